@@ -1,0 +1,638 @@
+/*
+ * mas_ref.c — ORACLE (test infrastructure only; see mas_ref.h header).
+ *
+ * Plain, slow, obviously-correct CPU implementation of the discretised MAS
+ * implicit parabolic operator and its Jacobi-PCG solve.  Every formula is the
+ * reading frozen in SURVEY.md §8(c) / DESIGN.md §3; the paper itself
+ * (Caplan et al. 2023) states no formula.
+ *
+ * Structure: the 1-D metric tables are the plain definitions of §8(c)
+ * "1-D metrics"; cell_L() is the per-cell operator written face by face
+ * exactly as "(L u)_P = c_P u_P + (1/V_P) sum_f G_f (u_P - u_N(f))";
+ * the PCG loop is the textbook order of §8(c) "PCG, exact order".
+ * No blocking, fusion or reordering beyond that.
+ *
+ * Build: gcc -O2 -ffp-contract=off -fopenmp -shared -fPIC (oracle/build.py).
+ */
+#include "mas_ref.h"
+
+#include <math.h>
+#include <stdlib.h>
+#include <string.h>
+#ifdef _OPENMP
+#include <omp.h>
+#endif
+
+#define TWO_PI (2.0 * 3.14159265358979323846)
+
+void mas_ref_set_threads(int n) {
+#ifdef _OPENMP
+    if (n > 0) omp_set_num_threads(n);
+#else
+    (void)n;
+#endif
+}
+
+/* ---------------------------------------------------------------------------
+ * 1-D metric tables (SURVEY §8(c) "1-D metrics"; readings R1, R3, R7).
+ * ------------------------------------------------------------------------- */
+typedef struct {
+    int nr, nt, np;
+    double *dr, *dt, *dp;   /* cell widths                                    */
+    double *hr;             /* [nr+1] centre distance across r-face i (R3)    */
+    double *ht;             /* [nt+1] centre distance across theta-face j     */
+    double *hp;             /* [np]   centre distance across phi-face k (wrap)*/
+    double *sC, *sF;        /* sin(theta) at centres [nt] and faces [nt+1]    */
+} tables;
+
+static void tables_free(tables* T) {
+    free(T->dr); free(T->dt); free(T->dp); free(T->hr); free(T->ht);
+    free(T->hp); free(T->sC); free(T->sF);
+}
+
+static int tables_make(const mas_ref_grid* g, tables* T) {
+    int nr = g->nr, nt = g->nt, np = g->np, i, j, k;
+    memset(T, 0, sizeof(*T));
+    if (nr < 1 || nt < 1 || np < 2) return MAS_REF_ERR_ARG;
+    T->nr = nr; T->nt = nt; T->np = np;
+    T->dr = malloc(sizeof(double) * nr);
+    T->dt = malloc(sizeof(double) * nt);
+    T->dp = malloc(sizeof(double) * np);
+    T->hr = malloc(sizeof(double) * (nr + 1));
+    T->ht = malloc(sizeof(double) * (nt + 1));
+    T->hp = malloc(sizeof(double) * np);
+    T->sC = malloc(sizeof(double) * nt);
+    T->sF = malloc(sizeof(double) * (nt + 1));
+    if (!T->dr || !T->dt || !T->dp || !T->hr || !T->ht || !T->hp || !T->sC || !T->sF) {
+        tables_free(T);
+        return MAS_REF_ERR_ARG;
+    }
+    for (i = 0; i < nr; i++) T->dr[i] = g->rF[i + 1] - g->rF[i];
+    for (j = 0; j < nt; j++) T->dt[j] = g->tF[j + 1] - g->tF[j];
+    for (k = 0; k < np; k++) T->dp[k] = g->pF[k + 1] - g->pF[k];
+    /* hr: interior faces centre-to-centre; boundary faces half-cell (R3). */
+    T->hr[0] = g->rC[0] - g->rF[0];
+    for (i = 1; i < nr; i++) T->hr[i] = g->rC[i] - g->rC[i - 1];
+    T->hr[nr] = g->rF[nr] - g->rC[nr - 1];
+    /* ht only for interior theta faces; faces 0 and nt carry no flux (R5). */
+    T->ht[0] = 0.0; T->ht[nt] = 0.0;
+    for (j = 1; j < nt; j++) T->ht[j] = g->tC[j] - g->tC[j - 1];
+    /* hp: periodic, face 0 lies between cell np-1 and cell 0 (R7). */
+    T->hp[0] = g->pC[0] + TWO_PI - g->pC[np - 1];
+    for (k = 1; k < np; k++) T->hp[k] = g->pC[k] - g->pC[k - 1];
+    for (j = 0; j < nt; j++) T->sC[j] = sin(g->tC[j]);
+    T->sF[0] = 0.0; T->sF[nt] = 0.0;       /* never used: pole / wall faces */
+    for (j = 1; j < nt; j++) T->sF[j] = sin(g->tF[j]);
+    return MAS_REF_OK;
+}
+
+/* Cell volume (R4): V = rC^2 dr * sC dt * dp. */
+static double cell_V(const mas_ref_grid* g, const tables* T, int i, int j, int k) {
+    return g->rC[i] * g->rC[i] * T->dr[i] * T->sC[j] * T->dt[j] * T->dp[k];
+}
+
+/* Face geometric conductances (R4), faces numbered:
+ *   0: r-face i (toward i-1)   1: r-face i+1 (toward i+1)
+ *   2: t-face j (toward j-1)   3: t-face j+1 (toward j+1)
+ *   4: p-face k (toward k-1)   5: p-face k+1 (toward k+1), periodic
+ *   gR(i;j,k) = rF[i]^2 * sC[j]*dt[j]*dp[k] / hr[i]
+ *   gT(j;i,k) = dr[i] * sF[j]*dp[k] / ht[j]
+ *   gP(k;i,j) = dr[i] * dt[j] / (sC[j]*hp[k])                                */
+static double gR(const mas_ref_grid* g, const tables* T, int iface, int j, int k) {
+    return g->rF[iface] * g->rF[iface] * T->sC[j] * T->dt[j] * T->dp[k] / T->hr[iface];
+}
+static double gT(const tables* T, int i, int jface, int k) {
+    return T->dr[i] * T->sF[jface] * T->dp[k] / T->ht[jface];
+}
+static double gP(const tables* T, int i, int j, int kface) {
+    return T->dr[i] * T->dt[j] / (T->sC[j] * T->hp[kface]);
+}
+
+enum { FACE_NONE = 0, FACE_INTERIOR = 1, FACE_DIRICHLET = 2 };
+
+/* Face kinds of cell (i,j,k) in the GLOBAL grid (R3, R5, R7). */
+static void face_kinds(const mas_ref_grid* g, int i, int j, int kind[6]) {
+    kind[0] = (i > 0) ? FACE_INTERIOR
+              : (g->bc_inner == MAS_REF_DIRICHLET ? FACE_DIRICHLET : FACE_NONE);
+    kind[1] = (i < g->nr - 1) ? FACE_INTERIOR
+              : (g->bc_outer == MAS_REF_DIRICHLET ? FACE_DIRICHLET : FACE_NONE);
+    kind[2] = (j > 0) ? FACE_INTERIOR : FACE_NONE;          /* pole / wall (R5) */
+    kind[3] = (j < g->nt - 1) ? FACE_INTERIOR : FACE_NONE;
+    kind[4] = FACE_INTERIOR;                                /* periodic phi (R7) */
+    kind[5] = FACE_INTERIOR;
+}
+
+static void face_geoms(const mas_ref_grid* g, const tables* T, int i, int j, int k,
+                       const int kind[6], double gf[6]) {
+    int np = g->np;
+    gf[0] = kind[0] ? gR(g, T, i, j, k) : 0.0;
+    gf[1] = kind[1] ? gR(g, T, i + 1, j, k) : 0.0;
+    gf[2] = kind[2] ? gT(T, i, j, k) : 0.0;
+    gf[3] = kind[3] ? gT(T, i, j + 1, k) : 0.0;
+    gf[4] = gP(T, i, j, k);
+    gf[5] = gP(T, i, j, (k + 1) % np);
+}
+
+/* (L u)_P = c_P u_P + (1/V_P) * sum_f G_f (u_P - u_N(f)),
+ * G_f = kappa_f g_f, kappa_f = (kappa_P + kappa_N)/2 on interior faces (R6),
+ * kappa_f = kappa_P and u_N = 0 on a Dirichlet face (homogeneous).          */
+static double cell_L(double V, double cP, double kP, double uP, const int kind[6],
+                     const double gf[6], const double kN[6], const double uN[6]) {
+    double acc = 0.0;
+    int f;
+    for (f = 0; f < 6; f++) {
+        if (kind[f] == FACE_INTERIOR) {
+            double G = 0.5 * (kP + kN[f]) * gf[f];
+            acc += G * (uP - uN[f]);
+        } else if (kind[f] == FACE_DIRICHLET) {
+            double G = kP * gf[f];
+            acc += G * uP;
+        }
+    }
+    return cP * uP + acc / V;
+}
+
+/* Jacobi diagonal D_P = c_P + (1/V_P) sum_f G_f (R8). */
+static double cell_D(double V, double cP, double kP, const int kind[6],
+                     const double gf[6], const double kN[6]) {
+    double acc = 0.0;
+    int f;
+    for (f = 0; f < 6; f++) {
+        if (kind[f] == FACE_INTERIOR) acc += 0.5 * (kP + kN[f]) * gf[f];
+        else if (kind[f] == FACE_DIRICHLET) acc += kP * gf[f];
+    }
+    return cP + acc / V;
+}
+
+#define IDX(g, i, j, k) (((size_t)(i) * (g)->nt + (size_t)(j)) * (g)->np + (size_t)(k))
+
+/* Gather the 6 neighbour values of a monolithic field a at (i,j,k). */
+static void gather(const mas_ref_grid* g, const double* a, int i, int j, int k,
+                   const int kind[6], double out[6]) {
+    int np = g->np;
+    out[0] = (kind[0] == FACE_INTERIOR) ? a[IDX(g, i - 1, j, k)] : 0.0;
+    out[1] = (kind[1] == FACE_INTERIOR) ? a[IDX(g, i + 1, j, k)] : 0.0;
+    out[2] = (kind[2] == FACE_INTERIOR) ? a[IDX(g, i, j - 1, k)] : 0.0;
+    out[3] = (kind[3] == FACE_INTERIOR) ? a[IDX(g, i, j + 1, k)] : 0.0;
+    out[4] = a[IDX(g, i, j, (k + np - 1) % np)];
+    out[5] = a[IDX(g, i, j, (k + 1) % np)];
+}
+
+int mas_ref_volumes(const mas_ref_grid* g, double* V) {
+    tables T;
+    int i;
+    if (!g || !V || tables_make(g, &T)) return MAS_REF_ERR_ARG;
+#pragma omp parallel for schedule(static)
+    for (i = 0; i < g->nr; i++) {
+        int j, k;
+        for (j = 0; j < g->nt; j++)
+            for (k = 0; k < g->np; k++) V[IDX(g, i, j, k)] = cell_V(g, &T, i, j, k);
+    }
+    tables_free(&T);
+    return MAS_REF_OK;
+}
+
+int mas_ref_op_apply(const mas_ref_grid* g, int ncomp, const double* kappa,
+                     const double* c, const double* x, double* y) {
+    tables T;
+    size_t N;
+    int i;
+    if (!g || !kappa || !x || !y || ncomp < 1 || tables_make(g, &T)) return MAS_REF_ERR_ARG;
+    N = (size_t)g->nr * g->nt * g->np;
+#pragma omp parallel for schedule(static)
+    for (i = 0; i < g->nr; i++) {
+        int j, k, m, kind[6];
+        double gf[6], kN[6], uN[6];
+        for (j = 0; j < g->nt; j++) {
+            face_kinds(g, i, j, kind);
+            for (k = 0; k < g->np; k++) {
+                size_t P = IDX(g, i, j, k);
+                double V = cell_V(g, &T, i, j, k);
+                double cP = c ? c[P] : 0.0;
+                face_geoms(g, &T, i, j, k, kind, gf);
+                gather(g, kappa, i, j, k, kind, kN);
+                for (m = 0; m < ncomp; m++) {
+                    const double* u = x + (size_t)m * N;
+                    gather(g, u, i, j, k, kind, uN);
+                    y[(size_t)m * N + P] = cell_L(V, cP, kappa[P], u[P], kind, gf, kN, uN);
+                }
+            }
+        }
+    }
+    tables_free(&T);
+    return MAS_REF_OK;
+}
+
+int mas_ref_op_diag(const mas_ref_grid* g, const double* kappa, const double* c,
+                    double* D) {
+    tables T;
+    int i;
+    if (!g || !kappa || !D || tables_make(g, &T)) return MAS_REF_ERR_ARG;
+#pragma omp parallel for schedule(static)
+    for (i = 0; i < g->nr; i++) {
+        int j, k, kind[6];
+        double gf[6], kN[6];
+        for (j = 0; j < g->nt; j++) {
+            face_kinds(g, i, j, kind);
+            for (k = 0; k < g->np; k++) {
+                size_t P = IDX(g, i, j, k);
+                face_geoms(g, &T, i, j, k, kind, gf);
+                gather(g, kappa, i, j, k, kind, kN);
+                D[P] = cell_D(cell_V(g, &T, i, j, k), c ? c[P] : 0.0, kappa[P], kind, gf, kN);
+            }
+        }
+    }
+    tables_free(&T);
+    return MAS_REF_OK;
+}
+
+int mas_ref_dirichlet_rhs(const mas_ref_grid* g, int ncomp, const double* kappa,
+                          const double* ub_inner, const double* ub_outer, double* f) {
+    tables T;
+    size_t N, plane;
+    int j, k, m;
+    if (!g || !kappa || !f || ncomp < 1 || tables_make(g, &T)) return MAS_REF_ERR_ARG;
+    N = (size_t)g->nr * g->nt * g->np;
+    plane = (size_t)g->nt * g->np;
+    for (m = 0; m < ncomp; m++)
+        for (j = 0; j < g->nt; j++)
+            for (k = 0; k < g->np; k++) {
+                if (ub_inner && g->bc_inner == MAS_REF_DIRICHLET) {
+                    size_t P = IDX(g, 0, j, k);
+                    double G = kappa[P] * gR(g, &T, 0, j, k);
+                    f[(size_t)m * N + P] += G * ub_inner[(size_t)m * plane + (size_t)j * g->np + k]
+                                            / cell_V(g, &T, 0, j, k);
+                }
+                if (ub_outer && g->bc_outer == MAS_REF_DIRICHLET) {
+                    int i = g->nr - 1;
+                    size_t P = IDX(g, i, j, k);
+                    double G = kappa[P] * gR(g, &T, g->nr, j, k);
+                    f[(size_t)m * N + P] += G * ub_outer[(size_t)m * plane + (size_t)j * g->np + k]
+                                            / cell_V(g, &T, i, j, k);
+                }
+            }
+    tables_free(&T);
+    return MAS_REF_OK;
+}
+
+/* V-weighted dot over planes [i0, i0+nl) of arrays holding exactly those
+ * planes; per-plane partials in (j,k) order, then planes in order, then
+ * components (R9). */
+static double dot_planes(const mas_ref_grid* g, const tables* T, int i0, int nl,
+                         int ncomp, const double* a, const double* b) {
+    size_t plane = (size_t)g->nt * g->np, Nl = plane * nl;
+    double* part = malloc(sizeof(double) * (size_t)nl * ncomp);
+    double s = 0.0;
+    int il, m;
+    if (!part) return NAN;
+    for (m = 0; m < ncomp; m++) {
+#pragma omp parallel for schedule(static)
+        for (il = 0; il < nl; il++) {
+            int j, k, i = i0 + il;
+            double ps = 0.0;
+            for (j = 0; j < g->nt; j++)
+                for (k = 0; k < g->np; k++) {
+                    size_t P = (size_t)m * Nl + (size_t)il * plane + (size_t)j * g->np + k;
+                    ps += cell_V(g, T, i, j, k) * a[P] * b[P];
+                }
+            part[(size_t)m * nl + il] = ps;
+        }
+    }
+    for (m = 0; m < ncomp; m++)
+        for (il = 0; il < nl; il++) s += part[(size_t)m * nl + il];
+    free(part);
+    return s;
+}
+
+int mas_ref_dot(const mas_ref_grid* g, int ncomp, const double* a, const double* b,
+                double* out) {
+    tables T;
+    if (!g || !a || !b || !out || ncomp < 1 || tables_make(g, &T)) return MAS_REF_ERR_ARG;
+    *out = dot_planes(g, &T, 0, g->nr, ncomp, a, b);
+    tables_free(&T);
+    return MAS_REF_OK;
+}
+
+/* ---------------------------------------------------------------------------
+ * Jacobi-PCG (SURVEY §8(c) "PCG, exact order"; R10 stopping, R11 counting).
+ * ------------------------------------------------------------------------- */
+int mas_ref_pcg_solve(const mas_ref_grid* g, int ncomp, const double* kappa,
+                      const double* c, const double* f, double* x, double tol,
+                      int maxit, int* iters, double* relres, double* res_hist) {
+    tables T;
+    size_t N, n, e;
+    double *D, *r, *z, *p, *q;
+    double bn, rn, rho, sigma, alpha, rho_new, beta;
+    int k, status = MAS_REF_NOT_CONVERGED, m;
+    if (!g || !kappa || !f || !x || !iters || !relres || ncomp < 1 || maxit < 0 ||
+        !(tol >= 0.0) || tables_make(g, &T))
+        return MAS_REF_ERR_ARG;
+    N = (size_t)g->nr * g->nt * g->np;
+    n = N * ncomp;
+    D = malloc(sizeof(double) * N);
+    r = malloc(sizeof(double) * n);
+    z = malloc(sizeof(double) * n);
+    p = malloc(sizeof(double) * n);
+    q = malloc(sizeof(double) * n);
+    if (!D || !r || !z || !p || !q) { status = MAS_REF_ERR_ARG; goto done; }
+    mas_ref_op_diag(g, kappa, c, D);
+
+    bn = sqrt(dot_planes(g, &T, 0, g->nr, ncomp, f, f));
+    if (bn == 0.0) {
+        for (e = 0; e < n; e++) x[e] = 0.0;
+        *iters = 0; *relres = 0.0;
+        if (res_hist) res_hist[0] = 0.0;
+        status = MAS_REF_OK; goto done;
+    }
+    mas_ref_op_apply(g, ncomp, kappa, c, x, r);                  /* r = L x     */
+#pragma omp parallel for schedule(static)
+    for (e = 0; e < n; e++) r[e] = f[e] - r[e];                  /* r = f - L x */
+    rn = sqrt(dot_planes(g, &T, 0, g->nr, ncomp, r, r));
+    if (res_hist) res_hist[0] = rn;
+    if (rn <= tol * bn) { *iters = 0; *relres = rn / bn; status = MAS_REF_OK; goto done; }
+    for (m = 0; m < ncomp; m++)
+#pragma omp parallel for schedule(static)
+        for (e = 0; e < N; e++) z[m * N + e] = r[m * N + e] / D[e];   /* z = D^-1 r  */
+    memcpy(p, z, sizeof(double) * n);                            /* p = z       */
+    rho = dot_planes(g, &T, 0, g->nr, ncomp, r, z);
+
+    for (k = 1; k <= maxit; k++) {
+        mas_ref_op_apply(g, ncomp, kappa, c, p, q);              /* q = L p     */
+        sigma = dot_planes(g, &T, 0, g->nr, ncomp, p, q);
+        if (!(sigma > 0.0) || !isfinite(sigma)) {
+            *iters = k; *relres = rn / bn; status = MAS_REF_ERR_BREAKDOWN; goto done;
+        }
+        alpha = rho / sigma;
+#pragma omp parallel for schedule(static)
+        for (e = 0; e < n; e++) { x[e] += alpha * p[e]; r[e] -= alpha * q[e]; }
+        rn = sqrt(dot_planes(g, &T, 0, g->nr, ncomp, r, r));
+        if (res_hist) res_hist[k] = rn;
+        if (rn <= tol * bn) { *iters = k; *relres = rn / bn; status = MAS_REF_OK; goto done; }
+        for (m = 0; m < ncomp; m++)
+#pragma omp parallel for schedule(static)
+            for (e = 0; e < N; e++) z[m * N + e] = r[m * N + e] / D[e];
+        rho_new = dot_planes(g, &T, 0, g->nr, ncomp, r, z);
+        beta = rho_new / rho;
+        rho = rho_new;
+#pragma omp parallel for schedule(static)
+        for (e = 0; e < n; e++) p[e] = z[e] + beta * p[e];
+    }
+    *iters = maxit; *relres = rn / bn; status = MAS_REF_NOT_CONVERGED;
+done:
+    free(D); free(r); free(z); free(p); free(q);
+    tables_free(&T);
+    return status;
+}
+
+/* ---------------------------------------------------------------------------
+ * r-slab decomposition; "virtual ranks" in one process.
+ * ------------------------------------------------------------------------- */
+void mas_ref_partition(int nr, int nranks, int rank, int* i0, int* nl) {
+    int base = nr / nranks, rem = nr % nranks;
+    *nl = base + (rank < rem ? 1 : 0);
+    *i0 = rank * base + (rank < rem ? rank : rem);
+}
+
+int mas_ref_op_apply_slab(const mas_ref_grid* g, int i0, int nl, int ncomp,
+                          const double* kappa_ext, const double* c,
+                          const double* x_ext, double* y) {
+    tables T;
+    size_t plane, Ne, Nl;
+    int il;
+    if (!g || !kappa_ext || !x_ext || !y || ncomp < 1 || nl < 1 || i0 < 0 ||
+        i0 + nl > g->nr || tables_make(g, &T))
+        return MAS_REF_ERR_ARG;
+    plane = (size_t)g->nt * g->np;
+    Ne = plane * (nl + 2);
+    Nl = plane * nl;
+#pragma omp parallel for schedule(static)
+    for (il = 0; il < nl; il++) {
+        int i = i0 + il, j, k, m, kind[6], np = g->np;
+        double gf[6], kN[6], uN[6];
+        for (j = 0; j < g->nt; j++) {
+            face_kinds(g, i, j, kind);
+            for (k = 0; k < np; k++) {
+                /* extended index: local plane il sits at ext plane il+1 */
+                size_t Pe = (size_t)(il + 1) * plane + (size_t)j * np + k;
+                size_t Pl = (size_t)il * plane + (size_t)j * np + k;
+                size_t km = (size_t)j * np + (k + np - 1) % np, kp = (size_t)j * np + (k + 1) % np;
+                double V = cell_V(g, &T, i, j, k);
+                face_geoms(g, &T, i, j, k, kind, gf);
+                kN[0] = kappa_ext[Pe - plane];
+                kN[1] = kappa_ext[Pe + plane];
+                kN[2] = (j > 0) ? kappa_ext[Pe - np] : 0.0;
+                kN[3] = (j < g->nt - 1) ? kappa_ext[Pe + np] : 0.0;
+                kN[4] = kappa_ext[(size_t)(il + 1) * plane + km];
+                kN[5] = kappa_ext[(size_t)(il + 1) * plane + kp];
+                for (m = 0; m < ncomp; m++) {
+                    const double* u = x_ext + (size_t)m * Ne;
+                    uN[0] = u[Pe - plane];
+                    uN[1] = u[Pe + plane];
+                    uN[2] = (j > 0) ? u[Pe - np] : 0.0;
+                    uN[3] = (j < g->nt - 1) ? u[Pe + np] : 0.0;
+                    uN[4] = u[(size_t)(il + 1) * plane + km];
+                    uN[5] = u[(size_t)(il + 1) * plane + kp];
+                    y[(size_t)m * Nl + Pl] =
+                        cell_L(V, c ? c[Pl] : 0.0, kappa_ext[Pe], u[Pe], kind, gf, kN, uN);
+                }
+            }
+        }
+    }
+    tables_free(&T);
+    return MAS_REF_OK;
+}
+
+int mas_ref_dot_slab(const mas_ref_grid* g, int i0, int nl, int ncomp,
+                     const double* a, const double* b, double* out) {
+    tables T;
+    if (!g || !a || !b || !out || nl < 1 || tables_make(g, &T)) return MAS_REF_ERR_ARG;
+    *out = dot_planes(g, &T, i0, nl, ncomp, a, b);
+    tables_free(&T);
+    return MAS_REF_OK;
+}
+
+typedef struct {
+    int i0, nl;
+    double *k_ext, *c, *D, *f, *x_ext, *r, *z, *p_ext, *q;
+} vslab;
+
+/* Seam exchange: copy the edge planes of every slab's extended field into the
+ * ghost planes of its r-neighbours (what ncclSend/ncclRecv do per rank). */
+static void vseam(const mas_ref_grid* g, vslab* S, int P, int ncomp, int which) {
+    size_t plane = (size_t)g->nt * g->np, bytes = sizeof(double) * plane;
+    int s, m;
+    for (s = 0; s < P; s++)
+        for (m = 0; m < ncomp; m++) {
+            size_t Ne = plane * (S[s].nl + 2);
+            double* a = (which == 0 ? S[s].x_ext : which == 1 ? S[s].p_ext : S[s].k_ext) + m * Ne;
+            if (s > 0) {
+                vslab* L = &S[s - 1];
+                size_t NeL = plane * (L->nl + 2);
+                double* b = (which == 0 ? L->x_ext : which == 1 ? L->p_ext : L->k_ext) + m * NeL;
+                memcpy(a, b + (size_t)L->nl * plane, bytes);           /* ghost lo <- L's last  */
+                memcpy(b + (size_t)(L->nl + 1) * plane, a + plane, bytes); /* L's ghost hi <- my first */
+            }
+        }
+}
+
+int mas_ref_pcg_solve_vranks(const mas_ref_grid* g, int P, int ncomp,
+                             const double* kappa, const double* c, const double* f,
+                             double* x, double tol, int maxit, int* iters,
+                             double* relres, double* res_hist) {
+    size_t plane, N;
+    vslab* S;
+    int s, m, k, status = MAS_REF_NOT_CONVERGED;
+    double bn, rn, rho, sigma, alpha, rho_new, beta, part;
+    if (!g || P < 1 || P > g->nr || !kappa || !f || !x || !iters || !relres || ncomp < 1)
+        return MAS_REF_ERR_ARG;
+    plane = (size_t)g->nt * g->np;
+    N = plane * g->nr;
+    S = calloc(P, sizeof(vslab));
+    for (s = 0; s < P; s++) {
+        size_t Nl, Ne;
+        mas_ref_partition(g->nr, P, s, &S[s].i0, &S[s].nl);
+        Nl = plane * S[s].nl; Ne = plane * (S[s].nl + 2);
+        S[s].k_ext = calloc(Ne, sizeof(double));
+        S[s].c = calloc(Nl, sizeof(double));
+        S[s].D = calloc(Nl, sizeof(double));
+        S[s].f = calloc(Nl * ncomp, sizeof(double));
+        S[s].x_ext = calloc(Ne * ncomp, sizeof(double));
+        S[s].r = calloc(Nl * ncomp, sizeof(double));
+        S[s].z = calloc(Nl * ncomp, sizeof(double));
+        S[s].p_ext = calloc(Ne * ncomp, sizeof(double));
+        S[s].q = calloc(Nl * ncomp, sizeof(double));
+        memcpy(S[s].k_ext + plane, kappa + S[s].i0 * plane, sizeof(double) * Nl);
+        if (c) memcpy(S[s].c, c + S[s].i0 * plane, sizeof(double) * Nl);
+        for (m = 0; m < ncomp; m++) {
+            memcpy(S[s].f + m * Nl, f + m * N + S[s].i0 * plane, sizeof(double) * Nl);
+            memcpy(S[s].x_ext + m * Ne + plane, x + m * N + S[s].i0 * plane, sizeof(double) * Nl);
+        }
+    }
+    vseam(g, S, P, 1, 2);                                   /* static kappa seams */
+    /* Jacobi diagonal: setup-time quantity, taken from the monolithic routine
+     * restricted to each slab's planes. */
+    {
+        double* Dg = malloc(sizeof(double) * N);
+        mas_ref_op_diag(g, kappa, c, Dg);
+        for (s = 0; s < P; s++)
+            memcpy(S[s].D, Dg + S[s].i0 * plane, sizeof(double) * plane * S[s].nl);
+        free(Dg);
+    }
+    bn = 0.0;
+    for (s = 0; s < P; s++) { mas_ref_dot_slab(g, S[s].i0, S[s].nl, ncomp, S[s].f, S[s].f, &part); bn += part; }
+    bn = sqrt(bn);
+    if (bn == 0.0) {
+        memset(x, 0, sizeof(double) * N * ncomp);
+        *iters = 0; *relres = 0.0; if (res_hist) res_hist[0] = 0.0;
+        status = MAS_REF_OK; goto done;
+    }
+    vseam(g, S, P, ncomp, 0);
+    rn = 0.0;
+    for (s = 0; s < P; s++) {
+        size_t Nl = plane * S[s].nl, e;
+        mas_ref_op_apply_slab(g, S[s].i0, S[s].nl, ncomp, S[s].k_ext, c ? S[s].c : NULL, S[s].x_ext, S[s].r);
+        for (e = 0; e < Nl * ncomp; e++) S[s].r[e] = S[s].f[e] - S[s].r[e];
+        mas_ref_dot_slab(g, S[s].i0, S[s].nl, ncomp, S[s].r, S[s].r, &part); rn += part;
+    }
+    rn = sqrt(rn);
+    if (res_hist) res_hist[0] = rn;
+    if (rn <= tol * bn) { *iters = 0; *relres = rn / bn; status = MAS_REF_OK; goto copyout; }
+    rho = 0.0;
+    for (s = 0; s < P; s++) {
+        size_t Nl = plane * S[s].nl, Ne = plane * (S[s].nl + 2), e;
+        for (m = 0; m < ncomp; m++)
+            for (e = 0; e < Nl; e++) {
+                S[s].z[m * Nl + e] = S[s].r[m * Nl + e] / S[s].D[e];
+                S[s].p_ext[m * Ne + plane + e] = S[s].z[m * Nl + e];
+            }
+        mas_ref_dot_slab(g, S[s].i0, S[s].nl, ncomp, S[s].r, S[s].z, &part); rho += part;
+    }
+    for (k = 1; k <= maxit; k++) {
+        vseam(g, S, P, ncomp, 1);                           /* p seams        */
+        sigma = 0.0;
+        for (s = 0; s < P; s++) {
+            size_t Nl = plane * S[s].nl, Ne = plane * (S[s].nl + 2), e;
+            double* pl = malloc(sizeof(double) * Nl * ncomp);
+            mas_ref_op_apply_slab(g, S[s].i0, S[s].nl, ncomp, S[s].k_ext, c ? S[s].c : NULL, S[s].p_ext, S[s].q);
+            for (m = 0; m < ncomp; m++)
+                for (e = 0; e < Nl; e++) pl[m * Nl + e] = S[s].p_ext[m * Ne + plane + e];
+            mas_ref_dot_slab(g, S[s].i0, S[s].nl, ncomp, pl, S[s].q, &part); sigma += part;
+            free(pl);
+        }
+        if (!(sigma > 0.0) || !isfinite(sigma)) {
+            *iters = k; *relres = rn / bn; status = MAS_REF_ERR_BREAKDOWN; goto copyout;
+        }
+        alpha = rho / sigma;
+        rn = 0.0;
+        for (s = 0; s < P; s++) {
+            size_t Nl = plane * S[s].nl, Ne = plane * (S[s].nl + 2), e;
+            for (m = 0; m < ncomp; m++)
+                for (e = 0; e < Nl; e++) {
+                    S[s].x_ext[m * Ne + plane + e] += alpha * S[s].p_ext[m * Ne + plane + e];
+                    S[s].r[m * Nl + e] -= alpha * S[s].q[m * Nl + e];
+                }
+            mas_ref_dot_slab(g, S[s].i0, S[s].nl, ncomp, S[s].r, S[s].r, &part); rn += part;
+        }
+        rn = sqrt(rn);
+        if (res_hist) res_hist[k] = rn;
+        if (rn <= tol * bn) { *iters = k; *relres = rn / bn; status = MAS_REF_OK; goto copyout; }
+        rho_new = 0.0;
+        for (s = 0; s < P; s++) {
+            size_t Nl = plane * S[s].nl, e;
+            for (m = 0; m < ncomp; m++)
+                for (e = 0; e < Nl; e++) S[s].z[m * Nl + e] = S[s].r[m * Nl + e] / S[s].D[e];
+            mas_ref_dot_slab(g, S[s].i0, S[s].nl, ncomp, S[s].r, S[s].z, &part); rho_new += part;
+        }
+        beta = rho_new / rho;
+        rho = rho_new;
+        for (s = 0; s < P; s++) {
+            size_t Nl = plane * S[s].nl, Ne = plane * (S[s].nl + 2), e;
+            for (m = 0; m < ncomp; m++)
+                for (e = 0; e < Nl; e++)
+                    S[s].p_ext[m * Ne + plane + e] = S[s].z[m * Nl + e] + beta * S[s].p_ext[m * Ne + plane + e];
+        }
+    }
+    *iters = maxit; *relres = rn / bn; status = MAS_REF_NOT_CONVERGED;
+copyout:
+    for (s = 0; s < P; s++) {
+        size_t Nl = plane * S[s].nl, Ne = plane * (S[s].nl + 2);
+        for (m = 0; m < ncomp; m++)
+            memcpy(x + m * N + S[s].i0 * plane, S[s].x_ext + m * Ne + plane, sizeof(double) * Nl);
+    }
+done:
+    for (s = 0; s < P; s++) {
+        free(S[s].k_ext); free(S[s].c); free(S[s].D); free(S[s].f); free(S[s].x_ext);
+        free(S[s].r); free(S[s].z); free(S[s].p_ext); free(S[s].q);
+    }
+    free(S);
+    return status;
+}
+
+/* Per-cell evaluation of (L x) at a list of flat cell indices (comp-major
+ * flat index m*N + P): used to check GPU results sampled at full size. */
+int mas_ref_op_apply_cells(const mas_ref_grid* g, int ncomp, const double* kappa,
+                           const double* c, const double* x, long long ncells,
+                           const long long* idx, double* out) {
+    tables T;
+    size_t N;
+    long long s;
+    if (!g || !kappa || !x || !idx || !out || ncomp < 1 || tables_make(g, &T)) return MAS_REF_ERR_ARG;
+    N = (size_t)g->nr * g->nt * g->np;
+#pragma omp parallel for schedule(static)
+    for (s = 0; s < ncells; s++) {
+        size_t flat = (size_t)idx[s], P = flat % N;
+        int m = (int)(flat / N);
+        int i = (int)(P / ((size_t)g->nt * g->np));
+        int j = (int)((P / g->np) % g->nt);
+        int k = (int)(P % g->np), kind[6];
+        double gf[6], kN[6], uN[6];
+        const double* u = x + (size_t)m * N;
+        face_kinds(g, i, j, kind);
+        face_geoms(g, &T, i, j, k, kind, gf);
+        gather(g, kappa, i, j, k, kind, kN);
+        gather(g, u, i, j, k, kind, uN);
+        out[s] = cell_L(cell_V(g, &T, i, j, k), c ? c[P] : 0.0, kappa[P], u[P], kind, gf, kN, uN);
+    }
+    tables_free(&T);
+    return MAS_REF_OK;
+}

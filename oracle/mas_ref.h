@@ -1,0 +1,111 @@
+/*
+ * mas_ref.h — ORACLE for the MAS implicit-parabolic PCG path.
+ *
+ * TEST INFRASTRUCTURE ONLY.  Nothing in the product path
+ * (paper_conf_ipps_caplansl23_b200/, include/) may include, link or call this.
+ * Only tests/, __graft_entry__.smoke() and bench.py (cpu_baseline leg and
+ * --impl reference) may load it.  It shares no source with the CUDA path.
+ *
+ * What it computes (the paper, Caplan, Stulajter & Linker 2023, prints no
+ * formula; every definition below is a reading frozen in SURVEY.md §8(c) and
+ * DESIGN.md §3, R1..R16):
+ *   P:208-213 (§III)  "logically rectangular non-uniform staggered spherical
+ *                      grid", "finite-difference discretizations", implicit
+ *                      time stepping, "highly memory-bound".
+ *   P:1027-1030 (Fig.4) "viscosity solver iterations" with halo exchanges.
+ *   P:1212-1216 ([25])  implicit parabolic schemes "with krylov solvers".
+ *
+ * Arithmetic: IEEE fp64, compiled -O2 -ffp-contract=off (no FMA contraction,
+ * no fast-math).  Reductions are summed per r-plane in (j,k) order, planes in
+ * increasing i, then components, so results are independent of the OpenMP
+ * thread count.
+ *
+ * Layout: C order [comp][i=r][j=theta][k=phi], phi fastest (reading R15).
+ * All pointers are HOST pointers.  Return value 0 = OK; see codes below.
+ */
+#ifndef MAS_REF_H
+#define MAS_REF_H
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+enum { MAS_REF_OK = 0, MAS_REF_NOT_CONVERGED = 1, MAS_REF_ERR_ARG = 2,
+       MAS_REF_ERR_BREAKDOWN = 6 };
+enum { MAS_REF_DIRICHLET = 0, MAS_REF_NEUMANN = 1 };
+
+/* Grid description (R1): faces ("node"/main mesh) and centres ("half" mesh).
+ * rF[nr+1], rC[nr], tF[nt+1], tC[nt], pF[np+1], pC[np].
+ * bc_inner / bc_outer: r-boundary conditions (R3).  Theta faces 0 and nt never
+ * carry flux: pole faces have zero area, non-pole walls are Neumann (R5). */
+typedef struct {
+    int nr, nt, np;
+    const double *rF, *rC, *tF, *tC, *pF, *pC;
+    int bc_inner, bc_outer;
+} mas_ref_grid;
+
+void mas_ref_set_threads(int nthreads);
+
+/* Cell volumes V[i][j][k] = rC^2 dr * sin(tC) dt * dp   (R4). */
+int mas_ref_volumes(const mas_ref_grid* g, double* V);
+
+/* y = L x for ncomp components sharing kappa, c   (R2, R4-R7, R13).
+ * (L u)_P = c_P u_P + (1/V_P) sum_f G_f (u_P - u_N(f)), homogeneous BCs. */
+int mas_ref_op_apply(const mas_ref_grid* g, int ncomp, const double* kappa,
+                     const double* c, const double* x, double* y);
+
+/* Jacobi diagonal D_P = c_P + (1/V_P) sum_f G_f (Dirichlet faces included) (R8). */
+int mas_ref_op_diag(const mas_ref_grid* g, const double* kappa, const double* c,
+                    double* D);
+
+/* f += (1/V_P) G_b u_b on Dirichlet r-faces.  ub_inner/ub_outer: [ncomp][nt][np]
+ * or NULL (homogeneous).  A boundary whose bc is Neumann ignores its ub. */
+int mas_ref_dirichlet_rhs(const mas_ref_grid* g, int ncomp, const double* kappa,
+                          const double* ub_inner, const double* ub_outer,
+                          double* f);
+
+/* <a,b>_V = sum_m sum_P V_P a_mP b_mP   (R9). */
+int mas_ref_dot(const mas_ref_grid* g, int ncomp, const double* a,
+                const double* b, double* out);
+
+/* Jacobi-PCG, textbook order (R10-R12).  x: in x0, out solution.
+ * iters = number of L*p products in the loop; relres = ||r||_V/||f||_V.
+ * res_hist (NULL or maxit+1): ||r_k||_V for k = 0..iters. */
+int mas_ref_pcg_solve(const mas_ref_grid* g, int ncomp, const double* kappa,
+                      const double* c, const double* f, double* x, double tol,
+                      int maxit, int* iters, double* relres, double* res_hist);
+
+/* Slab-local operator for a rank owning r-planes [i0, i0+nl) of the global
+ * grid g.  kappa_ext and x_ext hold nl+2 planes per component: plane 0 is the
+ * ghost copy of global plane i0-1, plane nl+1 of i0+nl (ignored at a global
+ * boundary).  c and y hold nl interior planes. */
+int mas_ref_op_apply_slab(const mas_ref_grid* g, int i0, int nl, int ncomp,
+                          const double* kappa_ext, const double* c,
+                          const double* x_ext, double* y);
+
+/* Per-slab partial of <a,b>_V over planes [i0,i0+nl) (a,b interior, nl planes). */
+int mas_ref_dot_slab(const mas_ref_grid* g, int i0, int nl, int ncomp,
+                     const double* a, const double* b, double* out);
+
+/* The same PCG run on `nranks` virtual r-slabs inside one process: explicit
+ * ghost-plane copies between slab buffers, slab-local partial dots summed in
+ * rank order.  Models the multi-GPU decomposition. */
+int mas_ref_pcg_solve_vranks(const mas_ref_grid* g, int nranks, int ncomp,
+                             const double* kappa, const double* c,
+                             const double* f, double* x, double tol, int maxit,
+                             int* iters, double* relres, double* res_hist);
+
+/* (L x) evaluated only at the listed flat indices idx[s] = m*N + P (component
+ * major), for sampled checks at sizes where a full oracle pass is too slow. */
+int mas_ref_op_apply_cells(const mas_ref_grid* g, int ncomp, const double* kappa,
+                           const double* c, const double* x, long long ncells,
+                           const long long* idx, double* out);
+
+/* The r-slab partition: rank p owns n_p = nr/P + (p < nr%P)
+ * planes starting at i0_p. */
+void mas_ref_partition(int nr, int nranks, int rank, int* i0, int* nl);
+
+#ifdef __cplusplus
+}
+#endif
+#endif
