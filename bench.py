@@ -1,0 +1,371 @@
+#!/usr/bin/env python
+"""bench.py — fp64 Jacobi-PCG of the MAS implicit viscosity operator on B200.
+
+Metric (BASELINE.json): "fp64 PCG iters/sec and HBM GB/s vs peak at 1/2/4/8
+B200, 36M-cell grid".  Workload: config C3 — 3-component
+viscosity, 256x256x512 = 33.5 M cells (the paper's 36 M-cell test problem,
+PAPER.md P:748-758, is the shape model), synthetic coronal-like fields
+(paper_conf_ipps_caplansl23_b200.workloads), tol 1e-12.
+
+One step = one implicit viscosity step of the hot path: mas_op_update
+(a2: copy kappa/c, Jacobi diagonal) + x := x0 + mas_pcg_solve (a3-a5) to
+tol 1e-12.  value = PCG iterations / s over all ranks (strong scaling: the
+same global grid for every N, r-slabs per rank).  Inputs (>= 268 MB per
+field) exceed the 126 MB L2, so no explicit flush is needed.
+
+Launch: python bench.py [--gpus N --steps K --warmup W]; N > 1 under
+torch.distributed.run (one process per GPU, NCCL).  --impl reference times
+the CPU oracle on the host cores (the only other place oracle/ runs).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from paper_conf_ipps_caplansl23_b200 import workloads as W  # noqa: E402
+
+METRIC = "fp64 PCG iters/sec and HBM GB/s vs peak at 1/2/4/8 B200, 36M-cell grid"
+UNIT = "PCG iters/s"
+CONFIGS = {
+    # name: (kind, nr, nt, np)
+    "C3": ("viscosity", 256, 256, 512),
+    "C2": ("conduction", 128, 128, 256),
+    "C1": ("mms", 16, 24, 32),
+}
+# algorithmic bytes per cell per iteration: kernel A reads
+# r, p_old, x (ncomp each) + dinv, kappa, c and writes p, q, x (ncomp each);
+# kernel B reads r, q (ncomp) + dinv and writes r (ncomp).
+def alg_bytes_per_cell(ncomp):
+    a = 8 * (3 * ncomp + 3 + 3 * ncomp)
+    b = 8 * (2 * ncomp + 1 + ncomp)
+    return a, b
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return float(d.get("hbm_gbs", 6650.0)), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    return 6650.0, "fallback (B200_PROFILING.md)"
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+    FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.proc = None
+        self.lines = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}",
+                 "--format=csv,noheader,nounits", "-lms", "200"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if not self.proc:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        sm, smax, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            parts = [p.strip() for p in ln.split(",")]
+            if len(parts) < 8:
+                continue
+            try:
+                sm.append(float(parts[0]))
+                smax = float(parts[1])
+            except ValueError:
+                continue
+            for nm, v in zip(names, parts[4:8]):
+                if v.lower() == "active":
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": smax,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def make_problem(cfg: str):
+    kind, nr, nt, np_ = CONFIGS[cfg]
+    return W.make(kind, nr=nr, nt=nt, np_=np_)
+
+
+def cpu_cores() -> int:
+    try:
+        return len(os.sched_getaffinity(0))
+    except Exception:
+        return os.cpu_count() or 1
+
+
+def oracle_sample(prob, iters: int, threads: int):
+    """Time the oracle (as it stands) on a bounded sample: `iters` fixed PCG
+    iterations (tol = 0) on the full grid, minus a 1-iteration run to remove
+    the setup (diagonal, initial residual).  Returns iters/s."""
+    import oracle
+    o = oracle.Oracle.for_problem(prob, threads)
+    f = o.dirichlet_rhs(prob.kappa, prob.f, prob.ub_inner, prob.ub_outer)
+    t0 = time.perf_counter()
+    o.pcg(prob.kappa, prob.c, f, prob.x0, 0.0, 1)
+    t1 = time.perf_counter()
+    o.pcg(prob.kappa, prob.c, f, prob.x0, 0.0, 1 + iters)
+    t2 = time.perf_counter()
+    per_iter = max((t2 - t1) - (t1 - t0), 1e-9) / iters
+    return 1.0 / per_iter, per_iter
+
+
+def run_reference(args):
+    """--impl reference: the CPU oracle on this box's host cores, same config,
+    metric and unit; each step = 2 fixed oracle PCG iterations on the full grid."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    import oracle
+    oracle.build()
+    prob = make_problem(args.config)
+    cores = cpu_cores()
+    o = oracle.Oracle.for_problem(prob, cores)
+    f = o.dirichlet_rhs(prob.kappa, prob.f, prob.ub_inner, prob.ub_outer)
+    per_step_iters = 2
+    for _ in range(args.warmup):
+        o.pcg(prob.kappa, prob.c, f, prob.x0, 0.0, per_step_iters)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        o.pcg(prob.kappa, prob.c, f, prob.x0, 0.0, per_step_iters)
+    dt = time.perf_counter() - t0
+    value = args.steps * per_step_iters / dt
+    sample = (f"{args.config} full grid {prob.shape}, ncomp {prob.ncomp}: {per_step_iters} fixed "
+              f"oracle PCG iterations per step incl. its setup (diag + initial residual)")
+    line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * dt / args.steps,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic", "impl": "reference",
+            "config": {"workload": args.config, "grid": list(prob.shape), "ncomp": prob.ncomp},
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle",
+                             "sample": sample},
+            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0,
+                    "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=3)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="C3", choices=sorted(CONFIGS))
+    ap.add_argument("--tol", type=float, default=1e-12)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--cpu-iters", type=int, default=3)
+    args = ap.parse_args()
+    if args.impl == "reference":
+        return run_reference(args)
+
+    import torch
+    import torch.distributed as dist
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    from paper_conf_ipps_caplansl23_b200 import build as B
+    if rank == 0:
+        B.build()
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+        dist.barrier()
+    from paper_conf_ipps_caplansl23_b200 import maspcg as M
+
+    prob = make_problem(args.config)
+    nr, nt, np_ = prob.shape
+    distinfo = None
+    if world > 1:
+        obj = [M.mas_comm_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=0)
+        distinfo = (world, rank, obj[0])
+    grid = M.Grid(prob.mesh, distinfo)
+    i0, nl = grid.i0, grid.nl
+    sl = slice(i0, i0 + nl)
+    nc = prob.ncomp
+
+    def to_dev(a):
+        return torch.from_numpy(np.ascontiguousarray(a)).to(dev)
+
+    kappa = to_dev(prob.kappa[sl])
+    cmass = to_dev(prob.c[sl])
+    f = to_dev(prob.f[:, sl])
+    x0 = to_dev(prob.x0[:, sl])
+    x = x0.clone()
+    op = M.Operator(grid, nc, kappa, cmass, prob.bc_inner, prob.bc_outer)
+    ubi = to_dev(prob.ub_inner) if prob.ub_inner is not None else None
+    ubo = to_dev(prob.ub_outer) if prob.ub_outer is not None else None
+    rhs = f.clone()
+    if ubi is not None or ubo is not None:
+        op.dirichlet_rhs(ubi, ubo, rhs)
+    stream = torch.cuda.current_stream()
+    maxit = 20000
+
+    def step(prof=False):
+        op.update(kappa, cmass)           # a2: coefficients + Jacobi diagonal (1 kernel)
+        x.copy_(x0)                       # warm start x0 = v^n (R12)
+        st, it, rel, _ = op.solve(rhs, x, args.tol, maxit)
+        if st != M.MAS_OK:
+            raise RuntimeError(f"solve status {st}")
+        return it, op.launch_count + 1
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    op.set_profiling(True)
+    clocks = ClockSampler(local)
+    clocks.start()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    e0.record(stream)
+    iters_total, launches, ka, kb = 0, 0, [], []
+    for _ in range(args.steps):
+        it, nlaunch = step()
+        iters_total += it
+        launches += nlaunch
+        a_ms, b_ms, n = op.kernel_times()
+        ka.append(a_ms)
+        kb.append(b_ms)
+    e1.record(stream)
+    torch.cuda.synchronize()
+    clk = clocks.stop()
+    op.set_profiling(False)
+    t_ms = e0.elapsed_time(e1)
+    if world > 1:
+        tt = torch.tensor([t_ms], device=dev, dtype=torch.float64)
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        t_ms = float(tt.item())
+        dist.barrier()
+    iters_per_solve = iters_total / args.steps
+    value = iters_total / (t_ms / 1e3)  # the solve is one global problem: iterations are shared
+
+    # roofline of the dominant kernel (kernel A), algorithmic bytes / its
+    # average CUDA-event duration over the timed region
+    cells = nr * nt * np_
+    cells_local = nl * nt * np_
+    a_b, b_b = alg_bytes_per_cell(nc)
+    a_ms = statistics.mean(ka)
+    b_ms = statistics.mean(kb)
+    peak, peak_src = load_peaks()
+    achieved = a_b * cells_local / (a_ms / 1e3) / 1e9
+    iter_gbs = (a_b + b_b) * cells / (t_ms / 1e3 / iters_total) / 1e9
+    traffic = None
+    prof_json = os.path.join(ROOT, "profiles", f"ncu_{args.config}_kernelA.json")
+    if os.path.exists(prof_json):
+        with open(prof_json) as fh:
+            traffic = json.load(fh).get("dram_bytes_per_launch")
+
+    # e2e: the same step through the C ABI with HOST buffers (pinned): the
+    # library stages kappa, c, rhs, x0 to the device and copies x back.
+    e2e = None
+    if not args.no_e2e:
+        pin = lambda a: torch.from_numpy(np.ascontiguousarray(a)).pin_memory()
+        hk, hc, hf, hx0 = pin(prob.kappa[sl]), pin(prob.c[sl]), rhs.cpu().pin_memory(), \
+            pin(prob.x0[:, sl])
+        hx = hx0.clone().pin_memory()
+        ksteps = max(1, min(args.steps, 2))
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        h0, h1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        h0.record(stream)
+        e2e_iters = 0
+        for _ in range(ksteps):
+            op.update(hk, hc)
+            hx.copy_(hx0)
+            st, it, rel, _ = op.solve(hf, hx, args.tol, maxit)
+            e2e_iters += it
+        h1.record(stream)
+        torch.cuda.synchronize()
+        te = h0.elapsed_time(h1)
+        if world > 1:
+            tt = torch.tensor([te], device=dev, dtype=torch.float64)
+            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+            te = float(tt.item())
+        h2d = (2 + 2 * nc) * cells_local * 8
+        e2e = {"value": e2e_iters / (te / 1e3), "unit": UNIT, "h2d_bytes_per_step": h2d,
+               "d2h_bytes_per_step": nc * cells_local * 8,
+               "note": "pinned host kappa, c, rhs, x0 -> device inside the timed region; x -> host"}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        cores = cpu_cores()
+        v, per = oracle_sample(prob, args.cpu_iters, cores)
+        cpu = {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle",
+               "sample": f"{args.config} full grid, {args.cpu_iters} fixed oracle PCG iterations "
+                         f"(setup subtracted via a 1-iteration run); {per:.3f} s/iteration"}
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": t_ms / args.steps,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
+            "dtype": "f64", "data": "synthetic",
+            "config": {"workload": args.config, "grid": [nr, nt, np_], "ncomp": nc,
+                       "cells": cells, "tol": args.tol, "iters_per_solve": iters_per_solve,
+                       "parallelism": f"r-slab x{world}",
+                       "l2": "inputs > L2 (268 MB per field vs 126 MB); no flush",
+                       "step": "mas_op_update + x:=x0 + mas_pcg_solve"},
+            "roofline": {"bound": "hbm", "kernel": "k_stencil<PCGA> (kernel A)",
+                         "achieved": achieved, "peak": peak, "unit": "GB/s",
+                         "frac": achieved / peak, "traffic": traffic,
+                         "alg_bytes_per_cell": a_b, "avg_ms": a_ms, "peak_source": peak_src},
+            "kernels": {"A_ms": a_ms, "B_ms": b_ms,
+                        "A_GBs": achieved,
+                        "B_GBs": b_b * cells_local / (b_ms / 1e3) / 1e9,
+                        "iter_alg_GBs": iter_gbs, "iter_frac": iter_gbs / peak,
+                        "alg_bytes_per_cell_iter": a_b + b_b},
+            "e2e": e2e,
+            "gpu_launches": launches,
+            "clocks": clk,
+            "cpu_baseline": cpu,
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -1,0 +1,179 @@
+/*
+ * mas_pcg.h — C ABI of the B200-native MAS implicit-parabolic PCG library.
+ *
+ * What the library computes.  The MAS solar MHD code (Caplan, Stulajter &
+ * Linker 2023, PAPER.md) uses "a logically rectangular non-uniform staggered
+ * spherical grid and finite-difference discretizations with a combination of
+ * explicit and implicit time-stepping methods" and is "highly memory-bound"
+ * (§III).  Its hot loop is the "viscosity solver iterations" with
+ * GPU peer-to-peer halo exchanges (Fig. 4; §V-C),
+ * i.e. a Krylov solve of the implicit parabolic operators (ref. [25],
+ * P:1212-1216).  The paper gives no formula; the operator, boundary handling,
+ * preconditioner and stopping rule are the readings R1..R16 of DESIGN.md §3
+ * (SURVEY.md §8(c)), summarised here:
+ *
+ *   (L u)_P = c_P u_P + (1/V_P) sum_{faces f of P} G_f (u_P - u_N(f))
+ *   G_f = kappa_f g_f,  kappa_f = (kappa_P + kappa_N)/2,  midpoint FD metrics
+ *   periodic phi, zero-flux pole / theta-wall faces, r-faces Dirichlet
+ *   (homogeneous, half-cell distance) or Neumann;
+ *   <a,b> = sum_m sum_P V_P a_mP b_mP;  Jacobi (diagonal) preconditioner;
+ *   stop when ||r_k||_V <= tol * ||f||_V.
+ *
+ * Conventions for every call:
+ *   - Per-cell arrays are fp64, C order [comp][i=r][j=theta][k=phi] (phi
+ *     fastest), interior cells of the caller's LOCAL r-slab only (no ghosts),
+ *     16-byte aligned.  Pointers may be device pointers or host pointers
+ *     (pageable or pinned); host pointers are staged through library-owned
+ *     device buffers, device pointers are used in place.
+ *   - 1-D mesh arrays are host pointers, copied at create.
+ *   - Handles are opaque and library-owned.  After a call returns the library
+ *     keeps no user pointer.
+ *   - Setup/update/apply/rhs calls are asynchronous on the given stream;
+ *     mas_pcg_solve returns when the solve is complete (it reports the
+ *     iteration count).  Stream 0 means the legacy default stream.
+ *   - No exception crosses the ABI.  On failure the status is returned and
+ *     mas_last_error() gives a thread-local detail string.
+ *   - With a mas_dist_t (multi-GPU, one process per GPU, r-slab
+ *     decomposition), every call is collective over the ranks: all ranks call
+ *     the same functions in the same order.
+ */
+#ifndef MAS_PCG_H
+#define MAS_PCG_H
+
+#include <cuda_runtime_api.h>
+
+#if defined(__GNUC__)
+#define MAS_API __attribute__((visibility("default")))
+#else
+#define MAS_API
+#endif
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct mas_grid mas_grid_t;
+typedef struct mas_op mas_op_t;
+
+typedef enum {
+    MAS_OK = 0,
+    MAS_NOT_CONVERGED = 1, /* warning: x holds the last iterate               */
+    MAS_ERR_ARG = 2,       /* invalid argument / mesh / coefficient           */
+    MAS_ERR_CUDA = 3,
+    MAS_ERR_NCCL = 4,
+    MAS_ERR_NOMEM = 5,
+    MAS_ERR_BREAKDOWN = 6  /* <p, L p>_V <= 0 or non-finite                    */
+} mas_status_t;
+
+typedef enum { MAS_BC_DIRICHLET = 0, MAS_BC_NEUMANN = 1 } mas_bc_t;
+enum { MAS_POLE_NORTH = 1, MAS_POLE_SOUTH = 2 };
+
+/* Multi-GPU description.  NULL => single GPU.  nccl_id: 128 bytes from
+ * mas_comm_unique_id() on rank 0, broadcast by the caller (e.g. with
+ * torch.distributed).  The current CUDA device is used. */
+typedef struct {
+    int nranks;
+    int rank;
+    unsigned char nccl_id[128];
+} mas_dist_t;
+
+/* Rank 0 only: a fresh NCCL unique id for mas_dist_t.nccl_id. */
+MAS_API mas_status_t mas_comm_unique_id(unsigned char out[128]);
+
+/* Create the grid (reading R1: the node/"main" mesh = cell faces, the
+ * half mesh = cell centres; "staggered spherical grid").
+ *   r_node[nr+1], r_half[nr], t_node[nt+1], t_half[nt], p_node[np+1],
+ *   p_half[np]: strictly increasing, half[i] in (node[i], node[i+1]).
+ *   t_node within [0, pi]; MAS_POLE_NORTH requires t_node[0] == 0,
+ *   MAS_POLE_SOUTH requires |t_node[nt] - pi| <= 4 eps.  Pole faces and
+ *   non-pole theta walls carry no flux (R5).
+ *   periodic_phi must be 1 and p_node[np]-p_node[0] must equal 2 pi to
+ *   1e-12 relative (R7); np must be even (16-byte phi pairs).
+ *   nr >= nranks.  On a mas_dist_t each rank owns the r-slab given by
+ *   mas_grid_local_extent (rank p: nr/P + (p < nr%P) planes).
+ * Errors: MAS_ERR_ARG (validation; checked before any device work),
+ *         MAS_ERR_CUDA, MAS_ERR_NCCL, MAS_ERR_NOMEM. */
+MAS_API mas_status_t mas_grid_create(int nr, int nt, int np,
+                             const double* r_node, const double* r_half,
+                             const double* t_node, const double* t_half,
+                             const double* p_node, const double* p_half,
+                             int pole_flags, int periodic_phi,
+                             const mas_dist_t* dist, mas_grid_t** out);
+
+/* First global r-plane and number of planes owned by this rank. */
+MAS_API mas_status_t mas_grid_local_extent(const mas_grid_t* g, int* i0, int* nr_local);
+
+MAS_API mas_status_t mas_grid_destroy(mas_grid_t* g);
+
+/* Set up the operator of ncomp (1: conduction, 3: viscosity, R13)
+ * uncoupled components sharing kappa (>= 0) and mass c (>= 0; NULL => 0),
+ * both [nr_local][nt][np].  Copies kappa and c, computes the Jacobi
+ * diagonal D = c + (1/V) sum_f G_f (R8) and exchanges the static kappa / D
+ * seams once.  bc_r_inner / bc_r_outer: r-boundary conditions (R3).
+ * Errors: MAS_ERR_ARG if ncomp not 1 or 3, a coefficient is negative or
+ * non-finite, or some D_P <= 0 (checked on the device; this call then
+ * synchronises the stream). */
+MAS_API mas_status_t mas_op_setup(mas_grid_t* g, int ncomp, const double* kappa,
+                          const double* mass, mas_bc_t bc_r_inner,
+                          mas_bc_t bc_r_outer, cudaStream_t stream,
+                          mas_op_t** out);
+
+/* Replace kappa and c (e.g. kappa = T^{5/2} each implicit step); same checks. */
+MAS_API mas_status_t mas_op_update(mas_op_t* op, const double* kappa, const double* mass,
+                           cudaStream_t stream);
+
+/* y = L x with homogeneous boundary conditions.  x, y: [ncomp][nr_local][nt][np]. */
+MAS_API mas_status_t mas_op_apply(const mas_op_t* op, const double* x, double* y,
+                          cudaStream_t stream);
+
+/* Jacobi diagonal D (before inversion), [nr_local][nt][np]. */
+MAS_API mas_status_t mas_op_diag(const mas_op_t* op, double* D, cudaStream_t stream);
+
+/* f += (1/V_P) G_b u_b on Dirichlet r-faces.  ub_inner / ub_outer:
+ * [ncomp][nt][np] boundary values or NULL (homogeneous); ignored on a
+ * Neumann boundary and on ranks that do not own that boundary. */
+MAS_API mas_status_t mas_op_dirichlet_rhs(const mas_op_t* op, const double* ub_inner,
+                                  const double* ub_outer, double* f_inout,
+                                  cudaStream_t stream);
+
+/* <a,b>_V over all ranks (R9).  Synchronises the stream. */
+MAS_API mas_status_t mas_op_dot(const mas_op_t* op, const double* a, const double* b,
+                        double* out, cudaStream_t stream);
+
+/* Jacobi-PCG solve of L x = rhs (R10-R12): x in = x0, out = solution.
+ *   tol >= 0: stop when ||r_k||_V <= tol ||rhs||_V (k = 0 included);
+ *   maxit >= 0: at most maxit L*p products.
+ *   iters: products used; relres: ||r||_V/||rhs||_V (recursive residual);
+ *   res_hist: NULL or host array of maxit+1 doubles, ||r_k||_V, k=0..iters.
+ * Returns MAS_OK, MAS_NOT_CONVERGED (x = last iterate) or MAS_ERR_BREAKDOWN
+ * (x = iterate before the breaking step), or an error.  rhs == 0 gives
+ * x = 0, iters = 0.  Blocks until done. */
+MAS_API mas_status_t mas_pcg_solve(const mas_op_t* op, const double* rhs, double* x,
+                           double tol, int maxit, int* iters, double* relres,
+                           double* res_hist, cudaStream_t stream);
+
+/* Kernel launches issued by the last mas_pcg_solve on this op (its CUDA path
+ * evidence; includes early-exit launches after convergence). */
+MAS_API long long mas_op_launch_count(const mas_op_t* op);
+
+/* Per-kernel timing of mas_pcg_solve: when on, every kernel A / kernel B
+ * launch of a solve is bracketed by CUDA events on the solve stream. */
+MAS_API mas_status_t mas_op_set_profiling(mas_op_t* op, int on);
+
+/* Average device time (ms) of kernel A (fused p-update + stencil + <p,q>)
+ * and kernel B (r-update + Jacobi + two dots) over the iterations 1..iters
+ * of the last profiled solve; n = number of iterations averaged. */
+MAS_API mas_status_t mas_op_kernel_times(const mas_op_t* op, double* a_ms, double* b_ms, int* n);
+
+MAS_API mas_status_t mas_op_destroy(mas_op_t* op);
+
+MAS_API const char* mas_status_string(mas_status_t s);
+MAS_API const char* mas_last_error(void);
+
+/* Library/build identification: "maspcg <version> sm_100a". */
+MAS_API const char* mas_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* MAS_PCG_H */

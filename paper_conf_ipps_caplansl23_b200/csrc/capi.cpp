@@ -1,0 +1,684 @@
+// capi.cpp — the extern "C" boundary (include/mas_pcg.h) and the PCG driver.
+//
+// Host logic only: argument checking, device buffers, the iteration loop
+// that enqueues kernel A / kernel B (kernels.cu) with NCCL allreduces and
+// seam exchanges between them (multi-GPU), and the convergence handshake.
+// The host never sees alpha/beta/residuals during the solve: they live in
+// PcgState on the device (PAPER.md lesson: avoid host involvement and launch
+// gaps; asynchronous launches).
+#include <cuda_runtime.h>
+
+#include <cmath>
+#include <cstring>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "grid.h"
+
+namespace mas {
+
+static thread_local std::string g_last_error;
+void set_last_error(const std::string& msg) { g_last_error = msg; }
+
+#define CU(call)                                                                        \
+    do {                                                                                \
+        cudaError_t e_ = (call);                                                        \
+        if (e_ != cudaSuccess) {                                                        \
+            set_last_error(std::string(#call) + ": " + cudaGetErrorString(e_));         \
+            return MAS_ERR_CUDA;                                                        \
+        }                                                                               \
+    } while (0)
+
+#define ST(call)                                   \
+    do {                                           \
+        mas_status_t s_ = (call);                  \
+        if (s_ != MAS_OK) return s_;               \
+    } while (0)
+
+static mas_status_t arg_error(const std::string& why) {
+    set_last_error(why);
+    return MAS_ERR_ARG;
+}
+
+static bool is_device_ptr(const void* p) {
+    cudaPointerAttributes at;
+    if (cudaPointerGetAttributes(&at, p) != cudaSuccess) {
+        cudaGetLastError();
+        return false;
+    }
+    return at.type == cudaMemoryTypeDevice || at.type == cudaMemoryTypeManaged;
+}
+
+template <class T>
+static mas_status_t dmalloc(T** p, size_t n) {
+    if (n == 0) { *p = nullptr; return MAS_OK; }
+    cudaError_t e = cudaMalloc(reinterpret_cast<void**>(p), n * sizeof(T));
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        set_last_error(std::string("cudaMalloc: ") + cudaGetErrorString(e));
+        return e == cudaErrorMemoryAllocation ? MAS_ERR_NOMEM : MAS_ERR_CUDA;
+    }
+    return MAS_OK;
+}
+
+}  // namespace mas
+
+using namespace mas;
+
+struct mas_op {
+    mas_grid* g = nullptr;
+    int ncomp = 1;
+    mas_bc_t bci = MAS_BC_DIRICHLET, bco = MAS_BC_NEUMANN;
+    long long Nl = 0;           // local cells per component
+    double *kappa = nullptr, *c = nullptr, *dinv = nullptr;
+    double *kg = nullptr;       // kappa ghosts [2][plane] (lo, hi)
+    double *dg = nullptr;       // dinv ghosts
+    double *wR = nullptr;       // [2*nl] bc-folded radial tables (wRm, wRp)
+    Geo geo{};
+    // PCG work vectors [ncomp][nl][plane]
+    double *r = nullptr, *p[2] = {nullptr, nullptr}, *q = nullptr;
+    double *rg = nullptr;       // r ghosts [2][ncomp][plane]
+    double *pg[2] = {nullptr, nullptr};
+    double *xg = nullptr;       // x ghosts (init residual)
+    double *stage_a = nullptr, *stage_b = nullptr;  // host-pointer staging
+    PcgState* st = nullptr;
+    double* hist = nullptr;     // [3][cap]: rho, sigma, rr
+    int hist_cap = 0;
+    Scratch scr{};
+    double* dot_out = nullptr;
+    int* bad = nullptr;
+    int* host_flag = nullptr;   // mapped pinned
+    int* host_flag_dev = nullptr;
+    int chunk = 16;
+    int b_blocks = 0;
+    int max_blocks = 0;
+    cudaEvent_t ev[2] = {nullptr, nullptr};
+    long long launches = 0;
+    // optional per-kernel timing of the solve (CUDA events on its stream)
+    int prof = 0;
+    std::vector<cudaEvent_t> pev;  // 4 per iteration: A start/end, B start/end
+    double prof_a_ms = 0.0, prof_b_ms = 0.0, prof_init_ms = 0.0;
+    int prof_n = 0;
+};
+
+extern "C" {
+
+const char* mas_version(void) { return "maspcg 0.1 sm_100a"; }
+
+const char* mas_status_string(mas_status_t s) {
+    switch (s) {
+        case MAS_OK: return "ok";
+        case MAS_NOT_CONVERGED: return "not converged (x holds the last iterate)";
+        case MAS_ERR_ARG: return "invalid argument";
+        case MAS_ERR_CUDA: return "CUDA error";
+        case MAS_ERR_NCCL: return "NCCL error";
+        case MAS_ERR_NOMEM: return "out of device memory";
+        case MAS_ERR_BREAKDOWN: return "PCG breakdown (<p,Lp> <= 0 or non-finite)";
+    }
+    return "unknown status";
+}
+
+const char* mas_last_error(void) { return g_last_error.c_str(); }
+
+mas_status_t mas_comm_unique_id(unsigned char out[128]) {
+    if (!out) return arg_error("null out");
+    return comm_unique_id(out);
+}
+
+mas_status_t mas_grid_create(int nr, int nt, int np, const double* r_node, const double* r_half,
+                             const double* t_node, const double* t_half, const double* p_node,
+                             const double* p_half, int pole_flags, int periodic_phi,
+                             const mas_dist_t* dist, mas_grid_t** out) {
+    if (!out) return arg_error("null out");
+    *out = nullptr;
+    const int nranks = dist ? dist->nranks : 1;
+    const int rank = dist ? dist->rank : 0;
+    if (dist && (rank < 0 || rank >= nranks)) return arg_error("bad rank");
+    std::string why;
+    if (!validate_mesh(nr, nt, np, r_node, r_half, t_node, t_half, p_node, p_half, pole_flags,
+                       periodic_phi, nranks, &why))
+        return arg_error(why);
+    mas_grid* g = new (std::nothrow) mas_grid();
+    if (!g) return MAS_ERR_NOMEM;
+    g->nr = nr; g->nt = nt; g->np = np;
+    g->pole_flags = pole_flags;
+    g->nranks = nranks; g->rank = rank;
+    g->rF.assign(r_node, r_node + nr + 1); g->rC.assign(r_half, r_half + nr);
+    g->tF.assign(t_node, t_node + nt + 1); g->tC.assign(t_half, t_half + nt);
+    g->pF.assign(p_node, p_node + np + 1); g->pC.assign(p_half, p_half + np);
+    partition(nr, nranks, rank, &g->i0, &g->nl);
+    build_tables(g);
+    if (cudaGetDevice(&g->device) != cudaSuccess) {
+        cudaGetLastError();
+        delete g;
+        set_last_error("no CUDA device");
+        return MAS_ERR_CUDA;
+    }
+    // device tables: [irc2 vr](nl) [wTm wTp isc2 vt](nt) [wPm wPp vp](np)
+    const Tables& T = g->tab;
+    std::vector<double> h;
+    for (auto* v : {&T.irc2, &T.vr, &T.wTm, &T.wTp, &T.isc2, &T.vt, &T.wPm, &T.wPp, &T.vp})
+        h.insert(h.end(), v->begin(), v->end());
+    mas_status_t s = dmalloc(&g->d_tab, h.size());
+    if (s != MAS_OK) { delete g; return s; }
+    if (cudaMemcpy(g->d_tab, h.data(), h.size() * sizeof(double), cudaMemcpyHostToDevice) !=
+        cudaSuccess) {
+        cudaFree(g->d_tab);
+        delete g;
+        set_last_error("cudaMemcpy tables");
+        return MAS_ERR_CUDA;
+    }
+    if (dist && nranks > 1) {
+        s = comm_create(dist, &g->comm);
+        if (s != MAS_OK) { cudaFree(g->d_tab); delete g; return s; }
+    }
+    *out = g;
+    return MAS_OK;
+}
+
+mas_status_t mas_grid_local_extent(const mas_grid_t* g, int* i0, int* nr_local) {
+    if (!g || !i0 || !nr_local) return arg_error("null argument");
+    *i0 = g->i0;
+    *nr_local = g->nl;
+    return MAS_OK;
+}
+
+mas_status_t mas_grid_destroy(mas_grid_t* g) {
+    if (!g) return MAS_OK;
+    if (g->d_tab) cudaFree(g->d_tab);
+    comm_destroy(g->comm);
+    delete g;
+    return MAS_OK;
+}
+
+}  // extern "C"
+
+// ---------------------------------------------------------------------------
+// op internals
+// ---------------------------------------------------------------------------
+static Halo halo_of(const mas_op* op, const double* in, const double* ghosts, int ncomp) {
+    Halo h;
+    h.in = in;
+    const long long plane = op->geo.plane;
+    h.glo = (ghosts && !op->geo.glob_lo) ? ghosts : nullptr;
+    h.ghi = (ghosts && !op->geo.glob_hi) ? ghosts + (long long)ncomp * plane : nullptr;
+    return h;
+}
+
+// copy coefficients in (host or device pointers), compute D and 1/D, exchange
+// the static kappa / dinv seams, check the coefficients on the device.
+static mas_status_t op_load(mas_op* op, const double* kappa, const double* mass, cudaStream_t s,
+                            double* D_out) {
+    const size_t bytes = op->Nl * sizeof(double);
+    CU(cudaMemcpyAsync(op->kappa, kappa, bytes, cudaMemcpyDefault, s));
+    if (mass)
+        CU(cudaMemcpyAsync(op->c, mass, bytes, cudaMemcpyDefault, s));
+    else
+        CU(cudaMemsetAsync(op->c, 0, bytes, s));
+    const long long plane = op->geo.plane;
+    if (op->g->comm)
+        ST(comm_seams(op->g->comm, op->kappa, 1, op->g->nl, plane, op->kg, op->kg + plane, s));
+    CU(cudaMemsetAsync(op->bad, 0, sizeof(int), s));
+    CU(launch_diag(op->geo, halo_of(op, op->kappa, op->kg, 1), op->c, D_out, op->dinv, op->bad, s));
+    if (op->g->comm)
+        ST(comm_seams(op->g->comm, op->dinv, 1, op->g->nl, plane, op->dg, op->dg + plane, s));
+    int bad = 0;
+    CU(cudaMemcpyAsync(&bad, op->bad, sizeof(int), cudaMemcpyDeviceToHost, s));
+    CU(cudaStreamSynchronize(s));
+    if (op->g->comm) {  // agree on the verdict across ranks
+        double* d = op->dot_out;
+        double hb = bad;
+        CU(cudaMemcpyAsync(d, &hb, sizeof(double), cudaMemcpyHostToDevice, s));
+        ST(comm_allreduce(op->g->comm, d, 1, s));
+        CU(cudaMemcpyAsync(&hb, d, sizeof(double), cudaMemcpyDeviceToHost, s));
+        CU(cudaStreamSynchronize(s));
+        bad = hb != 0.0;
+    }
+    if (bad) return arg_error("kappa/c negative or non-finite, or Jacobi diagonal D <= 0");
+    return MAS_OK;
+}
+
+static void op_free(mas_op* op) {
+    if (!op) return;
+    for (double* p : {op->kappa, op->c, op->dinv, op->kg, op->dg, op->wR, op->r, op->p[0], op->p[1],
+                      op->q, op->rg, op->pg[0], op->pg[1], op->xg, op->stage_a, op->stage_b,
+                      op->hist, op->dot_out, op->scr.partials})
+        if (p) cudaFree(p);
+    if (op->st) cudaFree(op->st);
+    if (op->scr.ticket) cudaFree(op->scr.ticket);
+    if (op->bad) cudaFree(op->bad);
+    if (op->host_flag) cudaFreeHost(op->host_flag);
+    for (auto& e : op->ev)
+        if (e) cudaEventDestroy(e);
+    for (auto& e : op->pev) cudaEventDestroy(e);
+    delete op;
+}
+
+static mas_status_t ensure_hist(mas_op* op, int maxit) {
+    if (op->hist_cap >= maxit + 2) return MAS_OK;
+    if (op->hist) cudaFree(op->hist);
+    op->hist = nullptr;
+    op->hist_cap = 0;
+    ST(dmalloc(&op->hist, 3 * (size_t)(maxit + 2)));
+    op->hist_cap = maxit + 2;
+    return MAS_OK;
+}
+
+static mas_status_t ensure_prof_events(mas_op* op, int k) {
+    while (op->pev.size() < 4 * (size_t)k) {
+        cudaEvent_t e;
+        CU(cudaEventCreate(&e));
+        op->pev.push_back(e);
+    }
+    return MAS_OK;
+}
+
+static mas_status_t ensure_stage(mas_op* op) {
+    if (op->stage_a) return MAS_OK;
+    ST(dmalloc(&op->stage_a, op->ncomp * op->Nl));
+    ST(dmalloc(&op->stage_b, op->ncomp * op->Nl));
+    return MAS_OK;
+}
+
+extern "C" {
+
+mas_status_t mas_op_setup(mas_grid_t* g, int ncomp, const double* kappa, const double* mass,
+                          mas_bc_t bc_r_inner, mas_bc_t bc_r_outer, cudaStream_t stream,
+                          mas_op_t** out) {
+    if (!out) return arg_error("null out");
+    *out = nullptr;
+    if (!g || !kappa) return arg_error("null grid or kappa");
+    if (ncomp != 1 && ncomp != 3) return arg_error("ncomp must be 1 or 3");
+    if ((bc_r_inner != MAS_BC_DIRICHLET && bc_r_inner != MAS_BC_NEUMANN) ||
+        (bc_r_outer != MAS_BC_DIRICHLET && bc_r_outer != MAS_BC_NEUMANN))
+        return arg_error("bad boundary condition");
+    mas_op* op = new (std::nothrow) mas_op();
+    if (!op) return MAS_ERR_NOMEM;
+    op->g = g;
+    op->ncomp = ncomp;
+    op->bci = bc_r_inner;
+    op->bco = bc_r_outer;
+    const int nl = g->nl, nt = g->nt, np = g->np;
+    const long long plane = (long long)nt * np;
+    op->Nl = (long long)nl * plane;
+    const bool multi = g->comm != nullptr;
+    mas_status_t s;
+#define TRY(x)                         \
+    do {                               \
+        s = (x);                       \
+        if (s != MAS_OK) {             \
+            op_free(op);               \
+            return s;                  \
+        }                              \
+    } while (0)
+    TRY(dmalloc(&op->kappa, op->Nl));
+    TRY(dmalloc(&op->c, op->Nl));
+    TRY(dmalloc(&op->dinv, op->Nl));
+    TRY(dmalloc(&op->wR, 2 * (size_t)nl));
+    TRY(dmalloc(&op->r, ncomp * op->Nl));
+    TRY(dmalloc(&op->p[0], ncomp * op->Nl));
+    TRY(dmalloc(&op->p[1], ncomp * op->Nl));
+    TRY(dmalloc(&op->q, ncomp * op->Nl));
+    if (multi) {
+        TRY(dmalloc(&op->kg, 2 * plane));
+        TRY(dmalloc(&op->dg, 2 * plane));
+        TRY(dmalloc(&op->rg, 2 * ncomp * plane));
+        TRY(dmalloc(&op->pg[0], 2 * ncomp * plane));
+        TRY(dmalloc(&op->pg[1], 2 * ncomp * plane));
+        TRY(dmalloc(&op->xg, 2 * ncomp * plane));
+    }
+    TRY(dmalloc(&op->st, 1));
+    TRY(dmalloc(&op->dot_out, 1));
+    TRY(dmalloc(&op->bad, 1));
+    TRY(ensure_hist(op, 64));
+    // geometry with the boundary conditions folded into the radial tables:
+    // a Neumann face gets weight 0; a Dirichlet face keeps its weight and the
+    // kernels use kappa_ghost = kappa_P, u_ghost = 0 (R3).
+    {
+        std::vector<double> w(2 * nl);
+        for (int il = 0; il < nl; il++) {
+            w[il] = g->tab.wRm[il];
+            w[nl + il] = g->tab.wRp[il];
+        }
+        if (g->i0 == 0 && bc_r_inner == MAS_BC_NEUMANN) w[0] = 0.0;
+        if (g->i0 + nl == g->nr && bc_r_outer == MAS_BC_NEUMANN) w[2 * nl - 1] = 0.0;
+        if (cudaMemcpy(op->wR, w.data(), w.size() * sizeof(double), cudaMemcpyHostToDevice) !=
+            cudaSuccess) {
+            op_free(op);
+            set_last_error("cudaMemcpy wR");
+            return MAS_ERR_CUDA;
+        }
+    }
+    Geo& G = op->geo;
+    G.nl = nl; G.nt = nt; G.np = np; G.plane = plane;
+    G.glob_lo = g->i0 == 0;
+    G.glob_hi = g->i0 + nl == g->nr;
+    G.wRm = op->wR;
+    G.wRp = op->wR + nl;
+    const double* t = g->d_tab;
+    G.irc2 = t; t += nl;
+    G.vr = t; t += nl;
+    G.wTm = t; t += nt;
+    G.wTp = t; t += nt;
+    G.isc2 = t; t += nt;
+    G.vt = t; t += nt;
+    G.wPm = t; t += np;
+    G.wPp = t; t += np;
+    G.vp = t;
+    op->chunk = nl >= 64 ? 16 : (nl >= 16 ? 8 : 4);
+    op->max_blocks = stencil_blocks(G, op->chunk);
+    op->b_blocks = 148 * 8;
+    if (op->b_blocks > op->max_blocks) op->max_blocks = op->b_blocks;
+    TRY(dmalloc(&op->scr.partials, 4 * (size_t)op->max_blocks));
+    TRY(dmalloc(&op->scr.ticket, 8));
+    if (cudaMemset(op->scr.ticket, 0, 8 * sizeof(unsigned)) != cudaSuccess ||
+        cudaHostAlloc(reinterpret_cast<void**>(&op->host_flag), sizeof(int), cudaHostAllocMapped) !=
+            cudaSuccess ||
+        cudaHostGetDevicePointer(reinterpret_cast<void**>(&op->host_flag_dev), op->host_flag, 0) !=
+            cudaSuccess ||
+        cudaEventCreateWithFlags(&op->ev[0], cudaEventDisableTiming) != cudaSuccess ||
+        cudaEventCreateWithFlags(&op->ev[1], cudaEventDisableTiming) != cudaSuccess) {
+        cudaGetLastError();
+        op_free(op);
+        set_last_error("device scratch setup failed");
+        return MAS_ERR_CUDA;
+    }
+    TRY(op_load(op, kappa, mass, stream, nullptr));
+#undef TRY
+    *out = op;
+    return MAS_OK;
+}
+
+mas_status_t mas_op_update(mas_op_t* op, const double* kappa, const double* mass,
+                           cudaStream_t stream) {
+    if (!op || !kappa) return arg_error("null op or kappa");
+    return op_load(op, kappa, mass, stream, nullptr);
+}
+
+mas_status_t mas_op_diag(const mas_op_t* op_c, double* D, cudaStream_t stream) {
+    mas_op* op = const_cast<mas_op*>(op_c);
+    if (!op || !D) return arg_error("null argument");
+    double* Dd = D;
+    const bool host = !is_device_ptr(D);
+    if (host) {
+        ST(ensure_stage(op));
+        Dd = op->stage_b;
+    }
+    CU(cudaMemsetAsync(op->bad, 0, sizeof(int), stream));
+    CU(launch_diag(op->geo, halo_of(op, op->kappa, op->kg, 1), op->c, Dd, op->dinv, op->bad, stream));
+    if (host) {
+        CU(cudaMemcpyAsync(D, Dd, op->Nl * sizeof(double), cudaMemcpyDeviceToHost, stream));
+        CU(cudaStreamSynchronize(stream));
+    }
+    return MAS_OK;
+}
+
+mas_status_t mas_op_apply(const mas_op_t* op_c, const double* x, double* y, cudaStream_t stream) {
+    mas_op* op = const_cast<mas_op*>(op_c);
+    if (!op || !x || !y) return arg_error("null argument");
+    const size_t bytes = op->ncomp * op->Nl * sizeof(double);
+    const double* xd = x;
+    double* yd = y;
+    const bool hx = !is_device_ptr(x), hy = !is_device_ptr(y);
+    if (hx || hy) ST(ensure_stage(op));
+    if (hx) {
+        CU(cudaMemcpyAsync(op->stage_a, x, bytes, cudaMemcpyHostToDevice, stream));
+        xd = op->stage_a;
+    }
+    if (hy) yd = op->stage_b;
+    const long long plane = op->geo.plane;
+    if (op->g->comm)
+        ST(comm_seams(op->g->comm, xd, op->ncomp, op->g->nl, plane, op->xg,
+                      op->xg + op->ncomp * plane, stream));
+    StencilArgs a{};
+    a.g = op->geo;
+    a.chunk = op->chunk;
+    a.u = halo_of(op, xd, op->xg, op->ncomp);
+    a.kappa = halo_of(op, op->kappa, op->kg, 1);
+    a.c = op->c;
+    a.out = yd;
+    a.scr = op->scr;
+    CU(launch_stencil(MODE_APPLY, op->ncomp, a, stream));
+    if (hy) {
+        CU(cudaMemcpyAsync(y, yd, bytes, cudaMemcpyDeviceToHost, stream));
+        CU(cudaStreamSynchronize(stream));
+    }
+    return MAS_OK;
+}
+
+mas_status_t mas_op_dirichlet_rhs(const mas_op_t* op_c, const double* ub_inner,
+                                  const double* ub_outer, double* f_inout, cudaStream_t stream) {
+    mas_op* op = const_cast<mas_op*>(op_c);
+    if (!op || !f_inout) return arg_error("null argument");
+    const long long plane = op->geo.plane;
+    const size_t fbytes = op->ncomp * op->Nl * sizeof(double);
+    const size_t bbytes = op->ncomp * plane * sizeof(double);
+    const bool hf = !is_device_ptr(f_inout);
+    if (hf) ST(ensure_stage(op));
+    double* fd = hf ? op->stage_a : f_inout;
+    if (hf) CU(cudaMemcpyAsync(fd, f_inout, fbytes, cudaMemcpyHostToDevice, stream));
+    double* ubuf = nullptr;
+    for (int side = 0; side < 2; side++) {
+        const double* ub = side ? ub_outer : ub_inner;
+        const bool owns = side ? op->geo.glob_hi : op->geo.glob_lo;
+        const bool dir = (side ? op->bco : op->bci) == MAS_BC_DIRICHLET;
+        if (!ub || !owns || !dir) continue;
+        const double* ubd = ub;
+        if (!is_device_ptr(ub)) {
+            if (!ubuf) ST(dmalloc(&ubuf, op->ncomp * plane));
+            CU(cudaMemcpyAsync(ubuf, ub, bbytes, cudaMemcpyHostToDevice, stream));
+            ubd = ubuf;
+        }
+        CU(launch_dirichlet(op->geo, op->ncomp, op->kappa, ubd, side, fd, stream));
+    }
+    if (hf) CU(cudaMemcpyAsync(f_inout, fd, fbytes, cudaMemcpyDeviceToHost, stream));
+    if (ubuf || hf) CU(cudaStreamSynchronize(stream));
+    if (ubuf) cudaFree(ubuf);
+    return MAS_OK;
+}
+
+mas_status_t mas_op_dot(const mas_op_t* op_c, const double* a, const double* b, double* out,
+                        cudaStream_t stream) {
+    mas_op* op = const_cast<mas_op*>(op_c);
+    if (!op || !a || !b || !out) return arg_error("null argument");
+    const size_t bytes = op->ncomp * op->Nl * sizeof(double);
+    const double *ad = a, *bd = b;
+    if (!is_device_ptr(a) || !is_device_ptr(b)) {
+        ST(ensure_stage(op));
+        if (!is_device_ptr(a)) {
+            CU(cudaMemcpyAsync(op->stage_a, a, bytes, cudaMemcpyHostToDevice, stream));
+            ad = op->stage_a;
+        }
+        if (!is_device_ptr(b)) {
+            CU(cudaMemcpyAsync(op->stage_b, b, bytes, cudaMemcpyHostToDevice, stream));
+            bd = op->stage_b;
+        }
+    }
+    CU(launch_dot(op->geo, op->ncomp, ad, bd, op->scr, op->dot_out, op->b_blocks, stream));
+    if (op->g->comm) ST(comm_allreduce(op->g->comm, op->dot_out, 1, stream));
+    CU(cudaMemcpyAsync(out, op->dot_out, sizeof(double), cudaMemcpyDeviceToHost, stream));
+    CU(cudaStreamSynchronize(stream));
+    return MAS_OK;
+}
+
+long long mas_op_launch_count(const mas_op_t* op) { return op ? op->launches : -1; }
+
+mas_status_t mas_op_set_profiling(mas_op_t* op, int on) {
+    if (!op) return arg_error("null op");
+    op->prof = on ? 1 : 0;
+    return MAS_OK;
+}
+
+mas_status_t mas_op_kernel_times(const mas_op_t* op, double* a_ms, double* b_ms, int* n) {
+    if (!op || !a_ms || !b_ms || !n) return arg_error("null argument");
+    *a_ms = op->prof_a_ms;
+    *b_ms = op->prof_b_ms;
+    *n = op->prof_n;
+    return MAS_OK;
+}
+
+mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, double tol,
+                           int maxit, int* iters, double* relres, double* res_hist,
+                           cudaStream_t s) {
+    mas_op* op = const_cast<mas_op*>(op_c);
+    if (!op || !rhs || !x || !iters || !relres) return arg_error("null argument");
+    if (!(tol >= 0.0) || maxit < 0) return arg_error("need tol >= 0 and maxit >= 0");
+    const int nc = op->ncomp;
+    const long long plane = op->geo.plane;
+    const size_t bytes = nc * op->Nl * sizeof(double);
+    Comm* comm = op->g->comm;
+    ST(ensure_hist(op, maxit));
+    op->launches = 0;
+
+    // host buffers are staged through library-owned device memory
+    const double* fd = rhs;
+    double* xd = x;
+    const bool hf = !is_device_ptr(rhs), hx = !is_device_ptr(x);
+    if (hf || hx) ST(ensure_stage(op));
+    if (hf) {
+        CU(cudaMemcpyAsync(op->stage_a, rhs, bytes, cudaMemcpyHostToDevice, s));
+        fd = op->stage_a;
+    }
+    if (hx) {
+        CU(cudaMemcpyAsync(op->stage_b, x, bytes, cudaMemcpyHostToDevice, s));
+        xd = op->stage_b;
+    }
+
+    PcgState init{};
+    init.tol = tol;
+    init.maxit = maxit;
+    init.k = 1;
+    init.stopped = 0;
+    init.status = MAS_NOT_CONVERGED;
+    CU(cudaMemcpyAsync(op->st, &init, sizeof(init), cudaMemcpyHostToDevice, s));
+    *op->host_flag = 0;
+    double* rho_h = op->hist;
+    double* sig_h = op->hist + op->hist_cap;
+    double* rr_h = op->hist + 2 * op->hist_cap;
+
+    // a3: r = f - L x0 and the three initial dot products
+    if (comm) ST(comm_seams(comm, xd, nc, op->g->nl, plane, op->xg, op->xg + nc * plane, s));
+    StencilArgs a{};
+    a.g = op->geo;
+    a.chunk = op->chunk;
+    a.u = halo_of(op, xd, op->xg, nc);
+    a.kappa = halo_of(op, op->kappa, op->kg, 1);
+    a.dinv = halo_of(op, op->dinv, op->dg, 1);
+    a.c = op->c;
+    a.f = fd;
+    a.out = op->r;
+    a.st = op->st;
+    a.rho_hist = rho_h;
+    a.sigma_hist = sig_h;
+    a.rr_hist = rr_h;
+    a.scr = op->scr;
+    a.host_flag = op->host_flag_dev;
+    CU(launch_stencil(MODE_RESID, nc, a, s));
+    op->launches++;
+    if (comm) ST(comm_allreduce(comm, &op->st->pend_rho, 3, s));  // rho, rr, ff
+
+    StreamArgs b{};
+    b.g = op->geo;
+    b.ncomp = nc;
+    b.r = op->r;
+    b.q = op->q;
+    b.dinv = op->dinv;
+    b.st = op->st;
+    b.rho_hist = rho_h;
+    b.sigma_hist = sig_h;
+    b.rr_hist = rr_h;
+    b.scr = op->scr;
+    b.host_flag = op->host_flag_dev;
+
+    // a4: iterations.  Kernel A(k) reads k, alpha, beta and the convergence
+    // decision from PcgState; the host only keeps two iterations in flight
+    // and stops enqueueing once the device reports the stop (a decision all
+    // ranks take identically, so the collectives stay matched).
+    a.u = halo_of(op, op->r, op->rg, nc);
+    a.out = op->q;
+    a.x = xd;
+    a.f = nullptr;
+    int stop_seen_at = -1;
+    for (int k = 1; k <= maxit + 1; k++) {
+        double* pold = op->p[(k + 1) & 1];
+        double* pnew = op->p[k & 1];
+        if (comm) {
+            ST(comm_seams(comm, op->r, nc, op->g->nl, plane, op->rg, op->rg + nc * plane, s));
+            if (k > 1)
+                ST(comm_seams(comm, pold, nc, op->g->nl, plane, op->pg[(k + 1) & 1],
+                              op->pg[(k + 1) & 1] + nc * plane, s));
+        }
+        a.pold = halo_of(op, pold, op->pg[(k + 1) & 1], nc);
+        a.pnew = pnew;
+        cudaEvent_t* pe = nullptr;
+        if (op->prof) {
+            ST(ensure_prof_events(op, k));
+            pe = &op->pev[4 * (size_t)(k - 1)];
+            CU(cudaEventRecord(pe[0], s));
+        }
+        CU(launch_stencil(MODE_PCGA, nc, a, s));
+        op->launches++;
+        if (pe) CU(cudaEventRecord(pe[1], s));
+        if (comm) ST(comm_allreduce(comm, &op->st->pend_sigma, 1, s));
+        if (k <= maxit) {
+            if (pe) CU(cudaEventRecord(pe[2], s));
+            CU(launch_pcg_b(b, op->b_blocks, s));
+            op->launches++;
+            if (pe) CU(cudaEventRecord(pe[3], s));
+            if (comm) ST(comm_allreduce(comm, &op->st->pend_rho, 2, s));
+        }
+        CU(cudaEventRecord(op->ev[k & 1], s));
+        if (k >= 2) {
+            // wait for iteration k-1 to finish, then stop if the device
+            // decided at or before iteration k-1 (every rank sees the same
+            // decision at the same point, so the collectives stay matched)
+            CU(cudaEventSynchronize(op->ev[(k - 1) & 1]));
+            const int flag = *(volatile int*)op->host_flag;
+            if (flag > 0 && flag <= k - 1) {
+                stop_seen_at = k;
+                break;
+            }
+        }
+    }
+    (void)stop_seen_at;
+    CU(cudaStreamSynchronize(s));
+    PcgState fin{};
+    CU(cudaMemcpy(&fin, op->st, sizeof(fin), cudaMemcpyDeviceToHost));
+    if (!fin.stopped) {
+        set_last_error("internal: PCG loop ended without a stop decision");
+        return MAS_ERR_CUDA;
+    }
+    *iters = fin.iters;
+    *relres = fin.relres;
+    if (res_hist) {
+        // after a breakdown at iteration k only ||r_0..r_{k-1}|| exist
+        const int nh = fin.status == MAS_ERR_BREAKDOWN ? fin.iters : fin.iters + 1;
+        std::vector<double> rr(nh);
+        CU(cudaMemcpy(rr.data(), rr_h, rr.size() * sizeof(double), cudaMemcpyDeviceToHost));
+        for (int k = 0; k < nh; k++) res_hist[k] = std::sqrt(rr[k]);
+    }
+    if (op->prof) {  // average device time of the working launches 1..iters
+        double sa = 0.0, sb = 0.0;
+        int n = 0;
+        for (int k = 1; k <= fin.iters && 4 * (size_t)k <= op->pev.size(); k++, n++) {
+            float ta = 0.f, tb = 0.f;
+            CU(cudaEventElapsedTime(&ta, op->pev[4 * (k - 1)], op->pev[4 * (k - 1) + 1]));
+            CU(cudaEventElapsedTime(&tb, op->pev[4 * (k - 1) + 2], op->pev[4 * (k - 1) + 3]));
+            sa += ta;
+            sb += tb;
+        }
+        op->prof_n = n;
+        op->prof_a_ms = n ? sa / n : 0.0;
+        op->prof_b_ms = n ? sb / n : 0.0;
+    }
+    if (hx) CU(cudaMemcpy(x, xd, bytes, cudaMemcpyDeviceToHost));
+    return (mas_status_t)fin.status;
+}
+
+mas_status_t mas_op_destroy(mas_op_t* op) {
+    op_free(op);
+    return MAS_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,52 @@
+// grid.h — host-side objects behind the opaque ABI handles.
+#pragma once
+
+#include <string>
+#include <vector>
+
+#include "mas_internal.h"
+
+namespace mas {
+
+struct Tables {  // local 1-D tables, layout of Geo (mas_internal.h)
+    std::vector<double> wRm, wRp, irc2, vr, wTm, wTp, isc2, vt, wPm, wPp, vp;
+};
+
+struct Comm;  // comm.cpp (NCCL)
+
+}  // namespace mas
+
+struct mas_grid {
+    int nr = 0, nt = 0, np = 0;
+    int i0 = 0, nl = 0;
+    int pole_flags = 0;
+    int nranks = 1, rank = 0;
+    int device = 0;
+    std::vector<double> rF, rC, tF, tC, pF, pC;
+    mas::Tables tab;
+    double* d_tab = nullptr;  // device copy of the theta/phi tables + irc2/vr
+    mas::Comm* comm = nullptr;
+};
+
+namespace mas {
+
+int validate_mesh(int nr, int nt, int np, const double* rF, const double* rC, const double* tF,
+                  const double* tC, const double* pF, const double* pC, int pole_flags,
+                  int periodic_phi, int nranks, std::string* why);
+void partition(int nr, int nranks, int rank, int* i0, int* nl);
+void build_tables(mas_grid* g);
+
+// ---- comm.cpp -------------------------------------------------------------
+mas_status_t comm_unique_id(unsigned char out[128]);
+mas_status_t comm_create(const mas_dist_t* d, Comm** out);
+void comm_destroy(Comm* c);
+// sum n doubles in place over all ranks
+mas_status_t comm_allreduce(Comm* c, double* buf, int n, cudaStream_t s);
+// exchange r-seams of an ncomp-component field with interior `in`
+// ([ncomp][nl][plane]): send first/last plane to rank-1/rank+1, receive the
+// neighbours' edge planes into glo / ghi ([ncomp][plane]).
+mas_status_t comm_seams(Comm* c, const double* in, int ncomp, int nl, long long plane, double* glo,
+                        double* ghi, cudaStream_t s);
+mas_status_t comm_barrier(Comm* c, cudaStream_t s);
+
+}  // namespace mas

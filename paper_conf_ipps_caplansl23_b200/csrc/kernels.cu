@@ -1,0 +1,675 @@
+// kernels.cu — sm_100a kernels of the MAS implicit-parabolic PCG path.
+//
+// The path is HBM-bound ("highly memory-bound"; DESIGN.md
+// §5 roofline), so there are no tensor-core contractions here: every kernel
+// streams fp64 fields with 16-byte (double2) coalesced accesses along phi,
+// stages (theta,phi) plane tiles with a one-cell halo in shared memory and
+// marches along r with the r-neighbours in registers.  Kernel fusion follows
+// the paper's own lesson that OpenACC's fused, asynchronous kernels beat the
+// un-fused DC loops:
+//
+//   k_stencil<MODE_PCGA>  "kernel A":  beta, p = D^-1 r + beta p_old (also on
+//       the halo), deferred x += alpha_{k-1} p_old, q = L p, partial <p,q>_V
+//   k_pcg_b               "kernel B":  r -= alpha q, z = D^-1 r, <r,z>_V, <r,r>_V
+//   k_stencil<MODE_RESID> init:  r = f - L x, <f,f>_V, <r,r>_V, <r,D^-1 r>_V
+//   k_stencil<MODE_APPLY> y = L x (mas_op_apply)
+//
+// Scalars (alpha, beta, convergence, breakdown) never leave the device: each
+// reduction ends in a deterministic "last block" sum (fixed order, no fp64
+// atomics) whose result the next kernel reads.  See DESIGN.md §5.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdint>
+
+#include "mas_internal.h"
+
+namespace mas {
+
+constexpr int kThreads = 256;  // 8 warps
+constexpr int TJ = 8;          // theta rows per tile (one warp per row)
+constexpr int TK = 64;         // phi cells per tile (2 per lane, double2)
+constexpr int OFF = 2;         // smem column of the first tile cell (16B aligned)
+constexpr int ROW = TK + 4;    // smem row length: [pad][halo][64 cells][halo][pad]
+constexpr int HROWS = TJ + 2;  // tile rows + 2 halo rows
+
+enum { P_NORMAL = 0, P_FINAL = 1, P_ZERO = 2 };
+enum { TKT_STENCIL = 0, TKT_B = 1, TKT_DOT = 2 };
+
+// --------------------------------------------------------------------------
+// deterministic reductions
+// --------------------------------------------------------------------------
+__device__ __forceinline__ double warp_sum(double v) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_down_sync(0xffffffffu, v, o);
+    return v;  // valid in lane 0
+}
+
+// Block-reduce NS sums, publish the block partial, take a ticket.  Returns
+// true in the last block to finish, where `v` then holds the grid totals
+// (valid in thread 0), summed in a fixed order independent of scheduling.
+template <int NS>
+__device__ bool grid_reduce(double (&v)[NS], const Scratch& scr, int tkt) {
+    __shared__ double wsum[NS][kThreads / 32];
+    __shared__ bool last;
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+#pragma unroll
+    for (int s = 0; s < NS; s++) {
+        double t = warp_sum(v[s]);
+        if (lane == 0) wsum[s][w] = t;
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+#pragma unroll
+        for (int s = 0; s < NS; s++) {
+            double t = 0.0;
+            for (int q = 0; q < kThreads / 32; q++) t += wsum[s][q];
+            scr.partials[(size_t)blockIdx.x * NS + s] = t;
+        }
+        __threadfence();
+        unsigned old = atomicAdd(&scr.ticket[tkt], 1u);
+        last = (old == gridDim.x - 1);
+    }
+    __syncthreads();
+    if (!last) return false;
+    __threadfence();
+#pragma unroll
+    for (int s = 0; s < NS; s++) {
+        double t = 0.0;
+        for (unsigned b = threadIdx.x; b < gridDim.x; b += kThreads)
+            t += __ldcg(&scr.partials[(size_t)b * NS + s]);
+        t = warp_sum(t);
+        __syncthreads();
+        if (lane == 0) wsum[s][w] = t;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            double u = 0.0;
+            for (int q = 0; q < kThreads / 32; q++) u += wsum[s][q];
+            v[s] = u;
+        }
+    }
+    if (threadIdx.x == 0) scr.ticket[tkt] = 0u;
+    return true;
+}
+
+// --------------------------------------------------------------------------
+// field access
+// --------------------------------------------------------------------------
+__device__ __forceinline__ const double* plane_ptr(const Halo& h, int comp, int i, const Geo& g) {
+    if (i < 0) return h.glo + (long long)comp * g.plane;
+    if (i >= g.nl) return h.ghi + (long long)comp * g.plane;
+    return h.in + ((long long)comp * g.nl + i) * g.plane;
+}
+__device__ __forceinline__ double2 ld2(const double* p) {
+    return __ldg(reinterpret_cast<const double2*>(p));
+}
+__device__ __forceinline__ double2 dadd2(double2 a, double2 b) { return make_double2(a.x + b.x, a.y + b.y); }
+
+// The value entering the stencil at (plane i, offset off) for NC components,
+// plus kappa; PCGA also returns p_old (for the deferred x update).
+template <int MODE, int NC>
+struct Prod {
+    double2 u[NC];
+    double2 kap;
+    double2 po[NC];
+};
+
+template <int MODE, int NC>
+__device__ __forceinline__ void produce2(const StencilArgs& a, int i, long long off, bool first,
+                                         double beta, Prod<MODE, NC>& o) {
+    const Geo& g = a.g;
+    o.kap = ld2(plane_ptr(a.kappa, 0, i, g) + off);
+    if (MODE == MODE_PCGA) {
+        const double2 di = ld2(plane_ptr(a.dinv, 0, i, g) + off);
+#pragma unroll
+        for (int c = 0; c < NC; c++) {
+            const double2 r = ld2(plane_ptr(a.u, c, i, g) + off);
+            double2 z = make_double2(di.x * r.x, di.y * r.y);
+            if (!first) {
+                o.po[c] = ld2(plane_ptr(a.pold, c, i, g) + off);
+                z.x = fma(beta, o.po[c].x, z.x);
+                z.y = fma(beta, o.po[c].y, z.y);
+            } else {
+                o.po[c] = make_double2(0.0, 0.0);
+            }
+            o.u[c] = z;
+        }
+    } else {
+#pragma unroll
+        for (int c = 0; c < NC; c++) o.u[c] = ld2(plane_ptr(a.u, c, i, g) + off);
+    }
+}
+
+template <int MODE, int NC>
+__device__ __forceinline__ void produce1(const StencilArgs& a, int i, long long off, bool first,
+                                         double beta, double (&u)[NC], double& kap) {
+    const Geo& g = a.g;
+    kap = __ldg(plane_ptr(a.kappa, 0, i, g) + off);
+    if (MODE == MODE_PCGA) {
+        const double di = __ldg(plane_ptr(a.dinv, 0, i, g) + off);
+#pragma unroll
+        for (int c = 0; c < NC; c++) {
+            double z = di * __ldg(plane_ptr(a.u, c, i, g) + off);
+            if (!first) z = fma(beta, __ldg(plane_ptr(a.pold, c, i, g) + off), z);
+            u[c] = z;
+        }
+    } else {
+#pragma unroll
+        for (int c = 0; c < NC; c++) u[c] = __ldg(plane_ptr(a.u, c, i, g) + off);
+    }
+}
+
+// smem plane buffer: field f (0..NC-1 = u components, NC = kappa), row, col
+template <int NC>
+__device__ __forceinline__ double* sfield(double* buf, int f) { return buf + f * (HROWS * ROW); }
+
+// Produce plane i for the whole tile (own cells + 1-cell theta/phi halo) into
+// smem buffer `buf`; returns the own-cell product in `own`.
+template <int MODE, int NC>
+__device__ __forceinline__ void produce_tile(const StencilArgs& a, int i, double* buf, int j0, int k0,
+                                             int height, int width, bool first, double beta,
+                                             Prod<MODE, NC>& own, bool halo) {
+    const Geo& g = a.g;
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const int kc = 2 * lane;
+    if (w < height && kc < width) {
+        const long long off = (long long)(j0 + w) * g.np + k0 + kc;
+        produce2<MODE, NC>(a, i, off, first, beta, own);
+        const int idx = (1 + w) * ROW + OFF + kc;
+#pragma unroll
+        for (int c = 0; c < NC; c++) *reinterpret_cast<double2*>(sfield<NC>(buf, c) + idx) = own.u[c];
+        *reinterpret_cast<double2*>(sfield<NC>(buf, NC) + idx) = own.kap;
+    }
+    if (!halo) return;
+    if (w < 2) {  // theta halo rows: warp 0 -> j0-1, warp 1 -> j0+height
+        const int jr = (w == 0) ? 0 : height + 1;
+        const int j = j0 + jr - 1;
+        if (kc < width) {
+            const int idx = jr * ROW + OFF + kc;
+            if (j >= 0 && j < g.nt) {
+                Prod<MODE, NC> h;
+                produce2<MODE, NC>(a, i, (long long)j * g.np + k0 + kc, first, beta, h);
+#pragma unroll
+                for (int c = 0; c < NC; c++) *reinterpret_cast<double2*>(sfield<NC>(buf, c) + idx) = h.u[c];
+                *reinterpret_cast<double2*>(sfield<NC>(buf, NC) + idx) = h.kap;
+            } else {  // beyond a pole / theta wall: zero-flux face, value unused but finite
+#pragma unroll
+                for (int c = 0; c <= NC; c++)
+                    *reinterpret_cast<double2*>(sfield<NC>(buf, c) + idx) = make_double2(0.0, 0.0);
+            }
+        }
+    } else if (w == 2) {  // phi halo columns (periodic wrap)
+        const int side = lane >> 4, jr = lane & 15;
+        if (jr < height) {
+            const int k = side == 0 ? (k0 - 1 + g.np) % g.np : (k0 + width) % g.np;
+            const int col = side == 0 ? OFF - 1 : OFF + width;
+            double u[NC], kap;
+            produce1<MODE, NC>(a, i, (long long)(j0 + jr) * g.np + k, first, beta, u, kap);
+            const int idx = (1 + jr) * ROW + col;
+#pragma unroll
+            for (int c = 0; c < NC; c++) sfield<NC>(buf, c)[idx] = u[c];
+            sfield<NC>(buf, NC)[idx] = kap;
+        }
+    }
+}
+
+// --------------------------------------------------------------------------
+// the fused stencil kernel
+// --------------------------------------------------------------------------
+template <int MODE, int NC>
+__global__ void __launch_bounds__(kThreads, (NC == 1 ? 3 : 2)) k_stencil(const StencilArgs a) {
+    extern __shared__ __align__(16) double smem[];
+    constexpr int BUF = (NC + 1) * HROWS * ROW;
+    const Geo& g = a.g;
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+
+    // ---- PCG scalars (all threads read the same device values) ----------
+    int pmode = P_NORMAL;
+    bool first = false;
+    double beta = 0.0, alpha_prev = 0.0;
+    int kit = 0;
+    if (MODE == MODE_PCGA) {
+        const volatile PcgState* st = a.st;
+        if (st->stopped) return;
+        kit = st->k;
+        const double ff = st->pend_ff, rr = st->pend_rr;
+        first = (kit == 1);
+        if (kit >= 2) alpha_prev = a.rho_hist[kit - 2] / a.sigma_hist[kit - 1];
+        if (first && ff == 0.0)
+            pmode = P_ZERO;
+        else if (sqrt(rr) <= st->tol * sqrt(ff) || kit > st->maxit)
+            pmode = P_FINAL;
+        else if (!first)
+            beta = st->pend_rho / a.rho_hist[kit - 2];
+    }
+
+    // ---- work item ------------------------------------------------------
+    const int item = blockIdx.x;
+    const int tk = item % a.ntk;
+    const int tj = (item / a.ntk) % a.ntj;
+    const int ch = item / (a.ntk * a.ntj);
+    const int j0 = tj * TJ, k0 = tk * TK;
+    const int height = min(TJ, g.nt - j0), width = min(TK, g.np - k0);
+    const int ia = ch * a.chunk, ib = min(ia + a.chunk, g.nl);
+    const int kc = 2 * lane;
+    const bool own = (w < height) && (kc < width);
+    const int j = j0 + w, k = k0 + kc;
+    const long long off = (long long)j * g.np + k;
+    const long long Nl = (long long)g.nl * g.plane;
+
+    double acc[3] = {0.0, 0.0, 0.0};
+
+    if (MODE == MODE_PCGA && pmode != P_NORMAL) {
+        // final deferred update x += alpha_{k-1} p_{k-1} (or x = 0 if f == 0)
+        if (own) {
+            for (int i = ia; i < ib; i++) {
+#pragma unroll
+                for (int c = 0; c < NC; c++) {
+                    double2* xp = reinterpret_cast<double2*>(a.x + c * Nl + (long long)i * g.plane + off);
+                    if (pmode == P_ZERO) {
+                        *xp = make_double2(0.0, 0.0);
+                    } else if (kit >= 2) {
+                        const double2 po = ld2(plane_ptr(a.pold, c, i, g) + off);
+                        double2 xv = *xp;
+                        xv.x = fma(alpha_prev, po.x, xv.x);
+                        xv.y = fma(alpha_prev, po.y, xv.y);
+                        *xp = xv;
+                    }
+                }
+            }
+        }
+        double v1[1] = {0.0};
+        if (grid_reduce<1>(v1, a.scr, TKT_STENCIL) && threadIdx.x == 0) {
+            PcgState* st = a.st;
+            const double ff = st->pend_ff, rr = st->pend_rr;
+            a.rr_hist[kit - 1] = rr;
+            a.rho_hist[kit - 1] = st->pend_rho;
+            if (pmode == P_ZERO) {
+                st->iters = 0;
+                st->relres = 0.0;
+                st->status = MAS_OK;
+                a.rr_hist[0] = 0.0;
+            } else {
+                const bool conv = sqrt(rr) <= st->tol * sqrt(ff);
+                st->iters = kit - 1;
+                st->relres = sqrt(rr) / sqrt(ff);
+                st->status = conv ? MAS_OK : MAS_NOT_CONVERGED;
+            }
+            __threadfence();
+            st->stopped = 1;
+            if (a.host_flag) {
+                __threadfence_system();
+                *(volatile int*)a.host_flag = kit;
+            }
+        }
+        return;
+    }
+
+    // ---- march along r ----------------------------------------------------
+    double* buf0 = smem;
+    Prod<MODE, NC> cur, nxt;   // own-cell products at planes i (cur) and i+1 (nxt)
+    double2 um[NC], km;        // own u and kappa at plane i-1
+    double2 un[NC], kn;        // own u and kappa at plane i+1
+
+    // plane ia-1: own cell only (r-neighbour of the first plane)
+    const bool lo_ghost = (ia == 0) && g.glob_lo;
+    if (own && !lo_ghost) {
+        Prod<MODE, NC> pm;
+        produce2<MODE, NC>(a, ia - 1, off, first, beta, pm);
+#pragma unroll
+        for (int c = 0; c < NC; c++) um[c] = pm.u[c];
+        km = pm.kap;
+    }
+    produce_tile<MODE, NC>(a, ia, buf0, j0, k0, height, width, first, beta, cur, true);
+    if (lo_ghost && own) {  // global boundary ghost: u = 0, kappa_ghost = kappa_P
+#pragma unroll
+        for (int c = 0; c < NC; c++) um[c] = make_double2(0.0, 0.0);
+        km = cur.kap;
+    }
+
+    // per-cell geometry constant over the march
+    double wpm[2], wpp[2], vpk[2];
+    double wtm = 0.0, wtp = 0.0, isc = 0.0, vtj = 0.0;
+    if (own) {
+        wtm = __ldg(g.wTm + j);
+        wtp = __ldg(g.wTp + j);
+        isc = __ldg(g.isc2 + j);
+        vtj = __ldg(g.vt + j);
+#pragma unroll
+        for (int e = 0; e < 2; e++) {
+            wpm[e] = __ldg(g.wPm + k + e);
+            wpp[e] = __ldg(g.wPp + k + e);
+            vpk[e] = __ldg(g.vp + k + e);
+        }
+    }
+
+    for (int i = ia; i < ib; i++) {
+        double* bc = smem + ((i - ia) % 3) * BUF;
+        double* bn = smem + ((i + 1 - ia) % 3) * BUF;
+        const bool hi_ghost = (i + 1 == g.nl) && g.glob_hi;
+        if (!hi_ghost) {
+            // the next plane needs its halo only if it will be a stencil plane
+            produce_tile<MODE, NC>(a, i + 1, bn, j0, k0, height, width, first, beta, nxt, i + 1 < ib);
+            if (own) {
+#pragma unroll
+                for (int c = 0; c < NC; c++) un[c] = nxt.u[c];
+                kn = nxt.kap;
+            }
+        } else if (own) {
+#pragma unroll
+            for (int c = 0; c < NC; c++) un[c] = make_double2(0.0, 0.0);
+            kn = cur.kap;
+        }
+        __syncthreads();
+
+        if (own) {
+            const int idx = (1 + w) * ROW + OFF + kc;
+            const double* sk = sfield<NC>(bc, NC);
+            const double wrm = __ldg(g.wRm + i), wrp = __ldg(g.wRp + i), irc = __ldg(g.irc2 + i);
+            const double vri = __ldg(g.vr + i);
+            double2 cP = make_double2(0.0, 0.0);
+            if (a.c) cP = ld2(a.c + (long long)i * g.plane + off);
+            const long long pofs = (long long)i * g.plane + off;
+
+            double aRm[2], aRp[2], aTm[2], aTp[2], aPm[2], aPp[2], kP[2];
+            kP[0] = sk[idx];
+            kP[1] = sk[idx + 1];
+            const double kM[2] = {km.x, km.y}, kN[2] = {kn.x, kn.y};
+#pragma unroll
+            for (int e = 0; e < 2; e++) {
+                const double kp = kP[e];
+                aRm[e] = wrm * (0.5 * (kp + kM[e]));
+                aRp[e] = wrp * (0.5 * (kp + kN[e]));
+                aTm[e] = irc * wtm * (0.5 * (kp + sk[idx + e - ROW]));
+                aTp[e] = irc * wtp * (0.5 * (kp + sk[idx + e + ROW]));
+                aPm[e] = irc * isc * wpm[e] * (0.5 * (kp + sk[idx + e - 1]));
+                aPp[e] = irc * isc * wpp[e] * (0.5 * (kp + sk[idx + e + 1]));
+            }
+            const double cc[2] = {cP.x, cP.y};
+            const double V[2] = {vri * vtj * vpk[0], vri * vtj * vpk[1]};
+            double2 di = make_double2(0.0, 0.0);
+            if (MODE == MODE_RESID) di = ld2(a.dinv.in + pofs);
+
+#pragma unroll
+            for (int c = 0; c < NC; c++) {
+                const double* su = sfield<NC>(bc, c);
+                const double uM[2] = {um[c].x, um[c].y}, uN[2] = {un[c].x, un[c].y};
+                double L[2], uu[2];
+#pragma unroll
+                for (int e = 0; e < 2; e++) {
+                    const double u = su[idx + e];
+                    uu[e] = u;
+                    double s = cc[e] * u;
+                    s = fma(aRm[e], u - uM[e], s);
+                    s = fma(aRp[e], u - uN[e], s);
+                    s = fma(aTm[e], u - su[idx + e - ROW], s);
+                    s = fma(aTp[e], u - su[idx + e + ROW], s);
+                    s = fma(aPm[e], u - su[idx + e - 1], s);
+                    s = fma(aPp[e], u - su[idx + e + 1], s);
+                    L[e] = s;
+                }
+                const long long o = c * Nl + pofs;
+                if (MODE == MODE_APPLY) {
+                    *reinterpret_cast<double2*>(a.out + o) = make_double2(L[0], L[1]);
+                } else if (MODE == MODE_RESID) {
+                    const double2 f = ld2(a.f + o);
+                    const double r0 = f.x - L[0], r1 = f.y - L[1];
+                    *reinterpret_cast<double2*>(a.out + o) = make_double2(r0, r1);
+                    acc[0] += V[0] * f.x * f.x + V[1] * f.y * f.y;
+                    acc[1] += V[0] * r0 * r0 + V[1] * r1 * r1;
+                    acc[2] += V[0] * r0 * (di.x * r0) + V[1] * r1 * (di.y * r1);
+                } else {  // PCGA
+                    *reinterpret_cast<double2*>(a.out + o) = make_double2(L[0], L[1]);
+                    *reinterpret_cast<double2*>(a.pnew + o) = make_double2(uu[0], uu[1]);
+                    if (kit >= 2) {
+                        double2* xp = reinterpret_cast<double2*>(a.x + o);
+                        double2 xv = *xp;
+                        xv.x = fma(alpha_prev, cur.po[c].x, xv.x);
+                        xv.y = fma(alpha_prev, cur.po[c].y, xv.y);
+                        *xp = xv;
+                    }
+                    acc[0] += V[0] * uu[0] * L[0] + V[1] * uu[1] * L[1];
+                }
+                um[c] = make_double2(uu[0], uu[1]);
+            }
+            km = make_double2(kP[0], kP[1]);
+            cur = nxt;
+        }
+    }
+
+    // ---- reductions -------------------------------------------------------
+    if (MODE == MODE_RESID) {
+        if (grid_reduce<3>(acc, a.scr, TKT_STENCIL) && threadIdx.x == 0) {
+            PcgState* st = a.st;
+            st->pend_ff = acc[0];
+            st->pend_rr = acc[1];
+            st->pend_rho = acc[2];
+        }
+    } else if (MODE == MODE_PCGA) {
+        double v[1] = {acc[0]};
+        if (grid_reduce<1>(v, a.scr, TKT_STENCIL) && threadIdx.x == 0) {
+            PcgState* st = a.st;
+            st->pend_sigma = v[0];
+            a.rr_hist[kit - 1] = st->pend_rr;
+            a.rho_hist[kit - 1] = st->pend_rho;
+        }
+    }
+}
+
+// --------------------------------------------------------------------------
+// kernel B: r -= alpha q ; z = D^-1 r ; <r,z>_V, <r,r>_V
+// --------------------------------------------------------------------------
+template <int NC>
+__global__ void __launch_bounds__(kThreads) k_pcg_b(const StreamArgs a) {
+    const volatile PcgState* vst = a.st;
+    if (vst->stopped) return;
+    const Geo& g = a.g;
+    const int kit = vst->k;
+    const double sigma = vst->pend_sigma;
+    const bool brk = !(sigma > 0.0) || !isfinite(sigma);
+    const double alpha = a.rho_hist[kit - 1] / sigma;
+    double acc[2] = {0.0, 0.0};
+    if (!brk) {
+        const long long Nl = (long long)g.nl * g.plane;
+        const int rows = g.nl * g.nt;
+        const int half = g.np >> 1;
+        for (int row = blockIdx.x; row < rows; row += gridDim.x) {
+            const int i = row / g.nt, j = row - i * g.nt;
+            const double wrow = __ldg(g.vr + i) * __ldg(g.vt + j);
+            const long long base = (long long)row * g.np;
+            for (int h = threadIdx.x; h < half; h += kThreads) {
+                const int k = 2 * h;
+                const double2 di = ld2(a.dinv + base + k);
+                const double V0 = wrow * __ldg(g.vp + k), V1 = wrow * __ldg(g.vp + k + 1);
+                double2 r[NC], q[NC];
+#pragma unroll
+                for (int c = 0; c < NC; c++) {
+                    r[c] = ld2(a.r + c * Nl + base + k);
+                    q[c] = ld2(a.q + c * Nl + base + k);
+                }
+#pragma unroll
+                for (int c = 0; c < NC; c++) {
+                    double2 rv = r[c];
+                    rv.x = fma(-alpha, q[c].x, rv.x);
+                    rv.y = fma(-alpha, q[c].y, rv.y);
+                    *reinterpret_cast<double2*>(a.r + c * Nl + base + k) = rv;
+                    const double z0 = di.x * rv.x, z1 = di.y * rv.y;
+                    acc[0] += V0 * rv.x * z0 + V1 * rv.y * z1;
+                    acc[1] += V0 * rv.x * rv.x + V1 * rv.y * rv.y;
+                }
+            }
+        }
+    }
+    if (grid_reduce<2>(acc, a.scr, TKT_B) && threadIdx.x == 0) {
+        PcgState* st = a.st;
+        if (brk) {
+            st->iters = kit;
+            st->relres = sqrt(st->pend_rr) / sqrt(st->pend_ff);
+            st->status = MAS_ERR_BREAKDOWN;
+            a.rr_hist[kit - 1] = st->pend_rr;
+            __threadfence();
+            st->stopped = 1;
+            if (a.host_flag) {
+                __threadfence_system();
+                *(volatile int*)a.host_flag = kit;
+            }
+        } else {
+            a.sigma_hist[kit] = sigma;
+            st->pend_rho = acc[0];
+            st->pend_rr = acc[1];
+            st->k = kit + 1;
+        }
+    }
+}
+
+// --------------------------------------------------------------------------
+// setup kernels
+// --------------------------------------------------------------------------
+__device__ __forceinline__ double kap_at(const Halo& h, int i, long long off, const Geo& g) {
+    return __ldg(plane_ptr(h, 0, i, g) + off);
+}
+
+// D = c + sum_f a_f (Dirichlet faces included via kappa_ghost = kappa_P),
+// dinv = 1/D; flags negative / non-finite coefficients and D <= 0.
+__global__ void __launch_bounds__(kThreads) k_diag(const Geo g, const Halo kappa, const double* c,
+                                                   double* D, double* dinv, int* bad) {
+    const long long Nl = (long long)g.nl * g.plane;
+    for (long long P = blockIdx.x * (long long)kThreads + threadIdx.x; P < Nl;
+         P += (long long)gridDim.x * kThreads) {
+        const int i = (int)(P / g.plane);
+        const long long off = P - (long long)i * g.plane;
+        const int j = (int)(off / g.np), k = (int)(off - (long long)j * g.np);
+        const double kp = kappa.in[P];
+        const double cp = c ? c[P] : 0.0;
+        const double kim = (i == 0 && g.glob_lo) ? kp : kap_at(kappa, i - 1, off, g);
+        const double kip = (i == g.nl - 1 && g.glob_hi) ? kp : kap_at(kappa, i + 1, off, g);
+        const double kjm = j > 0 ? kappa.in[P - g.np] : 0.0;
+        const double kjp = j < g.nt - 1 ? kappa.in[P + g.np] : 0.0;
+        const int km = k == 0 ? g.np - 1 : k - 1, kq = k == g.np - 1 ? 0 : k + 1;
+        const double kkm = kappa.in[P - k + km], kkp = kappa.in[P - k + kq];
+        const double irc = g.irc2[i];
+        double s = cp;
+        s += g.wRm[i] * (0.5 * (kp + kim));
+        s += g.wRp[i] * (0.5 * (kp + kip));
+        s += irc * g.wTm[j] * (0.5 * (kp + kjm));
+        s += irc * g.wTp[j] * (0.5 * (kp + kjp));
+        s += irc * g.isc2[j] * g.wPm[k] * (0.5 * (kp + kkm));
+        s += irc * g.isc2[j] * g.wPp[k] * (0.5 * (kp + kkp));
+        if (D) D[P] = s;
+        dinv[P] = 1.0 / s;
+        const bool ok = (kp >= 0.0) && isfinite(kp) && (cp >= 0.0) && isfinite(cp) && (s > 0.0) &&
+                        isfinite(s);
+        if (!ok) atomicOr(bad, 1);
+    }
+}
+
+// f += w_b kappa_P u_b on a Dirichlet boundary plane (inner: plane 0, wRm;
+// outer: plane nl-1, wRp).
+__global__ void k_dirichlet(const Geo g, int ncomp, const double* kappa, const double* ub, int outer,
+                            double* f) {
+    const long long plane = g.plane;
+    const long long Nl = (long long)g.nl * plane;
+    const int i = outer ? g.nl - 1 : 0;
+    const double wgt = outer ? g.wRp[i] : g.wRm[i];
+    for (long long t = blockIdx.x * (long long)blockDim.x + threadIdx.x; t < plane * ncomp;
+         t += (long long)gridDim.x * blockDim.x) {
+        const int c = (int)(t / plane);
+        const long long off = t - c * plane;
+        const long long P = (long long)i * plane + off;
+        f[c * Nl + P] += wgt * kappa[P] * ub[t];
+    }
+}
+
+__global__ void __launch_bounds__(kThreads) k_dot(const Geo g, int ncomp, const double* x,
+                                                  const double* y, Scratch scr, double* out) {
+    double acc[1] = {0.0};
+    const long long Nl = (long long)g.nl * g.plane;
+    const int rows = g.nl * g.nt;
+    for (int row = blockIdx.x; row < rows; row += gridDim.x) {
+        const int i = row / g.nt, j = row - i * g.nt;
+        const double wrow = g.vr[i] * g.vt[j];
+        const long long base = (long long)row * g.np;
+        for (int k = threadIdx.x; k < g.np; k += kThreads) {
+            const double V = wrow * g.vp[k];
+            for (int c = 0; c < ncomp; c++) acc[0] += V * x[c * Nl + base + k] * y[c * Nl + base + k];
+        }
+    }
+    if (grid_reduce<1>(acc, scr, TKT_DOT) && threadIdx.x == 0) *out = acc[0];
+}
+
+// --------------------------------------------------------------------------
+// launchers
+// --------------------------------------------------------------------------
+int stencil_blocks(const Geo& g, int chunk) {
+    const int ntj = (g.nt + TJ - 1) / TJ, ntk = (g.np + TK - 1) / TK;
+    const int nch = (g.nl + chunk - 1) / chunk;
+    return ntj * ntk * nch;
+}
+
+template <int MODE, int NC>
+static cudaError_t launch_one(const StencilArgs& a0, cudaStream_t s) {
+    StencilArgs a = a0;
+    a.ntj = (a.g.nt + TJ - 1) / TJ;
+    a.ntk = (a.g.np + TK - 1) / TK;
+    a.nchunk = (a.g.nl + a.chunk - 1) / a.chunk;
+    const int smem = 3 * (NC + 1) * HROWS * ROW * (int)sizeof(double);
+    static bool attr_done = false;
+    if (!attr_done) {
+        cudaError_t e = cudaFuncSetAttribute(k_stencil<MODE, NC>,
+                                             cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+        if (e != cudaSuccess) return e;
+        attr_done = true;
+    }
+    const int blocks = a.ntj * a.ntk * a.nchunk;
+    k_stencil<MODE, NC><<<blocks, kThreads, smem, s>>>(a);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_stencil(int mode, int ncomp, const StencilArgs& a, cudaStream_t s) {
+    if (ncomp == 1) {
+        if (mode == MODE_APPLY) return launch_one<MODE_APPLY, 1>(a, s);
+        if (mode == MODE_RESID) return launch_one<MODE_RESID, 1>(a, s);
+        return launch_one<MODE_PCGA, 1>(a, s);
+    }
+    if (ncomp == 3) {
+        if (mode == MODE_APPLY) return launch_one<MODE_APPLY, 3>(a, s);
+        if (mode == MODE_RESID) return launch_one<MODE_RESID, 3>(a, s);
+        return launch_one<MODE_PCGA, 3>(a, s);
+    }
+    return cudaErrorInvalidValue;
+}
+
+cudaError_t launch_pcg_b(const StreamArgs& a, int nblocks, cudaStream_t s) {
+    if (a.ncomp == 1)
+        k_pcg_b<1><<<nblocks, kThreads, 0, s>>>(a);
+    else if (a.ncomp == 3)
+        k_pcg_b<3><<<nblocks, kThreads, 0, s>>>(a);
+    else
+        return cudaErrorInvalidValue;
+    return cudaGetLastError();
+}
+
+cudaError_t launch_diag(const Geo& g, Halo kappa, const double* c, double* D, double* dinv, int* bad,
+                        cudaStream_t s) {
+    const long long Nl = (long long)g.nl * g.plane;
+    const int blocks = (int)std::min<long long>((Nl + kThreads - 1) / kThreads, 148LL * 16);
+    k_diag<<<blocks, kThreads, 0, s>>>(g, kappa, c, D, dinv, bad);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_dirichlet(const Geo& g, int ncomp, const double* kappa, const double* ub, int outer,
+                             double* f, cudaStream_t s) {
+    const long long n = g.plane * ncomp;
+    const int blocks = (int)std::min<long long>((n + 255) / 256, 148LL * 8);
+    k_dirichlet<<<blocks, 256, 0, s>>>(g, ncomp, kappa, ub, outer, f);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_dot(const Geo& g, int ncomp, const double* a, const double* b, Scratch scr,
+                       double* out, int nblocks, cudaStream_t s) {
+    k_dot<<<nblocks, kThreads, 0, s>>>(g, ncomp, a, b, scr, out);
+    return cudaGetLastError();
+}
+
+}  // namespace mas

@@ -1,0 +1,122 @@
+// mas_internal.h — structures shared by the host driver (C++) and the CUDA
+// kernels of the B200 MAS-PCG library.  Not part of the ABI.
+#pragma once
+
+#include <cuda_runtime.h>
+
+#include <cstdint>
+#include <string>
+
+#include "../../include/mas_pcg.h"
+
+namespace mas {
+
+// ---------------------------------------------------------------------------
+// Geometry: 1-D coefficient tables (device pointers), computed once on the
+// host from the node/half meshes (grid.cpp).  With them the per-cell operator
+// of DESIGN.md §5.1 is
+//   (L u)_P = c u + aRm (u-u_{i-1}) + aRp (u-u_{i+1}) + aTm (u-u_{j-1})
+//           + aTp (u-u_{j+1}) + aPm (u-u_{k-1}) + aPp (u-u_{k+1})
+//   aRm = wRm[i] kf,   aTm = irc2[i] wTm[j] kf,   aPm = irc2[i] isc2[j] wPm[k] kf
+// with kf = (kappa_P + kappa_N)/2 of that face.  V_P = vr[i] vt[j] vp[k].
+// ---------------------------------------------------------------------------
+struct Geo {
+    int nl, nt, np;        // local r-planes, theta, phi
+    long long plane;       // nt*np
+    int glob_lo, glob_hi;  // this slab owns the global inner / outer r-boundary
+    const double* wRm;     // [nl] r-face i   / V  (0 on a global Neumann face)
+    const double* wRp;     // [nl] r-face i+1 / V
+    const double* irc2;    // [nl] 1/rC^2
+    const double* vr;      // [nl] rC^2 dr
+    const double* wTm;     // [nt] theta-face j   / (V/r^2)   (0 at pole/wall)
+    const double* wTp;     // [nt] theta-face j+1 / (V/r^2)
+    const double* isc2;    // [nt] 1/sin^2(tC)
+    const double* vt;      // [nt] sin(tC) dt
+    const double* wPm;     // [np] phi-face k   / (V/(r^2 sin^2))
+    const double* wPp;     // [np] phi-face k+1 / (V/(r^2 sin^2))
+    const double* vp;      // [np] dp
+};
+
+// A field read with an r-halo: interior planes plus optional ghost planes
+// (multi-GPU seams).  ghost == nullptr at a global boundary or on one GPU.
+struct Halo {
+    const double* in;   // [ncomp][nl][nt][np]
+    const double* glo;  // [ncomp][nt][np]  copy of global plane i0-1
+    const double* ghi;  // [ncomp][nt][np]  copy of global plane i0+nl
+};
+
+// Device-resident PCG state (one per op).  "pend_*" are the current
+// rank-local -> (allreduced) sums; the *_hist arrays are archived values.
+struct PcgState {
+    double pend_sigma;  // <p_k, q_k>_V           written by A(k), read by B(k)
+    double pend_rho;    // <r_k, z_k>_V           written by B(k), read by A(k+1)
+    double pend_rr;     // <r_k, r_k>_V
+    double pend_ff;     // <f, f>_V               written by init
+    double tol;
+    double relres;
+    int k;              // current iteration (A(k), B(k)); B's last block increments
+    int maxit;
+    int stopped;        // 1 once a kernel decided the solve is over
+    int iters;
+    int status;         // mas_status_t
+    int pad;
+};
+
+struct Scratch {
+    double* partials;    // [max_blocks * 4]
+    unsigned* ticket;    // one counter per kernel kind
+};
+
+enum { MODE_APPLY = 0, MODE_RESID = 1, MODE_PCGA = 2 };
+
+struct StencilArgs {
+    Geo g;
+    int chunk;                // r-planes per work item
+    int ntj, ntk, nchunk;     // tiles in theta, phi; chunks in r
+    Halo u;                   // APPLY/RESID: x;  PCGA: r (p = D^-1 r + beta p_old)
+    Halo pold;                // PCGA: p_{k-1}
+    Halo dinv;                // PCGA: 1/D with halo;  RESID: own only
+    Halo kappa;
+    const double* c;          // [nl][nt][np] or nullptr
+    const double* f;          // RESID: rhs [ncomp][nl][nt][np]
+    double* out;              // APPLY: y;  RESID: r;  PCGA: q
+    double* pnew;             // PCGA: p_k
+    double* x;                // PCGA: x (deferred update x += alpha_{k-1} p_{k-1})
+    PcgState* st;             // RESID / PCGA
+    double* rho_hist;         // [maxit+2]
+    double* sigma_hist;       // [maxit+2]
+    double* rr_hist;          // [maxit+2]
+    Scratch scr;
+    int* host_flag;           // mapped pinned int set to 1 when the solve stops
+};
+
+struct StreamArgs {  // kernel B
+    Geo g;
+    int ncomp;
+    double* r;
+    const double* q;
+    const double* dinv;
+    PcgState* st;
+    double* rho_hist;
+    double* sigma_hist;
+    double* rr_hist;
+    Scratch scr;
+    int* host_flag;
+};
+
+// launchers (kernels.cu)
+int stencil_blocks(const Geo& g, int chunk);
+cudaError_t launch_stencil(int mode, int ncomp, const StencilArgs& a, cudaStream_t s);
+cudaError_t launch_pcg_b(const StreamArgs& a, int nblocks, cudaStream_t s);
+cudaError_t launch_diag(const Geo& g, Halo kappa, const double* c, double* D, double* dinv,
+                        int* bad, cudaStream_t s);
+cudaError_t launch_dirichlet(const Geo& g, int ncomp, const double* kappa, const double* ub,
+                             int outer, double* f, cudaStream_t s);
+cudaError_t launch_dot(const Geo& g, int ncomp, const double* a, const double* b, Scratch scr,
+                       double* out, int nblocks, cudaStream_t s);
+cudaError_t launch_check_coeffs(long long n, const double* kappa, const double* c, int* bad,
+                                cudaStream_t s);
+
+void set_last_error(const std::string& msg);
+
+}  // namespace mas

@@ -1,0 +1,299 @@
+"""Thin Python binding of the C ABI in include/mas_pcg.h (argument marshalling
+only: every step of the solve runs in lib/libmaspcg.so's CUDA kernels).
+
+Functions keep the C names (mas_grid_create, mas_op_setup, mas_op_apply,
+mas_pcg_solve, ...) and accept torch tensors (CUDA or CPU) or numpy arrays;
+they pass data pointers and the current torch CUDA stream.  There is no CPU
+fallback: if the shared library is missing, import fails loudly.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+from typing import Optional
+
+import numpy as np
+
+from . import build as _build
+
+MAS_OK, MAS_NOT_CONVERGED, MAS_ERR_ARG, MAS_ERR_CUDA, MAS_ERR_NCCL, MAS_ERR_NOMEM, \
+    MAS_ERR_BREAKDOWN = range(7)
+MAS_BC_DIRICHLET, MAS_BC_NEUMANN = 0, 1
+MAS_POLE_NORTH, MAS_POLE_SOUTH = 1, 2
+
+# every symbol include/mas_pcg.h declares
+ABI_SYMBOLS = ("mas_comm_unique_id", "mas_grid_create", "mas_grid_local_extent",
+               "mas_grid_destroy", "mas_op_setup", "mas_op_update", "mas_op_apply", "mas_op_diag",
+               "mas_op_dirichlet_rhs", "mas_op_dot", "mas_pcg_solve", "mas_op_launch_count",
+               "mas_op_set_profiling", "mas_op_kernel_times", "mas_op_destroy", "mas_status_string", "mas_last_error", "mas_version")
+
+
+class MasError(RuntimeError):
+    def __init__(self, status: int, where: str, detail: str):
+        super().__init__(f"{where}: {status_string(status)} ({detail})")
+        self.status = status
+
+
+class mas_dist_t(C.Structure):
+    _fields_ = [("nranks", C.c_int), ("rank", C.c_int), ("nccl_id", C.c_ubyte * 128)]
+
+
+_lib: Optional[C.CDLL] = None
+_vp, _i, _d = C.c_void_p, C.c_int, C.c_double
+
+
+def lib() -> C.CDLL:
+    """Load lib/libmaspcg.so (never rebuilt here; see build.py / build())."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(_build.SO):
+            raise ImportError(f"{_build.SO} missing: run __graft_entry__.build() "
+                              "(there is no CPU fallback)")
+        L = C.CDLL(_build.SO)
+        sig = {
+            "mas_comm_unique_id": (_i, [_vp]),
+            "mas_grid_create": (_i, [_i, _i, _i, _vp, _vp, _vp, _vp, _vp, _vp, _i, _i, _vp, _vp]),
+            "mas_grid_local_extent": (_i, [_vp, _vp, _vp]),
+            "mas_grid_destroy": (_i, [_vp]),
+            "mas_op_setup": (_i, [_vp, _i, _vp, _vp, _i, _i, _vp, _vp]),
+            "mas_op_update": (_i, [_vp, _vp, _vp, _vp]),
+            "mas_op_apply": (_i, [_vp, _vp, _vp, _vp]),
+            "mas_op_diag": (_i, [_vp, _vp, _vp]),
+            "mas_op_dirichlet_rhs": (_i, [_vp, _vp, _vp, _vp, _vp]),
+            "mas_op_dot": (_i, [_vp, _vp, _vp, _vp, _vp]),
+            "mas_pcg_solve": (_i, [_vp, _vp, _vp, _d, _i, _vp, _vp, _vp, _vp]),
+            "mas_op_launch_count": (C.c_longlong, [_vp]),
+            "mas_op_set_profiling": (_i, [_vp, _i]),
+            "mas_op_kernel_times": (_i, [_vp, _vp, _vp, _vp]),
+            "mas_op_destroy": (_i, [_vp]),
+            "mas_status_string": (C.c_char_p, [_i]),
+            "mas_last_error": (C.c_char_p, []),
+            "mas_version": (C.c_char_p, []),
+        }
+        for name, (res, args) in sig.items():
+            f = getattr(L, name)
+            f.restype, f.argtypes = res, args
+        _lib = L
+    return _lib
+
+
+def status_string(s: int) -> str:
+    return lib().mas_status_string(s).decode()
+
+
+def last_error() -> str:
+    return lib().mas_last_error().decode()
+
+
+def _check(s: int, where: str, ok=(MAS_OK,)) -> int:
+    if s not in ok:
+        raise MasError(s, where, last_error())
+    return s
+
+
+def _ptr(a) -> Optional[int]:
+    """Data pointer of a torch tensor or numpy array (must be contiguous fp64)."""
+    if a is None:
+        return None
+    if isinstance(a, np.ndarray):
+        if a.dtype != np.float64 or not a.flags.c_contiguous:
+            raise TypeError("need C-contiguous float64 arrays")
+        return a.ctypes.data
+    import torch
+    if isinstance(a, torch.Tensor):
+        if a.dtype != torch.float64 or not a.is_contiguous():
+            raise TypeError("need contiguous float64 tensors")
+        return a.data_ptr()
+    raise TypeError(f"unsupported array type {type(a)}")
+
+
+def _stream(stream=None) -> Optional[int]:
+    if stream is not None:
+        return stream if isinstance(stream, int) else stream.cuda_stream
+    import torch
+    if torch.cuda.is_available():
+        return torch.cuda.current_stream().cuda_stream
+    return None
+
+
+# ---------------------------------------------------------------------------
+# C-named entry points
+# ---------------------------------------------------------------------------
+def mas_comm_unique_id() -> bytes:
+    buf = (C.c_ubyte * 128)()
+    _check(lib().mas_comm_unique_id(buf), "mas_comm_unique_id")
+    return bytes(buf)
+
+
+def mas_grid_create(r_node, r_half, t_node, t_half, p_node, p_half, pole_flags=3,
+                    periodic_phi=1, dist: Optional[tuple] = None) -> int:
+    """dist = (nranks, rank, nccl_id_bytes) or None.  Returns the handle."""
+    arrs = [np.ascontiguousarray(a, dtype=np.float64) for a in
+            (r_node, r_half, t_node, t_half, p_node, p_half)]
+    nr, nt, np_ = len(arrs[1]), len(arrs[3]), len(arrs[5])
+    for a, n in zip(arrs[::2], (nr, nt, np_)):
+        if len(a) != n + 1:
+            raise ValueError("node arrays must have n+1 entries")
+    d = None
+    if dist is not None:
+        d = mas_dist_t(dist[0], dist[1])
+        C.memmove(d.nccl_id, dist[2], 128)
+    out = C.c_void_p()
+    _check(lib().mas_grid_create(nr, nt, np_, *[a.ctypes.data for a in arrs], pole_flags,
+                                 periodic_phi, C.byref(d) if d is not None else None,
+                                 C.byref(out)), "mas_grid_create")
+    return out.value
+
+
+def mas_grid_local_extent(g: int):
+    i0, nl = C.c_int(), C.c_int()
+    _check(lib().mas_grid_local_extent(g, C.byref(i0), C.byref(nl)), "mas_grid_local_extent")
+    return i0.value, nl.value
+
+
+def mas_grid_destroy(g: int) -> None:
+    _check(lib().mas_grid_destroy(g), "mas_grid_destroy")
+
+
+def mas_op_setup(g: int, ncomp: int, kappa, mass=None, bc_r_inner=MAS_BC_DIRICHLET,
+                 bc_r_outer=MAS_BC_NEUMANN, stream=None) -> int:
+    out = C.c_void_p()
+    _check(lib().mas_op_setup(g, ncomp, _ptr(kappa), _ptr(mass), bc_r_inner, bc_r_outer,
+                              _stream(stream), C.byref(out)), "mas_op_setup")
+    return out.value
+
+
+def mas_op_update(op: int, kappa, mass=None, stream=None) -> None:
+    _check(lib().mas_op_update(op, _ptr(kappa), _ptr(mass), _stream(stream)), "mas_op_update")
+
+
+def mas_op_apply(op: int, x, y, stream=None) -> None:
+    _check(lib().mas_op_apply(op, _ptr(x), _ptr(y), _stream(stream)), "mas_op_apply")
+
+
+def mas_op_diag(op: int, D, stream=None) -> None:
+    _check(lib().mas_op_diag(op, _ptr(D), _stream(stream)), "mas_op_diag")
+
+
+def mas_op_dirichlet_rhs(op: int, ub_inner, ub_outer, f, stream=None) -> None:
+    _check(lib().mas_op_dirichlet_rhs(op, _ptr(ub_inner), _ptr(ub_outer), _ptr(f),
+                                      _stream(stream)), "mas_op_dirichlet_rhs")
+
+
+def mas_op_dot(op: int, a, b, stream=None) -> float:
+    out = C.c_double()
+    _check(lib().mas_op_dot(op, _ptr(a), _ptr(b), C.byref(out), _stream(stream)), "mas_op_dot")
+    return out.value
+
+
+def mas_pcg_solve(op: int, rhs, x, tol: float, maxit: int, want_hist: bool = False,
+                  stream=None):
+    """Returns (status, iters, relres, res_hist or None)."""
+    it, rel = C.c_int(), C.c_double()
+    hist = np.zeros(maxit + 1) if want_hist else None
+    s = lib().mas_pcg_solve(op, _ptr(rhs), _ptr(x), float(tol), int(maxit), C.byref(it),
+                            C.byref(rel), hist.ctypes.data if want_hist else None,
+                            _stream(stream))
+    _check(s, "mas_pcg_solve", ok=(MAS_OK, MAS_NOT_CONVERGED, MAS_ERR_BREAKDOWN))
+    if hist is not None:
+        n = it.value if s == MAS_ERR_BREAKDOWN else it.value + 1
+        hist = hist[:n]
+    return s, it.value, rel.value, hist
+
+
+def mas_op_launch_count(op: int) -> int:
+    return int(lib().mas_op_launch_count(op))
+
+
+def mas_op_set_profiling(op: int, on: bool) -> None:
+    _check(lib().mas_op_set_profiling(op, int(bool(on))), "mas_op_set_profiling")
+
+
+def mas_op_kernel_times(op: int):
+    """(avg ms kernel A, avg ms kernel B, iterations averaged) of the last solve."""
+    a, b, n = C.c_double(), C.c_double(), C.c_int()
+    _check(lib().mas_op_kernel_times(op, C.byref(a), C.byref(b), C.byref(n)),
+           "mas_op_kernel_times")
+    return a.value, b.value, n.value
+
+
+def mas_op_destroy(op: int) -> None:
+    _check(lib().mas_op_destroy(op), "mas_op_destroy")
+
+
+def mas_version() -> str:
+    return lib().mas_version().decode()
+
+
+# ---------------------------------------------------------------------------
+# small RAII helpers over the same calls
+# ---------------------------------------------------------------------------
+class Grid:
+    def __init__(self, mesh, dist=None):
+        flags = (MAS_POLE_NORTH if getattr(mesh, "pole_north", True) else 0) | \
+                (MAS_POLE_SOUTH if getattr(mesh, "pole_south", True) else 0)
+        if mesh.tF[0] != 0.0:
+            flags &= ~MAS_POLE_NORTH
+        if abs(mesh.tF[-1] - np.pi) > 1e-15:
+            flags &= ~MAS_POLE_SOUTH
+        self.h = mas_grid_create(mesh.rF, mesh.rC, mesh.tF, mesh.tC, mesh.pF, mesh.pC, flags, 1,
+                                 dist)
+        self.i0, self.nl = mas_grid_local_extent(self.h)
+        self.shape = (len(mesh.rC), len(mesh.tC), len(mesh.pC))
+
+    def close(self):
+        if self.h:
+            mas_grid_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+class Operator:
+    def __init__(self, grid: Grid, ncomp, kappa, mass, bc_inner, bc_outer, stream=None):
+        self.grid = grid
+        self.ncomp = ncomp
+        self.h = mas_op_setup(grid.h, ncomp, kappa, mass, bc_inner, bc_outer, stream)
+
+    def update(self, kappa, mass, stream=None):
+        mas_op_update(self.h, kappa, mass, stream)
+
+    def apply(self, x, y, stream=None):
+        mas_op_apply(self.h, x, y, stream)
+
+    def diag(self, D, stream=None):
+        mas_op_diag(self.h, D, stream)
+
+    def dirichlet_rhs(self, ub_inner, ub_outer, f, stream=None):
+        mas_op_dirichlet_rhs(self.h, ub_inner, ub_outer, f, stream)
+
+    def dot(self, a, b, stream=None):
+        return mas_op_dot(self.h, a, b, stream)
+
+    def solve(self, rhs, x, tol, maxit, want_hist=False, stream=None):
+        return mas_pcg_solve(self.h, rhs, x, tol, maxit, want_hist, stream)
+
+    def set_profiling(self, on=True):
+        mas_op_set_profiling(self.h, on)
+
+    def kernel_times(self):
+        return mas_op_kernel_times(self.h)
+
+    @property
+    def launch_count(self):
+        return mas_op_launch_count(self.h)
+
+    def close(self):
+        if self.h:
+            mas_op_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
