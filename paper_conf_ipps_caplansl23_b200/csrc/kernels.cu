@@ -104,40 +104,79 @@ __device__ __forceinline__ const double* plane_ptr(const Halo& h, int comp, int 
 __device__ __forceinline__ double2 ld2(const double* p) {
     return __ldg(reinterpret_cast<const double2*>(p));
 }
-__device__ __forceinline__ double2 dadd2(double2 a, double2 b) { return make_double2(a.x + b.x, a.y + b.y); }
+__device__ __forceinline__ double2 lds2(const double* p) { return *reinterpret_cast<const double2*>(p); }
+__device__ __forceinline__ void sts2(double* p, double2 v) { *reinterpret_cast<double2*>(p) = v; }
+__device__ __forceinline__ void stg2(double* p, double2 v) { *reinterpret_cast<double2*>(p) = v; }
 
-// The value entering the stencil at (plane i, offset off) for NC components,
-// plus kappa; PCGA also returns p_old (for the deferred x update).
-template <int MODE, int NC>
-struct Prod {
-    double2 u[NC];
-    double2 kap;
-    double2 po[NC];
+// Values that the stencil phase of a plane needs besides the smem ring.
+template <int NC>
+struct OwnRegs {
+    double2 c;      // mass term
+    double2 f[NC];  // RESID: rhs
+    double2 di;     // RESID: 1/D
 };
 
+// The field entering the stencil at plane i, cell pair `off`:
+//   APPLY / RESID: u = x;   PCGA: u = p_k = D^-1 r + beta p_{k-1} (p_1 = D^-1 r).
+// When `own_work` (own cells of a plane this block owns), PCGA also applies
+// the deferred x += alpha_{k-1} p_{k-1} and stores p_k, and the mass / rhs
+// terms of the stencil phase are loaded into `o`.
 template <int MODE, int NC>
 __device__ __forceinline__ void produce2(const StencilArgs& a, int i, long long off, bool first,
-                                         double beta, Prod<MODE, NC>& o) {
+                                         double beta, double alpha_prev, bool xupd,
+                                         double2 (&u)[NC], double2& kap, bool own_work,
+                                         OwnRegs<NC>& o) {
     const Geo& g = a.g;
-    o.kap = ld2(plane_ptr(a.kappa, 0, i, g) + off);
+    kap = ld2(plane_ptr(a.kappa, 0, i, g) + off);
     if (MODE == MODE_PCGA) {
         const double2 di = ld2(plane_ptr(a.dinv, 0, i, g) + off);
+        double2 r[NC], po[NC], xv[NC];
+#pragma unroll
+        for (int c = 0; c < NC; c++) r[c] = ld2(plane_ptr(a.u, c, i, g) + off);
+        if (!first) {
+#pragma unroll
+            for (int c = 0; c < NC; c++) po[c] = ld2(plane_ptr(a.pold, c, i, g) + off);
+        }
+        const long long o3 = (long long)i * g.plane + off;
+        const long long Nl = (long long)g.nl * g.plane;
+        if (own_work && xupd) {
+#pragma unroll
+            for (int c = 0; c < NC; c++) xv[c] = *reinterpret_cast<const double2*>(a.x + c * Nl + o3);
+        }
+        if (own_work && a.c) o.c = ld2(a.c + o3);
 #pragma unroll
         for (int c = 0; c < NC; c++) {
-            const double2 r = ld2(plane_ptr(a.u, c, i, g) + off);
-            double2 z = make_double2(di.x * r.x, di.y * r.y);
+            double2 z = make_double2(di.x * r[c].x, di.y * r[c].y);
             if (!first) {
-                o.po[c] = ld2(plane_ptr(a.pold, c, i, g) + off);
-                z.x = fma(beta, o.po[c].x, z.x);
-                z.y = fma(beta, o.po[c].y, z.y);
-            } else {
-                o.po[c] = make_double2(0.0, 0.0);
+                z.x = fma(beta, po[c].x, z.x);
+                z.y = fma(beta, po[c].y, z.y);
             }
-            o.u[c] = z;
+            u[c] = z;
+        }
+        if (own_work) {
+#pragma unroll
+            for (int c = 0; c < NC; c++) {
+                stg2(a.pnew + c * Nl + o3, u[c]);
+                if (xupd) {
+                    xv[c].x = fma(alpha_prev, po[c].x, xv[c].x);
+                    xv[c].y = fma(alpha_prev, po[c].y, xv[c].y);
+                    stg2(a.x + c * Nl + o3, xv[c]);
+                }
+            }
         }
     } else {
 #pragma unroll
-        for (int c = 0; c < NC; c++) o.u[c] = ld2(plane_ptr(a.u, c, i, g) + off);
+        for (int c = 0; c < NC; c++) u[c] = ld2(plane_ptr(a.u, c, i, g) + off);
+        if (own_work) {
+            const long long o3 = (long long)i * g.plane + off;
+            const long long Nl = (long long)g.nl * g.plane;
+            if (a.c) o.c = ld2(a.c + o3);
+            if (MODE == MODE_RESID) {
+                o.di = ld2(a.dinv.in + o3);
+#pragma unroll
+                for (int c = 0; c < NC; c++) o.f[c] = ld2(a.f + c * Nl + o3);
+            }
+        }
     }
 }
 
@@ -160,26 +199,28 @@ __device__ __forceinline__ void produce1(const StencilArgs& a, int i, long long 
     }
 }
 
-// smem plane buffer: field f (0..NC-1 = u components, NC = kappa), row, col
-template <int NC>
+// smem ring buffer of one plane: field f (0..NC-1 = u components, NC = kappa)
 __device__ __forceinline__ double* sfield(double* buf, int f) { return buf + f * (HROWS * ROW); }
 
-// Produce plane i for the whole tile (own cells + 1-cell theta/phi halo) into
-// smem buffer `buf`; returns the own-cell product in `own`.
+// Produce plane i for the tile into ring slot `buf`: own cells (registers ->
+// smem) and, if `halo`, the 1-cell theta/phi halo (periodic in phi, zeros
+// beyond a pole / theta wall where the face weight is 0).
 template <int MODE, int NC>
 __device__ __forceinline__ void produce_tile(const StencilArgs& a, int i, double* buf, int j0, int k0,
                                              int height, int width, bool first, double beta,
-                                             Prod<MODE, NC>& own, bool halo) {
+                                             double alpha_prev, bool xupd, bool halo, bool own_work,
+                                             double2& kown, OwnRegs<NC>& o) {
     const Geo& g = a.g;
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     const int kc = 2 * lane;
     if (w < height && kc < width) {
-        const long long off = (long long)(j0 + w) * g.np + k0 + kc;
-        produce2<MODE, NC>(a, i, off, first, beta, own);
+        double2 u[NC];
+        produce2<MODE, NC>(a, i, (long long)(j0 + w) * g.np + k0 + kc, first, beta, alpha_prev,
+                           xupd, u, kown, own_work, o);
         const int idx = (1 + w) * ROW + OFF + kc;
 #pragma unroll
-        for (int c = 0; c < NC; c++) *reinterpret_cast<double2*>(sfield<NC>(buf, c) + idx) = own.u[c];
-        *reinterpret_cast<double2*>(sfield<NC>(buf, NC) + idx) = own.kap;
+        for (int c = 0; c < NC; c++) sts2(sfield(buf, c) + idx, u[c]);
+        sts2(sfield(buf, NC) + idx, kown);
     }
     if (!halo) return;
     if (w < 2) {  // theta halo rows: warp 0 -> j0-1, warp 1 -> j0+height
@@ -188,15 +229,16 @@ __device__ __forceinline__ void produce_tile(const StencilArgs& a, int i, double
         if (kc < width) {
             const int idx = jr * ROW + OFF + kc;
             if (j >= 0 && j < g.nt) {
-                Prod<MODE, NC> h;
-                produce2<MODE, NC>(a, i, (long long)j * g.np + k0 + kc, first, beta, h);
+                double2 u[NC], kap;
+                OwnRegs<NC> dummy;
+                produce2<MODE, NC>(a, i, (long long)j * g.np + k0 + kc, first, beta, alpha_prev,
+                                   false, u, kap, false, dummy);
 #pragma unroll
-                for (int c = 0; c < NC; c++) *reinterpret_cast<double2*>(sfield<NC>(buf, c) + idx) = h.u[c];
-                *reinterpret_cast<double2*>(sfield<NC>(buf, NC) + idx) = h.kap;
-            } else {  // beyond a pole / theta wall: zero-flux face, value unused but finite
+                for (int c = 0; c < NC; c++) sts2(sfield(buf, c) + idx, u[c]);
+                sts2(sfield(buf, NC) + idx, kap);
+            } else {
 #pragma unroll
-                for (int c = 0; c <= NC; c++)
-                    *reinterpret_cast<double2*>(sfield<NC>(buf, c) + idx) = make_double2(0.0, 0.0);
+                for (int c = 0; c <= NC; c++) sts2(sfield(buf, c) + idx, make_double2(0.0, 0.0));
             }
         }
     } else if (w == 2) {  // phi halo columns (periodic wrap)
@@ -208,15 +250,36 @@ __device__ __forceinline__ void produce_tile(const StencilArgs& a, int i, double
             produce1<MODE, NC>(a, i, (long long)(j0 + jr) * g.np + k, first, beta, u, kap);
             const int idx = (1 + jr) * ROW + col;
 #pragma unroll
-            for (int c = 0; c < NC; c++) sfield<NC>(buf, c)[idx] = u[c];
-            sfield<NC>(buf, NC)[idx] = kap;
+            for (int c = 0; c < NC; c++) sfield(buf, c)[idx] = u[c];
+            sfield(buf, NC)[idx] = kap;
         }
+    }
+}
+
+// Own-cell region of a ring slot as the global-boundary ghost plane:
+// u = 0 (homogeneous Dirichlet; irrelevant under Neumann, weight 0) and
+// kappa_ghost = kappa_P so that the face kappa is kappa_P (reading R3).
+template <int NC>
+__device__ __forceinline__ void ghost_plane(double* buf, int height, int width, double2 kP) {
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const int kc = 2 * lane;
+    if (w < height && kc < width) {
+        const int idx = (1 + w) * ROW + OFF + kc;
+#pragma unroll
+        for (int c = 0; c < NC; c++) sts2(sfield(buf, c) + idx, make_double2(0.0, 0.0));
+        sts2(sfield(buf, NC) + idx, kP);
     }
 }
 
 // --------------------------------------------------------------------------
 // the fused stencil kernel
 // --------------------------------------------------------------------------
+// One block = one (TJ x TK) theta-phi tile x one chunk of r-planes.  It
+// marches along r keeping the last three produced planes (p and kappa with
+// halo) in a shared-memory ring: slot(i) = (i - ia + 1) % 3.  Per plane:
+//   produce(i+1): global loads of r, p_old, D^-1, kappa (+x, c for own cells)
+//                 -> p_{i+1} into the ring (and x-update / p store)
+//   sync; stencil(i) from the ring only (r-neighbours = adjacent slots); sync
 template <int MODE, int NC>
 __global__ void __launch_bounds__(kThreads, (NC == 1 ? 3 : 2)) k_stencil(const StencilArgs a) {
     extern __shared__ __align__(16) double smem[];
@@ -243,6 +306,7 @@ __global__ void __launch_bounds__(kThreads, (NC == 1 ? 3 : 2)) k_stencil(const S
         else if (!first)
             beta = st->pend_rho / a.rho_hist[kit - 2];
     }
+    const bool xupd = (MODE == MODE_PCGA) && kit >= 2;
 
     // ---- work item ------------------------------------------------------
     const int item = blockIdx.x;
@@ -266,15 +330,15 @@ __global__ void __launch_bounds__(kThreads, (NC == 1 ? 3 : 2)) k_stencil(const S
             for (int i = ia; i < ib; i++) {
 #pragma unroll
                 for (int c = 0; c < NC; c++) {
-                    double2* xp = reinterpret_cast<double2*>(a.x + c * Nl + (long long)i * g.plane + off);
+                    double* xp = a.x + c * Nl + (long long)i * g.plane + off;
                     if (pmode == P_ZERO) {
-                        *xp = make_double2(0.0, 0.0);
+                        stg2(xp, make_double2(0.0, 0.0));
                     } else if (kit >= 2) {
                         const double2 po = ld2(plane_ptr(a.pold, c, i, g) + off);
-                        double2 xv = *xp;
+                        double2 xv = lds2(xp);
                         xv.x = fma(alpha_prev, po.x, xv.x);
                         xv.y = fma(alpha_prev, po.y, xv.y);
-                        *xp = xv;
+                        stg2(xp, xv);
                     }
                 }
             }
@@ -306,30 +370,21 @@ __global__ void __launch_bounds__(kThreads, (NC == 1 ? 3 : 2)) k_stencil(const S
         return;
     }
 
-    // ---- march along r ----------------------------------------------------
-    double* buf0 = smem;
-    Prod<MODE, NC> cur, nxt;   // own-cell products at planes i (cur) and i+1 (nxt)
-    double2 um[NC], km;        // own u and kappa at plane i-1
-    double2 un[NC], kn;        // own u and kappa at plane i+1
+    auto slot = [&](int i) { return smem + ((i - ia + 1) % 3) * BUF; };
 
-    // plane ia-1: own cell only (r-neighbour of the first plane)
+    // ---- prologue: planes ia-1 (own cells only) and ia --------------------
+    OwnRegs<NC> oc, on;  // own-cell stencil inputs for the current / next plane
+    double2 kown = make_double2(0.0, 0.0), kdummy;
     const bool lo_ghost = (ia == 0) && g.glob_lo;
-    if (own && !lo_ghost) {
-        Prod<MODE, NC> pm;
-        produce2<MODE, NC>(a, ia - 1, off, first, beta, pm);
-#pragma unroll
-        for (int c = 0; c < NC; c++) um[c] = pm.u[c];
-        km = pm.kap;
-    }
-    produce_tile<MODE, NC>(a, ia, buf0, j0, k0, height, width, first, beta, cur, true);
-    if (lo_ghost && own) {  // global boundary ghost: u = 0, kappa_ghost = kappa_P
-#pragma unroll
-        for (int c = 0; c < NC; c++) um[c] = make_double2(0.0, 0.0);
-        km = cur.kap;
-    }
+    if (!lo_ghost)
+        produce_tile<MODE, NC>(a, ia - 1, slot(ia - 1), j0, k0, height, width, first, beta,
+                               alpha_prev, false, false, false, kdummy, on);
+    produce_tile<MODE, NC>(a, ia, slot(ia), j0, k0, height, width, first, beta, alpha_prev, xupd,
+                           true, true, kown, oc);
+    if (lo_ghost) ghost_plane<NC>(slot(ia - 1), height, width, kown);
 
     // per-cell geometry constant over the march
-    double wpm[2], wpp[2], vpk[2];
+    double wpm[2] = {0.0, 0.0}, wpp[2] = {0.0, 0.0}, vpk[2] = {0.0, 0.0};
     double wtm = 0.0, wtp = 0.0, isc = 0.0, vtj = 0.0;
     if (own) {
         wtm = __ldg(g.wTm + j);
@@ -345,97 +400,79 @@ __global__ void __launch_bounds__(kThreads, (NC == 1 ? 3 : 2)) k_stencil(const S
     }
 
     for (int i = ia; i < ib; i++) {
-        double* bc = smem + ((i - ia) % 3) * BUF;
-        double* bn = smem + ((i + 1 - ia) % 3) * BUF;
-        const bool hi_ghost = (i + 1 == g.nl) && g.glob_hi;
-        if (!hi_ghost) {
-            // the next plane needs its halo only if it will be a stencil plane
-            produce_tile<MODE, NC>(a, i + 1, bn, j0, k0, height, width, first, beta, nxt, i + 1 < ib);
-            if (own) {
-#pragma unroll
-                for (int c = 0; c < NC; c++) un[c] = nxt.u[c];
-                kn = nxt.kap;
-            }
-        } else if (own) {
-#pragma unroll
-            for (int c = 0; c < NC; c++) un[c] = make_double2(0.0, 0.0);
-            kn = cur.kap;
-        }
+        // produce plane i+1 (halo only if it is a stencil plane of this block)
+        if ((i + 1 == g.nl) && g.glob_hi)
+            ghost_plane<NC>(slot(i + 1), height, width, kown);
+        else
+            produce_tile<MODE, NC>(a, i + 1, slot(i + 1), j0, k0, height, width, first, beta,
+                                   alpha_prev, xupd && (i + 1 < ib), i + 1 < ib, i + 1 < ib, kown, on);
         __syncthreads();
 
         if (own) {
+            const double* S0 = slot(i);
+            const double* Sm = slot(i - 1);
+            const double* Sp = slot(i + 1);
             const int idx = (1 + w) * ROW + OFF + kc;
-            const double* sk = sfield<NC>(bc, NC);
             const double wrm = __ldg(g.wRm + i), wrp = __ldg(g.wRp + i), irc = __ldg(g.irc2 + i);
             const double vri = __ldg(g.vr + i);
-            double2 cP = make_double2(0.0, 0.0);
-            if (a.c) cP = ld2(a.c + (long long)i * g.plane + off);
+
+            const double2 kP = lds2(sfield(const_cast<double*>(S0), NC) + idx);
+            const double2 kM = lds2(sfield(const_cast<double*>(Sm), NC) + idx);
+            const double2 kN = lds2(sfield(const_cast<double*>(Sp), NC) + idx);
+            const double2 kS = lds2(sfield(const_cast<double*>(S0), NC) + idx - ROW);
+            const double2 kT = lds2(sfield(const_cast<double*>(S0), NC) + idx + ROW);
+            const double kL = sfield(const_cast<double*>(S0), NC)[idx - 1];
+            const double kR = sfield(const_cast<double*>(S0), NC)[idx + 2];
+            const double it = irc * wtm, ip = irc * wtp, ic = irc * isc;
+            // face coefficients a_f = w_f * (kappa_P + kappa_N)/2, cells e = 0, 1
+            const double aRm0 = wrm * (0.5 * (kP.x + kM.x)), aRm1 = wrm * (0.5 * (kP.y + kM.y));
+            const double aRp0 = wrp * (0.5 * (kP.x + kN.x)), aRp1 = wrp * (0.5 * (kP.y + kN.y));
+            const double aTm0 = it * (0.5 * (kP.x + kS.x)), aTm1 = it * (0.5 * (kP.y + kS.y));
+            const double aTp0 = ip * (0.5 * (kP.x + kT.x)), aTp1 = ip * (0.5 * (kP.y + kT.y));
+            const double aPm0 = ic * wpm[0] * (0.5 * (kP.x + kL));
+            const double aPm1 = ic * wpm[1] * (0.5 * (kP.y + kP.x));
+            const double aPp0 = ic * wpp[0] * (0.5 * (kP.x + kP.y));
+            const double aPp1 = ic * wpp[1] * (0.5 * (kP.y + kR));
+            const double V0 = vri * vtj * vpk[0], V1 = vri * vtj * vpk[1];
+            const double2 cP = a.c ? oc.c : make_double2(0.0, 0.0);
             const long long pofs = (long long)i * g.plane + off;
-
-            double aRm[2], aRp[2], aTm[2], aTp[2], aPm[2], aPp[2], kP[2];
-            kP[0] = sk[idx];
-            kP[1] = sk[idx + 1];
-            const double kM[2] = {km.x, km.y}, kN[2] = {kn.x, kn.y};
-#pragma unroll
-            for (int e = 0; e < 2; e++) {
-                const double kp = kP[e];
-                aRm[e] = wrm * (0.5 * (kp + kM[e]));
-                aRp[e] = wrp * (0.5 * (kp + kN[e]));
-                aTm[e] = irc * wtm * (0.5 * (kp + sk[idx + e - ROW]));
-                aTp[e] = irc * wtp * (0.5 * (kp + sk[idx + e + ROW]));
-                aPm[e] = irc * isc * wpm[e] * (0.5 * (kp + sk[idx + e - 1]));
-                aPp[e] = irc * isc * wpp[e] * (0.5 * (kp + sk[idx + e + 1]));
-            }
-            const double cc[2] = {cP.x, cP.y};
-            const double V[2] = {vri * vtj * vpk[0], vri * vtj * vpk[1]};
-            double2 di = make_double2(0.0, 0.0);
-            if (MODE == MODE_RESID) di = ld2(a.dinv.in + pofs);
-
 #pragma unroll
             for (int c = 0; c < NC; c++) {
-                const double* su = sfield<NC>(bc, c);
-                const double uM[2] = {um[c].x, um[c].y}, uN[2] = {un[c].x, un[c].y};
-                double L[2], uu[2];
-#pragma unroll
-                for (int e = 0; e < 2; e++) {
-                    const double u = su[idx + e];
-                    uu[e] = u;
-                    double s = cc[e] * u;
-                    s = fma(aRm[e], u - uM[e], s);
-                    s = fma(aRp[e], u - uN[e], s);
-                    s = fma(aTm[e], u - su[idx + e - ROW], s);
-                    s = fma(aTp[e], u - su[idx + e + ROW], s);
-                    s = fma(aPm[e], u - su[idx + e - 1], s);
-                    s = fma(aPp[e], u - su[idx + e + 1], s);
-                    L[e] = s;
-                }
+                const double* s0 = sfield(const_cast<double*>(S0), c);
+                const double2 u = lds2(s0 + idx);
+                const double2 uM = lds2(sfield(const_cast<double*>(Sm), c) + idx);
+                const double2 uN = lds2(sfield(const_cast<double*>(Sp), c) + idx);
+                const double2 uS = lds2(s0 + idx - ROW);
+                const double2 uT = lds2(s0 + idx + ROW);
+                const double uL = s0[idx - 1], uR = s0[idx + 2];
+                double L0 = cP.x * u.x, L1 = cP.y * u.y;
+                L0 = fma(aRm0, u.x - uM.x, L0);
+                L1 = fma(aRm1, u.y - uM.y, L1);
+                L0 = fma(aRp0, u.x - uN.x, L0);
+                L1 = fma(aRp1, u.y - uN.y, L1);
+                L0 = fma(aTm0, u.x - uS.x, L0);
+                L1 = fma(aTm1, u.y - uS.y, L1);
+                L0 = fma(aTp0, u.x - uT.x, L0);
+                L1 = fma(aTp1, u.y - uT.y, L1);
+                L0 = fma(aPm0, u.x - uL, L0);
+                L1 = fma(aPm1, u.y - u.x, L1);
+                L0 = fma(aPp0, u.x - u.y, L0);
+                L1 = fma(aPp1, u.y - uR, L1);
                 const long long o = c * Nl + pofs;
-                if (MODE == MODE_APPLY) {
-                    *reinterpret_cast<double2*>(a.out + o) = make_double2(L[0], L[1]);
-                } else if (MODE == MODE_RESID) {
-                    const double2 f = ld2(a.f + o);
-                    const double r0 = f.x - L[0], r1 = f.y - L[1];
-                    *reinterpret_cast<double2*>(a.out + o) = make_double2(r0, r1);
-                    acc[0] += V[0] * f.x * f.x + V[1] * f.y * f.y;
-                    acc[1] += V[0] * r0 * r0 + V[1] * r1 * r1;
-                    acc[2] += V[0] * r0 * (di.x * r0) + V[1] * r1 * (di.y * r1);
-                } else {  // PCGA
-                    *reinterpret_cast<double2*>(a.out + o) = make_double2(L[0], L[1]);
-                    *reinterpret_cast<double2*>(a.pnew + o) = make_double2(uu[0], uu[1]);
-                    if (kit >= 2) {
-                        double2* xp = reinterpret_cast<double2*>(a.x + o);
-                        double2 xv = *xp;
-                        xv.x = fma(alpha_prev, cur.po[c].x, xv.x);
-                        xv.y = fma(alpha_prev, cur.po[c].y, xv.y);
-                        *xp = xv;
-                    }
-                    acc[0] += V[0] * uu[0] * L[0] + V[1] * uu[1] * L[1];
+                if (MODE == MODE_RESID) {
+                    const double r0 = oc.f[c].x - L0, r1 = oc.f[c].y - L1;
+                    stg2(a.out + o, make_double2(r0, r1));
+                    acc[0] += V0 * oc.f[c].x * oc.f[c].x + V1 * oc.f[c].y * oc.f[c].y;
+                    acc[1] += V0 * r0 * r0 + V1 * r1 * r1;
+                    acc[2] += V0 * r0 * (oc.di.x * r0) + V1 * r1 * (oc.di.y * r1);
+                } else {
+                    stg2(a.out + o, make_double2(L0, L1));
+                    if (MODE == MODE_PCGA) acc[0] += V0 * u.x * L0 + V1 * u.y * L1;
                 }
-                um[c] = make_double2(uu[0], uu[1]);
             }
-            km = make_double2(kP[0], kP[1]);
-            cur = nxt;
         }
+        oc = on;
+        __syncthreads();
     }
 
     // ---- reductions -------------------------------------------------------
@@ -456,7 +493,6 @@ __global__ void __launch_bounds__(kThreads, (NC == 1 ? 3 : 2)) k_stencil(const S
         }
     }
 }
-
 // --------------------------------------------------------------------------
 // kernel B: r -= alpha q ; z = D^-1 r ; <r,z>_V, <r,r>_V
 // --------------------------------------------------------------------------

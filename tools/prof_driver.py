@@ -1,0 +1,30 @@
+"""Small driver for ncu: set up config C3 (or --config) and run one PCG solve
+with a few iterations through the C ABI.  Launch order: k_diag (setup),
+k_stencil<RESID>, then per iteration k_stencil<PCGA>, k_pcg_b."""
+import argparse
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+import numpy as np
+import torch
+
+from paper_conf_ipps_caplansl23_b200 import maspcg as M
+from paper_conf_ipps_caplansl23_b200 import workloads as W
+
+ap = argparse.ArgumentParser()
+ap.add_argument("--config", default="C3")
+ap.add_argument("--maxit", type=int, default=4)
+args = ap.parse_args()
+shapes = {"C3": ("viscosity", 256, 256, 512), "C2": ("conduction", 128, 128, 256)}
+kind, nr, nt, np_ = shapes[args.config]
+prob = W.make(kind, nr=nr, nt=nt, np_=np_)
+d = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()
+g = M.Grid(prob.mesh)
+op = M.Operator(g, prob.ncomp, d(prob.kappa), d(prob.c), prob.bc_inner, prob.bc_outer)
+f = d(prob.f)
+x = d(prob.x0)
+st, it, rel, _ = op.solve(f, x, 0.0, args.maxit)
+torch.cuda.synchronize()
+print("iters", it, "status", st)
