@@ -116,95 +116,81 @@ struct OwnRegs {
     double2 di;     // RESID: 1/D
 };
 
-// The field entering the stencil at plane i, cell pair `off`:
-//   APPLY / RESID: u = x;   PCGA: u = p_k = D^-1 r + beta p_{k-1} (p_1 = D^-1 r).
-// When `own_work` (own cells of a plane this block owns), PCGA also applies
-// the deferred x += alpha_{k-1} p_{k-1} and stores p_k, and the mass / rhs
-// terms of the stencil phase are loaded into `o`.
+// Raw inputs of one cell pair (or one cell in .x for a phi-halo column).
+template <int NC>
+struct Raw {
+    double2 u[NC];   // PCGA: r;  APPLY/RESID: x
+    double2 po[NC];  // PCGA: p_{k-1}
+    double2 di;      // PCGA: 1/D
+    double2 kap;
+};
+
+template <bool SCALAR>
+__device__ __forceinline__ double2 ldv(const double* p) {
+    if (SCALAR) return make_double2(__ldg(p), 0.0);
+    return ld2(p);
+}
+
+// Block-uniform base pointers of plane i of every field the producer reads.
+template <int NC>
+struct PlanePtrs {
+    const double* u[NC];
+    const double* po[NC];
+    const double* di;
+    const double* kap;
+};
+
 template <int MODE, int NC>
-__device__ __forceinline__ void produce2(const StencilArgs& a, int i, long long off, bool first,
-                                         double beta, double alpha_prev, bool xupd,
-                                         double2 (&u)[NC], double2& kap, bool own_work,
-                                         OwnRegs<NC>& o) {
+__device__ __forceinline__ PlanePtrs<NC> plane_ptrs(const StencilArgs& a, int i, bool first) {
     const Geo& g = a.g;
-    kap = ld2(plane_ptr(a.kappa, 0, i, g) + off);
-    if (MODE == MODE_PCGA) {
-        const double2 di = ld2(plane_ptr(a.dinv, 0, i, g) + off);
-        double2 r[NC], po[NC], xv[NC];
+    PlanePtrs<NC> P;
+    P.kap = plane_ptr(a.kappa, 0, i, g);
 #pragma unroll
-        for (int c = 0; c < NC; c++) r[c] = ld2(plane_ptr(a.u, c, i, g) + off);
+    for (int c = 0; c < NC; c++) P.u[c] = plane_ptr(a.u, c, i, g);
+    P.di = (MODE == MODE_PCGA) ? plane_ptr(a.dinv, 0, i, g) : nullptr;
+#pragma unroll
+    for (int c = 0; c < NC; c++) P.po[c] = (MODE == MODE_PCGA && !first) ? plane_ptr(a.pold, c, i, g) : nullptr;
+    return P;
+}
+
+template <int MODE, int NC, bool SCALAR>
+__device__ __forceinline__ void load_raw(const PlanePtrs<NC>& P, long long off, bool first, Raw<NC>& R) {
+    R.kap = ldv<SCALAR>(P.kap + off);
+#pragma unroll
+    for (int c = 0; c < NC; c++) R.u[c] = ldv<SCALAR>(P.u[c] + off);
+    if (MODE == MODE_PCGA) {
+        R.di = ldv<SCALAR>(P.di + off);
         if (!first) {
 #pragma unroll
-            for (int c = 0; c < NC; c++) po[c] = ld2(plane_ptr(a.pold, c, i, g) + off);
-        }
-        const long long o3 = (long long)i * g.plane + off;
-        const long long Nl = (long long)g.nl * g.plane;
-        if (own_work && xupd) {
-#pragma unroll
-            for (int c = 0; c < NC; c++) xv[c] = *reinterpret_cast<const double2*>(a.x + c * Nl + o3);
-        }
-        if (own_work && a.c) o.c = ld2(a.c + o3);
-#pragma unroll
-        for (int c = 0; c < NC; c++) {
-            double2 z = make_double2(di.x * r[c].x, di.y * r[c].y);
-            if (!first) {
-                z.x = fma(beta, po[c].x, z.x);
-                z.y = fma(beta, po[c].y, z.y);
-            }
-            u[c] = z;
-        }
-        if (own_work) {
-#pragma unroll
-            for (int c = 0; c < NC; c++) {
-                stg2(a.pnew + c * Nl + o3, u[c]);
-                if (xupd) {
-                    xv[c].x = fma(alpha_prev, po[c].x, xv[c].x);
-                    xv[c].y = fma(alpha_prev, po[c].y, xv[c].y);
-                    stg2(a.x + c * Nl + o3, xv[c]);
-                }
-            }
-        }
-    } else {
-#pragma unroll
-        for (int c = 0; c < NC; c++) u[c] = ld2(plane_ptr(a.u, c, i, g) + off);
-        if (own_work) {
-            const long long o3 = (long long)i * g.plane + off;
-            const long long Nl = (long long)g.nl * g.plane;
-            if (a.c) o.c = ld2(a.c + o3);
-            if (MODE == MODE_RESID) {
-                o.di = ld2(a.dinv.in + o3);
-#pragma unroll
-                for (int c = 0; c < NC; c++) o.f[c] = ld2(a.f + c * Nl + o3);
-            }
+            for (int c = 0; c < NC; c++) R.po[c] = ldv<SCALAR>(P.po[c] + off);
         }
     }
 }
 
+// u entering the stencil: APPLY/RESID x;  PCGA p_k = D^-1 r + beta p_{k-1}
 template <int MODE, int NC>
-__device__ __forceinline__ void produce1(const StencilArgs& a, int i, long long off, bool first,
-                                         double beta, double (&u)[NC], double& kap) {
-    const Geo& g = a.g;
-    kap = __ldg(plane_ptr(a.kappa, 0, i, g) + off);
-    if (MODE == MODE_PCGA) {
-        const double di = __ldg(plane_ptr(a.dinv, 0, i, g) + off);
+__device__ __forceinline__ void finish_raw(Raw<NC>& R, bool first, double beta) {
+    if constexpr (MODE != MODE_PCGA) return;
 #pragma unroll
-        for (int c = 0; c < NC; c++) {
-            double z = di * __ldg(plane_ptr(a.u, c, i, g) + off);
-            if (!first) z = fma(beta, __ldg(plane_ptr(a.pold, c, i, g) + off), z);
-            u[c] = z;
+    for (int c = 0; c < NC; c++) {
+        double2 z = make_double2(R.di.x * R.u[c].x, R.di.y * R.u[c].y);
+        if (!first) {
+            z.x = fma(beta, R.po[c].x, z.x);
+            z.y = fma(beta, R.po[c].y, z.y);
         }
-    } else {
-#pragma unroll
-        for (int c = 0; c < NC; c++) u[c] = __ldg(plane_ptr(a.u, c, i, g) + off);
+        R.u[c] = z;
     }
 }
 
 // smem ring buffer of one plane: field f (0..NC-1 = u components, NC = kappa)
 __device__ __forceinline__ double* sfield(double* buf, int f) { return buf + f * (HROWS * ROW); }
 
-// Produce plane i for the tile into ring slot `buf`: own cells (registers ->
-// smem) and, if `halo`, the 1-cell theta/phi halo (periodic in phi, zeros
-// beyond a pole / theta wall where the face weight is 0).
+// Produce plane i for the tile into ring slot `buf`: own cells and, if
+// `halo`, the 1-cell theta/phi halo (periodic in phi; zeros beyond a pole /
+// theta wall, where the face weight is 0).  All global loads of the thread
+// (own pair, one halo item, x and c) are issued before any is consumed.
+// For own cells of planes this block owns (`own_work`), PCGA also stores
+// p_k and applies the deferred x += alpha_{k-1} p_{k-1}.
 template <int MODE, int NC>
 __device__ __forceinline__ void produce_tile(const StencilArgs& a, int i, double* buf, int j0, int k0,
                                              int height, int width, bool first, double beta,
@@ -213,46 +199,91 @@ __device__ __forceinline__ void produce_tile(const StencilArgs& a, int i, double
     const Geo& g = a.g;
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     const int kc = 2 * lane;
-    if (w < height && kc < width) {
-        double2 u[NC];
-        produce2<MODE, NC>(a, i, (long long)(j0 + w) * g.np + k0 + kc, first, beta, alpha_prev,
-                           xupd, u, kown, own_work, o);
-        const int idx = (1 + w) * ROW + OFF + kc;
-#pragma unroll
-        for (int c = 0; c < NC; c++) sts2(sfield(buf, c) + idx, u[c]);
-        sts2(sfield(buf, NC) + idx, kown);
-    }
-    if (!halo) return;
-    if (w < 2) {  // theta halo rows: warp 0 -> j0-1, warp 1 -> j0+height
-        const int jr = (w == 0) ? 0 : height + 1;
-        const int j = j0 + jr - 1;
-        if (kc < width) {
-            const int idx = jr * ROW + OFF + kc;
-            if (j >= 0 && j < g.nt) {
-                double2 u[NC], kap;
-                OwnRegs<NC> dummy;
-                produce2<MODE, NC>(a, i, (long long)j * g.np + k0 + kc, first, beta, alpha_prev,
-                                   false, u, kap, false, dummy);
-#pragma unroll
-                for (int c = 0; c < NC; c++) sts2(sfield(buf, c) + idx, u[c]);
-                sts2(sfield(buf, NC) + idx, kap);
-            } else {
-#pragma unroll
-                for (int c = 0; c <= NC; c++) sts2(sfield(buf, c) + idx, make_double2(0.0, 0.0));
+    const bool has_own = (w < height) && (kc < width);
+    // this thread's halo item: 1 = theta row pair (warps 0, 1), 2 = phi column cell (warp 2)
+    int hkind = 0, hidx = 0;
+    long long hoff = 0;
+    if (halo) {
+        if (w < 2) {
+            const int jr = (w == 0) ? 0 : height + 1;
+            const int j = j0 + jr - 1;
+            if (kc < width) {
+                hidx = jr * ROW + OFF + kc;
+                hkind = (j >= 0 && j < g.nt) ? 1 : 3;  // 3 = beyond the pole/wall: zeros
+                hoff = (long long)j * g.np + k0 + kc;
+            }
+        } else if (w == 2) {
+            const int side = lane >> 4, jr = lane & 15;
+            if (jr < height) {
+                const int k = side == 0 ? (k0 - 1 + g.np) % g.np : (k0 + width) % g.np;
+                hidx = (1 + jr) * ROW + (side == 0 ? OFF - 1 : OFF + width);
+                hkind = 2;
+                hoff = (long long)(j0 + jr) * g.np + k;
             }
         }
-    } else if (w == 2) {  // phi halo columns (periodic wrap)
-        const int side = lane >> 4, jr = lane & 15;
-        if (jr < height) {
-            const int k = side == 0 ? (k0 - 1 + g.np) % g.np : (k0 + width) % g.np;
-            const int col = side == 0 ? OFF - 1 : OFF + width;
-            double u[NC], kap;
-            produce1<MODE, NC>(a, i, (long long)(j0 + jr) * g.np + k, first, beta, u, kap);
-            const int idx = (1 + jr) * ROW + col;
+    }
+    const long long off = (long long)(j0 + w) * g.np + k0 + kc;
+    const long long o3 = (long long)i * g.plane + off;
+    const long long Nl = (long long)g.nl * g.plane;
+
+    // ---- issue every load ---------------------------------------------------
+    const PlanePtrs<NC> P = plane_ptrs<MODE, NC>(a, i, first);
+    Raw<NC> R, H;
+    double2 xv[NC];
+    if (has_own) {
+        load_raw<MODE, NC, false>(P, off, first, R);
+        if (own_work) {
+            if (a.c) o.c = ld2(a.c + o3);
+            if (MODE == MODE_PCGA && xupd) {
 #pragma unroll
-            for (int c = 0; c < NC; c++) sfield(buf, c)[idx] = u[c];
-            sfield(buf, NC)[idx] = kap;
+                for (int c = 0; c < NC; c++) xv[c] = lds2(a.x + c * Nl + o3);
+            }
+            if (MODE == MODE_RESID) {
+                o.di = ld2(a.dinv.in + o3);
+#pragma unroll
+                for (int c = 0; c < NC; c++) o.f[c] = ld2(a.f + c * Nl + o3);
+            }
         }
+    }
+    if (hkind == 1)
+        load_raw<MODE, NC, false>(P, hoff, first, H);
+    else if (hkind == 2)
+        load_raw<MODE, NC, true>(P, hoff, first, H);
+
+    // ---- consume ----------------------------------------------------------
+    if (has_own) {
+        finish_raw<MODE, NC>(R, first, beta);
+        const int idx = (1 + w) * ROW + OFF + kc;
+#pragma unroll
+        for (int c = 0; c < NC; c++) sts2(sfield(buf, c) + idx, R.u[c]);
+        sts2(sfield(buf, NC) + idx, R.kap);
+        kown = R.kap;
+        if (MODE == MODE_PCGA && own_work) {
+#pragma unroll
+            for (int c = 0; c < NC; c++) {
+                stg2(a.pnew + c * Nl + o3, R.u[c]);
+                if (xupd) {
+                    xv[c].x = fma(alpha_prev, R.po[c].x, xv[c].x);
+                    xv[c].y = fma(alpha_prev, R.po[c].y, xv[c].y);
+                    stg2(a.x + c * Nl + o3, xv[c]);
+                }
+            }
+        }
+    }
+    if (hkind == 1 || hkind == 2) {
+        finish_raw<MODE, NC>(H, first, beta);
+        if (hkind == 1) {
+#pragma unroll
+            for (int c = 0; c < NC; c++) sts2(sfield(buf, c) + hidx, H.u[c]);
+            sts2(sfield(buf, NC) + hidx, H.kap);
+        } else {
+#pragma unroll
+            for (int c = 0; c < NC; c++) sfield(buf, c)[hidx] = H.u[c].x;
+            sfield(buf, NC)[hidx] = H.kap.x;
+        }
+    } else if (hkind == 3) {
+#pragma unroll
+        for (int c = 0; c <= NC; c++) sts2(sfield(buf, c) + hidx, make_double2(0.0, 0.0));
     }
 }
 
@@ -383,22 +414,6 @@ __global__ void __launch_bounds__(kThreads, (NC == 1 ? 3 : 2)) k_stencil(const S
                            true, true, kown, oc);
     if (lo_ghost) ghost_plane<NC>(slot(ia - 1), height, width, kown);
 
-    // per-cell geometry constant over the march
-    double wpm[2] = {0.0, 0.0}, wpp[2] = {0.0, 0.0}, vpk[2] = {0.0, 0.0};
-    double wtm = 0.0, wtp = 0.0, isc = 0.0, vtj = 0.0;
-    if (own) {
-        wtm = __ldg(g.wTm + j);
-        wtp = __ldg(g.wTp + j);
-        isc = __ldg(g.isc2 + j);
-        vtj = __ldg(g.vt + j);
-#pragma unroll
-        for (int e = 0; e < 2; e++) {
-            wpm[e] = __ldg(g.wPm + k + e);
-            wpp[e] = __ldg(g.wPp + k + e);
-            vpk[e] = __ldg(g.vp + k + e);
-        }
-    }
-
     for (int i = ia; i < ib; i++) {
         // produce plane i+1 (halo only if it is a stencil plane of this block)
         if ((i + 1 == g.nl) && g.glob_hi)
@@ -415,6 +430,11 @@ __global__ void __launch_bounds__(kThreads, (NC == 1 ? 3 : 2)) k_stencil(const S
             const int idx = (1 + w) * ROW + OFF + kc;
             const double wrm = __ldg(g.wRm + i), wrp = __ldg(g.wRp + i), irc = __ldg(g.irc2 + i);
             const double vri = __ldg(g.vr + i);
+            // 1-D geometry (L1-resident tables, re-read per plane to save registers)
+            const double wtm = __ldg(g.wTm + j), wtp = __ldg(g.wTp + j), isc = __ldg(g.isc2 + j);
+            const double vtj = __ldg(g.vt + j);
+            const double2 wpm2 = ld2(g.wPm + k), wpp2 = ld2(g.wPp + k), vpk2 = ld2(g.vp + k);
+            const double wpm[2] = {wpm2.x, wpm2.y}, wpp[2] = {wpp2.x, wpp2.y}, vpk[2] = {vpk2.x, vpk2.y};
 
             const double2 kP = lds2(sfield(const_cast<double*>(S0), NC) + idx);
             const double2 kM = lds2(sfield(const_cast<double*>(Sm), NC) + idx);
