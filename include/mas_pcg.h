@@ -100,6 +100,12 @@ MAS_API mas_status_t mas_grid_create(int nr, int nt, int np,
                              int pole_flags, int periodic_phi,
                              const mas_dist_t* dist, mas_grid_t** out);
 
+/* The r-slab partition without a grid (host only, no device work): rank
+ * owns nr/nranks + (rank < nr % nranks) planes starting at *i0 (SURVEY.md
+ * §8(e)).  Lets a caller size its slab buffers before mas_grid_create.
+ * Errors: MAS_ERR_ARG unless 1 <= nranks <= nr and 0 <= rank < nranks. */
+MAS_API mas_status_t mas_partition(int nr, int nranks, int rank, int* i0, int* nr_local);
+
 /* First global r-plane and number of planes owned by this rank. */
 MAS_API mas_status_t mas_grid_local_extent(const mas_grid_t* g, int* i0, int* nr_local);
 

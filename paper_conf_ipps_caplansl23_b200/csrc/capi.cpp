@@ -177,6 +177,14 @@ mas_status_t mas_grid_create(int nr, int nt, int np, const double* r_node, const
     return MAS_OK;
 }
 
+mas_status_t mas_partition(int nr, int nranks, int rank, int* i0, int* nr_local) {
+    if (!i0 || !nr_local) return arg_error("null argument");
+    if (nranks < 1 || nr < nranks || rank < 0 || rank >= nranks)
+        return arg_error("need 1 <= nranks <= nr and 0 <= rank < nranks");
+    partition(nr, nranks, rank, i0, nr_local);
+    return MAS_OK;
+}
+
 mas_status_t mas_grid_local_extent(const mas_grid_t* g, int* i0, int* nr_local) {
     if (!g || !i0 || !nr_local) return arg_error("null argument");
     *i0 = g->i0;

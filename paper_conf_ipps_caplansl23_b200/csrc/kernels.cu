@@ -170,15 +170,16 @@ __device__ __forceinline__ void load_raw(const PlanePtrs<NC>& P, long long off, 
 // u entering the stencil: APPLY/RESID x;  PCGA p_k = D^-1 r + beta p_{k-1}
 template <int MODE, int NC>
 __device__ __forceinline__ void finish_raw(Raw<NC>& R, bool first, double beta) {
-    if constexpr (MODE != MODE_PCGA) return;
+    if constexpr (MODE == MODE_PCGA) {
 #pragma unroll
-    for (int c = 0; c < NC; c++) {
-        double2 z = make_double2(R.di.x * R.u[c].x, R.di.y * R.u[c].y);
-        if (!first) {
-            z.x = fma(beta, R.po[c].x, z.x);
-            z.y = fma(beta, R.po[c].y, z.y);
+        for (int c = 0; c < NC; c++) {
+            double2 z = make_double2(R.di.x * R.u[c].x, R.di.y * R.u[c].y);
+            if (!first) {
+                z.x = fma(beta, R.po[c].x, z.x);
+                z.y = fma(beta, R.po[c].y, z.y);
+            }
+            R.u[c] = z;
         }
-        R.u[c] = z;
     }
 }
 

@@ -22,7 +22,7 @@ MAS_BC_DIRICHLET, MAS_BC_NEUMANN = 0, 1
 MAS_POLE_NORTH, MAS_POLE_SOUTH = 1, 2
 
 # every symbol include/mas_pcg.h declares
-ABI_SYMBOLS = ("mas_comm_unique_id", "mas_grid_create", "mas_grid_local_extent",
+ABI_SYMBOLS = ("mas_comm_unique_id", "mas_partition", "mas_grid_create", "mas_grid_local_extent",
                "mas_grid_destroy", "mas_op_setup", "mas_op_update", "mas_op_apply", "mas_op_diag",
                "mas_op_dirichlet_rhs", "mas_op_dot", "mas_pcg_solve", "mas_op_launch_count",
                "mas_op_set_profiling", "mas_op_kernel_times", "mas_op_destroy", "mas_status_string", "mas_last_error", "mas_version")
@@ -53,6 +53,7 @@ def lib() -> C.CDLL:
         sig = {
             "mas_comm_unique_id": (_i, [_vp]),
             "mas_grid_create": (_i, [_i, _i, _i, _vp, _vp, _vp, _vp, _vp, _vp, _i, _i, _vp, _vp]),
+            "mas_partition": (_i, [_i, _i, _i, _vp, _vp]),
             "mas_grid_local_extent": (_i, [_vp, _vp, _vp]),
             "mas_grid_destroy": (_i, [_vp]),
             "mas_op_setup": (_i, [_vp, _i, _vp, _vp, _i, _i, _vp, _vp]),
@@ -143,6 +144,12 @@ def mas_grid_create(r_node, r_half, t_node, t_half, p_node, p_half, pole_flags=3
                                  periodic_phi, C.byref(d) if d is not None else None,
                                  C.byref(out)), "mas_grid_create")
     return out.value
+
+
+def mas_partition(nr: int, nranks: int, rank: int):
+    i0, nl = C.c_int(), C.c_int()
+    _check(lib().mas_partition(nr, nranks, rank, C.byref(i0), C.byref(nl)), "mas_partition")
+    return i0.value, nl.value
 
 
 def mas_grid_local_extent(g: int):
