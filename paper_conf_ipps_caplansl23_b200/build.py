@@ -52,6 +52,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
     cmd = [nvcc, *ARCH, "-O3", "-lineinfo", "-std=c++17", "-shared", "-Xcompiler", "-fPIC",
            "-Xcompiler", "-fvisibility=hidden", "-cudart", "static",
            "-I", INCLUDE, "-I", os.path.join(nccl, "include"),
+           *os.environ.get("MAS_NVCC_FLAGS", "").split(),
            *sources(), "-o", tmp,
            "-L", os.path.join(nccl, "lib"), "-l:libnccl.so.2",
            "-Xlinker", "-rpath," + os.path.join(nccl, "lib")]

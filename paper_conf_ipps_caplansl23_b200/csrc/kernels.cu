@@ -27,8 +27,16 @@
 
 namespace mas {
 
-constexpr int kThreads = 256;  // 8 warps
-constexpr int TJ = 8;          // theta rows per tile (one warp per row)
+constexpr int kThreads = 256;  // 8 warps (stream kernels)
+#ifndef MAS_TJ
+#define MAS_TJ 8
+#endif
+#ifndef MAS_MINB
+#define MAS_MINB 2
+#endif
+constexpr int TJ = MAS_TJ;     // theta rows per stencil tile (one warp per row)
+constexpr int kSThreads = 32 * TJ;
+constexpr int kMaxChunk = 16;  // r-planes per stencil work item (host picks <= this)
 constexpr int TK = 64;         // phi cells per tile (2 per lane, double2)
 constexpr int OFF = 2;         // smem column of the first tile cell (16B aligned)
 constexpr int ROW = TK + 4;    // smem row length: [pad][halo][64 cells][halo][pad]
@@ -49,9 +57,9 @@ __device__ __forceinline__ double warp_sum(double v) {
 // Block-reduce NS sums, publish the block partial, take a ticket.  Returns
 // true in the last block to finish, where `v` then holds the grid totals
 // (valid in thread 0), summed in a fixed order independent of scheduling.
-template <int NS>
+template <int NS, int NTHR = kThreads>
 __device__ bool grid_reduce(double (&v)[NS], const Scratch& scr, int tkt) {
-    __shared__ double wsum[NS][kThreads / 32];
+    __shared__ double wsum[NS][NTHR / 32];
     __shared__ bool last;
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
 #pragma unroll
@@ -64,7 +72,7 @@ __device__ bool grid_reduce(double (&v)[NS], const Scratch& scr, int tkt) {
 #pragma unroll
         for (int s = 0; s < NS; s++) {
             double t = 0.0;
-            for (int q = 0; q < kThreads / 32; q++) t += wsum[s][q];
+            for (int q = 0; q < NTHR / 32; q++) t += wsum[s][q];
             scr.partials[(size_t)blockIdx.x * NS + s] = t;
         }
         __threadfence();
@@ -77,7 +85,7 @@ __device__ bool grid_reduce(double (&v)[NS], const Scratch& scr, int tkt) {
 #pragma unroll
     for (int s = 0; s < NS; s++) {
         double t = 0.0;
-        for (unsigned b = threadIdx.x; b < gridDim.x; b += kThreads)
+        for (unsigned b = threadIdx.x; b < gridDim.x; b += NTHR)
             t += __ldcg(&scr.partials[(size_t)b * NS + s]);
         t = warp_sum(t);
         __syncthreads();
@@ -85,7 +93,7 @@ __device__ bool grid_reduce(double (&v)[NS], const Scratch& scr, int tkt) {
         __syncthreads();
         if (threadIdx.x == 0) {
             double u = 0.0;
-            for (int q = 0; q < kThreads / 32; q++) u += wsum[s][q];
+            for (int q = 0; q < NTHR / 32; q++) u += wsum[s][q];
             v[s] = u;
         }
     }
@@ -313,7 +321,7 @@ __device__ __forceinline__ void ghost_plane(double* buf, int height, int width, 
 //                 -> p_{i+1} into the ring (and x-update / p store)
 //   sync; stencil(i) from the ring only (r-neighbours = adjacent slots); sync
 template <int MODE, int NC>
-__global__ void __launch_bounds__(kThreads, (NC == 1 ? 3 : 2)) k_stencil(const StencilArgs a) {
+__global__ void __launch_bounds__(kSThreads, MAS_MINB) k_stencil(const StencilArgs a) {
     extern __shared__ __align__(16) double smem[];
     constexpr int BUF = (NC + 1) * HROWS * ROW;
     const Geo& g = a.g;
@@ -376,7 +384,7 @@ __global__ void __launch_bounds__(kThreads, (NC == 1 ? 3 : 2)) k_stencil(const S
             }
         }
         double v1[1] = {0.0};
-        if (grid_reduce<1>(v1, a.scr, TKT_STENCIL) && threadIdx.x == 0) {
+        if (grid_reduce<1, kSThreads>(v1, a.scr, TKT_STENCIL) && threadIdx.x == 0) {
             PcgState* st = a.st;
             const double ff = st->pend_ff, rr = st->pend_rr;
             a.rr_hist[kit - 1] = rr;
@@ -404,6 +412,32 @@ __global__ void __launch_bounds__(kThreads, (NC == 1 ? 3 : 2)) k_stencil(const S
 
     auto slot = [&](int i) { return smem + ((i - ia + 1) % 3) * BUF; };
 
+    // 1-D geometry of this work item staged in shared memory once (visible to
+    // the stencil after the first barrier of the march)
+    __shared__ __align__(16) double sgR[4][kMaxChunk];
+    __shared__ __align__(16) double sgT[4][TJ];
+    __shared__ __align__(16) double sgP[3][TK];
+    for (int t = threadIdx.x; t < kMaxChunk; t += kSThreads) {
+        const int i = min(ia + t, g.nl - 1);
+        sgR[0][t] = g.wRm[i];
+        sgR[1][t] = g.wRp[i];
+        sgR[2][t] = g.irc2[i];
+        sgR[3][t] = g.vr[i];
+    }
+    for (int t = threadIdx.x; t < TJ; t += kSThreads) {
+        const int jj = min(j0 + t, g.nt - 1);
+        sgT[0][t] = g.wTm[jj];
+        sgT[1][t] = g.wTp[jj];
+        sgT[2][t] = g.isc2[jj];
+        sgT[3][t] = g.vt[jj];
+    }
+    for (int t = threadIdx.x; t < TK; t += kSThreads) {
+        const int kk = min(k0 + t, g.np - 1);
+        sgP[0][t] = g.wPm[kk];
+        sgP[1][t] = g.wPp[kk];
+        sgP[2][t] = g.vp[kk];
+    }
+
     // ---- prologue: planes ia-1 (own cells only) and ia --------------------
     OwnRegs<NC> oc, on;  // own-cell stencil inputs for the current / next plane
     double2 kown = make_double2(0.0, 0.0), kdummy;
@@ -429,12 +463,11 @@ __global__ void __launch_bounds__(kThreads, (NC == 1 ? 3 : 2)) k_stencil(const S
             const double* Sm = slot(i - 1);
             const double* Sp = slot(i + 1);
             const int idx = (1 + w) * ROW + OFF + kc;
-            const double wrm = __ldg(g.wRm + i), wrp = __ldg(g.wRp + i), irc = __ldg(g.irc2 + i);
-            const double vri = __ldg(g.vr + i);
-            // 1-D geometry (L1-resident tables, re-read per plane to save registers)
-            const double wtm = __ldg(g.wTm + j), wtp = __ldg(g.wTp + j), isc = __ldg(g.isc2 + j);
-            const double vtj = __ldg(g.vt + j);
-            const double2 wpm2 = ld2(g.wPm + k), wpp2 = ld2(g.wPp + k), vpk2 = ld2(g.vp + k);
+            // 1-D geometry from the block's shared-memory copy (no global latency per plane)
+            const int ir = i - ia;
+            const double wrm = sgR[0][ir], wrp = sgR[1][ir], irc = sgR[2][ir], vri = sgR[3][ir];
+            const double wtm = sgT[0][w], wtp = sgT[1][w], isc = sgT[2][w], vtj = sgT[3][w];
+            const double2 wpm2 = lds2(&sgP[0][kc]), wpp2 = lds2(&sgP[1][kc]), vpk2 = lds2(&sgP[2][kc]);
             const double wpm[2] = {wpm2.x, wpm2.y}, wpp[2] = {wpp2.x, wpp2.y}, vpk[2] = {vpk2.x, vpk2.y};
 
             const double2 kP = lds2(sfield(const_cast<double*>(S0), NC) + idx);
@@ -498,7 +531,7 @@ __global__ void __launch_bounds__(kThreads, (NC == 1 ? 3 : 2)) k_stencil(const S
 
     // ---- reductions -------------------------------------------------------
     if (MODE == MODE_RESID) {
-        if (grid_reduce<3>(acc, a.scr, TKT_STENCIL) && threadIdx.x == 0) {
+        if (grid_reduce<3, kSThreads>(acc, a.scr, TKT_STENCIL) && threadIdx.x == 0) {
             PcgState* st = a.st;
             st->pend_ff = acc[0];
             st->pend_rr = acc[1];
@@ -506,7 +539,7 @@ __global__ void __launch_bounds__(kThreads, (NC == 1 ? 3 : 2)) k_stencil(const S
         }
     } else if (MODE == MODE_PCGA) {
         double v[1] = {acc[0]};
-        if (grid_reduce<1>(v, a.scr, TKT_STENCIL) && threadIdx.x == 0) {
+        if (grid_reduce<1, kSThreads>(v, a.scr, TKT_STENCIL) && threadIdx.x == 0) {
             PcgState* st = a.st;
             st->pend_sigma = v[0];
             a.rr_hist[kit - 1] = st->pend_rr;
@@ -679,7 +712,7 @@ static cudaError_t launch_one(const StencilArgs& a0, cudaStream_t s) {
         attr_done = true;
     }
     const int blocks = a.ntj * a.ntk * a.nchunk;
-    k_stencil<MODE, NC><<<blocks, kThreads, smem, s>>>(a);
+    k_stencil<MODE, NC><<<blocks, kSThreads, smem, s>>>(a);
     return cudaGetLastError();
 }
 
