@@ -194,106 +194,151 @@ __device__ __forceinline__ void finish_raw(Raw<NC>& R, bool first, double beta) 
 // smem ring buffer of one plane: field f (0..NC-1 = u components, NC = kappa)
 __device__ __forceinline__ double* sfield(double* buf, int f) { return buf + f * (HROWS * ROW); }
 
-// Produce plane i for the tile into ring slot `buf`: own cells and, if
-// `halo`, the 1-cell theta/phi halo (periodic in phi; zeros beyond a pole /
-// theta wall, where the face weight is 0).  All global loads of the thread
-// (own pair, one halo item, x and c) are issued before any is consumed.
-// For own cells of planes this block owns (`own_work`), PCGA also stores
-// p_k and applies the deferred x += alpha_{k-1} p_{k-1}.
+// Halo item of a thread (plane independent), one scalar cell: threads
+// 0..2TK-1 cover the theta halo rows j0-1 and j0+height, threads
+// 2TK..2TK+2TJ-1 the periodic phi halo columns.
+struct HaloMeta {
+    long long hoff;  // offset in the plane
+    int hidx;        // index in a ring field
+    int hkind;       // 0 none, 1 load, 3 zeros (beyond a pole / theta wall)
+};
+
+__device__ __forceinline__ HaloMeta halo_meta(const Geo& g, int j0, int k0, int height, int width) {
+    const int t = threadIdx.x;
+    HaloMeta m{0, 0, 0};
+    if (t < 2 * TK) {
+        const bool top = t < TK;
+        const int kk = top ? t : t - TK;
+        const int hr = top ? 0 : height + 1;
+        const int j = j0 + hr - 1;
+        if (kk < width) {
+            m.hidx = hr * ROW + OFF + kk;
+            m.hkind = (j >= 0 && j < g.nt) ? 1 : 3;
+            m.hoff = (long long)j * g.np + k0 + kk;
+        }
+    } else if (t < 2 * TK + 2 * TJ) {
+        const int q = t - 2 * TK, side = q / TJ, r = q % TJ;
+        if (r < height) {
+            const int k = side == 0 ? (k0 - 1 + g.np) % g.np : (k0 + width) % g.np;
+            m.hidx = (1 + r) * ROW + (side == 0 ? OFF - 1 : OFF + width);
+            m.hkind = 1;
+            m.hoff = (long long)(j0 + r) * g.np + k;
+        }
+    }
+    return m;
+}
+
+// One plane's loads of this thread, in flight in registers (the software
+// pipeline issues plane i+2 before the stencil of plane i).
+template <int NC>
+struct Stage {
+    Raw<NC> R;                          // own double2 pair
+    double hu[NC], hpo[NC], hdi, hkap;  // halo scalar cell
+    double2 xv[NC];                     // own x (PCGA deferred update)
+    OwnRegs<NC> o;                      // own c (+ f, D^-1 for RESID)
+};
+
 template <int MODE, int NC>
-__device__ __forceinline__ void produce_tile(const StencilArgs& a, int i, double* buf, int j0, int k0,
-                                             int height, int width, bool first, double beta,
-                                             double alpha_prev, bool xupd, bool halo, bool own_work,
-                                             double2& kown, OwnRegs<NC>& o) {
+__device__ __forceinline__ void stage_issue(const StencilArgs& a, int i, int j0, int k0, int height,
+                                            int width, const HaloMeta& hm, bool first, bool xupd,
+                                            bool halo, bool own_work, Stage<NC>& S) {
     const Geo& g = a.g;
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     const int kc = 2 * lane;
-    const bool has_own = (w < height) && (kc < width);
-    // this thread's halo item: 1 = theta row pair (warps 0, 1), 2 = phi column cell (warp 2)
-    int hkind = 0, hidx = 0;
-    long long hoff = 0;
-    if (halo) {
-        if (w < 2) {
-            const int jr = (w == 0) ? 0 : height + 1;
-            const int j = j0 + jr - 1;
-            if (kc < width) {
-                hidx = jr * ROW + OFF + kc;
-                hkind = (j >= 0 && j < g.nt) ? 1 : 3;  // 3 = beyond the pole/wall: zeros
-                hoff = (long long)j * g.np + k0 + kc;
-            }
-        } else if (w == 2) {
-            const int side = lane >> 4, jr = lane & 15;
-            if (jr < height) {
-                const int k = side == 0 ? (k0 - 1 + g.np) % g.np : (k0 + width) % g.np;
-                hidx = (1 + jr) * ROW + (side == 0 ? OFF - 1 : OFF + width);
-                hkind = 2;
-                hoff = (long long)(j0 + jr) * g.np + k;
-            }
-        }
-    }
-    const long long off = (long long)(j0 + w) * g.np + k0 + kc;
-    const long long o3 = (long long)i * g.plane + off;
     const long long Nl = (long long)g.nl * g.plane;
-
-    // ---- issue every load ---------------------------------------------------
     const PlanePtrs<NC> P = plane_ptrs<MODE, NC>(a, i, first);
-    Raw<NC> R, H;
-    double2 xv[NC];
-    if (has_own) {
-        load_raw<MODE, NC, false>(P, off, first, R);
+    if (w < height && kc < width) {
+        const long long off = (long long)(j0 + w) * g.np + k0 + kc;
+        const long long o3 = (long long)i * g.plane + off;
+        load_raw<MODE, NC, false>(P, off, first, S.R);
         if (own_work) {
-            if (a.c) o.c = ld2(a.c + o3);
+            if (a.c) S.o.c = ld2(a.c + o3);
             if (MODE == MODE_PCGA && xupd) {
 #pragma unroll
-                for (int c = 0; c < NC; c++) xv[c] = lds2(a.x + c * Nl + o3);
+                for (int c = 0; c < NC; c++) S.xv[c] = lds2(a.x + c * Nl + o3);
             }
             if (MODE == MODE_RESID) {
-                o.di = ld2(a.dinv.in + o3);
+                S.o.di = ld2(a.dinv.in + o3);
 #pragma unroll
-                for (int c = 0; c < NC; c++) o.f[c] = ld2(a.f + c * Nl + o3);
+                for (int c = 0; c < NC; c++) S.o.f[c] = ld2(a.f + c * Nl + o3);
             }
         }
     }
-    if (hkind == 1)
-        load_raw<MODE, NC, false>(P, hoff, first, H);
-    else if (hkind == 2)
-        load_raw<MODE, NC, true>(P, hoff, first, H);
+    if (halo && hm.hkind == 1) {
+        S.hkap = __ldg(P.kap + hm.hoff);
+#pragma unroll
+        for (int c = 0; c < NC; c++) S.hu[c] = __ldg(P.u[c] + hm.hoff);
+        if (MODE == MODE_PCGA) {
+            S.hdi = __ldg(P.di + hm.hoff);
+            if (!first) {
+#pragma unroll
+                for (int c = 0; c < NC; c++) S.hpo[c] = __ldg(P.po[c] + hm.hoff);
+            }
+        }
+    }
+}
 
-    // ---- consume ----------------------------------------------------------
-    if (has_own) {
-        finish_raw<MODE, NC>(R, first, beta);
+template <int MODE, int NC>
+__device__ __forceinline__ void stage_commit(const StencilArgs& a, int i, int j0, int k0, int height,
+                                             int width, const HaloMeta& hm, bool first, double beta,
+                                             double alpha_prev, bool xupd, bool halo, bool own_work,
+                                             Stage<NC>& S, double* buf, double2& kown,
+                                             OwnRegs<NC>& o) {
+    const Geo& g = a.g;
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const int kc = 2 * lane;
+    const long long Nl = (long long)g.nl * g.plane;
+    if (w < height && kc < width) {
+        finish_raw<MODE, NC>(S.R, first, beta);
         const int idx = (1 + w) * ROW + OFF + kc;
 #pragma unroll
-        for (int c = 0; c < NC; c++) sts2(sfield(buf, c) + idx, R.u[c]);
-        sts2(sfield(buf, NC) + idx, R.kap);
-        kown = R.kap;
-        if (MODE == MODE_PCGA && own_work) {
+        for (int c = 0; c < NC; c++) sts2(sfield(buf, c) + idx, S.R.u[c]);
+        sts2(sfield(buf, NC) + idx, S.R.kap);
+        kown = S.R.kap;
+        if (own_work) {
+            o = S.o;
+            if (MODE == MODE_PCGA) {
+                const long long o3 = (long long)i * g.plane + (long long)(j0 + w) * g.np + k0 + kc;
 #pragma unroll
-            for (int c = 0; c < NC; c++) {
-                stg2(a.pnew + c * Nl + o3, R.u[c]);
-                if (xupd) {
-                    xv[c].x = fma(alpha_prev, R.po[c].x, xv[c].x);
-                    xv[c].y = fma(alpha_prev, R.po[c].y, xv[c].y);
-                    stg2(a.x + c * Nl + o3, xv[c]);
+                for (int c = 0; c < NC; c++) {
+                    stg2(a.pnew + c * Nl + o3, S.R.u[c]);
+                    if (xupd) {
+                        double2 xv = S.xv[c];
+                        xv.x = fma(alpha_prev, S.R.po[c].x, xv.x);
+                        xv.y = fma(alpha_prev, S.R.po[c].y, xv.y);
+                        stg2(a.x + c * Nl + o3, xv);
+                    }
                 }
             }
         }
     }
-    if (hkind == 1 || hkind == 2) {
-        finish_raw<MODE, NC>(H, first, beta);
-        if (hkind == 1) {
+    if (halo && hm.hkind == 1) {
 #pragma unroll
-            for (int c = 0; c < NC; c++) sts2(sfield(buf, c) + hidx, H.u[c]);
-            sts2(sfield(buf, NC) + hidx, H.kap);
-        } else {
-#pragma unroll
-            for (int c = 0; c < NC; c++) sfield(buf, c)[hidx] = H.u[c].x;
-            sfield(buf, NC)[hidx] = H.kap.x;
+        for (int c = 0; c < NC; c++) {
+            double u = S.hu[c];
+            if (MODE == MODE_PCGA) {
+                const double z = S.hdi * u;
+                u = first ? z : fma(beta, S.hpo[c], z);
+            }
+            sfield(buf, c)[hm.hidx] = u;
         }
-    } else if (hkind == 3) {
+        sfield(buf, NC)[hm.hidx] = S.hkap;
+    } else if (halo && hm.hkind == 3) {
 #pragma unroll
-        for (int c = 0; c <= NC; c++) sts2(sfield(buf, c) + hidx, make_double2(0.0, 0.0));
+        for (int c = 0; c <= NC; c++) sfield(buf, c)[hm.hidx] = 0.0;
     }
+}
+
+// Produce plane i into ring slot `buf` right away (issue + commit).
+template <int MODE, int NC>
+__device__ __forceinline__ void produce_tile(const StencilArgs& a, int i, double* buf, int j0, int k0,
+                                             int height, int width, const HaloMeta& hm, bool first,
+                                             double beta, double alpha_prev, bool xupd, bool halo,
+                                             bool own_work, double2& kown, OwnRegs<NC>& o) {
+    Stage<NC> S;
+    stage_issue<MODE, NC>(a, i, j0, k0, height, width, hm, first, xupd, halo, own_work, S);
+    stage_commit<MODE, NC>(a, i, j0, k0, height, width, hm, first, beta, alpha_prev, xupd, halo,
+                           own_work, S, buf, kown, o);
 }
 
 // Own-cell region of a ring slot as the global-boundary ghost plane:
@@ -410,7 +455,11 @@ __global__ void __launch_bounds__(kSThreads, MAS_MINB) k_stencil(const StencilAr
         return;
     }
 
-    auto slot = [&](int i) { return smem + ((i - ia + 1) % 3) * BUF; };
+    // 4-slot ring: stencil(i) reads slots i-1, i, i+1 while plane i+2's loads
+    // are in flight; plane i+2 is committed into the slot of plane i-2, so
+    // one barrier per plane suffices.
+    auto slot = [&](int i) { return smem + ((i - ia + 1) & 3) * BUF; };
+    auto real_plane = [&](int p) { return !(p == g.nl && g.glob_hi); };
 
     // 1-D geometry of this work item staged in shared memory once (visible to
     // the stencil after the first barrier of the march)
@@ -442,21 +491,31 @@ __global__ void __launch_bounds__(kSThreads, MAS_MINB) k_stencil(const StencilAr
     OwnRegs<NC> oc, on;  // own-cell stencil inputs for the current / next plane
     double2 kown = make_double2(0.0, 0.0), kdummy;
     const bool lo_ghost = (ia == 0) && g.glob_lo;
+    const HaloMeta hm = halo_meta(g, j0, k0, height, width);
     if (!lo_ghost)
-        produce_tile<MODE, NC>(a, ia - 1, slot(ia - 1), j0, k0, height, width, first, beta,
+        produce_tile<MODE, NC>(a, ia - 1, slot(ia - 1), j0, k0, height, width, hm, first, beta,
                                alpha_prev, false, false, false, kdummy, on);
-    produce_tile<MODE, NC>(a, ia, slot(ia), j0, k0, height, width, first, beta, alpha_prev, xupd,
+    produce_tile<MODE, NC>(a, ia, slot(ia), j0, k0, height, width, hm, first, beta, alpha_prev, xupd,
                            true, true, kown, oc);
     if (lo_ghost) ghost_plane<NC>(slot(ia - 1), height, width, kown);
+    Stage<NC> S;
+    if (real_plane(ia + 1))
+        stage_issue<MODE, NC>(a, ia + 1, j0, k0, height, width, hm, first, xupd && (ia + 1 < ib),
+                              ia + 1 < ib, ia + 1 < ib, S);
 
     for (int i = ia; i < ib; i++) {
-        // produce plane i+1 (halo only if it is a stencil plane of this block)
-        if ((i + 1 == g.nl) && g.glob_hi)
-            ghost_plane<NC>(slot(i + 1), height, width, kown);
+        // commit plane i+1 (its loads were issued one plane earlier)
+        if (real_plane(i + 1))
+            stage_commit<MODE, NC>(a, i + 1, j0, k0, height, width, hm, first, beta, alpha_prev,
+                                   xupd && (i + 1 < ib), i + 1 < ib, i + 1 < ib, S, slot(i + 1),
+                                   kown, on);
         else
-            produce_tile<MODE, NC>(a, i + 1, slot(i + 1), j0, k0, height, width, first, beta,
-                                   alpha_prev, xupd && (i + 1 < ib), i + 1 < ib, i + 1 < ib, kown, on);
+            ghost_plane<NC>(slot(i + 1), height, width, kown);
         __syncthreads();
+        // issue plane i+2: its latency overlaps the stencil of plane i
+        if (i + 2 <= ib && real_plane(i + 2))
+            stage_issue<MODE, NC>(a, i + 2, j0, k0, height, width, hm, first, xupd && (i + 2 < ib),
+                                  i + 2 < ib, i + 2 < ib, S);
 
         if (own) {
             const double* S0 = slot(i);
@@ -526,7 +585,6 @@ __global__ void __launch_bounds__(kSThreads, MAS_MINB) k_stencil(const StencilAr
             }
         }
         oc = on;
-        __syncthreads();
     }
 
     // ---- reductions -------------------------------------------------------
@@ -703,7 +761,7 @@ static cudaError_t launch_one(const StencilArgs& a0, cudaStream_t s) {
     a.ntj = (a.g.nt + TJ - 1) / TJ;
     a.ntk = (a.g.np + TK - 1) / TK;
     a.nchunk = (a.g.nl + a.chunk - 1) / a.chunk;
-    const int smem = 3 * (NC + 1) * HROWS * ROW * (int)sizeof(double);
+    const int smem = 4 * (NC + 1) * HROWS * ROW * (int)sizeof(double);
     static bool attr_done = false;
     if (!attr_done) {
         cudaError_t e = cudaFuncSetAttribute(k_stencil<MODE, NC>,
