@@ -9,6 +9,7 @@
 #include <cuda_runtime.h>
 
 #include <cmath>
+#include <cstdlib>
 #include <cstring>
 #include <new>
 #include <string>
@@ -374,7 +375,9 @@ mas_status_t mas_op_setup(mas_grid_t* g, int ncomp, const double* kappa, const d
     G.wPm = t; t += np;
     G.wPp = t; t += np;
     G.vp = t;
-    op->chunk = nl >= 64 ? 16 : (nl >= 16 ? 8 : 4);
+    const char* ch_env = getenv("MAS_CHUNK");  // experiment hook
+    op->chunk = ch_env ? atoi(ch_env) : (nl >= 128 ? 32 : nl >= 64 ? 16 : (nl >= 16 ? 8 : 4));
+    if (op->chunk < 1 || op->chunk > 32) op->chunk = 16;
     op->max_blocks = stencil_blocks(G, op->chunk);
     op->b_blocks = 148 * 8;
     if (op->b_blocks > op->max_blocks) op->max_blocks = op->b_blocks;

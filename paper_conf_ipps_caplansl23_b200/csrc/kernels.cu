@@ -36,7 +36,7 @@ constexpr int kThreads = 256;  // 8 warps (stream kernels)
 #endif
 constexpr int TJ = MAS_TJ;     // theta rows per stencil tile (one warp per row)
 constexpr int kSThreads = 32 * TJ;
-constexpr int kMaxChunk = 16;  // r-planes per stencil work item (host picks <= this)
+constexpr int kMaxChunk = 32;  // r-planes per stencil work item (host picks <= this)
 constexpr int TK = 64;         // phi cells per tile (2 per lane, double2)
 constexpr int OFF = 2;         // smem column of the first tile cell (16B aligned)
 constexpr int ROW = TK + 4;    // smem row length: [pad][halo][64 cells][halo][pad]
