@@ -101,6 +101,14 @@ struct mas_op {
     std::vector<cudaEvent_t> pev;  // 4 per iteration: A start/end, B start/end
     double prof_a_ms = 0.0, prof_b_ms = 0.0, prof_init_ms = 0.0;
     int prof_n = 0;
+    // single-GPU solve loop as one CUDA graph: a device-side while node whose
+    // body is two PCG iterations (A, B, A, B); rebuilt when x or the history
+    // buffers move.
+    cudaGraphExec_t gexec = nullptr;
+    cudaStream_t cap_stream = nullptr;
+    const double* g_x = nullptr;
+    const double* g_hist = nullptr;
+    int use_graph = 1;
 };
 
 extern "C" {
@@ -261,6 +269,8 @@ static void op_free(mas_op* op) {
     for (auto& e : op->ev)
         if (e) cudaEventDestroy(e);
     for (auto& e : op->pev) cudaEventDestroy(e);
+    if (op->gexec) cudaGraphExecDestroy(op->gexec);
+    if (op->cap_stream) cudaStreamDestroy(op->cap_stream);
     delete op;
 }
 
@@ -280,6 +290,59 @@ static mas_status_t ensure_prof_events(mas_op* op, int k) {
         CU(cudaEventCreate(&e));
         op->pev.push_back(e);
     }
+    return MAS_OK;
+}
+
+// Build (or reuse) the graph of the iteration loop: while (!stopped) {A B A B}.
+// Kernels read k, alpha, beta and the stop decision from PcgState; the
+// deciding kernel's last block sets the while-condition to 0.
+static mas_status_t loop_graph(mas_op* op, StencilArgs a, StreamArgs b) {
+    if (op->gexec && op->g_x == a.x && op->g_hist == a.rho_hist) return MAS_OK;
+    if (op->gexec) {
+        cudaGraphExecDestroy(op->gexec);
+        op->gexec = nullptr;
+    }
+    if (!op->cap_stream) CU(cudaStreamCreateWithFlags(&op->cap_stream, cudaStreamNonBlocking));
+    cudaGraph_t g;
+    CU(cudaGraphCreate(&g, 0));
+    cudaGraphConditionalHandle h;
+    cudaError_t e = cudaGraphConditionalHandleCreate(&h, g, 1, cudaGraphCondAssignDefault);
+    cudaGraphNodeParams p = {};
+    p.type = cudaGraphNodeTypeConditional;
+    p.conditional.handle = h;
+    p.conditional.type = cudaGraphCondTypeWhile;
+    p.conditional.size = 1;
+    cudaGraphNode_t node;
+    if (e == cudaSuccess) e = cudaGraphAddNode(&node, g, nullptr, 0, &p);
+    if (e == cudaSuccess) {
+        cudaGraph_t body = p.conditional.phGraph_out[0];
+        e = cudaStreamBeginCaptureToGraph(op->cap_stream, body, nullptr, nullptr, 0,
+                                          cudaStreamCaptureModeThreadLocal);
+        if (e == cudaSuccess) {
+            a.cond = (unsigned long long)h;
+            b.cond = (unsigned long long)h;
+            const int nc = op->ncomp;
+            for (int kk = 1; kk <= 2 && e == cudaSuccess; kk++) {
+                a.pold = halo_of(op, op->p[(kk + 1) & 1], nullptr, nc);
+                a.pnew = op->p[kk & 1];
+                e = launch_stencil(MODE_PCGA, nc, a, op->cap_stream);
+                if (e == cudaSuccess) e = launch_pcg_b(b, op->b_blocks, op->cap_stream);
+            }
+            cudaGraph_t out = body;
+            cudaError_t e2 = cudaStreamEndCapture(op->cap_stream, &out);
+            if (e == cudaSuccess) e = e2;
+        }
+    }
+    if (e == cudaSuccess) e = cudaGraphInstantiate(&op->gexec, g, 0);
+    cudaGraphDestroy(g);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        op->gexec = nullptr;
+        set_last_error(std::string("loop graph: ") + cudaGetErrorString(e));
+        return MAS_ERR_CUDA;
+    }
+    op->g_x = a.x;
+    op->g_hist = a.rho_hist;
     return MAS_OK;
 }
 
@@ -375,6 +438,8 @@ mas_status_t mas_op_setup(mas_grid_t* g, int ncomp, const double* kappa, const d
     G.wPm = t; t += np;
     G.wPp = t; t += np;
     G.vp = t;
+    const char* g_env = getenv("MAS_NO_GRAPH");  // experiment hook: host-driven loop
+    op->use_graph = !(g_env && atoi(g_env));
     const char* ch_env = getenv("MAS_CHUNK");  // experiment hook
     op->chunk = ch_env ? atoi(ch_env) : (nl >= 128 ? 32 : nl >= 64 ? 16 : (nl >= 16 ? 8 : 4));
     if (op->chunk < 1 || op->chunk > 32) op->chunk = 16;
@@ -610,8 +675,13 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
     a.out = op->q;
     a.x = xd;
     a.f = nullptr;
+    const bool graph = !comm && !op->prof && op->use_graph;
+    if (graph) {
+        ST(loop_graph(op, a, b));
+        CU(cudaGraphLaunch(op->gexec, s));
+    }
     int stop_seen_at = -1;
-    for (int k = 1; k <= maxit + 1; k++) {
+    for (int k = 1; !graph && k <= maxit + 1; k++) {
         double* pold = op->p[(k + 1) & 1];
         double* pnew = op->p[k & 1];
         if (comm) {
@@ -662,6 +732,10 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
     }
     *iters = fin.iters;
     *relres = fin.relres;
+    if (graph) {  // init + 4 kernels per executed loop body (two iterations)
+        const int last_a = fin.status == MAS_ERR_BREAKDOWN ? fin.iters : fin.iters + 1;
+        op->launches += 4LL * ((last_a + 1) / 2);
+    }
     if (res_hist) {
         // after a breakdown at iteration k only ||r_0..r_{k-1}|| exist
         const int nh = fin.status == MAS_ERR_BREAKDOWN ? fin.iters : fin.iters + 1;

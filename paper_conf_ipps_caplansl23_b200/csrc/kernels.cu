@@ -451,6 +451,7 @@ __global__ void __launch_bounds__(kSThreads, MAS_MINB) k_stencil(const StencilAr
                 __threadfence_system();
                 *(volatile int*)a.host_flag = kit;
             }
+            if (a.cond) cudaGraphSetConditional((cudaGraphConditionalHandle)a.cond, 0);
         }
         return;
     }
@@ -662,6 +663,7 @@ __global__ void __launch_bounds__(kThreads) k_pcg_b(const StreamArgs a) {
                 __threadfence_system();
                 *(volatile int*)a.host_flag = kit;
             }
+            if (a.cond) cudaGraphSetConditional((cudaGraphConditionalHandle)a.cond, 0);
         } else {
             a.sigma_hist[kit] = sigma;
             st->pend_rho = acc[0];

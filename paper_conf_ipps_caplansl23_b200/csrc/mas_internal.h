@@ -87,7 +87,8 @@ struct StencilArgs {
     double* sigma_hist;       // [maxit+2]
     double* rr_hist;          // [maxit+2]
     Scratch scr;
-    int* host_flag;           // mapped pinned int set to 1 when the solve stops
+    int* host_flag;           // mapped pinned int: iteration at which the solve stopped
+    unsigned long long cond;  // CUDA graph while-loop handle (0: not in a graph)
 };
 
 struct StreamArgs {  // kernel B
@@ -102,6 +103,7 @@ struct StreamArgs {  // kernel B
     double* rr_hist;
     Scratch scr;
     int* host_flag;
+    unsigned long long cond;
 };
 
 // launchers (kernels.cu)
