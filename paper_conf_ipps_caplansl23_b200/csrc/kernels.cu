@@ -34,6 +34,9 @@ constexpr int kThreads = 256;  // 8 warps (stream kernels)
 #ifndef MAS_MINB
 #define MAS_MINB 2
 #endif
+#ifndef MAS_MINB1
+#define MAS_MINB1 3
+#endif
 constexpr int TJ = MAS_TJ;     // theta rows per stencil tile (one warp per row)
 constexpr int kSThreads = 32 * TJ;
 constexpr int kMaxChunk = 32;  // r-planes per stencil work item (host picks <= this)
@@ -366,7 +369,7 @@ __device__ __forceinline__ void ghost_plane(double* buf, int height, int width, 
 //                 -> p_{i+1} into the ring (and x-update / p store)
 //   sync; stencil(i) from the ring only (r-neighbours = adjacent slots); sync
 template <int MODE, int NC>
-__global__ void __launch_bounds__(kSThreads, MAS_MINB) k_stencil(const StencilArgs a) {
+__global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_stencil(const StencilArgs a) {
     extern __shared__ __align__(16) double smem[];
     constexpr int BUF = (NC + 1) * HROWS * ROW;
     const Geo& g = a.g;
@@ -623,11 +626,16 @@ __global__ void __launch_bounds__(kThreads) k_pcg_b(const StreamArgs a) {
         const long long Nl = (long long)g.nl * g.plane;
         const int rows = g.nl * g.nt;
         const int half = g.np >> 1;
-        for (int row = blockIdx.x; row < rows; row += gridDim.x) {
+        // a block covers rpi whole (r,theta) rows per step when a row has
+        // fewer double2 pairs than the block has threads
+        const int tpr = min(kThreads, half), rpi = kThreads / tpr;
+        const int sub = threadIdx.x / tpr, col = threadIdx.x - sub * tpr;
+        if (sub >= rpi) goto reduce;
+        for (int row = blockIdx.x * rpi + sub; row < rows; row += gridDim.x * rpi) {
             const int i = row / g.nt, j = row - i * g.nt;
             const double wrow = __ldg(g.vr + i) * __ldg(g.vt + j);
             const long long base = (long long)row * g.np;
-            for (int h = threadIdx.x; h < half; h += kThreads) {
+            for (int h = col; h < half; h += tpr) {
                 const int k = 2 * h;
                 const double2 di = ld2(a.dinv + base + k);
                 const double V0 = wrow * __ldg(g.vp + k), V1 = wrow * __ldg(g.vp + k + 1);
@@ -650,6 +658,7 @@ __global__ void __launch_bounds__(kThreads) k_pcg_b(const StreamArgs a) {
             }
         }
     }
+reduce:
     if (grid_reduce<2>(acc, a.scr, TKT_B) && threadIdx.x == 0) {
         PcgState* st = a.st;
         if (brk) {
