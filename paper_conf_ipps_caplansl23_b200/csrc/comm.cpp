@@ -6,23 +6,76 @@
 // per GPU (as the paper's launch script, Listing 6), NCCL
 // send/recv of the contiguous r-seam planes (layout R15 makes them
 // contiguous, no packing) and an in-place fp64 allreduce of 1-3 scalars.
+//
+// A second transport, "virtual ranks", runs P ranks as P host threads of one
+// process on ONE GPU (each with its own stream).  It implements the same two
+// collectives with device copies, CUDA events and host barriers, so the
+// multi-rank driver, ghost-plane kernels and stop handshake can be validated
+// on a single B200 (this run has no multi-GPU box).  It is selected by a
+// mas_dist_t.nccl_id beginning with "MASVIRT\0" followed by an 8-byte group
+// key.  It is a test transport, not a performance path.
 #include <nccl.h>
 
+#include <condition_variable>
 #include <cstring>
+#include <map>
+#include <mutex>
 #include <string>
+#include <vector>
 
 #include "grid.h"
 
 namespace mas {
 
+// ---------------------------------------------------------------------------
+// virtual-rank group
+// ---------------------------------------------------------------------------
+struct VGroup {
+    int n = 0;
+    int refs = 0;
+    std::mutex m;
+    std::condition_variable cv;
+    int arrived = 0;
+    long gen = 0;
+    double* stage = nullptr;                   // [n][8] allreduce staging (device)
+    std::vector<cudaEvent_t> ev_in, ev_out;    // per rank: staged / summed
+    std::vector<cudaEvent_t> ev_seam, ev_pull; // per rank: seam data ready / pulls done
+    std::vector<const double*> seam_src;       // per rank: interior field of this seam call
+    std::vector<int> seam_nl;
+
+    void barrier() {
+        std::unique_lock<std::mutex> lk(m);
+        const long g = gen;
+        if (++arrived == n) {
+            arrived = 0;
+            gen++;
+            cv.notify_all();
+        } else {
+            cv.wait(lk, [&] { return gen != g; });
+        }
+    }
+};
+
+static std::mutex g_vmap_mutex;
+static std::map<unsigned long long, VGroup*> g_vmap;
+
 struct Comm {
     ncclComm_t nccl = nullptr;
     int nranks = 1, rank = 0;
+    VGroup* vg = nullptr;
+    unsigned long long vkey = 0;
 };
+
+static const char kVirtMagic[8] = {'M', 'A', 'S', 'V', 'I', 'R', 'T', 0};
 
 static mas_status_t nccl_fail(ncclResult_t r, const char* what) {
     set_last_error(std::string(what) + ": " + ncclGetErrorString(r));
     return MAS_ERR_NCCL;
+}
+
+static mas_status_t cuda_fail(cudaError_t e, const char* what) {
+    set_last_error(std::string(what) + ": " + cudaGetErrorString(e));
+    return MAS_ERR_CUDA;
 }
 
 mas_status_t comm_unique_id(unsigned char out[128]) {
@@ -34,10 +87,59 @@ mas_status_t comm_unique_id(unsigned char out[128]) {
     return MAS_OK;
 }
 
+static mas_status_t vgroup_join(const mas_dist_t* d, Comm* c) {
+    unsigned long long key;
+    memcpy(&key, d->nccl_id + 8, 8);
+    VGroup* g;
+    {
+        std::lock_guard<std::mutex> lk(g_vmap_mutex);
+        auto it = g_vmap.find(key);
+        if (it == g_vmap.end()) {
+            g = new VGroup();
+            g->n = d->nranks;
+            g->ev_in.resize(g->n);
+            g->ev_out.resize(g->n);
+            g->ev_seam.resize(g->n);
+            g->ev_pull.resize(g->n);
+            g->seam_src.assign(g->n, nullptr);
+            g->seam_nl.assign(g->n, 0);
+            cudaError_t e = cudaMalloc(&g->stage, sizeof(double) * 8 * g->n);
+            for (int r = 0; r < g->n && e == cudaSuccess; r++) {
+                e = cudaEventCreateWithFlags(&g->ev_in[r], cudaEventDisableTiming);
+                if (e == cudaSuccess) e = cudaEventCreateWithFlags(&g->ev_out[r], cudaEventDisableTiming);
+                if (e == cudaSuccess) e = cudaEventCreateWithFlags(&g->ev_seam[r], cudaEventDisableTiming);
+                if (e == cudaSuccess) e = cudaEventCreateWithFlags(&g->ev_pull[r], cudaEventDisableTiming);
+            }
+            if (e != cudaSuccess) return cuda_fail(e, "virtual group setup");
+            g_vmap[key] = g;
+        } else {
+            g = it->second;
+            if (g->n != d->nranks) {
+                set_last_error("virtual group: nranks mismatch");
+                return MAS_ERR_ARG;
+            }
+        }
+        g->refs++;
+    }
+    c->vg = g;
+    c->vkey = key;
+    g->barrier();  // collective create
+    return MAS_OK;
+}
+
 mas_status_t comm_create(const mas_dist_t* d, Comm** out) {
     Comm* c = new Comm();
     c->nranks = d->nranks;
     c->rank = d->rank;
+    if (memcmp(d->nccl_id, kVirtMagic, 8) == 0) {
+        mas_status_t s = vgroup_join(d, c);
+        if (s != MAS_OK) {
+            delete c;
+            return s;
+        }
+        *out = c;
+        return MAS_OK;
+    }
     ncclUniqueId id;
     memcpy(id.internal, d->nccl_id, 128);
     ncclResult_t r = ncclCommInitRank(&c->nccl, d->nranks, id, d->rank);
@@ -52,18 +154,99 @@ mas_status_t comm_create(const mas_dist_t* d, Comm** out) {
 void comm_destroy(Comm* c) {
     if (!c) return;
     if (c->nccl) ncclCommDestroy(c->nccl);
+    if (c->vg) {
+        VGroup* g = c->vg;
+        g->barrier();
+        std::lock_guard<std::mutex> lk(g_vmap_mutex);
+        if (--g->refs == 0) {
+            for (int r = 0; r < g->n; r++) {
+                cudaEventDestroy(g->ev_in[r]);
+                cudaEventDestroy(g->ev_out[r]);
+                cudaEventDestroy(g->ev_seam[r]);
+                cudaEventDestroy(g->ev_pull[r]);
+            }
+            cudaFree(g->stage);
+            g_vmap.erase(c->vkey);
+            delete g;
+        }
+    }
     delete c;
+}
+
+// ---------------------------------------------------------------------------
+// allreduce (sum, fp64, n <= 8)
+// ---------------------------------------------------------------------------
+static mas_status_t v_allreduce(Comm* c, double* buf, int n, cudaStream_t s) {
+    VGroup* g = c->vg;
+    const int r = c->rank;
+    cudaError_t e;
+    // stage[r] may still be read by the previous call's sums of other ranks
+    for (int j = 0; j < g->n; j++)
+        if (j != r && (e = cudaStreamWaitEvent(s, g->ev_out[j], 0)) != cudaSuccess)
+            return cuda_fail(e, "virtual allreduce wait");
+    if ((e = cudaMemcpyAsync(g->stage + 8 * r, buf, sizeof(double) * n, cudaMemcpyDeviceToDevice, s)) !=
+            cudaSuccess ||
+        (e = cudaEventRecord(g->ev_in[r], s)) != cudaSuccess)
+        return cuda_fail(e, "virtual allreduce stage");
+    g->barrier();
+    for (int j = 0; j < g->n; j++)
+        if ((e = cudaStreamWaitEvent(s, g->ev_in[j], 0)) != cudaSuccess)
+            return cuda_fail(e, "virtual allreduce wait");
+    if ((e = launch_rank_sum(buf, g->stage, g->n, n, s)) != cudaSuccess ||
+        (e = cudaEventRecord(g->ev_out[r], s)) != cudaSuccess)
+        return cuda_fail(e, "virtual allreduce sum");
+    g->barrier();
+    return MAS_OK;
 }
 
 mas_status_t comm_allreduce(Comm* c, double* buf, int n, cudaStream_t s) {
     if (!c || c->nranks == 1) return MAS_OK;
+    if (c->vg) return v_allreduce(c, buf, n, s);
     ncclResult_t r = ncclAllReduce(buf, buf, n, ncclFloat64, ncclSum, c->nccl, s);
     return r == ncclSuccess ? MAS_OK : nccl_fail(r, "ncclAllReduce");
+}
+
+// ---------------------------------------------------------------------------
+// seams: edge r-planes to the r-neighbours' ghost planes
+// ---------------------------------------------------------------------------
+static mas_status_t v_seams(Comm* c, const double* in, int ncomp, int nl, long long plane,
+                            double* glo, double* ghi, cudaStream_t s) {
+    VGroup* g = c->vg;
+    const int r = c->rank;
+    cudaError_t e;
+    g->seam_src[r] = in;
+    g->seam_nl[r] = nl;
+    if ((e = cudaEventRecord(g->ev_seam[r], s)) != cudaSuccess) return cuda_fail(e, "virtual seam record");
+    g->barrier();
+    const size_t bytes = sizeof(double) * plane;
+    for (int side = 0; side < 2; side++) {
+        const int nb = side == 0 ? r - 1 : r + 1;
+        if (nb < 0 || nb >= g->n) continue;
+        if ((e = cudaStreamWaitEvent(s, g->ev_seam[nb], 0)) != cudaSuccess)
+            return cuda_fail(e, "virtual seam wait");
+        const double* src = g->seam_src[nb];
+        const int nbl = g->seam_nl[nb];
+        for (int m = 0; m < ncomp; m++) {
+            // lower neighbour's last plane -> my glo; upper neighbour's first plane -> my ghi
+            const double* from = src + ((long long)m * nbl + (side == 0 ? nbl - 1 : 0)) * plane;
+            double* to = (side == 0 ? glo : ghi) + (long long)m * plane;
+            if ((e = cudaMemcpyAsync(to, from, bytes, cudaMemcpyDeviceToDevice, s)) != cudaSuccess)
+                return cuda_fail(e, "virtual seam copy");
+        }
+    }
+    if ((e = cudaEventRecord(g->ev_pull[r], s)) != cudaSuccess) return cuda_fail(e, "virtual seam record");
+    g->barrier();
+    // my edge planes must not be overwritten before the neighbours pulled them
+    for (int nb : {r - 1, r + 1})
+        if (nb >= 0 && nb < g->n && (e = cudaStreamWaitEvent(s, g->ev_pull[nb], 0)) != cudaSuccess)
+            return cuda_fail(e, "virtual seam wait");
+    return MAS_OK;
 }
 
 mas_status_t comm_seams(Comm* c, const double* in, int ncomp, int nl, long long plane, double* glo,
                         double* ghi, cudaStream_t s) {
     if (!c || c->nranks == 1) return MAS_OK;
+    if (c->vg) return v_seams(c, in, ncomp, nl, plane, glo, ghi, s);
     const long long Nl = (long long)nl * plane;
     ncclResult_t r = ncclGroupStart();
     if (r != ncclSuccess) return nccl_fail(r, "ncclGroupStart");
@@ -85,6 +268,11 @@ mas_status_t comm_seams(Comm* c, const double* in, int ncomp, int nl, long long 
 
 mas_status_t comm_barrier(Comm* c, cudaStream_t s) {
     if (!c || c->nranks == 1) return MAS_OK;
+    if (c->vg) {
+        if (cudaStreamSynchronize(s) != cudaSuccess) return MAS_ERR_CUDA;
+        c->vg->barrier();
+        return MAS_OK;
+    }
     double* d = nullptr;
     if (cudaMallocAsync(&d, sizeof(double), s) != cudaSuccess) return MAS_ERR_CUDA;
     cudaMemsetAsync(d, 0, sizeof(double), s);

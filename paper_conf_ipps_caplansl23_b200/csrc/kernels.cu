@@ -825,6 +825,20 @@ cudaError_t launch_dirichlet(const Geo& g, int ncomp, const double* kappa, const
     return cudaGetLastError();
 }
 
+__global__ void k_rank_sum(double* out, const double* stage, int nranks, int n) {
+    const int t = threadIdx.x;
+    if (t < n) {
+        double s = 0.0;
+        for (int r = 0; r < nranks; r++) s += stage[8 * r + t];
+        out[t] = s;
+    }
+}
+
+cudaError_t launch_rank_sum(double* out, const double* stage, int nranks, int n, cudaStream_t s) {
+    k_rank_sum<<<1, 32, 0, s>>>(out, stage, nranks, n);
+    return cudaGetLastError();
+}
+
 cudaError_t launch_dot(const Geo& g, int ncomp, const double* a, const double* b, Scratch scr,
                        double* out, int nblocks, cudaStream_t s) {
     k_dot<<<nblocks, kThreads, 0, s>>>(g, ncomp, a, b, scr, out);

@@ -116,8 +116,8 @@ cudaError_t launch_dirichlet(const Geo& g, int ncomp, const double* kappa, const
                              int outer, double* f, cudaStream_t s);
 cudaError_t launch_dot(const Geo& g, int ncomp, const double* a, const double* b, Scratch scr,
                        double* out, int nblocks, cudaStream_t s);
-cudaError_t launch_check_coeffs(long long n, const double* kappa, const double* c, int* bad,
-                                cudaStream_t s);
+// out[t] = sum_r stage[8r + t], t < n, ranks summed in rank order (virtual-rank allreduce)
+cudaError_t launch_rank_sum(double* out, const double* stage, int nranks, int n, cudaStream_t s);
 
 void set_last_error(const std::string& msg);
 

@@ -126,6 +126,12 @@ def mas_comm_unique_id() -> bytes:
     return bytes(buf)
 
 
+def virtual_ranks_id(key: int) -> bytes:
+    """mas_dist_t.nccl_id selecting the in-process "virtual ranks" transport:
+    P ranks as P host threads on one GPU (test transport, see comm.cpp)."""
+    return b"MASVIRT\0" + int(key).to_bytes(8, "little") + bytes(112)
+
+
 def mas_grid_create(r_node, r_half, t_node, t_half, p_node, p_half, pole_flags=3,
                     periodic_phi=1, dist: Optional[tuple] = None) -> int:
     """dist = (nranks, rank, nccl_id_bytes) or None.  Returns the handle."""

@@ -1,0 +1,115 @@
+"""The multi-rank (r-slab) path of the library on ONE B200: P ranks run as P
+host threads, each with its own CUDA stream, connected by the library's
+"virtual ranks" transport (comm.cpp) instead of NCCL.  Everything else is the
+production multi-rank code: the slab partition, ghost-plane kernels,
+seam/allreduce placement in the host-driven PCG loop and the stop handshake.
+
+Parity: P slabs vs the oracle on the same global problem:
+matvec <= 1e-13, PCG iterations +-1 and x <= 1e-10.
+"""
+import math
+import threading
+
+import numpy as np
+import pytest
+
+from paper_conf_ipps_caplansl23_b200 import workloads as W
+
+pytestmark = pytest.mark.gpu
+torch = pytest.importorskip("torch")
+
+_key = [1000]
+
+
+@pytest.fixture(scope="module")
+def mp():
+    if not torch.cuda.is_available():
+        pytest.skip("needs a GPU")
+    from paper_conf_ipps_caplansl23_b200 import build
+    build.build()
+    from paper_conf_ipps_caplansl23_b200 import maspcg
+    return maspcg
+
+
+def run_ranks(mp, prob, P, x_apply, want_solve=True, maxit=None, tol=None):
+    _key[0] += 1
+    vid = mp.virtual_ranks_id(_key[0])
+    res, errs = {}, []
+
+    def rank_main(r):
+        try:
+            torch.cuda.set_device(0)
+            s = torch.cuda.Stream()
+            with torch.cuda.stream(s):
+                g = mp.Grid(prob.mesh, dist=(P, r, vid))
+                i0, nl = g.i0, g.nl
+                sl = slice(i0, i0 + nl)
+                d = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()
+                op = mp.Operator(g, prob.ncomp, d(prob.kappa[sl]), d(prob.c[sl]), prob.bc_inner,
+                                 prob.bc_outer)
+                y = torch.empty((prob.ncomp, nl) + prob.shape[1:], dtype=torch.float64, device="cuda")
+                op.apply(d(x_apply[:, sl]), y)
+                out = {"i0": i0, "nl": nl, "y": None, "dot": None}
+                torch.cuda.current_stream().synchronize()
+                out["y"] = y.cpu().numpy()
+                out["dot"] = op.dot(d(x_apply[:, sl]), d(x_apply[:, sl]))
+                if want_solve:
+                    f = d(prob.f[:, sl])
+                    ubi = d(prob.ub_inner) if prob.ub_inner is not None else None
+                    op.dirichlet_rhs(ubi, None, f)
+                    x = d(prob.x0[:, sl])
+                    st, it, rel, hist = op.solve(f, x, prob.tol if tol is None else tol,
+                                                 prob.maxit if maxit is None else maxit, True)
+                    torch.cuda.current_stream().synchronize()
+                    out.update(st=st, it=it, rel=rel, x=x.cpu().numpy(), launches=op.launch_count)
+                op.close()
+                g.close()
+                res[r] = out
+        except Exception as e:  # noqa: BLE001
+            errs.append((r, repr(e)))
+
+    th = [threading.Thread(target=rank_main, args=(r,)) for r in range(P)]
+    for t in th:
+        t.start()
+    for t in th:
+        t.join(timeout=600)
+    assert not errs, errs
+    assert len(res) == P
+    return [res[r] for r in range(P)]
+
+
+@pytest.mark.parametrize("P", [2, 3, 4])
+def test_virtual_ranks_apply_dot_and_pcg(mp, oracle_mod, P):
+    prob = W.viscosity_problem(13, 16, 64, warm=False)
+    x = W.random_field((3,) + prob.shape, 42)
+    out = run_ranks(mp, prob, P, x)
+    o = oracle_mod.Oracle.for_problem(prob)
+    V = o.volumes()[None]
+    # matvec, assembled from the slabs
+    y = np.concatenate([r["y"] for r in out], axis=1)
+    yo = o.apply(prob.kappa, prob.c, x)
+    assert math.sqrt((V * (y - yo) ** 2).sum() / (V * yo ** 2).sum()) <= 1e-13
+    # global dot through the allreduce
+    for r in out:
+        assert abs(r["dot"] - o.dot(x, x)) <= 1e-13 * o.dot(x, x)
+    # PCG
+    rc, xo, ito, _, _ = oracle_mod.solve_problem(prob)
+    its = {r["it"] for r in out}
+    assert len(its) == 1, its  # every rank stopped at the same iteration
+    it = its.pop()
+    assert all(r["st"] == mp.MAS_OK for r in out)
+    assert abs(it - ito) <= 1
+    xg = np.concatenate([r["x"] for r in out], axis=1)
+    if it == ito:
+        assert math.sqrt((V * (xg - xo) ** 2).sum() / (V * xo ** 2).sum()) <= 1e-10
+
+
+def test_virtual_ranks_conduction_dirichlet_and_fixed_iterations(mp, oracle_mod):
+    prob = W.conduction_problem(10, 24, 32)
+    x = W.random_field((1,) + prob.shape, 43)
+    out = run_ranks(mp, prob, 3, x, tol=0.0, maxit=25)
+    rc, xo, ito, _, _ = oracle_mod.solve_problem(prob, tol=0.0, maxit=25)
+    assert all(r["st"] == mp.MAS_NOT_CONVERGED and r["it"] == 25 for r in out)
+    xg = np.concatenate([r["x"] for r in out], axis=1)
+    V = oracle_mod.Oracle.for_problem(prob).volumes()[None]
+    assert math.sqrt((V * (xg - xo) ** 2).sum() / (V * xo ** 2).sum()) <= 1e-10
