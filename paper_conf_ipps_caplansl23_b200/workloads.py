@@ -210,6 +210,44 @@ def viscosity_problem(nr=256, nt=256, np_=512, r0=1.0, r1=30.0, R=200.0, D_max=1
                    tol, maxit, extra={"dt": dt})
 
 
+@dataclasses.dataclass
+class LongRun:
+    """C5: repeated implicit steps of conduction then viscosity,
+    warm-started, Delta t frozen at step 0.  Per step n (harness arithmetic,
+    not the PCG path): kappa_T = (T^n)^(5/2), rhs_T = c_T T^n (+ Dirichlet
+    T_b at r0); rhs_v = c_v v^n."""
+    mesh: Mesh
+    T0: np.ndarray      # [nr,nt,np]
+    v0: np.ndarray      # [3,nr,nt,np]
+    rho: np.ndarray     # [nr,nt,np]
+    c_T: np.ndarray     # rho / ((gamma-1) dt_T)
+    c_v: np.ndarray     # rho / dt_v
+    T_b: np.ndarray     # [1,nt,np] inner Dirichlet temperature
+    dt_T: float
+    dt_v: float
+    tol: float = 1e-12
+    maxit: int = 20000
+
+
+def longrun_problem(nr=320, nt=300, np_=600, r0=1.0, r1=30.0, R=200.0, D_T=1000.0,
+                    D_v=100.0) -> LongRun:
+    m = stretched_mesh(nr, nt, np_, r0, r1, R)
+    gT = texture(m.tC, m.pC, 1)
+    grho = texture(m.tC, m.pC, 2)
+    r = m.rC[:, None, None]
+    T = np.ascontiguousarray(np.broadcast_to(_temperature(r, gT[None]), (nr, nt, np_)))
+    rho = np.ascontiguousarray(np.broadcast_to(_density(r, grho[None]), (nr, nt, np_)))
+    rho_c = rho / (GAMMA - 1.0)
+    dt_T = D_T / _diffusion_number_scale(m, T ** 2.5, rho_c)
+    dt_v = D_v / _diffusion_number_scale(m, rho, rho)
+    v = np.empty((3, nr, nt, np_))
+    prof = np.sin(math.pi * (m.rC - r0) / (r1 - r0))[:, None, None]
+    for comp in range(3):
+        v[comp] = prof * texture(m.tC, m.pC, 10 + comp)[None]
+    return LongRun(m, T, v, rho, rho_c / dt_T, rho / dt_v,
+                   _temperature(np.float64(m.rF[0]), gT)[None].copy(), dt_T, dt_v)
+
+
 def random_field(shape, seed=42) -> np.ndarray:
     """Matvec-parity input: U[-1,1] i.i.d."""
     return np.random.default_rng(seed).uniform(-1.0, 1.0, size=shape)
