@@ -236,10 +236,29 @@ __device__ __forceinline__ HaloMeta halo_meta(const Geo& g, int j0, int k0, int 
 template <int NC>
 struct Stage {
     Raw<NC> R;                          // own double2 pair
-    double hu[NC], hpo[NC], hdi, hkap;  // halo scalar cell
     double2 xv[NC];                     // own x (PCGA deferred update)
     OwnRegs<NC> o;                      // own c (+ f, D^-1 for RESID)
 };
+
+// --- cp.async (LDGSTS) for the halo items --------------------------------
+// The scalar halo items do not fit in registers next to the own pair's
+// in-flight loads (ptxas spilled them, forcing an early wait), so each halo
+// thread copies its item into a private shared-memory slot instead:
+// layout [field][kHaloSlots], fields 0 kappa, 1 1/D, 2.. u[NC], po[NC].
+constexpr int kHaloSlots = 2 * TK + 2 * TJ;
+__device__ __forceinline__ void cpa8(double* sdst, const double* gsrc) {
+    const unsigned sa = (unsigned)__cvta_generic_to_shared(sdst);
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"(sa), "l"(gsrc) : "memory");
+}
+__device__ __forceinline__ void cpa_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
+__device__ __forceinline__ void cpa_wait_all() { asm volatile("cp.async.wait_group 0;\n" ::: "memory"); }
+
+// dynamic shared memory: [4-slot ring][halo staging]
+template <int NC>
+__device__ __forceinline__ double* halo_stage() {
+    extern __shared__ __align__(16) double dyn_smem[];
+    return dyn_smem + 4 * (NC + 1) * HROWS * ROW;
+}
 
 template <int MODE, int NC>
 __device__ __forceinline__ void stage_issue(const StencilArgs& a, int i, int j0, int k0, int height,
@@ -250,6 +269,7 @@ __device__ __forceinline__ void stage_issue(const StencilArgs& a, int i, int j0,
     const int kc = 2 * lane;
     const long long Nl = (long long)g.nl * g.plane;
     const PlanePtrs<NC> P = plane_ptrs<MODE, NC>(a, i, first);
+    double* hst = halo_stage<NC>();
     if (w < height && kc < width) {
         const long long off = (long long)(j0 + w) * g.np + k0 + kc;
         const long long o3 = (long long)i * g.plane + off;
@@ -268,17 +288,19 @@ __device__ __forceinline__ void stage_issue(const StencilArgs& a, int i, int j0,
         }
     }
     if (halo && hm.hkind == 1) {
-        S.hkap = __ldg(P.kap + hm.hoff);
+        double* h = hst + threadIdx.x;
+        cpa8(h, P.kap + hm.hoff);
 #pragma unroll
-        for (int c = 0; c < NC; c++) S.hu[c] = __ldg(P.u[c] + hm.hoff);
+        for (int c = 0; c < NC; c++) cpa8(h + (2 + c) * kHaloSlots, P.u[c] + hm.hoff);
         if (MODE == MODE_PCGA) {
-            S.hdi = __ldg(P.di + hm.hoff);
+            cpa8(h + kHaloSlots, P.di + hm.hoff);
             if (!first) {
 #pragma unroll
-                for (int c = 0; c < NC; c++) S.hpo[c] = __ldg(P.po[c] + hm.hoff);
+                for (int c = 0; c < NC; c++) cpa8(h + (2 + NC + c) * kHaloSlots, P.po[c] + hm.hoff);
             }
         }
     }
+    cpa_commit();
 }
 
 template <int MODE, int NC>
@@ -316,16 +338,19 @@ __device__ __forceinline__ void stage_commit(const StencilArgs& a, int i, int j0
         }
     }
     if (halo && hm.hkind == 1) {
+        double* hst = halo_stage<NC>();
+        cpa_wait_all();  // this thread's own copies; read back below by the same thread
+        const double* h = hst + threadIdx.x;
 #pragma unroll
         for (int c = 0; c < NC; c++) {
-            double u = S.hu[c];
+            double u = h[(2 + c) * kHaloSlots];
             if (MODE == MODE_PCGA) {
-                const double z = S.hdi * u;
-                u = first ? z : fma(beta, S.hpo[c], z);
+                const double z = h[kHaloSlots] * u;
+                u = first ? z : fma(beta, h[(2 + NC + c) * kHaloSlots], z);
             }
             sfield(buf, c)[hm.hidx] = u;
         }
-        sfield(buf, NC)[hm.hidx] = S.hkap;
+        sfield(buf, NC)[hm.hidx] = h[0];
     } else if (halo && hm.hkind == 3) {
 #pragma unroll
         for (int c = 0; c <= NC; c++) sfield(buf, c)[hm.hidx] = 0.0;
@@ -772,7 +797,7 @@ static cudaError_t launch_one(const StencilArgs& a0, cudaStream_t s) {
     a.ntj = (a.g.nt + TJ - 1) / TJ;
     a.ntk = (a.g.np + TK - 1) / TK;
     a.nchunk = (a.g.nl + a.chunk - 1) / a.chunk;
-    const int smem = 4 * (NC + 1) * HROWS * ROW * (int)sizeof(double);
+    const int smem = (4 * (NC + 1) * HROWS * ROW + (2 + 2 * NC) * kHaloSlots) * (int)sizeof(double);
     static bool attr_done = false;
     if (!attr_done) {
         cudaError_t e = cudaFuncSetAttribute(k_stencil<MODE, NC>,
