@@ -442,7 +442,7 @@ mas_status_t mas_op_setup(mas_grid_t* g, int ncomp, const double* kappa, const d
     op->use_graph = !(g_env && atoi(g_env));
     const char* ch_env = getenv("MAS_CHUNK");  // experiment hook
     op->chunk = ch_env ? atoi(ch_env) : (nl >= 128 ? 32 : nl >= 64 ? 16 : (nl >= 16 ? 8 : 4));
-    if (op->chunk < 1 || op->chunk > 32) op->chunk = 16;
+    if (op->chunk < 1 || op->chunk > 64) op->chunk = 16;
     op->max_blocks = stencil_blocks(G, op->chunk);
     op->b_blocks = 148 * 8;
     if (op->b_blocks > op->max_blocks) op->max_blocks = op->b_blocks;

@@ -39,7 +39,10 @@ constexpr int kThreads = 256;  // 8 warps (stream kernels)
 #endif
 constexpr int TJ = MAS_TJ;     // theta rows per stencil tile (one warp per row)
 constexpr int kSThreads = 32 * TJ;
-constexpr int kMaxChunk = 32;  // r-planes per stencil work item (host picks <= this)
+#ifndef MAS_MAXCHUNK
+#define MAS_MAXCHUNK 32
+#endif
+constexpr int kMaxChunk = MAS_MAXCHUNK;  // r-planes per stencil work item (host picks <= this)
 constexpr int TK = 64;         // phi cells per tile (2 per lane, double2)
 constexpr int OFF = 2;         // smem column of the first tile cell (16B aligned)
 constexpr int ROW = TK + 4;    // smem row length: [pad][halo][64 cells][halo][pad]
@@ -521,13 +524,17 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
     double2 kown = make_double2(0.0, 0.0), kdummy;
     const bool lo_ghost = (ia == 0) && g.glob_lo;
     const HaloMeta hm = halo_meta(g, j0, k0, height, width);
+    // planes ia-1 (own cells only) and ia: both loads in flight together
+    Stage<NC> S0, S;
     if (!lo_ghost)
-        produce_tile<MODE, NC>(a, ia - 1, slot(ia - 1), j0, k0, height, width, hm, first, beta,
-                               alpha_prev, false, false, false, kdummy, on);
-    produce_tile<MODE, NC>(a, ia, slot(ia), j0, k0, height, width, hm, first, beta, alpha_prev, xupd,
-                           true, true, kown, oc);
+        stage_issue<MODE, NC>(a, ia - 1, j0, k0, height, width, hm, first, false, false, false, S0);
+    stage_issue<MODE, NC>(a, ia, j0, k0, height, width, hm, first, xupd, true, true, S);
+    if (!lo_ghost)
+        stage_commit<MODE, NC>(a, ia - 1, j0, k0, height, width, hm, first, beta, alpha_prev, false,
+                               false, false, S0, slot(ia - 1), kdummy, on);
+    stage_commit<MODE, NC>(a, ia, j0, k0, height, width, hm, first, beta, alpha_prev, xupd, true, true,
+                           S, slot(ia), kown, oc);
     if (lo_ghost) ghost_plane<NC>(slot(ia - 1), height, width, kown);
-    Stage<NC> S;
     if (real_plane(ia + 1))
         stage_issue<MODE, NC>(a, ia + 1, j0, k0, height, width, hm, first, xupd && (ia + 1 < ib),
                               ia + 1 < ib, ia + 1 < ib, S);
