@@ -41,6 +41,8 @@ UNIT = "PCG iters/s"
 CONFIGS = {
     # name: (kind, nr, nt, np)
     "C3": ("viscosity", 256, 256, 512),
+    # C4: weak scaling, (256 * N) x 256 x 512 on N GPUs (nr scaled below)
+    "C4": ("viscosity", 256, 256, 512),
     "C2": ("conduction", 128, 128, 256),
     "C1": ("mms", 16, 24, 32),
 }
@@ -114,9 +116,15 @@ class ClockSampler:
                 "reasons": sorted(reasons), "samples": len(sm)}
 
 
-def make_problem(cfg: str):
+def make_problem(cfg: str, world: int = 1):
     kind, nr, nt, np_ = CONFIGS[cfg]
+    if cfg == "C4":
+        nr *= world
     return W.make(kind, nr=nr, nt=nt, np_=np_)
+
+
+def scaling_of(cfg: str) -> str:
+    return "weak" if cfg == "C4" else "strong"
 
 
 def cpu_cores() -> int:
@@ -166,7 +174,8 @@ def run_reference(args):
               f"oracle PCG iterations per step incl. its setup (diag + initial residual)")
     line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * dt / args.steps,
-            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
+            "higher_is_better": True, "scaling": scaling_of(args.config), "vs_baseline": None,
+            "dtype": "f64",
             "data": "synthetic", "impl": "reference",
             "config": {"workload": args.config, "grid": list(prob.shape), "ncomp": prob.ncomp},
             "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle",
@@ -208,7 +217,7 @@ def main():
         dist.barrier()
     from paper_conf_ipps_caplansl23_b200 import maspcg as M
 
-    prob = make_problem(args.config)
+    prob = make_problem(args.config, world)
     nr, nt, np_ = prob.shape
     distinfo = None
     if world > 1:
@@ -352,7 +361,7 @@ def main():
         line = {
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": t_ms / args.steps,
-            "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
+            "higher_is_better": True, "scaling": scaling_of(args.config), "vs_baseline": None,
             "dtype": "f64", "data": "synthetic",
             "config": {"workload": args.config, "grid": [nr, nt, np_], "ncomp": nc,
                        "cells": cells, "tol": args.tol, "iters_per_solve": iters_per_solve,
