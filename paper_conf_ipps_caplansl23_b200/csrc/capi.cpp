@@ -95,6 +95,10 @@ struct mas_op {
     int b_blocks = 0;
     int max_blocks = 0;
     cudaEvent_t ev[2] = {nullptr, nullptr};
+    // multi-GPU: seams run on their own stream while kernel A works on the
+    // interior chunks (which need no ghost plane)
+    cudaStream_t cs = nullptr;
+    cudaEvent_t ev_ready = nullptr, ev_seam = nullptr;
     long long launches = 0;
     // optional per-kernel timing of the solve (CUDA events on its stream)
     int prof = 0;
@@ -270,6 +274,9 @@ static void op_free(mas_op* op) {
         if (e) cudaEventDestroy(e);
     for (auto& e : op->pev) cudaEventDestroy(e);
     if (op->gexec) cudaGraphExecDestroy(op->gexec);
+    if (op->cs) cudaStreamDestroy(op->cs);
+    if (op->ev_ready) cudaEventDestroy(op->ev_ready);
+    if (op->ev_seam) cudaEventDestroy(op->ev_seam);
     if (op->cap_stream) cudaStreamDestroy(op->cap_stream);
     delete op;
 }
@@ -404,6 +411,14 @@ mas_status_t mas_op_setup(mas_grid_t* g, int ncomp, const double* kappa, const d
     TRY(dmalloc(&op->dot_out, 1));
     TRY(dmalloc(&op->bad, 1));
     TRY(ensure_hist(op, 64));
+    if (multi && (cudaStreamCreateWithFlags(&op->cs, cudaStreamNonBlocking) != cudaSuccess ||
+                  cudaEventCreateWithFlags(&op->ev_ready, cudaEventDisableTiming) != cudaSuccess ||
+                  cudaEventCreateWithFlags(&op->ev_seam, cudaEventDisableTiming) != cudaSuccess)) {
+        cudaGetLastError();
+        op_free(op);
+        set_last_error("comm stream setup failed");
+        return MAS_ERR_CUDA;
+    }
     // geometry with the boundary conditions folded into the radial tables:
     // a Neumann face gets weight 0; a Dirichlet face keeps its weight and the
     // kernels use kappa_ghost = kappa_P, u_ghost = 0 (R3).
@@ -442,6 +457,10 @@ mas_status_t mas_op_setup(mas_grid_t* g, int ncomp, const double* kappa, const d
     op->use_graph = !(g_env && atoi(g_env));
     const char* ch_env = getenv("MAS_CHUNK");  // experiment hook
     op->chunk = ch_env ? atoi(ch_env) : (nl >= 128 ? 32 : nl >= 64 ? 16 : (nl >= 16 ? 8 : 4));
+    if (!ch_env && multi && nl >= 12) {
+        // at least 3 chunks so that the interior ones can overlap the seams
+        op->chunk = nl / 4 < 4 ? 4 : (nl / 4 > 32 ? 32 : nl / 4);
+    }
     if (op->chunk < 1 || op->chunk > 64) op->chunk = 16;
     op->max_blocks = stencil_blocks(G, op->chunk);
     op->b_blocks = 148 * 8;
@@ -684,22 +703,43 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
     for (int k = 1; !graph && k <= maxit + 1; k++) {
         double* pold = op->p[(k + 1) & 1];
         double* pnew = op->p[k & 1];
-        if (comm) {
-            ST(comm_seams(comm, op->r, nc, op->g->nl, plane, op->rg, op->rg + nc * plane, s));
-            if (k > 1)
-                ST(comm_seams(comm, pold, nc, op->g->nl, plane, op->pg[(k + 1) & 1],
-                              op->pg[(k + 1) & 1] + nc * plane, s));
-        }
         a.pold = halo_of(op, pold, op->pg[(k + 1) & 1], nc);
         a.pnew = pnew;
         cudaEvent_t* pe = nullptr;
         if (op->prof) {
             ST(ensure_prof_events(op, k));
             pe = &op->pev[4 * (size_t)(k - 1)];
-            CU(cudaEventRecord(pe[0], s));
         }
-        CU(launch_stencil(MODE_PCGA, nc, a, s));
-        op->launches++;
+        if (comm) {
+            // seams of r and p_{k-1} on the comm stream, overlapped with kernel
+            // A on the interior chunks; the two edge chunks wait for them
+            CU(cudaEventRecord(op->ev_ready, s));
+            CU(cudaStreamWaitEvent(op->cs, op->ev_ready, 0));
+            ST(comm_seams(comm, op->r, nc, op->g->nl, plane, op->rg, op->rg + nc * plane, op->cs));
+            if (k > 1)
+                ST(comm_seams(comm, pold, nc, op->g->nl, plane, op->pg[(k + 1) & 1],
+                              op->pg[(k + 1) & 1] + nc * plane, op->cs));
+            CU(cudaEventRecord(op->ev_seam, op->cs));
+            if (pe) CU(cudaEventRecord(pe[0], s));
+            const int nchunk = (op->g->nl + op->chunk - 1) / op->chunk;
+            if (nchunk >= 3) {
+                a.part = 1;
+                CU(launch_stencil(MODE_PCGA, nc, a, s));
+                CU(cudaStreamWaitEvent(s, op->ev_seam, 0));
+                a.part = 2;
+                CU(launch_stencil(MODE_PCGA, nc, a, s));
+                a.part = 0;
+                op->launches += 2;
+            } else {
+                CU(cudaStreamWaitEvent(s, op->ev_seam, 0));
+                CU(launch_stencil(MODE_PCGA, nc, a, s));
+                op->launches++;
+            }
+        } else {
+            if (pe) CU(cudaEventRecord(pe[0], s));
+            CU(launch_stencil(MODE_PCGA, nc, a, s));
+            op->launches++;
+        }
         if (pe) CU(cudaEventRecord(pe[1], s));
         if (comm) ST(comm_allreduce(comm, &op->st->pend_sigma, 1, s));
         if (k <= maxit) {

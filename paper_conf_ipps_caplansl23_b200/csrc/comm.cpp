@@ -61,6 +61,7 @@ static std::map<unsigned long long, VGroup*> g_vmap;
 
 struct Comm {
     ncclComm_t nccl = nullptr;
+    ncclComm_t nccl_seam = nullptr;  // split communicator: seams run on their own stream
     int nranks = 1, rank = 0;
     VGroup* vg = nullptr;
     unsigned long long vkey = 0;
@@ -147,12 +148,21 @@ mas_status_t comm_create(const mas_dist_t* d, Comm** out) {
         delete c;
         return nccl_fail(r, "ncclCommInitRank");
     }
+    // NCCL operations of one communicator must not run concurrently on two
+    // streams: the seams (comm stream) get their own communicator
+    r = ncclCommSplit(c->nccl, 0, d->rank, &c->nccl_seam, nullptr);
+    if (r != ncclSuccess) {
+        ncclCommDestroy(c->nccl);
+        delete c;
+        return nccl_fail(r, "ncclCommSplit");
+    }
     *out = c;
     return MAS_OK;
 }
 
 void comm_destroy(Comm* c) {
     if (!c) return;
+    if (c->nccl_seam) ncclCommDestroy(c->nccl_seam);
     if (c->nccl) ncclCommDestroy(c->nccl);
     if (c->vg) {
         VGroup* g = c->vg;
@@ -254,12 +264,12 @@ mas_status_t comm_seams(Comm* c, const double* in, int ncomp, int nl, long long 
         const double* first = in + m * Nl;
         const double* last = in + m * Nl + (long long)(nl - 1) * plane;
         if (c->rank > 0) {
-            ncclSend(first, plane, ncclFloat64, c->rank - 1, c->nccl, s);
-            ncclRecv(glo + m * plane, plane, ncclFloat64, c->rank - 1, c->nccl, s);
+            ncclSend(first, plane, ncclFloat64, c->rank - 1, c->nccl_seam, s);
+            ncclRecv(glo + m * plane, plane, ncclFloat64, c->rank - 1, c->nccl_seam, s);
         }
         if (c->rank < c->nranks - 1) {
-            ncclSend(last, plane, ncclFloat64, c->rank + 1, c->nccl, s);
-            ncclRecv(ghi + m * plane, plane, ncclFloat64, c->rank + 1, c->nccl, s);
+            ncclSend(last, plane, ncclFloat64, c->rank + 1, c->nccl_seam, s);
+            ncclRecv(ghi + m * plane, plane, ncclFloat64, c->rank + 1, c->nccl_seam, s);
         }
     }
     r = ncclGroupEnd();

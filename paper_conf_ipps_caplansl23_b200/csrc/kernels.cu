@@ -425,7 +425,12 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
     const bool xupd = (MODE == MODE_PCGA) && kit >= 2;
 
     // ---- work item ------------------------------------------------------
-    const int item = blockIdx.x;
+    // work item; a split launch (multi-GPU seam overlap) covers either the
+    // interior chunks 1..nchunk-2 or the edge chunks 0 and nchunk-1
+    const int T = a.ntk * a.ntj;
+    const int item = a.part == 1 ? T + (int)blockIdx.x
+                     : a.part == 2 ? ((int)blockIdx.x < T ? (int)blockIdx.x : T * (a.nchunk - 2) + (int)blockIdx.x)
+                                   : (int)blockIdx.x;
     const int tk = item % a.ntk;
     const int tj = (item / a.ntk) % a.ntj;
     const int ch = item / (a.ntk * a.ntj);
@@ -460,7 +465,7 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
             }
         }
         double v1[1] = {0.0};
-        if (grid_reduce<1, kSThreads>(v1, a.scr, TKT_STENCIL) && threadIdx.x == 0) {
+        if (grid_reduce<1, kSThreads>(v1, a.scr, TKT_STENCIL) && threadIdx.x == 0 && a.part != 1) {
             PcgState* st = a.st;
             const double ff = st->pend_ff, rr = st->pend_rr;
             a.rr_hist[kit - 1] = rr;
@@ -635,9 +640,13 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
         double v[1] = {acc[0]};
         if (grid_reduce<1, kSThreads>(v, a.scr, TKT_STENCIL) && threadIdx.x == 0) {
             PcgState* st = a.st;
-            st->pend_sigma = v[0];
-            a.rr_hist[kit - 1] = st->pend_rr;
-            a.rho_hist[kit - 1] = st->pend_rho;
+            if (a.part == 1) {
+                st->sigma_part = v[0];  // completed by the edge launch
+            } else {
+                st->pend_sigma = a.part == 2 ? st->sigma_part + v[0] : v[0];
+                a.rr_hist[kit - 1] = st->pend_rr;
+                a.rho_hist[kit - 1] = st->pend_rho;
+            }
         }
     }
 }
@@ -812,7 +821,9 @@ static cudaError_t launch_one(const StencilArgs& a0, cudaStream_t s) {
         if (e != cudaSuccess) return e;
         attr_done = true;
     }
-    const int blocks = a.ntj * a.ntk * a.nchunk;
+    const int T = a.ntj * a.ntk;
+    const int blocks = a.part == 1 ? T * (a.nchunk - 2) : a.part == 2 ? 2 * T : T * a.nchunk;
+    if (blocks <= 0) return cudaErrorInvalidValue;
     k_stencil<MODE, NC><<<blocks, kSThreads, smem, s>>>(a);
     return cudaGetLastError();
 }

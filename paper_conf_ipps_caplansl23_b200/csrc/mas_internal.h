@@ -52,6 +52,7 @@ struct PcgState {
     double pend_rho;    // <r_k, z_k>_V           written by B(k), read by A(k+1)
     double pend_rr;     // <r_k, r_k>_V
     double pend_ff;     // <f, f>_V               written by init
+    double sigma_part;  // <p,q> of the interior launch of a split kernel A (multi-GPU overlap)
     double tol;
     double relres;
     int k;              // current iteration (A(k), B(k)); B's last block increments
@@ -88,6 +89,8 @@ struct StencilArgs {
     double* rr_hist;          // [maxit+2]
     Scratch scr;
     int* host_flag;           // mapped pinned int: iteration at which the solve stopped
+    int part;                 // 0: all work items; 1: interior chunks; 2: the two edge chunks
+                              // (interior runs while the seams are in flight)
     unsigned long long cond;  // CUDA graph while-loop handle (0: not in a graph)
 };
 

@@ -104,6 +104,23 @@ def test_virtual_ranks_apply_dot_and_pcg(mp, oracle_mod, P):
         assert math.sqrt((V * (xg - xo) ** 2).sum() / (V * xo ** 2).sum()) <= 1e-10
 
 
+@pytest.mark.parametrize("P", [2, 3])
+def test_virtual_ranks_seam_overlap_split_kernel(mp, oracle_mod, P):
+    """Slabs of >= 12 planes use >= 3 chunks: kernel A runs the interior
+    chunks while the seams are in flight, then the two edge chunks."""
+    prob = W.viscosity_problem(15 * P, 16, 64, warm=False)
+    x = W.random_field((3,) + prob.shape, 44)
+    out = run_ranks(mp, prob, P, x)
+    rc, xo, ito, _, _ = oracle_mod.solve_problem(prob)
+    its = {r["it"] for r in out}
+    assert len(its) == 1 and abs(its.pop() - ito) <= 1
+    V = oracle_mod.Oracle.for_problem(prob).volumes()[None]
+    xg = np.concatenate([r["x"] for r in out], axis=1)
+    assert math.sqrt((V * (xg - xo) ** 2).sum() / (V * xo ** 2).sum()) <= 1e-10
+    # the split kernel A shows up as one extra launch per iteration
+    assert all(r["launches"] >= 3 * r["it"] for r in out)
+
+
 def test_virtual_ranks_conduction_dirichlet_and_fixed_iterations(mp, oracle_mod):
     prob = W.conduction_problem(10, 24, 32)
     x = W.random_field((1,) + prob.shape, 43)
