@@ -409,18 +409,22 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
     double beta = 0.0, alpha_prev = 0.0;
     int kit = 0;
     if (MODE == MODE_PCGA) {
-        const volatile PcgState* st = a.st;
-        if (st->stopped) return;
-        kit = st->k;
-        const double ff = st->pend_ff, rr = st->pend_rr;
+        // one round trip: everything A(k) needs sits in PcgState (written by
+        // earlier kernels; read through L2)
+        const PcgState* st = a.st;
+        if (__ldcg(&st->stopped)) return;
+        kit = __ldcg(&st->k);
+        const double ff = __ldcg(&st->pend_ff), rr = __ldcg(&st->pend_rr);
+        const double rho1 = __ldcg(&st->pend_rho), rho2 = __ldcg(&st->rho_prev);
+        const double sig1 = __ldcg(&st->sigma_prev);
         first = (kit == 1);
-        if (kit >= 2) alpha_prev = a.rho_hist[kit - 2] / a.sigma_hist[kit - 1];
+        if (kit >= 2) alpha_prev = rho2 / sig1;
         if (first && ff == 0.0)
             pmode = P_ZERO;
-        else if (sqrt(rr) <= st->tol * sqrt(ff) || kit > st->maxit)
+        else if (sqrt(rr) <= __ldcg(&st->tol) * sqrt(ff) || kit > __ldcg(&st->maxit))
             pmode = P_FINAL;
         else if (!first)
-            beta = st->pend_rho / a.rho_hist[kit - 2];
+            beta = rho1 / rho2;
     }
     const bool xupd = (MODE == MODE_PCGA) && kit >= 2;
 
@@ -646,6 +650,7 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
                 st->pend_sigma = a.part == 2 ? st->sigma_part + v[0] : v[0];
                 a.rr_hist[kit - 1] = st->pend_rr;
                 a.rho_hist[kit - 1] = st->pend_rho;
+                st->rho_prev = st->pend_rho;  // rho_{k-1}, read as rho_{(k+1)-2} by A(k+1)
             }
         }
     }
@@ -655,13 +660,13 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
 // --------------------------------------------------------------------------
 template <int NC>
 __global__ void __launch_bounds__(kThreads) k_pcg_b(const StreamArgs a) {
-    const volatile PcgState* vst = a.st;
-    if (vst->stopped) return;
+    const PcgState* vst = a.st;
+    if (__ldcg(&vst->stopped)) return;
     const Geo& g = a.g;
-    const int kit = vst->k;
-    const double sigma = vst->pend_sigma;
+    const int kit = __ldcg(&vst->k);
+    const double sigma = __ldcg(&vst->pend_sigma);
     const bool brk = !(sigma > 0.0) || !isfinite(sigma);
-    const double alpha = a.rho_hist[kit - 1] / sigma;
+    const double alpha = __ldcg(&vst->pend_rho) / sigma;  // rho_{k-1} / sigma_k
     double acc[2] = {0.0, 0.0};
     if (!brk) {
         const long long Nl = (long long)g.nl * g.plane;
@@ -716,6 +721,7 @@ reduce:
             if (a.cond) cudaGraphSetConditional((cudaGraphConditionalHandle)a.cond, 0);
         } else {
             a.sigma_hist[kit] = sigma;
+            st->sigma_prev = sigma;
             st->pend_rho = acc[0];
             st->pend_rr = acc[1];
             st->k = kit + 1;

@@ -53,6 +53,8 @@ struct PcgState {
     double pend_rr;     // <r_k, r_k>_V
     double pend_ff;     // <f, f>_V               written by init
     double sigma_part;  // <p,q> of the interior launch of a split kernel A (multi-GPU overlap)
+    double rho_prev;    // rho of the previous A: at A(k) it is rho_{k-2} (A's last block updates)
+    double sigma_prev;  // sigma_{k-1}, saved by B(k-1)'s last block
     double tol;
     double relres;
     int k;              // current iteration (A(k), B(k)); B's last block increments
