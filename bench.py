@@ -43,6 +43,9 @@ CONFIGS = {
     "C3": ("viscosity", 256, 256, 512),
     # C4: weak scaling, (256 * N) x 256 x 512 on N GPUs (nr scaled below)
     "C4": ("viscosity", 256, 256, 512),
+    # one rank's share of C3 at P = 8 (32 r-planes), to study the per-GPU
+    # kernel efficiency that bounds 8-GPU strong scaling
+    "C3s8": ("viscosity", 32, 256, 512),
     "C2": ("conduction", 128, 128, 256),
     "C1": ("mms", 16, 24, 32),
 }

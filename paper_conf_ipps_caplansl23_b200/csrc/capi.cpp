@@ -391,6 +391,10 @@ mas_status_t mas_op_setup(mas_grid_t* g, int ncomp, const double* kappa, const d
     const int nl = g->nl, nt = g->nt, np = g->np;
     const long long plane = (long long)nt * np;
     op->Nl = (long long)nl * plane;
+    if ((long long)ncomp * op->Nl >= (1LL << 31)) {  // the stencil kernels index with 32-bit offsets
+        delete op;
+        return arg_error("local slab too large: ncomp * cells must be < 2^31 per rank");
+    }
     const bool multi = g->comm != nullptr;
     mas_status_t s;
 #define TRY(x)                         \

@@ -35,7 +35,7 @@ constexpr int kThreads = 256;  // 8 warps (stream kernels)
 #define MAS_MINB 2
 #endif
 #ifndef MAS_MINB1
-#define MAS_MINB1 3
+#define MAS_MINB1 2
 #endif
 constexpr int TJ = MAS_TJ;     // theta rows per stencil tile (one warp per row)
 constexpr int kSThreads = 32 * TJ;
@@ -110,10 +110,14 @@ __device__ bool grid_reduce(double (&v)[NS], const Scratch& scr, int tkt) {
 // --------------------------------------------------------------------------
 // field access
 // --------------------------------------------------------------------------
+// The stencil kernels index with 32-bit offsets (the host rejects slabs with
+// ncomp * cells >= 2^31): fewer integer instructions on the address path.
+__device__ __forceinline__ int plane32(const Geo& g) { return (int)g.plane; }
+// --------------------------------------------------------------------------
 __device__ __forceinline__ const double* plane_ptr(const Halo& h, int comp, int i, const Geo& g) {
-    if (i < 0) return h.glo + (long long)comp * g.plane;
-    if (i >= g.nl) return h.ghi + (long long)comp * g.plane;
-    return h.in + ((long long)comp * g.nl + i) * g.plane;
+    if (i < 0) return h.glo + (int)comp * plane32(g);
+    if (i >= g.nl) return h.ghi + (int)comp * plane32(g);
+    return h.in + ((int)comp * g.nl + i) * plane32(g);
 }
 __device__ __forceinline__ double2 ld2(const double* p) {
     return __ldg(reinterpret_cast<const double2*>(p));
@@ -168,7 +172,7 @@ __device__ __forceinline__ PlanePtrs<NC> plane_ptrs(const StencilArgs& a, int i,
 }
 
 template <int MODE, int NC, bool SCALAR>
-__device__ __forceinline__ void load_raw(const PlanePtrs<NC>& P, long long off, bool first, Raw<NC>& R) {
+__device__ __forceinline__ void load_raw(const PlanePtrs<NC>& P, int off, bool first, Raw<NC>& R) {
     R.kap = ldv<SCALAR>(P.kap + off);
 #pragma unroll
     for (int c = 0; c < NC; c++) R.u[c] = ldv<SCALAR>(P.u[c] + off);
@@ -204,7 +208,7 @@ __device__ __forceinline__ double* sfield(double* buf, int f) { return buf + f *
 // 0..2TK-1 cover the theta halo rows j0-1 and j0+height, threads
 // 2TK..2TK+2TJ-1 the periodic phi halo columns.
 struct HaloMeta {
-    long long hoff;  // offset in the plane
+    int hoff;  // offset in the plane
     int hidx;        // index in a ring field
     int hkind;       // 0 none, 1 load, 3 zeros (beyond a pole / theta wall)
 };
@@ -220,7 +224,7 @@ __device__ __forceinline__ HaloMeta halo_meta(const Geo& g, int j0, int k0, int 
         if (kk < width) {
             m.hidx = hr * ROW + OFF + kk;
             m.hkind = (j >= 0 && j < g.nt) ? 1 : 3;
-            m.hoff = (long long)j * g.np + k0 + kk;
+            m.hoff = (int)j * g.np + k0 + kk;
         }
     } else if (t < 2 * TK + 2 * TJ) {
         const int q = t - 2 * TK, side = q / TJ, r = q % TJ;
@@ -228,7 +232,7 @@ __device__ __forceinline__ HaloMeta halo_meta(const Geo& g, int j0, int k0, int 
             const int k = side == 0 ? (k0 - 1 + g.np) % g.np : (k0 + width) % g.np;
             m.hidx = (1 + r) * ROW + (side == 0 ? OFF - 1 : OFF + width);
             m.hkind = 1;
-            m.hoff = (long long)(j0 + r) * g.np + k;
+            m.hoff = (int)(j0 + r) * g.np + k;
         }
     }
     return m;
@@ -270,12 +274,12 @@ __device__ __forceinline__ void stage_issue(const StencilArgs& a, int i, int j0,
     const Geo& g = a.g;
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     const int kc = 2 * lane;
-    const long long Nl = (long long)g.nl * g.plane;
+    const int Nl = (int)g.nl * plane32(g);
     const PlanePtrs<NC> P = plane_ptrs<MODE, NC>(a, i, first);
     double* hst = halo_stage<NC>();
     if (w < height && kc < width) {
-        const long long off = (long long)(j0 + w) * g.np + k0 + kc;
-        const long long o3 = (long long)i * g.plane + off;
+        const int off = (int)(j0 + w) * g.np + k0 + kc;
+        const int o3 = (int)i * plane32(g) + off;
         load_raw<MODE, NC, false>(P, off, first, S.R);
         if (own_work) {
             if (a.c) S.o.c = ld2(a.c + o3);
@@ -315,7 +319,7 @@ __device__ __forceinline__ void stage_commit(const StencilArgs& a, int i, int j0
     const Geo& g = a.g;
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     const int kc = 2 * lane;
-    const long long Nl = (long long)g.nl * g.plane;
+    const int Nl = (int)g.nl * plane32(g);
     if (w < height && kc < width) {
         finish_raw<MODE, NC>(S.R, first, beta);
         const int idx = (1 + w) * ROW + OFF + kc;
@@ -326,7 +330,7 @@ __device__ __forceinline__ void stage_commit(const StencilArgs& a, int i, int j0
         if (own_work) {
             o = S.o;
             if (MODE == MODE_PCGA) {
-                const long long o3 = (long long)i * g.plane + (long long)(j0 + w) * g.np + k0 + kc;
+                const int o3 = (int)i * plane32(g) + (int)(j0 + w) * g.np + k0 + kc;
 #pragma unroll
                 for (int c = 0; c < NC; c++) {
                     stg2(a.pnew + c * Nl + o3, S.R.u[c]);
@@ -444,8 +448,8 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
     const int kc = 2 * lane;
     const bool own = (w < height) && (kc < width);
     const int j = j0 + w, k = k0 + kc;
-    const long long off = (long long)j * g.np + k;
-    const long long Nl = (long long)g.nl * g.plane;
+    const int off = (int)j * g.np + k;
+    const int Nl = (int)g.nl * plane32(g);
 
     double acc[3] = {0.0, 0.0, 0.0};
 
@@ -455,7 +459,7 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
             for (int i = ia; i < ib; i++) {
 #pragma unroll
                 for (int c = 0; c < NC; c++) {
-                    double* xp = a.x + c * Nl + (long long)i * g.plane + off;
+                    double* xp = a.x + c * Nl + (int)i * plane32(g) + off;
                     if (pmode == P_ZERO) {
                         stg2(xp, make_double2(0.0, 0.0));
                     } else if (kit >= 2) {
@@ -593,7 +597,7 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
             const double aPp1 = ic * wpp[1] * (0.5 * (kP.y + kR));
             const double V0 = vri * vtj * vpk[0], V1 = vri * vtj * vpk[1];
             const double2 cP = a.c ? oc.c : make_double2(0.0, 0.0);
-            const long long pofs = (long long)i * g.plane + off;
+            const int pofs = (int)i * plane32(g) + off;
 #pragma unroll
             for (int c = 0; c < NC; c++) {
                 const double* s0 = sfield(const_cast<double*>(S0), c);
@@ -616,7 +620,7 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
                 L1 = fma(aPm1, u.y - u.x, L1);
                 L0 = fma(aPp0, u.x - u.y, L0);
                 L1 = fma(aPp1, u.y - uR, L1);
-                const long long o = c * Nl + pofs;
+                const int o = c * Nl + pofs;
                 if (MODE == MODE_RESID) {
                     const double r0 = oc.f[c].x - L0, r1 = oc.f[c].y - L1;
                     stg2(a.out + o, make_double2(r0, r1));
