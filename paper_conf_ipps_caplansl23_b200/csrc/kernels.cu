@@ -3,10 +3,10 @@
 // The path is HBM-bound ("highly memory-bound"; DESIGN.md
 // §5 roofline), so there are no tensor-core contractions here: every kernel
 // streams fp64 fields with 16-byte (double2) coalesced accesses along phi,
-// stages (theta,phi) plane tiles with a one-cell halo in shared memory and
-// marches along r with the r-neighbours in registers.  Kernel fusion follows
-// the paper's own lesson that OpenACC's fused, asynchronous kernels beat the
-// un-fused DC loops:
+// stages (theta,phi) plane tiles with a one-cell halo in a shared-memory
+// ring and marches along r (the r-neighbours are the adjacent ring slots).
+// Kernel fusion follows the paper's own lesson that OpenACC's fused,
+// asynchronous kernels beat the un-fused DC loops:
 //
 //   k_stencil<MODE_PCGA>  "kernel A":  beta, p = D^-1 r + beta p_old (also on
 //       the halo), deferred x += alpha_{k-1} p_old, q = L p, partial <p,q>_V
@@ -362,18 +362,6 @@ __device__ __forceinline__ void stage_commit(const StencilArgs& a, int i, int j0
 #pragma unroll
         for (int c = 0; c <= NC; c++) sfield(buf, c)[hm.hidx] = 0.0;
     }
-}
-
-// Produce plane i into ring slot `buf` right away (issue + commit).
-template <int MODE, int NC>
-__device__ __forceinline__ void produce_tile(const StencilArgs& a, int i, double* buf, int j0, int k0,
-                                             int height, int width, const HaloMeta& hm, bool first,
-                                             double beta, double alpha_prev, bool xupd, bool halo,
-                                             bool own_work, double2& kown, OwnRegs<NC>& o) {
-    Stage<NC> S;
-    stage_issue<MODE, NC>(a, i, j0, k0, height, width, hm, first, xupd, halo, own_work, S);
-    stage_commit<MODE, NC>(a, i, j0, k0, height, width, hm, first, beta, alpha_prev, xupd, halo,
-                           own_work, S, buf, kown, o);
 }
 
 // Own-cell region of a ring slot as the global-boundary ghost plane:
