@@ -548,9 +548,16 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
                                    kown, on);
         else
             ghost_plane<NC>(slot(i + 1), height, width, kown);
+        // issue plane i+2 (registers and private cp.async slots only): its
+        // latency overlaps the stencil of plane i.  Issuing it before the
+        // barrier measured faster for the scalar kernel and slower for the
+        // 3-component one (tools/abtest.sh), hence the split.
+        constexpr bool kIssueEarly = (NC == 1);
+        if (kIssueEarly && i + 2 <= ib && real_plane(i + 2))
+            stage_issue<MODE, NC>(a, i + 2, j0, k0, height, width, hm, first, xupd && (i + 2 < ib),
+                                  i + 2 < ib, i + 2 < ib, S);
         __syncthreads();
-        // issue plane i+2: its latency overlaps the stencil of plane i
-        if (i + 2 <= ib && real_plane(i + 2))
+        if (!kIssueEarly && i + 2 <= ib && real_plane(i + 2))
             stage_issue<MODE, NC>(a, i + 2, j0, k0, height, width, hm, first, xupd && (i + 2 < ib),
                                   i + 2 < ib, i + 2 < ib, S);
 
