@@ -260,23 +260,16 @@ __device__ __forceinline__ void cpa8(double* sdst, const double* gsrc) {
 __device__ __forceinline__ void cpa_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
 __device__ __forceinline__ void cpa_wait_all() { asm volatile("cp.async.wait_group 0;\n" ::: "memory"); }
 
-// dynamic shared memory: [4-slot ring][halo staging]
-template <int NC>
-__device__ __forceinline__ double* halo_stage() {
-    extern __shared__ __align__(16) double dyn_smem[];
-    return dyn_smem + 4 * (NC + 1) * HROWS * ROW;
-}
 
 template <int MODE, int NC>
 __device__ __forceinline__ void stage_issue(const StencilArgs& a, int i, int j0, int k0, int height,
                                             int width, const HaloMeta& hm, bool first, bool xupd,
-                                            bool halo, bool own_work, Stage<NC>& S) {
+                                            bool halo, bool own_work, Stage<NC>& S, double* hst) {
     const Geo& g = a.g;
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     const int kc = 2 * lane;
     const int Nl = (int)g.nl * plane32(g);
     const PlanePtrs<NC> P = plane_ptrs<MODE, NC>(a, i, first);
-    double* hst = halo_stage<NC>();
     if (w < height && kc < width) {
         const int off = (int)(j0 + w) * g.np + k0 + kc;
         const int o3 = (int)i * plane32(g) + off;
@@ -315,7 +308,7 @@ __device__ __forceinline__ void stage_commit(const StencilArgs& a, int i, int j0
                                              int width, const HaloMeta& hm, bool first, double beta,
                                              double alpha_prev, bool xupd, bool halo, bool own_work,
                                              Stage<NC>& S, double* buf, double2& kown,
-                                             OwnRegs<NC>& o) {
+                                             OwnRegs<NC>& o, const double* hst) {
     const Geo& g = a.g;
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     const int kc = 2 * lane;
@@ -345,7 +338,6 @@ __device__ __forceinline__ void stage_commit(const StencilArgs& a, int i, int j0
         }
     }
     if (halo && hm.hkind == 1) {
-        double* hst = halo_stage<NC>();
         cpa_wait_all();  // this thread's own copies; read back below by the same thread
         const double* h = hst + threadIdx.x;
 #pragma unroll
@@ -492,6 +484,9 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
     // are in flight; plane i+2 is committed into the slot of plane i-2, so
     // one barrier per plane suffices.
     auto slot = [&](int i) { return smem + ((i - ia + 1) & 3) * BUF; };
+    // private cp.async slots of the halo items: static shared memory, so the
+    // shared-window address needs no runtime conversion
+    __shared__ __align__(16) double hst_arr[(2 + 2 * NC) * kHaloSlots];
     auto real_plane = [&](int p) { return !(p == g.nl && g.glob_hi); };
 
     // 1-D geometry of this work item staged in shared memory once (visible to
@@ -528,24 +523,24 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
     // planes ia-1 (own cells only) and ia: both loads in flight together
     Stage<NC> S0, S;
     if (!lo_ghost)
-        stage_issue<MODE, NC>(a, ia - 1, j0, k0, height, width, hm, first, false, false, false, S0);
-    stage_issue<MODE, NC>(a, ia, j0, k0, height, width, hm, first, xupd, true, true, S);
+        stage_issue<MODE, NC>(a, ia - 1, j0, k0, height, width, hm, first, false, false, false, S0, hst_arr);
+    stage_issue<MODE, NC>(a, ia, j0, k0, height, width, hm, first, xupd, true, true, S, hst_arr);
     if (!lo_ghost)
         stage_commit<MODE, NC>(a, ia - 1, j0, k0, height, width, hm, first, beta, alpha_prev, false,
-                               false, false, S0, slot(ia - 1), kdummy, on);
+                               false, false, S0, slot(ia - 1), kdummy, on, hst_arr);
     stage_commit<MODE, NC>(a, ia, j0, k0, height, width, hm, first, beta, alpha_prev, xupd, true, true,
-                           S, slot(ia), kown, oc);
+                           S, slot(ia), kown, oc, hst_arr);
     if (lo_ghost) ghost_plane<NC>(slot(ia - 1), height, width, kown);
     if (real_plane(ia + 1))
         stage_issue<MODE, NC>(a, ia + 1, j0, k0, height, width, hm, first, xupd && (ia + 1 < ib),
-                              ia + 1 < ib, ia + 1 < ib, S);
+                              ia + 1 < ib, ia + 1 < ib, S, hst_arr);
 
     for (int i = ia; i < ib; i++) {
         // commit plane i+1 (its loads were issued one plane earlier)
         if (real_plane(i + 1))
             stage_commit<MODE, NC>(a, i + 1, j0, k0, height, width, hm, first, beta, alpha_prev,
                                    xupd && (i + 1 < ib), i + 1 < ib, i + 1 < ib, S, slot(i + 1),
-                                   kown, on);
+                                   kown, on, hst_arr);
         else
             ghost_plane<NC>(slot(i + 1), height, width, kown);
         // issue plane i+2 (registers and private cp.async slots only): its
@@ -555,11 +550,11 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
         constexpr bool kIssueEarly = (NC == 1);
         if (kIssueEarly && i + 2 <= ib && real_plane(i + 2))
             stage_issue<MODE, NC>(a, i + 2, j0, k0, height, width, hm, first, xupd && (i + 2 < ib),
-                                  i + 2 < ib, i + 2 < ib, S);
+                                  i + 2 < ib, i + 2 < ib, S, hst_arr);
         __syncthreads();
         if (!kIssueEarly && i + 2 <= ib && real_plane(i + 2))
             stage_issue<MODE, NC>(a, i + 2, j0, k0, height, width, hm, first, xupd && (i + 2 < ib),
-                                  i + 2 < ib, i + 2 < ib, S);
+                                  i + 2 < ib, i + 2 < ib, S, hst_arr);
 
         if (own) {
             const double* S0 = slot(i);
@@ -818,7 +813,7 @@ static cudaError_t launch_one(const StencilArgs& a0, cudaStream_t s) {
     a.ntj = (a.g.nt + TJ - 1) / TJ;
     a.ntk = (a.g.np + TK - 1) / TK;
     a.nchunk = (a.g.nl + a.chunk - 1) / a.chunk;
-    const int smem = (4 * (NC + 1) * HROWS * ROW + (2 + 2 * NC) * kHaloSlots) * (int)sizeof(double);
+    const int smem = 4 * (NC + 1) * HROWS * ROW * (int)sizeof(double);
     static bool attr_done = false;
     if (!attr_done) {
         cudaError_t e = cudaFuncSetAttribute(k_stencil<MODE, NC>,
