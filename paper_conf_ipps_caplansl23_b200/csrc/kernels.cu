@@ -185,6 +185,23 @@ __device__ __forceinline__ void load_raw(const PlanePtrs<NC>& P, int off, bool f
     }
 }
 
+// Interior planes (no ghost buffer involved): every field is addressed as
+// base + comp * Nl + idx with one 32-bit idx = i * plane + offset, so the
+// per-load address is a single wide multiply-add on a uniform base.
+template <int MODE, int NC, bool SCALAR>
+__device__ __forceinline__ void load_raw_in(const StencilArgs& a, int Nl, int idx, bool first, Raw<NC>& R) {
+    R.kap = ldv<SCALAR>(a.kappa.in + idx);
+#pragma unroll
+    for (int c = 0; c < NC; c++) R.u[c] = ldv<SCALAR>(a.u.in + c * Nl + idx);
+    if (MODE == MODE_PCGA) {
+        R.di = ldv<SCALAR>(a.dinv.in + idx);
+        if (!first) {
+#pragma unroll
+            for (int c = 0; c < NC; c++) R.po[c] = ldv<SCALAR>(a.pold.in + c * Nl + idx);
+        }
+    }
+}
+
 // u entering the stencil: APPLY/RESID x;  PCGA p_k = D^-1 r + beta p_{k-1}
 template <int MODE, int NC>
 __device__ __forceinline__ void finish_raw(Raw<NC>& R, bool first, double beta) {
@@ -269,11 +286,17 @@ __device__ __forceinline__ void stage_issue(const StencilArgs& a, int i, int j0,
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     const int kc = 2 * lane;
     const int Nl = (int)g.nl * plane32(g);
-    const PlanePtrs<NC> P = plane_ptrs<MODE, NC>(a, i, first);
+    const bool interior = (i >= 0) && (i < g.nl);  // uniform: no ghost buffer involved
+    const int pl = plane32(g), ipl = i * pl;
     if (w < height && kc < width) {
         const int off = (int)(j0 + w) * g.np + k0 + kc;
-        const int o3 = (int)i * plane32(g) + off;
-        load_raw<MODE, NC, false>(P, off, first, S.R);
+        const int o3 = ipl + off;
+        if (interior) {
+            load_raw_in<MODE, NC, false>(a, Nl, o3, first, S.R);
+        } else {
+            const PlanePtrs<NC> P = plane_ptrs<MODE, NC>(a, i, first);
+            load_raw<MODE, NC, false>(P, off, first, S.R);
+        }
         if (own_work) {
             if (a.c) S.o.c = ld2(a.c + o3);
             if (MODE == MODE_PCGA && xupd) {
@@ -289,14 +312,18 @@ __device__ __forceinline__ void stage_issue(const StencilArgs& a, int i, int j0,
     }
     if (halo && hm.hkind == 1) {
         double* h = hst + threadIdx.x;
-        cpa8(h, P.kap + hm.hoff);
+        if (interior) {  // halo planes are stencil planes: always interior here
+            const int hi = ipl + (int)hm.hoff;
+            cpa8(h, a.kappa.in + hi);
 #pragma unroll
-        for (int c = 0; c < NC; c++) cpa8(h + (2 + c) * kHaloSlots, P.u[c] + hm.hoff);
-        if (MODE == MODE_PCGA) {
-            cpa8(h + kHaloSlots, P.di + hm.hoff);
-            if (!first) {
+            for (int c = 0; c < NC; c++) cpa8(h + (2 + c) * kHaloSlots, a.u.in + c * Nl + hi);
+            if (MODE == MODE_PCGA) {
+                cpa8(h + kHaloSlots, a.dinv.in + hi);
+                if (!first) {
 #pragma unroll
-                for (int c = 0; c < NC; c++) cpa8(h + (2 + NC + c) * kHaloSlots, P.po[c] + hm.hoff);
+                    for (int c = 0; c < NC; c++)
+                        cpa8(h + (2 + NC + c) * kHaloSlots, a.pold.in + c * Nl + hi);
+                }
             }
         }
     }
