@@ -338,7 +338,9 @@ static mas_status_t loop_graph(mas_op* op, StencilArgs a, StreamArgs b) {
             a.cond = (unsigned long long)h;
             b.cond = (unsigned long long)h;
             const int nc = op->ncomp;
-            for (int kk = 1; kk <= 2 && e == cudaSuccess; kk++) {
+            // iteration 1 runs before the loop (its own kernel-A instantiation);
+            // the body covers an even and an odd iteration: k = 2, 3, 4, ...
+            for (int kk = 2; kk <= 3 && e == cudaSuccess; kk++) {
                 a.pold = halo_of(op, op->p[(kk + 1) & 1], nullptr, nc);
                 a.pnew = op->p[kk & 1];
                 e = launch_stencil(MODE_PCGA, nc, a, op->cap_stream);
@@ -713,6 +715,10 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
     const bool graph = !comm && !op->prof && op->use_graph;
     if (graph) {
         ST(loop_graph(op, a, b));
+        a.pold = halo_of(op, op->p[0], nullptr, nc);  // iteration 1
+        a.pnew = op->p[1];
+        CU(launch_stencil(MODE_PCGA, nc, a, s, true));
+        CU(launch_pcg_b(b, op->b_blocks, s));
         CU(cudaGraphLaunch(op->gexec, s));
     }
     int stop_seen_at = -1;
@@ -741,20 +747,20 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
             const int nchunk = (op->g->nl + op->chunk - 1) / op->chunk;
             if (nchunk >= 3) {
                 a.part = 1;
-                CU(launch_stencil(MODE_PCGA, nc, a, s));
+                CU(launch_stencil(MODE_PCGA, nc, a, s, k == 1));
                 CU(cudaStreamWaitEvent(s, op->ev_seam, 0));
                 a.part = 2;
-                CU(launch_stencil(MODE_PCGA, nc, a, s));
+                CU(launch_stencil(MODE_PCGA, nc, a, s, k == 1));
                 a.part = 0;
                 op->launches += 2;
             } else {
                 CU(cudaStreamWaitEvent(s, op->ev_seam, 0));
-                CU(launch_stencil(MODE_PCGA, nc, a, s));
+                CU(launch_stencil(MODE_PCGA, nc, a, s, k == 1));
                 op->launches++;
             }
         } else {
             if (pe) CU(cudaEventRecord(pe[0], s));
-            CU(launch_stencil(MODE_PCGA, nc, a, s));
+            CU(launch_stencil(MODE_PCGA, nc, a, s, k == 1));
             op->launches++;
         }
         if (pe) CU(cudaEventRecord(pe[1], s));
@@ -789,9 +795,10 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
     }
     *iters = fin.iters;
     *relres = fin.relres;
-    if (graph) {  // init + 4 kernels per executed loop body (two iterations)
+    if (graph) {  // iteration 1 + 4 kernels per executed loop body (iterations 2k, 2k+1)
         const int last_a = fin.status == MAS_ERR_BREAKDOWN ? fin.iters : fin.iters + 1;
-        op->launches += 4LL * ((last_a + 1) / 2);
+        const int bodies = last_a <= 2 ? 1 : last_a / 2;
+        op->launches += 2 + 4LL * bodies;
     }
     if (res_hist) {
         // after a breakdown at iteration k only ||r_0..r_{k-1}|| exist

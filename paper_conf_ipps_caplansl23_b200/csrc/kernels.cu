@@ -407,7 +407,10 @@ __device__ __forceinline__ void ghost_plane(double* buf, int height, int width, 
 //   produce(i+1): global loads of r, p_old, D^-1, kappa (+x, c for own cells)
 //                 -> p_{i+1} into the ring (and x-update / p store)
 //   sync; stencil(i) from the ring only (r-neighbours = adjacent slots); sync
-template <int MODE, int NC>
+// FIRSTK: kernel A of iteration 1 (p = D^-1 r, no x update) is its own
+// instantiation, so the per-plane code of every other iteration carries no
+// first-iteration branches.
+template <int MODE, int NC, bool FIRSTK = false>
 __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_stencil(const StencilArgs a) {
     extern __shared__ __align__(16) double smem[];
     constexpr int BUF = (NC + 1) * HROWS * ROW;
@@ -423,7 +426,13 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
         // one round trip: everything A(k) needs sits in PcgState (written by
         // earlier kernels; read through L2)
         const PcgState* st = a.st;
-        if (__ldcg(&st->stopped)) return;
+        if (__ldcg(&st->stopped)) {
+            // already decided (possibly before the graph's while loop started):
+            // end the loop
+            if (a.cond && blockIdx.x == 0 && threadIdx.x == 0)
+                cudaGraphSetConditional((cudaGraphConditionalHandle)a.cond, 0);
+            return;
+        }
         kit = __ldcg(&st->k);
         const double ff = __ldcg(&st->pend_ff), rr = __ldcg(&st->pend_rr);
         const double rho1 = __ldcg(&st->pend_rho), rho2 = __ldcg(&st->rho_prev);
@@ -437,7 +446,8 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
         else if (!first)
             beta = rho1 / rho2;
     }
-    const bool xupd = (MODE == MODE_PCGA) && kit >= 2;
+    const bool xupd = (MODE == MODE_PCGA) && !FIRSTK;
+    if (MODE == MODE_PCGA && pmode == P_NORMAL && FIRSTK != first) __trap();  // host dispatch bug
 
     // ---- work item ------------------------------------------------------
     // work item; a split launch (multi-GPU seam overlap) covers either the
@@ -550,22 +560,22 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
     // planes ia-1 (own cells only) and ia: both loads in flight together
     Stage<NC> S0, S;
     if (!lo_ghost)
-        stage_issue<MODE, NC>(a, ia - 1, j0, k0, height, width, hm, first, false, false, false, S0, hst_arr);
-    stage_issue<MODE, NC>(a, ia, j0, k0, height, width, hm, first, xupd, true, true, S, hst_arr);
+        stage_issue<MODE, NC>(a, ia - 1, j0, k0, height, width, hm, FIRSTK, false, false, false, S0, hst_arr);
+    stage_issue<MODE, NC>(a, ia, j0, k0, height, width, hm, FIRSTK, xupd, true, true, S, hst_arr);
     if (!lo_ghost)
-        stage_commit<MODE, NC>(a, ia - 1, j0, k0, height, width, hm, first, beta, alpha_prev, false,
+        stage_commit<MODE, NC>(a, ia - 1, j0, k0, height, width, hm, FIRSTK, beta, alpha_prev, false,
                                false, false, S0, slot(ia - 1), kdummy, on, hst_arr);
-    stage_commit<MODE, NC>(a, ia, j0, k0, height, width, hm, first, beta, alpha_prev, xupd, true, true,
+    stage_commit<MODE, NC>(a, ia, j0, k0, height, width, hm, FIRSTK, beta, alpha_prev, xupd, true, true,
                            S, slot(ia), kown, oc, hst_arr);
     if (lo_ghost) ghost_plane<NC>(slot(ia - 1), height, width, kown);
     if (real_plane(ia + 1))
-        stage_issue<MODE, NC>(a, ia + 1, j0, k0, height, width, hm, first, xupd && (ia + 1 < ib),
+        stage_issue<MODE, NC>(a, ia + 1, j0, k0, height, width, hm, FIRSTK, xupd && (ia + 1 < ib),
                               ia + 1 < ib, ia + 1 < ib, S, hst_arr);
 
     for (int i = ia; i < ib; i++) {
         // commit plane i+1 (its loads were issued one plane earlier)
         if (real_plane(i + 1))
-            stage_commit<MODE, NC>(a, i + 1, j0, k0, height, width, hm, first, beta, alpha_prev,
+            stage_commit<MODE, NC>(a, i + 1, j0, k0, height, width, hm, FIRSTK, beta, alpha_prev,
                                    xupd && (i + 1 < ib), i + 1 < ib, i + 1 < ib, S, slot(i + 1),
                                    kown, on, hst_arr);
         else
@@ -576,11 +586,11 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
         // 3-component one (tools/abtest.sh), hence the split.
         constexpr bool kIssueEarly = (NC == 1);
         if (kIssueEarly && i + 2 <= ib && real_plane(i + 2))
-            stage_issue<MODE, NC>(a, i + 2, j0, k0, height, width, hm, first, xupd && (i + 2 < ib),
+            stage_issue<MODE, NC>(a, i + 2, j0, k0, height, width, hm, FIRSTK, xupd && (i + 2 < ib),
                                   i + 2 < ib, i + 2 < ib, S, hst_arr);
         __syncthreads();
         if (!kIssueEarly && i + 2 <= ib && real_plane(i + 2))
-            stage_issue<MODE, NC>(a, i + 2, j0, k0, height, width, hm, first, xupd && (i + 2 < ib),
+            stage_issue<MODE, NC>(a, i + 2, j0, k0, height, width, hm, FIRSTK, xupd && (i + 2 < ib),
                                   i + 2 < ib, i + 2 < ib, S, hst_arr);
 
         if (own) {
@@ -682,7 +692,11 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
 template <int NC>
 __global__ void __launch_bounds__(kThreads) k_pcg_b(const StreamArgs a) {
     const PcgState* vst = a.st;
-    if (__ldcg(&vst->stopped)) return;
+    if (__ldcg(&vst->stopped)) {
+        if (a.cond && blockIdx.x == 0 && threadIdx.x == 0)
+            cudaGraphSetConditional((cudaGraphConditionalHandle)a.cond, 0);
+        return;
+    }
     const Geo& g = a.g;
     const int kit = __ldcg(&vst->k);
     const double sigma = __ldcg(&vst->pend_sigma);
@@ -834,7 +848,7 @@ int stencil_blocks(const Geo& g, int chunk) {
     return ntj * ntk * nch;
 }
 
-template <int MODE, int NC>
+template <int MODE, int NC, bool FIRSTK = false>
 static cudaError_t launch_one(const StencilArgs& a0, cudaStream_t s) {
     StencilArgs a = a0;
     a.ntj = (a.g.nt + TJ - 1) / TJ;
@@ -843,7 +857,7 @@ static cudaError_t launch_one(const StencilArgs& a0, cudaStream_t s) {
     const int smem = 4 * (NC + 1) * HROWS * ROW * (int)sizeof(double);
     static bool attr_done = false;
     if (!attr_done) {
-        cudaError_t e = cudaFuncSetAttribute(k_stencil<MODE, NC>,
+        cudaError_t e = cudaFuncSetAttribute(k_stencil<MODE, NC, FIRSTK>,
                                              cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
         if (e != cudaSuccess) return e;
         attr_done = true;
@@ -851,20 +865,20 @@ static cudaError_t launch_one(const StencilArgs& a0, cudaStream_t s) {
     const int T = a.ntj * a.ntk;
     const int blocks = a.part == 1 ? T * (a.nchunk - 2) : a.part == 2 ? 2 * T : T * a.nchunk;
     if (blocks <= 0) return cudaErrorInvalidValue;
-    k_stencil<MODE, NC><<<blocks, kSThreads, smem, s>>>(a);
+    k_stencil<MODE, NC, FIRSTK><<<blocks, kSThreads, smem, s>>>(a);
     return cudaGetLastError();
 }
 
-cudaError_t launch_stencil(int mode, int ncomp, const StencilArgs& a, cudaStream_t s) {
+cudaError_t launch_stencil(int mode, int ncomp, const StencilArgs& a, cudaStream_t s, bool first) {
     if (ncomp == 1) {
         if (mode == MODE_APPLY) return launch_one<MODE_APPLY, 1>(a, s);
         if (mode == MODE_RESID) return launch_one<MODE_RESID, 1>(a, s);
-        return launch_one<MODE_PCGA, 1>(a, s);
+        return first ? launch_one<MODE_PCGA, 1, true>(a, s) : launch_one<MODE_PCGA, 1>(a, s);
     }
     if (ncomp == 3) {
         if (mode == MODE_APPLY) return launch_one<MODE_APPLY, 3>(a, s);
         if (mode == MODE_RESID) return launch_one<MODE_RESID, 3>(a, s);
-        return launch_one<MODE_PCGA, 3>(a, s);
+        return first ? launch_one<MODE_PCGA, 3, true>(a, s) : launch_one<MODE_PCGA, 3>(a, s);
     }
     return cudaErrorInvalidValue;
 }

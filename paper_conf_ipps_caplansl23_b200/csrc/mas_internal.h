@@ -113,7 +113,9 @@ struct StreamArgs {  // kernel B
 
 // launchers (kernels.cu)
 int stencil_blocks(const Geo& g, int chunk);
-cudaError_t launch_stencil(int mode, int ncomp, const StencilArgs& a, cudaStream_t s);
+// first: kernel A of iteration 1 (its own instantiation)
+cudaError_t launch_stencil(int mode, int ncomp, const StencilArgs& a, cudaStream_t s,
+                           bool first = false);
 cudaError_t launch_pcg_b(const StreamArgs& a, int nblocks, cudaStream_t s);
 cudaError_t launch_diag(const Geo& g, Halo kappa, const double* c, double* D, double* dinv,
                         int* bad, cudaStream_t s);
