@@ -479,7 +479,8 @@ mas_status_t mas_op_setup(mas_grid_t* g, int ncomp, const double* kappa, const d
     }
     if (op->chunk < 1 || op->chunk > 64) op->chunk = 16;
     op->max_blocks = stencil_blocks(G, op->chunk);
-    op->b_blocks = 148 * 8;
+    const char* bb_env = getenv("MAS_BBLOCKS");  // experiment hook
+    op->b_blocks = bb_env ? atoi(bb_env) : 148 * 8;
     if (op->b_blocks > op->max_blocks) op->max_blocks = op->b_blocks;
     TRY(dmalloc(&op->scr.partials, 4 * (size_t)op->max_blocks));
     TRY(dmalloc(&op->scr.ticket, 8));
