@@ -46,6 +46,8 @@ CONFIGS = {
     # one rank's share of C3 at P = 8 (32 r-planes), to study the per-GPU
     # kernel efficiency that bounds 8-GPU strong scaling
     "C3s8": ("viscosity", 32, 256, 512),
+    # the whole C4 problem of 8 GPUs (268 M cells) on one B200
+    "C4x8": ("viscosity", 2048, 256, 512),
     "C2": ("conduction", 128, 128, 256),
     "C1": ("mms", 16, 24, 32),
 }
