@@ -202,6 +202,10 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--cpu-iters", type=int, default=3)
+    ap.add_argument("--transport", default="auto", choices=["auto", "p2p", "nccl"],
+                    help="multi-GPU PCG loop: P2P (NVLink peer memory: mailbox allreduce + "
+                         "in-place seam reads, one CUDA graph per rank) or NCCL; auto = P2P "
+                         "if every rank can map its peers, else NCCL")
     args = ap.parse_args()
     if args.impl == "reference":
         return run_reference(args)
@@ -243,6 +247,17 @@ def main():
     x0 = to_dev(prob.x0[:, sl])
     x = x0.clone()
     op = M.Operator(grid, nc, kappa, cmass, prob.bc_inner, prob.bc_outer)
+    transport = "single-gpu"
+    if world > 1:
+        transport = "nccl"
+        if args.transport != "nccl":
+            try:
+                op.enable_p2p()
+                transport = "p2p"
+            except M.MasError as e:  # collective verdict: every rank keeps NCCL
+                if args.transport == "p2p":
+                    raise
+                transport = f"nccl (p2p unavailable: {e})"
     ubi = to_dev(prob.ub_inner) if prob.ub_inner is not None else None
     ubo = to_dev(prob.ub_outer) if prob.ub_outer is not None else None
     rhs = f.clone()
@@ -264,9 +279,10 @@ def main():
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
-    # timed region: the production path (single GPU: the whole PCG loop is one
-    # CUDA graph with a device-side while node; multi-GPU: host-driven loop
-    # with NCCL between the kernels)
+    # timed region: the production path (one GPU, or multi-GPU with the P2P
+    # transport: the whole PCG loop is one CUDA graph per rank with a
+    # device-side while node; multi-GPU NCCL: host-driven loop with NCCL
+    # between the kernels)
     clocks = ClockSampler(local)
     clocks.start()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -370,7 +386,7 @@ def main():
             "dtype": "f64", "data": "synthetic",
             "config": {"workload": args.config, "grid": [nr, nt, np_], "ncomp": nc,
                        "cells": cells, "tol": args.tol, "iters_per_solve": iters_per_solve,
-                       "parallelism": f"r-slab x{world}",
+                       "parallelism": f"r-slab x{world}", "transport": transport,
                        "l2": "inputs > L2 (268 MB per field vs 126 MB); no flush",
                        "step": "mas_op_update + x:=x0 + mas_pcg_solve"},
             "roofline": {"bound": "hbm", "kernel": "k_stencil<PCGA> (kernel A)",

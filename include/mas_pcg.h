@@ -158,6 +158,31 @@ MAS_API mas_status_t mas_pcg_solve(const mas_op_t* op, const double* rhs, double
                            double tol, int maxit, int* iters, double* relres,
                            double* res_hist, cudaStream_t stream);
 
+/* Collective (all ranks, after mas_op_setup): switch this op's PCG iteration
+ * loop from NCCL to the P2P transport over NVLink / NVSwitch peer memory.
+ * Multi-GPU PCG needs two exchange steps per iteration (
+ * the paper's halo exchanges use GPU peer-to-peer transfers, P:1005-1007,
+ * Fig. 4):
+ *   - seams: kernel A reads the r-neighbours' edge planes of r_{k-1} and
+ *     p_{k-1} in place from their device memory (no send/recv, no ghost copy);
+ *   - the two scalar allreduces: the reducing kernel's last block writes its
+ *     rank-local partials into every rank's mailbox (one-shot NVLink stores
+ *     + a sequence number); the consuming kernel sums all ranks' entries in
+ *     rank order, so every rank gets identical bits and the same stop
+ *     decision.  The loop then runs as one CUDA graph per rank with no host
+ *     round trip.
+ * Setup uses CUDA IPC (cudaIpcGetMemHandle / cudaIpcOpenMemHandle) on the
+ * library-owned r, p and mailbox buffers, with the handles all-gathered over
+ * the grid's NCCL communicator; the init residual, op setup/update seams and
+ * mas_op_dot keep NCCL.  With one rank the mailbox path runs against itself.
+ * Errors: MAS_ERR_CUDA on every rank if any rank cannot map its peers (the op
+ * then keeps the NCCL loop); MAS_ERR_NCCL.  A mailbox wait longer than 60 s
+ * traps the kernel (fails loudly rather than hanging). */
+MAS_API mas_status_t mas_op_enable_p2p(mas_op_t* op, cudaStream_t stream);
+
+/* Transport of the op's PCG loop: 0 NCCL (or one GPU), 1 P2P; -1 if op is NULL. */
+MAS_API int mas_op_transport(const mas_op_t* op);
+
 /* Kernel launches issued by the last mas_pcg_solve on this op (its CUDA path
  * evidence; includes early-exit launches after convergence). */
 MAS_API long long mas_op_launch_count(const mas_op_t* op);

@@ -122,6 +122,16 @@ struct mas_op {
     const double* g_x = nullptr;
     const double* g_hist = nullptr;
     int use_graph = 1;
+    // P2P transport (mas_op_enable_p2p): mailbox allreduce + in-place reads of
+    // the r-neighbours' edge planes over NVLink instead of NCCL in the loop
+    int p2p = 0;
+    Mail* mbox = nullptr;              // own mailbox [2 slots][nranks]
+    Mail** d_peers = nullptr;          // device array [nranks] of every rank's mailbox
+    std::vector<void*> ipc_opened;     // cudaIpcOpenMemHandle mappings (closed at destroy)
+    const double* nb_r[2] = {nullptr, nullptr};  // rank-1 / rank+1 r arrays
+    const double* nb_p[2][2] = {{nullptr, nullptr}, {nullptr, nullptr}};  // [parity][lo/hi]
+    int nb_nl[2] = {0, 0};             // their slab sizes
+    unsigned long long epoch = 0;      // solves so far (mailbox sequence numbers)
 };
 
 extern "C" {
@@ -233,7 +243,42 @@ static Halo halo_of(const mas_op* op, const double* in, const double* ghosts, in
     const long long plane = op->geo.plane;
     h.glo = (ghosts && !op->geo.glob_lo) ? ghosts : nullptr;
     h.ghi = (ghosts && !op->geo.glob_hi) ? ghosts + (long long)ncomp * plane : nullptr;
+    h.slo = h.shi = (int)plane;
     return h;
+}
+
+// P2P transport: the ghost planes are the r-neighbours' own edge planes,
+// read in place (lo: last plane of rank-1's array, hi: first plane of rank+1's)
+static Halo peer_halo(const mas_op* op, const double* in, const double* lo, const double* hi) {
+    Halo h;
+    h.in = in;
+    const long long plane = op->geo.plane;
+    h.glo = (lo && !op->geo.glob_lo) ? lo + (long long)(op->nb_nl[0] - 1) * plane : nullptr;
+    h.ghi = (hi && !op->geo.glob_hi) ? hi : nullptr;
+    h.slo = (int)(op->nb_nl[0] * plane);
+    h.shi = (int)(op->nb_nl[1] * plane);
+    return h;
+}
+
+// the fields kernel A reads with an r-halo in iteration k: r_{k-1}, p_{k-1}
+static Halo r_halo(const mas_op* op) {
+    return op->p2p ? peer_halo(op, op->r, op->nb_r[0], op->nb_r[1])
+                   : halo_of(op, op->r, op->rg, op->ncomp);
+}
+static Halo pold_halo(const mas_op* op, int k) {
+    const int par = (k + 1) & 1;
+    return op->p2p ? peer_halo(op, op->p[par], op->nb_p[par][0], op->nb_p[par][1])
+                   : halo_of(op, op->p[par], op->g->comm ? op->pg[par] : nullptr, op->ncomp);
+}
+static P2P p2p_args(const mas_op* op) {
+    P2P t{};
+    if (op->p2p) {
+        t.own = op->mbox;
+        t.peers = op->d_peers;
+        t.nranks = comm_nranks(op->g->comm);
+        t.rank = comm_rank(op->g->comm);
+    }
+    return t;
 }
 
 // copy coefficients in (host or device pointers), compute D and 1/D, exchange
@@ -287,6 +332,9 @@ static void op_free(mas_op* op) {
     if (op->ev_ready) cudaEventDestroy(op->ev_ready);
     if (op->ev_seam) cudaEventDestroy(op->ev_seam);
     if (op->cap_stream) cudaStreamDestroy(op->cap_stream);
+    for (void* p : op->ipc_opened) cudaIpcCloseMemHandle(p);
+    if (op->mbox) cudaFree(op->mbox);
+    if (op->d_peers) cudaFree(op->d_peers);
     delete op;
 }
 
@@ -341,7 +389,7 @@ static mas_status_t loop_graph(mas_op* op, StencilArgs a, StreamArgs b) {
             // iteration 1 runs before the loop (its own kernel-A instantiation);
             // the body covers an even and an odd iteration: k = 2, 3, 4, ...
             for (int kk = 2; kk <= 3 && e == cudaSuccess; kk++) {
-                a.pold = halo_of(op, op->p[(kk + 1) & 1], nullptr, nc);
+                a.pold = pold_halo(op, kk);
                 a.pnew = op->p[kk & 1];
                 e = launch_stencil(MODE_PCGA, nc, a, op->cap_stream);
                 if (e == cudaSuccess) e = launch_pcg_b(b, op->b_blocks, op->cap_stream);
@@ -615,6 +663,102 @@ mas_status_t mas_op_dot(const mas_op_t* op_c, const double* a, const double* b, 
     return MAS_OK;
 }
 
+// Collective: switch the iteration loop of this op to the P2P transport.
+// Every rank exports (CUDA IPC) its r, p[0], p[1] and mailbox; the records
+// are all-gathered once; each rank maps its r-neighbours' r / p arrays and
+// every rank's mailbox.  Virtual ranks (one process) share raw pointers.
+mas_status_t mas_op_enable_p2p(mas_op_t* op, cudaStream_t s) {
+    if (!op) return arg_error("null op");
+    if (op->p2p) return MAS_OK;
+    Comm* comm = op->g->comm;
+    const int P = comm_nranks(comm), rank = comm_rank(comm);
+    const bool virt = comm_is_virtual(comm);
+    ST(dmalloc(&op->mbox, 2 * (size_t)P));
+    CU(cudaMemset(op->mbox, 0, 2 * (size_t)P * sizeof(Mail)));
+    struct Rec {
+        cudaIpcMemHandle_t h[4];
+        unsigned long long raw[4];
+        int nl;
+        int ok;
+    };
+    Rec mine;
+    memset(&mine, 0, sizeof(mine));
+    const void* bufs[4] = {op->r, op->p[0], op->p[1], op->mbox};
+    mine.nl = op->g->nl;
+    mine.ok = 1;
+    for (int b = 0; b < 4; b++) {
+        mine.raw[b] = (unsigned long long)(uintptr_t)bufs[b];
+        if (P > 1 && !virt && cudaIpcGetMemHandle(&mine.h[b], const_cast<void*>(bufs[b])) != cudaSuccess) {
+            cudaGetLastError();
+            mine.ok = 0;
+        }
+    }
+    std::vector<Rec> all(P);
+    ST(comm_allgather_bytes(comm, &mine, all.data(), sizeof(Rec), s));
+    bool ok = true;
+    for (int q = 0; q < P; q++) ok = ok && all[q].ok;
+    std::string why = ok ? "" : "cudaIpcGetMemHandle failed on some rank";
+    auto map = [&](int q, int b) -> void* {
+        if (q == rank || virt) return (void*)(uintptr_t)all[q].raw[b];
+        void* p = nullptr;
+        if (cudaIpcOpenMemHandle(&p, all[q].h[b], cudaIpcMemLazyEnablePeerAccess) != cudaSuccess) {
+            why = std::string("cudaIpcOpenMemHandle: ") + cudaGetErrorString(cudaGetLastError());
+            ok = false;
+            return nullptr;
+        }
+        op->ipc_opened.push_back(p);
+        return p;
+    };
+    std::vector<Mail*> peers(P, nullptr);
+    for (int q = 0; q < P && ok; q++) peers[q] = (Mail*)map(q, 3);
+    for (int side = 0; side < 2 && ok; side++) {
+        const int q = side == 0 ? rank - 1 : rank + 1;
+        if (q < 0 || q >= P) continue;
+        op->nb_r[side] = (const double*)map(q, 0);
+        op->nb_p[0][side] = (const double*)map(q, 1);
+        op->nb_p[1][side] = (const double*)map(q, 2);
+        op->nb_nl[side] = all[q].nl;
+    }
+    if (ok && dmalloc(&op->d_peers, (size_t)P) == MAS_OK &&
+        cudaMemcpy(op->d_peers, peers.data(), P * sizeof(Mail*), cudaMemcpyHostToDevice) != cudaSuccess) {
+        cudaGetLastError();
+        ok = false;
+        why = "peer table copy";
+    }
+    if (comm && P > 1) {  // every rank adopts the transport, or none does
+        double* d = op->dot_out;
+        double flag = ok ? 0.0 : 1.0;
+        CU(cudaMemcpyAsync(d, &flag, sizeof(double), cudaMemcpyHostToDevice, s));
+        ST(comm_allreduce(comm, d, 1, s));
+        CU(cudaMemcpyAsync(&flag, d, sizeof(double), cudaMemcpyDeviceToHost, s));
+        CU(cudaStreamSynchronize(s));
+        if (flag != 0.0 && ok) {
+            ok = false;
+            why = "P2P setup failed on another rank";
+        }
+    }
+    if (!ok) {
+        for (void* p : op->ipc_opened) cudaIpcCloseMemHandle(p);
+        op->ipc_opened.clear();
+        cudaFree(op->mbox);
+        op->mbox = nullptr;
+        if (op->d_peers) cudaFree(op->d_peers);
+        op->d_peers = nullptr;
+        op->nb_r[0] = op->nb_r[1] = nullptr;
+        op->nb_p[0][0] = op->nb_p[0][1] = op->nb_p[1][0] = op->nb_p[1][1] = nullptr;
+        set_last_error("P2P transport unavailable: " + why);
+        return MAS_ERR_CUDA;
+    }
+    op->p2p = 1;
+    if (op->gexec) {  // the loop graph reads the ghost planes differently now
+        cudaGraphExecDestroy(op->gexec);
+        op->gexec = nullptr;
+    }
+    return MAS_OK;
+}
+
+int mas_op_transport(const mas_op_t* op) { return !op ? -1 : op->p2p ? 1 : 0; }
+
 long long mas_op_launch_count(const mas_op_t* op) { return op ? op->launches : -1; }
 
 mas_status_t mas_op_set_profiling(mas_op_t* op, int on) {
@@ -659,7 +803,9 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
         xd = op->stage_b;
     }
 
+    const bool p2p = op->p2p;
     PcgState init{};
+    if (p2p) init.epoch = ++op->epoch;
     init.tol = tol;
     init.maxit = maxit;
     init.k = 1;
@@ -688,9 +834,10 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
     a.rr_hist = rr_h;
     a.scr = op->scr;
     a.host_flag = op->host_flag_dev;
+    a.p2p = p2p_args(op);
     CU(launch_stencil(MODE_RESID, nc, a, s));
     op->launches++;
-    if (comm) ST(comm_allreduce(comm, &op->st->pend_rho, 3, s));  // rho, rr, ff
+    if (comm && !p2p) ST(comm_allreduce(comm, &op->st->pend_rho, 3, s));  // rho, rr, ff
 
     StreamArgs b{};
     b.g = op->geo;
@@ -704,19 +851,22 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
     b.rr_hist = rr_h;
     b.scr = op->scr;
     b.host_flag = op->host_flag_dev;
+    b.p2p = p2p_args(op);
 
     // a4: iterations.  Kernel A(k) reads k, alpha, beta and the convergence
     // decision from PcgState; the host only keeps two iterations in flight
     // and stops enqueueing once the device reports the stop (a decision all
     // ranks take identically, so the collectives stay matched).
-    a.u = halo_of(op, op->r, op->rg, nc);
+    a.u = r_halo(op);
     a.out = op->q;
     a.x = xd;
     a.f = nullptr;
-    const bool graph = !comm && !op->prof && op->use_graph;
+    // no host involvement per iteration on one GPU and with the P2P transport
+    // (virtual P2P ranks share one GPU and need host ordering: comm_vsync)
+    const bool graph = !op->prof && op->use_graph && (!comm || (p2p && !comm_is_virtual(comm)));
     if (graph) {
         ST(loop_graph(op, a, b));
-        a.pold = halo_of(op, op->p[0], nullptr, nc);  // iteration 1
+        a.pold = pold_halo(op, 1);  // iteration 1 (not read)
         a.pnew = op->p[1];
         CU(launch_stencil(MODE_PCGA, nc, a, s, true));
         CU(launch_pcg_b(b, op->b_blocks, s));
@@ -727,14 +877,14 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
         NvtxRange nvtx_it("pcg iteration (A, [seams, allreduce], B)");
         double* pold = op->p[(k + 1) & 1];
         double* pnew = op->p[k & 1];
-        a.pold = halo_of(op, pold, op->pg[(k + 1) & 1], nc);
+        a.pold = pold_halo(op, k);
         a.pnew = pnew;
         cudaEvent_t* pe = nullptr;
         if (op->prof) {
             ST(ensure_prof_events(op, k));
             pe = &op->pev[4 * (size_t)(k - 1)];
         }
-        if (comm) {
+        if (comm && !p2p) {
             // seams of r and p_{k-1} on the comm stream, overlapped with kernel
             // A on the interior chunks; the two edge chunks wait for them
             CU(cudaEventRecord(op->ev_ready, s));
@@ -760,18 +910,20 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
                 op->launches++;
             }
         } else {
+            if (p2p) ST(comm_vsync(comm, s));  // virtual P2P ranks: all B(k-1) done
             if (pe) CU(cudaEventRecord(pe[0], s));
             CU(launch_stencil(MODE_PCGA, nc, a, s, k == 1));
             op->launches++;
         }
         if (pe) CU(cudaEventRecord(pe[1], s));
-        if (comm) ST(comm_allreduce(comm, &op->st->pend_sigma, 1, s));
+        if (comm && !p2p) ST(comm_allreduce(comm, &op->st->pend_sigma, 1, s));
         if (k <= maxit) {
+            if (p2p) ST(comm_vsync(comm, s));  // virtual P2P ranks: all A(k) done
             if (pe) CU(cudaEventRecord(pe[2], s));
             CU(launch_pcg_b(b, op->b_blocks, s));
             op->launches++;
             if (pe) CU(cudaEventRecord(pe[3], s));
-            if (comm) ST(comm_allreduce(comm, &op->st->pend_rho, 2, s));
+            if (comm && !p2p) ST(comm_allreduce(comm, &op->st->pend_rho, 2, s));
         }
         CU(cudaEventRecord(op->ev[k & 1], s));
         if (k >= 2) {
@@ -788,6 +940,9 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
     }
     (void)stop_seen_at;
     CU(cudaStreamSynchronize(s));
+    // P2P: no rank may publish the next solve's partials while another rank's
+    // kernels of this solve can still read its mailbox
+    if (p2p && comm) ST(comm_barrier(comm, s));
     PcgState fin{};
     CU(cudaMemcpy(&fin, op->st, sizeof(fin), cudaMemcpyDeviceToHost));
     if (!fin.stopped) {

@@ -42,6 +42,8 @@ struct VGroup {
     std::vector<cudaEvent_t> ev_seam, ev_pull; // per rank: seam data ready / pulls done
     std::vector<const double*> seam_src;       // per rank: interior field of this seam call
     std::vector<int> seam_nl;
+    std::vector<std::vector<unsigned char>> gather;  // allgather staging (host)
+    std::vector<cudaEvent_t> ev_sync;          // per rank: comm_vsync
 
     void barrier() {
         std::unique_lock<std::mutex> lk(m);
@@ -104,12 +106,15 @@ static mas_status_t vgroup_join(const mas_dist_t* d, Comm* c) {
             g->ev_pull.resize(g->n);
             g->seam_src.assign(g->n, nullptr);
             g->seam_nl.assign(g->n, 0);
+            g->gather.resize(g->n);
+            g->ev_sync.resize(g->n);
             cudaError_t e = cudaMalloc(&g->stage, sizeof(double) * 8 * g->n);
             for (int r = 0; r < g->n && e == cudaSuccess; r++) {
                 e = cudaEventCreateWithFlags(&g->ev_in[r], cudaEventDisableTiming);
                 if (e == cudaSuccess) e = cudaEventCreateWithFlags(&g->ev_out[r], cudaEventDisableTiming);
                 if (e == cudaSuccess) e = cudaEventCreateWithFlags(&g->ev_seam[r], cudaEventDisableTiming);
                 if (e == cudaSuccess) e = cudaEventCreateWithFlags(&g->ev_pull[r], cudaEventDisableTiming);
+                if (e == cudaSuccess) e = cudaEventCreateWithFlags(&g->ev_sync[r], cudaEventDisableTiming);
             }
             if (e != cudaSuccess) return cuda_fail(e, "virtual group setup");
             g_vmap[key] = g;
@@ -174,6 +179,7 @@ void comm_destroy(Comm* c) {
                 cudaEventDestroy(g->ev_out[r]);
                 cudaEventDestroy(g->ev_seam[r]);
                 cudaEventDestroy(g->ev_pull[r]);
+                cudaEventDestroy(g->ev_sync[r]);
             }
             cudaFree(g->stage);
             g_vmap.erase(c->vkey);
@@ -274,6 +280,63 @@ mas_status_t comm_seams(Comm* c, const double* in, int ncomp, int nl, long long 
     }
     r = ncclGroupEnd();
     return r == ncclSuccess ? MAS_OK : nccl_fail(r, "seam send/recv");
+}
+
+// ---------------------------------------------------------------------------
+// setup-time helpers of the P2P transport
+// ---------------------------------------------------------------------------
+bool comm_is_virtual(const Comm* c) { return c && c->vg; }
+int comm_rank(const Comm* c) { return c ? c->rank : 0; }
+int comm_nranks(const Comm* c) { return c ? c->nranks : 1; }
+
+// all[r * n .. r * n + n) = rank r's `mine` (host buffers), for every rank r
+mas_status_t comm_allgather_bytes(Comm* c, const void* mine, void* all, size_t n, cudaStream_t s) {
+    if (!c || c->nranks == 1) {
+        memcpy(all, mine, n);
+        return MAS_OK;
+    }
+    if (c->vg) {
+        VGroup* g = c->vg;
+        g->gather[c->rank].assign((const unsigned char*)mine, (const unsigned char*)mine + n);
+        g->barrier();
+        for (int r = 0; r < g->n; r++) memcpy((unsigned char*)all + r * n, g->gather[r].data(), n);
+        g->barrier();
+        return MAS_OK;
+    }
+    unsigned char* d = nullptr;
+    cudaError_t e = cudaMalloc(&d, n * (c->nranks + 1));
+    if (e != cudaSuccess) return cuda_fail(e, "allgather buffer");
+    mas_status_t st = MAS_OK;
+    if ((e = cudaMemcpyAsync(d, mine, n, cudaMemcpyHostToDevice, s)) != cudaSuccess) {
+        st = cuda_fail(e, "allgather copy");
+    } else {
+        ncclResult_t r = ncclAllGather(d, d + n, n, ncclChar, c->nccl, s);
+        if (r != ncclSuccess)
+            st = nccl_fail(r, "ncclAllGather");
+        else if ((e = cudaMemcpyAsync(all, d + n, n * c->nranks, cudaMemcpyDeviceToHost, s)) !=
+                     cudaSuccess ||
+                 (e = cudaStreamSynchronize(s)) != cudaSuccess)
+            st = cuda_fail(e, "allgather copy back");
+    }
+    cudaFree(d);
+    return st;
+}
+
+// Virtual ranks only: order stream s after the work every rank has enqueued
+// so far.  The P2P kernels' mailbox waits are then already satisfied when a
+// kernel starts: on one GPU a spinning consumer could otherwise occupy the
+// SMs its producer (another virtual rank's kernel) needs.
+mas_status_t comm_vsync(Comm* c, cudaStream_t s) {
+    if (!c || !c->vg) return MAS_OK;
+    VGroup* g = c->vg;
+    cudaError_t e;
+    if ((e = cudaEventRecord(g->ev_sync[c->rank], s)) != cudaSuccess) return cuda_fail(e, "vsync record");
+    g->barrier();
+    for (int r = 0; r < g->n; r++)
+        if (r != c->rank && (e = cudaStreamWaitEvent(s, g->ev_sync[r], 0)) != cudaSuccess)
+            return cuda_fail(e, "vsync wait");
+    g->barrier();  // every rank captured the events before they are recorded again
+    return MAS_OK;
 }
 
 mas_status_t comm_barrier(Comm* c, cudaStream_t s) {

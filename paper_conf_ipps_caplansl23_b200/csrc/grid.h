@@ -48,5 +48,11 @@ mas_status_t comm_allreduce(Comm* c, double* buf, int n, cudaStream_t s);
 mas_status_t comm_seams(Comm* c, const double* in, int ncomp, int nl, long long plane, double* glo,
                         double* ghi, cudaStream_t s);
 mas_status_t comm_barrier(Comm* c, cudaStream_t s);
+// P2P transport setup helpers
+bool comm_is_virtual(const Comm* c);
+int comm_rank(const Comm* c);
+int comm_nranks(const Comm* c);
+mas_status_t comm_allgather_bytes(Comm* c, const void* mine, void* all, size_t n, cudaStream_t s);
+mas_status_t comm_vsync(Comm* c, cudaStream_t s);
 
 }  // namespace mas

@@ -63,8 +63,10 @@ __device__ __forceinline__ double warp_sum(double v) {
 // Block-reduce NS sums, publish the block partial, take a ticket.  Returns
 // true in the last block to finish, where `v` then holds the grid totals
 // (valid in thread 0), summed in a fixed order independent of scheduling.
+// sysfence: the block's global writes are also read by peer GPUs (P2P
+// transport), so order them at system scope before the ticket.
 template <int NS, int NTHR = kThreads>
-__device__ bool grid_reduce(double (&v)[NS], const Scratch& scr, int tkt) {
+__device__ bool grid_reduce(double (&v)[NS], const Scratch& scr, int tkt, bool sysfence = false) {
     __shared__ double wsum[NS][NTHR / 32];
     __shared__ bool last;
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
@@ -81,7 +83,10 @@ __device__ bool grid_reduce(double (&v)[NS], const Scratch& scr, int tkt) {
             for (int q = 0; q < NTHR / 32; q++) t += wsum[s][q];
             scr.partials[(size_t)blockIdx.x * NS + s] = t;
         }
-        __threadfence();
+        if (sysfence)
+            __threadfence_system();
+        else
+            __threadfence();
         unsigned old = atomicAdd(&scr.ticket[tkt], 1u);
         last = (old == gridDim.x - 1);
     }
@@ -108,6 +113,71 @@ __device__ bool grid_reduce(double (&v)[NS], const Scratch& scr, int tkt) {
 }
 
 // --------------------------------------------------------------------------
+// P2P transport: one-shot allreduce through peer mailboxes (NVLink stores)
+// --------------------------------------------------------------------------
+// The reducing kernel's last block writes its rank-local partials into slot
+// [rank] of EVERY rank's mailbox, then (after a system-scope fence) the
+// sequence number.  A consumer kernel waits in thread 0 of each block until
+// all nranks entries of its own mailbox carry the expected sequence and sums
+// them in rank order: every rank obtains the same bits, so every rank takes
+// the same stop / breakdown decision and the loop needs no host handshake.
+// A publication of iteration k needs every rank past its consumer of
+// iteration k-1 (each kernel waits for all ranks' previous partials), so one
+// mailbox slot per kernel kind suffices.
+__device__ __forceinline__ unsigned long long p2p_seq(unsigned long long epoch, int k) {
+    return (epoch << 32) | (unsigned long long)(unsigned)(k + 1);
+}
+__device__ __forceinline__ unsigned long long gtimer_ns() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+constexpr unsigned long long kP2PTimeoutNs = 60ull * 1000000000ull;
+// slow path: spin (with a 60 s limit: fail loudly rather than hang)
+__device__ __noinline__ void p2p_wait(const volatile unsigned long long* sp, unsigned long long seq,
+                                      int rank, int slot, int from) {
+    const unsigned long long t0 = gtimer_ns();
+    while (*sp != seq) {
+        __nanosleep(100);
+        if (gtimer_ns() - t0 > kP2PTimeoutNs) {
+            printf("maspcg: P2P mailbox wait timed out (rank %d, slot %d, from rank %d)\n", rank,
+                   slot, from);
+            __trap();
+        }
+    }
+}
+
+// the calling thread waits for and sums the nranks entries (rank order)
+template <int N>
+__device__ __forceinline__ void p2p_gather_one(const P2P& t, int slot, unsigned long long seq,
+                                               double (&out)[N]) {
+    const Mail* mb = t.own + slot * t.nranks;
+#pragma unroll
+    for (int n = 0; n < N; n++) out[n] = 0.0;
+    for (int q = 0; q < t.nranks; q++) {
+        const volatile unsigned long long* sp = &mb[q].seq;
+        if (*sp != seq) p2p_wait(sp, seq, t.rank, slot, q);
+        __threadfence_system();  // the values were written before the sequence
+        const volatile double* v = mb[q].v;
+#pragma unroll
+        for (int n = 0; n < N; n++) out[n] += v[n];
+    }
+}
+
+// thread 0 of the last block: publish n rank-local partials to every rank
+__device__ void p2p_publish(const P2P& t, int slot, unsigned long long seq, const double* v, int n) {
+    for (int q = 0; q < t.nranks; q++) {
+        volatile Mail* m = t.peers[q] + slot * t.nranks + t.rank;
+        for (int i = 0; i < n; i++) m->v[i] = v[i];
+    }
+    __threadfence_system();
+    for (int q = 0; q < t.nranks; q++) {
+        volatile Mail* m = t.peers[q] + slot * t.nranks + t.rank;
+        m->seq = seq;
+    }
+}
+
+// --------------------------------------------------------------------------
 // field access
 // --------------------------------------------------------------------------
 // The stencil kernels index with 32-bit offsets (the host rejects slabs with
@@ -115,8 +185,8 @@ __device__ bool grid_reduce(double (&v)[NS], const Scratch& scr, int tkt) {
 __device__ __forceinline__ int plane32(const Geo& g) { return (int)g.plane; }
 // --------------------------------------------------------------------------
 __device__ __forceinline__ const double* plane_ptr(const Halo& h, int comp, int i, const Geo& g) {
-    if (i < 0) return h.glo + (int)comp * plane32(g);
-    if (i >= g.nl) return h.ghi + (int)comp * plane32(g);
+    if (i < 0) return h.glo + (int)comp * h.slo;
+    if (i >= g.nl) return h.ghi + (int)comp * h.shi;
     return h.in + ((int)comp * g.nl + i) * plane32(g);
 }
 __device__ __forceinline__ double2 ld2(const double* p) {
@@ -398,6 +468,34 @@ __device__ __forceinline__ void ghost_plane(double* buf, int height, int width, 
     }
 }
 
+// Global <f,f>, <r_{k-1},r_{k-1}>, <r_{k-1},z_{k-1}> entering A(k): from
+// PcgState (one GPU / NCCL allreduce in place), or summed from the mailbox of
+// B(k-1) (init at k = 1) under the P2P transport.  block: every thread of
+// the block calls (thread 0 waits, the others read its sums); otherwise the
+// calling thread alone.
+__device__ __forceinline__ void a_globals(const StencilArgs& a, int kit, double& ff, double& rr,
+                                          double& rho1, bool block = false) {
+    const PcgState* st = a.st;
+    ff = __ldcg(&st->pend_ff);
+    rr = __ldcg(&st->pend_rr);
+    rho1 = __ldcg(&st->pend_rho);
+    if (a.p2p.nranks > 0) {
+        __shared__ double sh[3];
+        double v[3];
+        if (!block || threadIdx.x == 0) {
+            p2p_gather_one<3>(a.p2p, MB_B, p2p_seq(__ldcg(&st->epoch), kit - 1), v);
+            if (block) sh[0] = v[0], sh[1] = v[1], sh[2] = v[2];
+        }
+        if (block) {
+            __syncthreads();
+            v[0] = sh[0], v[1] = sh[1], v[2] = sh[2];
+        }
+        rho1 = v[0];
+        rr = v[1];
+        if (kit == 1) ff = v[2];
+    }
+}
+
 // --------------------------------------------------------------------------
 // the fused stencil kernel
 // --------------------------------------------------------------------------
@@ -422,6 +520,8 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
     bool first = false;
     double beta = 0.0, alpha_prev = 0.0;
     int kit = 0;
+    const bool p2p = a.p2p.nranks > 0;
+    __shared__ double final_g[3];
     if (MODE == MODE_PCGA) {
         // one round trip: everything A(k) needs sits in PcgState (written by
         // earlier kernels; read through L2)
@@ -434,8 +534,10 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
             return;
         }
         kit = __ldcg(&st->k);
-        const double ff = __ldcg(&st->pend_ff), rr = __ldcg(&st->pend_rr);
-        const double rho1 = __ldcg(&st->pend_rho), rho2 = __ldcg(&st->rho_prev);
+        double ff, rr, rho1;
+        a_globals(a, kit, ff, rr, rho1, true);
+        final_g[0] = ff, final_g[1] = rr, final_g[2] = rho1;  // for the stop branch below
+        const double rho2 = __ldcg(&st->rho_prev);
         const double sig1 = __ldcg(&st->sigma_prev);
         first = (kit == 1);
         if (kit >= 2) alpha_prev = rho2 / sig1;
@@ -492,9 +594,9 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
         double v1[1] = {0.0};
         if (grid_reduce<1, kSThreads>(v1, a.scr, TKT_STENCIL) && threadIdx.x == 0 && a.part != 1) {
             PcgState* st = a.st;
-            const double ff = st->pend_ff, rr = st->pend_rr;
+            const double ff = final_g[0], rr = final_g[1], rho1 = final_g[2];
             a.rr_hist[kit - 1] = rr;
-            a.rho_hist[kit - 1] = st->pend_rho;
+            a.rho_hist[kit - 1] = rho1;
             if (pmode == P_ZERO) {
                 st->iters = 0;
                 st->relres = 0.0;
@@ -665,23 +767,36 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
 
     // ---- reductions -------------------------------------------------------
     if (MODE == MODE_RESID) {
-        if (grid_reduce<3, kSThreads>(acc, a.scr, TKT_STENCIL) && threadIdx.x == 0) {
+        if (grid_reduce<3, kSThreads>(acc, a.scr, TKT_STENCIL, p2p) && threadIdx.x == 0) {
             PcgState* st = a.st;
             st->pend_ff = acc[0];
             st->pend_rr = acc[1];
             st->pend_rho = acc[2];
+            if (p2p) {
+                const double pub[3] = {acc[2], acc[1], acc[0]};  // {rho, rr, ff}
+                p2p_publish(a.p2p, MB_B, p2p_seq(st->epoch, 0), pub, 3);
+            }
         }
     } else if (MODE == MODE_PCGA) {
         double v[1] = {acc[0]};
-        if (grid_reduce<1, kSThreads>(v, a.scr, TKT_STENCIL) && threadIdx.x == 0) {
+        if (grid_reduce<1, kSThreads>(v, a.scr, TKT_STENCIL, p2p) && threadIdx.x == 0) {
             PcgState* st = a.st;
             if (a.part == 1) {
                 st->sigma_part = v[0];  // completed by the edge launch
             } else {
+                double ff, rr, rho1;
+                a_globals(a, kit, ff, rr, rho1);
                 st->pend_sigma = a.part == 2 ? st->sigma_part + v[0] : v[0];
-                a.rr_hist[kit - 1] = st->pend_rr;
-                a.rho_hist[kit - 1] = st->pend_rho;
-                st->rho_prev = st->pend_rho;  // rho_{k-1}, read as rho_{(k+1)-2} by A(k+1)
+                a.rr_hist[kit - 1] = rr;
+                a.rho_hist[kit - 1] = rho1;
+                st->rho_prev = rho1;  // rho_{k-1}, read as rho_{(k+1)-2} by A(k+1)
+                if (p2p) {
+                    // globals for B(k) (alpha, breakdown report) and later A's
+                    st->pend_rho = rho1;
+                    st->pend_rr = rr;
+                    st->pend_ff = ff;
+                    p2p_publish(a.p2p, MB_A, p2p_seq(st->epoch, kit), v, 1);
+                }
             }
         }
     }
@@ -699,7 +814,18 @@ __global__ void __launch_bounds__(kThreads) k_pcg_b(const StreamArgs a) {
     }
     const Geo& g = a.g;
     const int kit = __ldcg(&vst->k);
-    const double sigma = __ldcg(&vst->pend_sigma);
+    const bool p2p = a.p2p.nranks > 0;
+    double sigma = __ldcg(&vst->pend_sigma);
+    if (p2p) {  // the allreduce of A(k): sigma_k (thread 0 waits, the block reads)
+        __shared__ double sh_sigma;
+        if (threadIdx.x == 0) {
+            double v[1];
+            p2p_gather_one<1>(a.p2p, MB_A, p2p_seq(__ldcg(&vst->epoch), kit), v);
+            sh_sigma = v[0];
+        }
+        __syncthreads();
+        sigma = sh_sigma;
+    }
     const bool brk = !(sigma > 0.0) || !isfinite(sigma);
     const double alpha = __ldcg(&vst->pend_rho) / sigma;  // rho_{k-1} / sigma_k
     double acc[2] = {0.0, 0.0};
@@ -740,7 +866,7 @@ __global__ void __launch_bounds__(kThreads) k_pcg_b(const StreamArgs a) {
         }
     }
 reduce:
-    if (grid_reduce<2>(acc, a.scr, TKT_B) && threadIdx.x == 0) {
+    if (grid_reduce<2>(acc, a.scr, TKT_B, p2p) && threadIdx.x == 0) {
         PcgState* st = a.st;
         if (brk) {
             st->iters = kit;
@@ -760,6 +886,7 @@ reduce:
             st->pend_rho = acc[0];
             st->pend_rr = acc[1];
             st->k = kit + 1;
+            if (p2p) p2p_publish(a.p2p, MB_B, p2p_seq(st->epoch, kit), acc, 2);
         }
     }
 }

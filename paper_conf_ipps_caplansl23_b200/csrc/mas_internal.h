@@ -41,8 +41,30 @@ struct Geo {
 // (multi-GPU seams).  ghost == nullptr at a global boundary or on one GPU.
 struct Halo {
     const double* in;   // [ncomp][nl][nt][np]
-    const double* glo;  // [ncomp][nt][np]  copy of global plane i0-1
-    const double* ghi;  // [ncomp][nt][np]  copy of global plane i0+nl
+    const double* glo;  // plane i0-1 of component 0: a ghost copy [ncomp][nt][np], or (P2P
+                        // transport) the last plane of rank-1's own array, read over NVLink
+    const double* ghi;  // plane i0+nl of component 0 (ghost copy, or rank+1's first plane)
+    int slo, shi;       // component strides of glo / ghi (plane for a ghost copy,
+                        // nl_neighbour * plane for a neighbour's array)
+};
+
+// ---------------------------------------------------------------------------
+// P2P transport (multi-GPU over NVLink / NVSwitch peer memory): the two
+// per-iteration scalar allreduces become one-shot mailbox writes fused into
+// the reducing kernel's last block, and kernel A reads the r-neighbours'
+// edge planes in place (no seam exchange).  See DESIGN.md §7.
+// ---------------------------------------------------------------------------
+struct Mail {                 // one rank's published partial sums
+    double v[4];
+    unsigned long long seq;   // (epoch << 32) | (k + 1) once v is valid
+    unsigned long long pad[3];
+};
+enum { MB_A = 0, MB_B = 1 };  // mailbox slots: A(k) -> B(k) (sigma); B(k)/init -> A(k+1)
+struct P2P {
+    Mail* own;                // this rank's mailbox [2 slots][nranks]
+    Mail* const* peers;       // [nranks] every rank's mailbox (device-visible pointers)
+    int nranks;               // 0: transport off
+    int rank;
 };
 
 // Device-resident PCG state (one per op).  "pend_*" are the current
@@ -63,6 +85,7 @@ struct PcgState {
     int iters;
     int status;         // mas_status_t
     int pad;
+    unsigned long long epoch;  // P2P: solve counter (mailbox sequence numbers)
 };
 
 struct Scratch {
@@ -94,6 +117,7 @@ struct StencilArgs {
     int part;                 // 0: all work items; 1: interior chunks; 2: the two edge chunks
                               // (interior runs while the seams are in flight)
     unsigned long long cond;  // CUDA graph while-loop handle (0: not in a graph)
+    P2P p2p;                  // RESID / PCGA: mailbox transport (nranks == 0: off)
 };
 
 struct StreamArgs {  // kernel B
@@ -109,6 +133,7 @@ struct StreamArgs {  // kernel B
     Scratch scr;
     int* host_flag;
     unsigned long long cond;
+    P2P p2p;
 };
 
 // launchers (kernels.cu)

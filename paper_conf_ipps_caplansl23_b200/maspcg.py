@@ -24,7 +24,8 @@ MAS_POLE_NORTH, MAS_POLE_SOUTH = 1, 2
 # every symbol include/mas_pcg.h declares
 ABI_SYMBOLS = ("mas_comm_unique_id", "mas_partition", "mas_grid_create", "mas_grid_local_extent",
                "mas_grid_destroy", "mas_op_setup", "mas_op_update", "mas_op_apply", "mas_op_diag",
-               "mas_op_dirichlet_rhs", "mas_op_dot", "mas_pcg_solve", "mas_op_launch_count",
+               "mas_op_dirichlet_rhs", "mas_op_dot", "mas_pcg_solve", "mas_op_enable_p2p",
+               "mas_op_transport", "mas_op_launch_count",
                "mas_op_set_profiling", "mas_op_kernel_times", "mas_op_destroy", "mas_status_string", "mas_last_error", "mas_version")
 
 
@@ -63,6 +64,8 @@ def lib() -> C.CDLL:
             "mas_op_dirichlet_rhs": (_i, [_vp, _vp, _vp, _vp, _vp]),
             "mas_op_dot": (_i, [_vp, _vp, _vp, _vp, _vp]),
             "mas_pcg_solve": (_i, [_vp, _vp, _vp, _d, _i, _vp, _vp, _vp, _vp]),
+            "mas_op_enable_p2p": (_i, [_vp, _vp]),
+            "mas_op_transport": (_i, [_vp]),
             "mas_op_launch_count": (C.c_longlong, [_vp]),
             "mas_op_set_profiling": (_i, [_vp, _i]),
             "mas_op_kernel_times": (_i, [_vp, _vp, _vp, _vp]),
@@ -214,6 +217,15 @@ def mas_pcg_solve(op: int, rhs, x, tol: float, maxit: int, want_hist: bool = Fal
     return s, it.value, rel.value, hist
 
 
+def mas_op_enable_p2p(op: int, stream=None) -> None:
+    """Collective: the op's PCG loop uses the P2P (NVLink peer-memory) transport."""
+    _check(lib().mas_op_enable_p2p(op, _stream(stream)), "mas_op_enable_p2p")
+
+
+def mas_op_transport(op: int) -> str:
+    return {0: "nccl", 1: "p2p"}.get(int(lib().mas_op_transport(op)), "invalid")
+
+
 def mas_op_launch_count(op: int) -> int:
     return int(lib().mas_op_launch_count(op))
 
@@ -289,6 +301,13 @@ class Operator:
 
     def solve(self, rhs, x, tol, maxit, want_hist=False, stream=None):
         return mas_pcg_solve(self.h, rhs, x, tol, maxit, want_hist, stream)
+
+    def enable_p2p(self, stream=None):
+        mas_op_enable_p2p(self.h, stream)
+
+    @property
+    def transport(self):
+        return mas_op_transport(self.h)
 
     def set_profiling(self, on=True):
         mas_op_set_profiling(self.h, on)

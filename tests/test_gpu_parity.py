@@ -233,3 +233,29 @@ def test_deterministic_repeat(mp):
     b = gpu_solve(mp, prob)
     assert a[2] == b[2]
     np.testing.assert_array_equal(a[1], b[1])
+
+
+@pytest.mark.parametrize("mk", ["viscosity", "conduction"])
+def test_p2p_transport_one_rank_is_bitwise_identical(mp, mk):
+    """mas_op_enable_p2p on one GPU: the mailbox allreduce runs against the
+    rank itself inside the CUDA-graph loop (0 + v = v exactly), so the solve
+    must be bit-identical to the plain path, over repeated solves (epochs)."""
+    prob = (W.viscosity_problem(12, 16, 64) if mk == "viscosity" else
+            W.conduction_problem(10, 16, 32))
+    st, xd, it, rel, hist, op = gpu_solve(mp, prob)
+    op.enable_p2p()
+    assert op.transport == "p2p"
+    f = dev(prob.f)
+    op.dirichlet_rhs(None if prob.ub_inner is None else dev(prob.ub_inner), None, f)
+    for _ in range(3):
+        x = dev(prob.x0)
+        st2, it2, rel2, hist2 = op.solve(f, x, prob.tol, prob.maxit, True)
+        assert (st2, it2, rel2) == (st, it, rel)
+        np.testing.assert_array_equal(host(x), xd)
+        np.testing.assert_array_equal(np.asarray(hist2), np.asarray(hist))
+    # fixed-iteration and zero-rhs paths through the mailbox
+    x = dev(prob.x0)
+    assert op.solve(f, x, 0.0, 5)[:2] == (mp.MAS_NOT_CONVERGED, 5)
+    z = torch.zeros_like(f)
+    st3, it3, _, _ = op.solve(z, x, prob.tol, prob.maxit)
+    assert (st3, it3) == (mp.MAS_OK, 0) and float(x.abs().max()) == 0.0

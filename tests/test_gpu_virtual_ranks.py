@@ -31,7 +31,8 @@ def mp():
     return maspcg
 
 
-def run_ranks(mp, prob, P, x_apply, want_solve=True, maxit=None, tol=None):
+def run_ranks(mp, prob, P, x_apply, want_solve=True, maxit=None, tol=None, p2p=False,
+              solves=1):
     _key[0] += 1
     vid = mp.virtual_ranks_id(_key[0])
     res, errs = {}, []
@@ -47,6 +48,9 @@ def run_ranks(mp, prob, P, x_apply, want_solve=True, maxit=None, tol=None):
                 d = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()
                 op = mp.Operator(g, prob.ncomp, d(prob.kappa[sl]), d(prob.c[sl]), prob.bc_inner,
                                  prob.bc_outer)
+                if p2p:
+                    op.enable_p2p()
+                    assert op.transport == "p2p"
                 y = torch.empty((prob.ncomp, nl) + prob.shape[1:], dtype=torch.float64, device="cuda")
                 op.apply(d(x_apply[:, sl]), y)
                 out = {"i0": i0, "nl": nl, "y": None, "dot": None}
@@ -57,11 +61,13 @@ def run_ranks(mp, prob, P, x_apply, want_solve=True, maxit=None, tol=None):
                     f = d(prob.f[:, sl])
                     ubi = d(prob.ub_inner) if prob.ub_inner is not None else None
                     op.dirichlet_rhs(ubi, None, f)
-                    x = d(prob.x0[:, sl])
-                    st, it, rel, hist = op.solve(f, x, prob.tol if tol is None else tol,
-                                                 prob.maxit if maxit is None else maxit, True)
-                    torch.cuda.current_stream().synchronize()
-                    out.update(st=st, it=it, rel=rel, x=x.cpu().numpy(), launches=op.launch_count)
+                    for _ in range(solves):  # repeated solves: mailbox epochs
+                        x = d(prob.x0[:, sl])
+                        st, it, rel, hist = op.solve(f, x, prob.tol if tol is None else tol,
+                                                     prob.maxit if maxit is None else maxit, True)
+                        torch.cuda.current_stream().synchronize()
+                    out.update(st=st, it=it, rel=rel, x=x.cpu().numpy(), launches=op.launch_count,
+                               hist=np.asarray(hist))
                 op.close()
                 g.close()
                 res[r] = out
@@ -125,6 +131,60 @@ def test_virtual_ranks_conduction_dirichlet_and_fixed_iterations(mp, oracle_mod)
     prob = W.conduction_problem(10, 24, 32)
     x = W.random_field((1,) + prob.shape, 43)
     out = run_ranks(mp, prob, 3, x, tol=0.0, maxit=25)
+    rc, xo, ito, _, _ = oracle_mod.solve_problem(prob, tol=0.0, maxit=25)
+    assert all(r["st"] == mp.MAS_NOT_CONVERGED and r["it"] == 25 for r in out)
+    xg = np.concatenate([r["x"] for r in out], axis=1)
+    V = oracle_mod.Oracle.for_problem(prob).volumes()[None]
+    assert math.sqrt((V * (xg - xo) ** 2).sum() / (V * xo ** 2).sum()) <= 1e-10
+
+
+# ---------------------------------------------------------------------------
+# P2P transport (mas_op_enable_p2p): mailbox allreduce fused into the reducing
+# kernels' last blocks and in-place reads of the neighbours' edge planes.  On
+# one GPU the virtual ranks' buffers are plain device pointers of one process;
+# the kernels run exactly the code of the multi-GPU path.
+# ---------------------------------------------------------------------------
+@pytest.mark.parametrize("P", [2, 3, 4])
+def test_virtual_ranks_p2p_transport_matches_nccl_path_bitwise(mp, oracle_mod, P):
+    """Both transports sum the ranks' partials in rank order, so the P2P loop
+    must reproduce the NCCL-placement loop bit for bit (and the oracle).  Slabs
+    of 8 planes: the NCCL loop does not split kernel A (which would change the
+    block-partial summation order)."""
+    prob = W.viscosity_problem(8 * P, 16, 64, warm=False)
+    x = W.random_field((3,) + prob.shape, 45)
+    ref = run_ranks(mp, prob, P, x)
+    out = run_ranks(mp, prob, P, x, p2p=True, solves=2)
+    assert [r["it"] for r in out] == [r["it"] for r in ref]
+    assert all(r["st"] == mp.MAS_OK for r in out)
+    for a, b in zip(out, ref):
+        assert np.array_equal(a["x"], b["x"])
+        assert np.array_equal(a["hist"], b["hist"])
+    rc, xo, ito, _, _ = oracle_mod.solve_problem(prob)
+    assert abs(out[0]["it"] - ito) <= 1
+    V = oracle_mod.Oracle.for_problem(prob).volumes()[None]
+    xg = np.concatenate([r["x"] for r in out], axis=1)
+    assert math.sqrt((V * (xg - xo) ** 2).sum() / (V * xo ** 2).sum()) <= 1e-10
+    # no seam split: one kernel A and one kernel B per iteration
+    assert all(r["launches"] <= 2 * r["it"] + 6 for r in out)
+
+
+@pytest.mark.parametrize("P", [2, 4])
+def test_virtual_ranks_p2p_long_slabs(mp, oracle_mod, P):
+    prob = W.viscosity_problem(17 * P + 1, 16, 64, warm=False)
+    x = W.random_field((3,) + prob.shape, 46)
+    out = run_ranks(mp, prob, P, x, p2p=True)
+    rc, xo, ito, _, _ = oracle_mod.solve_problem(prob)
+    its = {r["it"] for r in out}
+    assert len(its) == 1 and abs(its.pop() - ito) <= 1
+    V = oracle_mod.Oracle.for_problem(prob).volumes()[None]
+    xg = np.concatenate([r["x"] for r in out], axis=1)
+    assert math.sqrt((V * (xg - xo) ** 2).sum() / (V * xo ** 2).sum()) <= 1e-10
+
+
+def test_virtual_ranks_p2p_dirichlet_fixed_iterations(mp, oracle_mod):
+    prob = W.conduction_problem(10, 24, 32)
+    x = W.random_field((1,) + prob.shape, 43)
+    out = run_ranks(mp, prob, 3, x, tol=0.0, maxit=25, p2p=True)
     rc, xo, ito, _, _ = oracle_mod.solve_problem(prob, tol=0.0, maxit=25)
     assert all(r["st"] == mp.MAS_NOT_CONVERGED and r["it"] == 25 for r in out)
     xg = np.concatenate([r["x"] for r in out], axis=1)
