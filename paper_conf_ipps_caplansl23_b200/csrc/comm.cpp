@@ -16,7 +16,10 @@
 // key.  It is a test transport, not a performance path.
 #include <nccl.h>
 
+#include <chrono>
 #include <condition_variable>
+#include <cstdio>
+#include <thread>
 #include <cstring>
 #include <map>
 #include <mutex>
@@ -67,9 +70,12 @@ struct Comm {
     int nranks = 1, rank = 0;
     VGroup* vg = nullptr;
     unsigned long long vkey = 0;
+    std::string hdir;                // host-exchange transport: shared directory
+    long hseq = 0;                   // host-exchange call counter
 };
 
 static const char kVirtMagic[8] = {'M', 'A', 'S', 'V', 'I', 'R', 'T', 0};
+static const char kHostMagic[8] = {'M', 'A', 'S', 'H', 'O', 'S', 'T', 0};
 
 static mas_status_t nccl_fail(ncclResult_t r, const char* what) {
     set_last_error(std::string(what) + ": " + ncclGetErrorString(r));
@@ -79,6 +85,103 @@ static mas_status_t nccl_fail(ncclResult_t r, const char* what) {
 static mas_status_t cuda_fail(cudaError_t e, const char* what) {
     set_last_error(std::string(what) + ": " + cudaGetErrorString(e));
     return MAS_ERR_CUDA;
+}
+
+// ---------------------------------------------------------------------------
+// host-exchange transport (tests): P processes sharing ONE GPU exchange the
+// setup-time collectives through files in a shared directory; everything
+// else (CUDA IPC mappings, the P2P kernels) is the multi-GPU code.  NCCL
+// cannot run two ranks on one device, so this is how the cross-process P2P
+// path is exercised on a single B200.  Selected by a mas_dist_t.nccl_id of
+// "MASHOST\0" + a NUL-terminated directory path.  Not a performance path.
+// ---------------------------------------------------------------------------
+static mas_status_t h_exchange(Comm* c, const void* mine, size_t n, std::vector<unsigned char>& all) {
+    const long seq = ++c->hseq;
+    auto name = [&](int r) { return c->hdir + "/x" + std::to_string(seq) + "." + std::to_string(r); };
+    {
+        const std::string tmp = name(c->rank) + ".tmp";
+        FILE* f = fopen(tmp.c_str(), "wb");
+        if (!f || fwrite(mine, 1, n, f) != n) {
+            if (f) fclose(f);
+            set_last_error("host exchange: cannot write " + tmp);
+            return MAS_ERR_NCCL;
+        }
+        fclose(f);
+        if (rename(tmp.c_str(), name(c->rank).c_str()) != 0) {
+            set_last_error("host exchange: rename failed");
+            return MAS_ERR_NCCL;
+        }
+    }
+    all.assign(n * c->nranks, 0);
+    for (int r = 0; r < c->nranks; r++) {
+        const auto t0 = std::chrono::steady_clock::now();
+        for (;;) {
+            FILE* f = fopen(name(r).c_str(), "rb");
+            if (f) {
+                const size_t got = fread(all.data() + r * n, 1, n, f);
+                fclose(f);
+                if (got == n) break;
+            }
+            if (std::chrono::steady_clock::now() - t0 > std::chrono::seconds(120)) {
+                set_last_error("host exchange: timed out waiting for rank " + std::to_string(r));
+                return MAS_ERR_NCCL;
+            }
+            std::this_thread::sleep_for(std::chrono::microseconds(200));
+        }
+    }
+    return MAS_OK;
+}
+
+static mas_status_t h_allreduce(Comm* c, double* buf, int n, cudaStream_t s) {
+    double mine[8] = {0};
+    cudaError_t e;
+    if ((e = cudaMemcpyAsync(mine, buf, n * sizeof(double), cudaMemcpyDeviceToHost, s)) != cudaSuccess ||
+        (e = cudaStreamSynchronize(s)) != cudaSuccess)
+        return cuda_fail(e, "host allreduce");
+    std::vector<unsigned char> all;
+    mas_status_t st = h_exchange(c, mine, sizeof(mine), all);
+    if (st != MAS_OK) return st;
+    double sum[8] = {0};
+    for (int r = 0; r < c->nranks; r++)
+        for (int t = 0; t < n; t++) sum[t] += reinterpret_cast<const double*>(all.data() + r * sizeof(mine))[t];
+    if ((e = cudaMemcpyAsync(buf, sum, n * sizeof(double), cudaMemcpyHostToDevice, s)) != cudaSuccess ||
+        (e = cudaStreamSynchronize(s)) != cudaSuccess)
+        return cuda_fail(e, "host allreduce");
+    return MAS_OK;
+}
+
+static mas_status_t h_seams(Comm* c, const double* in, int ncomp, int nl, long long plane, double* glo,
+                            double* ghi, cudaStream_t s) {
+    // payload: [first plane, last plane] of every component
+    const size_t pb = sizeof(double) * plane;
+    std::vector<unsigned char> mine(2 * ncomp * pb);
+    cudaError_t e;
+    for (int m = 0; m < ncomp; m++) {
+        const double* base = in + (long long)m * nl * plane;
+        if ((e = cudaMemcpyAsync(mine.data() + (2 * m) * pb, base, pb, cudaMemcpyDeviceToHost, s)) !=
+                cudaSuccess ||
+            (e = cudaMemcpyAsync(mine.data() + (2 * m + 1) * pb, base + (long long)(nl - 1) * plane, pb,
+                                 cudaMemcpyDeviceToHost, s)) != cudaSuccess)
+            return cuda_fail(e, "host seams");
+    }
+    if ((e = cudaStreamSynchronize(s)) != cudaSuccess) return cuda_fail(e, "host seams");
+    std::vector<unsigned char> all;
+    mas_status_t st = h_exchange(c, mine.data(), mine.size(), all);
+    if (st != MAS_OK) return st;
+    for (int m = 0; m < ncomp; m++) {
+        if (c->rank > 0) {  // rank-1's last plane
+            const unsigned char* src = all.data() + (c->rank - 1) * mine.size() + (2 * m + 1) * pb;
+            if ((e = cudaMemcpyAsync(glo + m * plane, src, pb, cudaMemcpyHostToDevice, s)) != cudaSuccess)
+                return cuda_fail(e, "host seams");
+        }
+        if (c->rank < c->nranks - 1) {  // rank+1's first plane
+            const unsigned char* src = all.data() + (c->rank + 1) * mine.size() + (2 * m) * pb;
+            if ((e = cudaMemcpyAsync(ghi + m * plane, src, pb, cudaMemcpyHostToDevice, s)) != cudaSuccess)
+                return cuda_fail(e, "host seams");
+        }
+    }
+    if ((e = cudaStreamSynchronize(s)) != cudaSuccess) return cuda_fail(e, "host seams");
+    return MAS_OK;
 }
 
 mas_status_t comm_unique_id(unsigned char out[128]) {
@@ -137,6 +240,21 @@ mas_status_t comm_create(const mas_dist_t* d, Comm** out) {
     Comm* c = new Comm();
     c->nranks = d->nranks;
     c->rank = d->rank;
+    if (memcmp(d->nccl_id, kHostMagic, 8) == 0) {
+        char path[121];
+        memcpy(path, d->nccl_id + 8, 120);
+        path[120] = 0;
+        c->hdir = path;
+        std::vector<unsigned char> all;
+        const unsigned char one = 1;
+        mas_status_t s = h_exchange(c, &one, 1, all);  // collective create
+        if (s != MAS_OK) {
+            delete c;
+            return s;
+        }
+        *out = c;
+        return MAS_OK;
+    }
     if (memcmp(d->nccl_id, kVirtMagic, 8) == 0) {
         mas_status_t s = vgroup_join(d, c);
         if (s != MAS_OK) {
@@ -218,6 +336,7 @@ static mas_status_t v_allreduce(Comm* c, double* buf, int n, cudaStream_t s) {
 mas_status_t comm_allreduce(Comm* c, double* buf, int n, cudaStream_t s) {
     if (!c || c->nranks == 1) return MAS_OK;
     if (c->vg) return v_allreduce(c, buf, n, s);
+    if (!c->hdir.empty()) return h_allreduce(c, buf, n, s);
     ncclResult_t r = ncclAllReduce(buf, buf, n, ncclFloat64, ncclSum, c->nccl, s);
     return r == ncclSuccess ? MAS_OK : nccl_fail(r, "ncclAllReduce");
 }
@@ -263,6 +382,7 @@ mas_status_t comm_seams(Comm* c, const double* in, int ncomp, int nl, long long 
                         double* ghi, cudaStream_t s) {
     if (!c || c->nranks == 1) return MAS_OK;
     if (c->vg) return v_seams(c, in, ncomp, nl, plane, glo, ghi, s);
+    if (!c->hdir.empty()) return h_seams(c, in, ncomp, nl, plane, glo, ghi, s);
     const long long Nl = (long long)nl * plane;
     ncclResult_t r = ncclGroupStart();
     if (r != ncclSuccess) return nccl_fail(r, "ncclGroupStart");
@@ -294,6 +414,12 @@ mas_status_t comm_allgather_bytes(Comm* c, const void* mine, void* all, size_t n
     if (!c || c->nranks == 1) {
         memcpy(all, mine, n);
         return MAS_OK;
+    }
+    if (!c->hdir.empty()) {
+        std::vector<unsigned char> v;
+        mas_status_t st = h_exchange(c, mine, n, v);
+        if (st == MAS_OK) memcpy(all, v.data(), n * c->nranks);
+        return st;
     }
     if (c->vg) {
         VGroup* g = c->vg;
@@ -345,6 +471,12 @@ mas_status_t comm_barrier(Comm* c, cudaStream_t s) {
         if (cudaStreamSynchronize(s) != cudaSuccess) return MAS_ERR_CUDA;
         c->vg->barrier();
         return MAS_OK;
+    }
+    if (!c->hdir.empty()) {
+        if (cudaStreamSynchronize(s) != cudaSuccess) return MAS_ERR_CUDA;
+        std::vector<unsigned char> all;
+        const unsigned char one = 1;
+        return h_exchange(c, &one, 1, all);
     }
     double* d = nullptr;
     if (cudaMallocAsync(&d, sizeof(double), s) != cudaSuccess) return MAS_ERR_CUDA;

@@ -135,6 +135,16 @@ def virtual_ranks_id(key: int) -> bytes:
     return b"MASVIRT\0" + int(key).to_bytes(8, "little") + bytes(112)
 
 
+def host_exchange_id(directory: str) -> bytes:
+    """mas_dist_t.nccl_id selecting the "host exchange" test transport: P
+    processes on ONE GPU exchange the setup-time collectives through files in
+    `directory` (comm.cpp); the P2P loop then runs across real processes."""
+    d = os.fsencode(directory)
+    if len(d) > 119:
+        raise ValueError("directory path too long (max 119 bytes)")
+    return b"MASHOST\0" + d + bytes(120 - len(d))
+
+
 def mas_grid_create(r_node, r_half, t_node, t_half, p_node, p_half, pole_flags=3,
                     periodic_phi=1, dist: Optional[tuple] = None) -> int:
     """dist = (nranks, rank, nccl_id_bytes) or None.  Returns the handle."""
