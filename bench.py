@@ -202,6 +202,8 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--cpu-iters", type=int, default=3)
+    ap.add_argument("--ptheta", type=int, default=1,
+                    help="(r, theta) decomposition: theta bands per r-slab (must divide --gpus)")
     ap.add_argument("--transport", default="auto", choices=["auto", "p2p", "nccl"],
                     help="multi-GPU PCG loop: P2P (NVLink peer memory: mailbox allreduce + "
                          "in-place seam reads, one CUDA graph per rank) or NCCL; auto = P2P "
@@ -233,9 +235,10 @@ def main():
         obj = [M.mas_comm_unique_id() if rank == 0 else None]
         dist.broadcast_object_list(obj, src=0)
         distinfo = (world, rank, obj[0])
-    grid = M.Grid(prob.mesh, distinfo)
-    i0, nl = grid.i0, grid.nl
-    sl = slice(i0, i0 + nl)
+    grid = M.Grid(prob.mesh, distinfo, ptheta=args.ptheta if world > 1 else 1)
+    i0, nl, j0, ntl = grid.i0, grid.nl, grid.j0, grid.ntl
+    sl = (slice(i0, i0 + nl), slice(j0, j0 + ntl))
+    slc = (slice(None),) + sl
     nc = prob.ncomp
 
     def to_dev(a):
@@ -243,8 +246,8 @@ def main():
 
     kappa = to_dev(prob.kappa[sl])
     cmass = to_dev(prob.c[sl])
-    f = to_dev(prob.f[:, sl])
-    x0 = to_dev(prob.x0[:, sl])
+    f = to_dev(prob.f[slc])
+    x0 = to_dev(prob.x0[slc])
     x = x0.clone()
     op = M.Operator(grid, nc, kappa, cmass, prob.bc_inner, prob.bc_outer)
     transport = "single-gpu"
@@ -258,8 +261,8 @@ def main():
                 if args.transport == "p2p":
                     raise
                 transport = f"nccl (p2p unavailable: {e})"
-    ubi = to_dev(prob.ub_inner) if prob.ub_inner is not None else None
-    ubo = to_dev(prob.ub_outer) if prob.ub_outer is not None else None
+    ubi = to_dev(prob.ub_inner[:, j0:j0 + ntl]) if prob.ub_inner is not None else None
+    ubo = to_dev(prob.ub_outer[:, j0:j0 + ntl]) if prob.ub_outer is not None else None
     rhs = f.clone()
     if ubi is not None or ubo is not None:
         op.dirichlet_rhs(ubi, ubo, rhs)
@@ -325,7 +328,7 @@ def main():
     # roofline of the dominant kernel (kernel A), algorithmic bytes / its
     # average CUDA-event duration over the timed region
     cells = nr * nt * np_
-    cells_local = nl * nt * np_
+    cells_local = nl * ntl * np_
     a_b, b_b = alg_bytes_per_cell(nc)
     a_ms = statistics.mean(ka)
     b_ms = statistics.mean(kb)
@@ -344,7 +347,7 @@ def main():
     if not args.no_e2e:
         pin = lambda a: torch.from_numpy(np.ascontiguousarray(a)).pin_memory()
         hk, hc, hf, hx0 = pin(prob.kappa[sl]), pin(prob.c[sl]), rhs.cpu().pin_memory(), \
-            pin(prob.x0[:, sl])
+            pin(prob.x0[slc])
         hx = hx0.clone().pin_memory()
         ksteps = max(1, min(args.steps, 2))
         torch.cuda.synchronize()
@@ -386,7 +389,9 @@ def main():
             "dtype": "f64", "data": "synthetic",
             "config": {"workload": args.config, "grid": [nr, nt, np_], "ncomp": nc,
                        "cells": cells, "tol": args.tol, "iters_per_solve": iters_per_solve,
-                       "parallelism": f"r-slab x{world}", "transport": transport,
+                       "parallelism": (f"r-slab x{world}" if args.ptheta == 1 or world == 1 else
+                                       f"(r,theta) {world // args.ptheta}x{args.ptheta}"),
+                       "transport": transport,
                        "l2": "inputs > L2 (268 MB per field vs 126 MB); no flush",
                        "step": "mas_op_update + x:=x0 + mas_pcg_solve"},
             "roofline": {"bound": "hbm", "kernel": "k_stencil<PCGA> (kernel A)",

@@ -100,6 +100,32 @@ MAS_API mas_status_t mas_grid_create(int nr, int nt, int np,
                              int pole_flags, int periodic_phi,
                              const mas_dist_t* dist, mas_grid_t** out);
 
+/* (r, theta) decomposition (the north_star's "slabs in
+ * r (and in theta where needed)"; the paper's domain decomposition with
+ * halo exchanges).  Same mesh arguments and checks as
+ * mas_grid_create; dist->nranks = pr * ptheta with ptheta >= 1 dividing it.
+ * Rank = rr * ptheta + rt (theta fastest): rank rt of r-slab rr owns r-planes
+ * [i0, i0 + nr_local) (the partition of nr over pr) and theta rows
+ * [j0, j0 + nt_local) (the partition of nt over ptheta), every phi.  Every
+ * per-cell array of every later call on this grid is then the local block
+ * [comp][nr_local][nt_local][np].  Needs nr >= pr and nt >= ptheta.
+ * ptheta == 1 is mas_grid_create.  The theta-ghost rows are exchanged by the
+ * library: packed copies over the grid's communicator at setup / apply / init
+ * and in the NCCL loop; read in place from the theta neighbours' arrays by
+ * kernel A under the P2P transport (mas_op_enable_p2p).
+ * Errors: as mas_grid_create; MAS_ERR_ARG if ptheta does not divide nranks. */
+MAS_API mas_status_t mas_grid_create_2d(int nr, int nt, int np,
+                             const double* r_node, const double* r_half,
+                             const double* t_node, const double* t_half,
+                             const double* p_node, const double* p_half,
+                             int pole_flags, int periodic_phi,
+                             const mas_dist_t* dist, int ptheta, mas_grid_t** out);
+
+/* This rank's block of a 2-D decomposition: r-planes [i0, i0 + nr_local),
+ * theta rows [j0, j0 + nt_local). */
+MAS_API mas_status_t mas_grid_local_extent_2d(const mas_grid_t* g, int* i0, int* nr_local,
+                                              int* j0, int* nt_local);
+
 /* The r-slab partition without a grid (host only, no device work): rank
  * owns nr/nranks + (rank < nr % nranks) planes starting at *i0 (SURVEY.md
  * §8(e)).  Lets a caller size its slab buffers before mas_grid_create.

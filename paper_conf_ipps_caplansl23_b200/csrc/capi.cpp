@@ -132,6 +132,15 @@ struct mas_op {
     const double* nb_p[2][2] = {{nullptr, nullptr}, {nullptr, nullptr}};  // [parity][lo/hi]
     int nb_nl[2] = {0, 0};             // their slab sizes
     unsigned long long epoch = 0;      // solves so far (mailbox sequence numbers)
+    // (r, theta) decomposition (NEXT-3): theta-ghost rows, packed [2][ncomp][nl][np]
+    int tlo = -1, thi = -1;            // theta-neighbour ranks (-1: pole / wall side)
+    double *kgt = nullptr, *dgt = nullptr;       // kappa, 1/D rows (static, per op_load)
+    double *xgt = nullptr, *rgt = nullptr;       // x (apply / init), r (NCCL loop)
+    double *pgt[2] = {nullptr, nullptr};         // p_{k-1} (NCCL loop)
+    double* tpack = nullptr;                     // pack buffer of the own first/last rows
+    const double* nbt_r[2] = {nullptr, nullptr};                         // P2P: theta nbrs' r
+    const double* nbt_p[2][2] = {{nullptr, nullptr}, {nullptr, nullptr}};  // [parity][lo/hi]
+    int nbt_ntl[2] = {0, 0};                     // their theta rows
 };
 
 extern "C" {
@@ -162,14 +171,24 @@ mas_status_t mas_grid_create(int nr, int nt, int np, const double* r_node, const
                              const double* t_node, const double* t_half, const double* p_node,
                              const double* p_half, int pole_flags, int periodic_phi,
                              const mas_dist_t* dist, mas_grid_t** out) {
+    return mas_grid_create_2d(nr, nt, np, r_node, r_half, t_node, t_half, p_node, p_half,
+                              pole_flags, periodic_phi, dist, 1, out);
+}
+
+mas_status_t mas_grid_create_2d(int nr, int nt, int np, const double* r_node, const double* r_half,
+                                const double* t_node, const double* t_half, const double* p_node,
+                                const double* p_half, int pole_flags, int periodic_phi,
+                                const mas_dist_t* dist, int ptheta, mas_grid_t** out) {
     if (!out) return arg_error("null out");
     *out = nullptr;
     const int nranks = dist ? dist->nranks : 1;
     const int rank = dist ? dist->rank : 0;
     if (dist && (rank < 0 || rank >= nranks)) return arg_error("bad rank");
+    if (ptheta < 1 || nranks % ptheta) return arg_error("ptheta must divide nranks");
+    const int pr = nranks / ptheta;
     std::string why;
     if (!validate_mesh(nr, nt, np, r_node, r_half, t_node, t_half, p_node, p_half, pole_flags,
-                       periodic_phi, nranks, &why))
+                       periodic_phi, pr, ptheta, &why))
         return arg_error(why);
     mas_grid* g = new (std::nothrow) mas_grid();
     if (!g) return MAS_ERR_NOMEM;
@@ -179,7 +198,12 @@ mas_status_t mas_grid_create(int nr, int nt, int np, const double* r_node, const
     g->rF.assign(r_node, r_node + nr + 1); g->rC.assign(r_half, r_half + nr);
     g->tF.assign(t_node, t_node + nt + 1); g->tC.assign(t_half, t_half + nt);
     g->pF.assign(p_node, p_node + np + 1); g->pC.assign(p_half, p_half + np);
-    partition(nr, nranks, rank, &g->i0, &g->nl);
+    g->ptheta = ptheta;
+    g->pr = pr;
+    g->rrank = rank / ptheta;  // theta fastest in the rank numbering
+    g->trank = rank % ptheta;
+    partition(nr, pr, g->rrank, &g->i0, &g->nl);
+    partition(nt, ptheta, g->trank, &g->j0, &g->ntl);
     build_tables(g);
     if (cudaGetDevice(&g->device) != cudaSuccess) {
         cudaGetLastError();
@@ -221,6 +245,16 @@ mas_status_t mas_grid_local_extent(const mas_grid_t* g, int* i0, int* nr_local) 
     if (!g || !i0 || !nr_local) return arg_error("null argument");
     *i0 = g->i0;
     *nr_local = g->nl;
+    return MAS_OK;
+}
+
+mas_status_t mas_grid_local_extent_2d(const mas_grid_t* g, int* i0, int* nr_local, int* j0,
+                                      int* nt_local) {
+    if (!g || !i0 || !nr_local || !j0 || !nt_local) return arg_error("null argument");
+    *i0 = g->i0;
+    *nr_local = g->nl;
+    *j0 = g->j0;
+    *nt_local = g->ntl;
     return MAS_OK;
 }
 
@@ -270,6 +304,53 @@ static Halo pold_halo(const mas_op* op, int k) {
     return op->p2p ? peer_halo(op, op->p[par], op->nb_p[par][0], op->nb_p[par][1])
                    : halo_of(op, op->p[par], op->g->comm ? op->pg[par] : nullptr, op->ncomp);
 }
+// theta-ghost rows (2-D decomposition): a packed copy, or the theta
+// neighbours' own arrays in place (P2P)
+static TRows packed_rows(const mas_op* op, const double* buf, int ncomp) {
+    TRows t{};
+    if (!buf) return t;
+    const int nl = op->geo.nl, np = op->geo.np;
+    t.lo = op->tlo >= 0 ? buf : nullptr;
+    t.hi = op->thi >= 0 ? buf + (long long)ncomp * nl * np : nullptr;
+    t.cs_lo = t.cs_hi = nl * np;
+    t.ps_lo = t.ps_hi = np;
+    return t;
+}
+static TRows peer_rows(const mas_op* op, const double* lo, const double* hi) {
+    TRows t{};
+    const int nl = op->geo.nl, np = op->geo.np;
+    if (lo) {
+        t.lo = lo + (long long)(op->nbt_ntl[0] - 1) * np;  // its last row
+        t.ps_lo = op->nbt_ntl[0] * np;
+        t.cs_lo = nl * t.ps_lo;
+    }
+    if (hi) {
+        t.hi = hi;  // its first row
+        t.ps_hi = op->nbt_ntl[1] * np;
+        t.cs_hi = nl * t.ps_hi;
+    }
+    return t;
+}
+static TRows r_trows(const mas_op* op) {
+    return op->p2p ? peer_rows(op, op->nbt_r[0], op->nbt_r[1]) : packed_rows(op, op->rgt, op->ncomp);
+}
+static TRows pold_trows(const mas_op* op, int k) {
+    const int par = (k + 1) & 1;
+    return op->p2p ? peer_rows(op, op->nbt_p[par][0], op->nbt_p[par][1])
+                   : packed_rows(op, op->pgt[par], op->ncomp);
+}
+static bool split_theta(const mas_op* op) { return op->g->ptheta > 1; }
+
+// exchange the first / last theta rows of `field` ([ncomp][nl][nt][np]) with
+// the theta neighbours into recv ([2][ncomp][nl][np]); collective
+static mas_status_t tseams(mas_op* op, const double* field, int ncomp, double* recv, cudaStream_t s) {
+    if (!split_theta(op)) return MAS_OK;
+    const size_t n = (size_t)ncomp * op->geo.nl * op->geo.np;
+    CU(launch_pack_rows(op->geo, ncomp, field, op->tpack, s));
+    return comm_exchange(op->g->comm, op->tlo, op->thi, op->tpack, op->tpack + n, recv, recv + n, n, s);
+}
+static int rstride(const mas_op* op) { return op->g->ptheta; }
+
 static P2P p2p_args(const mas_op* op) {
     P2P t{};
     if (op->p2p) {
@@ -293,11 +374,16 @@ static mas_status_t op_load(mas_op* op, const double* kappa, const double* mass,
         CU(cudaMemsetAsync(op->c, 0, bytes, s));
     const long long plane = op->geo.plane;
     if (op->g->comm)
-        ST(comm_seams(op->g->comm, op->kappa, 1, op->g->nl, plane, op->kg, op->kg + plane, s));
+        ST(comm_seams(op->g->comm, op->kappa, 1, op->g->nl, plane, op->kg, op->kg + plane, s,
+                      rstride(op)));
+    ST(tseams(op, op->kappa, 1, op->kgt, s));
     CU(cudaMemsetAsync(op->bad, 0, sizeof(int), s));
-    CU(launch_diag(op->geo, halo_of(op, op->kappa, op->kg, 1), op->c, D_out, op->dinv, op->bad, s));
+    CU(launch_diag(op->geo, halo_of(op, op->kappa, op->kg, 1), packed_rows(op, op->kgt, 1), op->c,
+                   D_out, op->dinv, op->bad, s));
     if (op->g->comm)
-        ST(comm_seams(op->g->comm, op->dinv, 1, op->g->nl, plane, op->dg, op->dg + plane, s));
+        ST(comm_seams(op->g->comm, op->dinv, 1, op->g->nl, plane, op->dg, op->dg + plane, s,
+                      rstride(op)));
+    ST(tseams(op, op->dinv, 1, op->dgt, s));
     int bad = 0;
     CU(cudaMemcpyAsync(&bad, op->bad, sizeof(int), cudaMemcpyDeviceToHost, s));
     CU(cudaStreamSynchronize(s));
@@ -316,6 +402,8 @@ static mas_status_t op_load(mas_op* op, const double* kappa, const double* mass,
 
 static void op_free(mas_op* op) {
     if (!op) return;
+    for (double* p : {op->kgt, op->dgt, op->xgt, op->rgt, op->pgt[0], op->pgt[1], op->tpack})
+        if (p) cudaFree(p);
     for (double* p : {op->kappa, op->c, op->dinv, op->kg, op->dg, op->wR, op->r, op->p[0], op->p[1],
                       op->q, op->rg, op->pg[0], op->pg[1], op->xg, op->stage_a, op->stage_b,
                       op->hist, op->dot_out, op->scr.partials})
@@ -390,6 +478,7 @@ static mas_status_t loop_graph(mas_op* op, StencilArgs a, StreamArgs b) {
             // the body covers an even and an odd iteration: k = 2, 3, 4, ...
             for (int kk = 2; kk <= 3 && e == cudaSuccess; kk++) {
                 a.pold = pold_halo(op, kk);
+                a.tpold = pold_trows(op, kk);
                 a.pnew = op->p[kk & 1];
                 e = launch_stencil(MODE_PCGA, nc, a, op->cap_stream);
                 if (e == cudaSuccess) e = launch_pcg_b(b, op->b_blocks, op->cap_stream);
@@ -438,7 +527,7 @@ mas_status_t mas_op_setup(mas_grid_t* g, int ncomp, const double* kappa, const d
     op->ncomp = ncomp;
     op->bci = bc_r_inner;
     op->bco = bc_r_outer;
-    const int nl = g->nl, nt = g->nt, np = g->np;
+    const int nl = g->nl, nt = g->ntl, np = g->np;  // local block [nl][ntl][np]
     const long long plane = (long long)nt * np;
     op->Nl = (long long)nl * plane;
     if ((long long)ncomp * op->Nl >= (1LL << 31)) {  // the stencil kernels index with 32-bit offsets
@@ -470,6 +559,18 @@ mas_status_t mas_op_setup(mas_grid_t* g, int ncomp, const double* kappa, const d
         TRY(dmalloc(&op->pg[0], 2 * ncomp * plane));
         TRY(dmalloc(&op->pg[1], 2 * ncomp * plane));
         TRY(dmalloc(&op->xg, 2 * ncomp * plane));
+    }
+    if (g->ptheta > 1) {  // theta neighbours: rank -/+ 1 within the same r-slab
+        op->tlo = g->trank > 0 ? g->rank - 1 : -1;
+        op->thi = g->trank < g->ptheta - 1 ? g->rank + 1 : -1;
+        const size_t rows = (size_t)nl * np;
+        TRY(dmalloc(&op->kgt, 2 * rows));
+        TRY(dmalloc(&op->dgt, 2 * rows));
+        TRY(dmalloc(&op->xgt, 2 * ncomp * rows));
+        TRY(dmalloc(&op->rgt, 2 * ncomp * rows));
+        TRY(dmalloc(&op->pgt[0], 2 * ncomp * rows));
+        TRY(dmalloc(&op->pgt[1], 2 * ncomp * rows));
+        TRY(dmalloc(&op->tpack, 2 * ncomp * rows));
     }
     TRY(dmalloc(&op->st, 1));
     TRY(dmalloc(&op->dot_out, 1));
@@ -567,7 +668,8 @@ mas_status_t mas_op_diag(const mas_op_t* op_c, double* D, cudaStream_t stream) {
         Dd = op->stage_b;
     }
     CU(cudaMemsetAsync(op->bad, 0, sizeof(int), stream));
-    CU(launch_diag(op->geo, halo_of(op, op->kappa, op->kg, 1), op->c, Dd, op->dinv, op->bad, stream));
+    CU(launch_diag(op->geo, halo_of(op, op->kappa, op->kg, 1), packed_rows(op, op->kgt, 1), op->c, Dd,
+                   op->dinv, op->bad, stream));
     if (host) {
         CU(cudaMemcpyAsync(D, Dd, op->Nl * sizeof(double), cudaMemcpyDeviceToHost, stream));
         CU(cudaStreamSynchronize(stream));
@@ -591,12 +693,15 @@ mas_status_t mas_op_apply(const mas_op_t* op_c, const double* x, double* y, cuda
     const long long plane = op->geo.plane;
     if (op->g->comm)
         ST(comm_seams(op->g->comm, xd, op->ncomp, op->g->nl, plane, op->xg,
-                      op->xg + op->ncomp * plane, stream));
+                      op->xg + op->ncomp * plane, stream, rstride(op)));
+    ST(tseams(op, xd, op->ncomp, op->xgt, stream));
     StencilArgs a{};
     a.g = op->geo;
     a.chunk = op->chunk;
     a.u = halo_of(op, xd, op->xg, op->ncomp);
     a.kappa = halo_of(op, op->kappa, op->kg, 1);
+    a.tu = packed_rows(op, op->xgt, op->ncomp);
+    a.tkappa = packed_rows(op, op->kgt, 1);
     a.c = op->c;
     a.out = yd;
     a.scr = op->scr;
@@ -678,13 +783,14 @@ mas_status_t mas_op_enable_p2p(mas_op_t* op, cudaStream_t s) {
     struct Rec {
         cudaIpcMemHandle_t h[4];
         unsigned long long raw[4];
-        int nl;
+        int nl, ntl;
         int ok;
     };
     Rec mine;
     memset(&mine, 0, sizeof(mine));
     const void* bufs[4] = {op->r, op->p[0], op->p[1], op->mbox};
     mine.nl = op->g->nl;
+    mine.ntl = op->g->ntl;
     mine.ok = 1;
     for (int b = 0; b < 4; b++) {
         mine.raw[b] = (unsigned long long)(uintptr_t)bufs[b];
@@ -711,13 +817,22 @@ mas_status_t mas_op_enable_p2p(mas_op_t* op, cudaStream_t s) {
     };
     std::vector<Mail*> peers(P, nullptr);
     for (int q = 0; q < P && ok; q++) peers[q] = (Mail*)map(q, 3);
-    for (int side = 0; side < 2 && ok; side++) {
-        const int q = side == 0 ? rank - 1 : rank + 1;
+    const int pt = op->g->ptheta;
+    for (int side = 0; side < 2 && ok; side++) {  // r-neighbours: rank -/+ ptheta
+        const int q = side == 0 ? rank - pt : rank + pt;
         if (q < 0 || q >= P) continue;
         op->nb_r[side] = (const double*)map(q, 0);
         op->nb_p[0][side] = (const double*)map(q, 1);
         op->nb_p[1][side] = (const double*)map(q, 2);
         op->nb_nl[side] = all[q].nl;
+    }
+    for (int side = 0; side < 2 && ok; side++) {  // theta neighbours (same r-slab)
+        const int q = side == 0 ? op->tlo : op->thi;
+        if (q < 0) continue;
+        op->nbt_r[side] = (const double*)map(q, 0);
+        op->nbt_p[0][side] = (const double*)map(q, 1);
+        op->nbt_p[1][side] = (const double*)map(q, 2);
+        op->nbt_ntl[side] = all[q].ntl;
     }
     if (ok && dmalloc(&op->d_peers, (size_t)P) == MAS_OK &&
         cudaMemcpy(op->d_peers, peers.data(), P * sizeof(Mail*), cudaMemcpyHostToDevice) != cudaSuccess) {
@@ -745,6 +860,8 @@ mas_status_t mas_op_enable_p2p(mas_op_t* op, cudaStream_t s) {
         if (op->d_peers) cudaFree(op->d_peers);
         op->d_peers = nullptr;
         op->nb_r[0] = op->nb_r[1] = nullptr;
+        op->nbt_r[0] = op->nbt_r[1] = nullptr;
+        op->nbt_p[0][0] = op->nbt_p[0][1] = op->nbt_p[1][0] = op->nbt_p[1][1] = nullptr;
         op->nb_p[0][0] = op->nb_p[0][1] = op->nb_p[1][0] = op->nb_p[1][1] = nullptr;
         set_last_error("P2P transport unavailable: " + why);
         return MAS_ERR_CUDA;
@@ -818,13 +935,17 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
     double* rr_h = op->hist + 2 * op->hist_cap;
 
     // a3: r = f - L x0 and the three initial dot products
-    if (comm) ST(comm_seams(comm, xd, nc, op->g->nl, plane, op->xg, op->xg + nc * plane, s));
+    if (comm) ST(comm_seams(comm, xd, nc, op->g->nl, plane, op->xg, op->xg + nc * plane, s, rstride(op)));
+    ST(tseams(op, xd, nc, op->xgt, s));
     StencilArgs a{};
     a.g = op->geo;
     a.chunk = op->chunk;
     a.u = halo_of(op, xd, op->xg, nc);
     a.kappa = halo_of(op, op->kappa, op->kg, 1);
     a.dinv = halo_of(op, op->dinv, op->dg, 1);
+    a.tu = packed_rows(op, op->xgt, nc);
+    a.tkappa = packed_rows(op, op->kgt, 1);
+    a.tdinv = packed_rows(op, op->dgt, 1);
     a.c = op->c;
     a.f = fd;
     a.out = op->r;
@@ -858,6 +979,7 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
     // and stops enqueueing once the device reports the stop (a decision all
     // ranks take identically, so the collectives stay matched).
     a.u = r_halo(op);
+    a.tu = r_trows(op);
     a.out = op->q;
     a.x = xd;
     a.f = nullptr;
@@ -867,6 +989,7 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
     if (graph) {
         ST(loop_graph(op, a, b));
         a.pold = pold_halo(op, 1);  // iteration 1 (not read)
+        a.tpold = pold_trows(op, 1);
         a.pnew = op->p[1];
         CU(launch_stencil(MODE_PCGA, nc, a, s, true));
         CU(launch_pcg_b(b, op->b_blocks, s));
@@ -878,21 +1001,37 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
         double* pold = op->p[(k + 1) & 1];
         double* pnew = op->p[k & 1];
         a.pold = pold_halo(op, k);
+        a.tpold = pold_trows(op, k);
         a.pnew = pnew;
         cudaEvent_t* pe = nullptr;
         if (op->prof) {
             ST(ensure_prof_events(op, k));
             pe = &op->pev[4 * (size_t)(k - 1)];
         }
-        if (comm && !p2p) {
+        if (comm && !p2p && split_theta(op)) {
+            // (r, theta) decomposition over NCCL: r-plane seams and packed
+            // theta rows of r and p_{k-1} on the solve stream, then kernel A
+            ST(comm_seams(comm, op->r, nc, op->g->nl, plane, op->rg, op->rg + nc * plane, s,
+                          rstride(op)));
+            ST(tseams(op, op->r, nc, op->rgt, s));
+            if (k > 1) {
+                ST(comm_seams(comm, pold, nc, op->g->nl, plane, op->pg[(k + 1) & 1],
+                              op->pg[(k + 1) & 1] + nc * plane, s, rstride(op)));
+                ST(tseams(op, pold, nc, op->pgt[(k + 1) & 1], s));
+            }
+            if (pe) CU(cudaEventRecord(pe[0], s));
+            CU(launch_stencil(MODE_PCGA, nc, a, s, k == 1));
+            op->launches++;
+        } else if (comm && !p2p) {
             // seams of r and p_{k-1} on the comm stream, overlapped with kernel
             // A on the interior chunks; the two edge chunks wait for them
             CU(cudaEventRecord(op->ev_ready, s));
             CU(cudaStreamWaitEvent(op->cs, op->ev_ready, 0));
-            ST(comm_seams(comm, op->r, nc, op->g->nl, plane, op->rg, op->rg + nc * plane, op->cs));
+            ST(comm_seams(comm, op->r, nc, op->g->nl, plane, op->rg, op->rg + nc * plane, op->cs,
+                          rstride(op)));
             if (k > 1)
                 ST(comm_seams(comm, pold, nc, op->g->nl, plane, op->pg[(k + 1) & 1],
-                              op->pg[(k + 1) & 1] + nc * plane, op->cs));
+                              op->pg[(k + 1) & 1] + nc * plane, op->cs, rstride(op)));
             CU(cudaEventRecord(op->ev_seam, op->cs));
             if (pe) CU(cudaEventRecord(pe[0], s));
             const int nchunk = (op->g->nl + op->chunk - 1) / op->chunk;

@@ -47,6 +47,7 @@ struct VGroup {
     std::vector<int> seam_nl;
     std::vector<std::vector<unsigned char>> gather;  // allgather staging (host)
     std::vector<cudaEvent_t> ev_sync;          // per rank: comm_vsync
+    std::vector<const double*> xsend;          // per rank: comm_exchange send buffers [lo, hi]
 
     void barrier() {
         std::unique_lock<std::mutex> lk(m);
@@ -151,7 +152,8 @@ static mas_status_t h_allreduce(Comm* c, double* buf, int n, cudaStream_t s) {
 }
 
 static mas_status_t h_seams(Comm* c, const double* in, int ncomp, int nl, long long plane, double* glo,
-                            double* ghi, cudaStream_t s) {
+                            double* ghi, cudaStream_t s, int stride) {
+    const int lo = c->rank - stride, hi = c->rank + stride;
     // payload: [first plane, last plane] of every component
     const size_t pb = sizeof(double) * plane;
     std::vector<unsigned char> mine(2 * ncomp * pb);
@@ -169,18 +171,41 @@ static mas_status_t h_seams(Comm* c, const double* in, int ncomp, int nl, long l
     mas_status_t st = h_exchange(c, mine.data(), mine.size(), all);
     if (st != MAS_OK) return st;
     for (int m = 0; m < ncomp; m++) {
-        if (c->rank > 0) {  // rank-1's last plane
-            const unsigned char* src = all.data() + (c->rank - 1) * mine.size() + (2 * m + 1) * pb;
+        if (lo >= 0) {  // the lower neighbour's last plane
+            const unsigned char* src = all.data() + lo * mine.size() + (2 * m + 1) * pb;
             if ((e = cudaMemcpyAsync(glo + m * plane, src, pb, cudaMemcpyHostToDevice, s)) != cudaSuccess)
                 return cuda_fail(e, "host seams");
         }
-        if (c->rank < c->nranks - 1) {  // rank+1's first plane
-            const unsigned char* src = all.data() + (c->rank + 1) * mine.size() + (2 * m) * pb;
+        if (hi < c->nranks) {  // the upper neighbour's first plane
+            const unsigned char* src = all.data() + hi * mine.size() + (2 * m) * pb;
             if ((e = cudaMemcpyAsync(ghi + m * plane, src, pb, cudaMemcpyHostToDevice, s)) != cudaSuccess)
                 return cuda_fail(e, "host seams");
         }
     }
     if ((e = cudaStreamSynchronize(s)) != cudaSuccess) return cuda_fail(e, "host seams");
+    return MAS_OK;
+}
+
+static mas_status_t h_xchg(Comm* c, int lo, int hi, const double* send_lo, const double* send_hi,
+                           double* recv_lo, double* recv_hi, size_t count, cudaStream_t s) {
+    const size_t b = count * sizeof(double);
+    std::vector<unsigned char> mine(2 * b, 0);
+    cudaError_t e;
+    if (lo >= 0 && (e = cudaMemcpyAsync(mine.data(), send_lo, b, cudaMemcpyDeviceToHost, s)) != cudaSuccess)
+        return cuda_fail(e, "host exchange");
+    if (hi >= 0 && (e = cudaMemcpyAsync(mine.data() + b, send_hi, b, cudaMemcpyDeviceToHost, s)) != cudaSuccess)
+        return cuda_fail(e, "host exchange");
+    if ((e = cudaStreamSynchronize(s)) != cudaSuccess) return cuda_fail(e, "host exchange");
+    std::vector<unsigned char> all;
+    mas_status_t st = h_exchange(c, mine.data(), mine.size(), all);
+    if (st != MAS_OK) return st;
+    if (lo >= 0 && (e = cudaMemcpyAsync(recv_lo, all.data() + lo * 2 * b + b, b, cudaMemcpyHostToDevice, s)) !=
+                       cudaSuccess)
+        return cuda_fail(e, "host exchange");
+    if (hi >= 0 && (e = cudaMemcpyAsync(recv_hi, all.data() + hi * 2 * b, b, cudaMemcpyHostToDevice, s)) !=
+                       cudaSuccess)
+        return cuda_fail(e, "host exchange");
+    if ((e = cudaStreamSynchronize(s)) != cudaSuccess) return cuda_fail(e, "host exchange");
     return MAS_OK;
 }
 
@@ -211,6 +236,7 @@ static mas_status_t vgroup_join(const mas_dist_t* d, Comm* c) {
             g->seam_nl.assign(g->n, 0);
             g->gather.resize(g->n);
             g->ev_sync.resize(g->n);
+            g->xsend.assign(2 * g->n, nullptr);
             cudaError_t e = cudaMalloc(&g->stage, sizeof(double) * 8 * g->n);
             for (int r = 0; r < g->n && e == cudaSuccess; r++) {
                 e = cudaEventCreateWithFlags(&g->ev_in[r], cudaEventDisableTiming);
@@ -345,7 +371,7 @@ mas_status_t comm_allreduce(Comm* c, double* buf, int n, cudaStream_t s) {
 // seams: edge r-planes to the r-neighbours' ghost planes
 // ---------------------------------------------------------------------------
 static mas_status_t v_seams(Comm* c, const double* in, int ncomp, int nl, long long plane,
-                            double* glo, double* ghi, cudaStream_t s) {
+                            double* glo, double* ghi, cudaStream_t s, int stride) {
     VGroup* g = c->vg;
     const int r = c->rank;
     cudaError_t e;
@@ -355,7 +381,7 @@ static mas_status_t v_seams(Comm* c, const double* in, int ncomp, int nl, long l
     g->barrier();
     const size_t bytes = sizeof(double) * plane;
     for (int side = 0; side < 2; side++) {
-        const int nb = side == 0 ? r - 1 : r + 1;
+        const int nb = side == 0 ? r - stride : r + stride;
         if (nb < 0 || nb >= g->n) continue;
         if ((e = cudaStreamWaitEvent(s, g->ev_seam[nb], 0)) != cudaSuccess)
             return cuda_fail(e, "virtual seam wait");
@@ -372,34 +398,87 @@ static mas_status_t v_seams(Comm* c, const double* in, int ncomp, int nl, long l
     if ((e = cudaEventRecord(g->ev_pull[r], s)) != cudaSuccess) return cuda_fail(e, "virtual seam record");
     g->barrier();
     // my edge planes must not be overwritten before the neighbours pulled them
-    for (int nb : {r - 1, r + 1})
+    for (int nb : {r - stride, r + stride})
         if (nb >= 0 && nb < g->n && (e = cudaStreamWaitEvent(s, g->ev_pull[nb], 0)) != cudaSuccess)
             return cuda_fail(e, "virtual seam wait");
     return MAS_OK;
 }
 
+// r-seams: the r-neighbours are rank -/+ nb_stride (nb_stride = ptheta under
+// an (r, theta) decomposition with theta fastest in the rank numbering)
 mas_status_t comm_seams(Comm* c, const double* in, int ncomp, int nl, long long plane, double* glo,
-                        double* ghi, cudaStream_t s) {
+                        double* ghi, cudaStream_t s, int nb_stride) {
     if (!c || c->nranks == 1) return MAS_OK;
-    if (c->vg) return v_seams(c, in, ncomp, nl, plane, glo, ghi, s);
-    if (!c->hdir.empty()) return h_seams(c, in, ncomp, nl, plane, glo, ghi, s);
+    if (c->vg) return v_seams(c, in, ncomp, nl, plane, glo, ghi, s, nb_stride);
+    if (!c->hdir.empty()) return h_seams(c, in, ncomp, nl, plane, glo, ghi, s, nb_stride);
+    const int lo = c->rank - nb_stride, hi = c->rank + nb_stride;
     const long long Nl = (long long)nl * plane;
     ncclResult_t r = ncclGroupStart();
     if (r != ncclSuccess) return nccl_fail(r, "ncclGroupStart");
     for (int m = 0; m < ncomp; m++) {
         const double* first = in + m * Nl;
         const double* last = in + m * Nl + (long long)(nl - 1) * plane;
-        if (c->rank > 0) {
-            ncclSend(first, plane, ncclFloat64, c->rank - 1, c->nccl_seam, s);
-            ncclRecv(glo + m * plane, plane, ncclFloat64, c->rank - 1, c->nccl_seam, s);
+        if (lo >= 0) {
+            ncclSend(first, plane, ncclFloat64, lo, c->nccl_seam, s);
+            ncclRecv(glo + m * plane, plane, ncclFloat64, lo, c->nccl_seam, s);
         }
-        if (c->rank < c->nranks - 1) {
-            ncclSend(last, plane, ncclFloat64, c->rank + 1, c->nccl_seam, s);
-            ncclRecv(ghi + m * plane, plane, ncclFloat64, c->rank + 1, c->nccl_seam, s);
+        if (hi < c->nranks) {
+            ncclSend(last, plane, ncclFloat64, hi, c->nccl_seam, s);
+            ncclRecv(ghi + m * plane, plane, ncclFloat64, hi, c->nccl_seam, s);
         }
     }
     r = ncclGroupEnd();
     return r == ncclSuccess ? MAS_OK : nccl_fail(r, "seam send/recv");
+}
+
+// ---------------------------------------------------------------------------
+// exchange of packed buffers (theta-ghost rows of the 2-D decomposition)
+// ---------------------------------------------------------------------------
+static mas_status_t v_xchg(Comm* c, int lo, int hi, const double* send_lo, const double* send_hi,
+                           double* recv_lo, double* recv_hi, size_t count, cudaStream_t s) {
+    VGroup* g = c->vg;
+    const int r = c->rank;
+    cudaError_t e;
+    g->xsend[2 * r] = send_lo;
+    g->xsend[2 * r + 1] = send_hi;
+    if ((e = cudaEventRecord(g->ev_seam[r], s)) != cudaSuccess) return cuda_fail(e, "virtual exchange");
+    g->barrier();
+    const size_t b = count * sizeof(double);
+    if (lo >= 0) {  // lower neighbour's send_hi -> my recv_lo
+        if ((e = cudaStreamWaitEvent(s, g->ev_seam[lo], 0)) != cudaSuccess ||
+            (e = cudaMemcpyAsync(recv_lo, g->xsend[2 * lo + 1], b, cudaMemcpyDeviceToDevice, s)) != cudaSuccess)
+            return cuda_fail(e, "virtual exchange");
+    }
+    if (hi >= 0) {  // upper neighbour's send_lo -> my recv_hi
+        if ((e = cudaStreamWaitEvent(s, g->ev_seam[hi], 0)) != cudaSuccess ||
+            (e = cudaMemcpyAsync(recv_hi, g->xsend[2 * hi], b, cudaMemcpyDeviceToDevice, s)) != cudaSuccess)
+            return cuda_fail(e, "virtual exchange");
+    }
+    if ((e = cudaEventRecord(g->ev_pull[r], s)) != cudaSuccess) return cuda_fail(e, "virtual exchange");
+    g->barrier();
+    for (int nb : {lo, hi})
+        if (nb >= 0 && (e = cudaStreamWaitEvent(s, g->ev_pull[nb], 0)) != cudaSuccess)
+            return cuda_fail(e, "virtual exchange");
+    return MAS_OK;
+}
+
+mas_status_t comm_exchange(Comm* c, int lo, int hi, const double* send_lo, const double* send_hi,
+                           double* recv_lo, double* recv_hi, size_t count, cudaStream_t s) {
+    if (!c || c->nranks == 1) return MAS_OK;  // collective: every rank calls (host/virtual barriers)
+    if (c->vg) return v_xchg(c, lo, hi, send_lo, send_hi, recv_lo, recv_hi, count, s);
+    if (!c->hdir.empty()) return h_xchg(c, lo, hi, send_lo, send_hi, recv_lo, recv_hi, count, s);
+    ncclResult_t r = ncclGroupStart();
+    if (r != ncclSuccess) return nccl_fail(r, "ncclGroupStart");
+    if (lo >= 0) {
+        ncclSend(send_lo, count, ncclFloat64, lo, c->nccl_seam, s);
+        ncclRecv(recv_lo, count, ncclFloat64, lo, c->nccl_seam, s);
+    }
+    if (hi >= 0) {
+        ncclSend(send_hi, count, ncclFloat64, hi, c->nccl_seam, s);
+        ncclRecv(recv_hi, count, ncclFloat64, hi, c->nccl_seam, s);
+    }
+    r = ncclGroupEnd();
+    return r == ncclSuccess ? MAS_OK : nccl_fail(r, "theta-row send/recv");
 }
 
 // ---------------------------------------------------------------------------

@@ -40,11 +40,12 @@ static bool strictly_inside(const double* node, const double* half, int n, std::
 
 int validate_mesh(int nr, int nt, int np, const double* rF, const double* rC, const double* tF,
                   const double* tC, const double* pF, const double* pC, int pole_flags,
-                  int periodic_phi, int nranks, std::string* why) {
+                  int periodic_phi, int pr, int ptheta, std::string* why) {
     if (!rF || !rC || !tF || !tC || !pF || !pC) { *why = "null mesh pointer"; return 0; }
     if (nr < 1 || nt < 1 || np < 2) { *why = "need nr >= 1, nt >= 1, np >= 2"; return 0; }
     if (np % 2) { *why = "np must be even (16-byte phi pairs)"; return 0; }
-    if (nranks < 1 || nr < nranks) { *why = "need nr >= nranks >= 1"; return 0; }
+    if (pr < 1 || nr < pr) { *why = "need nr >= nranks / ptheta >= 1"; return 0; }
+    if (ptheta < 1 || nt < ptheta) { *why = "need nt >= ptheta >= 1"; return 0; }
     if ((long long)nt * np > (1LL << 30)) { *why = "theta-phi plane too large"; return 0; }
     if (!periodic_phi) { *why = "periodic_phi must be 1 (reading R7)"; return 0; }
     if (pole_flags & ~(MAS_POLE_NORTH | MAS_POLE_SOUTH)) { *why = "unknown pole flag"; return 0; }
@@ -84,11 +85,12 @@ void partition(int nr, int nranks, int rank, int* i0, int* nl) {
 
 void build_tables(mas_grid* g) {
     const int nr = g->nr, nt = g->nt, np = g->np, i0 = g->i0, nl = g->nl;
+    const int j0 = g->j0, ntl = g->ntl;  // local theta rows (global faces 0 / nt stay flux-free)
     const double *rF = g->rF.data(), *rC = g->rC.data(), *tF = g->tF.data(), *tC = g->tC.data(),
                  *pF = g->pF.data(), *pC = g->pC.data();
     Tables& T = g->tab;
     T.wRm.assign(nl, 0.0); T.wRp.assign(nl, 0.0); T.irc2.assign(nl, 0.0); T.vr.assign(nl, 0.0);
-    T.wTm.assign(nt, 0.0); T.wTp.assign(nt, 0.0); T.isc2.assign(nt, 0.0); T.vt.assign(nt, 0.0);
+    T.wTm.assign(ntl, 0.0); T.wTp.assign(ntl, 0.0); T.isc2.assign(ntl, 0.0); T.vt.assign(ntl, 0.0);
     T.wPm.assign(np, 0.0); T.wPp.assign(np, 0.0); T.vp.assign(np, 0.0);
     auto hr = [&](int f) {  // centre distance across r-face f (R3 at the boundaries)
         if (f == 0) return rC[0] - rF[0];
@@ -103,12 +105,13 @@ void build_tables(mas_grid* g) {
         T.irc2[il] = 1.0 / rc2;
         T.vr[il] = rc2 * dr;
     }
-    for (int j = 0; j < nt; j++) {
+    for (int jl = 0; jl < ntl; jl++) {
+        const int j = j0 + jl;
         const double dt = tF[j + 1] - tF[j], sC = std::sin(tC[j]);
-        if (j > 0) T.wTm[j] = std::sin(tF[j]) / ((tC[j] - tC[j - 1]) * sC * dt);
-        if (j < nt - 1) T.wTp[j] = std::sin(tF[j + 1]) / ((tC[j + 1] - tC[j]) * sC * dt);
-        T.isc2[j] = 1.0 / (sC * sC);
-        T.vt[j] = sC * dt;
+        if (j > 0) T.wTm[jl] = std::sin(tF[j]) / ((tC[j] - tC[j - 1]) * sC * dt);
+        if (j < nt - 1) T.wTp[jl] = std::sin(tF[j + 1]) / ((tC[j + 1] - tC[j]) * sC * dt);
+        T.isc2[jl] = 1.0 / (sC * sC);
+        T.vt[jl] = sC * dt;
     }
     std::vector<double> hp(np);
     hp[0] = pC[0] + kTwoPi - pC[np - 1];

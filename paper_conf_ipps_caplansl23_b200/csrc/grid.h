@@ -19,6 +19,9 @@ struct Comm;  // comm.cpp (NCCL)
 struct mas_grid {
     int nr = 0, nt = 0, np = 0;
     int i0 = 0, nl = 0;
+    // (r, theta) decomposition: nranks = pr * ptheta, rank = rrank * ptheta + trank
+    int ptheta = 1, pr = 1, rrank = 0, trank = 0;
+    int j0 = 0, ntl = 0;      // this rank's theta rows [j0, j0 + ntl)
     int pole_flags = 0;
     int nranks = 1, rank = 0;
     int device = 0;
@@ -32,7 +35,7 @@ namespace mas {
 
 int validate_mesh(int nr, int nt, int np, const double* rF, const double* rC, const double* tF,
                   const double* tC, const double* pF, const double* pC, int pole_flags,
-                  int periodic_phi, int nranks, std::string* why);
+                  int periodic_phi, int pr, int ptheta, std::string* why);
 void partition(int nr, int nranks, int rank, int* i0, int* nl);
 void build_tables(mas_grid* g);
 
@@ -46,7 +49,11 @@ mas_status_t comm_allreduce(Comm* c, double* buf, int n, cudaStream_t s);
 // ([ncomp][nl][plane]): send first/last plane to rank-1/rank+1, receive the
 // neighbours' edge planes into glo / ghi ([ncomp][plane]).
 mas_status_t comm_seams(Comm* c, const double* in, int ncomp, int nl, long long plane, double* glo,
-                        double* ghi, cudaStream_t s);
+                        double* ghi, cudaStream_t s, int nb_stride = 1);
+// exchange contiguous buffers of `count` doubles with ranks lo / hi (-1: none):
+// send_lo -> lo, recv_lo <- lo's send_hi; send_hi -> hi, recv_hi <- hi's send_lo
+mas_status_t comm_exchange(Comm* c, int lo, int hi, const double* send_lo, const double* send_hi,
+                           double* recv_lo, double* recv_hi, size_t count, cudaStream_t s);
 mas_status_t comm_barrier(Comm* c, cudaStream_t s);
 // P2P transport setup helpers
 bool comm_is_virtual(const Comm* c);

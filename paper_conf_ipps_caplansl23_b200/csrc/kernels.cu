@@ -297,10 +297,14 @@ __device__ __forceinline__ double* sfield(double* buf, int f) { return buf + f *
 struct HaloMeta {
     int hoff;  // offset in the plane
     int hidx;        // index in a ring field
-    int hkind;       // 0 none, 1 load, 3 zeros (beyond a pole / theta wall)
+    int hkind;       // 0 none, 1 load, 3 zeros (beyond a pole / theta wall),
+                     // 4 / 5 load from the lower / upper theta neighbour's row
 };
 
-__device__ __forceinline__ HaloMeta halo_meta(const Geo& g, int j0, int k0, int height, int width) {
+// hkind 4 / 5: the row beyond the local theta range belongs to the theta
+// neighbour (2-D decomposition): hoff is then the phi index in that row.
+__device__ __forceinline__ HaloMeta halo_meta(const Geo& g, int j0, int k0, int height, int width,
+                                              bool tnb_lo, bool tnb_hi) {
     const int t = threadIdx.x;
     HaloMeta m{0, 0, 0};
     if (t < 2 * TK) {
@@ -310,8 +314,8 @@ __device__ __forceinline__ HaloMeta halo_meta(const Geo& g, int j0, int k0, int 
         const int j = j0 + hr - 1;
         if (kk < width) {
             m.hidx = hr * ROW + OFF + kk;
-            m.hkind = (j >= 0 && j < g.nt) ? 1 : 3;
-            m.hoff = (int)j * g.np + k0 + kk;
+            m.hkind = (j >= 0 && j < g.nt) ? 1 : j < 0 ? (tnb_lo ? 4 : 3) : (tnb_hi ? 5 : 3);
+            m.hoff = m.hkind >= 4 ? k0 + kk : (int)j * g.np + k0 + kk;
         }
     } else if (t < 2 * TK + 2 * TJ) {
         const int q = t - 2 * TK, side = q / TJ, r = q % TJ;
@@ -348,6 +352,28 @@ __device__ __forceinline__ void cpa_commit() { asm volatile("cp.async.commit_gro
 __device__ __forceinline__ void cpa_wait_all() { asm volatile("cp.async.wait_group 0;\n" ::: "memory"); }
 
 
+// theta-neighbour row item (2-D decomposition): same private cp.async slots
+// as a local halo item, addresses from the TRows descriptors
+__device__ __forceinline__ const double* trow_at(const TRows& T, bool hi, int comp, int i, int k) {
+    return hi ? T.hi + comp * T.cs_hi + i * T.ps_hi + k : T.lo + comp * T.cs_lo + i * T.ps_lo + k;
+}
+template <int MODE, int NC>
+__device__ __forceinline__ void trow_issue(const StencilArgs& a, int i, const HaloMeta& hm, bool first,
+                                        double* h) {
+    const bool hi = hm.hkind == 5;
+    const int k = hm.hoff;
+    cpa8(h, trow_at(a.tkappa, hi, 0, i, k));
+#pragma unroll
+    for (int c = 0; c < NC; c++) cpa8(h + (2 + c) * kHaloSlots, trow_at(a.tu, hi, c, i, k));
+    if (MODE == MODE_PCGA) {
+        cpa8(h + kHaloSlots, trow_at(a.tdinv, hi, 0, i, k));
+        if (!first) {
+#pragma unroll
+            for (int c = 0; c < NC; c++) cpa8(h + (2 + NC + c) * kHaloSlots, trow_at(a.tpold, hi, c, i, k));
+        }
+    }
+}
+
 template <int MODE, int NC>
 __device__ __forceinline__ void stage_issue(const StencilArgs& a, int i, int j0, int k0, int height,
                                             int width, const HaloMeta& hm, bool first, bool xupd,
@@ -380,7 +406,9 @@ __device__ __forceinline__ void stage_issue(const StencilArgs& a, int i, int j0,
             }
         }
     }
-    if (halo && hm.hkind == 1) {
+    if (halo && hm.hkind >= 4 && interior) {
+        trow_issue<MODE, NC>(a, i, hm, first, hst + threadIdx.x);
+    } else if (halo && hm.hkind == 1) {
         double* h = hst + threadIdx.x;
         if (interior) {  // halo planes are stencil planes: always interior here
             const int hi = ipl + (int)hm.hoff;
@@ -434,7 +462,7 @@ __device__ __forceinline__ void stage_commit(const StencilArgs& a, int i, int j0
             }
         }
     }
-    if (halo && hm.hkind == 1) {
+    if (halo && (hm.hkind == 1 || hm.hkind >= 4)) {
         cpa_wait_all();  // this thread's own copies; read back below by the same thread
         const double* h = hst + threadIdx.x;
 #pragma unroll
@@ -658,7 +686,8 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
     OwnRegs<NC> oc, on;  // own-cell stencil inputs for the current / next plane
     double2 kown = make_double2(0.0, 0.0), kdummy;
     const bool lo_ghost = (ia == 0) && g.glob_lo;
-    const HaloMeta hm = halo_meta(g, j0, k0, height, width);
+    const HaloMeta hm = halo_meta(g, j0, k0, height, width, a.tkappa.lo != nullptr,
+                                  a.tkappa.hi != nullptr);
     // planes ia-1 (own cells only) and ia: both loads in flight together
     Stage<NC> S0, S;
     if (!lo_ghost)
@@ -900,8 +929,8 @@ __device__ __forceinline__ double kap_at(const Halo& h, int i, long long off, co
 
 // D = c + sum_f a_f (Dirichlet faces included via kappa_ghost = kappa_P),
 // dinv = 1/D; flags negative / non-finite coefficients and D <= 0.
-__global__ void __launch_bounds__(kThreads) k_diag(const Geo g, const Halo kappa, const double* c,
-                                                   double* D, double* dinv, int* bad) {
+__global__ void __launch_bounds__(kThreads) k_diag(const Geo g, const Halo kappa, const TRows tk,
+                                                   const double* c, double* D, double* dinv, int* bad) {
     const long long Nl = (long long)g.nl * g.plane;
     for (long long P = blockIdx.x * (long long)kThreads + threadIdx.x; P < Nl;
          P += (long long)gridDim.x * kThreads) {
@@ -912,8 +941,10 @@ __global__ void __launch_bounds__(kThreads) k_diag(const Geo g, const Halo kappa
         const double cp = c ? c[P] : 0.0;
         const double kim = (i == 0 && g.glob_lo) ? kp : kap_at(kappa, i - 1, off, g);
         const double kip = (i == g.nl - 1 && g.glob_hi) ? kp : kap_at(kappa, i + 1, off, g);
-        const double kjm = j > 0 ? kappa.in[P - g.np] : 0.0;
-        const double kjp = j < g.nt - 1 ? kappa.in[P + g.np] : 0.0;
+        // beyond the local theta rows: the theta neighbour's row, else 0 (pole / wall, weight 0)
+        const double kjm = j > 0 ? kappa.in[P - g.np] : tk.lo ? tk.lo[(long long)i * tk.ps_lo + k] : 0.0;
+        const double kjp = j < g.nt - 1 ? kappa.in[P + g.np]
+                                        : tk.hi ? tk.hi[(long long)i * tk.ps_hi + k] : 0.0;
         const int km = k == 0 ? g.np - 1 : k - 1, kq = k == g.np - 1 ? 0 : k + 1;
         const double kkm = kappa.in[P - k + km], kkp = kappa.in[P - k + kq];
         const double irc = g.irc2[i];
@@ -1020,11 +1051,32 @@ cudaError_t launch_pcg_b(const StreamArgs& a, int nblocks, cudaStream_t s) {
     return cudaGetLastError();
 }
 
-cudaError_t launch_diag(const Geo& g, Halo kappa, const double* c, double* D, double* dinv, int* bad,
-                        cudaStream_t s) {
+cudaError_t launch_diag(const Geo& g, Halo kappa, TRows tkappa, const double* c, double* D,
+                        double* dinv, int* bad, cudaStream_t s) {
     const long long Nl = (long long)g.nl * g.plane;
     const int blocks = (int)std::min<long long>((Nl + kThreads - 1) / kThreads, 148LL * 16);
-    k_diag<<<blocks, kThreads, 0, s>>>(g, kappa, c, D, dinv, bad);
+    k_diag<<<blocks, kThreads, 0, s>>>(g, kappa, tkappa, c, D, dinv, bad);
+    return cudaGetLastError();
+}
+
+// first / last theta rows of every plane of a field, packed [2][ncomp][nl][np]
+__global__ void k_pack_rows(const Geo g, int ncomp, const double* in, double* out) {
+    const long long n = (long long)ncomp * g.nl * g.np;  // per side
+    for (long long t = blockIdx.x * (long long)blockDim.x + threadIdx.x; t < 2 * n;
+         t += (long long)gridDim.x * blockDim.x) {
+        const int side = t >= n;
+        const long long u = t - side * n;
+        const long long ci = u / g.np;  // comp * nl + i
+        const int k = (int)(u - ci * g.np);
+        const int j = side ? g.nt - 1 : 0;
+        out[t] = in[ci * g.plane + (long long)j * g.np + k];
+    }
+}
+
+cudaError_t launch_pack_rows(const Geo& g, int ncomp, const double* in, double* out, cudaStream_t s) {
+    const long long n = 2LL * ncomp * g.nl * g.np;
+    const int blocks = (int)std::min<long long>((n + 255) / 256, 148LL * 8);
+    k_pack_rows<<<blocks, 256, 0, s>>>(g, ncomp, in, out);
     return cudaGetLastError();
 }
 

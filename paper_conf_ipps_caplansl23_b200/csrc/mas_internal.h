@@ -21,7 +21,7 @@ namespace mas {
 // with kf = (kappa_P + kappa_N)/2 of that face.  V_P = vr[i] vt[j] vp[k].
 // ---------------------------------------------------------------------------
 struct Geo {
-    int nl, nt, np;        // local r-planes, theta, phi
+    int nl, nt, np;        // local r-planes, local theta rows, phi
     long long plane;       // nt*np
     int glob_lo, glob_hi;  // this slab owns the global inner / outer r-boundary
     const double* wRm;     // [nl] r-face i   / V  (0 on a global Neumann face)
@@ -46,6 +46,19 @@ struct Halo {
     const double* ghi;  // plane i0+nl of component 0 (ghost copy, or rank+1's first plane)
     int slo, shi;       // component strides of glo / ghi (plane for a ghost copy,
                         // nl_neighbour * plane for a neighbour's array)
+};
+
+// The theta-ghost rows of a field under an (r, theta) decomposition (NEXT-3):
+// rows j = -1 and j = nt_local of every local plane, taken from the theta
+// neighbours.  Either a packed copy [ncomp][nl][np] (static kappa / 1/D rows,
+// x at init, the NCCL loop) or, under the P2P transport, the neighbour's own
+// array read in place.  lo / hi == nullptr: no neighbour on that side (pole or
+// theta wall: the face carries no flux, the halo holds zeros).
+struct TRows {
+    const double* lo;  // row j = -1, component 0, plane 0
+    const double* hi;  // row j = nt_local
+    int cs_lo, ps_lo;  // component / plane strides of lo
+    int cs_hi, ps_hi;
 };
 
 // ---------------------------------------------------------------------------
@@ -103,6 +116,7 @@ struct StencilArgs {
     Halo pold;                // PCGA: p_{k-1}
     Halo dinv;                // PCGA: 1/D with halo;  RESID: own only
     Halo kappa;
+    TRows tu, tpold, tdinv, tkappa;  // theta-ghost rows (2-D decomposition; zero: none)
     const double* c;          // [nl][nt][np] or nullptr
     const double* f;          // RESID: rhs [ncomp][nl][nt][np]
     double* out;              // APPLY: y;  RESID: r;  PCGA: q
@@ -142,8 +156,10 @@ int stencil_blocks(const Geo& g, int chunk);
 cudaError_t launch_stencil(int mode, int ncomp, const StencilArgs& a, cudaStream_t s,
                            bool first = false);
 cudaError_t launch_pcg_b(const StreamArgs& a, int nblocks, cudaStream_t s);
-cudaError_t launch_diag(const Geo& g, Halo kappa, const double* c, double* D, double* dinv,
-                        int* bad, cudaStream_t s);
+cudaError_t launch_diag(const Geo& g, Halo kappa, TRows tkappa, const double* c, double* D,
+                        double* dinv, int* bad, cudaStream_t s);
+// out[side][c][i][k] = in[c][i][side ? nt-1 : 0][k]: a field's first / last theta rows
+cudaError_t launch_pack_rows(const Geo& g, int ncomp, const double* in, double* out, cudaStream_t s);
 cudaError_t launch_dirichlet(const Geo& g, int ncomp, const double* kappa, const double* ub,
                              int outer, double* f, cudaStream_t s);
 cudaError_t launch_dot(const Geo& g, int ncomp, const double* a, const double* b, Scratch scr,

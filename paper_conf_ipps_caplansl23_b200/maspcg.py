@@ -25,7 +25,8 @@ MAS_POLE_NORTH, MAS_POLE_SOUTH = 1, 2
 ABI_SYMBOLS = ("mas_comm_unique_id", "mas_partition", "mas_grid_create", "mas_grid_local_extent",
                "mas_grid_destroy", "mas_op_setup", "mas_op_update", "mas_op_apply", "mas_op_diag",
                "mas_op_dirichlet_rhs", "mas_op_dot", "mas_pcg_solve", "mas_op_enable_p2p",
-               "mas_op_transport", "mas_op_launch_count",
+               "mas_op_transport", "mas_op_launch_count", "mas_grid_create_2d",
+               "mas_grid_local_extent_2d",
                "mas_op_set_profiling", "mas_op_kernel_times", "mas_op_destroy", "mas_status_string", "mas_last_error", "mas_version")
 
 
@@ -56,6 +57,9 @@ def lib() -> C.CDLL:
             "mas_grid_create": (_i, [_i, _i, _i, _vp, _vp, _vp, _vp, _vp, _vp, _i, _i, _vp, _vp]),
             "mas_partition": (_i, [_i, _i, _i, _vp, _vp]),
             "mas_grid_local_extent": (_i, [_vp, _vp, _vp]),
+            "mas_grid_create_2d": (_i, [_i, _i, _i, _vp, _vp, _vp, _vp, _vp, _vp, _i, _i, _vp, _i,
+                                        _vp]),
+            "mas_grid_local_extent_2d": (_i, [_vp, _vp, _vp, _vp, _vp]),
             "mas_grid_destroy": (_i, [_vp]),
             "mas_op_setup": (_i, [_vp, _i, _vp, _vp, _i, _i, _vp, _vp]),
             "mas_op_update": (_i, [_vp, _vp, _vp, _vp]),
@@ -146,8 +150,9 @@ def host_exchange_id(directory: str) -> bytes:
 
 
 def mas_grid_create(r_node, r_half, t_node, t_half, p_node, p_half, pole_flags=3,
-                    periodic_phi=1, dist: Optional[tuple] = None) -> int:
-    """dist = (nranks, rank, nccl_id_bytes) or None.  Returns the handle."""
+                    periodic_phi=1, dist: Optional[tuple] = None, ptheta: int = 1) -> int:
+    """dist = (nranks, rank, nccl_id_bytes) or None.  ptheta > 1: (r, theta)
+    decomposition through mas_grid_create_2d.  Returns the handle."""
     arrs = [np.ascontiguousarray(a, dtype=np.float64) for a in
             (r_node, r_half, t_node, t_half, p_node, p_half)]
     nr, nt, np_ = len(arrs[1]), len(arrs[3]), len(arrs[5])
@@ -159,10 +164,17 @@ def mas_grid_create(r_node, r_half, t_node, t_half, p_node, p_half, pole_flags=3
         d = mas_dist_t(dist[0], dist[1])
         C.memmove(d.nccl_id, dist[2], 128)
     out = C.c_void_p()
-    _check(lib().mas_grid_create(nr, nt, np_, *[a.ctypes.data for a in arrs], pole_flags,
-                                 periodic_phi, C.byref(d) if d is not None else None,
-                                 C.byref(out)), "mas_grid_create")
+    _check(lib().mas_grid_create_2d(nr, nt, np_, *[a.ctypes.data for a in arrs], pole_flags,
+                                    periodic_phi, C.byref(d) if d is not None else None,
+                                    int(ptheta), C.byref(out)), "mas_grid_create_2d")
     return out.value
+
+
+def mas_grid_local_extent_2d(g: int):
+    i0, nl, j0, ntl = C.c_int(), C.c_int(), C.c_int(), C.c_int()
+    _check(lib().mas_grid_local_extent_2d(g, C.byref(i0), C.byref(nl), C.byref(j0), C.byref(ntl)),
+           "mas_grid_local_extent_2d")
+    return i0.value, nl.value, j0.value, ntl.value
 
 
 def mas_partition(nr: int, nranks: int, rank: int):
@@ -264,7 +276,7 @@ def mas_version() -> str:
 # small RAII helpers over the same calls
 # ---------------------------------------------------------------------------
 class Grid:
-    def __init__(self, mesh, dist=None):
+    def __init__(self, mesh, dist=None, ptheta=1):
         flags = (MAS_POLE_NORTH if getattr(mesh, "pole_north", True) else 0) | \
                 (MAS_POLE_SOUTH if getattr(mesh, "pole_south", True) else 0)
         if mesh.tF[0] != 0.0:
@@ -272,8 +284,8 @@ class Grid:
         if abs(mesh.tF[-1] - np.pi) > 1e-15:
             flags &= ~MAS_POLE_SOUTH
         self.h = mas_grid_create(mesh.rF, mesh.rC, mesh.tF, mesh.tC, mesh.pF, mesh.pC, flags, 1,
-                                 dist)
-        self.i0, self.nl = mas_grid_local_extent(self.h)
+                                 dist, ptheta)
+        self.i0, self.nl, self.j0, self.ntl = mas_grid_local_extent_2d(self.h)
         self.shape = (len(mesh.rC), len(mesh.tC), len(mesh.pC))
 
     def close(self):

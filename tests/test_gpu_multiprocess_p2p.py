@@ -31,34 +31,38 @@ import json, sys
 import numpy as np, torch
 sys.path.insert(0, {root!r})
 from paper_conf_ipps_caplansl23_b200 import maspcg as M, workloads as W
-P, rank, d, kind, nr, nt, np_, p2p = {P}, int(sys.argv[1]), {d!r}, {kind!r}, {nr}, {nt}, {np_}, {p2p}
+P, rank, d, kind, nr, nt, np_, p2p, pt = ({P}, int(sys.argv[1]), {d!r}, {kind!r}, {nr}, {nt}, {np_},
+                                          {p2p}, {ptheta})
 torch.cuda.set_device(0)
 prob = W.make(kind, nr=nr, nt=nt, np_=np_, warm=False)
-g = M.Grid(prob.mesh, dist=(P, rank, M.host_exchange_id(d)))
-sl = slice(g.i0, g.i0 + g.nl)
+g = M.Grid(prob.mesh, dist=(P, rank, M.host_exchange_id(d)), ptheta=pt)
+sl = (slice(g.i0, g.i0 + g.nl), slice(g.j0, g.j0 + g.ntl))
+slc = (slice(None),) + sl
 dv = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()
 op = M.Operator(g, prob.ncomp, dv(prob.kappa[sl]), dv(prob.c[sl]), prob.bc_inner, prob.bc_outer)
 if p2p:
     op.enable_p2p()
-f = dv(prob.f[:, sl])
-op.dirichlet_rhs(dv(prob.ub_inner) if prob.ub_inner is not None else None, None, f)
+f = dv(prob.f[slc])
+op.dirichlet_rhs(dv(prob.ub_inner[:, g.j0:g.j0 + g.ntl]) if prob.ub_inner is not None else None,
+                 None, f)
 res = []
 for _ in range(2):
-    x = dv(prob.x0[:, sl])
+    x = dv(prob.x0[slc])
     st, it, rel, hist = op.solve(f, x, prob.tol, prob.maxit, True)
     torch.cuda.synchronize()
     res.append((st, it))
 np.save(f"{{d}}/x.{{rank}}.npy", x.cpu().numpy())
-json.dump({{"res": res, "transport": op.transport, "i0": g.i0, "nl": g.nl, "hist": list(hist)}},
+json.dump({{"res": res, "transport": op.transport, "i0": g.i0, "nl": g.nl, "j0": g.j0,
+           "ntl": g.ntl, "hist": list(hist)}},
           open(f"{{d}}/out.{{rank}}.json", "w"))
 op.close(); g.close()
 """
 
 
-def run_procs(tmp_path, P, kind, shape, p2p=True, timeout=600):
+def run_procs(tmp_path, P, kind, shape, p2p=True, timeout=600, ptheta=1):
     d = str(tmp_path)
     src = WORKER.format(root=ROOT, P=P, d=d, kind=kind, nr=shape[0], nt=shape[1], np_=shape[2],
-                        p2p=p2p)
+                        p2p=p2p, ptheta=ptheta)
     script = os.path.join(d, "worker.py")
     with open(script, "w") as fh:
         fh.write(src)
@@ -88,10 +92,11 @@ def built():
     build.build()
 
 
-@pytest.mark.parametrize("P,kind,shape", [(2, "viscosity", (12, 16, 64)),
-                                          (3, "conduction", (13, 16, 32))])
-def test_p2p_across_processes_matches_oracle(built, oracle_mod, tmp_path, P, kind, shape):
-    res, xs = run_procs(tmp_path, P, kind, shape)
+@pytest.mark.parametrize("P,kind,shape,ptheta", [(2, "viscosity", (12, 16, 64), 1),
+                                                 (3, "conduction", (13, 16, 32), 1),
+                                                 (4, "viscosity", (10, 18, 64), 2)])
+def test_p2p_across_processes_matches_oracle(built, oracle_mod, tmp_path, P, kind, shape, ptheta):
+    res, xs = run_procs(tmp_path, P, kind, shape, ptheta=ptheta)
     assert all(r["transport"] == "p2p" for r in res)
     prob = W.make(kind, nr=shape[0], nt=shape[1], np_=shape[2], warm=False)
     rc, xo, ito, _, _ = oracle_mod.solve_problem(prob)
@@ -100,5 +105,8 @@ def test_p2p_across_processes_matches_oracle(built, oracle_mod, tmp_path, P, kin
     (st1, it1), (st2, it2) = its.pop()
     assert st1 == st2 == 0 and it1 == it2 and abs(it1 - ito) <= 1
     V = oracle_mod.Oracle.for_problem(prob).volumes()[None]
-    xg = np.concatenate(xs, axis=1)
+    xg = np.full(xo.shape, np.nan)
+    for r, xl in zip(res, xs):
+        xg[:, r["i0"]:r["i0"] + r["nl"], r["j0"]:r["j0"] + r["ntl"]] = xl
+    assert not np.isnan(xg).any()
     assert math.sqrt((V * (xg - xo) ** 2).sum() / (V * xo ** 2).sum()) <= 1e-10

@@ -31,8 +31,20 @@ def mp():
     return maspcg
 
 
+def assemble(out, key):
+    """Global [comp][r][theta][phi] field from the ranks' local blocks."""
+    nc = out[0][key].shape[0]
+    nr = max(r["i0"] + r["nl"] for r in out)
+    nt = max(r["j0"] + r["ntl"] for r in out)
+    g = np.full((nc, nr, nt, out[0][key].shape[3]), np.nan)
+    for r in out:
+        g[:, r["i0"]:r["i0"] + r["nl"], r["j0"]:r["j0"] + r["ntl"]] = r[key]
+    assert not np.isnan(g).any()
+    return g
+
+
 def run_ranks(mp, prob, P, x_apply, want_solve=True, maxit=None, tol=None, p2p=False,
-              solves=1):
+              solves=1, ptheta=1):
     _key[0] += 1
     vid = mp.virtual_ranks_id(_key[0])
     res, errs = {}, []
@@ -42,27 +54,29 @@ def run_ranks(mp, prob, P, x_apply, want_solve=True, maxit=None, tol=None, p2p=F
             torch.cuda.set_device(0)
             s = torch.cuda.Stream()
             with torch.cuda.stream(s):
-                g = mp.Grid(prob.mesh, dist=(P, r, vid))
-                i0, nl = g.i0, g.nl
-                sl = slice(i0, i0 + nl)
+                g = mp.Grid(prob.mesh, dist=(P, r, vid), ptheta=ptheta)
+                i0, nl, j0, ntl = g.i0, g.nl, g.j0, g.ntl
+                sl = (slice(i0, i0 + nl), slice(j0, j0 + ntl))     # [r, theta] of a field
+                slc = (slice(None),) + sl                           # [comp, r, theta]
                 d = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()
                 op = mp.Operator(g, prob.ncomp, d(prob.kappa[sl]), d(prob.c[sl]), prob.bc_inner,
                                  prob.bc_outer)
                 if p2p:
                     op.enable_p2p()
                     assert op.transport == "p2p"
-                y = torch.empty((prob.ncomp, nl) + prob.shape[1:], dtype=torch.float64, device="cuda")
-                op.apply(d(x_apply[:, sl]), y)
-                out = {"i0": i0, "nl": nl, "y": None, "dot": None}
+                y = torch.empty((prob.ncomp, nl, ntl, prob.shape[2]), dtype=torch.float64,
+                                device="cuda")
+                op.apply(d(x_apply[slc]), y)
+                out = {"i0": i0, "nl": nl, "j0": j0, "ntl": ntl, "y": None, "dot": None}
                 torch.cuda.current_stream().synchronize()
                 out["y"] = y.cpu().numpy()
-                out["dot"] = op.dot(d(x_apply[:, sl]), d(x_apply[:, sl]))
+                out["dot"] = op.dot(d(x_apply[slc]), d(x_apply[slc]))
                 if want_solve:
-                    f = d(prob.f[:, sl])
-                    ubi = d(prob.ub_inner) if prob.ub_inner is not None else None
+                    f = d(prob.f[slc])
+                    ubi = d(prob.ub_inner[:, j0:j0 + ntl]) if prob.ub_inner is not None else None
                     op.dirichlet_rhs(ubi, None, f)
                     for _ in range(solves):  # repeated solves: mailbox epochs
-                        x = d(prob.x0[:, sl])
+                        x = d(prob.x0[slc])
                         st, it, rel, hist = op.solve(f, x, prob.tol if tol is None else tol,
                                                      prob.maxit if maxit is None else maxit, True)
                         torch.cuda.current_stream().synchronize()
@@ -92,7 +106,7 @@ def test_virtual_ranks_apply_dot_and_pcg(mp, oracle_mod, P):
     o = oracle_mod.Oracle.for_problem(prob)
     V = o.volumes()[None]
     # matvec, assembled from the slabs
-    y = np.concatenate([r["y"] for r in out], axis=1)
+    y = assemble(out, "y")
     yo = o.apply(prob.kappa, prob.c, x)
     assert math.sqrt((V * (y - yo) ** 2).sum() / (V * yo ** 2).sum()) <= 1e-13
     # global dot through the allreduce
@@ -105,7 +119,7 @@ def test_virtual_ranks_apply_dot_and_pcg(mp, oracle_mod, P):
     it = its.pop()
     assert all(r["st"] == mp.MAS_OK for r in out)
     assert abs(it - ito) <= 1
-    xg = np.concatenate([r["x"] for r in out], axis=1)
+    xg = assemble(out, "x")
     if it == ito:
         assert math.sqrt((V * (xg - xo) ** 2).sum() / (V * xo ** 2).sum()) <= 1e-10
 
@@ -121,7 +135,7 @@ def test_virtual_ranks_seam_overlap_split_kernel(mp, oracle_mod, P):
     its = {r["it"] for r in out}
     assert len(its) == 1 and abs(its.pop() - ito) <= 1
     V = oracle_mod.Oracle.for_problem(prob).volumes()[None]
-    xg = np.concatenate([r["x"] for r in out], axis=1)
+    xg = assemble(out, "x")
     assert math.sqrt((V * (xg - xo) ** 2).sum() / (V * xo ** 2).sum()) <= 1e-10
     # the split kernel A shows up as one extra launch per iteration
     assert all(r["launches"] >= 3 * r["it"] for r in out)
@@ -133,7 +147,7 @@ def test_virtual_ranks_conduction_dirichlet_and_fixed_iterations(mp, oracle_mod)
     out = run_ranks(mp, prob, 3, x, tol=0.0, maxit=25)
     rc, xo, ito, _, _ = oracle_mod.solve_problem(prob, tol=0.0, maxit=25)
     assert all(r["st"] == mp.MAS_NOT_CONVERGED and r["it"] == 25 for r in out)
-    xg = np.concatenate([r["x"] for r in out], axis=1)
+    xg = assemble(out, "x")
     V = oracle_mod.Oracle.for_problem(prob).volumes()[None]
     assert math.sqrt((V * (xg - xo) ** 2).sum() / (V * xo ** 2).sum()) <= 1e-10
 
@@ -162,7 +176,7 @@ def test_virtual_ranks_p2p_transport_matches_nccl_path_bitwise(mp, oracle_mod, P
     rc, xo, ito, _, _ = oracle_mod.solve_problem(prob)
     assert abs(out[0]["it"] - ito) <= 1
     V = oracle_mod.Oracle.for_problem(prob).volumes()[None]
-    xg = np.concatenate([r["x"] for r in out], axis=1)
+    xg = assemble(out, "x")
     assert math.sqrt((V * (xg - xo) ** 2).sum() / (V * xo ** 2).sum()) <= 1e-10
     # no seam split: one kernel A and one kernel B per iteration
     assert all(r["launches"] <= 2 * r["it"] + 6 for r in out)
@@ -177,7 +191,7 @@ def test_virtual_ranks_p2p_long_slabs(mp, oracle_mod, P):
     its = {r["it"] for r in out}
     assert len(its) == 1 and abs(its.pop() - ito) <= 1
     V = oracle_mod.Oracle.for_problem(prob).volumes()[None]
-    xg = np.concatenate([r["x"] for r in out], axis=1)
+    xg = assemble(out, "x")
     assert math.sqrt((V * (xg - xo) ** 2).sum() / (V * xo ** 2).sum()) <= 1e-10
 
 
@@ -187,6 +201,52 @@ def test_virtual_ranks_p2p_dirichlet_fixed_iterations(mp, oracle_mod):
     out = run_ranks(mp, prob, 3, x, tol=0.0, maxit=25, p2p=True)
     rc, xo, ito, _, _ = oracle_mod.solve_problem(prob, tol=0.0, maxit=25)
     assert all(r["st"] == mp.MAS_NOT_CONVERGED and r["it"] == 25 for r in out)
-    xg = np.concatenate([r["x"] for r in out], axis=1)
+    xg = assemble(out, "x")
     V = oracle_mod.Oracle.for_problem(prob).volumes()[None]
     assert math.sqrt((V * (xg - xo) ** 2).sum() / (V * xo ** 2).sum()) <= 1e-10
+
+
+# ---------------------------------------------------------------------------
+# (r, theta) decomposition (NEXT-3): P = pr x ptheta ranks, theta fastest.
+# Theta-ghost rows: packed and exchanged (setup, apply, init, NCCL loop) or
+# read in place from the theta neighbours' arrays (P2P loop).
+# ---------------------------------------------------------------------------
+@pytest.mark.parametrize("P,ptheta,shape", [(2, 2, (9, 16, 64)), (4, 2, (12, 20, 64)),
+                                            (3, 3, (7, 13, 66)), (6, 3, (10, 25, 32))])
+def test_virtual_ranks_theta_split_matches_oracle(mp, oracle_mod, P, ptheta, shape):
+    prob = W.viscosity_problem(*shape, warm=False)
+    x = W.random_field((3,) + prob.shape, 47)
+    o = oracle_mod.Oracle.for_problem(prob)
+    V = o.volumes()[None]
+    rc, xo, ito, _, _ = oracle_mod.solve_problem(prob)
+    res = {}
+    for p2p in (False, True):
+        out = run_ranks(mp, prob, P, x, p2p=p2p, ptheta=ptheta)
+        y = assemble(out, "y")
+        yo = o.apply(prob.kappa, prob.c, x)
+        assert math.sqrt((V * (y - yo) ** 2).sum() / (V * yo ** 2).sum()) <= 1e-13
+        for r in out:
+            assert abs(r["dot"] - o.dot(x, x)) <= 1e-13 * o.dot(x, x)
+        its = {r["it"] for r in out}
+        assert len(its) == 1, its
+        it = its.pop()
+        assert all(r["st"] == mp.MAS_OK for r in out) and abs(it - ito) <= 1
+        xg = assemble(out, "x")
+        if it == ito:
+            assert math.sqrt((V * (xg - xo) ** 2).sum() / (V * xo ** 2).sum()) <= 1e-10
+        res[p2p] = (it, xg)
+    # both loops sum the same block partials in rank order
+    assert res[False][0] == res[True][0]
+    np.testing.assert_array_equal(res[False][1], res[True][1])
+
+
+def test_virtual_ranks_theta_split_conduction_dirichlet_fixed_iterations(mp, oracle_mod):
+    prob = W.conduction_problem(8, 24, 32)
+    x = W.random_field((1,) + prob.shape, 48)
+    rc, xo, ito, _, _ = oracle_mod.solve_problem(prob, tol=0.0, maxit=20)
+    V = oracle_mod.Oracle.for_problem(prob).volumes()[None]
+    for p2p in (False, True):
+        out = run_ranks(mp, prob, 4, x, tol=0.0, maxit=20, p2p=p2p, ptheta=4)
+        assert all(r["st"] == mp.MAS_NOT_CONVERGED and r["it"] == 20 for r in out)
+        xg = assemble(out, "x")
+        assert math.sqrt((V * (xg - xo) ** 2).sum() / (V * xo ** 2).sum()) <= 1e-10
