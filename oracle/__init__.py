@@ -158,6 +158,25 @@ class Oracle:
                                               _p(c_loc), _p(x_ext), _p(y)))
         return y
 
+    def apply_block(self, i0, nl, j0, ntl, kappa_ext, c_loc, x_ext):
+        """(r, theta) block operator; *_ext carry one ghost plane / row per side."""
+        x_ext = _f64(x_ext)
+        npp = self.shape[2]
+        ncomp = x_ext.size // ((nl + 2) * (ntl + 2) * npp)
+        y = np.empty((ncomp, nl, ntl, npp))
+        kappa_ext, c_loc = _f64(kappa_ext), _f64(c_loc)
+        self._chk(lib().mas_ref_op_apply_block(C.byref(self.g), i0, nl, j0, ntl, ncomp,
+                                               _p(kappa_ext), _p(c_loc), _p(x_ext), _p(y)))
+        return y
+
+    def dot_block(self, i0, nl, j0, ntl, a, b):
+        a, b = _f64(a), _f64(b)
+        out = C.c_double()
+        ncomp = a.size // (nl * ntl * self.shape[2])
+        self._chk(lib().mas_ref_dot_block(C.byref(self.g), i0, nl, j0, ntl, ncomp, _p(a), _p(b),
+                                          C.byref(out)))
+        return out.value
+
     def dot_slab(self, i0, nl, a, b):
         a, b = _f64(a), _f64(b)
         plane = self.shape[1] * self.shape[2]

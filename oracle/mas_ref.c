@@ -442,6 +442,91 @@ int mas_ref_op_apply_slab(const mas_ref_grid* g, int i0, int nl, int ncomp,
     return MAS_REF_OK;
 }
 
+/* (r, theta) block [i0,i0+nl) x [j0,j0+ntl) of the global grid (SURVEY §8(f)
+ * NEXT-3, the north_star's "slabs in r (and in theta where needed)"): the same
+ * cell_L as mas_ref_op_apply, with the neighbour values read from the
+ * block's extended arrays (one ghost plane / row on each side).  Face kinds,
+ * metrics and volumes use the GLOBAL indices (i, j), so a face on a block
+ * edge is an interior face and only the global r-boundaries, poles and theta
+ * walls are boundary faces (readings R3, R5). */
+int mas_ref_op_apply_block(const mas_ref_grid* g, int i0, int nl, int j0, int ntl, int ncomp,
+                           const double* kappa_ext, const double* c,
+                           const double* x_ext, double* y) {
+    tables T;
+    size_t te, pe, Ne, pl, Nl;
+    int il;
+    if (!g || !kappa_ext || !x_ext || !y || ncomp < 1 || nl < 1 || ntl < 1 || i0 < 0 || j0 < 0 ||
+        i0 + nl > g->nr || j0 + ntl > g->nt || tables_make(g, &T))
+        return MAS_REF_ERR_ARG;
+    te = (size_t)g->np;                 /* ext row stride   */
+    pe = (size_t)(ntl + 2) * g->np;     /* ext plane stride */
+    Ne = pe * (nl + 2);
+    pl = (size_t)ntl * g->np;
+    Nl = pl * nl;
+#pragma omp parallel for schedule(static)
+    for (il = 0; il < nl; il++) {
+        int i = i0 + il, jl, k, m, kind[6], np = g->np;
+        double gf[6], kN[6], uN[6];
+        for (jl = 0; jl < ntl; jl++) {
+            int j = j0 + jl;
+            face_kinds(g, i, j, kind);
+            for (k = 0; k < np; k++) {
+                size_t Pe = (size_t)(il + 1) * pe + (size_t)(jl + 1) * te + k;
+                size_t Pl = (size_t)il * pl + (size_t)jl * np + k;
+                size_t row = (size_t)(il + 1) * pe + (size_t)(jl + 1) * te;
+                size_t km = row + (k + np - 1) % np, kp = row + (k + 1) % np;
+                double V = cell_V(g, &T, i, j, k);
+                face_geoms(g, &T, i, j, k, kind, gf);
+                kN[0] = kappa_ext[Pe - pe];
+                kN[1] = kappa_ext[Pe + pe];
+                kN[2] = (kind[2] == FACE_INTERIOR) ? kappa_ext[Pe - te] : 0.0;
+                kN[3] = (kind[3] == FACE_INTERIOR) ? kappa_ext[Pe + te] : 0.0;
+                kN[4] = kappa_ext[km];
+                kN[5] = kappa_ext[kp];
+                for (m = 0; m < ncomp; m++) {
+                    const double* u = x_ext + (size_t)m * Ne;
+                    uN[0] = u[Pe - pe];
+                    uN[1] = u[Pe + pe];
+                    uN[2] = (kind[2] == FACE_INTERIOR) ? u[Pe - te] : 0.0;
+                    uN[3] = (kind[3] == FACE_INTERIOR) ? u[Pe + te] : 0.0;
+                    uN[4] = u[km];
+                    uN[5] = u[kp];
+                    y[(size_t)m * Nl + Pl] =
+                        cell_L(V, c ? c[Pl] : 0.0, kappa_ext[Pe], u[Pe], kind, gf, kN, uN);
+                }
+            }
+        }
+    }
+    tables_free(&T);
+    return MAS_REF_OK;
+}
+
+/* Per-block partial of <a,b>_V (a, b: [ncomp][nl][ntl][np]), summed per
+ * r-plane in (j,k) order, then planes, then components. */
+int mas_ref_dot_block(const mas_ref_grid* g, int i0, int nl, int j0, int ntl, int ncomp,
+                      const double* a, const double* b, double* out) {
+    tables T;
+    size_t pl, Nl;
+    int il, jl, k, m;
+    double s = 0.0;
+    if (!g || !a || !b || !out || nl < 1 || ntl < 1 || tables_make(g, &T)) return MAS_REF_ERR_ARG;
+    pl = (size_t)ntl * g->np;
+    Nl = pl * nl;
+    for (m = 0; m < ncomp; m++)
+        for (il = 0; il < nl; il++) {
+            double ps = 0.0;
+            for (jl = 0; jl < ntl; jl++)
+                for (k = 0; k < g->np; k++) {
+                    size_t P = (size_t)m * Nl + (size_t)il * pl + (size_t)jl * g->np + k;
+                    ps += cell_V(g, &T, i0 + il, j0 + jl, k) * a[P] * b[P];
+                }
+            s += ps;
+        }
+    tables_free(&T);
+    *out = s;
+    return MAS_REF_OK;
+}
+
 int mas_ref_dot_slab(const mas_ref_grid* g, int i0, int nl, int ncomp,
                      const double* a, const double* b, double* out) {
     tables T;

@@ -83,6 +83,16 @@ int mas_ref_op_apply_slab(const mas_ref_grid* g, int i0, int nl, int ncomp,
                           const double* kappa_ext, const double* c,
                           const double* x_ext, double* y);
 
+/* (r, theta) block [i0,i0+nl) x [j0,j0+ntl): kappa_ext [nl+2][ntl+2][np] and
+ * x_ext [ncomp][nl+2][ntl+2][np] carry one ghost plane / theta row on each side
+ * (ignored where the face is a global boundary, pole or wall); c [nl][ntl][np],
+ * y [ncomp][nl][ntl][np].  mas_ref_dot_block: the block's partial <a,b>_V. */
+int mas_ref_op_apply_block(const mas_ref_grid* g, int i0, int nl, int j0, int ntl, int ncomp,
+                           const double* kappa_ext, const double* c,
+                           const double* x_ext, double* y);
+int mas_ref_dot_block(const mas_ref_grid* g, int i0, int nl, int j0, int ntl, int ncomp,
+                      const double* a, const double* b, double* out);
+
 /* Per-slab partial of <a,b>_V over planes [i0,i0+nl) (a,b interior, nl planes). */
 int mas_ref_dot_slab(const mas_ref_grid* g, int i0, int nl, int ncomp,
                      const double* a, const double* b, double* out);

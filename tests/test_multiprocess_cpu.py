@@ -167,3 +167,138 @@ def test_gloo_r_slab_protocol(world):
     assert res[0]["matvec_bitwise"]
     it, ito, err = res[0]["pcg"]
     assert abs(it - ito) <= 1 and err <= 1e-10, (it, ito, err)
+
+
+# ---------------------------------------------------------------------------
+# (r, theta) decomposition (NEXT-3): ranks = pr x ptheta, theta fastest.  The
+# r-seams go to rank -/+ ptheta, the theta-ghost rows (packed [comp][i][phi])
+# to rank -/+ 1 within the r-slab, as in the library (capi.cpp tseams).
+# ---------------------------------------------------------------------------
+def block_exchange(ext, nl, ntl, rank, pr, pt):
+    """ext: [ncomp, nl+2, ntl+2, np] with the block at [1:nl+1, 1:ntl+1]."""
+    rr, rt = divmod(rank, pt)
+    reqs, recv = [], {}
+
+    def post(send, peer, key, like):
+        reqs.append(dist.isend(send.contiguous(), peer))
+        recv[key] = torch.empty_like(like)
+        reqs.append(dist.irecv(recv[key], peer))
+
+    inner = ext[:, :, 1:ntl + 1]
+    if rr > 0:
+        post(inner[:, 1], rank - pt, "rlo", inner[:, 0])
+    if rr < pr - 1:
+        post(inner[:, nl], rank + pt, "rhi", inner[:, 0])
+    rows = ext[:, 1:nl + 1]
+    if rt > 0:
+        post(rows[:, :, 1], rank - 1, "tlo", rows[:, :, 0])
+    if rt < pt - 1:
+        post(rows[:, :, ntl], rank + 1, "thi", rows[:, :, 0])
+    for q in reqs:
+        q.wait()
+    if "rlo" in recv:
+        ext[:, 0, 1:ntl + 1] = recv["rlo"]
+    if "rhi" in recv:
+        ext[:, nl + 1, 1:ntl + 1] = recv["rhi"]
+    if "tlo" in recv:
+        ext[:, 1:nl + 1, 0] = recv["tlo"]
+    if "thi" in recv:
+        ext[:, 1:nl + 1, ntl + 1] = recv["thi"]
+
+
+def worker_2d(rank, world, pt, port, q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    import sys
+    sys.path.insert(0, ROOT)
+    import oracle
+    from paper_conf_ipps_caplansl23_b200 import maspcg as M
+    from paper_conf_ipps_caplansl23_b200 import workloads as W
+    out = {}
+    try:
+        pr = world // pt
+        rr, rt = divmod(rank, pt)
+        prob = W.viscosity_problem(6, 11, 16, warm=False)
+        prob.kappa = prob.kappa * 40.0
+        nr, nt, np_ = prob.shape
+        i0, nl = M.mas_partition(nr, pr, rr)
+        j0, ntl = M.mas_partition(nt, pt, rt)
+        blk = (slice(i0, i0 + nl), slice(j0, j0 + ntl))
+        o = oracle.Oracle.for_problem(prob)
+        x = W.random_field((3,) + prob.shape, 42)
+
+        def ext_of(a):  # a: [ncomp, nl, ntl, np] block -> exchanged ext
+            e = torch.zeros((a.shape[0], nl + 2, ntl + 2, np_), dtype=torch.float64)
+            e[:, 1:nl + 1, 1:ntl + 1] = torch.from_numpy(np.ascontiguousarray(a))
+            block_exchange(e, nl, ntl, rank, pr, pt)
+            return e.numpy()
+
+        kext = ext_of(prob.kappa[None][(slice(None),) + blk])[0]
+        c = prob.c[blk]
+        y = o.apply_block(i0, nl, j0, ntl, kext, c, ext_of(x[(slice(None),) + blk]))
+        yall = [None] * world
+        dist.all_gather_object(yall, (i0, nl, j0, ntl, y))
+        if rank == 0:
+            yfull = np.full((3,) + prob.shape, np.nan)
+            for a, n, b, m, yb in yall:
+                yfull[:, a:a + n, b:b + m] = yb
+            out["matvec_bitwise"] = bool(np.array_equal(yfull, o.apply(prob.kappa, prob.c, x)))
+        # distributed Jacobi-PCG over the blocks (textbook order, SURVEY §8(c))
+        D = o.diag(prob.kappa, prob.c)[blk]
+        f = prob.f[(slice(None),) + blk]
+        dot = lambda a, b: allsum(o.dot_block(i0, nl, j0, ntl, a, b))
+        bn = math.sqrt(dot(f, f))
+        xs = np.zeros_like(f)
+        r = f.copy()
+        p = r / D[None]
+        rho = dot(r, p)
+        it = 0
+        for k in range(1, 500):
+            qv = o.apply_block(i0, nl, j0, ntl, kext, c, ext_of(p))
+            alpha = rho / dot(p, qv)
+            xs += alpha * p
+            r -= alpha * qv
+            if math.sqrt(dot(r, r)) <= prob.tol * bn:
+                it = k
+                break
+            z = r / D[None]
+            rn = dot(r, z)
+            p = z + (rn / rho) * p
+            rho = rn
+        xall = [None] * world
+        dist.all_gather_object(xall, (i0, nl, j0, ntl, xs, it))
+        if rank == 0:
+            xfull = np.full((3,) + prob.shape, np.nan)
+            for a, n, b, m, xb, _ in xall:
+                xfull[:, a:a + n, b:b + m] = xb
+            rc, xo, ito, _, _ = o.pcg(prob.kappa, prob.c, prob.f, np.zeros_like(prob.f), prob.tol, 500)
+            V = o.volumes()[None]
+            out["pcg"] = (it, ito, math.sqrt((V * (xfull - xo) ** 2).sum() / (V * xo ** 2).sum()),
+                          {t[5] for t in xall})
+        q.put((rank, out))
+    except Exception as e:  # surface errors to the parent
+        q.put((rank, {"error": repr(e)}))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world,pt", [(2, 2), (4, 2)])
+def test_gloo_r_theta_block_protocol(world, pt):
+    import oracle
+    oracle.build()
+    from paper_conf_ipps_caplansl23_b200 import build as B
+    B.build()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = free_port()
+    procs = [ctx.Process(target=worker_2d, args=(r, world, pt, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = dict(q.get(timeout=300) for _ in range(world))
+    for p in procs:
+        p.join(timeout=60)
+    for r in range(world):
+        assert "error" not in res[r], res[r]
+    assert res[0]["matvec_bitwise"]
+    it, ito, err, its = res[0]["pcg"]
+    assert len(its) == 1 and abs(it - ito) <= 1 and err <= 1e-10, (it, ito, err, its)

@@ -387,3 +387,40 @@ def test_partition_tiles_the_r_range(oracle_mod):
                 assert a + n == b
             assert parts[-1][0] + parts[-1][1] == nr
             assert max(n for _, n in parts) - min(n for _, n in parts) <= 1
+
+
+# ---------------------------------------------------------------------------
+# decomposition: (r, theta) blocks == monolithic (NEXT-3)
+# ---------------------------------------------------------------------------
+def block_ext(a, i0, nl, j0, ntl):
+    """[.., nl+2, ntl+2, np] copy of a block with one ghost plane / row per
+    side from the global array (zeros beyond the global index range)."""
+    nr, nt = a.shape[-3], a.shape[-2]
+    ext = np.zeros(a.shape[:-3] + (nl + 2, ntl + 2, a.shape[-1]))
+    ilo, ihi = max(i0 - 1, 0), min(i0 + nl + 1, nr)
+    jlo, jhi = max(j0 - 1, 0), min(j0 + ntl + 1, nt)
+    ext[..., ilo - (i0 - 1):ihi - (i0 - 1), jlo - (j0 - 1):jhi - (j0 - 1), :] = \
+        a[..., ilo:ihi, jlo:jhi, :]
+    return ext
+
+
+@pytest.mark.parametrize("pr,pt", [(1, 2), (2, 2), (3, 3), (1, 6)])
+@pytest.mark.parametrize("bc", [(0, 1), (1, 1)])
+def test_block_apply_bitwise(oracle_mod, pr, pt, bc):
+    shape = (9, 13, 8)
+    m = W.stretched_mesh(*shape)
+    o = oracle_mod.Oracle(m, *bc)
+    kappa, c = rand_coeffs(shape, 22)
+    x = np.random.default_rng(23).standard_normal((3,) + shape)
+    y = o.apply(kappa, c, x)
+    dots = []
+    for rr in range(pr):
+        i0, nl = oracle_mod.partition(shape[0], pr, rr)
+        for rt in range(pt):
+            j0, ntl = oracle_mod.partition(shape[1], pt, rt)
+            yb = o.apply_block(i0, nl, j0, ntl, block_ext(kappa, i0, nl, j0, ntl),
+                               c[i0:i0 + nl, j0:j0 + ntl], block_ext(x, i0, nl, j0, ntl))
+            assert np.array_equal(yb, y[:, i0:i0 + nl, j0:j0 + ntl])
+            xb = np.ascontiguousarray(x[:, i0:i0 + nl, j0:j0 + ntl])
+            dots.append(o.dot_block(i0, nl, j0, ntl, xb, xb))
+    assert abs(sum(dots) - o.dot(x, x)) <= 1e-14 * o.dot(x, x)
