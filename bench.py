@@ -348,18 +348,22 @@ def main():
         pin = lambda a: torch.from_numpy(np.ascontiguousarray(a)).pin_memory()
         hk, hc, hf, hx0 = pin(prob.kappa[sl]), pin(prob.c[sl]), rhs.cpu().pin_memory(), \
             pin(prob.x0[slc])
-        hx = hx0.clone().pin_memory()
         ksteps = max(1, min(args.steps, 2))
+        # one pinned x0 per step (the solve overwrites x in place), filled
+        # before the timed region; one untimed warm-up step allocates the
+        # library's host-staging buffers
+        hxs = [hx0.clone().pin_memory() for _ in range(ksteps + 1)]
+        op.update(hk, hc)
+        op.solve(hf, hxs[-1], args.tol, maxit)
         torch.cuda.synchronize()
         if world > 1:
             dist.barrier()
         h0, h1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         h0.record(stream)
         e2e_iters = 0
-        for _ in range(ksteps):
+        for sidx in range(ksteps):
             op.update(hk, hc)
-            hx.copy_(hx0)
-            st, it, rel, _ = op.solve(hf, hx, args.tol, maxit)
+            st, it, rel, _ = op.solve(hf, hxs[sidx], args.tol, maxit)
             e2e_iters += it
         h1.record(stream)
         torch.cuda.synchronize()
@@ -371,7 +375,8 @@ def main():
         h2d = (2 + 2 * nc) * cells_local * 8
         e2e = {"value": e2e_iters / (te / 1e3), "unit": UNIT, "h2d_bytes_per_step": h2d,
                "d2h_bytes_per_step": nc * cells_local * 8,
-               "note": "pinned host kappa, c, rhs, x0 -> device inside the timed region; x -> host"}
+               "note": "pinned host kappa, c, rhs, x0 -> device inside the timed region; x -> host; "
+                       "1 untimed warm-up step"}
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
