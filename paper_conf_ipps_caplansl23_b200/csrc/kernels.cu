@@ -374,6 +374,43 @@ __device__ __forceinline__ void trow_issue(const StencilArgs& a, int i, const Ha
     }
 }
 
+// --- L2 prefetch one plane ahead of the register pipeline -----------------
+// The own-tile loads of plane i+2 are issued (into registers) before the
+// stencil of plane i.  Before that, plane i+3's tile rows are prefetched into
+// L2 by the bulk-copy engine (one cp.async.bulk.prefetch per (field, row):
+// no registers, no LSU/MIO slots), so the DRAM queue stays fed while the
+// block computes and the register loads mostly hit L2.
+#ifndef MAS_NO_PREFETCH
+#ifndef MAS_PF_DIST
+#define MAS_PF_DIST 3
+#endif
+constexpr int kPfDist = MAS_PF_DIST;  // planes ahead of the stencil plane
+__device__ __forceinline__ void l2_prefetch_row(const double* p, int bytes) {
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;\n" ::"l"(p), "r"(bytes) : "memory");
+}
+template <int MODE, int NC>
+__device__ __forceinline__ void plane_prefetch(const StencilArgs& a, int i, int j0, int k0, int height,
+                                               int width, bool first, bool xupd) {
+    const Geo& g = a.g;
+    // fields: u[NC], po[NC] (PCGA, not first), x[NC] (xupd), dinv (PCGA), kappa, c
+    constexpr int NF = 3 * NC + 3;
+    const int t = threadIdx.x;
+    if (t >= NF * TJ) return;
+    const int f = t / TJ, w = t - f * TJ;
+    if (w >= height) return;
+    const int Nl = (int)g.nl * plane32(g);
+    const int off = i * plane32(g) + (j0 + w) * g.np + k0;
+    const double* base = nullptr;
+    if (f < NC) base = a.u.in + f * Nl;
+    else if (f < 2 * NC) base = (MODE == MODE_PCGA && !first) ? a.pold.in + (f - NC) * Nl : nullptr;
+    else if (f < 3 * NC) base = (MODE == MODE_PCGA && xupd) ? a.x + (f - 2 * NC) * Nl : nullptr;
+    else if (f == 3 * NC) base = MODE == MODE_PCGA ? a.dinv.in : nullptr;
+    else if (f == 3 * NC + 1) base = a.kappa.in;
+    else base = a.c;
+    if (base) l2_prefetch_row(base + off, width * 8);
+}
+#endif
+
 template <int MODE, int NC>
 __device__ __forceinline__ void stage_issue(const StencilArgs& a, int i, int j0, int k0, int height,
                                             int width, const HaloMeta& hm, bool first, bool xupd,
@@ -682,6 +719,12 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
         sgP[2][t] = g.vp[kk];
     }
 
+#ifndef MAS_NO_PREFETCH
+    // the planes the march reaches before its first in-loop prefetch
+    if (NC == 3)
+        for (int ip = ia + 1; ip < min(ia + kPfDist, ib); ip++)
+            plane_prefetch<MODE, NC>(a, ip, j0, k0, height, width, FIRSTK, xupd);
+#endif
     // ---- prologue: planes ia-1 (own cells only) and ia --------------------
     OwnRegs<NC> oc, on;  // own-cell stencil inputs for the current / next plane
     double2 kown = make_double2(0.0, 0.0), kdummy;
@@ -720,6 +763,12 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
             stage_issue<MODE, NC>(a, i + 2, j0, k0, height, width, hm, FIRSTK, xupd && (i + 2 < ib),
                                   i + 2 < ib, i + 2 < ib, S, hst_arr);
         __syncthreads();
+#ifndef MAS_NO_PREFETCH
+        // 3-component kernels only: for the scalar kernel (C2: 256 work items,
+        // under one wave) it measured slower (tools/abtest.sh)
+        if (NC == 3 && i + kPfDist < ib)
+            plane_prefetch<MODE, NC>(a, i + kPfDist, j0, k0, height, width, FIRSTK, xupd);
+#endif
         if (!kIssueEarly && i + 2 <= ib && real_plane(i + 2))
             stage_issue<MODE, NC>(a, i + 2, j0, k0, height, width, hm, FIRSTK, xupd && (i + 2 < ib),
                                   i + 2 < ib, i + 2 < ib, S, hst_arr);
