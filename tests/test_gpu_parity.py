@@ -259,3 +259,25 @@ def test_p2p_transport_one_rank_is_bitwise_identical(mp, mk):
     z = torch.zeros_like(f)
     st3, it3, _, _ = op.solve(z, x, prob.tol, prob.maxit)
     assert (st3, it3) == (mp.MAS_OK, 0) and float(x.abs().max()) == 0.0
+
+
+@pytest.mark.parametrize("mk", ["viscosity", "conduction", "mms"])
+def test_graph_loop_equals_host_loop_bitwise(mp, mk):
+    """The single-GPU solve runs as one CUDA graph (device-side while node);
+    with profiling on, the same kernels are launched one by one from the
+    host.  Both must give the same bits, iteration count and history."""
+    prob = {"viscosity": lambda: W.viscosity_problem(20, 16, 64),
+            "conduction": lambda: W.conduction_problem(40, 16, 32),
+            "mms": lambda: W.mms_problem(16, 24, 32)}[mk]()
+    st, xg, it, rel, hist, op = gpu_solve(mp, prob)
+    f = dev(prob.f)
+    ubi = dev(prob.ub_inner) if prob.ub_inner is not None else None
+    ubo = dev(prob.ub_outer) if prob.ub_outer is not None else None
+    if ubi is not None or ubo is not None:
+        op.dirichlet_rhs(ubi, ubo, f)
+    op.set_profiling(True)
+    x = dev(prob.x0)
+    st2, it2, rel2, hist2 = op.solve(f, x, prob.tol, prob.maxit, True)
+    assert (st2, it2, rel2) == (st, it, rel)
+    np.testing.assert_array_equal(host(x), xg)
+    np.testing.assert_array_equal(np.asarray(hist2), np.asarray(hist))
