@@ -195,6 +195,16 @@ __device__ __forceinline__ double2 ld2(const double* p) {
 __device__ __forceinline__ double2 lds2(const double* p) { return *reinterpret_cast<const double2*>(p); }
 __device__ __forceinline__ void sts2(double* p, double2 v) { *reinterpret_cast<double2*>(p) = v; }
 __device__ __forceinline__ void stg2(double* p, double2 v) { *reinterpret_cast<double2*>(p) = v; }
+// use-once streams of kernel B (r, q: far larger than L2): evict-first loads
+// and stores (A/B: kernel B -3..-5% at C3 and C2; the same hints in kernel A
+// measured +2.6% there, so kernel A keeps the default policy)
+#ifndef MAS_NO_CS
+__device__ __forceinline__ void sts_cs(double* p, double2 v) { __stcs(reinterpret_cast<double2*>(p), v); }
+__device__ __forceinline__ double2 ld_cs(const double* p) { return __ldcs(reinterpret_cast<const double2*>(p)); }
+#else
+__device__ __forceinline__ void sts_cs(double* p, double2 v) { *reinterpret_cast<double2*>(p) = v; }
+__device__ __forceinline__ double2 ld_cs(const double* p) { return *reinterpret_cast<const double2*>(p); }
+#endif
 
 // Values that the stencil phase of a plane needs besides the smem ring.
 template <int NC>
@@ -927,15 +937,15 @@ __global__ void __launch_bounds__(kThreads) k_pcg_b(const StreamArgs a) {
                 double2 r[NC], q[NC];
 #pragma unroll
                 for (int c = 0; c < NC; c++) {
-                    r[c] = ld2(a.r + c * Nl + base + k);
-                    q[c] = ld2(a.q + c * Nl + base + k);
+                    r[c] = ld_cs(a.r + c * Nl + base + k);
+                    q[c] = ld_cs(a.q + c * Nl + base + k);
                 }
 #pragma unroll
                 for (int c = 0; c < NC; c++) {
                     double2 rv = r[c];
                     rv.x = fma(-alpha, q[c].x, rv.x);
                     rv.y = fma(-alpha, q[c].y, rv.y);
-                    *reinterpret_cast<double2*>(a.r + c * Nl + base + k) = rv;
+                    sts_cs(a.r + c * Nl + base + k, rv);
                     const double z0 = di.x * rv.x, z1 = di.y * rv.y;
                     acc[0] += V0 * rv.x * z0 + V1 * rv.y * z1;
                     acc[1] += V0 * rv.x * rv.x + V1 * rv.y * rv.y;
