@@ -198,6 +198,15 @@ __device__ __forceinline__ void stg2(double* p, double2 v) { *reinterpret_cast<d
 // use-once streams of kernel B (r, q: far larger than L2): evict-first loads
 // and stores (A/B: kernel B -3..-5% at C3 and C2; the same hints in kernel A
 // measured +2.6% there, so kernel A keeps the default policy)
+// kernel A's stores (p, q, x): default policy (MAS_A_STCS, streaming stores,
+// measured +2.8% on kernel A)
+__device__ __forceinline__ void stg2a(double* p, double2 v) {
+#ifdef MAS_A_STCS
+    __stcs(reinterpret_cast<double2*>(p), v);
+#else
+    *reinterpret_cast<double2*>(p) = v;
+#endif
+}
 #ifndef MAS_NO_CS
 __device__ __forceinline__ void sts_cs(double* p, double2 v) { __stcs(reinterpret_cast<double2*>(p), v); }
 __device__ __forceinline__ double2 ld_cs(const double* p) { return __ldcs(reinterpret_cast<const double2*>(p)); }
@@ -395,8 +404,17 @@ __device__ __forceinline__ void trow_issue(const StencilArgs& a, int i, const Ha
 #define MAS_PF_DIST 3
 #endif
 constexpr int kPfDist = MAS_PF_DIST;  // planes ahead of the stencil plane
+// evict_last policy on the prefetched lines (A/B: kernel B -2%, kernel A equal)
 __device__ __forceinline__ void l2_prefetch_row(const double* p, int bytes) {
+#ifndef MAS_PF_NORMAL
+    unsigned long long pol;
+    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;\n" : "=l"(pol));
+    asm volatile("cp.async.bulk.prefetch.L2.global.L2::cache_hint [%0], %1, %2;\n" ::"l"(p), "r"(bytes),
+                 "l"(pol)
+                 : "memory");
+#else
     asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;\n" ::"l"(p), "r"(bytes) : "memory");
+#endif
 }
 template <int MODE, int NC>
 __device__ __forceinline__ void plane_prefetch(const StencilArgs& a, int i, int j0, int k0, int height,
@@ -498,12 +516,12 @@ __device__ __forceinline__ void stage_commit(const StencilArgs& a, int i, int j0
                 const int o3 = (int)i * plane32(g) + (int)(j0 + w) * g.np + k0 + kc;
 #pragma unroll
                 for (int c = 0; c < NC; c++) {
-                    stg2(a.pnew + c * Nl + o3, S.R.u[c]);
+                    stg2a(a.pnew + c * Nl + o3, S.R.u[c]);
                     if (xupd) {
                         double2 xv = S.xv[c];
                         xv.x = fma(alpha_prev, S.R.po[c].x, xv.x);
                         xv.y = fma(alpha_prev, S.R.po[c].y, xv.y);
-                        stg2(a.x + c * Nl + o3, xv);
+                        stg2a(a.x + c * Nl + o3, xv);
                     }
                 }
             }
@@ -845,7 +863,7 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
                     acc[1] += V0 * r0 * r0 + V1 * r1 * r1;
                     acc[2] += V0 * r0 * (oc.di.x * r0) + V1 * r1 * (oc.di.y * r1);
                 } else {
-                    stg2(a.out + o, make_double2(L0, L1));
+                    stg2a(a.out + o, make_double2(L0, L1));
                     if (MODE == MODE_PCGA) acc[0] += V0 * u.x * L0 + V1 * u.y * L1;
                 }
             }
