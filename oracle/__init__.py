@@ -185,6 +185,37 @@ class Oracle:
                                          _p(b), C.byref(out)))
         return out.value
 
+    # ---- field-aligned conduction (NEXT-4, readings R21-R26) ----------------
+    def aniso_apply(self, kpar, bhat, x):
+        """y = L_par x (kpar [nr,nt,np], bhat [3,nr,nt,np] at lower corners)."""
+        x = _f64(x)
+        ncomp = x.size // self.N
+        y = np.empty_like(x)
+        kpar, bhat = _f64(kpar), _f64(bhat)
+        self._chk(lib().mas_ref_aniso_apply(C.byref(self.g), ncomp, _p(kpar), _p(bhat), _p(x),
+                                            _p(y)))
+        return y
+
+    def aniso_diag(self, kpar, bhat):
+        D = np.empty(self.shape)
+        kpar, bhat = _f64(kpar), _f64(bhat)
+        self._chk(lib().mas_ref_aniso_diag(C.byref(self.g), _p(kpar), _p(bhat), _p(D)))
+        return D
+
+    def pcg_aniso(self, kappa, c, kpar, bhat, f, x0, tol, maxit):
+        """PCG on L_iso + L_par.  Returns (status, x, iters, relres, res_hist)."""
+        f = _f64(f)
+        x = _f64(x0).copy()
+        ncomp = f.size // self.N
+        kappa, c, kpar, bhat = _f64(kappa), _f64(c), _f64(kpar), _f64(bhat)
+        iters, relres = C.c_int(), C.c_double()
+        hist = np.zeros(maxit + 1)
+        rc = lib().mas_ref_pcg_solve_aniso(C.byref(self.g), ncomp, _p(kappa), _p(c), _p(kpar),
+                                           _p(bhat), _p(f), _p(x), C.c_double(tol), maxit,
+                                           C.byref(iters), C.byref(relres), _p(hist))
+        self._chk(rc)
+        return rc, x, iters.value, relres.value, hist[: iters.value + 1]
+
 
 def partition(nr: int, nranks: int, rank: int):
     i0, nl = C.c_int(), C.c_int()
@@ -196,6 +227,10 @@ def solve_problem(prob, tol=None, maxit=None, x0=None, threads: int = 0, nranks:
     """Full oracle solve of a workloads.Problem: rhs = f + Dirichlet terms."""
     o = Oracle.for_problem(prob, threads)
     f = o.dirichlet_rhs(prob.kappa, prob.f, prob.ub_inner, prob.ub_outer)
+    if prob.kpar is not None:  # field-aligned conduction (NEXT-4)
+        return o.pcg_aniso(prob.kappa, prob.c, prob.kpar, prob.bhat, f,
+                           prob.x0 if x0 is None else x0, prob.tol if tol is None else tol,
+                           prob.maxit if maxit is None else maxit)
     return o.pcg(prob.kappa, prob.c, f, prob.x0 if x0 is None else x0,
                  prob.tol if tol is None else tol, prob.maxit if maxit is None else maxit,
                  nranks=nranks)

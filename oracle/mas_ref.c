@@ -316,9 +316,16 @@ int mas_ref_dot(const mas_ref_grid* g, int ncomp, const double* a, const double*
 /* ---------------------------------------------------------------------------
  * Jacobi-PCG (SURVEY §8(c) "PCG, exact order"; R10 stopping, R11 counting).
  * ------------------------------------------------------------------------- */
-int mas_ref_pcg_solve(const mas_ref_grid* g, int ncomp, const double* kappa,
-                      const double* c, const double* f, double* x, double tol,
-                      int maxit, int* iters, double* relres, double* res_hist) {
+static int aniso_add(const mas_ref_grid* g, int ncomp, const double* kpar,
+                     const double* bhat, const double* x, double* y);
+static int aniso_diag_add(const mas_ref_grid* g, const double* kpar, const double* bhat,
+                          double* D);
+
+/* The PCG loop for L = L_iso (+ L_par when kpar != NULL, NEXT-4). */
+static int pcg_core(const mas_ref_grid* g, int ncomp, const double* kappa,
+                    const double* c, const double* kpar, const double* bhat,
+                    const double* f, double* x, double tol,
+                    int maxit, int* iters, double* relres, double* res_hist) {
     tables T;
     size_t N, n, e;
     double *D, *r, *z, *p, *q;
@@ -336,6 +343,7 @@ int mas_ref_pcg_solve(const mas_ref_grid* g, int ncomp, const double* kappa,
     q = malloc(sizeof(double) * n);
     if (!D || !r || !z || !p || !q) { status = MAS_REF_ERR_ARG; goto done; }
     mas_ref_op_diag(g, kappa, c, D);
+    if (kpar) aniso_diag_add(g, kpar, bhat, D);                  /* D += D_par  */
 
     bn = sqrt(dot_planes(g, &T, 0, g->nr, ncomp, f, f));
     if (bn == 0.0) {
@@ -345,6 +353,7 @@ int mas_ref_pcg_solve(const mas_ref_grid* g, int ncomp, const double* kappa,
         status = MAS_REF_OK; goto done;
     }
     mas_ref_op_apply(g, ncomp, kappa, c, x, r);                  /* r = L x     */
+    if (kpar) aniso_add(g, ncomp, kpar, bhat, x, r);
 #pragma omp parallel for schedule(static)
     for (e = 0; e < n; e++) r[e] = f[e] - r[e];                  /* r = f - L x */
     rn = sqrt(dot_planes(g, &T, 0, g->nr, ncomp, r, r));
@@ -358,6 +367,7 @@ int mas_ref_pcg_solve(const mas_ref_grid* g, int ncomp, const double* kappa,
 
     for (k = 1; k <= maxit; k++) {
         mas_ref_op_apply(g, ncomp, kappa, c, p, q);              /* q = L p     */
+        if (kpar) aniso_add(g, ncomp, kpar, bhat, p, q);
         sigma = dot_planes(g, &T, 0, g->nr, ncomp, p, q);
         if (!(sigma > 0.0) || !isfinite(sigma)) {
             *iters = k; *relres = rn / bn; status = MAS_REF_ERR_BREAKDOWN; goto done;
@@ -382,6 +392,12 @@ done:
     free(D); free(r); free(z); free(p); free(q);
     tables_free(&T);
     return status;
+}
+
+int mas_ref_pcg_solve(const mas_ref_grid* g, int ncomp, const double* kappa,
+                      const double* c, const double* f, double* x, double tol,
+                      int maxit, int* iters, double* relres, double* res_hist) {
+    return pcg_core(g, ncomp, kappa, c, NULL, NULL, f, x, tol, maxit, iters, relres, res_hist);
 }
 
 /* ---------------------------------------------------------------------------
@@ -720,4 +736,173 @@ int mas_ref_op_apply_cells(const mas_ref_grid* g, int ncomp, const double* kappa
     }
     tables_free(&T);
     return MAS_REF_OK;
+}
+
+/* ---------------------------------------------------------------------------
+ * Field-aligned (anisotropic) thermal conduction — SURVEY §8(f) NEXT-4.
+ * The paper names MAS's thermal conduction only through its test problem
+ * ("thermodynamic MHD") and the implicit parabolic Krylov solvers
+ * of ref. [25]; it prints no formula.  Readings (DESIGN.md
+ * §3.4, R21-R26):
+ *
+ *   R21  L = L_iso + L_par with L_par u = -div(kpar b (b . grad u)), written in
+ *        the symmetric corner ("dual-cell") form
+ *          V_P (L_par u)_P = sum_{corners c of P} W_c kpar_c (b_c . g_c(u))
+ *                                                      (b_c . d g_c / d u_P)
+ *        (so V L_par = G^T W K G is symmetric positive semi-definite).
+ *   R22  g_c = (d_r u, (1/r) d_theta u, (1/(r sin theta)) d_phi u) at the
+ *        corner c = (rF_I, tF_J, pF_K) from its 8 cells (I-1+a, J-1+b,
+ *        K-1+e mod np), a,b,e in {0,1}: each component is the mean of the 4
+ *        cell-centre differences across the corner in that direction,
+ *          g_r   = sum_{b,e} (u[I][..] - u[I-1][..]) / (4 hr_I)
+ *          g_t   = sum_{a,e} (u[..][J][..] - u[..][J-1][..]) / (4 rF_I ht_J)
+ *          g_p   = sum_{a,b} (u[..][..][K] - u[..][..][K-1]) / (4 rF_I sF_J hp_K)
+ *   R23  dual volume W_c = rF_I^2 sin(tF_J) hr_I ht_J hp_K (midpoint FD, R4).
+ *   R24  corners on the domain boundary (r faces 0 and nr, theta faces 0 and
+ *        nt: poles and walls) carry no weight: no field-aligned flux leaves
+ *        the domain; the boundary conditions stay with L_iso.
+ *   R25  kpar and b are given AT CORNERS, stored at the cell whose lower
+ *        corner it is: kpar[i][j][k] belongs to (rF_i, tF_j, pF_k); entries
+ *        with i = 0 or j = 0 are ignored.  b = (b_r, b_theta, b_phi) is used as
+ *        given (not renormalised), layout bhat[3][nr][nt][np].
+ *   R26  the Jacobi diagonal adds (1/V_P) sum_c W_c kpar_c (b_c . dg_c/du_P)^2.
+ * ------------------------------------------------------------------------- */
+static int corner_live(const mas_ref_grid* g, int I, int J) {          /* R24 */
+    return I >= 1 && I <= g->nr - 1 && J >= 1 && J <= g->nt - 1;
+}
+
+static double corner_W(const mas_ref_grid* g, const tables* T, int I, int J, int K) { /* R23 */
+    return g->rF[I] * g->rF[I] * T->sF[J] * T->hr[I] * T->ht[J] * T->hp[K];
+}
+
+/* R22: the corner gradient of u (one component, monolithic [nr][nt][np]). */
+static void corner_grad(const mas_ref_grid* g, const tables* T, const double* u, int I, int J,
+                        int K, double gr[3]) {
+    int np = g->np, Km = (K + np - 1) % np, a, b, e;
+    int ii[2] = {I - 1, I}, jj[2] = {J - 1, J}, kk[2] = {Km, K};
+    double sr = 0.0, st = 0.0, sp = 0.0;
+    for (b = 0; b < 2; b++)
+        for (e = 0; e < 2; e++)
+            sr += u[IDX(g, I, jj[b], kk[e])] - u[IDX(g, I - 1, jj[b], kk[e])];
+    for (a = 0; a < 2; a++)
+        for (e = 0; e < 2; e++)
+            st += u[IDX(g, ii[a], J, kk[e])] - u[IDX(g, ii[a], J - 1, kk[e])];
+    for (a = 0; a < 2; a++)
+        for (b = 0; b < 2; b++)
+            sp += u[IDX(g, ii[a], jj[b], K)] - u[IDX(g, ii[a], jj[b], Km)];
+    gr[0] = sr / (4.0 * T->hr[I]);
+    gr[1] = st / (4.0 * g->rF[I] * T->ht[J]);
+    gr[2] = sp / (4.0 * g->rF[I] * T->sF[J] * T->hp[K]);
+}
+
+/* d g_c / d u_Q for the cell Q = (I-1+a, J-1+b, K-1+e) of corner c. */
+static void corner_dgrad(const mas_ref_grid* g, const tables* T, int I, int J, int K, int a,
+                         int b, int e, double d[3]) {
+    d[0] = (a ? 1.0 : -1.0) / (4.0 * T->hr[I]);
+    d[1] = (b ? 1.0 : -1.0) / (4.0 * g->rF[I] * T->ht[J]);
+    d[2] = (e ? 1.0 : -1.0) / (4.0 * g->rF[I] * T->sF[J] * T->hp[K]);
+}
+
+/* R21 / R26 for cell (i,j,k): sum over its 8 corners of W kpar (b.g)(b.dg)
+ * (want_diag: W kpar (b.dg)^2), divided by V_P.  u may be NULL for the diagonal. */
+static double aniso_cell(const mas_ref_grid* g, const tables* T, const double* kpar,
+                         const double* bhat, const double* u, int i, int j, int k, int want_diag) {
+    size_t N = (size_t)g->nr * g->nt * g->np;
+    double acc = 0.0;
+    int a, b, e;
+    for (a = 0; a < 2; a++)           /* a = 1: the corner plane I = i (cell above it) */
+        for (b = 0; b < 2; b++)
+            for (e = 0; e < 2; e++) {
+                int I = a ? i : i + 1, J = b ? j : j + 1, K = e ? k : (k + 1) % g->np;
+                size_t C;
+                double W, kc, bv[3], d[3], bd, gr[3];
+                if (!corner_live(g, I, J)) continue;
+                C = IDX(g, I, J, K);
+                W = corner_W(g, T, I, J, K);
+                kc = kpar[C];
+                bv[0] = bhat[C]; bv[1] = bhat[N + C]; bv[2] = bhat[2 * N + C];
+                corner_dgrad(g, T, I, J, K, a, b, e, d);
+                bd = bv[0] * d[0] + bv[1] * d[1] + bv[2] * d[2];
+                if (want_diag) {
+                    acc += W * kc * bd * bd;
+                } else {
+                    corner_grad(g, T, u, I, J, K, gr);
+                    acc += W * kc * (bv[0] * gr[0] + bv[1] * gr[1] + bv[2] * gr[2]) * bd;
+                }
+            }
+    return acc / cell_V(g, T, i, j, k);
+}
+
+static int aniso_check(const mas_ref_grid* g, const double* kpar, const double* bhat) {
+    return g && kpar && bhat && g->nr >= 1 && g->nt >= 1 && g->np >= 2;
+}
+
+int mas_ref_aniso_apply(const mas_ref_grid* g, int ncomp, const double* kpar,
+                        const double* bhat, const double* x, double* y) {
+    tables T;
+    size_t N;
+    int i;
+    if (!aniso_check(g, kpar, bhat) || !x || !y || ncomp < 1 || tables_make(g, &T))
+        return MAS_REF_ERR_ARG;
+    N = (size_t)g->nr * g->nt * g->np;
+#pragma omp parallel for schedule(static)
+    for (i = 0; i < g->nr; i++) {
+        int j, k, m;
+        for (m = 0; m < ncomp; m++)
+            for (j = 0; j < g->nt; j++)
+                for (k = 0; k < g->np; k++)
+                    y[(size_t)m * N + IDX(g, i, j, k)] =
+                        aniso_cell(g, &T, kpar, bhat, x + (size_t)m * N, i, j, k, 0);
+    }
+    tables_free(&T);
+    return MAS_REF_OK;
+}
+
+int mas_ref_aniso_diag(const mas_ref_grid* g, const double* kpar, const double* bhat,
+                       double* D) {
+    tables T;
+    int i;
+    if (!aniso_check(g, kpar, bhat) || !D || tables_make(g, &T)) return MAS_REF_ERR_ARG;
+#pragma omp parallel for schedule(static)
+    for (i = 0; i < g->nr; i++) {
+        int j, k;
+        for (j = 0; j < g->nt; j++)
+            for (k = 0; k < g->np; k++)
+                D[IDX(g, i, j, k)] = aniso_cell(g, &T, kpar, bhat, NULL, i, j, k, 1);
+    }
+    tables_free(&T);
+    return MAS_REF_OK;
+}
+
+/* y += L_par x (the PCG's full operator is L_iso + L_par, summed per cell). */
+static int aniso_add(const mas_ref_grid* g, int ncomp, const double* kpar,
+                     const double* bhat, const double* x, double* y) {
+    size_t n = (size_t)g->nr * g->nt * g->np * ncomp, e;
+    double* t = malloc(sizeof(double) * n);
+    int rc;
+    if (!t) return MAS_REF_ERR_ARG;
+    rc = mas_ref_aniso_apply(g, ncomp, kpar, bhat, x, t);
+    for (e = 0; e < n; e++) y[e] += t[e];
+    free(t);
+    return rc;
+}
+
+static int aniso_diag_add(const mas_ref_grid* g, const double* kpar, const double* bhat,
+                          double* D) {
+    size_t n = (size_t)g->nr * g->nt * g->np, e;
+    double* t = malloc(sizeof(double) * n);
+    int rc;
+    if (!t) return MAS_REF_ERR_ARG;
+    rc = mas_ref_aniso_diag(g, kpar, bhat, t);
+    for (e = 0; e < n; e++) D[e] += t[e];
+    free(t);
+    return rc;
+}
+
+int mas_ref_pcg_solve_aniso(const mas_ref_grid* g, int ncomp, const double* kappa,
+                            const double* c, const double* kpar, const double* bhat,
+                            const double* f, double* x, double tol, int maxit, int* iters,
+                            double* relres, double* res_hist) {
+    if (!aniso_check(g, kpar, bhat)) return MAS_REF_ERR_ARG;
+    return pcg_core(g, ncomp, kappa, c, kpar, bhat, f, x, tol, maxit, iters, relres, res_hist);
 }

@@ -115,6 +115,22 @@ int mas_ref_op_apply_cells(const mas_ref_grid* g, int ncomp, const double* kappa
  * planes starting at i0_p. */
 void mas_ref_partition(int nr, int nranks, int rank, int* i0, int* nl);
 
+/* Field-aligned (anisotropic) conduction, readings
+ * R21-R26 (mas_ref.c): y = L_par x with
+ *   V_P (L_par u)_P = sum_{corners c of P} W_c kpar_c (b_c.g_c(u)) (b_c.dg_c/du_P),
+ * kpar [nr][nt][np] and bhat [3][nr][nt][np] given at the LOWER corner
+ * (rF_i, tF_j, pF_k) of cell (i,j,k); boundary corners carry no weight. */
+int mas_ref_aniso_apply(const mas_ref_grid* g, int ncomp, const double* kpar,
+                        const double* bhat, const double* x, double* y);
+/* Diagonal of L_par (R26). */
+int mas_ref_aniso_diag(const mas_ref_grid* g, const double* kpar, const double* bhat,
+                       double* D);
+/* The Jacobi-PCG of mas_ref_pcg_solve on L = L_iso + L_par, D = D_iso + D_par. */
+int mas_ref_pcg_solve_aniso(const mas_ref_grid* g, int ncomp, const double* kappa,
+                            const double* c, const double* kpar, const double* bhat,
+                            const double* f, double* x, double tol, int maxit, int* iters,
+                            double* relres, double* res_hist);
+
 #ifdef __cplusplus
 }
 #endif

@@ -66,6 +66,10 @@ class Problem:
     tol: float
     maxit: int
     extra: dict = dataclasses.field(default_factory=dict)
+    # field-aligned conduction (NEXT-4): kpar [nr,nt,np] and bhat [3,nr,nt,np]
+    # given at the LOWER corner (rF_i, tF_j, pF_k) of cell (i,j,k) (reading R25)
+    kpar: Optional[np.ndarray] = None
+    bhat: Optional[np.ndarray] = None
 
     @property
     def shape(self):
@@ -95,20 +99,26 @@ def stretched_mesh(nr: int, nt: int, np_: int, r0: float = 1.0, r1: float = 30.0
     return Mesh(rF=rF, rC=mid(rF), tF=tF, tC=mid(tF), pF=pF, pC=mid(pF))
 
 
-def texture(tC: np.ndarray, pC: np.ndarray, seed: int) -> np.ndarray:
+def texture(tC: np.ndarray, pC: np.ndarray, seed: int, at=None) -> np.ndarray:
     """g(theta,phi) = sum_{m=0..3} sin^m(theta) (a_m cos(theta) + b_m) cos(m phi + c_m),
     a_m, b_m ~ N(0,1), c_m ~ U[0, 2pi), normalised to max|g| = 1 on the cell
-    centres.  Smooth at the poles (sin^m factor)."""
+    centres.  Smooth at the poles (sin^m factor).  at = (t, p): evaluate the
+    same function (same normalisation) at other points, e.g. cell corners."""
     rng = np.random.default_rng(seed)
     am = rng.standard_normal(4)
     bm = rng.standard_normal(4)
     cm = rng.uniform(0.0, 2.0 * math.pi, 4)
-    th = tC[:, None]
-    ph = pC[None, :]
-    g = np.zeros((len(tC), len(pC)))
-    for m in range(4):
-        g += np.sin(th) ** m * (am[m] * np.cos(th) + bm[m]) * np.cos(m * ph + cm[m])
-    return g / np.abs(g).max()
+
+    def ev(t, p):
+        th = t[:, None]
+        ph = p[None, :]
+        g = np.zeros((len(t), len(p)))
+        for m in range(4):
+            g += np.sin(th) ** m * (am[m] * np.cos(th) + bm[m]) * np.cos(m * ph + cm[m])
+        return g
+
+    norm = np.abs(ev(tC, pC)).max()
+    return (ev(tC, pC) if at is None else ev(*at)) / norm
 
 
 def _temperature(r, gT):
@@ -210,6 +220,44 @@ def viscosity_problem(nr=256, nt=256, np_=512, r0=1.0, r1=30.0, R=200.0, D_max=1
                    tol, maxit, extra={"dt": dt})
 
 
+def spiral_dipole_field(r, t, p, omega=0.5, dip=0.3, b0=0.02):
+    """Unit magnetic-field direction b = B/|B| in spherical components
+    (b_r, b_theta, b_phi) for B = split monopole wound into a Parker spiral
+    (B_r = 1/r^2, B_phi = -omega sin(theta)/r) + a dipole of strength dip +
+    a uniform b0 x-hat field (breaks the axisymmetry).  Every term is a smooth
+    Cartesian field, so b is smooth at the poles (NEXT-4 workload input)."""
+    st, ct, sp, cp = np.sin(t), np.cos(t), np.sin(p), np.cos(p)
+    Br = 1.0 / r ** 2 + 2.0 * dip * ct / r ** 3 + b0 * st * cp
+    Bt = dip * st / r ** 3 + b0 * ct * cp
+    Bp = -omega * st / r - b0 * sp
+    n = np.sqrt(Br * Br + Bt * Bt + Bp * Bp)
+    return np.stack([Br / n, Bt / n, Bp / n])
+
+
+def aniso_conduction_problem(nr=128, nt=128, np_=256, r0=1.0, r1=30.0, R=200.0,
+                             D_max=1000.0, eps_iso=1e-2, tol=1e-12, maxit=20000,
+                             warm=True) -> Problem:
+    """C2a: field-aligned thermal conduction.  As C2, but
+    the conductivity is split into kpar = T^(5/2) along b (at the cell corners,
+    reading R25) and an isotropic kappa = eps_iso T^(5/2) at the cell centres;
+    b from spiral_dipole_field.  Same dt rule, c, boundary data, f and x0 as C2."""
+    prob = conduction_problem(nr, nt, np_, r0, r1, R, D_max, tol, maxit, warm)
+    m = prob.mesh
+    gT = texture(m.tC, m.pC, 1, at=(m.tF[:-1], m.pF[:-1]))
+    rc = m.rF[:-1][:, None, None]
+    Tc = _temperature(rc, gT[None])
+    tc = m.tF[:-1][None, :, None]
+    pc = m.pF[:-1][None, None, :]
+    bhat = spiral_dipole_field(rc, tc, pc)
+    shape = (nr, nt, np_)
+    prob.kpar = np.ascontiguousarray(np.broadcast_to(Tc ** 2.5, shape))
+    prob.bhat = np.ascontiguousarray(np.broadcast_to(bhat, (3,) + shape))
+    prob.kappa = eps_iso * prob.kappa
+    prob.name = "C2a-aniso-conduction"
+    prob.extra["eps_iso"] = eps_iso
+    return prob
+
+
 @dataclasses.dataclass
 class LongRun:
     """C5: repeated implicit steps of conduction then viscosity,
@@ -257,9 +305,10 @@ CONFIGS = {
     "C1": dict(kind="mms", nr=16, nt=24, np_=32),
     "C2": dict(kind="conduction", nr=128, nt=128, np_=256),
     "C3": dict(kind="viscosity", nr=256, nt=256, np_=512),
+    "C2a": dict(kind="aniso", nr=128, nt=128, np_=256),
 }
 
 
 def make(kind: str, **kw) -> Problem:
     return {"mms": mms_problem, "conduction": conduction_problem,
-            "viscosity": viscosity_problem}[kind](**kw)
+            "viscosity": viscosity_problem, "aniso": aniso_conduction_problem}[kind](**kw)
