@@ -49,6 +49,9 @@ CONFIGS = {
     # the whole C4 problem of 8 GPUs (268 M cells) on one B200
     "C4x8": ("viscosity", 2048, 256, 512),
     "C2": ("conduction", 128, 128, 256),
+    # C2 with field-aligned conduction: kernel A, the
+    # L_par kernel and kernel B per iteration (one GPU)
+    "C2a": ("aniso", 128, 128, 256),
     "C1": ("mms", 16, 24, 32),
 }
 # algorithmic bytes per cell per iteration: kernel A reads
@@ -58,6 +61,11 @@ def alg_bytes_per_cell(ncomp):
     a = 8 * (3 * ncomp + 3 + 3 * ncomp)
     b = 8 * (2 * ncomp + 1 + ncomp)
     return a, b
+
+
+# the L_par kernel (NEXT-4, scalar): reads p_k and the 3 corner coefficients,
+# reads and writes q
+ANISO_BYTES_PER_CELL = 8 * (1 + 3 + 2)
 
 
 def load_peaks():
@@ -146,13 +154,21 @@ def oracle_sample(prob, iters: int, threads: int):
     import oracle
     o = oracle.Oracle.for_problem(prob, threads)
     f = o.dirichlet_rhs(prob.kappa, prob.f, prob.ub_inner, prob.ub_outer)
+    run = oracle_runner(o, prob, f)
     t0 = time.perf_counter()
-    o.pcg(prob.kappa, prob.c, f, prob.x0, 0.0, 1)
+    run(1)
     t1 = time.perf_counter()
-    o.pcg(prob.kappa, prob.c, f, prob.x0, 0.0, 1 + iters)
+    run(1 + iters)
     t2 = time.perf_counter()
     per_iter = max((t2 - t1) - (t1 - t0), 1e-9) / iters
     return 1.0 / per_iter, per_iter
+
+
+def oracle_runner(o, prob, f):
+    """k fixed oracle PCG iterations (tol = 0) on the problem's operator."""
+    if prob.kpar is not None:
+        return lambda k: o.pcg_aniso(prob.kappa, prob.c, prob.kpar, prob.bhat, f, prob.x0, 0.0, k)
+    return lambda k: o.pcg(prob.kappa, prob.c, f, prob.x0, 0.0, k)
 
 
 def run_reference(args):
@@ -168,11 +184,12 @@ def run_reference(args):
     o = oracle.Oracle.for_problem(prob, cores)
     f = o.dirichlet_rhs(prob.kappa, prob.f, prob.ub_inner, prob.ub_outer)
     per_step_iters = 2
+    run = oracle_runner(o, prob, f)
     for _ in range(args.warmup):
-        o.pcg(prob.kappa, prob.c, f, prob.x0, 0.0, per_step_iters)
+        run(per_step_iters)
     t0 = time.perf_counter()
     for _ in range(args.steps):
-        o.pcg(prob.kappa, prob.c, f, prob.x0, 0.0, per_step_iters)
+        run(per_step_iters)
     dt = time.perf_counter() - t0
     value = args.steps * per_step_iters / dt
     sample = (f"{args.config} full grid {prob.shape}, ncomp {prob.ncomp}: {per_step_iters} fixed "
@@ -250,6 +267,13 @@ def main():
     x0 = to_dev(prob.x0[slc])
     x = x0.clone()
     op = M.Operator(grid, nc, kappa, cmass, prob.bc_inner, prob.bc_outer)
+    aniso = prob.kpar is not None
+    if aniso:
+        if world > 1:
+            raise SystemExit("C2a (field-aligned conduction) is single-GPU in this version")
+        kpar = to_dev(prob.kpar)
+        bhat = to_dev(prob.bhat)
+        op.set_aniso(kpar, bhat)
     transport = "single-gpu"
     if world > 1:
         transport = "nccl"
@@ -271,6 +295,8 @@ def main():
 
     def step(prof=False):
         op.update(kappa, cmass)           # a2: coefficients + Jacobi diagonal (1 kernel)
+        if aniso:                         # NEXT-4: corner coefficients + their diagonal
+            op.set_aniso(kpar, bhat)
         x.copy_(x0)                       # warm start x0 = v^n (R12)
         st, it, rel, _ = op.solve(rhs, x, args.tol, maxit)
         if st != M.MAS_OK:
@@ -310,7 +336,7 @@ def main():
     # the same K steps again with every kernel A / kernel B launch bracketed by
     # CUDA events on the solve stream (host-driven loop): per-kernel durations
     op.set_profiling(True)
-    ka, kb = [], []
+    ka, kb, kc = [], [], []
     e2, e3 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     e2.record(stream)
     for _ in range(args.steps):
@@ -318,6 +344,7 @@ def main():
         a_ms, b_ms, n = op.kernel_times()
         ka.append(a_ms)
         kb.append(b_ms)
+        kc.append(op.aniso_time())
     e3.record(stream)
     torch.cuda.synchronize()
     op.set_profiling(False)
@@ -334,7 +361,9 @@ def main():
     b_ms = statistics.mean(kb)
     peak, peak_src = load_peaks()
     achieved = a_b * cells_local / (a_ms / 1e3) / 1e9
-    iter_gbs = (a_b + b_b) * cells / (t_ms / 1e3 / iters_total) / 1e9
+    c_b = ANISO_BYTES_PER_CELL if aniso else 0
+    c_ms = statistics.mean(kc)
+    iter_gbs = (a_b + b_b + c_b) * cells / (t_ms / 1e3 / iters_total) / 1e9
     traffic = None
     prof_json = os.path.join(ROOT, "profiles", f"ncu_{args.config}_kernelA.json")
     if os.path.exists(prof_json):
@@ -353,7 +382,11 @@ def main():
         # before the timed region; one untimed warm-up step allocates the
         # library's host-staging buffers
         hxs = [hx0.clone().pin_memory() for _ in range(ksteps + 1)]
+        if aniso:
+            hkp, hb = pin(prob.kpar), pin(prob.bhat)
         op.update(hk, hc)
+        if aniso:
+            op.set_aniso(hkp, hb)
         op.solve(hf, hxs[-1], args.tol, maxit)
         torch.cuda.synchronize()
         if world > 1:
@@ -363,6 +396,8 @@ def main():
         e2e_iters = 0
         for sidx in range(ksteps):
             op.update(hk, hc)
+            if aniso:
+                op.set_aniso(hkp, hb)
             st, it, rel, _ = op.solve(hf, hxs[sidx], args.tol, maxit)
             e2e_iters += it
         h1.record(stream)
@@ -372,10 +407,11 @@ def main():
             tt = torch.tensor([te], device=dev, dtype=torch.float64)
             dist.all_reduce(tt, op=dist.ReduceOp.MAX)
             te = float(tt.item())
-        h2d = (2 + 2 * nc) * cells_local * 8
+        h2d = (2 + 2 * nc + (4 if aniso else 0)) * cells_local * 8
         e2e = {"value": e2e_iters / (te / 1e3), "unit": UNIT, "h2d_bytes_per_step": h2d,
                "d2h_bytes_per_step": nc * cells_local * 8,
-               "note": "pinned host kappa, c, rhs, x0 -> device inside the timed region; x -> host; "
+               "note": "pinned host kappa, c, rhs, x0 (+ kpar, bhat for C2a) -> device inside the "
+                       "timed region; x -> host; "
                        "1 untimed warm-up step"}
 
     cpu = None
@@ -397,8 +433,10 @@ def main():
                        "parallelism": (f"r-slab x{world}" if args.ptheta == 1 or world == 1 else
                                        f"(r,theta) {world // args.ptheta}x{args.ptheta}"),
                        "transport": transport,
-                       "l2": "inputs > L2 (268 MB per field vs 126 MB); no flush",
-                       "step": "mas_op_update + x:=x0 + mas_pcg_solve"},
+                       "l2": (f"no flush: one iteration streams {(a_b + b_b + c_b) * cells_local / 1e6:.0f}"
+                              f" MB ({8 * cells_local / 1e6:.0f} MB per field) through the 126 MB L2"),
+                       "step": "mas_op_update + " + ("mas_op_set_aniso + " if aniso else "") +
+                               "x:=x0 + mas_pcg_solve"},
             "roofline": {"bound": "hbm", "kernel": "k_stencil<PCGA> (kernel A)",
                          "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic,
@@ -408,9 +446,11 @@ def main():
                                   "(host-driven loop); value is the graph-mode pass",
                         "profiled_pass_ms_per_step": t_prof_ms / args.steps,
                         "A_GBs": achieved,
+                        **({"Lpar_ms": c_ms, "Lpar_GBs": c_b * cells_local / (c_ms / 1e3) / 1e9,
+                            "Lpar_alg_bytes_per_cell": c_b} if aniso and c_ms > 0 else {}),
                         "B_GBs": b_b * cells_local / (b_ms / 1e3) / 1e9,
                         "iter_alg_GBs": iter_gbs, "iter_frac": iter_gbs / peak,
-                        "alg_bytes_per_cell_iter": a_b + b_b},
+                        "alg_bytes_per_cell_iter": a_b + b_b + c_b},
             "e2e": e2e,
             "gpu_launches": launches,
             "clocks": clk,

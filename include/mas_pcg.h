@@ -222,6 +222,33 @@ MAS_API mas_status_t mas_op_set_profiling(mas_op_t* op, int on);
  * of the last profiled solve; n = number of iterations averaged. */
 MAS_API mas_status_t mas_op_kernel_times(const mas_op_t* op, double* a_ms, double* b_ms, int* n);
 
+/* Field-aligned (anisotropic) thermal conduction.
+ * MAS conducts heat along the magnetic field; the paper names the
+ * thermodynamic model of its test problem and the implicit
+ * parabolic Krylov schemes of ref. [25] but prints no formula,
+ * so the term is the reading R21-R26 of DESIGN.md §3.4:
+ *   L = L_iso + L_par,  L_par u = -div(kpar b (b . grad u)) in the symmetric
+ *   corner form  V_P (L_par u)_P = sum_{corners c of P} W_c kpar_c (b_c.g_c(u))
+ *   (b_c . dg_c/du_P), g_c the 8-cell corner gradient, W_c the corner dual
+ *   volume; corners on the r boundaries, poles and theta walls carry no
+ *   weight (no field-aligned flux leaves the domain).
+ * kpar: [nr][nt][np] >= 0 and bhat: [3][nr][nt][np] (b_r, b_theta, b_phi,
+ * used as given) at the LOWER corner (rF_i, tF_j, pF_k) of each cell; the
+ * entries of boundary corners (i = 0 or j = 0) are ignored.  Device or host
+ * pointers; the library keeps only the derived corner coefficients
+ * (3 fields).  The Jacobi diagonal gains the term's diagonal (R26); apply,
+ * the residual and every PCG iteration add it (one extra kernel per
+ * iteration).  kpar == NULL switches the term off.  Synchronises the stream.
+ * Errors: MAS_ERR_ARG if ncomp != 1, the grid is distributed (single GPU in
+ * this version), kpar < 0 or non-finite, b non-finite, or some D_P <= 0
+ * (the term is then off). */
+MAS_API mas_status_t mas_op_set_aniso(mas_op_t* op, const double* kpar, const double* bhat,
+                                      cudaStream_t stream);
+
+/* Average device time (ms) of the L_par kernel over the last profiled solve
+ * (mas_op_set_profiling); 0 when the term is off. */
+MAS_API mas_status_t mas_op_aniso_time(const mas_op_t* op, double* ms);
+
 MAS_API mas_status_t mas_op_destroy(mas_op_t* op);
 
 MAS_API const char* mas_status_string(mas_status_t s);

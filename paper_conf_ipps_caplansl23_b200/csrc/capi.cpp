@@ -111,8 +111,8 @@ struct mas_op {
     long long launches = 0;
     // optional per-kernel timing of the solve (CUDA events on its stream)
     int prof = 0;
-    std::vector<cudaEvent_t> pev;  // 4 per iteration: A start/end, B start/end
-    double prof_a_ms = 0.0, prof_b_ms = 0.0, prof_init_ms = 0.0;
+    std::vector<cudaEvent_t> pev;  // 6 per iteration: A, B, L_par start/end
+    double prof_a_ms = 0.0, prof_b_ms = 0.0, prof_c_ms = 0.0, prof_init_ms = 0.0;
     int prof_n = 0;
     // single-GPU solve loop as one CUDA graph: a device-side while node whose
     // body is two PCG iterations (A, B, A, B); rebuilt when x or the history
@@ -121,6 +121,7 @@ struct mas_op {
     cudaStream_t cap_stream = nullptr;
     const double* g_x = nullptr;
     const double* g_hist = nullptr;
+    int g_aniso = -1;
     int use_graph = 1;
     // P2P transport (mas_op_enable_p2p): mailbox allreduce + in-place reads of
     // the r-neighbours' edge planes over NVLink instead of NCCL in the loop
@@ -141,6 +142,11 @@ struct mas_op {
     const double* nbt_r[2] = {nullptr, nullptr};                         // P2P: theta nbrs' r
     const double* nbt_p[2][2] = {{nullptr, nullptr}, {nullptr, nullptr}};  // [parity][lo/hi]
     int nbt_ntl[2] = {0, 0};                     // their theta rows
+    // field-aligned conduction term L_par (NEXT-4, mas_op_set_aniso)
+    int aniso = 0;
+    double* ca = nullptr;                        // corner coefficients [3][nl][nt][np]
+    double* atab = nullptr;                      // AnisoTab arrays (device)
+    AnisoTab at{};
 };
 
 extern "C" {
@@ -362,6 +368,31 @@ static P2P p2p_args(const mas_op* op) {
     return t;
 }
 
+// D (optional) and 1/D: the 7-point diagonal (k_diag), plus the field-aligned
+// term's diagonal (R26) when L_par is on (D then goes through a device buffer:
+// the caller's, or q, which is free outside a solve).
+static mas_status_t op_diag(mas_op* op, double* D_out, cudaStream_t s) {
+    double* D = op->aniso && !D_out ? op->q : D_out;
+    CU(launch_diag(op->geo, halo_of(op, op->kappa, op->kg, 1), packed_rows(op, op->kgt, 1), op->c, D,
+                   op->dinv, op->bad, s));
+    if (op->aniso) CU(launch_aniso_diag(op->geo, op->ca, D, op->dinv, op->bad, s));
+    return MAS_OK;
+}
+
+static AnisoArgs aniso_args(const mas_op* op, int mode, const double* u, double* out) {
+    AnisoArgs a{};
+    a.g = op->geo;
+    a.chunk = op->chunk;
+    a.max_blocks = op->max_blocks;
+    a.ca = op->ca;
+    a.u = u;
+    a.out = out;
+    a.st = op->st;
+    a.scr = op->scr;
+    (void)mode;
+    return a;
+}
+
 // copy coefficients in (host or device pointers), compute D and 1/D, exchange
 // the static kappa / dinv seams, check the coefficients on the device.
 static mas_status_t op_load(mas_op* op, const double* kappa, const double* mass, cudaStream_t s,
@@ -378,8 +409,7 @@ static mas_status_t op_load(mas_op* op, const double* kappa, const double* mass,
                       rstride(op)));
     ST(tseams(op, op->kappa, 1, op->kgt, s));
     CU(cudaMemsetAsync(op->bad, 0, sizeof(int), s));
-    CU(launch_diag(op->geo, halo_of(op, op->kappa, op->kg, 1), packed_rows(op, op->kgt, 1), op->c,
-                   D_out, op->dinv, op->bad, s));
+    ST(op_diag(op, D_out, s));
     if (op->g->comm)
         ST(comm_seams(op->g->comm, op->dinv, 1, op->g->nl, plane, op->dg, op->dg + plane, s,
                       rstride(op)));
@@ -402,7 +432,8 @@ static mas_status_t op_load(mas_op* op, const double* kappa, const double* mass,
 
 static void op_free(mas_op* op) {
     if (!op) return;
-    for (double* p : {op->kgt, op->dgt, op->xgt, op->rgt, op->pgt[0], op->pgt[1], op->tpack})
+    for (double* p : {op->kgt, op->dgt, op->xgt, op->rgt, op->pgt[0], op->pgt[1], op->tpack, op->ca,
+                      op->atab})
         if (p) cudaFree(p);
     for (double* p : {op->kappa, op->c, op->dinv, op->kg, op->dg, op->wR, op->r, op->p[0], op->p[1],
                       op->q, op->rg, op->pg[0], op->pg[1], op->xg, op->stage_a, op->stage_b,
@@ -437,7 +468,7 @@ static mas_status_t ensure_hist(mas_op* op, int maxit) {
 }
 
 static mas_status_t ensure_prof_events(mas_op* op, int k) {
-    while (op->pev.size() < 4 * (size_t)k) {
+    while (op->pev.size() < 6 * (size_t)k) {
         cudaEvent_t e;
         CU(cudaEventCreate(&e));
         op->pev.push_back(e);
@@ -448,8 +479,9 @@ static mas_status_t ensure_prof_events(mas_op* op, int k) {
 // Build (or reuse) the graph of the iteration loop: while (!stopped) {A B A B}.
 // Kernels read k, alpha, beta and the stop decision from PcgState; the
 // deciding kernel's last block sets the while-condition to 0.
-static mas_status_t loop_graph(mas_op* op, StencilArgs a, StreamArgs b) {
-    if (op->gexec && op->g_x == a.x && op->g_hist == a.rho_hist) return MAS_OK;
+static mas_status_t loop_graph(mas_op* op, StencilArgs a, StreamArgs b, AnisoArgs an) {
+    if (op->gexec && op->g_x == a.x && op->g_hist == a.rho_hist && op->g_aniso == op->aniso)
+        return MAS_OK;
     if (op->gexec) {
         cudaGraphExecDestroy(op->gexec);
         op->gexec = nullptr;
@@ -473,6 +505,7 @@ static mas_status_t loop_graph(mas_op* op, StencilArgs a, StreamArgs b) {
         if (e == cudaSuccess) {
             a.cond = (unsigned long long)h;
             b.cond = (unsigned long long)h;
+            an.cond = (unsigned long long)h;
             const int nc = op->ncomp;
             // iteration 1 runs before the loop (its own kernel-A instantiation);
             // the body covers an even and an odd iteration: k = 2, 3, 4, ...
@@ -481,6 +514,8 @@ static mas_status_t loop_graph(mas_op* op, StencilArgs a, StreamArgs b) {
                 a.tpold = pold_trows(op, kk);
                 a.pnew = op->p[kk & 1];
                 e = launch_stencil(MODE_PCGA, nc, a, op->cap_stream);
+                an.u = a.pnew;
+                if (e == cudaSuccess && op->aniso) e = launch_aniso(MODE_PCGA, an, op->cap_stream);
                 if (e == cudaSuccess) e = launch_pcg_b(b, op->b_blocks, op->cap_stream);
             }
             cudaGraph_t out = body;
@@ -498,6 +533,7 @@ static mas_status_t loop_graph(mas_op* op, StencilArgs a, StreamArgs b) {
     }
     op->g_x = a.x;
     op->g_hist = a.rho_hist;
+    op->g_aniso = op->aniso;
     return MAS_OK;
 }
 
@@ -668,8 +704,7 @@ mas_status_t mas_op_diag(const mas_op_t* op_c, double* D, cudaStream_t stream) {
         Dd = op->stage_b;
     }
     CU(cudaMemsetAsync(op->bad, 0, sizeof(int), stream));
-    CU(launch_diag(op->geo, halo_of(op, op->kappa, op->kg, 1), packed_rows(op, op->kgt, 1), op->c, Dd,
-                   op->dinv, op->bad, stream));
+    ST(op_diag(op, Dd, stream));
     if (host) {
         CU(cudaMemcpyAsync(D, Dd, op->Nl * sizeof(double), cudaMemcpyDeviceToHost, stream));
         CU(cudaStreamSynchronize(stream));
@@ -706,6 +741,7 @@ mas_status_t mas_op_apply(const mas_op_t* op_c, const double* x, double* y, cuda
     a.out = yd;
     a.scr = op->scr;
     CU(launch_stencil(MODE_APPLY, op->ncomp, a, stream));
+    if (op->aniso) CU(launch_aniso(MODE_APPLY, aniso_args(op, MODE_APPLY, xd, yd), stream));
     if (hy) {
         CU(cudaMemcpyAsync(y, yd, bytes, cudaMemcpyDeviceToHost, stream));
         CU(cudaStreamSynchronize(stream));
@@ -892,6 +928,83 @@ mas_status_t mas_op_kernel_times(const mas_op_t* op, double* a_ms, double* b_ms,
     return MAS_OK;
 }
 
+mas_status_t mas_op_aniso_time(const mas_op_t* op, double* ms) {
+    if (!op || !ms) return arg_error("null argument");
+    *ms = op->prof_c_ms;
+    return MAS_OK;
+}
+
+mas_status_t mas_op_set_aniso(mas_op_t* op, const double* kpar, const double* bhat,
+                              cudaStream_t stream) {
+    NvtxRange nvtx("mas_op_set_aniso");
+    if (!op) return arg_error("null op");
+    if (!kpar) {  // switch the term off
+        op->aniso = 0;
+        CU(cudaMemsetAsync(op->bad, 0, sizeof(int), stream));
+        ST(op_diag(op, nullptr, stream));
+        return MAS_OK;
+    }
+    if (!bhat) return arg_error("null bhat");
+    if (op->ncomp != 1) return arg_error("field-aligned conduction needs ncomp == 1");
+    if (op->g->comm || op->g->nranks > 1)
+        return arg_error("field-aligned conduction is single-GPU in this version");
+    mas_grid* g = op->g;
+    const int nl = g->nl, nt = g->ntl, np = g->np;
+    const long long N = op->Nl;
+    if (!op->atab) {  // 1-D corner metrics (R22, R23), 0 on dead corners (R24)
+        std::vector<double> t(2 * (size_t)nl + 2 * (size_t)nt + np, 0.0);
+        double *rF = t.data(), *hr = rF + nl, *sF = hr + nl, *ht = sF + nt, *hp = ht + nt;
+        for (int il = 0; il < nl; il++) {
+            const int i = g->i0 + il;
+            rF[il] = g->rF[i];
+            hr[il] = i > 0 ? g->rC[i] - g->rC[i - 1] : 0.0;
+        }
+        for (int j = 1; j < nt; j++) {
+            sF[j] = std::sin(g->tF[j]);
+            ht[j] = g->tC[j] - g->tC[j - 1];
+        }
+        hp[0] = g->pC[0] + 2.0 * M_PI - g->pC[np - 1];
+        for (int k = 1; k < np; k++) hp[k] = g->pC[k] - g->pC[k - 1];
+        ST(dmalloc(&op->atab, t.size()));
+        CU(cudaMemcpy(op->atab, t.data(), t.size() * sizeof(double), cudaMemcpyHostToDevice));
+        op->at.rF = op->atab;
+        op->at.hr = op->atab + nl;
+        op->at.sF = op->atab + 2 * nl;
+        op->at.ht = op->atab + 2 * nl + nt;
+        op->at.hp = op->atab + 2 * nl + 2 * nt;
+    }
+    if (!op->ca) ST(dmalloc(&op->ca, 3 * (size_t)N));
+    // host inputs are staged through a temporary device buffer
+    const double *kd = kpar, *bd = bhat;
+    double* tmp = nullptr;
+    const bool hk = !is_device_ptr(kpar), hb = !is_device_ptr(bhat);
+    if (hk || hb) {
+        ST(dmalloc(&tmp, 4 * (size_t)N));
+        if (hk) {
+            CU(cudaMemcpyAsync(tmp, kpar, N * sizeof(double), cudaMemcpyHostToDevice, stream));
+            kd = tmp;
+        }
+        if (hb) {
+            CU(cudaMemcpyAsync(tmp + N, bhat, 3 * N * sizeof(double), cudaMemcpyHostToDevice, stream));
+            bd = tmp + N;
+        }
+    }
+    CU(cudaMemsetAsync(op->bad, 0, sizeof(int), stream));
+    CU(launch_aniso_coef(op->geo, op->at, kd, bd, op->ca, op->bad, stream));
+    op->aniso = 1;
+    ST(op_diag(op, nullptr, stream));
+    int bad = 0;
+    CU(cudaMemcpyAsync(&bad, op->bad, sizeof(int), cudaMemcpyDeviceToHost, stream));
+    CU(cudaStreamSynchronize(stream));
+    if (tmp) cudaFree(tmp);
+    if (bad) {
+        op->aniso = 0;
+        op_diag(op, nullptr, stream);
+        return arg_error("kpar negative or non-finite, b non-finite, or Jacobi diagonal D <= 0");
+    }
+    return MAS_OK;
+}
+
 mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, double tol,
                            int maxit, int* iters, double* relres, double* res_hist,
                            cudaStream_t s) {
@@ -958,6 +1071,15 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
     a.p2p = p2p_args(op);
     CU(launch_stencil(MODE_RESID, nc, a, s));
     op->launches++;
+    AnisoArgs an{};
+    if (op->aniso) {  // r -= L_par x0 and the three initial dots again (one GPU only)
+        an = aniso_args(op, MODE_RESID, xd, op->r);
+        an.f = fd;
+        an.dinv = op->dinv;
+        CU(launch_aniso(MODE_RESID, an, s));
+        op->launches++;
+        an = aniso_args(op, MODE_PCGA, nullptr, op->q);
+    }
     if (comm && !p2p) ST(comm_allreduce(comm, &op->st->pend_rho, 3, s));  // rho, rr, ff
 
     StreamArgs b{};
@@ -987,11 +1109,15 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
     // (virtual P2P ranks share one GPU and need host ordering: comm_vsync)
     const bool graph = !op->prof && op->use_graph && (!comm || (p2p && !comm_is_virtual(comm)));
     if (graph) {
-        ST(loop_graph(op, a, b));
+        ST(loop_graph(op, a, b, an));
         a.pold = pold_halo(op, 1);  // iteration 1 (not read)
         a.tpold = pold_trows(op, 1);
         a.pnew = op->p[1];
         CU(launch_stencil(MODE_PCGA, nc, a, s, true));
+        if (op->aniso) {
+            an.u = a.pnew;
+            CU(launch_aniso(MODE_PCGA, an, s));
+        }
         CU(launch_pcg_b(b, op->b_blocks, s));
         CU(cudaGraphLaunch(op->gexec, s));
     }
@@ -1006,7 +1132,7 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
         cudaEvent_t* pe = nullptr;
         if (op->prof) {
             ST(ensure_prof_events(op, k));
-            pe = &op->pev[4 * (size_t)(k - 1)];
+            pe = &op->pev[6 * (size_t)(k - 1)];
         }
         if (comm && !p2p && split_theta(op)) {
             // (r, theta) decomposition over NCCL: r-plane seams and packed
@@ -1055,6 +1181,13 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
             op->launches++;
         }
         if (pe) CU(cudaEventRecord(pe[1], s));
+        if (op->aniso) {  // q += L_par p_k, sigma += <p_k, L_par p_k> (one GPU only)
+            an.u = pnew;
+            if (pe) CU(cudaEventRecord(pe[4], s));
+            CU(launch_aniso(MODE_PCGA, an, s));
+            if (pe) CU(cudaEventRecord(pe[5], s));
+            op->launches++;
+        }
         if (comm && !p2p) ST(comm_allreduce(comm, &op->st->pend_sigma, 1, s));
         if (k <= maxit) {
             if (p2p) ST(comm_vsync(comm, s));  // virtual P2P ranks: all A(k) done
@@ -1093,7 +1226,8 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
     if (graph) {  // iteration 1 + 4 kernels per executed loop body (iterations 2k, 2k+1)
         const int last_a = fin.status == MAS_ERR_BREAKDOWN ? fin.iters : fin.iters + 1;
         const int bodies = last_a <= 2 ? 1 : last_a / 2;
-        op->launches += 2 + 4LL * bodies;
+        const int per = op->aniso ? 3 : 2;  // kernels per iteration
+        op->launches += per + 2LL * per * bodies;
     }
     if (res_hist) {
         // after a breakdown at iteration k only ||r_0..r_{k-1}|| exist
@@ -1103,15 +1237,19 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
         for (int k = 0; k < nh; k++) res_hist[k] = std::sqrt(rr[k]);
     }
     if (op->prof) {  // average device time of the working launches 1..iters
-        double sa = 0.0, sb = 0.0;
+        double sa = 0.0, sb = 0.0, sc = 0.0;
         int n = 0;
-        for (int k = 1; k <= fin.iters && 4 * (size_t)k <= op->pev.size(); k++, n++) {
-            float ta = 0.f, tb = 0.f;
-            CU(cudaEventElapsedTime(&ta, op->pev[4 * (k - 1)], op->pev[4 * (k - 1) + 1]));
-            CU(cudaEventElapsedTime(&tb, op->pev[4 * (k - 1) + 2], op->pev[4 * (k - 1) + 3]));
+        for (int k = 1; k <= fin.iters && 6 * (size_t)k <= op->pev.size(); k++, n++) {
+            float ta = 0.f, tb = 0.f, tc = 0.f;
+            const cudaEvent_t* e = &op->pev[6 * (size_t)(k - 1)];
+            CU(cudaEventElapsedTime(&ta, e[0], e[1]));
+            CU(cudaEventElapsedTime(&tb, e[2], e[3]));
+            if (op->aniso) CU(cudaEventElapsedTime(&tc, e[4], e[5]));
             sa += ta;
             sb += tb;
+            sc += tc;
         }
+        op->prof_c_ms = n ? sc / n : 0.0;
         op->prof_n = n;
         op->prof_a_ms = n ? sa / n : 0.0;
         op->prof_b_ms = n ? sb / n : 0.0;

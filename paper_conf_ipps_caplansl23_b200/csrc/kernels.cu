@@ -24,10 +24,10 @@
 #include <cstdint>
 
 #include "mas_internal.h"
+#include "reduce.cuh"
 
 namespace mas {
 
-constexpr int kThreads = 256;  // 8 warps (stream kernels)
 #ifndef MAS_TJ
 #define MAS_TJ 8
 #endif
@@ -50,67 +50,6 @@ constexpr int HROWS = TJ + 2;  // tile rows + 2 halo rows
 
 enum { P_NORMAL = 0, P_FINAL = 1, P_ZERO = 2 };
 enum { TKT_STENCIL = 0, TKT_B = 1, TKT_DOT = 2 };
-
-// --------------------------------------------------------------------------
-// deterministic reductions
-// --------------------------------------------------------------------------
-__device__ __forceinline__ double warp_sum(double v) {
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) v += __shfl_down_sync(0xffffffffu, v, o);
-    return v;  // valid in lane 0
-}
-
-// Block-reduce NS sums, publish the block partial, take a ticket.  Returns
-// true in the last block to finish, where `v` then holds the grid totals
-// (valid in thread 0), summed in a fixed order independent of scheduling.
-// sysfence: the block's global writes are also read by peer GPUs (P2P
-// transport), so order them at system scope before the ticket.
-template <int NS, int NTHR = kThreads>
-__device__ bool grid_reduce(double (&v)[NS], const Scratch& scr, int tkt, bool sysfence = false) {
-    __shared__ double wsum[NS][NTHR / 32];
-    __shared__ bool last;
-    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-#pragma unroll
-    for (int s = 0; s < NS; s++) {
-        double t = warp_sum(v[s]);
-        if (lane == 0) wsum[s][w] = t;
-    }
-    __syncthreads();
-    if (threadIdx.x == 0) {
-#pragma unroll
-        for (int s = 0; s < NS; s++) {
-            double t = 0.0;
-            for (int q = 0; q < NTHR / 32; q++) t += wsum[s][q];
-            scr.partials[(size_t)blockIdx.x * NS + s] = t;
-        }
-        if (sysfence)
-            __threadfence_system();
-        else
-            __threadfence();
-        unsigned old = atomicAdd(&scr.ticket[tkt], 1u);
-        last = (old == gridDim.x - 1);
-    }
-    __syncthreads();
-    if (!last) return false;
-    __threadfence();
-#pragma unroll
-    for (int s = 0; s < NS; s++) {
-        double t = 0.0;
-        for (unsigned b = threadIdx.x; b < gridDim.x; b += NTHR)
-            t += __ldcg(&scr.partials[(size_t)b * NS + s]);
-        t = warp_sum(t);
-        __syncthreads();
-        if (lane == 0) wsum[s][w] = t;
-        __syncthreads();
-        if (threadIdx.x == 0) {
-            double u = 0.0;
-            for (int q = 0; q < NTHR / 32; q++) u += wsum[s][q];
-            v[s] = u;
-        }
-    }
-    if (threadIdx.x == 0) scr.ticket[tkt] = 0u;
-    return true;
-}
 
 // --------------------------------------------------------------------------
 // P2P transport: one-shot allreduce through peer mailboxes (NVLink stores)

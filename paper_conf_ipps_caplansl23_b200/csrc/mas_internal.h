@@ -150,6 +150,38 @@ struct StreamArgs {  // kernel B
     P2P p2p;
 };
 
+// ---------------------------------------------------------------------------
+// Field-aligned conduction (readings R21-R26, DESIGN.md
+// §3.4):  V_P (L_par u)_P = sum_{corners c of P} s_c (sr a_c + st b_c + sp e_c),
+//   s_c = a_c Dr_c(u) + b_c Dt_c(u) + e_c Dp_c(u)
+// with Dr / Dt / Dp the sums of the 4 cell differences across corner c in r /
+// theta / phi, sr, st, sp = +-1 the side of P, and the corner coefficients
+//   (a, b, e) = sqrt(W_c kpar_c) (b_r/(4 hr), b_t/(4 rF ht), b_p/(4 rF sF hp))
+// precomputed once per mas_op_set_aniso (k_aniso_coef), stored at the cell
+// whose lower corner c is: ca[3][nl][nt][np].  Single GPU (one r-slab).
+// ---------------------------------------------------------------------------
+struct AnisoTab {          // 1-D corner metrics (device), 0 on dead corners (R24)
+    const double* rF;      // [nl]  r of the lower r-face of plane I
+    const double* hr;      // [nl]  rC_I - rC_{I-1}; 0 at the global inner face
+    const double* sF;      // [nt]  sin(tF_J); 0 at J = 0
+    const double* ht;      // [nt]  tC_J - tC_{J-1}; 0 at J = 0
+    const double* hp;      // [np]  centre distance across phi-face K (periodic)
+};
+
+struct AnisoArgs {
+    Geo g;
+    int chunk, ntj, ntk, nchunk;  // set by launch_aniso
+    int max_blocks;               // capacity of scr.partials (blocks)
+    const double* ca;      // [3][nl][nt][np] corner coefficients a, b, e
+    const double* u;       // APPLY / RESID: x;  PCGA: p_k (written by kernel A(k))
+    double* out;           // APPLY: y += L_par x;  RESID: r -= L_par x;  PCGA: q += L_par p
+    const double* f;       // RESID: rhs
+    const double* dinv;    // RESID: 1/D (for <r, D^-1 r>)
+    PcgState* st;
+    Scratch scr;
+    unsigned long long cond;
+};
+
 // launchers (kernels.cu)
 int stencil_blocks(const Geo& g, int chunk);
 // first: kernel A of iteration 1 (its own instantiation)
@@ -166,6 +198,16 @@ cudaError_t launch_dot(const Geo& g, int ncomp, const double* a, const double* b
                        double* out, int nblocks, cudaStream_t s);
 // out[t] = sum_r stage[8r + t], t < n, ranks summed in rank order (virtual-rank allreduce)
 cudaError_t launch_rank_sum(double* out, const double* stage, int nranks, int n, cudaStream_t s);
+
+// launchers (aniso.cu)
+cudaError_t launch_aniso(int mode, const AnisoArgs& a, cudaStream_t s);
+// ca from kpar [nl][nt][np] and bhat [3][nl][nt][np]; *bad |= 1 on a negative
+// or non-finite kpar / non-finite b
+cudaError_t launch_aniso_coef(const Geo& g, AnisoTab t, const double* kpar, const double* bhat,
+                              double* ca, int* bad, cudaStream_t s);
+// D += (1/V) sum_c (sr a + st b + sp e)^2 (R26); dinv = 1/D; *bad |= 1 if D <= 0
+cudaError_t launch_aniso_diag(const Geo& g, const double* ca, double* D, double* dinv, int* bad,
+                              cudaStream_t s);
 
 void set_last_error(const std::string& msg);
 

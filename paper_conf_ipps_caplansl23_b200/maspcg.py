@@ -27,7 +27,8 @@ ABI_SYMBOLS = ("mas_comm_unique_id", "mas_partition", "mas_grid_create", "mas_gr
                "mas_op_dirichlet_rhs", "mas_op_dot", "mas_pcg_solve", "mas_op_enable_p2p",
                "mas_op_transport", "mas_op_launch_count", "mas_grid_create_2d",
                "mas_grid_local_extent_2d",
-               "mas_op_set_profiling", "mas_op_kernel_times", "mas_op_destroy", "mas_status_string", "mas_last_error", "mas_version")
+               "mas_op_set_profiling", "mas_op_kernel_times", "mas_op_set_aniso",
+               "mas_op_aniso_time", "mas_op_destroy", "mas_status_string", "mas_last_error", "mas_version")
 
 
 class MasError(RuntimeError):
@@ -73,6 +74,8 @@ def lib() -> C.CDLL:
             "mas_op_launch_count": (C.c_longlong, [_vp]),
             "mas_op_set_profiling": (_i, [_vp, _i]),
             "mas_op_kernel_times": (_i, [_vp, _vp, _vp, _vp]),
+            "mas_op_set_aniso": (_i, [_vp, _vp, _vp, _vp]),
+            "mas_op_aniso_time": (_i, [_vp, _vp]),
             "mas_op_destroy": (_i, [_vp]),
             "mas_status_string": (C.c_char_p, [_i]),
             "mas_last_error": (C.c_char_p, []),
@@ -264,6 +267,19 @@ def mas_op_kernel_times(op: int):
     return a.value, b.value, n.value
 
 
+def mas_op_set_aniso(op: int, kpar, bhat, stream=None) -> None:
+    """Field-aligned conduction term L_par (NEXT-4): kpar [nr,nt,np],
+    bhat [3,nr,nt,np] at the lower cell corners; kpar None switches it off."""
+    _check(lib().mas_op_set_aniso(op, _ptr(kpar), _ptr(bhat), _stream(stream)),
+           "mas_op_set_aniso")
+
+
+def mas_op_aniso_time(op: int) -> float:
+    ms = C.c_double()
+    _check(lib().mas_op_aniso_time(op, C.byref(ms)), "mas_op_aniso_time")
+    return ms.value
+
+
 def mas_op_destroy(op: int) -> None:
     _check(lib().mas_op_destroy(op), "mas_op_destroy")
 
@@ -336,6 +352,12 @@ class Operator:
 
     def kernel_times(self):
         return mas_op_kernel_times(self.h)
+
+    def set_aniso(self, kpar, bhat, stream=None):
+        mas_op_set_aniso(self.h, kpar, bhat, stream)
+
+    def aniso_time(self):
+        return mas_op_aniso_time(self.h)
 
     @property
     def launch_count(self):

@@ -1,6 +1,8 @@
 """Small driver for ncu: set up config C3 (or --config) and run one PCG solve
 with a few iterations through the C ABI.  Launch order: k_diag (setup),
-k_stencil<RESID>, then per iteration k_stencil<PCGA>, k_pcg_b."""
+k_stencil<RESID>, then per iteration k_stencil<PCGA>, k_pcg_b (C2a: k_aniso_coef,
+k_diag, k_aniso_diag at setup; k_aniso<RESID> after the init; k_aniso<PCGA>
+after every kernel A)."""
 import argparse
 import os
 import sys
@@ -17,12 +19,15 @@ ap = argparse.ArgumentParser()
 ap.add_argument("--config", default="C3")
 ap.add_argument("--maxit", type=int, default=4)
 args = ap.parse_args()
-shapes = {"C3": ("viscosity", 256, 256, 512), "C2": ("conduction", 128, 128, 256)}
+shapes = {"C3": ("viscosity", 256, 256, 512), "C2": ("conduction", 128, 128, 256),
+          "C2a": ("aniso", 128, 128, 256)}
 kind, nr, nt, np_ = shapes[args.config]
 prob = W.make(kind, nr=nr, nt=nt, np_=np_)
 d = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()
 g = M.Grid(prob.mesh)
 op = M.Operator(g, prob.ncomp, d(prob.kappa), d(prob.c), prob.bc_inner, prob.bc_outer)
+if prob.kpar is not None:  # C2a: + k_aniso<PCGA> after each kernel A
+    op.set_aniso(d(prob.kpar), d(prob.bhat))
 f = d(prob.f)
 x = d(prob.x0)
 st, it, rel, _ = op.solve(f, x, 0.0, args.maxit)
