@@ -169,224 +169,236 @@ __global__ void __launch_bounds__(kThreads, MAS_ANISO_MINB) k_aniso(const AnisoA
         return;
     }
     const Geo& g = a.g;
-    const int item = blockIdx.x;
-    const int tk = item % a.ntk, tj = (item / a.ntk) % a.ntj, ch = item / (a.ntk * a.ntj);
-    const int j0 = tj * AJ, k0 = tk * AK;
-    const int height = min(AJ, g.nt - j0), width = min(AK, g.np - k0);  // width is even
-    const int ia = ch * a.chunk, ib = min(ia + a.chunk, g.nl);
     const int plane = (int)g.plane;
     const long long Nl = (long long)g.nl * plane;
-    const int hw = width >> 1;  // 16-byte pairs per row
     double acc[3] = {0.0, 0.0, 0.0};
+    // Balanced partition: the (tile, r-plane) units, tile-major, are split
+    // into gridDim.x equal ranges; a block's range covers one or two
+    // segments (a run of planes of one tile), each marched with its own
+    // pipeline (one resident wave of blocks, no tail).
+    const long long units = (long long)a.ntj * a.ntk * g.nl;
+    long long u0 = units * blockIdx.x / gridDim.x;
+    const long long u1 = units * (blockIdx.x + 1) / gridDim.x;
+    while (u0 < u1) {
+        const int tile = (int)(u0 / g.nl);
+        const int ia = (int)(u0 - (long long)tile * g.nl);
+        const int ib = (int)min((long long)g.nl, ia + (u1 - u0));
+        u0 += ib - ia;
+        const int tk = tile % a.ntk, tj = tile / a.ntk;
+        const int j0 = tj * AJ, k0 = tk * AK;
+        const int height = min(AJ, g.nt - j0), width = min(AK, g.np - k0);  // width is even
+        const int hw = width >> 1;  // 16-byte pairs per row
 
-    // ---- per-thread work lists ---------------------------------------------
-    // copies: smem offset within the slot (-1: none), in-plane source offset,
-    // 16 B (1) or 8 B (0), row valid (rows beyond a pole / the tile: zero-fill)
-    int pd[NP_IT], ps[NP_IT];
-    unsigned pflag = 0;  // bit 2s: 16 B, bit 2s+1: row valid
-    for (int s = 0; s < NP_IT; s++) {
-        const int t = threadIdx.x + s * kThreads;
-        pd[s] = -1;
-        ps[s] = 0;
-        if (t < PR * (hw + 2)) {
-            const int r = t / (hw + 2), c = t - r * (hw + 2);
-            const int j = j0 - 1 + r;
-            const bool ok = j >= 0 && j < g.nt && r <= height + 1;
-            if (c < hw) {
-                pd[s] = r * PW + 2 + 2 * c;
-                ps[s] = (ok ? j : 0) * g.np + k0 + 2 * c;
-                pflag |= 1u << (2 * s);
-            } else {
-                const int side = c - hw;  // 0: k0-1, 1: k0+width (periodic)
-                int k = side ? k0 + width : k0 - 1;
-                k = k < 0 ? k + g.np : (k >= g.np ? k - g.np : k);
-                pd[s] = r * PW + (side ? 2 + width : 1);
-                ps[s] = (ok ? j : 0) * g.np + k;
-            }
-            if (ok) pflag |= 2u << (2 * s);
-        }
-    }
-    int cd[NC_IT], cs[NC_IT];
-    unsigned cflag = 0;  // bits as pflag, + bits 16+2s..: field f
-    for (int s = 0; s < NC_IT; s++) {
-        const int t = threadIdx.x + s * kThreads;
-        cd[s] = -1;
-        cs[s] = 0;
-        const int crow = hw + 1;
-        if (t < 3 * CR * crow) {
-            const int fr = t / crow, c = t - fr * crow;
-            const int f = fr / CR, r = fr - f * CR;
-            const int J = j0 + r;
-            const bool ok = r <= height && J < g.nt;
-            if (c < hw) {
-                cd[s] = f * CA + r * CW + 2 * c;
-                cs[s] = (ok ? J : 0) * g.np + k0 + 2 * c;
-                cflag |= 1u << (2 * s);
-            } else {
-                int K = k0 + width;
-                if (K >= g.np) K -= g.np;
-                cd[s] = f * CA + r * CW + width;
-                cs[s] = (ok ? J : 0) * g.np + K;
-            }
-            if (ok) cflag |= 2u << (2 * s);
-            cflag |= (unsigned)f << (16 + 2 * s);
-        }
-    }
-    int qd[NQ_IT], qs[NQ_IT];
-    for (int s = 0; s < NQ_IT; s++) {
-        const int t = threadIdx.x + s * kThreads;
-        qd[s] = -1;
-        qs[s] = 0;
-        if (t < height * hw) {
-            const int r = t / hw, c = t - r * hw;
-            qd[s] = r * AK + 2 * c;
-            qs[s] = (j0 + r) * g.np + k0 + 2 * c;
-        }
-    }
-    // corners (smem offsets into the coefficient / p slots) and cells
-    int kc[NK_IT], kp[NK_IT];
-    unsigned kown = 0;  // bit s: the corner belongs to this tile (row < height, col < width):
-                        // the last row / col is the next tile's first (sigma counts each once)
-    for (int s = 0; s < NK_IT; s++) {
-        const int t = threadIdx.x + s * kThreads;
-        kc[s] = -1;
-        kp[s] = 0;
-        if (t < (height + 1) * (width + 1)) {
-            const int r = t / (width + 1), c = t - r * (width + 1);
-            kc[s] = r * CW + c;
-            kp[s] = r * PW + c + 1;
-            if (r < height && c < width) kown |= 1u << s;
-        }
-    }
-    int lc[NL_IT], lq[NL_IT], lo_[NL_IT];
-    double lw[NL_IT];  // 1 / (vt_j vp_k)
-    for (int s = 0; s < NL_IT; s++) {
-        const int t = threadIdx.x + s * kThreads;
-        lc[s] = -1;
-        lq[s] = 0;
-        lo_[s] = 0;
-        lw[s] = 0.0;
-        if (t < height * width) {
-            const int r = t / width, c = t - r * width;
-            lc[s] = r * CW + c;
-            lq[s] = r * AK + c;
-            lo_[s] = (j0 + r) * g.np + k0 + c;
-            lw[s] = 1.0 / (__ldg(g.vt + j0 + r) * __ldg(g.vp + k0 + c));
-        }
-    }
-
-    // ---- stages ------------------------------------------------------------
-    auto issue = [&](int I) {
-        if (I <= ib) {
-            double* P = Ps + (I & 3) * P_SLOT;
-            const bool pl = I >= 0 && I < g.nl;
-            const double* pb = a.u + (size_t)(pl ? I : 0) * plane;
-#pragma unroll
-            for (int s = 0; s < NP_IT; s++) {
-                if (pd[s] < 0) continue;
-                const bool ok = pl && ((pflag >> (2 * s + 1)) & 1u);
-                if ((pflag >> (2 * s)) & 1u)
-                    cpa16(P + pd[s], pb + ps[s], ok);
-                else
-                    cpa8(P + pd[s], pb + ps[s], ok);
-            }
-            double* Cf = Cs + (I & 3) * C_SLOT;
-            const bool cl = I < g.nl;
-            const double* cb0 = a.ca + (size_t)(cl ? I : 0) * plane;
-#pragma unroll
-            for (int s = 0; s < NC_IT; s++) {
-                if (cd[s] < 0) continue;
-                const bool ok = cl && ((cflag >> (2 * s + 1)) & 1u);
-                const int f = (cflag >> (16 + 2 * s)) & 3u;
-                const double* src = cb0 + f * Nl + cs[s];
-                if ((cflag >> (2 * s)) & 1u)
-                    cpa16(Cf + cd[s], src, ok);
-                else
-                    cpa8(Cf + cd[s], src, ok);
+        // ---- per-thread work lists ---------------------------------------------
+        // copies: smem offset within the slot (-1: none), in-plane source offset,
+        // 16 B (1) or 8 B (0), row valid (rows beyond a pole / the tile: zero-fill)
+        int pd[NP_IT], ps[NP_IT];
+        unsigned pflag = 0;  // bit 2s: 16 B, bit 2s+1: row valid
+        for (int s = 0; s < NP_IT; s++) {
+            const int t = threadIdx.x + s * kThreads;
+            pd[s] = -1;
+            ps[s] = 0;
+            if (t < PR * (hw + 2)) {
+                const int r = t / (hw + 2), c = t - r * (hw + 2);
+                const int j = j0 - 1 + r;
+                const bool ok = j >= 0 && j < g.nt && r <= height + 1;
+                if (c < hw) {
+                    pd[s] = r * PW + 2 + 2 * c;
+                    ps[s] = (ok ? j : 0) * g.np + k0 + 2 * c;
+                    pflag |= 1u << (2 * s);
+                } else {
+                    const int side = c - hw;  // 0: k0-1, 1: k0+width (periodic)
+                    int k = side ? k0 + width : k0 - 1;
+                    k = k < 0 ? k + g.np : (k >= g.np ? k - g.np : k);
+                    pd[s] = r * PW + (side ? 2 + width : 1);
+                    ps[s] = (ok ? j : 0) * g.np + k;
+                }
+                if (ok) pflag |= 2u << (2 * s);
             }
         }
-        const int iq = I - 1;  // out plane I-1: its cells are computed at step I
-        if (iq >= ia && iq < ib) {
-            double* Q = Qs + ((iq + 3) % 3) * Q_SLOT;
-            const double* qb = a.out + (size_t)iq * plane;
-#pragma unroll
-            for (int s = 0; s < NQ_IT; s++)
-                if (qd[s] >= 0) cpa16(Q + qd[s], qb + qs[s], true);
+        int cd[NC_IT], cs[NC_IT];
+        unsigned cflag = 0;  // bits as pflag, + bits 16+2s..: field f
+        for (int s = 0; s < NC_IT; s++) {
+            const int t = threadIdx.x + s * kThreads;
+            cd[s] = -1;
+            cs[s] = 0;
+            const int crow = hw + 1;
+            if (t < 3 * CR * crow) {
+                const int fr = t / crow, c = t - fr * crow;
+                const int f = fr / CR, r = fr - f * CR;
+                const int J = j0 + r;
+                const bool ok = r <= height && J < g.nt;
+                if (c < hw) {
+                    cd[s] = f * CA + r * CW + 2 * c;
+                    cs[s] = (ok ? J : 0) * g.np + k0 + 2 * c;
+                    cflag |= 1u << (2 * s);
+                } else {
+                    int K = k0 + width;
+                    if (K >= g.np) K -= g.np;
+                    cd[s] = f * CA + r * CW + width;
+                    cs[s] = (ok ? J : 0) * g.np + K;
+                }
+                if (ok) cflag |= 2u << (2 * s);
+                cflag |= (unsigned)f << (16 + 2 * s);
+            }
         }
-        cpa_commit_group();
-    };
-
-    // corner products of corner plane I: corner (J, K) = (j0 + r, k0 + c)
-    // sits between cell rows J-1, J (p rows r, r+1) and cols K-1, K
-    // (p cols c+1, c+2)
-    auto corners = [&](int I) {
-        const double* p0 = Ps + ((I - 1) & 3) * P_SLOT;
-        const double* p1 = Ps + (I & 3) * P_SLOT;
-        double* Cf = Cs + (I & 3) * C_SLOT;
-#pragma unroll
+        int qd[NQ_IT], qs[NQ_IT];
+        for (int s = 0; s < NQ_IT; s++) {
+            const int t = threadIdx.x + s * kThreads;
+            qd[s] = -1;
+            qs[s] = 0;
+            if (t < height * hw) {
+                const int r = t / hw, c = t - r * hw;
+                qd[s] = r * AK + 2 * c;
+                qs[s] = (j0 + r) * g.np + k0 + 2 * c;
+            }
+        }
+        // corners (smem offsets into the coefficient / p slots) and cells
+        int kc[NK_IT], kp[NK_IT];
+        unsigned kown = 0;  // bit s: the corner belongs to this tile (row < height, col < width):
+                            // the last row / col is the next tile's first (sigma counts each once)
         for (int s = 0; s < NK_IT; s++) {
-            if (kc[s] < 0) continue;
-            double* c0 = Cf + kc[s];
-            const double A0 = c0[0], B0 = c0[CA], E0 = c0[2 * CA];
-            const double* q0 = p0 + kp[s];
-            const double* q1 = p1 + kp[s];
-            const double a00 = q0[0], a01 = q0[1], a10 = q0[PW], a11 = q0[PW + 1];
-            const double b00 = q1[0], b01 = q1[1], b10 = q1[PW], b11 = q1[PW + 1];
-            const double Dr = ((b00 - a00) + (b01 - a01)) + ((b10 - a10) + (b11 - a11));
-            const double Dt = ((a10 - a00) + (a11 - a01)) + ((b10 - b00) + (b11 - b01));
-            const double Dp = ((a01 - a00) + (a11 - a10)) + ((b01 - b00) + (b11 - b10));
-            const double sc = A0 * Dr + B0 * Dt + E0 * Dp;
-            const double A = sc * A0, B = sc * B0, E = sc * E0;
-            c0[0] = (A + B) + E;       // st +, sp +
-            c0[CA] = (A + B) - E;      // st +, sp -
-            c0[2 * CA] = (A - B) + E;  // st -, sp +
-            c0[3 * CA] = (A - B) - E;  // st -, sp -
-            // corner plane ib is the next chunk's first (or the dead outer face)
-            if (MODE == MODE_PCGA && I < ib && ((kown >> s) & 1u)) acc[0] += sc * sc;
-        }
-    };
-
-    // cells of plane i: corner planes i (sr = +1) and i+1 (sr = -1); corner
-    // rows r (st = +1), r+1 (st = -1); corner cols c (sp = +1), c+1 (sp = -1)
-    auto cells = [&](int i) {
-        const double* lo = Cs + (i & 3) * C_SLOT;
-        const double* hi = Cs + ((i + 1) & 3) * C_SLOT;
-        const double* Q = Qs + ((i + 3) % 3) * Q_SLOT;
-        const double ivr = 1.0 / __ldg(g.vr + i);
-        double* ob = a.out + (size_t)i * plane;
-#pragma unroll
-        for (int s = 0; s < NL_IT; s++) {
-            if (lc[s] < 0) continue;
-            const double* l = lo + lc[s];
-            const double* h = hi + lc[s];
-            const double sl = (l[0] + l[CA + 1]) + (l[2 * CA + CW] + l[3 * CA + CW + 1]);
-            const double sh = (h[3 * CA] + h[2 * CA + 1]) + (h[CA + CW] + h[CW + 1]);
-            const double y = (sl - sh) * (ivr * lw[s]);
-            const double qv = Q[lq[s]];
-            if (MODE == MODE_RESID) {
-                const double rv = qv - y;
-                ob[lo_[s]] = rv;
-                const double V = __ldg(g.vr + i) / lw[s];
-                const double f = a.f[(size_t)i * plane + lo_[s]];
-                acc[0] += V * f * f;
-                acc[1] += V * rv * rv;
-                acc[2] += V * rv * (a.dinv[(size_t)i * plane + lo_[s]] * rv);
-            } else {
-                ob[lo_[s]] = qv + y;
+            const int t = threadIdx.x + s * kThreads;
+            kc[s] = -1;
+            kp[s] = 0;
+            if (t < (height + 1) * (width + 1)) {
+                const int r = t / (width + 1), c = t - r * (width + 1);
+                kc[s] = r * CW + c;
+                kp[s] = r * PW + c + 1;
+                if (r < height && c < width) kown |= 1u << s;
             }
         }
-    };
+        int lc[NL_IT], lq[NL_IT], lo_[NL_IT];
+        double lw[NL_IT];  // 1 / (vt_j vp_k)
+        for (int s = 0; s < NL_IT; s++) {
+            const int t = threadIdx.x + s * kThreads;
+            lc[s] = -1;
+            lq[s] = 0;
+            lo_[s] = 0;
+            lw[s] = 0.0;
+            if (t < height * width) {
+                const int r = t / width, c = t - r * width;
+                lc[s] = r * CW + c;
+                lq[s] = r * AK + c;
+                lo_[s] = (j0 + r) * g.np + k0 + c;
+                lw[s] = 1.0 / (__ldg(g.vt + j0 + r) * __ldg(g.vp + k0 + c));
+            }
+        }
 
-    issue(ia - 1);  // p plane ia-1 (zeros below the slab)
-    issue(ia);
-    issue(ia + 1);
-    for (int I = ia; I <= ib; I++) {
-        cpa_wait_1();  // this thread's copies of stages <= I are done (I+1 may be in flight)
-        __syncthreads();
-        issue(I + 2);
-        corners(I);
-        __syncthreads();
-        if (I > ia) cells(I - 1);
+        // ---- stages ------------------------------------------------------------
+        auto issue = [&](int I) {
+            if (I <= ib) {
+                double* P = Ps + (I & 3) * P_SLOT;
+                const bool pl = I >= 0 && I < g.nl;
+                const double* pb = a.u + (size_t)(pl ? I : 0) * plane;
+    #pragma unroll
+                for (int s = 0; s < NP_IT; s++) {
+                    if (pd[s] < 0) continue;
+                    const bool ok = pl && ((pflag >> (2 * s + 1)) & 1u);
+                    if ((pflag >> (2 * s)) & 1u)
+                        cpa16(P + pd[s], pb + ps[s], ok);
+                    else
+                        cpa8(P + pd[s], pb + ps[s], ok);
+                }
+                double* Cf = Cs + (I & 3) * C_SLOT;
+                const bool cl = I >= 0 && I < g.nl;  // plane ia-1 (p only) may be -1
+                const double* cb0 = a.ca + (size_t)(cl ? I : 0) * plane;
+    #pragma unroll
+                for (int s = 0; s < NC_IT; s++) {
+                    if (cd[s] < 0) continue;
+                    const bool ok = cl && ((cflag >> (2 * s + 1)) & 1u);
+                    const int f = (cflag >> (16 + 2 * s)) & 3u;
+                    const double* src = cb0 + f * Nl + cs[s];
+                    if ((cflag >> (2 * s)) & 1u)
+                        cpa16(Cf + cd[s], src, ok);
+                    else
+                        cpa8(Cf + cd[s], src, ok);
+                }
+            }
+            const int iq = I - 1;  // out plane I-1: its cells are computed at step I
+            if (iq >= ia && iq < ib) {
+                double* Q = Qs + ((iq + 3) % 3) * Q_SLOT;
+                const double* qb = a.out + (size_t)iq * plane;
+    #pragma unroll
+                for (int s = 0; s < NQ_IT; s++)
+                    if (qd[s] >= 0) cpa16(Q + qd[s], qb + qs[s], true);
+            }
+            cpa_commit_group();
+        };
+
+        // corner products of corner plane I: corner (J, K) = (j0 + r, k0 + c)
+        // sits between cell rows J-1, J (p rows r, r+1) and cols K-1, K
+        // (p cols c+1, c+2)
+        auto corners = [&](int I) {
+            const double* p0 = Ps + ((I - 1) & 3) * P_SLOT;
+            const double* p1 = Ps + (I & 3) * P_SLOT;
+            double* Cf = Cs + (I & 3) * C_SLOT;
+    #pragma unroll
+            for (int s = 0; s < NK_IT; s++) {
+                if (kc[s] < 0) continue;
+                double* c0 = Cf + kc[s];
+                const double A0 = c0[0], B0 = c0[CA], E0 = c0[2 * CA];
+                const double* q0 = p0 + kp[s];
+                const double* q1 = p1 + kp[s];
+                const double a00 = q0[0], a01 = q0[1], a10 = q0[PW], a11 = q0[PW + 1];
+                const double b00 = q1[0], b01 = q1[1], b10 = q1[PW], b11 = q1[PW + 1];
+                const double Dr = ((b00 - a00) + (b01 - a01)) + ((b10 - a10) + (b11 - a11));
+                const double Dt = ((a10 - a00) + (a11 - a01)) + ((b10 - b00) + (b11 - b01));
+                const double Dp = ((a01 - a00) + (a11 - a10)) + ((b01 - b00) + (b11 - b10));
+                const double sc = A0 * Dr + B0 * Dt + E0 * Dp;
+                const double A = sc * A0, B = sc * B0, E = sc * E0;
+                c0[0] = (A + B) + E;       // st +, sp +
+                c0[CA] = (A + B) - E;      // st +, sp -
+                c0[2 * CA] = (A - B) + E;  // st -, sp +
+                c0[3 * CA] = (A - B) - E;  // st -, sp -
+                // corner plane ib is the next chunk's first (or the dead outer face)
+                if (MODE == MODE_PCGA && I < ib && ((kown >> s) & 1u)) acc[0] += sc * sc;
+            }
+        };
+
+        // cells of plane i: corner planes i (sr = +1) and i+1 (sr = -1); corner
+        // rows r (st = +1), r+1 (st = -1); corner cols c (sp = +1), c+1 (sp = -1)
+        auto cells = [&](int i) {
+            const double* lo = Cs + (i & 3) * C_SLOT;
+            const double* hi = Cs + ((i + 1) & 3) * C_SLOT;
+            const double* Q = Qs + ((i + 3) % 3) * Q_SLOT;
+            const double ivr = 1.0 / __ldg(g.vr + i);
+            double* ob = a.out + (size_t)i * plane;
+    #pragma unroll
+            for (int s = 0; s < NL_IT; s++) {
+                if (lc[s] < 0) continue;
+                const double* l = lo + lc[s];
+                const double* h = hi + lc[s];
+                const double sl = (l[0] + l[CA + 1]) + (l[2 * CA + CW] + l[3 * CA + CW + 1]);
+                const double sh = (h[3 * CA] + h[2 * CA + 1]) + (h[CA + CW] + h[CW + 1]);
+                const double y = (sl - sh) * (ivr * lw[s]);
+                const double qv = Q[lq[s]];
+                if (MODE == MODE_RESID) {
+                    const double rv = qv - y;
+                    ob[lo_[s]] = rv;
+                    const double V = __ldg(g.vr + i) / lw[s];
+                    const double f = a.f[(size_t)i * plane + lo_[s]];
+                    acc[0] += V * f * f;
+                    acc[1] += V * rv * rv;
+                    acc[2] += V * rv * (a.dinv[(size_t)i * plane + lo_[s]] * rv);
+                } else {
+                    ob[lo_[s]] = qv + y;
+                }
+            }
+        };
+
+        issue(ia - 1);  // p plane ia-1 (zeros below the slab)
+        issue(ia);
+        issue(ia + 1);
+        for (int I = ia; I <= ib; I++) {
+            cpa_wait_1();  // this thread's copies of stages <= I are done (I+1 may be in flight)
+            __syncthreads();
+            issue(I + 2);
+            corners(I);
+            __syncthreads();
+            if (I > ia) cells(I - 1);
+        }
+        __syncthreads();  // the next segment refills the rings
     }
 
     if (MODE == MODE_PCGA) {
@@ -405,8 +417,8 @@ __global__ void __launch_bounds__(kThreads, MAS_ANISO_MINB) k_aniso(const AnisoA
 // ---------------------------------------------------------------------------
 // launchers
 // ---------------------------------------------------------------------------
-// r-chunking: as many chunks as keep every block resident at once (one wave
-// of MAS_ANISO_MINB blocks per SM), bounded by the reduction scratch
+// one resident wave: MAS_ANISO_MINB blocks per SM, each with an equal share of
+// the (tile, r-plane) units (bounded by the reduction scratch)
 cudaError_t launch_aniso(int mode, const AnisoArgs& a0, cudaStream_t s) {
     AnisoArgs a = a0;
     a.ntj = (a.g.nt + AJ - 1) / AJ;
@@ -419,13 +431,13 @@ cudaError_t launch_aniso(int mode, const AnisoArgs& a0, cudaStream_t s) {
         cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
         if (sms <= 0) sms = 148;
     }
-    int want = std::max(1, (MAS_ANISO_MINB * sms) / std::max(tiles, 1));
-    if (const char* e = getenv("MAS_ACHUNKS")) want = std::max(1, atoi(e));  // experiment hook
-    want = std::min(want, std::max(1, a.max_blocks / std::max(tiles, 1)));
-    want = std::min(want, a.g.nl);
-    a.chunk = (a.g.nl + want - 1) / want;
-    a.nchunk = (a.g.nl + a.chunk - 1) / a.chunk;
-    const int blocks = a.ntj * a.ntk * a.nchunk;
+    long long want = (long long)MAS_ANISO_MINB * sms;
+    if (const char* e = getenv("MAS_ABLOCKS")) want = std::max(1, atoi(e));  // experiment hook
+    want = std::min<long long>(want, (long long)tiles * a.g.nl);
+    want = std::min<long long>(want, a.max_blocks);
+    a.chunk = 0;
+    a.nchunk = 0;
+    const int blocks = (int)want;
     if (blocks <= 0) return cudaErrorInvalidValue;
     static bool attr = false;
     if (!attr) {

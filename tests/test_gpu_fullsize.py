@@ -112,3 +112,34 @@ def test_fullsize_pcg_vs_oracle(mp, oracle_mod, cfg):
     r = fo - o.apply(prob.kappa, prob.c, xg)
     true_rel = math.sqrt((V * r * r).sum() / (V * fo * fo).sum())
     assert true_rel <= 10 * prob.tol, true_rel
+
+
+# ---------------------------------------------------------------------------
+# C2a: field-aligned conduction (NEXT-4) at its bench size, bench launch
+# configuration (k_aniso r-chunks sized for one resident wave)
+# ---------------------------------------------------------------------------
+def test_fullsize_c2a_apply_and_solve(mp, oracle_mod):
+    prob = W.aniso_conduction_problem(128, 128, 256)
+    o = oracle_mod.Oracle.for_problem(prob)
+    d = lambda a: torch.from_numpy(np.array(a)).cuda()
+    g = mp.Grid(prob.mesh)
+    op = mp.Operator(g, 1, d(prob.kappa), d(prob.c), prob.bc_inner, prob.bc_outer)
+    op.set_aniso(d(prob.kpar), d(prob.bhat))
+    x = W.random_field((1,) + prob.shape, 42)
+    y = torch.empty((1,) + prob.shape, dtype=torch.float64, device="cuda")
+    op.apply(d(x), y)
+    yo = o.apply(prob.kappa, prob.c, x) + o.aniso_apply(prob.kpar, prob.bhat, x)
+    V = o.volumes()[None]
+    yg = y.cpu().numpy()
+    assert math.sqrt((V * (yg - yo) ** 2).sum() / (V * yo ** 2).sum()) <= 1e-13
+    # the full solve, warm start as in bench.py
+    f = d(prob.f)
+    op.dirichlet_rhs(d(prob.ub_inner), None, f)
+    xs = d(prob.x0)
+    st, it, rel, _ = op.solve(f, xs, prob.tol, prob.maxit)
+    rc, xo, ito, relo, _ = oracle_mod.solve_problem(prob)
+    assert st == mp.MAS_OK and rc == oracle_mod.OK
+    assert abs(it - ito) <= 1, (it, ito)
+    xg = xs.cpu().numpy()
+    if it == ito:
+        assert math.sqrt((V * (xg - xo) ** 2).sum() / (V * xo ** 2).sum()) <= 1e-10
