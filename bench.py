@@ -171,6 +171,32 @@ def oracle_runner(o, prob, f):
     return lambda k: o.pcg(prob.kappa, prob.c, f, prob.x0, 0.0, k)
 
 
+def host_dram_gbs(threads: int):
+    """Host DRAM copy bandwidth (tools/hostbw.c, OpenMP, 2 GiB per array),
+    the CPU roofline the oracle's time is set against."""
+    import ctypes
+    src = os.path.join(ROOT, "tools", "hostbw.c")
+    so = os.path.join(ROOT, "tools", "libhostbw.so")
+    try:
+        if not os.path.exists(so) or os.path.getmtime(so) < os.path.getmtime(src):
+            subprocess.check_call(["gcc", "-O2", "-fopenmp", "-shared", "-fPIC", "-o", so, src])
+        lib = ctypes.CDLL(so)
+        lib.host_copy_gbs.restype = ctypes.c_double
+        lib.host_copy_gbs.argtypes = [ctypes.c_longlong, ctypes.c_int]
+        os.environ.setdefault("OMP_NUM_THREADS", str(threads))
+        return float(lib.host_copy_gbs(1 << 28, 3))
+    except Exception:
+        return None
+
+
+# bytes per cell per iteration of the oracle's textbook (unfused) PCG, per
+# component: L p reads p, writes q (kappa, c shared: 2); <p,q> 2; x += a p,
+# r -= a q 6; ||r|| 1; z = r / D 3; <r,z> 2; p = z + b p 3 -> 19 passes
+# (SURVEY §8(d) counts 22 for the scalar case).
+def oracle_bytes_per_cell(ncomp):
+    return 8 * (2 + 19 * ncomp)
+
+
 def run_reference(args):
     """--impl reference: the CPU oracle on this box's host cores, same config,
     metric and unit; each step = 2 fixed oracle PCG iterations on the full grid."""
@@ -418,7 +444,11 @@ def main():
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         cores = cpu_cores()
         v, per = oracle_sample(prob, args.cpu_iters, cores)
+        hbw = host_dram_gbs(cores)
+        ob = oracle_bytes_per_cell(nc) * cells * v / 1e9
         cpu = {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle",
+               "host_dram_copy_gbs": hbw, "oracle_alg_gbs": ob,
+               "oracle_frac_of_host_dram": (ob / hbw) if hbw else None,
                "sample": f"{args.config} full grid, {args.cpu_iters} fixed oracle PCG iterations "
                          f"(setup subtracted via a 1-iteration run); {per:.3f} s/iteration"}
 
