@@ -120,6 +120,15 @@ __device__ __forceinline__ void cpa8(double* dst, const double* src, bool ok) {
     asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;\n" ::"r"(sa), "l"(src), "r"(ok ? 8 : 0)
                  : "memory");
 }
+// the same with a precomputed 32-bit shared-window address
+__device__ __forceinline__ void cpa16s(unsigned sa, const double* src, bool ok) {
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(sa), "l"(src), "r"(ok ? 16 : 0)
+                 : "memory");
+}
+__device__ __forceinline__ void cpa8s(unsigned sa, const double* src, bool ok) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;\n" ::"r"(sa), "l"(src), "r"(ok ? 8 : 0)
+                 : "memory");
+}
 __device__ __forceinline__ void cpa_commit_group() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
 __device__ __forceinline__ void cpa_wait_1() { asm volatile("cp.async.wait_group 1;\n" ::: "memory"); }
 
@@ -136,7 +145,7 @@ constexpr int Q_SLOT = AJ * AK;        // 512 doubles
 constexpr int SMEM_DOUBLES = 4 * P_SLOT + 4 * C_SLOT + 3 * Q_SLOT;
 // per-thread work lists (plane independent, computed once per block)
 constexpr int NP_IT = (PR * (AK / 2 + 2) + kThreads - 1) / kThreads;  // p copies
-constexpr int NC_IT = (3 * CR * (AK / 2 + 1) + kThreads - 1) / kThreads;  // coefficient copies
+constexpr int NC_IT = (CR * (AK / 2 + 1) + kThreads - 1) / kThreads;  // coefficient copies per field
 constexpr int NQ_IT = (AJ * AK / 2 + kThreads - 1) / kThreads;         // out copies
 constexpr int NK_IT = (CR * (AK + 1) + kThreads - 1) / kThreads;       // corners
 constexpr int NL_IT = (AJ * AK + kThreads - 1) / kThreads;             // cells
@@ -190,8 +199,13 @@ __global__ void __launch_bounds__(kThreads, MAS_ANISO_MINB) k_aniso(const AnisoA
         const int hw = width >> 1;  // 16-byte pairs per row
 
         // ---- per-thread work lists ---------------------------------------------
-        // copies: smem offset within the slot (-1: none), in-plane source offset,
-        // 16 B (1) or 8 B (0), row valid (rows beyond a pole / the tile: zero-fill)
+        // copies: byte offset within the slot (-1: none), in-plane source
+        // offset (elements), 16 B (1) or 8 B (0), row valid (rows beyond a
+        // pole / the tile: zero-fill).  The coefficient items are the same for
+        // the 3 fields (a, b, e) up to the field's array offset.
+        const unsigned sP = (unsigned)__cvta_generic_to_shared(Ps);
+        const unsigned sC = (unsigned)__cvta_generic_to_shared(Cs);
+        const unsigned sQ = (unsigned)__cvta_generic_to_shared(Qs);
         int pd[NP_IT], ps[NP_IT];
         unsigned pflag = 0;  // bit 2s: 16 B, bit 2s+1: row valid
         for (int s = 0; s < NP_IT; s++) {
@@ -203,43 +217,41 @@ __global__ void __launch_bounds__(kThreads, MAS_ANISO_MINB) k_aniso(const AnisoA
                 const int j = j0 - 1 + r;
                 const bool ok = j >= 0 && j < g.nt && r <= height + 1;
                 if (c < hw) {
-                    pd[s] = r * PW + 2 + 2 * c;
+                    pd[s] = 8 * (r * PW + 2 + 2 * c);
                     ps[s] = (ok ? j : 0) * g.np + k0 + 2 * c;
                     pflag |= 1u << (2 * s);
                 } else {
                     const int side = c - hw;  // 0: k0-1, 1: k0+width (periodic)
                     int k = side ? k0 + width : k0 - 1;
                     k = k < 0 ? k + g.np : (k >= g.np ? k - g.np : k);
-                    pd[s] = r * PW + (side ? 2 + width : 1);
+                    pd[s] = 8 * (r * PW + (side ? 2 + width : 1));
                     ps[s] = (ok ? j : 0) * g.np + k;
                 }
                 if (ok) pflag |= 2u << (2 * s);
             }
         }
         int cd[NC_IT], cs[NC_IT];
-        unsigned cflag = 0;  // bits as pflag, + bits 16+2s..: field f
+        unsigned cflag = 0;  // bits as pflag
         for (int s = 0; s < NC_IT; s++) {
             const int t = threadIdx.x + s * kThreads;
             cd[s] = -1;
             cs[s] = 0;
             const int crow = hw + 1;
-            if (t < 3 * CR * crow) {
-                const int fr = t / crow, c = t - fr * crow;
-                const int f = fr / CR, r = fr - f * CR;
+            if (t < CR * crow) {
+                const int r = t / crow, c = t - r * crow;
                 const int J = j0 + r;
                 const bool ok = r <= height && J < g.nt;
                 if (c < hw) {
-                    cd[s] = f * CA + r * CW + 2 * c;
+                    cd[s] = 8 * (r * CW + 2 * c);
                     cs[s] = (ok ? J : 0) * g.np + k0 + 2 * c;
                     cflag |= 1u << (2 * s);
                 } else {
                     int K = k0 + width;
                     if (K >= g.np) K -= g.np;
-                    cd[s] = f * CA + r * CW + width;
+                    cd[s] = 8 * (r * CW + width);
                     cs[s] = (ok ? J : 0) * g.np + K;
                 }
                 if (ok) cflag |= 2u << (2 * s);
-                cflag |= (unsigned)f << (16 + 2 * s);
             }
         }
         int qd[NQ_IT], qs[NQ_IT];
@@ -249,7 +261,7 @@ __global__ void __launch_bounds__(kThreads, MAS_ANISO_MINB) k_aniso(const AnisoA
             qs[s] = 0;
             if (t < height * hw) {
                 const int r = t / hw, c = t - r * hw;
-                qd[s] = r * AK + 2 * c;
+                qd[s] = 8 * (r * AK + 2 * c);
                 qs[s] = (j0 + r) * g.np + k0 + 2 * c;
             }
         }
@@ -288,7 +300,7 @@ __global__ void __launch_bounds__(kThreads, MAS_ANISO_MINB) k_aniso(const AnisoA
         // ---- stages ------------------------------------------------------------
         auto issue = [&](int I) {
             if (I <= ib) {
-                double* P = Ps + (I & 3) * P_SLOT;
+                const unsigned P = sP + (unsigned)((I & 3) * P_SLOT * 8);
                 const bool pl = I >= 0 && I < g.nl;
                 const double* pb = a.u + (size_t)(pl ? I : 0) * plane;
     #pragma unroll
@@ -296,32 +308,34 @@ __global__ void __launch_bounds__(kThreads, MAS_ANISO_MINB) k_aniso(const AnisoA
                     if (pd[s] < 0) continue;
                     const bool ok = pl && ((pflag >> (2 * s + 1)) & 1u);
                     if ((pflag >> (2 * s)) & 1u)
-                        cpa16(P + pd[s], pb + ps[s], ok);
+                        cpa16s(P + pd[s], pb + ps[s], ok);
                     else
-                        cpa8(P + pd[s], pb + ps[s], ok);
+                        cpa8s(P + pd[s], pb + ps[s], ok);
                 }
-                double* Cf = Cs + (I & 3) * C_SLOT;
+                const unsigned Cf = sC + (unsigned)((I & 3) * C_SLOT * 8);
                 const bool cl = I >= 0 && I < g.nl;  // plane ia-1 (p only) may be -1
-                const double* cb0 = a.ca + (size_t)(cl ? I : 0) * plane;
     #pragma unroll
-                for (int s = 0; s < NC_IT; s++) {
-                    if (cd[s] < 0) continue;
-                    const bool ok = cl && ((cflag >> (2 * s + 1)) & 1u);
-                    const int f = (cflag >> (16 + 2 * s)) & 3u;
-                    const double* src = cb0 + f * Nl + cs[s];
-                    if ((cflag >> (2 * s)) & 1u)
-                        cpa16(Cf + cd[s], src, ok);
-                    else
-                        cpa8(Cf + cd[s], src, ok);
+                for (int f = 0; f < 3; f++) {
+                    const double* cb = a.ca + f * Nl + (size_t)(cl ? I : 0) * plane;
+                    const unsigned Cff = Cf + (unsigned)(f * CA * 8);
+    #pragma unroll
+                    for (int s = 0; s < NC_IT; s++) {
+                        if (cd[s] < 0) continue;
+                        const bool ok = cl && ((cflag >> (2 * s + 1)) & 1u);
+                        if ((cflag >> (2 * s)) & 1u)
+                            cpa16s(Cff + cd[s], cb + cs[s], ok);
+                        else
+                            cpa8s(Cff + cd[s], cb + cs[s], ok);
+                    }
                 }
             }
             const int iq = I - 1;  // out plane I-1: its cells are computed at step I
             if (iq >= ia && iq < ib) {
-                double* Q = Qs + ((iq + 3) % 3) * Q_SLOT;
+                const unsigned Q = sQ + (unsigned)(((iq + 3) % 3) * Q_SLOT * 8);
                 const double* qb = a.out + (size_t)iq * plane;
     #pragma unroll
                 for (int s = 0; s < NQ_IT; s++)
-                    if (qd[s] >= 0) cpa16(Q + qd[s], qb + qs[s], true);
+                    if (qd[s] >= 0) cpa16s(Q + qd[s], qb + qs[s], true);
             }
             cpa_commit_group();
         };
@@ -362,7 +376,7 @@ __global__ void __launch_bounds__(kThreads, MAS_ANISO_MINB) k_aniso(const AnisoA
             const double* lo = Cs + (i & 3) * C_SLOT;
             const double* hi = Cs + ((i + 1) & 3) * C_SLOT;
             const double* Q = Qs + ((i + 3) % 3) * Q_SLOT;
-            const double ivr = 1.0 / __ldg(g.vr + i);
+            const double ivr = __ldg(a.ivr + i);
             double* ob = a.out + (size_t)i * plane;
     #pragma unroll
             for (int s = 0; s < NL_IT; s++) {

@@ -385,6 +385,7 @@ static AnisoArgs aniso_args(const mas_op* op, int mode, const double* u, double*
     a.chunk = op->chunk;
     a.max_blocks = op->max_blocks;
     a.ca = op->ca;
+    a.ivr = op->at.ivr;
     a.u = u;
     a.out = out;
     a.st = op->st;
@@ -952,12 +953,14 @@ mas_status_t mas_op_set_aniso(mas_op_t* op, const double* kpar, const double* bh
     const int nl = g->nl, nt = g->ntl, np = g->np;
     const long long N = op->Nl;
     if (!op->atab) {  // 1-D corner metrics (R22, R23), 0 on dead corners (R24)
-        std::vector<double> t(2 * (size_t)nl + 2 * (size_t)nt + np, 0.0);
+        std::vector<double> t(3 * (size_t)nl + 2 * (size_t)nt + np, 0.0);
         double *rF = t.data(), *hr = rF + nl, *sF = hr + nl, *ht = sF + nt, *hp = ht + nt;
+        double* ivr = hp + np;
         for (int il = 0; il < nl; il++) {
             const int i = g->i0 + il;
             rF[il] = g->rF[i];
             hr[il] = i > 0 ? g->rC[i] - g->rC[i - 1] : 0.0;
+            ivr[il] = 1.0 / g->tab.vr[il];
         }
         for (int j = 1; j < nt; j++) {
             sF[j] = std::sin(g->tF[j]);
@@ -972,6 +975,7 @@ mas_status_t mas_op_set_aniso(mas_op_t* op, const double* kpar, const double* bh
         op->at.sF = op->atab + 2 * nl;
         op->at.ht = op->atab + 2 * nl + nt;
         op->at.hp = op->atab + 2 * nl + 2 * nt;
+        op->at.ivr = op->atab + 2 * nl + 2 * nt + np;
     }
     if (!op->ca) ST(dmalloc(&op->ca, 3 * (size_t)N));
     // host inputs are staged through a temporary device buffer

@@ -166,6 +166,7 @@ struct AnisoTab {          // 1-D corner metrics (device), 0 on dead corners (R2
     const double* sF;      // [nt]  sin(tF_J); 0 at J = 0
     const double* ht;      // [nt]  tC_J - tC_{J-1}; 0 at J = 0
     const double* hp;      // [np]  centre distance across phi-face K (periodic)
+    const double* ivr;     // [nl]  1 / (rC^2 dr) of plane i (the kernel never divides)
 };
 
 struct AnisoArgs {
@@ -173,6 +174,7 @@ struct AnisoArgs {
     int chunk, ntj, ntk, nchunk;  // set by launch_aniso
     int max_blocks;               // capacity of scr.partials (blocks)
     const double* ca;      // [3][nl][nt][np] corner coefficients a, b, e
+    const double* ivr;     // AnisoTab::ivr
     const double* u;       // APPLY / RESID: x;  PCGA: p_k (written by kernel A(k))
     double* out;           // APPLY: y += L_par x;  RESID: r -= L_par x;  PCGA: q += L_par p
     const double* f;       // RESID: rhs
