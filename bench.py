@@ -294,14 +294,16 @@ def main():
     x = x0.clone()
     op = M.Operator(grid, nc, kappa, cmass, prob.bc_inner, prob.bc_outer)
     aniso = prob.kpar is not None
-    if aniso:
-        if world > 1:
-            raise SystemExit("C2a (field-aligned conduction) is single-GPU in this version")
-        kpar = to_dev(prob.kpar)
-        bhat = to_dev(prob.bhat)
+    if aniso:  # NEXT-4; on r-slabs it runs the NCCL loop (no P2P mailbox for its sigma)
+        if args.ptheta != 1:
+            raise SystemExit("C2a (field-aligned conduction) needs r-slabs (--ptheta 1)")
+        kpar = to_dev(prob.kpar[sl])
+        bhat = to_dev(prob.bhat[(slice(None),) + sl])
         op.set_aniso(kpar, bhat)
     transport = "single-gpu"
-    if world > 1:
+    if world > 1 and aniso:
+        transport = "nccl"
+    elif world > 1:
         transport = "nccl"
         if args.transport != "nccl":
             try:
@@ -409,7 +411,7 @@ def main():
         # library's host-staging buffers
         hxs = [hx0.clone().pin_memory() for _ in range(ksteps + 1)]
         if aniso:
-            hkp, hb = pin(prob.kpar), pin(prob.bhat)
+            hkp, hb = pin(prob.kpar[sl]), pin(prob.bhat[(slice(None),) + sl])
         op.update(hk, hc)
         if aniso:
             op.set_aniso(hkp, hb)

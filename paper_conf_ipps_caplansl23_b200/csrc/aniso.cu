@@ -68,18 +68,21 @@ __global__ void __launch_bounds__(kThreads) k_aniso_coef(const Geo g, const Anis
 }
 
 // corner coefficient f (0 a, 1 b, 2 e) of corner (I, J, K); 0 beyond the array
-// (I = nl: the global outer r-face; J = nt: the south pole / wall)
-__device__ __forceinline__ double corner_coef(const Geo& g, const double* ca, int f, int I, int J,
-                                              int K) {
-    if (I >= g.nl || J >= g.nt) return 0.0;
+// (J = nt: the south pole / wall; I = nl: the global outer r-face, or on an
+// r-slab rank+1's plane 0, taken from the ghost copy ca_hi)
+__device__ __forceinline__ double corner_coef(const Geo& g, const double* ca, const double* ca_hi,
+                                              int f, int I, int J, int K) {
+    if (J >= g.nt) return 0.0;
     if (K >= g.np) K -= g.np;
+    if (I >= g.nl) return ca_hi ? __ldg(ca_hi + f * g.plane + (long long)J * g.np + K) : 0.0;
     const long long N = (long long)g.nl * g.plane;
     return __ldg(ca + f * N + ((long long)I * g.nt + J) * g.np + K);
 }
 
 // D += (1/V) sum over the 8 corners of (sr a + st b + sp e)^2  (R26)
-__global__ void __launch_bounds__(kThreads) k_aniso_diag(const Geo g, const double* ca, double* D,
-                                                         double* dinv, int* bad) {
+__global__ void __launch_bounds__(kThreads) k_aniso_diag(const Geo g, const double* ca,
+                                                         const double* ca_hi, double* D, double* dinv,
+                                                         int* bad) {
     const long long N = (long long)g.nl * g.plane;
     for (long long P = blockIdx.x * (long long)kThreads + threadIdx.x; P < N;
          P += (long long)gridDim.x * kThreads) {
@@ -92,9 +95,9 @@ __global__ void __launch_bounds__(kThreads) k_aniso_diag(const Geo g, const doub
                 for (int dk = 0; dk < 2; dk++) {
                     const int I = i + di, J = j + dj, K = k + dk;
                     const double sr = di ? -1.0 : 1.0, st = dj ? -1.0 : 1.0, sp = dk ? -1.0 : 1.0;
-                    const double d = sr * corner_coef(g, ca, 0, I, J, K) +
-                                     st * corner_coef(g, ca, 1, I, J, K) +
-                                     sp * corner_coef(g, ca, 2, I, J, K);
+                    const double d = sr * corner_coef(g, ca, ca_hi, 0, I, J, K) +
+                                     st * corner_coef(g, ca, ca_hi, 1, I, J, K) +
+                                     sp * corner_coef(g, ca, ca_hi, 2, I, J, K);
                     s += d * d;
                 }
         const double V = g.vr[i] * g.vt[j] * g.vp[k];
@@ -108,6 +111,10 @@ __global__ void __launch_bounds__(kThreads) k_aniso_diag(const Geo g, const doub
 // ---------------------------------------------------------------------------
 // the operator term
 // ---------------------------------------------------------------------------
+__device__ __forceinline__ double2 lds2(const double* p) { return *reinterpret_cast<const double2*>(p); }
+__device__ __forceinline__ void sts2(double* p, double2 v) { *reinterpret_cast<double2*>(p) = v; }
+__device__ __forceinline__ void stg2(double* p, double2 v) { *reinterpret_cast<double2*>(p) = v; }
+__device__ __forceinline__ double2 ld2(const double* p) { return __ldg(reinterpret_cast<const double2*>(p)); }
 // cp.async (LDGSTS) with zero-fill: src_bytes = 0 writes zeros and reads
 // nothing (dead corners, rows beyond a pole, planes outside the slab)
 __device__ __forceinline__ void cpa16(double* dst, const double* src, bool ok) {
@@ -147,8 +154,6 @@ constexpr int SMEM_DOUBLES = 4 * P_SLOT + 4 * C_SLOT + 3 * Q_SLOT;
 constexpr int NP_IT = (PR * (AK / 2 + 2) + kThreads - 1) / kThreads;  // p copies
 constexpr int NC_IT = (CR * (AK / 2 + 1) + kThreads - 1) / kThreads;  // coefficient copies per field
 constexpr int NQ_IT = (AJ * AK / 2 + kThreads - 1) / kThreads;         // out copies
-constexpr int NK_IT = (CR * (AK + 1) + kThreads - 1) / kThreads;       // corners
-constexpr int NL_IT = (AJ * AK + kThreads - 1) / kThreads;             // cells
 }  // namespace
 constexpr int kAnisoSmem = SMEM_DOUBLES * (int)sizeof(double);  // 110,336 B: 2 blocks per SM
 
@@ -265,44 +270,39 @@ __global__ void __launch_bounds__(kThreads, MAS_ANISO_MINB) k_aniso(const AnisoA
                 qs[s] = (j0 + r) * g.np + k0 + 2 * c;
             }
         }
-        // corners (smem offsets into the coefficient / p slots) and cells
-        int kc[NK_IT], kp[NK_IT];
-        unsigned kown = 0;  // bit s: the corner belongs to this tile (row < height, col < width):
-                            // the last row / col is the next tile's first (sigma counts each once)
-        for (int s = 0; s < NK_IT; s++) {
-            const int t = threadIdx.x + s * kThreads;
-            kc[s] = -1;
-            kp[s] = 0;
-            if (t < (height + 1) * (width + 1)) {
-                const int r = t / (width + 1), c = t - r * (width + 1);
-                kc[s] = r * CW + c;
-                kp[s] = r * PW + c + 1;
-                if (r < height && c < width) kown |= 1u << s;
+        // compute mapping: warp w = tile row, lane l = the column pair 2l, 2l+1
+        // (cells (w, 2l..2l+1) and corners (w, 2l..2l+1)); the corners of row
+        // 8 and column 64 (the next tiles' first row / column) are an extra
+        // item of threads 0..72
+        const int w = threadIdx.x >> 5, c2 = 2 * (threadIdx.x & 31);
+        const bool crow_ok = w <= height && c2 <= width;  // corner pair in use
+        const bool cell_ok = w < height && c2 < width;    // cell pair in use (width even)
+        int xr = -1, xc = 0;  // extra corner of this thread
+        {
+            const int t = threadIdx.x;
+            if (height == AJ && t <= width) {
+                xr = AJ, xc = t;
+            } else if (width == AK && t >= AK + 1 && t - (AK + 1) < min(height + 1, AJ)) {
+                xr = t - (AK + 1), xc = AK;
             }
         }
-        int lc[NL_IT], lq[NL_IT], lo_[NL_IT];
-        double lw[NL_IT];  // 1 / (vt_j vp_k)
-        for (int s = 0; s < NL_IT; s++) {
-            const int t = threadIdx.x + s * kThreads;
-            lc[s] = -1;
-            lq[s] = 0;
-            lo_[s] = 0;
-            lw[s] = 0.0;
-            if (t < height * width) {
-                const int r = t / width, c = t - r * width;
-                lc[s] = r * CW + c;
-                lq[s] = r * AK + c;
-                lo_[s] = (j0 + r) * g.np + k0 + c;
-                lw[s] = 1.0 / (__ldg(g.vt + j0 + r) * __ldg(g.vp + k0 + c));
-            }
+        double cw0 = 0.0, cw1 = 0.0;  // 1 / (vt_j vp_k) of the two cells
+        if (cell_ok) {
+            const double vt = __ldg(g.vt + j0 + w);
+            cw0 = 1.0 / (vt * __ldg(g.vp + k0 + c2));
+            cw1 = 1.0 / (vt * __ldg(g.vp + k0 + c2 + 1));
         }
 
         // ---- stages ------------------------------------------------------------
         auto issue = [&](int I) {
             if (I <= ib) {
                 const unsigned P = sP + (unsigned)((I & 3) * P_SLOT * 8);
-                const bool pl = I >= 0 && I < g.nl;
-                const double* pb = a.u + (size_t)(pl ? I : 0) * plane;
+                // p plane I: own planes, or the r-slab ghost planes -1 / nl
+                const double* pb = I >= 0 && I < g.nl ? a.u.in + (size_t)I * plane
+                                   : I < 0            ? a.u.glo
+                                                      : a.u.ghi;
+                const bool pl = pb != nullptr;
+                if (!pl) pb = a.u.in;
     #pragma unroll
                 for (int s = 0; s < NP_IT; s++) {
                     if (pd[s] < 0) continue;
@@ -313,10 +313,14 @@ __global__ void __launch_bounds__(kThreads, MAS_ANISO_MINB) k_aniso(const AnisoA
                         cpa8s(P + pd[s], pb + ps[s], ok);
                 }
                 const unsigned Cf = sC + (unsigned)((I & 3) * C_SLOT * 8);
-                const bool cl = I >= 0 && I < g.nl;  // plane ia-1 (p only) may be -1
+                // corner plane I (plane ia-1, p only, may be -1); plane nl: the
+                // ghost copy of rank+1's plane 0, else the dead outer face
+                const bool cin = I >= 0 && I < g.nl;
+                const bool cl = cin || (I == g.nl && a.ca_hi != nullptr);
     #pragma unroll
                 for (int f = 0; f < 3; f++) {
-                    const double* cb = a.ca + f * Nl + (size_t)(cl ? I : 0) * plane;
+                    const double* cb = cin ? a.ca + f * Nl + (size_t)I * plane
+                                           : (cl ? a.ca_hi + (size_t)f * plane : a.ca);
                     const unsigned Cff = Cf + (unsigned)(f * CA * 8);
     #pragma unroll
                     for (int s = 0; s < NC_IT; s++) {
@@ -342,62 +346,92 @@ __global__ void __launch_bounds__(kThreads, MAS_ANISO_MINB) k_aniso(const AnisoA
 
         // corner products of corner plane I: corner (J, K) = (j0 + r, k0 + c)
         // sits between cell rows J-1, J (p rows r, r+1) and cols K-1, K
-        // (p cols c+1, c+2)
+        // (p cols c+1, c+2).  Each corner's raw (a, b, e) are replaced by the
+        // 4 sign combinations c[st,sp] = s a + st s b + sp s e.
+        auto corner_math = [&](double a00, double a01, double a10, double a11, double b00, double b01,
+                               double b10, double b11, double A0, double B0, double E0, double& o0,
+                               double& o1, double& o2, double& o3) -> double {
+            const double Dr = ((b00 - a00) + (b01 - a01)) + ((b10 - a10) + (b11 - a11));
+            const double Dt = ((a10 - a00) + (a11 - a01)) + ((b10 - b00) + (b11 - b01));
+            const double Dp = ((a01 - a00) + (a11 - a10)) + ((b01 - b00) + (b11 - b10));
+            const double sc = A0 * Dr + B0 * Dt + E0 * Dp;
+            const double A = sc * A0, B = sc * B0, E = sc * E0;
+            o0 = (A + B) + E;  // st +, sp +
+            o1 = (A + B) - E;  // st +, sp -
+            o2 = (A - B) + E;  // st -, sp +
+            o3 = (A - B) - E;  // st -, sp -
+            return sc;
+        };
         auto corners = [&](int I) {
             const double* p0 = Ps + ((I - 1) & 3) * P_SLOT;
             const double* p1 = Ps + (I & 3) * P_SLOT;
             double* Cf = Cs + (I & 3) * C_SLOT;
-    #pragma unroll
-            for (int s = 0; s < NK_IT; s++) {
-                if (kc[s] < 0) continue;
-                double* c0 = Cf + kc[s];
-                const double A0 = c0[0], B0 = c0[CA], E0 = c0[2 * CA];
-                const double* q0 = p0 + kp[s];
-                const double* q1 = p1 + kp[s];
-                const double a00 = q0[0], a01 = q0[1], a10 = q0[PW], a11 = q0[PW + 1];
-                const double b00 = q1[0], b01 = q1[1], b10 = q1[PW], b11 = q1[PW + 1];
-                const double Dr = ((b00 - a00) + (b01 - a01)) + ((b10 - a10) + (b11 - a11));
-                const double Dt = ((a10 - a00) + (a11 - a01)) + ((b10 - b00) + (b11 - b01));
-                const double Dp = ((a01 - a00) + (a11 - a10)) + ((b01 - b00) + (b11 - b10));
-                const double sc = A0 * Dr + B0 * Dt + E0 * Dp;
-                const double A = sc * A0, B = sc * B0, E = sc * E0;
-                c0[0] = (A + B) + E;       // st +, sp +
-                c0[CA] = (A + B) - E;      // st +, sp -
-                c0[2 * CA] = (A - B) + E;  // st -, sp +
-                c0[3 * CA] = (A - B) - E;  // st -, sp -
-                // corner plane ib is the next chunk's first (or the dead outer face)
-                if (MODE == MODE_PCGA && I < ib && ((kown >> s) & 1u)) acc[0] += sc * sc;
+            const bool own_plane = MODE == MODE_PCGA && I < ib;  // plane ib: the next segment's
+            if (crow_ok) {
+                // p cols c2+1 (scalar), c2+2..c2+3 (aligned pair), rows w, w+1
+                const double* q0 = p0 + w * PW + c2;
+                const double* q1 = p1 + w * PW + c2;
+                const double x0 = q0[1], y0 = q0[PW + 1], X0 = q1[1], Y0 = q1[PW + 1];
+                const double2 x12 = lds2(q0 + 2), y12 = lds2(q0 + PW + 2);
+                const double2 X12 = lds2(q1 + 2), Y12 = lds2(q1 + PW + 2);
+                double* c0 = Cf + w * CW + c2;
+                const double2 A0 = lds2(c0), B0 = lds2(c0 + CA), E0 = lds2(c0 + 2 * CA);
+                double o[2][4];
+                const double s0 = corner_math(x0, x12.x, y0, y12.x, X0, X12.x, Y0, Y12.x, A0.x, B0.x, E0.x,
+                                              o[0][0], o[0][1], o[0][2], o[0][3]);
+                const double s1 = corner_math(x12.x, x12.y, y12.x, y12.y, X12.x, X12.y, Y12.x, Y12.y, A0.y,
+                                              B0.y, E0.y, o[1][0], o[1][1], o[1][2], o[1][3]);
+#pragma unroll
+                for (int q = 0; q < 4; q++) sts2(c0 + q * CA, make_double2(o[0][q], o[1][q]));
+                // sigma: corners of this tile (row < height, col < width) only
+                if (own_plane && w < height && c2 < width) acc[0] += s0 * s0 + s1 * s1;
+            }
+            if (xr >= 0) {  // row 8 / column 64: counted by the neighbouring tile
+                const double* q0 = p0 + xr * PW + xc + 1;
+                const double* q1 = p1 + xr * PW + xc + 1;
+                double* c0 = Cf + xr * CW + xc;
+                double o0, o1, o2, o3;
+                corner_math(q0[0], q0[1], q0[PW], q0[PW + 1], q1[0], q1[1], q1[PW], q1[PW + 1], c0[0],
+                            c0[CA], c0[2 * CA], o0, o1, o2, o3);
+                c0[0] = o0;
+                c0[CA] = o1;
+                c0[2 * CA] = o2;
+                c0[3 * CA] = o3;
             }
         };
 
-        // cells of plane i: corner planes i (sr = +1) and i+1 (sr = -1); corner
-        // rows r (st = +1), r+1 (st = -1); corner cols c (sp = +1), c+1 (sp = -1)
+        // cells (w, c2), (w, c2+1) of plane i: corner planes i (sr = +1) and
+        // i+1 (sr = -1); corner rows w (st = +1), w+1 (st = -1); corner cols
+        // c (sp = +1), c+1 (sp = -1).  Plane i gives c[st,sp] of the 4 corners,
+        // plane i+1 gives -c[-st,-sp].
         auto cells = [&](int i) {
-            const double* lo = Cs + (i & 3) * C_SLOT;
-            const double* hi = Cs + ((i + 1) & 3) * C_SLOT;
-            const double* Q = Qs + ((i + 3) % 3) * Q_SLOT;
+            if (!cell_ok) return;
+            const double* l = Cs + (i & 3) * C_SLOT + w * CW + c2;
+            const double* h = Cs + ((i + 1) & 3) * C_SLOT + w * CW + c2;
+            const double2 l0 = lds2(l), l2 = lds2(l + 2 * CA + CW);
+            const double2 h3 = lds2(h + 3 * CA), h1 = lds2(h + CA + CW);
+            const double l1a = l[CA + 1], l1b = l[CA + 2];
+            const double l3a = l[3 * CA + CW + 1], l3b = l[3 * CA + CW + 2];
+            const double h2a = h[2 * CA + 1], h2b = h[2 * CA + 2];
+            const double h0a = h[CW + 1], h0b = h[CW + 2];
+            const double s0 = ((l0.x + l1a) + (l2.x + l3a)) - ((h3.x + h2a) + (h1.x + h0a));
+            const double s1 = ((l0.y + l1b) + (l2.y + l3b)) - ((h3.y + h2b) + (h1.y + h0b));
             const double ivr = __ldg(a.ivr + i);
-            double* ob = a.out + (size_t)i * plane;
-    #pragma unroll
-            for (int s = 0; s < NL_IT; s++) {
-                if (lc[s] < 0) continue;
-                const double* l = lo + lc[s];
-                const double* h = hi + lc[s];
-                const double sl = (l[0] + l[CA + 1]) + (l[2 * CA + CW] + l[3 * CA + CW + 1]);
-                const double sh = (h[3 * CA] + h[2 * CA + 1]) + (h[CA + CW] + h[CW + 1]);
-                const double y = (sl - sh) * (ivr * lw[s]);
-                const double qv = Q[lq[s]];
-                if (MODE == MODE_RESID) {
-                    const double rv = qv - y;
-                    ob[lo_[s]] = rv;
-                    const double V = __ldg(g.vr + i) / lw[s];
-                    const double f = a.f[(size_t)i * plane + lo_[s]];
-                    acc[0] += V * f * f;
-                    acc[1] += V * rv * rv;
-                    acc[2] += V * rv * (a.dinv[(size_t)i * plane + lo_[s]] * rv);
-                } else {
-                    ob[lo_[s]] = qv + y;
-                }
+            const double y0 = s0 * (ivr * cw0), y1 = s1 * (ivr * cw1);
+            const double2 qv = lds2(Qs + ((i + 3) % 3) * Q_SLOT + w * AK + c2);
+            double* o = a.out + (size_t)i * plane + (j0 + w) * g.np + k0 + c2;
+            if (MODE == MODE_RESID) {
+                const double r0 = qv.x - y0, r1 = qv.y - y1;
+                stg2(o, make_double2(r0, r1));
+                const double vr = __ldg(g.vr + i);
+                const double V0 = vr / cw0, V1 = vr / cw1;
+                const double2 f = ld2(a.f + (o - a.out));
+                const double2 di = ld2(a.dinv + (o - a.out));
+                acc[0] += V0 * f.x * f.x + V1 * f.y * f.y;
+                acc[1] += V0 * r0 * r0 + V1 * r1 * r1;
+                acc[2] += V0 * r0 * (di.x * r0) + V1 * r1 * (di.y * r1);
+            } else {
+                stg2(o, make_double2(qv.x + y0, qv.y + y1));
             }
         };
 
@@ -477,11 +511,11 @@ cudaError_t launch_aniso_coef(const Geo& g, AnisoTab t, const double* kpar, cons
     return cudaGetLastError();
 }
 
-cudaError_t launch_aniso_diag(const Geo& g, const double* ca, double* D, double* dinv, int* bad,
-                              cudaStream_t s) {
+cudaError_t launch_aniso_diag(const Geo& g, const double* ca, const double* ca_hi, double* D,
+                              double* dinv, int* bad, cudaStream_t s) {
     const long long N = (long long)g.nl * g.plane;
     const int blocks = (int)std::min<long long>((N + kThreads - 1) / kThreads, 148LL * 16);
-    k_aniso_diag<<<blocks, kThreads, 0, s>>>(g, ca, D, dinv, bad);
+    k_aniso_diag<<<blocks, kThreads, 0, s>>>(g, ca, ca_hi, D, dinv, bad);
     return cudaGetLastError();
 }
 

@@ -145,6 +145,8 @@ struct mas_op {
     // field-aligned conduction term L_par (NEXT-4, mas_op_set_aniso)
     int aniso = 0;
     double* ca = nullptr;                        // corner coefficients [3][nl][nt][np]
+    double* cag = nullptr;                       // r-slabs: their ghost planes [2][3][plane]
+    double* pkg = nullptr;                       // r-slabs: p_k ghost planes [2][plane]
     double* atab = nullptr;                      // AnisoTab arrays (device)
     AnisoTab at{};
 };
@@ -368,6 +370,11 @@ static P2P p2p_args(const mas_op* op) {
     return t;
 }
 
+// r-slabs: the corner plane above the slab is rank+1's plane 0 (ghost copy)
+static const double* aniso_ca_hi(const mas_op* op) {
+    return (op->cag && !op->geo.glob_hi) ? op->cag + 3 * op->geo.plane : nullptr;
+}
+
 // D (optional) and 1/D: the 7-point diagonal (k_diag), plus the field-aligned
 // term's diagonal (R26) when L_par is on (D then goes through a device buffer:
 // the caller's, or q, which is free outside a solve).
@@ -375,16 +382,17 @@ static mas_status_t op_diag(mas_op* op, double* D_out, cudaStream_t s) {
     double* D = op->aniso && !D_out ? op->q : D_out;
     CU(launch_diag(op->geo, halo_of(op, op->kappa, op->kg, 1), packed_rows(op, op->kgt, 1), op->c, D,
                    op->dinv, op->bad, s));
-    if (op->aniso) CU(launch_aniso_diag(op->geo, op->ca, D, op->dinv, op->bad, s));
+    if (op->aniso) CU(launch_aniso_diag(op->geo, op->ca, aniso_ca_hi(op), D, op->dinv, op->bad, s));
     return MAS_OK;
 }
 
-static AnisoArgs aniso_args(const mas_op* op, int mode, const double* u, double* out) {
+static AnisoArgs aniso_args(const mas_op* op, int mode, Halo u, double* out) {
     AnisoArgs a{};
     a.g = op->geo;
     a.chunk = op->chunk;
     a.max_blocks = op->max_blocks;
     a.ca = op->ca;
+    a.ca_hi = aniso_ca_hi(op);
     a.ivr = op->at.ivr;
     a.u = u;
     a.out = out;
@@ -434,7 +442,7 @@ static mas_status_t op_load(mas_op* op, const double* kappa, const double* mass,
 static void op_free(mas_op* op) {
     if (!op) return;
     for (double* p : {op->kgt, op->dgt, op->xgt, op->rgt, op->pgt[0], op->pgt[1], op->tpack, op->ca,
-                      op->atab})
+                      op->atab, op->cag, op->pkg})
         if (p) cudaFree(p);
     for (double* p : {op->kappa, op->c, op->dinv, op->kg, op->dg, op->wR, op->r, op->p[0], op->p[1],
                       op->q, op->rg, op->pg[0], op->pg[1], op->xg, op->stage_a, op->stage_b,
@@ -515,7 +523,7 @@ static mas_status_t loop_graph(mas_op* op, StencilArgs a, StreamArgs b, AnisoArg
                 a.tpold = pold_trows(op, kk);
                 a.pnew = op->p[kk & 1];
                 e = launch_stencil(MODE_PCGA, nc, a, op->cap_stream);
-                an.u = a.pnew;
+                an.u = Halo{a.pnew, nullptr, nullptr, 0, 0};  // one GPU
                 if (e == cudaSuccess && op->aniso) e = launch_aniso(MODE_PCGA, an, op->cap_stream);
                 if (e == cudaSuccess) e = launch_pcg_b(b, op->b_blocks, op->cap_stream);
             }
@@ -742,7 +750,8 @@ mas_status_t mas_op_apply(const mas_op_t* op_c, const double* x, double* y, cuda
     a.out = yd;
     a.scr = op->scr;
     CU(launch_stencil(MODE_APPLY, op->ncomp, a, stream));
-    if (op->aniso) CU(launch_aniso(MODE_APPLY, aniso_args(op, MODE_APPLY, xd, yd), stream));
+    if (op->aniso)
+        CU(launch_aniso(MODE_APPLY, aniso_args(op, MODE_APPLY, halo_of(op, xd, op->xg, 1), yd), stream));
     if (hy) {
         CU(cudaMemcpyAsync(y, yd, bytes, cudaMemcpyDeviceToHost, stream));
         CU(cudaStreamSynchronize(stream));
@@ -812,6 +821,8 @@ mas_status_t mas_op_dot(const mas_op_t* op_c, const double* a, const double* b, 
 mas_status_t mas_op_enable_p2p(mas_op_t* op, cudaStream_t s) {
     if (!op) return arg_error("null op");
     if (op->p2p) return MAS_OK;
+    if (op->aniso)  // the mailbox carries kernel A's sigma only; L_par runs the NCCL loop
+        return arg_error("P2P transport with the field-aligned term (mas_op_set_aniso) is not supported");
     Comm* comm = op->g->comm;
     const int P = comm_nranks(comm), rank = comm_rank(comm);
     const bool virt = comm_is_virtual(comm);
@@ -943,12 +954,16 @@ mas_status_t mas_op_set_aniso(mas_op_t* op, const double* kpar, const double* bh
         op->aniso = 0;
         CU(cudaMemsetAsync(op->bad, 0, sizeof(int), stream));
         ST(op_diag(op, nullptr, stream));
+        if (op->g->comm)
+            ST(comm_seams(op->g->comm, op->dinv, 1, op->g->nl, op->geo.plane, op->dg,
+                          op->dg + op->geo.plane, stream, rstride(op)));
         return MAS_OK;
     }
     if (!bhat) return arg_error("null bhat");
     if (op->ncomp != 1) return arg_error("field-aligned conduction needs ncomp == 1");
-    if (op->g->comm || op->g->nranks > 1)
-        return arg_error("field-aligned conduction is single-GPU in this version");
+    if (op->g->ptheta > 1)
+        return arg_error("field-aligned conduction: r-slab decompositions only (ptheta == 1)");
+    if (op->p2p) return arg_error("field-aligned conduction runs the NCCL loop (P2P transport is on)");
     mas_grid* g = op->g;
     const int nl = g->nl, nt = g->ntl, np = g->np;
     const long long N = op->Nl;
@@ -978,6 +993,10 @@ mas_status_t mas_op_set_aniso(mas_op_t* op, const double* kpar, const double* bh
         op->at.ivr = op->atab + 2 * nl + 2 * nt + np;
     }
     if (!op->ca) ST(dmalloc(&op->ca, 3 * (size_t)N));
+    if (op->g->comm && !op->cag) {
+        ST(dmalloc(&op->cag, 6 * (size_t)op->geo.plane));
+        ST(dmalloc(&op->pkg, 2 * (size_t)op->geo.plane));
+    }
     // host inputs are staged through a temporary device buffer
     const double *kd = kpar, *bd = bhat;
     double* tmp = nullptr;
@@ -995,15 +1014,32 @@ mas_status_t mas_op_set_aniso(mas_op_t* op, const double* kpar, const double* bh
     }
     CU(cudaMemsetAsync(op->bad, 0, sizeof(int), stream));
     CU(launch_aniso_coef(op->geo, op->at, kd, bd, op->ca, op->bad, stream));
+    Comm* comm = op->g->comm;
+    const long long plane = op->geo.plane;
+    if (comm)  // the corner plane above the slab: rank+1's plane 0 of (a, b, e)
+        ST(comm_seams(comm, op->ca, 3, op->g->nl, plane, op->cag, op->cag + 3 * plane, stream,
+                      rstride(op)));
     op->aniso = 1;
     ST(op_diag(op, nullptr, stream));
+    if (comm)
+        ST(comm_seams(comm, op->dinv, 1, op->g->nl, plane, op->dg, op->dg + plane, stream, rstride(op)));
     int bad = 0;
     CU(cudaMemcpyAsync(&bad, op->bad, sizeof(int), cudaMemcpyDeviceToHost, stream));
     CU(cudaStreamSynchronize(stream));
     if (tmp) cudaFree(tmp);
+    if (comm) {  // agree on the verdict across ranks
+        double* d = op->dot_out;
+        double hb = bad;
+        CU(cudaMemcpyAsync(d, &hb, sizeof(double), cudaMemcpyHostToDevice, stream));
+        ST(comm_allreduce(comm, d, 1, stream));
+        CU(cudaMemcpyAsync(&hb, d, sizeof(double), cudaMemcpyDeviceToHost, stream));
+        CU(cudaStreamSynchronize(stream));
+        bad = hb != 0.0;
+    }
     if (bad) {
         op->aniso = 0;
         op_diag(op, nullptr, stream);
+        if (comm) comm_seams(comm, op->dinv, 1, op->g->nl, plane, op->dg, op->dg + plane, stream, rstride(op));
         return arg_error("kpar negative or non-finite, b non-finite, or Jacobi diagonal D <= 0");
     }
     return MAS_OK;
@@ -1076,13 +1112,13 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
     CU(launch_stencil(MODE_RESID, nc, a, s));
     op->launches++;
     AnisoArgs an{};
-    if (op->aniso) {  // r -= L_par x0 and the three initial dots again (one GPU only)
-        an = aniso_args(op, MODE_RESID, xd, op->r);
+    if (op->aniso) {  // r -= L_par x0 and the three initial dots again (rank-local sums)
+        an = aniso_args(op, MODE_RESID, halo_of(op, xd, op->xg, 1), op->r);
         an.f = fd;
         an.dinv = op->dinv;
         CU(launch_aniso(MODE_RESID, an, s));
         op->launches++;
-        an = aniso_args(op, MODE_PCGA, nullptr, op->q);
+        an = aniso_args(op, MODE_PCGA, Halo{}, op->q);
     }
     if (comm && !p2p) ST(comm_allreduce(comm, &op->st->pend_rho, 3, s));  // rho, rr, ff
 
@@ -1119,7 +1155,7 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
         a.pnew = op->p[1];
         CU(launch_stencil(MODE_PCGA, nc, a, s, true));
         if (op->aniso) {
-            an.u = a.pnew;
+            an.u = Halo{a.pnew, nullptr, nullptr, 0, 0};  // one GPU
             CU(launch_aniso(MODE_PCGA, an, s));
         }
         CU(launch_pcg_b(b, op->b_blocks, s));
@@ -1185,8 +1221,11 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
             op->launches++;
         }
         if (pe) CU(cudaEventRecord(pe[1], s));
-        if (op->aniso) {  // q += L_par p_k, sigma += <p_k, L_par p_k> (one GPU only)
-            an.u = pnew;
+        if (op->aniso) {  // q += L_par p_k, sigma += <p_k, L_par p_k> (rank-local)
+            if (comm)  // the p_k planes of the r-neighbours (kernel A(k) just wrote them)
+                ST(comm_seams(comm, pnew, 1, op->g->nl, plane, op->pkg, op->pkg + plane, s,
+                              rstride(op)));
+            an.u = halo_of(op, pnew, op->pkg, 1);
             if (pe) CU(cudaEventRecord(pe[4], s));
             CU(launch_aniso(MODE_PCGA, an, s));
             if (pe) CU(cudaEventRecord(pe[5], s));

@@ -174,8 +174,10 @@ struct AnisoArgs {
     int chunk, ntj, ntk, nchunk;  // set by launch_aniso
     int max_blocks;               // capacity of scr.partials (blocks)
     const double* ca;      // [3][nl][nt][np] corner coefficients a, b, e
+    const double* ca_hi;   // r-slabs: corner plane nl = rank+1's plane 0, [3][plane]; or nullptr
     const double* ivr;     // AnisoTab::ivr
-    const double* u;       // APPLY / RESID: x;  PCGA: p_k (written by kernel A(k))
+    Halo u;                // APPLY / RESID: x;  PCGA: p_k (written by kernel A(k)); r-slab
+                           // ghost planes -1 / nl (nullptr at a global boundary)
     double* out;           // APPLY: y += L_par x;  RESID: r -= L_par x;  PCGA: q += L_par p
     const double* f;       // RESID: rhs
     const double* dinv;    // RESID: 1/D (for <r, D^-1 r>)
@@ -208,8 +210,8 @@ cudaError_t launch_aniso(int mode, const AnisoArgs& a, cudaStream_t s);
 cudaError_t launch_aniso_coef(const Geo& g, AnisoTab t, const double* kpar, const double* bhat,
                               double* ca, int* bad, cudaStream_t s);
 // D += (1/V) sum_c (sr a + st b + sp e)^2 (R26); dinv = 1/D; *bad |= 1 if D <= 0
-cudaError_t launch_aniso_diag(const Geo& g, const double* ca, double* D, double* dinv, int* bad,
-                              cudaStream_t s);
+cudaError_t launch_aniso_diag(const Geo& g, const double* ca, const double* ca_hi, double* D,
+                              double* dinv, int* bad, cudaStream_t s);
 
 void set_last_error(const std::string& msg);
 
