@@ -674,7 +674,13 @@ mas_status_t mas_op_setup(mas_grid_t* g, int ncomp, const double* kappa, const d
     if (op->chunk < 1 || op->chunk > 64) op->chunk = 16;
     op->max_blocks = stencil_blocks(G, op->chunk);
     const char* bb_env = getenv("MAS_BBLOCKS");  // experiment hook
-    op->b_blocks = bb_env ? atoi(bb_env) : 148 * 8;
+    // kernel B: 4 blocks per SM (a sweep over 3..8 per SM: 4 and 8 are best at
+    // C3, 4 is 13% faster than 8 at C2, profiles/README.md r1g)
+    int sms = 148, dev = 0;
+    if (cudaGetDevice(&dev) == cudaSuccess)
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    if (sms <= 0) sms = 148;
+    op->b_blocks = bb_env ? atoi(bb_env) : 4 * sms;
     if (op->b_blocks > op->max_blocks) op->max_blocks = op->b_blocks;
     TRY(dmalloc(&op->scr.partials, 4 * (size_t)op->max_blocks));
     TRY(dmalloc(&op->scr.ticket, 8));

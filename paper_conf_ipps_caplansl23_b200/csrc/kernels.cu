@@ -883,6 +883,48 @@ __global__ void __launch_bounds__(kThreads) k_pcg_b(const StreamArgs a) {
         const int tpr = min(kThreads, half), rpi = kThreads / tpr;
         const int sub = threadIdx.x / tpr, col = threadIdx.x - sub * tpr;
         if (sub >= rpi) goto reduce;
+#ifndef MAS_B_NO_U2
+        if (NC == 1) {
+            // scalar operator (C2: 4 M cells, ~7 rows per block): two rows per
+            // step, all six loads in flight before the arithmetic
+            const int stride = gridDim.x * rpi;
+            for (int row = blockIdx.x * rpi + sub; row < rows; row += 2 * stride) {
+                const int row2 = row + stride;
+                const bool two = row2 < rows;
+                const int i1 = row / g.nt, j1 = row - i1 * g.nt;
+                const int i2 = two ? row2 / g.nt : i1, j2 = two ? row2 - i2 * g.nt : j1;
+                const double w1 = __ldg(g.vr + i1) * __ldg(g.vt + j1);
+                const double w2 = __ldg(g.vr + i2) * __ldg(g.vt + j2);
+                const long long b1 = (long long)row * g.np, b2 = (long long)(two ? row2 : row) * g.np;
+                for (int h = col; h < half; h += tpr) {
+                    const int k = 2 * h;
+                    const double2 d1 = ld2(a.dinv + b1 + k), r1 = ld_cs(a.r + b1 + k), q1 = ld_cs(a.q + b1 + k);
+                    double2 d2 = make_double2(0.0, 0.0), r2 = d2, q2 = d2;
+                    if (two) {
+                        d2 = ld2(a.dinv + b2 + k);
+                        r2 = ld_cs(a.r + b2 + k);
+                        q2 = ld_cs(a.q + b2 + k);
+                    }
+                    const double vp0 = __ldg(g.vp + k), vp1 = __ldg(g.vp + k + 1);
+                    double2 rv = r1;
+                    rv.x = fma(-alpha, q1.x, rv.x);
+                    rv.y = fma(-alpha, q1.y, rv.y);
+                    sts_cs(a.r + b1 + k, rv);
+                    acc[0] += w1 * vp0 * rv.x * (d1.x * rv.x) + w1 * vp1 * rv.y * (d1.y * rv.y);
+                    acc[1] += w1 * vp0 * rv.x * rv.x + w1 * vp1 * rv.y * rv.y;
+                    if (two) {
+                        double2 rw = r2;
+                        rw.x = fma(-alpha, q2.x, rw.x);
+                        rw.y = fma(-alpha, q2.y, rw.y);
+                        sts_cs(a.r + b2 + k, rw);
+                        acc[0] += w2 * vp0 * rw.x * (d2.x * rw.x) + w2 * vp1 * rw.y * (d2.y * rw.y);
+                        acc[1] += w2 * vp0 * rw.x * rw.x + w2 * vp1 * rw.y * rw.y;
+                    }
+                }
+            }
+            goto reduce;
+        }
+#endif
         for (int row = blockIdx.x * rpi + sub; row < rows; row += gridDim.x * rpi) {
             const int i = row / g.nt, j = row - i * g.nt;
             const double wrow = __ldg(g.vr + i) * __ldg(g.vt + j);
