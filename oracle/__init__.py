@@ -202,6 +202,18 @@ class Oracle:
         self._chk(lib().mas_ref_aniso_diag(C.byref(self.g), _p(kpar), _p(bhat), _p(D)))
         return D
 
+    def aniso_apply_slab(self, i0, nl, kpar_ext, bhat_ext, x_ext):
+        """Slab-local L_par: x_ext with ghost planes, corner fields with the
+        corner plane above the slab."""
+        x_ext = _f64(x_ext)
+        plane = self.shape[1] * self.shape[2]
+        ncomp = x_ext.size // (plane * (nl + 2))
+        y = np.empty((ncomp, nl, self.shape[1], self.shape[2]))
+        kpar_ext, bhat_ext = _f64(kpar_ext), _f64(bhat_ext)
+        self._chk(lib().mas_ref_aniso_apply_slab(C.byref(self.g), i0, nl, ncomp, _p(kpar_ext),
+                                                 _p(bhat_ext), _p(x_ext), _p(y)))
+        return y
+
     def pcg_aniso(self, kappa, c, kpar, bhat, f, x0, tol, maxit):
         """PCG on L_iso + L_par.  Returns (status, x, iters, relres, res_hist)."""
         f = _f64(f)

@@ -775,21 +775,24 @@ static double corner_W(const mas_ref_grid* g, const tables* T, int I, int J, int
     return g->rF[I] * g->rF[I] * T->sF[J] * T->hr[I] * T->ht[J] * T->hp[K];
 }
 
-/* R22: the corner gradient of u (one component, monolithic [nr][nt][np]). */
-static void corner_grad(const mas_ref_grid* g, const tables* T, const double* u, int I, int J,
-                        int K, double gr[3]) {
+/* R22: the corner gradient of u (one component).  u holds global r-planes
+ * uo .. (array plane 0 = global plane uo): uo = 0 for a monolithic field,
+ * i0 - 1 for a slab with its ghost planes. */
+#define UIDX(g, uo, i, j, k) IDX(g, (i) - (uo), j, k)
+static void corner_grad(const mas_ref_grid* g, const tables* T, const double* u, int uo, int I,
+                        int J, int K, double gr[3]) {
     int np = g->np, Km = (K + np - 1) % np, a, b, e;
     int ii[2] = {I - 1, I}, jj[2] = {J - 1, J}, kk[2] = {Km, K};
     double sr = 0.0, st = 0.0, sp = 0.0;
     for (b = 0; b < 2; b++)
         for (e = 0; e < 2; e++)
-            sr += u[IDX(g, I, jj[b], kk[e])] - u[IDX(g, I - 1, jj[b], kk[e])];
+            sr += u[UIDX(g, uo, I, jj[b], kk[e])] - u[UIDX(g, uo, I - 1, jj[b], kk[e])];
     for (a = 0; a < 2; a++)
         for (e = 0; e < 2; e++)
-            st += u[IDX(g, ii[a], J, kk[e])] - u[IDX(g, ii[a], J - 1, kk[e])];
+            st += u[UIDX(g, uo, ii[a], J, kk[e])] - u[UIDX(g, uo, ii[a], J - 1, kk[e])];
     for (a = 0; a < 2; a++)
         for (b = 0; b < 2; b++)
-            sp += u[IDX(g, ii[a], jj[b], K)] - u[IDX(g, ii[a], jj[b], Km)];
+            sp += u[UIDX(g, uo, ii[a], jj[b], K)] - u[UIDX(g, uo, ii[a], jj[b], Km)];
     gr[0] = sr / (4.0 * T->hr[I]);
     gr[1] = st / (4.0 * g->rF[I] * T->ht[J]);
     gr[2] = sp / (4.0 * g->rF[I] * T->sF[J] * T->hp[K]);
@@ -804,10 +807,13 @@ static void corner_dgrad(const mas_ref_grid* g, const tables* T, int I, int J, i
 }
 
 /* R21 / R26 for cell (i,j,k): sum over its 8 corners of W kpar (b.g)(b.dg)
- * (want_diag: W kpar (b.dg)^2), divided by V_P.  u may be NULL for the diagonal. */
-static double aniso_cell(const mas_ref_grid* g, const tables* T, const double* kpar,
-                         const double* bhat, const double* u, int i, int j, int k, int want_diag) {
-    size_t N = (size_t)g->nr * g->nt * g->np;
+ * (want_diag: W kpar (b.dg)^2), divided by V_P.  u may be NULL for the diagonal.
+ * The corner fields hold global corner planes co .. (bhat components Nc apart),
+ * u holds global planes uo .. (UIDX); monolithic: co = uo = 0, Nc = N. */
+static double aniso_cell_at(const mas_ref_grid* g, const tables* T, const double* kpar,
+                            const double* bhat, size_t Nc, int co, const double* u, int uo,
+                            int i, int j, int k, int want_diag) {
+    size_t N = Nc;
     double acc = 0.0;
     int a, b, e;
     for (a = 0; a < 2; a++)           /* a = 1: the corner plane I = i (cell above it) */
@@ -817,7 +823,7 @@ static double aniso_cell(const mas_ref_grid* g, const tables* T, const double* k
                 size_t C;
                 double W, kc, bv[3], d[3], bd, gr[3];
                 if (!corner_live(g, I, J)) continue;
-                C = IDX(g, I, J, K);
+                C = IDX(g, I - co, J, K);
                 W = corner_W(g, T, I, J, K);
                 kc = kpar[C];
                 bv[0] = bhat[C]; bv[1] = bhat[N + C]; bv[2] = bhat[2 * N + C];
@@ -826,11 +832,17 @@ static double aniso_cell(const mas_ref_grid* g, const tables* T, const double* k
                 if (want_diag) {
                     acc += W * kc * bd * bd;
                 } else {
-                    corner_grad(g, T, u, I, J, K, gr);
+                    corner_grad(g, T, u, uo, I, J, K, gr);
                     acc += W * kc * (bv[0] * gr[0] + bv[1] * gr[1] + bv[2] * gr[2]) * bd;
                 }
             }
     return acc / cell_V(g, T, i, j, k);
+}
+
+static double aniso_cell(const mas_ref_grid* g, const tables* T, const double* kpar,
+                         const double* bhat, const double* u, int i, int j, int k, int want_diag) {
+    return aniso_cell_at(g, T, kpar, bhat, (size_t)g->nr * g->nt * g->np, 0, u, 0, i, j, k,
+                         want_diag);
 }
 
 static int aniso_check(const mas_ref_grid* g, const double* kpar, const double* bhat) {
@@ -905,4 +917,37 @@ int mas_ref_pcg_solve_aniso(const mas_ref_grid* g, int ncomp, const double* kapp
                             double* relres, double* res_hist) {
     if (!aniso_check(g, kpar, bhat)) return MAS_REF_ERR_ARG;
     return pcg_core(g, ncomp, kappa, c, kpar, bhat, f, x, tol, maxit, iters, relres, res_hist);
+}
+
+/* Slab-local L_par for a rank owning r-planes [i0, i0+nl) (the r-slab
+ * protocol of the library): x_ext [ncomp][nl+2][nt][np] with
+ * the ghost planes i0-1 / i0+nl at ext planes 0 / nl+1; the corner fields
+ * kpar_ext [nl+1][nt][np], bhat_ext [3][nl+1][nt][np] hold corner planes
+ * i0 .. i0+nl (the last one is rank+1's first; ignored at the global outer
+ * face).  y [ncomp][nl][nt][np]. */
+int mas_ref_aniso_apply_slab(const mas_ref_grid* g, int i0, int nl, int ncomp,
+                             const double* kpar_ext, const double* bhat_ext,
+                             const double* x_ext, double* y) {
+    tables T;
+    size_t plane, Nc, Ne, Nl;
+    int il;
+    if (!aniso_check(g, kpar_ext, bhat_ext) || !x_ext || !y || ncomp < 1 || nl < 1 || i0 < 0 ||
+        i0 + nl > g->nr || tables_make(g, &T))
+        return MAS_REF_ERR_ARG;
+    plane = (size_t)g->nt * g->np;
+    Nc = plane * (nl + 1);
+    Ne = plane * (nl + 2);
+    Nl = plane * nl;
+#pragma omp parallel for schedule(static)
+    for (il = 0; il < nl; il++) {
+        int j, k, m, i = i0 + il;
+        for (m = 0; m < ncomp; m++)
+            for (j = 0; j < g->nt; j++)
+                for (k = 0; k < g->np; k++)
+                    y[(size_t)m * Nl + IDX(g, il, j, k)] =
+                        aniso_cell_at(g, &T, kpar_ext, bhat_ext, Nc, i0, x_ext + (size_t)m * Ne,
+                                      i0 - 1, i, j, k, 0);
+    }
+    tables_free(&T);
+    return MAS_REF_OK;
 }

@@ -125,6 +125,12 @@ int mas_ref_aniso_apply(const mas_ref_grid* g, int ncomp, const double* kpar,
 /* Diagonal of L_par (R26). */
 int mas_ref_aniso_diag(const mas_ref_grid* g, const double* kpar, const double* bhat,
                        double* D);
+/* Slab-local L_par (r-slab protocol): x_ext [ncomp][nl+2][nt][np] with ghost
+ * planes i0-1 / i0+nl; kpar_ext [nl+1][nt][np], bhat_ext [3][nl+1][nt][np]
+ * hold corner planes i0 .. i0+nl; y [ncomp][nl][nt][np]. */
+int mas_ref_aniso_apply_slab(const mas_ref_grid* g, int i0, int nl, int ncomp,
+                             const double* kpar_ext, const double* bhat_ext,
+                             const double* x_ext, double* y);
 /* The Jacobi-PCG of mas_ref_pcg_solve on L = L_iso + L_par, D = D_iso + D_par. */
 int mas_ref_pcg_solve_aniso(const mas_ref_grid* g, int ncomp, const double* kappa,
                             const double* c, const double* kpar, const double* bhat,
