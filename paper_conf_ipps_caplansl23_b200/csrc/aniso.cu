@@ -13,17 +13,25 @@
 // k_aniso runs right after the fused stencil kernel of the same mode and adds
 // its term in place (APPLY: y += L_par x; RESID: r -= L_par x and the three
 // initial dots; PCGA: q += L_par p_k and sigma += <p_k, L_par p_k>_V), so
-// kernel A and kernel B are unchanged.  Work item: one 8 (theta) x 64 (phi)
-// cell tile x one chunk of r-planes; the block marches the corner planes
-// I = ia..ib: p plane I (tile + 1-cell halo, periodic in phi) into a 2-slot
-// shared ring, the (9 x 65) corner products (s a, s b, s e) of plane I into a
-// second 2-slot ring, then the cells of plane I-1 gather their 8 corners.
-// Bytes per cell (PCGA): p 8 + (a, b, e) 24 + q read/write 16 = 48 B.
+// kernel A and kernel B are unchanged.  One block per SM, warp-specialised:
+// a producer warp streams stages {p plane I with its phi halo, the 3
+// corner-coefficient fields of corner plane I, out plane I-1} into a 4-slot
+// shared ring with tensor copies (TMA, cuTensorMapEncodeTiled maps, one box
+// per field; rows beyond a pole and planes outside the slab arrive as zeros)
+// (the periodic phi-wrap cells come as 2-wide side boxes); 16 consumer warps (one per tile
+// row) compute the corner products and gather them into the cells.  Full /
+// empty mbarriers order the two sides.  Bytes per cell (PCGA):
+// p 8 + (a, b, e) 24 + q read/write 16 = 48 B.
+#include <cuda.h>
 #include <cuda_runtime.h>
+#include <cudaTypedefs.h>
 
 #include <algorithm>
 #include <cmath>
 #include <cstdlib>
+#include <cstring>
+#include <mutex>
+#include <vector>
 
 #include "mas_internal.h"
 #include "reduce.cuh"
@@ -31,9 +39,6 @@
 namespace mas {
 
 namespace {
-constexpr int AJ = 8, AK = 64;           // cell tile: theta rows x phi cells
-constexpr int PR = AJ + 2;               // p tile rows with a 1-cell halo
-constexpr int CR = AJ + 1;               // corner rows of the tile
 constexpr int TKT_ANISO = 3;
 }  // namespace
 
@@ -115,68 +120,104 @@ __device__ __forceinline__ double2 lds2(const double* p) { return *reinterpret_c
 __device__ __forceinline__ void sts2(double* p, double2 v) { *reinterpret_cast<double2*>(p) = v; }
 __device__ __forceinline__ void stg2(double* p, double2 v) { *reinterpret_cast<double2*>(p) = v; }
 __device__ __forceinline__ double2 ld2(const double* p) { return __ldg(reinterpret_cast<const double2*>(p)); }
-// cp.async (LDGSTS) with zero-fill: src_bytes = 0 writes zeros and reads
-// nothing (dead corners, rows beyond a pole, planes outside the slab)
-__device__ __forceinline__ void cpa16(double* dst, const double* src, bool ok) {
-    const unsigned sa = (unsigned)__cvta_generic_to_shared(dst);
-    asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(sa), "l"(src), "r"(ok ? 16 : 0)
-                 : "memory");
-}
-__device__ __forceinline__ void cpa8(double* dst, const double* src, bool ok) {
-    const unsigned sa = (unsigned)__cvta_generic_to_shared(dst);
-    asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;\n" ::"r"(sa), "l"(src), "r"(ok ? 8 : 0)
-                 : "memory");
-}
-// the same with a precomputed 32-bit shared-window address
-__device__ __forceinline__ void cpa16s(unsigned sa, const double* src, bool ok) {
-    asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(sa), "l"(src), "r"(ok ? 16 : 0)
-                 : "memory");
-}
-__device__ __forceinline__ void cpa8s(unsigned sa, const double* src, bool ok) {
-    asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;\n" ::"r"(sa), "l"(src), "r"(ok ? 8 : 0)
-                 : "memory");
-}
-__device__ __forceinline__ void cpa_commit_group() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
-__device__ __forceinline__ void cpa_wait_1() { asm volatile("cp.async.wait_group 1;\n" ::: "memory"); }
 
+// ---- warp-specialised pipeline ---------------------------------------------
+// One block per SM: 16 consumer warps (warp w = tile row w, lane l = the
+// column pair 2l, 2l+1) and one producer warp that streams the stages with
+// bulk copies (cp.async.bulk, the TMA engine) into a 4-slot ring, signalled by
+// mbarriers (full: bytes landed; empty: the 16 consumer warps are done).
 namespace {
-// Shared-memory rings.  A "stage" I is {p plane I, corner coefficients of
-// corner plane I, out/q plane I-1}; p and the coefficients use 4 slots
-// (slot = plane & 3), out uses 3 (slot = (plane + 3) % 3).
-constexpr int PW = AK + 4;             // p row: [pad][k0-1][64 cells][k0+width][pad], 16 B aligned
-constexpr int CW = AK + 2;             // corner row: corners k0 .. k0+64 (+ pad), 16 B aligned
-constexpr int CA = CR * CW;            // one corner array of a slot
-constexpr int P_SLOT = PR * PW;        // 680 doubles
-constexpr int C_SLOT = 4 * CA;         // raw a, b, e -> the 4 sign combinations (see corners)
-constexpr int Q_SLOT = AJ * AK;        // 512 doubles
-constexpr int SMEM_DOUBLES = 4 * P_SLOT + 4 * C_SLOT + 3 * Q_SLOT;
-// per-thread work lists (plane independent, computed once per block)
-constexpr int NP_IT = (PR * (AK / 2 + 2) + kThreads - 1) / kThreads;  // p copies
-constexpr int NC_IT = (CR * (AK / 2 + 1) + kThreads - 1) / kThreads;  // coefficient copies per field
-constexpr int NQ_IT = (AJ * AK / 2 + kThreads - 1) / kThreads;         // out copies
+constexpr int WJ = 16;                 // tile rows (one consumer warp each)
+constexpr int WK = 64;                 // tile columns (32 lanes x 2)
+constexpr int NCW = WJ;                // consumer warps
+constexpr int WTHREADS = 32 * (NCW + 1);
+constexpr int WPR = WJ + 2;            // p rows: j0-1 .. j0+16
+constexpr int WPW = WK + 4;            // p row: [k0-2][k0-1][64 cells][k0+64][k0+65]
+constexpr int WCR = WJ + 1;            // corner rows
+constexpr int WCW = WK + 2;            // corner row: K = k0 .. k0+64 (+1)
+constexpr int WCA = WCR * WCW;         // one corner array
+// every component of a slot starts 128-byte aligned (tensor-copy destinations)
+constexpr int WP_SLOT = 1232;          // p box [18][68] (1224) + pad
+constexpr int WC_SLOT = 4496;          // coefficient box [3][17][66] + combinations array 3 (4488) + pad
+constexpr int WQ_SLOT = WJ * WK;       // out box [16][64]
+constexpr int WPL = 48, WPRT = 48;     // phi-wrap side boxes of p: [18][2] (left k0-2.., right 0..)
+constexpr int WCS = 112;               // phi-wrap side box of the coefficients: [3][17][2]
+constexpr int O_C = WP_SLOT, O_Q = O_C + WC_SLOT, O_PL = O_Q + WQ_SLOT, O_PR = O_PL + WPL,
+              O_CS = O_PR + WPRT;
+constexpr int W_SLOT = O_CS + WCS;     // 6960 doubles
+constexpr int W_NSLOT = 4;
+// tensor-copy transaction bytes (whole boxes, out-of-bounds elements included)
+constexpr unsigned TX_P = WPR * WPW * 8, TX_PS = WPR * 2 * 8, TX_C = 3 * WCR * WCW * 8,
+                   TX_CS = 3 * WCR * 2 * 8, TX_Q = WJ * WK * 8;
 }  // namespace
-constexpr int kAnisoSmem = SMEM_DOUBLES * (int)sizeof(double);  // 110,336 B: 2 blocks per SM
+constexpr int kAnisoSmem = W_NSLOT * W_SLOT * (int)sizeof(double) + 3 * W_NSLOT * 8;  // 222,816 B
 
-#ifndef MAS_ANISO_MINB
-#define MAS_ANISO_MINB 2
-#endif
-// Per step I (corner plane I, cells of plane I-1):
-//   wait for stage I -> barrier A -> issue stage I+2 -> corners(I) ->
-//   barrier B -> cells(I-1)
-// Stage I+2 is issued after barrier A of step I, when every thread is past
-// step I-1, so the slots it overwrites are free.  The corner thread replaces
-// the raw (a, b, e) of its corner by the 4 sign combinations
-//   c[st,sp] = s a + st s b + sp s e   (st, sp = +-1)
-// so that a cell reads one value per corner: corner plane i (sr = +1) gives
-// c[st,sp] of its 4 corners, plane i+1 (sr = -1) gives -c[-st,-sp].
-// sigma_par = <p, L_par p>_V = sum_c s_c^2 (V L_par = G^T W K G), summed in
-// the corner phase.
+// Tensor maps of one launch (host-encoded, cuTensorMapEncodeTiled): boxes of
+// the field u, of its r-slab ghost planes, of the corner coefficients (all 3
+// fields in one box), of the corner plane above the slab, and of out.  The
+// *_s maps are the 2-wide phi-wrap side boxes (TMA does not wrap).
+struct __align__(64) AnisoMaps {
+    CUtensorMap u, u_s, lo, lo_s, hi, hi_s, ca, ca_s, cahi, cahi_s, out;
+    int has_lo, has_hi, has_cahi, pad;
+};
+
+__device__ __forceinline__ unsigned smem_u32(const void* p) { return (unsigned)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(unsigned bar, unsigned count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;\n" ::"r"(bar), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(unsigned bar, unsigned bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;\n" ::"r"(bar), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(unsigned bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];\n" ::"r"(bar) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(unsigned bar, unsigned parity) {
+    asm volatile(
+        "{\n"
+        ".reg .pred P1;\n"
+        "WAIT_%=:\n"
+        "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n"
+        "@!P1 bra WAIT_%=;\n"
+        "}\n" ::"r"(bar), "r"(parity) : "memory");
+}
+// tensor copies (TMA): one box of a tensor map into shared memory, completing
+// the box bytes on the mbarrier; out-of-bounds box elements land as zeros
+__device__ __forceinline__ void tma3(unsigned dst, const CUtensorMap* m, int c0, int c1, int c2, unsigned bar) {
+    asm volatile(
+        "cp.async.bulk.tensor.3d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4}], [%5];\n"
+        ::"r"(dst), "l"(m), "r"(c0), "r"(c1), "r"(c2), "r"(bar) : "memory");
+}
+__device__ __forceinline__ void tma2(unsigned dst, const CUtensorMap* m, int c0, int c1, unsigned bar) {
+    asm volatile(
+        "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];\n"
+        ::"r"(dst), "l"(m), "r"(c0), "r"(c1), "r"(bar) : "memory");
+}
+__device__ __forceinline__ void tma4(unsigned dst, const CUtensorMap* m, int c0, int c1, int c2, int c3,
+                                     unsigned bar) {
+    asm volatile(
+        "cp.async.bulk.tensor.4d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4, %5}], [%6];\n"
+        ::"r"(dst), "l"(m), "r"(c0), "r"(c1), "r"(c2), "r"(c3), "r"(bar) : "memory");
+}
+__device__ __forceinline__ void fence_proxy_async() {
+    asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
+}
+__device__ __forceinline__ void consumer_sync() {  // the 16 consumer warps only
+    asm volatile("bar.sync 1, %0;\n" ::"n"(32 * NCW) : "memory");
+}
+
+// Per step I (corner plane I, cells of plane I-1), consumer side:
+//   wait full(stage I) -> corners(I) -> consumer barrier -> cells(I-1) ->
+//   release stage I-1 (every read of its p, coefficients and out rows done).
+// A stage I is {p plane I, corner coefficients of corner plane I, out/q plane
+// I-1}.  The corner thread replaces the raw (a, b, e) of its corner by the 4
+// sign combinations c[st,sp] = s a + st s b + sp s e, so that a cell reads
+// one value per corner: corner plane i (sr = +1) gives c[st,sp] of its 4
+// corners, plane i+1 (sr = -1) gives -c[-st,-sp].  sigma_par = <p, L_par p>_V
+// = sum_c s_c^2 (V L_par = G^T W K G), summed in the corner phase.
 template <int MODE>
-__global__ void __launch_bounds__(kThreads, MAS_ANISO_MINB) k_aniso(const AnisoArgs a) {
-    extern __shared__ __align__(16) double sm[];
-    double* Ps = sm;
-    double* Cs = Ps + 4 * P_SLOT;
-    double* Qs = Cs + 4 * C_SLOT;
+__global__ void __launch_bounds__(WTHREADS, 1) k_aniso(const AnisoArgs a, const __grid_constant__ AnisoMaps M) {
+    extern __shared__ __align__(128) double sm[];
+    unsigned long long* bars = reinterpret_cast<unsigned long long*>(sm + W_NSLOT * W_SLOT);
     if (MODE == MODE_PCGA && __ldcg(&a.st->stopped)) {
         if (a.cond && blockIdx.x == 0 && threadIdx.x == 0)
             cudaGraphSetConditional((cudaGraphConditionalHandle)a.cond, 0);
@@ -184,12 +225,16 @@ __global__ void __launch_bounds__(kThreads, MAS_ANISO_MINB) k_aniso(const AnisoA
     }
     const Geo& g = a.g;
     const int plane = (int)g.plane;
-    const long long Nl = (long long)g.nl * plane;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const bool producer = warp == NCW;
     double acc[3] = {0.0, 0.0, 0.0};
-    // Balanced partition: the (tile, r-plane) units, tile-major, are split
-    // into gridDim.x equal ranges; a block's range covers one or two
-    // segments (a run of planes of one tile), each marched with its own
-    // pipeline (one resident wave of blocks, no tail).
+    auto P_of = [&](int slot) { return sm + slot * W_SLOT; };
+    auto C_of = [&](int slot) { return sm + slot * W_SLOT + O_C; };
+    auto Q_of = [&](int slot) { return sm + slot * W_SLOT + O_Q; };
+    const unsigned full0 = smem_u32(bars), empty0 = smem_u32(bars + W_NSLOT);
+
+    // balanced partition of the (tile, r-plane) units, tile-major (one or two
+    // segments per block)
     const long long units = (long long)a.ntj * a.ntk * g.nl;
     long long u0 = units * blockIdx.x / gridDim.x;
     const long long u1 = units * (blockIdx.x + 1) / gridDim.x;
@@ -199,262 +244,220 @@ __global__ void __launch_bounds__(kThreads, MAS_ANISO_MINB) k_aniso(const AnisoA
         const int ib = (int)min((long long)g.nl, ia + (u1 - u0));
         u0 += ib - ia;
         const int tk = tile % a.ntk, tj = tile / a.ntk;
-        const int j0 = tj * AJ, k0 = tk * AK;
-        const int height = min(AJ, g.nt - j0), width = min(AK, g.np - k0);  // width is even
-        const int hw = width >> 1;  // 16-byte pairs per row
+        const int j0 = tj * WJ, k0 = tk * WK;
+        const int height = min(WJ, g.nt - j0), width = min(WK, g.np - k0);  // width is even
 
-        // ---- per-thread work lists ---------------------------------------------
-        // copies: byte offset within the slot (-1: none), in-plane source
-        // offset (elements), 16 B (1) or 8 B (0), row valid (rows beyond a
-        // pole / the tile: zero-fill).  The coefficient items are the same for
-        // the 3 fields (a, b, e) up to the field's array offset.
-        const unsigned sP = (unsigned)__cvta_generic_to_shared(Ps);
-        const unsigned sC = (unsigned)__cvta_generic_to_shared(Cs);
-        const unsigned sQ = (unsigned)__cvta_generic_to_shared(Qs);
-        int pd[NP_IT], ps[NP_IT];
-        unsigned pflag = 0;  // bit 2s: 16 B, bit 2s+1: row valid
-        for (int s = 0; s < NP_IT; s++) {
-            const int t = threadIdx.x + s * kThreads;
-            pd[s] = -1;
-            ps[s] = 0;
-            if (t < PR * (hw + 2)) {
-                const int r = t / (hw + 2), c = t - r * (hw + 2);
-                const int j = j0 - 1 + r;
-                const bool ok = j >= 0 && j < g.nt && r <= height + 1;
-                if (c < hw) {
-                    pd[s] = 8 * (r * PW + 2 + 2 * c);
-                    ps[s] = (ok ? j : 0) * g.np + k0 + 2 * c;
-                    pflag |= 1u << (2 * s);
-                } else {
-                    const int side = c - hw;  // 0: k0-1, 1: k0+width (periodic)
-                    int k = side ? k0 + width : k0 - 1;
-                    k = k < 0 ? k + g.np : (k >= g.np ? k - g.np : k);
-                    pd[s] = 8 * (r * PW + (side ? 2 + width : 1));
-                    ps[s] = (ok ? j : 0) * g.np + k;
-                }
-                if (ok) pflag |= 2u << (2 * s);
+        // fresh rings (finite values in the cells no copy writes) and barriers
+        for (int t = threadIdx.x; t < W_NSLOT * W_SLOT; t += WTHREADS) sm[t] = 0.0;
+        if (threadIdx.x == 0) {
+            for (int q = 0; q < W_NSLOT; q++) {
+                mbar_init(full0 + 8 * q, 1);    // expect_tx by the producer; the tensor bytes
+                mbar_init(empty0 + 8 * q, NCW);
             }
         }
-        int cd[NC_IT], cs[NC_IT];
-        unsigned cflag = 0;  // bits as pflag
-        for (int s = 0; s < NC_IT; s++) {
-            const int t = threadIdx.x + s * kThreads;
-            cd[s] = -1;
-            cs[s] = 0;
-            const int crow = hw + 1;
-            if (t < CR * crow) {
-                const int r = t / crow, c = t - r * crow;
-                const int J = j0 + r;
-                const bool ok = r <= height && J < g.nt;
-                if (c < hw) {
-                    cd[s] = 8 * (r * CW + 2 * c);
-                    cs[s] = (ok ? J : 0) * g.np + k0 + 2 * c;
-                    cflag |= 1u << (2 * s);
-                } else {
-                    int K = k0 + width;
-                    if (K >= g.np) K -= g.np;
-                    cd[s] = 8 * (r * CW + width);
-                    cs[s] = (ok ? J : 0) * g.np + K;
-                }
-                if (ok) cflag |= 2u << (2 * s);
-            }
-        }
-        int qd[NQ_IT], qs[NQ_IT];
-        for (int s = 0; s < NQ_IT; s++) {
-            const int t = threadIdx.x + s * kThreads;
-            qd[s] = -1;
-            qs[s] = 0;
-            if (t < height * hw) {
-                const int r = t / hw, c = t - r * hw;
-                qd[s] = 8 * (r * AK + 2 * c);
-                qs[s] = (j0 + r) * g.np + k0 + 2 * c;
-            }
-        }
-        // compute mapping: warp w = tile row, lane l = the column pair 2l, 2l+1
-        // (cells (w, 2l..2l+1) and corners (w, 2l..2l+1)); the corners of row
-        // 8 and column 64 (the next tiles' first row / column) are an extra
-        // item of threads 0..72
-        const int w = threadIdx.x >> 5, c2 = 2 * (threadIdx.x & 31);
-        const bool crow_ok = w <= height && c2 <= width;  // corner pair in use
-        const bool cell_ok = w < height && c2 < width;    // cell pair in use (width even)
-        int xr = -1, xc = 0;  // extra corner of this thread
-        {
-            const int t = threadIdx.x;
-            if (height == AJ && t <= width) {
-                xr = AJ, xc = t;
-            } else if (width == AK && t >= AK + 1 && t - (AK + 1) < min(height + 1, AJ)) {
-                xr = t - (AK + 1), xc = AK;
-            }
-        }
-        double cw0 = 0.0, cw1 = 0.0;  // 1 / (vt_j vp_k) of the two cells
-        if (cell_ok) {
-            const double vt = __ldg(g.vt + j0 + w);
-            cw0 = 1.0 / (vt * __ldg(g.vp + k0 + c2));
-            cw1 = 1.0 / (vt * __ldg(g.vp + k0 + c2 + 1));
-        }
+        fence_proxy_async();
+        __syncthreads();
+        // stages ia-1 .. ib; stage number n = I - (ia - 1), slot n & 3, use n >> 2
+        const int nst = ib - ia + 2;
 
-        // ---- stages ------------------------------------------------------------
-        auto issue = [&](int I) {
-            if (I <= ib) {
-                const unsigned P = sP + (unsigned)((I & 3) * P_SLOT * 8);
-                // p plane I: own planes, or the r-slab ghost planes -1 / nl
-                const double* pb = I >= 0 && I < g.nl ? a.u.in + (size_t)I * plane
-                                   : I < 0            ? a.u.glo
-                                                      : a.u.ghi;
-                const bool pl = pb != nullptr;
-                if (!pl) pb = a.u.in;
-    #pragma unroll
-                for (int s = 0; s < NP_IT; s++) {
-                    if (pd[s] < 0) continue;
-                    const bool ok = pl && ((pflag >> (2 * s + 1)) & 1u);
-                    if ((pflag >> (2 * s)) & 1u)
-                        cpa16s(P + pd[s], pb + ps[s], ok);
-                    else
-                        cpa8s(P + pd[s], pb + ps[s], ok);
+        if (producer) {
+            // one lane issues the stage's tensor copies: one box per field, plus
+            // the 2-wide phi-wrap side boxes on the first / last phi tile (the
+            // consumers read the wrap cells from those)
+            const bool first = k0 == 0, last = k0 + width == g.np;
+            auto p_src = [&](int I) -> int {  // 0 dead, 1 own, 2 lo ghost, 3 hi ghost
+                return I >= 0 && I < g.nl ? 1 : (I < 0 ? (M.has_lo ? 2 : 0) : (M.has_hi ? 3 : 0));
+            };
+            auto c_src = [&](int n, int I) -> int {  // 0 none (stage ia-1), 1 own, 2 above, 3 dead
+                return n == 0 ? 0 : (I >= 0 && I < g.nl ? 1 : (M.has_cahi ? 2 : 3));
+            };
+            auto issue = [&](int n) {
+                const int I = ia - 1 + n, slot = n & 3;
+                if (n >= W_NSLOT) mbar_wait(empty0 + 8 * slot, ((n >> 2) - 1) & 1);
+                const int ps = p_src(I), cs = c_src(n, I);
+                const bool ql = I - 1 >= ia && I - 1 < ib;
+                double* base = sm + slot * W_SLOT;
+                __syncwarp();
+                if (lane == 0) {
+                    const unsigned full = full0 + 8 * slot;
+                    unsigned bytes = 0;
+                    if (ps) bytes += TX_P + (first ? TX_PS : 0u) + (last ? TX_PS : 0u);
+                    if (cs) bytes += TX_C + (last ? TX_CS : 0u);
+                    if (ql) bytes += TX_Q;
+                    mbar_expect_tx(full, bytes);
+                    const unsigned sb = smem_u32(base);
+                    const int jr = j0 - 1;
+                    if (ps == 1) {
+                        tma3(sb, &M.u, k0 - 2, jr, I, full);
+                        if (first) tma3(sb + 8 * O_PL, &M.u_s, g.np - 2, jr, I, full);
+                        if (last) tma3(sb + 8 * O_PR, &M.u_s, 0, jr, I, full);
+                    } else if (ps >= 2) {
+                        const CUtensorMap* m = ps == 2 ? &M.lo : &M.hi;
+                        const CUtensorMap* m_s = ps == 2 ? &M.lo_s : &M.hi_s;
+                        tma2(sb, m, k0 - 2, jr, full);
+                        if (first) tma2(sb + 8 * O_PL, m_s, g.np - 2, jr, full);
+                        if (last) tma2(sb + 8 * O_PR, m_s, 0, jr, full);
+                    }
+                    if (cs == 1 || cs == 3) {  // 3: the dead outer face, a box beyond the
+                                                 // last plane (read as zeros)
+                        const int Ic = cs == 1 ? I : g.nl;
+                        tma4(sb + 8 * O_C, &M.ca, k0, j0, Ic, 0, full);
+                        if (last) tma4(sb + 8 * O_CS, &M.ca_s, 0, j0, Ic, 0, full);
+                    } else if (cs == 2) {
+                        tma3(sb + 8 * O_C, &M.cahi, k0, j0, 0, full);
+                        if (last) tma3(sb + 8 * O_CS, &M.cahi_s, 0, j0, 0, full);
+                    }
+                    if (ql) tma3(sb + 8 * O_Q, &M.out, k0, j0, I - 1, full);
                 }
-                const unsigned Cf = sC + (unsigned)((I & 3) * C_SLOT * 8);
-                // corner plane I (plane ia-1, p only, may be -1); plane nl: the
-                // ghost copy of rank+1's plane 0, else the dead outer face
-                const bool cin = I >= 0 && I < g.nl;
-                const bool cl = cin || (I == g.nl && a.ca_hi != nullptr);
-    #pragma unroll
-                for (int f = 0; f < 3; f++) {
-                    const double* cb = cin ? a.ca + f * Nl + (size_t)I * plane
-                                           : (cl ? a.ca_hi + (size_t)f * plane : a.ca);
-                    const unsigned Cff = Cf + (unsigned)(f * CA * 8);
-    #pragma unroll
-                    for (int s = 0; s < NC_IT; s++) {
-                        if (cd[s] < 0) continue;
-                        const bool ok = cl && ((cflag >> (2 * s + 1)) & 1u);
-                        if ((cflag >> (2 * s)) & 1u)
-                            cpa16s(Cff + cd[s], cb + cs[s], ok);
-                        else
-                            cpa8s(Cff + cd[s], cb + cs[s], ok);
+            };
+            for (int n = 0; n < nst; n++) issue(n);
+        } else {
+            // ---- consumers --------------------------------------------------
+            const int w = warp, c2 = 2 * lane;
+            const bool first = k0 == 0, last = k0 + width == g.np;
+            const bool lfix = first && c2 == 0, rfix = last && c2 == width;
+            const bool crow_ok = w <= height && c2 <= width;  // corner pair in use
+            const bool cell_ok = w < height && c2 < width;    // cell pair in use
+            int xr = -1, xc = 0;  // extra corner: row 16 / column 64
+            {
+                const int t = threadIdx.x;
+                if (height == WJ && t <= width) {
+                    xr = WJ, xc = t;
+                } else if (width == WK && t >= WK + 1 && t - (WK + 1) < min(height + 1, WJ)) {
+                    xr = t - (WK + 1), xc = WK;
+                }
+            }
+            double cw0 = 0.0, cw1 = 0.0;  // 1 / (vt_j vp_k) of the two cells
+            if (cell_ok) {
+                const double vt = __ldg(g.vt + j0 + w);
+                cw0 = 1.0 / (vt * __ldg(g.vp + k0 + c2));
+                cw1 = 1.0 / (vt * __ldg(g.vp + k0 + c2 + 1));
+            }
+            auto corner_math = [&](double a00, double a01, double a10, double a11, double b00, double b01,
+                                   double b10, double b11, double A0, double B0, double E0, double& o0,
+                                   double& o1, double& o2, double& o3) -> double {
+                const double Dr = ((b00 - a00) + (b01 - a01)) + ((b10 - a10) + (b11 - a11));
+                const double Dt = ((a10 - a00) + (a11 - a01)) + ((b10 - b00) + (b11 - b01));
+                const double Dp = ((a01 - a00) + (a11 - a10)) + ((b01 - b00) + (b11 - b10));
+                const double sc = A0 * Dr + B0 * Dt + E0 * Dp;
+                const double A = sc * A0, B = sc * B0, E = sc * E0;
+                o0 = (A + B) + E;  // st +, sp +
+                o1 = (A + B) - E;  // st +, sp -
+                o2 = (A - B) + E;  // st -, sp +
+                o3 = (A - B) - E;  // st -, sp -
+                return sc;
+            };
+            for (int n = 0; n < nst; n++) {
+                const int I = ia - 1 + n, slot = n & 3;
+                mbar_wait(full0 + 8 * slot, (n >> 2) & 1);
+                if (n == 0) continue;  // stage ia-1: p plane ia-1 only
+                // ---- corners of plane I: p rows w, w+1 (cell rows J-1, J),
+                // p cols c2+1 .. c2+3 (cells K-1, K of the corner pair)
+                const double* p0 = P_of((n - 1) & 3);
+                const double* p1 = P_of(slot);
+                double* Cf = C_of(slot);
+                if (crow_ok) {
+                    const double* q0 = p0 + w * WPW + c2;
+                    const double* q1 = p1 + w * WPW + c2;
+                    double x0 = q0[1], y0 = q0[WPW + 1], X0 = q1[1], Y0 = q1[WPW + 1];
+                    double2 x12 = lds2(q0 + 2), y12 = lds2(q0 + WPW + 2);
+                    double2 X12 = lds2(q1 + 2), Y12 = lds2(q1 + WPW + 2);
+                    double* c0 = Cf + w * WCW + c2;
+                    double2 A0 = lds2(c0), B0 = lds2(c0 + WCA), E0 = lds2(c0 + 2 * WCA);
+                    if (lfix) {  // cell column k0-1 = np-1: the left phi-wrap box
+                        const double *L0 = p0 + O_PL, *L1 = p1 + O_PL;
+                        x0 = L0[2 * w + 1], y0 = L0[2 * w + 3], X0 = L1[2 * w + 1], Y0 = L1[2 * w + 3];
+                    }
+                    if (rfix) {  // cell column k0+width = 0 and corner column width: the right boxes
+                        const double *R0 = p0 + O_PR, *R1 = p1 + O_PR, *CS = p1 + O_CS;
+                        x12.x = R0[2 * w], y12.x = R0[2 * w + 2], X12.x = R1[2 * w], Y12.x = R1[2 * w + 2];
+                        A0.x = CS[2 * w], B0.x = CS[2 * (WCR + w)], E0.x = CS[2 * (2 * WCR + w)];
+                    }
+                    double o[2][4];
+                    const double s0 = corner_math(x0, x12.x, y0, y12.x, X0, X12.x, Y0, Y12.x, A0.x, B0.x,
+                                                  E0.x, o[0][0], o[0][1], o[0][2], o[0][3]);
+                    const double s1 = corner_math(x12.x, x12.y, y12.x, y12.y, X12.x, X12.y, Y12.x, Y12.y,
+                                                  A0.y, B0.y, E0.y, o[1][0], o[1][1], o[1][2], o[1][3]);
+#pragma unroll
+                    for (int q = 0; q < 4; q++) sts2(c0 + q * WCA, make_double2(o[0][q], o[1][q]));
+                    // sigma: this tile's corners (row < height, col < width) of the
+                    // segment's own planes (plane ib is the next segment's first)
+                    if (MODE == MODE_PCGA && I < ib && w < height && c2 < width)
+                        acc[0] += s0 * s0 + s1 * s1;
+                }
+                if (xr >= 0) {  // row 16 / column 64: counted by the neighbouring tile
+                    const double* q0 = p0 + xr * WPW + xc + 1;
+                    const double* q1 = p1 + xr * WPW + xc + 1;
+                    double* c0 = Cf + xr * WCW + xc;
+                    double a00 = q0[0], a01 = q0[1], a10 = q0[WPW], a11 = q0[WPW + 1];
+                    double b00 = q1[0], b01 = q1[1], b10 = q1[WPW], b11 = q1[WPW + 1];
+                    double A = c0[0], B = c0[WCA], E = c0[2 * WCA];
+                    if (first && xc == 0) {
+                        const double *L0 = p0 + O_PL, *L1 = p1 + O_PL;
+                        a00 = L0[2 * xr + 1], a10 = L0[2 * xr + 3], b00 = L1[2 * xr + 1], b10 = L1[2 * xr + 3];
+                    }
+                    if (last && xc == width) {
+                        const double *R0 = p0 + O_PR, *R1 = p1 + O_PR, *CS = p1 + O_CS;
+                        a01 = R0[2 * xr], a11 = R0[2 * xr + 2], b01 = R1[2 * xr], b11 = R1[2 * xr + 2];
+                        A = CS[2 * xr], B = CS[2 * (WCR + xr)], E = CS[2 * (2 * WCR + xr)];
+                    }
+                    double o0, o1, o2, o3;
+                    corner_math(a00, a01, a10, a11, b00, b01, b10, b11, A, B, E, o0, o1, o2, o3);
+                    c0[0] = o0;
+                    c0[WCA] = o1;
+                    c0[2 * WCA] = o2;
+                    c0[3 * WCA] = o3;
+                }
+                consumer_sync();
+                // ---- cells (w, c2..c2+1) of plane i = I-1: corner planes i
+                // (sr = +1) and I (sr = -1); out/q plane i from this stage
+                if (n >= 2 && cell_ok) {
+                    const int i = I - 1;
+                    const double* l = C_of((n - 1) & 3) + w * WCW + c2;
+                    const double* h = Cf + w * WCW + c2;
+                    const double2 l0 = lds2(l), l2 = lds2(l + 2 * WCA + WCW);
+                    const double2 h3 = lds2(h + 3 * WCA), h1 = lds2(h + WCA + WCW);
+                    const double l1a = l[WCA + 1], l1b = l[WCA + 2];
+                    const double l3a = l[3 * WCA + WCW + 1], l3b = l[3 * WCA + WCW + 2];
+                    const double h2a = h[2 * WCA + 1], h2b = h[2 * WCA + 2];
+                    const double h0a = h[WCW + 1], h0b = h[WCW + 2];
+                    const double s0 = ((l0.x + l1a) + (l2.x + l3a)) - ((h3.x + h2a) + (h1.x + h0a));
+                    const double s1 = ((l0.y + l1b) + (l2.y + l3b)) - ((h3.y + h2b) + (h1.y + h0b));
+                    const double ivr = __ldg(a.ivr + i);
+                    const double y0 = s0 * (ivr * cw0), y1 = s1 * (ivr * cw1);
+                    const double2 qv = lds2(Q_of(slot) + w * WK + c2);
+                    double* o = a.out + (size_t)i * plane + (size_t)(j0 + w) * g.np + k0 + c2;
+                    if (MODE == MODE_RESID) {
+                        const double r0 = qv.x - y0, r1 = qv.y - y1;
+                        stg2(o, make_double2(r0, r1));
+                        const double vr = __ldg(g.vr + i);
+                        const double V0 = vr / cw0, V1 = vr / cw1;
+                        const double2 f = ld2(a.f + (o - a.out));
+                        const double2 di = ld2(a.dinv + (o - a.out));
+                        acc[0] += V0 * f.x * f.x + V1 * f.y * f.y;
+                        acc[1] += V0 * r0 * r0 + V1 * r1 * r1;
+                        acc[2] += V0 * r0 * (di.x * r0) + V1 * r1 * (di.y * r1);
+                    } else {
+                        stg2(o, make_double2(qv.x + y0, qv.y + y1));
                     }
                 }
+                // stage n-1 is no longer read (p by corners(I), products by
+                // cells(I-1)); the combination writes went through the generic
+                // proxy, the next fill of the slot is a tensor copy
+                fence_proxy_async();
+                __syncwarp();
+                if (lane == 0) mbar_arrive(empty0 + 8 * ((n - 1) & 3));
             }
-            const int iq = I - 1;  // out plane I-1: its cells are computed at step I
-            if (iq >= ia && iq < ib) {
-                const unsigned Q = sQ + (unsigned)(((iq + 3) % 3) * Q_SLOT * 8);
-                const double* qb = a.out + (size_t)iq * plane;
-    #pragma unroll
-                for (int s = 0; s < NQ_IT; s++)
-                    if (qd[s] >= 0) cpa16s(Q + qd[s], qb + qs[s], true);
-            }
-            cpa_commit_group();
-        };
-
-        // corner products of corner plane I: corner (J, K) = (j0 + r, k0 + c)
-        // sits between cell rows J-1, J (p rows r, r+1) and cols K-1, K
-        // (p cols c+1, c+2).  Each corner's raw (a, b, e) are replaced by the
-        // 4 sign combinations c[st,sp] = s a + st s b + sp s e.
-        auto corner_math = [&](double a00, double a01, double a10, double a11, double b00, double b01,
-                               double b10, double b11, double A0, double B0, double E0, double& o0,
-                               double& o1, double& o2, double& o3) -> double {
-            const double Dr = ((b00 - a00) + (b01 - a01)) + ((b10 - a10) + (b11 - a11));
-            const double Dt = ((a10 - a00) + (a11 - a01)) + ((b10 - b00) + (b11 - b01));
-            const double Dp = ((a01 - a00) + (a11 - a10)) + ((b01 - b00) + (b11 - b10));
-            const double sc = A0 * Dr + B0 * Dt + E0 * Dp;
-            const double A = sc * A0, B = sc * B0, E = sc * E0;
-            o0 = (A + B) + E;  // st +, sp +
-            o1 = (A + B) - E;  // st +, sp -
-            o2 = (A - B) + E;  // st -, sp +
-            o3 = (A - B) - E;  // st -, sp -
-            return sc;
-        };
-        auto corners = [&](int I) {
-            const double* p0 = Ps + ((I - 1) & 3) * P_SLOT;
-            const double* p1 = Ps + (I & 3) * P_SLOT;
-            double* Cf = Cs + (I & 3) * C_SLOT;
-            const bool own_plane = MODE == MODE_PCGA && I < ib;  // plane ib: the next segment's
-            if (crow_ok) {
-                // p cols c2+1 (scalar), c2+2..c2+3 (aligned pair), rows w, w+1
-                const double* q0 = p0 + w * PW + c2;
-                const double* q1 = p1 + w * PW + c2;
-                const double x0 = q0[1], y0 = q0[PW + 1], X0 = q1[1], Y0 = q1[PW + 1];
-                const double2 x12 = lds2(q0 + 2), y12 = lds2(q0 + PW + 2);
-                const double2 X12 = lds2(q1 + 2), Y12 = lds2(q1 + PW + 2);
-                double* c0 = Cf + w * CW + c2;
-                const double2 A0 = lds2(c0), B0 = lds2(c0 + CA), E0 = lds2(c0 + 2 * CA);
-                double o[2][4];
-                const double s0 = corner_math(x0, x12.x, y0, y12.x, X0, X12.x, Y0, Y12.x, A0.x, B0.x, E0.x,
-                                              o[0][0], o[0][1], o[0][2], o[0][3]);
-                const double s1 = corner_math(x12.x, x12.y, y12.x, y12.y, X12.x, X12.y, Y12.x, Y12.y, A0.y,
-                                              B0.y, E0.y, o[1][0], o[1][1], o[1][2], o[1][3]);
-#pragma unroll
-                for (int q = 0; q < 4; q++) sts2(c0 + q * CA, make_double2(o[0][q], o[1][q]));
-                // sigma: corners of this tile (row < height, col < width) only
-                if (own_plane && w < height && c2 < width) acc[0] += s0 * s0 + s1 * s1;
-            }
-            if (xr >= 0) {  // row 8 / column 64: counted by the neighbouring tile
-                const double* q0 = p0 + xr * PW + xc + 1;
-                const double* q1 = p1 + xr * PW + xc + 1;
-                double* c0 = Cf + xr * CW + xc;
-                double o0, o1, o2, o3;
-                corner_math(q0[0], q0[1], q0[PW], q0[PW + 1], q1[0], q1[1], q1[PW], q1[PW + 1], c0[0],
-                            c0[CA], c0[2 * CA], o0, o1, o2, o3);
-                c0[0] = o0;
-                c0[CA] = o1;
-                c0[2 * CA] = o2;
-                c0[3 * CA] = o3;
-            }
-        };
-
-        // cells (w, c2), (w, c2+1) of plane i: corner planes i (sr = +1) and
-        // i+1 (sr = -1); corner rows w (st = +1), w+1 (st = -1); corner cols
-        // c (sp = +1), c+1 (sp = -1).  Plane i gives c[st,sp] of the 4 corners,
-        // plane i+1 gives -c[-st,-sp].
-        auto cells = [&](int i) {
-            if (!cell_ok) return;
-            const double* l = Cs + (i & 3) * C_SLOT + w * CW + c2;
-            const double* h = Cs + ((i + 1) & 3) * C_SLOT + w * CW + c2;
-            const double2 l0 = lds2(l), l2 = lds2(l + 2 * CA + CW);
-            const double2 h3 = lds2(h + 3 * CA), h1 = lds2(h + CA + CW);
-            const double l1a = l[CA + 1], l1b = l[CA + 2];
-            const double l3a = l[3 * CA + CW + 1], l3b = l[3 * CA + CW + 2];
-            const double h2a = h[2 * CA + 1], h2b = h[2 * CA + 2];
-            const double h0a = h[CW + 1], h0b = h[CW + 2];
-            const double s0 = ((l0.x + l1a) + (l2.x + l3a)) - ((h3.x + h2a) + (h1.x + h0a));
-            const double s1 = ((l0.y + l1b) + (l2.y + l3b)) - ((h3.y + h2b) + (h1.y + h0b));
-            const double ivr = __ldg(a.ivr + i);
-            const double y0 = s0 * (ivr * cw0), y1 = s1 * (ivr * cw1);
-            const double2 qv = lds2(Qs + ((i + 3) % 3) * Q_SLOT + w * AK + c2);
-            double* o = a.out + (size_t)i * plane + (j0 + w) * g.np + k0 + c2;
-            if (MODE == MODE_RESID) {
-                const double r0 = qv.x - y0, r1 = qv.y - y1;
-                stg2(o, make_double2(r0, r1));
-                const double vr = __ldg(g.vr + i);
-                const double V0 = vr / cw0, V1 = vr / cw1;
-                const double2 f = ld2(a.f + (o - a.out));
-                const double2 di = ld2(a.dinv + (o - a.out));
-                acc[0] += V0 * f.x * f.x + V1 * f.y * f.y;
-                acc[1] += V0 * r0 * r0 + V1 * r1 * r1;
-                acc[2] += V0 * r0 * (di.x * r0) + V1 * r1 * (di.y * r1);
-            } else {
-                stg2(o, make_double2(qv.x + y0, qv.y + y1));
-            }
-        };
-
-        issue(ia - 1);  // p plane ia-1 (zeros below the slab)
-        issue(ia);
-        issue(ia + 1);
-        for (int I = ia; I <= ib; I++) {
-            cpa_wait_1();  // this thread's copies of stages <= I are done (I+1 may be in flight)
-            __syncthreads();
-            issue(I + 2);
-            corners(I);
-            __syncthreads();
-            if (I > ia) cells(I - 1);
         }
-        __syncthreads();  // the next segment refills the rings
+        __syncthreads();  // the next segment re-initialises the rings and barriers
     }
 
     if (MODE == MODE_PCGA) {
         double v[1] = {acc[0]};
-        if (grid_reduce<1>(v, a.scr, TKT_ANISO) && threadIdx.x == 0)
+        if (grid_reduce<1, WTHREADS>(v, a.scr, TKT_ANISO) && threadIdx.x == 0)
             a.st->pend_sigma = a.st->pend_sigma + v[0];  // <p,L_iso p> (kernel A) + <p,L_par p>
     } else if (MODE == MODE_RESID) {
-        if (grid_reduce<3>(acc, a.scr, TKT_ANISO) && threadIdx.x == 0) {
+        if (grid_reduce<3, WTHREADS>(acc, a.scr, TKT_ANISO) && threadIdx.x == 0) {
             a.st->pend_ff = acc[0];
             a.st->pend_rr = acc[1];
             a.st->pend_rho = acc[2];
@@ -467,10 +470,66 @@ __global__ void __launch_bounds__(kThreads, MAS_ANISO_MINB) k_aniso(const AnisoA
 // ---------------------------------------------------------------------------
 // one resident wave: MAS_ANISO_MINB blocks per SM, each with an equal share of
 // the (tile, r-plane) units (bounded by the reduction scratch)
+static PFN_cuTensorMapEncodeTiled_v12000 tmap_encode_fn() {
+    static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+    static std::once_flag once;
+    std::call_once(once, [] {
+        void* p = nullptr;
+        cudaDriverEntryPointQueryResult q{};
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(p);
+    });
+    return fn;
+}
+
+// fp64 tiled tensor map, no swizzle, out-of-bounds elements read as zero
+static bool tmap(CUtensorMap* m, const double* base, int rank, const cuuint64_t* dims,
+                 const cuuint64_t* strides, const cuuint32_t* box) {
+    auto fn = tmap_encode_fn();
+    if (!fn || !base) return false;
+    const cuuint32_t es[5] = {1, 1, 1, 1, 1};
+    return fn(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, (cuuint32_t)rank, const_cast<double*>(base), dims, strides,
+              box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+              CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+static bool build_maps(const AnisoArgs& a, AnisoMaps* M) {
+    std::memset(M, 0, sizeof(*M));
+    const Geo& g = a.g;
+    const cuuint64_t np = (cuuint64_t)g.np, nt = (cuuint64_t)g.nt, nl = (cuuint64_t)g.nl;
+    const cuuint64_t rs = np * 8, ps = np * nt * 8, fs = np * nt * nl * 8;
+    const cuuint64_t d3[3] = {np, nt, nl}, s3[2] = {rs, ps};
+    const cuuint64_t d2[2] = {np, nt}, s2[1] = {rs};
+    const cuuint64_t d4[4] = {np, nt, nl, 3}, s4[3] = {rs, ps, fs};
+    const cuuint64_t dh[3] = {np, nt, 3}, sh[2] = {rs, ps};
+    const cuuint32_t bp[3] = {WPW, WPR, 1}, bps[3] = {2, WPR, 1};
+    const cuuint32_t bp2[2] = {WPW, WPR}, bps2[2] = {2, WPR};
+    const cuuint32_t bc[4] = {WCW, WCR, 1, 3}, bcs[4] = {2, WCR, 1, 3};
+    const cuuint32_t bh[3] = {WCW, WCR, 3}, bhs[3] = {2, WCR, 3};
+    const cuuint32_t bq[3] = {WK, WJ, 1};
+    bool ok = tmap(&M->u, a.u.in, 3, d3, s3, bp) && tmap(&M->u_s, a.u.in, 3, d3, s3, bps) &&
+              tmap(&M->ca, a.ca, 4, d4, s4, bc) && tmap(&M->ca_s, a.ca, 4, d4, s4, bcs) &&
+              tmap(&M->out, a.out, 3, d3, s3, bq);
+    if (ok && a.u.glo) {
+        M->has_lo = 1;
+        ok = tmap(&M->lo, a.u.glo, 2, d2, s2, bp2) && tmap(&M->lo_s, a.u.glo, 2, d2, s2, bps2);
+    }
+    if (ok && a.u.ghi) {
+        M->has_hi = 1;
+        ok = tmap(&M->hi, a.u.ghi, 2, d2, s2, bp2) && tmap(&M->hi_s, a.u.ghi, 2, d2, s2, bps2);
+    }
+    if (ok && a.ca_hi) {
+        M->has_cahi = 1;
+        ok = tmap(&M->cahi, a.ca_hi, 3, dh, sh, bh) && tmap(&M->cahi_s, a.ca_hi, 3, dh, sh, bhs);
+    }
+    return ok;
+}
+
 cudaError_t launch_aniso(int mode, const AnisoArgs& a0, cudaStream_t s) {
     AnisoArgs a = a0;
-    a.ntj = (a.g.nt + AJ - 1) / AJ;
-    a.ntk = (a.g.np + AK - 1) / AK;
+    a.ntj = (a.g.nt + WJ - 1) / WJ;
+    a.ntk = (a.g.np + WK - 1) / WK;
     const int tiles = a.ntj * a.ntk;
     static int sms = 0;
     if (!sms) {
@@ -479,7 +538,7 @@ cudaError_t launch_aniso(int mode, const AnisoArgs& a0, cudaStream_t s) {
         cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
         if (sms <= 0) sms = 148;
     }
-    long long want = (long long)MAS_ANISO_MINB * sms;
+    long long want = sms;  // one block per SM (223 KB of rings each)
     if (const char* e = getenv("MAS_ABLOCKS")) want = std::max(1, atoi(e));  // experiment hook
     want = std::min<long long>(want, (long long)tiles * a.g.nl);
     want = std::min<long long>(want, a.max_blocks);
@@ -487,6 +546,11 @@ cudaError_t launch_aniso(int mode, const AnisoArgs& a0, cudaStream_t s) {
     a.nchunk = 0;
     const int blocks = (int)want;
     if (blocks <= 0) return cudaErrorInvalidValue;
+    AnisoMaps M;
+    if (!build_maps(a, &M)) {
+        set_last_error("k_aniso: cuTensorMapEncodeTiled failed");
+        return cudaErrorInvalidValue;
+    }
     static bool attr = false;
     if (!attr) {
         cudaFuncSetAttribute(k_aniso<MODE_APPLY>, cudaFuncAttributeMaxDynamicSharedMemorySize, kAnisoSmem);
@@ -495,11 +559,11 @@ cudaError_t launch_aniso(int mode, const AnisoArgs& a0, cudaStream_t s) {
         attr = true;
     }
     if (mode == MODE_APPLY)
-        k_aniso<MODE_APPLY><<<blocks, kThreads, kAnisoSmem, s>>>(a);
+        k_aniso<MODE_APPLY><<<blocks, WTHREADS, kAnisoSmem, s>>>(a, M);
     else if (mode == MODE_RESID)
-        k_aniso<MODE_RESID><<<blocks, kThreads, kAnisoSmem, s>>>(a);
+        k_aniso<MODE_RESID><<<blocks, WTHREADS, kAnisoSmem, s>>>(a, M);
     else
-        k_aniso<MODE_PCGA><<<blocks, kThreads, kAnisoSmem, s>>>(a);
+        k_aniso<MODE_PCGA><<<blocks, WTHREADS, kAnisoSmem, s>>>(a, M);
     return cudaGetLastError();
 }
 
