@@ -884,7 +884,7 @@ __global__ void __launch_bounds__(kThreads) k_pcg_b(const StreamArgs a) {
         const int sub = threadIdx.x / tpr, col = threadIdx.x - sub * tpr;
         if (sub >= rpi) goto reduce;
 #ifndef MAS_B_NO_U2
-        if (NC == 1) {
+        if constexpr (NC == 1) {
             // scalar operator (C2: 4 M cells, ~7 rows per block): two rows per
             // step, all six loads in flight before the arithmetic
             const int stride = gridDim.x * rpi;
@@ -922,8 +922,7 @@ __global__ void __launch_bounds__(kThreads) k_pcg_b(const StreamArgs a) {
                     }
                 }
             }
-            goto reduce;
-        }
+        } else
 #endif
         for (int row = blockIdx.x * rpi + sub; row < rows; row += gridDim.x * rpi) {
             const int i = row / g.nt, j = row - i * g.nt;
