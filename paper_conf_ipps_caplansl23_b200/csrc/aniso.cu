@@ -347,37 +347,49 @@ __global__ void __launch_bounds__(WTHREADS, 1) k_aniso(const AnisoArgs a, const 
                 o3 = (A - B) - E;  // st -, sp -
                 return sc;
             };
+            // p of the previous plane for this thread's corners, carried in
+            // registers from one step to the next (rows w, w+1 of the pair;
+            // the extra corner's 4 cells); wrap cells from the side boxes
+            double x0 = 0.0, y0 = 0.0, e0 = 0.0, e1 = 0.0, e2 = 0.0, e3 = 0.0;
+            double2 x12 = make_double2(0.0, 0.0), y12 = x12;
             for (int n = 0; n < nst; n++) {
                 const int I = ia - 1 + n, slot = n & 3;
                 mbar_wait(full0 + 8 * slot, (n >> 2) & 1);
-                if (n == 0) continue;  // stage ia-1: p plane ia-1 only
-                // ---- corners of plane I: p rows w, w+1 (cell rows J-1, J),
-                // p cols c2+1 .. c2+3 (cells K-1, K of the corner pair)
-                const double* p0 = P_of((n - 1) & 3);
                 const double* p1 = P_of(slot);
+                double X0 = 0.0, Y0 = 0.0, E0 = 0.0, E1 = 0.0, E2 = 0.0, E3 = 0.0;
+                double2 X12 = make_double2(0.0, 0.0), Y12 = X12;
+                if (crow_ok) {
+                    const double* q1 = p1 + w * WPW + c2;
+                    X0 = q1[1], Y0 = q1[WPW + 1];
+                    X12 = lds2(q1 + 2), Y12 = lds2(q1 + WPW + 2);
+                    if (lfix) X0 = p1[O_PL + 2 * w + 1], Y0 = p1[O_PL + 2 * w + 3];
+                    if (rfix) X12.x = p1[O_PR + 2 * w], Y12.x = p1[O_PR + 2 * w + 2];
+                }
+                if (xr >= 0) {
+                    const double* q1 = p1 + xr * WPW + xc + 1;
+                    E0 = q1[0], E1 = q1[1], E2 = q1[WPW], E3 = q1[WPW + 1];
+                    if (first && xc == 0) E0 = p1[O_PL + 2 * xr + 1], E2 = p1[O_PL + 2 * xr + 3];
+                    if (last && xc == width) E1 = p1[O_PR + 2 * xr], E3 = p1[O_PR + 2 * xr + 2];
+                }
+                if (n == 0) {  // stage ia-1: p plane ia-1 only
+                    x0 = X0, y0 = Y0, x12 = X12, y12 = Y12, e0 = E0, e1 = E1, e2 = E2, e3 = E3;
+                    continue;
+                }
+                // ---- corners of plane I: p(I-1) rows w, w+1 (cell rows J-1, J)
+                // from registers, p(I) from the stage
                 double* Cf = C_of(slot);
                 if (crow_ok) {
-                    const double* q0 = p0 + w * WPW + c2;
-                    const double* q1 = p1 + w * WPW + c2;
-                    double x0 = q0[1], y0 = q0[WPW + 1], X0 = q1[1], Y0 = q1[WPW + 1];
-                    double2 x12 = lds2(q0 + 2), y12 = lds2(q0 + WPW + 2);
-                    double2 X12 = lds2(q1 + 2), Y12 = lds2(q1 + WPW + 2);
                     double* c0 = Cf + w * WCW + c2;
-                    double2 A0 = lds2(c0), B0 = lds2(c0 + WCA), E0 = lds2(c0 + 2 * WCA);
-                    if (lfix) {  // cell column k0-1 = np-1: the left phi-wrap box
-                        const double *L0 = p0 + O_PL, *L1 = p1 + O_PL;
-                        x0 = L0[2 * w + 1], y0 = L0[2 * w + 3], X0 = L1[2 * w + 1], Y0 = L1[2 * w + 3];
-                    }
-                    if (rfix) {  // cell column k0+width = 0 and corner column width: the right boxes
-                        const double *R0 = p0 + O_PR, *R1 = p1 + O_PR, *CS = p1 + O_CS;
-                        x12.x = R0[2 * w], y12.x = R0[2 * w + 2], X12.x = R1[2 * w], Y12.x = R1[2 * w + 2];
-                        A0.x = CS[2 * w], B0.x = CS[2 * (WCR + w)], E0.x = CS[2 * (2 * WCR + w)];
+                    double2 A0 = lds2(c0), B0 = lds2(c0 + WCA), C0 = lds2(c0 + 2 * WCA);
+                    if (rfix) {  // corner column width = k0 + width: the right box
+                        const double* CS = p1 + O_CS;
+                        A0.x = CS[2 * w], B0.x = CS[2 * (WCR + w)], C0.x = CS[2 * (2 * WCR + w)];
                     }
                     double o[2][4];
                     const double s0 = corner_math(x0, x12.x, y0, y12.x, X0, X12.x, Y0, Y12.x, A0.x, B0.x,
-                                                  E0.x, o[0][0], o[0][1], o[0][2], o[0][3]);
+                                                  C0.x, o[0][0], o[0][1], o[0][2], o[0][3]);
                     const double s1 = corner_math(x12.x, x12.y, y12.x, y12.y, X12.x, X12.y, Y12.x, Y12.y,
-                                                  A0.y, B0.y, E0.y, o[1][0], o[1][1], o[1][2], o[1][3]);
+                                                  A0.y, B0.y, C0.y, o[1][0], o[1][1], o[1][2], o[1][3]);
 #pragma unroll
                     for (int q = 0; q < 4; q++) sts2(c0 + q * WCA, make_double2(o[0][q], o[1][q]));
                     // sigma: this tile's corners (row < height, col < width) of the
@@ -386,28 +398,20 @@ __global__ void __launch_bounds__(WTHREADS, 1) k_aniso(const AnisoArgs a, const 
                         acc[0] += s0 * s0 + s1 * s1;
                 }
                 if (xr >= 0) {  // row 16 / column 64: counted by the neighbouring tile
-                    const double* q0 = p0 + xr * WPW + xc + 1;
-                    const double* q1 = p1 + xr * WPW + xc + 1;
                     double* c0 = Cf + xr * WCW + xc;
-                    double a00 = q0[0], a01 = q0[1], a10 = q0[WPW], a11 = q0[WPW + 1];
-                    double b00 = q1[0], b01 = q1[1], b10 = q1[WPW], b11 = q1[WPW + 1];
                     double A = c0[0], B = c0[WCA], E = c0[2 * WCA];
-                    if (first && xc == 0) {
-                        const double *L0 = p0 + O_PL, *L1 = p1 + O_PL;
-                        a00 = L0[2 * xr + 1], a10 = L0[2 * xr + 3], b00 = L1[2 * xr + 1], b10 = L1[2 * xr + 3];
-                    }
                     if (last && xc == width) {
-                        const double *R0 = p0 + O_PR, *R1 = p1 + O_PR, *CS = p1 + O_CS;
-                        a01 = R0[2 * xr], a11 = R0[2 * xr + 2], b01 = R1[2 * xr], b11 = R1[2 * xr + 2];
+                        const double* CS = p1 + O_CS;
                         A = CS[2 * xr], B = CS[2 * (WCR + xr)], E = CS[2 * (2 * WCR + xr)];
                     }
                     double o0, o1, o2, o3;
-                    corner_math(a00, a01, a10, a11, b00, b01, b10, b11, A, B, E, o0, o1, o2, o3);
+                    corner_math(e0, e1, e2, e3, E0, E1, E2, E3, A, B, E, o0, o1, o2, o3);
                     c0[0] = o0;
                     c0[WCA] = o1;
                     c0[2 * WCA] = o2;
                     c0[3 * WCA] = o3;
                 }
+                x0 = X0, y0 = Y0, x12 = X12, y12 = Y12, e0 = E0, e1 = E1, e2 = E2, e3 = E3;
                 consumer_sync();
                 // ---- cells (w, c2..c2+1) of plane i = I-1: corner planes i
                 // (sr = +1) and I (sr = -1); out/q plane i from this stage
