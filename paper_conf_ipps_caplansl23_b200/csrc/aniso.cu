@@ -17,10 +17,10 @@
 // a producer warp streams stages {p plane I with its phi halo, the 3
 // corner-coefficient fields of corner plane I, out plane I-1} into a 4-slot
 // shared ring with tensor copies (TMA, cuTensorMapEncodeTiled maps, one box
-// per field; rows beyond a pole and planes outside the slab arrive as zeros)
-// (the periodic phi-wrap cells come as 2-wide side boxes); 16 consumer warps (one per tile
-// row) compute the corner products and gather them into the cells.  Full /
-// empty mbarriers order the two sides.  Bytes per cell (PCGA):
+// per field; rows beyond a pole and planes outside the slab arrive as zeros;
+// the periodic phi-wrap cells come as 2-wide side boxes); 16 consumer warps
+// (one per tile row) compute the corner products and gather them into the
+// cells.  Full / empty mbarriers order the two sides.  Bytes per cell (PCGA):
 // p 8 + (a, b, e) 24 + q read/write 16 = 48 B.
 #include <cuda.h>
 #include <cuda_runtime.h>
@@ -123,9 +123,10 @@ __device__ __forceinline__ double2 ld2(const double* p) { return __ldg(reinterpr
 
 // ---- warp-specialised pipeline ---------------------------------------------
 // One block per SM: 16 consumer warps (warp w = tile row w, lane l = the
-// column pair 2l, 2l+1) and one producer warp that streams the stages with
-// bulk copies (cp.async.bulk, the TMA engine) into a 4-slot ring, signalled by
-// mbarriers (full: bytes landed; empty: the 16 consumer warps are done).
+// column pair 2l, 2l+1) and one producer warp whose lane 0 streams the stages
+// with tensor copies (cp.async.bulk.tensor, the TMA engine) into a 4-slot
+// ring, signalled by mbarriers (full: the box bytes landed; empty: the 16
+// consumer warps are done with the slot).
 namespace {
 constexpr int WJ = 16;                 // tile rows (one consumer warp each)
 constexpr int WK = 64;                 // tile columns (32 lanes x 2)
