@@ -214,6 +214,14 @@ class Oracle:
                                                  _p(bhat_ext), _p(x_ext), _p(y)))
         return y
 
+    def radial_sums(self, x, w):
+        """sum0[m][i] = sum_{j,k} w[j][k] x[m][i][j][k] (Listings 3-5, R27)."""
+        x, w = _f64(x), _f64(w)
+        ncomp = x.size // self.N
+        out = np.empty((ncomp, self.shape[0]))
+        self._chk(lib().mas_ref_radial_sums(C.byref(self.g), ncomp, _p(x), _p(w), _p(out)))
+        return out
+
     def pcg_aniso(self, kappa, c, kpar, bhat, f, x0, tol, maxit):
         """PCG on L_iso + L_par.  Returns (status, x, iters, relres, res_hist)."""
         f = _f64(f)

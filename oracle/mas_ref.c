@@ -951,3 +951,30 @@ int mas_ref_aniso_apply_slab(const mas_ref_grid* g, int i0, int nl, int ncomp,
     tables_free(&T);
     return MAS_REF_OK;
 }
+
+/* ---------------------------------------------------------------------------
+ * Per-radius array reductions, the paper's Listings 3-5 (P:428-445,
+ * P:592-645, §IV): "sum0(i)=sum0(i)+array(i,j)*..." over the angular index,
+ * one sum per radius i.  MAS uses them e.g. for the phi-averaged values of
+ * node-in-theta variables at the poles.  Reading R27:
+ * the elided factor "..." is a caller-supplied angular weight w[j][k], so
+ *   sum0[m][i] = sum_{j,k} w[j][k] x[m][i][j][k]     (summed in (j,k) order).
+ * ------------------------------------------------------------------------- */
+int mas_ref_radial_sums(const mas_ref_grid* g, int ncomp, const double* x, const double* w,
+                        double* out) {
+    size_t plane, N;
+    int m, i;
+    if (!g || !x || !w || !out || ncomp < 1 || g->nr < 1 || g->nt < 1 || g->np < 1)
+        return MAS_REF_ERR_ARG;
+    plane = (size_t)g->nt * g->np;
+    N = plane * g->nr;
+    for (m = 0; m < ncomp; m++)
+        for (i = 0; i < g->nr; i++) {
+            const double* xp = x + (size_t)m * N + (size_t)i * plane;
+            double s = 0.0;
+            size_t e;
+            for (e = 0; e < plane; e++) s += w[e] * xp[e];
+            out[(size_t)m * g->nr + i] = s;
+        }
+    return MAS_REF_OK;
+}

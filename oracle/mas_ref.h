@@ -137,6 +137,11 @@ int mas_ref_pcg_solve_aniso(const mas_ref_grid* g, int ncomp, const double* kapp
                             const double* f, double* x, double tol, int maxit, int* iters,
                             double* relres, double* res_hist);
 
+/* Per-radius array reduction (the paper's Listings 3-5, "sum0"; reading R27):
+ * out[m][i] = sum_{j,k} w[j][k] x[m][i][j][k], w [nt][np], out [ncomp][nr]. */
+int mas_ref_radial_sums(const mas_ref_grid* g, int ncomp, const double* x, const double* w,
+                        double* out);
+
 #ifdef __cplusplus
 }
 #endif
