@@ -254,6 +254,21 @@ MAS_API mas_status_t mas_op_set_aniso(mas_op_t* op, const double* kpar, const do
  * (mas_op_set_profiling); 0 when the term is off. */
 MAS_API mas_status_t mas_op_aniso_time(const mas_op_t* op, double* ms);
 
+/* Per-radius array reduction, the paper's Listings 3-5 ("sum0(i) =
+ * sum0(i) + array(i,j)*...", §IV; MAS uses such sums
+ * e.g. for phi-averaged pole values).  Reading R27:
+ * the elided factor is an angular weight, so
+ *   out[m][i] = sum_{j,k} w[j][k] x[m][i][j][k]
+ * for every component m and LOCAL r-plane i of this rank.  x [ncomp][nl][nt][np],
+ * w [nt][np] (16-byte aligned), out [ncomp][nl]; each may be a host or a
+ * device pointer (a host out makes the call synchronous).  Deterministic:
+ * one fixed-order block reduction per plane, no atomics (the paper's DC
+ * rewrite replaced the OpenACC atomics by a reduce).  Local to each rank (no
+ * communication: r-slab ranks own whole planes).
+ * Errors: MAS_ERR_ARG on a null pointer or a grid with ptheta > 1. */
+MAS_API mas_status_t mas_op_radial_sums(const mas_op_t* op, const double* x, const double* w,
+                                        double* out, cudaStream_t stream);
+
 MAS_API mas_status_t mas_op_destroy(mas_op_t* op);
 
 MAS_API const char* mas_status_string(mas_status_t s);

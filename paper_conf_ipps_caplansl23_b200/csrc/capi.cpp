@@ -147,6 +147,9 @@ struct mas_op {
     double* ca = nullptr;                        // corner coefficients [3][nl][nt][np]
     double* cag = nullptr;                       // r-slabs: their ghost planes [2][3][plane]
     double* pkg = nullptr;                       // r-slabs: p_k ghost planes [2][plane]
+    // per-radius sums (mas_op_radial_sums): weights and results, device
+    double* rs_w = nullptr;
+    double* rs_out = nullptr;
     double* atab = nullptr;                      // AnisoTab arrays (device)
     AnisoTab at{};
 };
@@ -442,7 +445,7 @@ static mas_status_t op_load(mas_op* op, const double* kappa, const double* mass,
 static void op_free(mas_op* op) {
     if (!op) return;
     for (double* p : {op->kgt, op->dgt, op->xgt, op->rgt, op->pgt[0], op->pgt[1], op->tpack, op->ca,
-                      op->atab, op->cag, op->pkg})
+                      op->atab, op->cag, op->pkg, op->rs_w, op->rs_out})
         if (p) cudaFree(p);
     for (double* p : {op->kappa, op->c, op->dinv, op->kg, op->dg, op->wR, op->r, op->p[0], op->p[1],
                       op->q, op->rg, op->pg[0], op->pg[1], op->xg, op->stage_a, op->stage_b,
@@ -817,6 +820,39 @@ mas_status_t mas_op_dot(const mas_op_t* op_c, const double* a, const double* b, 
     if (op->g->comm) ST(comm_allreduce(op->g->comm, op->dot_out, 1, stream));
     CU(cudaMemcpyAsync(out, op->dot_out, sizeof(double), cudaMemcpyDeviceToHost, stream));
     CU(cudaStreamSynchronize(stream));
+    return MAS_OK;
+}
+
+mas_status_t mas_op_radial_sums(const mas_op_t* op_c, const double* x, const double* w, double* out,
+                                cudaStream_t stream) {
+    mas_op* op = const_cast<mas_op*>(op_c);
+    if (!op || !x || !w || !out) return arg_error("null argument");
+    if (op->g->ptheta > 1) return arg_error("radial sums: r-slab decompositions only (ptheta == 1)");
+    const size_t plane = (size_t)op->geo.plane;
+    const size_t nout = (size_t)op->ncomp * op->g->nl;
+    const double *xd = x, *wd = w;
+    if (!is_device_ptr(x)) {
+        ST(ensure_stage(op));
+        CU(cudaMemcpyAsync(op->stage_a, x, op->ncomp * op->Nl * sizeof(double), cudaMemcpyHostToDevice,
+                           stream));
+        xd = op->stage_a;
+    }
+    if (!is_device_ptr(w)) {
+        if (!op->rs_w) ST(dmalloc(&op->rs_w, plane));
+        CU(cudaMemcpyAsync(op->rs_w, w, plane * sizeof(double), cudaMemcpyHostToDevice, stream));
+        wd = op->rs_w;
+    }
+    const bool hout = !is_device_ptr(out);
+    double* od = out;
+    if (hout) {
+        if (!op->rs_out) ST(dmalloc(&op->rs_out, nout));
+        od = op->rs_out;
+    }
+    CU(launch_radial_sums(op->geo, op->ncomp, xd, wd, od, stream));
+    if (hout) {
+        CU(cudaMemcpyAsync(out, od, nout * sizeof(double), cudaMemcpyDeviceToHost, stream));
+        CU(cudaStreamSynchronize(stream));
+    }
     return MAS_OK;
 }
 

@@ -1054,9 +1054,45 @@ __global__ void __launch_bounds__(kThreads) k_dot(const Geo g, int ncomp, const 
     if (grid_reduce<1>(acc, scr, TKT_DOT) && threadIdx.x == 0) *out = acc[0];
 }
 
+// Per-radius array reduction, the paper's Listings 3-5 (P:428-445,
+// P:592-645): sum0(i) = sum_j array(i,j) * w(j), here with the angular index
+// (j,k) and a caller-supplied weight (reading R27).  MAS's OpenACC version
+// uses atomic updates; the paper's DC rewrite reduces each i in an inner
+// loop.  On the GPU: one block per (component, r-plane), double2 loads, a
+// fixed-order block tree (deterministic, no atomics).
+__global__ void __launch_bounds__(kThreads) k_radial_sums(const Geo g, const double* x, const double* w,
+                                                          double* out) {
+    __shared__ double ws[kThreads / 32];
+    const int b = blockIdx.x;  // m * nl + i
+    const long long plane = g.plane;
+    const double* xp = x + (long long)b * plane;
+    double s = 0.0;
+    for (long long e = 2 * threadIdx.x; e < plane; e += 2 * kThreads) {
+        const double2 xv = ld2(xp + e), wv = ld2(w + e);
+        s = fma(wv.x, xv.x, s);
+        s = fma(wv.y, xv.y, s);
+    }
+    s = warp_sum(s);
+    if ((threadIdx.x & 31) == 0) ws[threadIdx.x >> 5] = s;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        double t = 0.0;
+        for (int q = 0; q < kThreads / 32; q++) t += ws[q];
+        out[b] = t;
+    }
+}
+
 // --------------------------------------------------------------------------
 // launchers
 // --------------------------------------------------------------------------
+cudaError_t launch_radial_sums(const Geo& g, int ncomp, const double* x, const double* w, double* out,
+                               cudaStream_t s) {
+    const int blocks = ncomp * g.nl;
+    if (blocks <= 0) return cudaErrorInvalidValue;
+    k_radial_sums<<<blocks, kThreads, 0, s>>>(g, x, w, out);
+    return cudaGetLastError();
+}
+
 int stencil_blocks(const Geo& g, int chunk) {
     const int ntj = (g.nt + TJ - 1) / TJ, ntk = (g.np + TK - 1) / TK;
     const int nch = (g.nl + chunk - 1) / chunk;

@@ -203,6 +203,9 @@ cudaError_t launch_dot(const Geo& g, int ncomp, const double* a, const double* b
 // out[t] = sum_r stage[8r + t], t < n, ranks summed in rank order (virtual-rank allreduce)
 cudaError_t launch_rank_sum(double* out, const double* stage, int nranks, int n, cudaStream_t s);
 
+// out[m * nl + i] = sum_{j,k} w[j][k] x[m][i][j][k] (the paper's sum0, Listings 3-5)
+cudaError_t launch_radial_sums(const Geo& g, int ncomp, const double* x, const double* w, double* out,
+                               cudaStream_t s);
 // launchers (aniso.cu)
 cudaError_t launch_aniso(int mode, const AnisoArgs& a, cudaStream_t s);
 // ca from kpar [nl][nt][np] and bhat [3][nl][nt][np]; *bad |= 1 on a negative

@@ -28,7 +28,7 @@ ABI_SYMBOLS = ("mas_comm_unique_id", "mas_partition", "mas_grid_create", "mas_gr
                "mas_op_transport", "mas_op_launch_count", "mas_grid_create_2d",
                "mas_grid_local_extent_2d",
                "mas_op_set_profiling", "mas_op_kernel_times", "mas_op_set_aniso",
-               "mas_op_aniso_time", "mas_op_destroy", "mas_status_string", "mas_last_error", "mas_version")
+               "mas_op_aniso_time", "mas_op_radial_sums", "mas_op_destroy", "mas_status_string", "mas_last_error", "mas_version")
 
 
 class MasError(RuntimeError):
@@ -76,6 +76,7 @@ def lib() -> C.CDLL:
             "mas_op_kernel_times": (_i, [_vp, _vp, _vp, _vp]),
             "mas_op_set_aniso": (_i, [_vp, _vp, _vp, _vp]),
             "mas_op_aniso_time": (_i, [_vp, _vp]),
+            "mas_op_radial_sums": (_i, [_vp, _vp, _vp, _vp, _vp]),
             "mas_op_destroy": (_i, [_vp]),
             "mas_status_string": (C.c_char_p, [_i]),
             "mas_last_error": (C.c_char_p, []),
@@ -280,6 +281,12 @@ def mas_op_aniso_time(op: int) -> float:
     return ms.value
 
 
+def mas_op_radial_sums(op: int, x, w, out, stream=None) -> None:
+    """out[m][i] = sum_{j,k} w[j][k] x[m][i][j][k] (the paper's sum0)."""
+    _check(lib().mas_op_radial_sums(op, _ptr(x), _ptr(w), _ptr(out), _stream(stream)),
+           "mas_op_radial_sums")
+
+
 def mas_op_destroy(op: int) -> None:
     _check(lib().mas_op_destroy(op), "mas_op_destroy")
 
@@ -358,6 +365,9 @@ class Operator:
 
     def aniso_time(self):
         return mas_op_aniso_time(self.h)
+
+    def radial_sums(self, x, w, out, stream=None):
+        mas_op_radial_sums(self.h, x, w, out, stream)
 
     @property
     def launch_count(self):
