@@ -1066,12 +1066,28 @@ __global__ void __launch_bounds__(kThreads) k_radial_sums(const Geo g, const dou
     const int b = blockIdx.x;  // m * nl + i
     const long long plane = g.plane;
     const double* xp = x + (long long)b * plane;
-    double s = 0.0;
-    for (long long e = 2 * threadIdx.x; e < plane; e += 2 * kThreads) {
-        const double2 xv = ld2(xp + e), wv = ld2(w + e);
-        s = fma(wv.x, xv.x, s);
-        s = fma(wv.y, xv.y, s);
+    // four independent pairs in flight per thread, summed in a fixed order
+    double s4[4] = {0.0, 0.0, 0.0, 0.0};
+    long long e = 2 * threadIdx.x;
+    for (; e + 6 * kThreads < plane; e += 8 * kThreads) {
+        double2 xv[4], wv[4];
+#pragma unroll
+        for (int u = 0; u < 4; u++) {
+            xv[u] = ld2(xp + e + 2 * u * kThreads);
+            wv[u] = ld2(w + e + 2 * u * kThreads);
+        }
+#pragma unroll
+        for (int u = 0; u < 4; u++) {
+            s4[u] = fma(wv[u].x, xv[u].x, s4[u]);
+            s4[u] = fma(wv[u].y, xv[u].y, s4[u]);
+        }
     }
+    for (; e < plane; e += 2 * kThreads) {
+        const double2 xv = ld2(xp + e), wv = ld2(w + e);
+        s4[0] = fma(wv.x, xv.x, s4[0]);
+        s4[0] = fma(wv.y, xv.y, s4[0]);
+    }
+    double s = (s4[0] + s4[1]) + (s4[2] + s4[3]);
     s = warp_sum(s);
     if ((threadIdx.x & 31) == 0) ws[threadIdx.x >> 5] = s;
     __syncthreads();
