@@ -207,3 +207,24 @@ def test_graph_loop_equals_host_loop_bitwise(mp, oracle_mod):
     assert a[1] == b[1]
     assert np.array_equal(a[2], b[2])
     assert b[8].aniso_time() > 0.0
+
+
+@pytest.mark.parametrize("shape", [(1, 8, 16), (6, 1, 16), (5, 6, 2), (3, 2, 130)])
+def test_degenerate_grids(mp, oracle_mod, shape):
+    """One r-plane or one theta row: every corner is on the boundary, L_par = 0;
+    np = 2: the phi-wrap boxes cover the whole row; a 2-row theta band with a
+    ragged phi tile.  Apply and diagonal against the oracle."""
+    mesh = W.stretched_mesh(*shape)
+    kappa, c, kpar, b = rand_fields(shape, 21)
+    g, op = setup(mp, mesh, kappa, c, kpar, b)
+    x = W.random_field((1,) + shape, 22)
+    y = torch.empty((1,) + shape, dtype=torch.float64, device="cuda")
+    op.apply(dev(x), y)
+    o = oracle_mod.Oracle(mesh, 0, 1)
+    yo = o.apply(kappa, c, x) + o.aniso_apply(kpar, b, x)
+    assert rel_l2_V(o.volumes(), host(y), yo) <= 1e-13
+    if shape[0] == 1 or shape[1] == 1:
+        assert np.array_equal(o.aniso_apply(kpar, b, x), np.zeros_like(x))
+    D = torch.empty(shape, dtype=torch.float64, device="cuda")
+    op.diag(D)
+    np.testing.assert_allclose(host(D), o.diag(kappa, c) + o.aniso_diag(kpar, b), rtol=1e-13, atol=0)
