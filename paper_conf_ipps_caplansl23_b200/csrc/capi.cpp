@@ -1041,7 +1041,16 @@ mas_status_t mas_op_set_aniso(mas_op_t* op, const double* kpar, const double* bh
     }
     // host inputs are staged through a temporary device buffer
     const double *kd = kpar, *bd = bhat;
-    double* tmp = nullptr;
+    // host inputs: a temporary device copy, freed on every return path
+    // (cudaFree waits for the device, so the pending copies and the
+    // coefficient kernel have consumed it)
+    struct DevTmp {
+        double* p = nullptr;
+        ~DevTmp() {
+            if (p) cudaFree(p);
+        }
+    } tmp_guard;
+    double*& tmp = tmp_guard.p;
     const bool hk = !is_device_ptr(kpar), hb = !is_device_ptr(bhat);
     if (hk || hb) {
         ST(dmalloc(&tmp, 4 * (size_t)N));
@@ -1062,13 +1071,19 @@ mas_status_t mas_op_set_aniso(mas_op_t* op, const double* kpar, const double* bh
         ST(comm_seams(comm, op->ca, 3, op->g->nl, plane, op->cag, op->cag + 3 * plane, stream,
                       rstride(op)));
     op->aniso = 1;
+    struct AnisoOff {  // an error return below leaves the term off
+        mas_op* op;
+        bool keep = false;
+        ~AnisoOff() {
+            if (!keep) op->aniso = 0;
+        }
+    } on_error{op};
     ST(op_diag(op, nullptr, stream));
     if (comm)
         ST(comm_seams(comm, op->dinv, 1, op->g->nl, plane, op->dg, op->dg + plane, stream, rstride(op)));
     int bad = 0;
     CU(cudaMemcpyAsync(&bad, op->bad, sizeof(int), cudaMemcpyDeviceToHost, stream));
     CU(cudaStreamSynchronize(stream));
-    if (tmp) cudaFree(tmp);
     if (comm) {  // agree on the verdict across ranks
         double* d = op->dot_out;
         double hb = bad;
@@ -1084,6 +1099,7 @@ mas_status_t mas_op_set_aniso(mas_op_t* op, const double* kpar, const double* bh
         if (comm) comm_seams(comm, op->dinv, 1, op->g->nl, plane, op->dg, op->dg + plane, stream, rstride(op));
         return arg_error("kpar negative or non-finite, b non-finite, or Jacobi diagonal D <= 0");
     }
+    on_error.keep = true;
     return MAS_OK;
 }
 
