@@ -343,6 +343,9 @@ __device__ __forceinline__ void trow_issue(const StencilArgs& a, int i, const Ha
 #define MAS_PF_DIST 3
 #endif
 constexpr int kPfDist = MAS_PF_DIST;  // planes ahead of the stencil plane
+#ifndef MAS_PF_SCALAR
+#define MAS_PF_SCALAR 0  // the scalar kernel measured slower with the prefetch (r1e)
+#endif
 // evict_last policy on the prefetched lines (A/B: kernel B -2%, kernel A equal)
 __device__ __forceinline__ void l2_prefetch_row(const double* p, int bytes) {
 #ifndef MAS_PF_NORMAL
@@ -688,7 +691,7 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
 
 #ifndef MAS_NO_PREFETCH
     // the planes the march reaches before its first in-loop prefetch
-    if (NC == 3)
+    if (NC == 3 || MAS_PF_SCALAR)
         for (int ip = ia + 1; ip < min(ia + kPfDist, ib); ip++)
             plane_prefetch<MODE, NC>(a, ip, j0, k0, height, width, FIRSTK, xupd);
 #endif
@@ -733,7 +736,7 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
 #ifndef MAS_NO_PREFETCH
         // 3-component kernels only: for the scalar kernel (C2: 256 work items,
         // under one wave) it measured slower (tools/abtest.sh)
-        if (NC == 3 && i + kPfDist < ib)
+        if ((NC == 3 || MAS_PF_SCALAR) && i + kPfDist < ib)
             plane_prefetch<MODE, NC>(a, i + kPfDist, j0, k0, height, width, FIRSTK, xupd);
 #endif
         if (!kIssueEarly && i + 2 <= ib && real_plane(i + 2))
