@@ -150,6 +150,7 @@ struct mas_op {
     // per-radius sums (mas_op_radial_sums): weights and results, device
     double* rs_w = nullptr;
     double* rs_out = nullptr;
+    double* astage = nullptr;                    // host kpar / b staging [4][nl][nt][np]
     double* atab = nullptr;                      // AnisoTab arrays (device)
     AnisoTab at{};
 };
@@ -445,7 +446,7 @@ static mas_status_t op_load(mas_op* op, const double* kappa, const double* mass,
 static void op_free(mas_op* op) {
     if (!op) return;
     for (double* p : {op->kgt, op->dgt, op->xgt, op->rgt, op->pgt[0], op->pgt[1], op->tpack, op->ca,
-                      op->atab, op->cag, op->pkg, op->rs_w, op->rs_out})
+                      op->atab, op->cag, op->pkg, op->rs_w, op->rs_out, op->astage})
         if (p) cudaFree(p);
     for (double* p : {op->kappa, op->c, op->dinv, op->kg, op->dg, op->wR, op->r, op->p[0], op->p[1],
                       op->q, op->rg, op->pg[0], op->pg[1], op->xg, op->stage_a, op->stage_b,
@@ -1041,19 +1042,13 @@ mas_status_t mas_op_set_aniso(mas_op_t* op, const double* kpar, const double* bh
     }
     // host inputs are staged through a temporary device buffer
     const double *kd = kpar, *bd = bhat;
-    // host inputs: a temporary device copy, freed on every return path
-    // (cudaFree waits for the device, so the pending copies and the
-    // coefficient kernel have consumed it)
-    struct DevTmp {
-        double* p = nullptr;
-        ~DevTmp() {
-            if (p) cudaFree(p);
-        }
-    } tmp_guard;
-    double*& tmp = tmp_guard.p;
+    // host inputs are staged through a library-owned device buffer (kept for
+    // the next call: a time-stepping caller refreshes kpar and b every step)
     const bool hk = !is_device_ptr(kpar), hb = !is_device_ptr(bhat);
+    double* tmp = nullptr;
     if (hk || hb) {
-        ST(dmalloc(&tmp, 4 * (size_t)N));
+        if (!op->astage) ST(dmalloc(&op->astage, 4 * (size_t)N));
+        tmp = op->astage;
         if (hk) {
             CU(cudaMemcpyAsync(tmp, kpar, N * sizeof(double), cudaMemcpyHostToDevice, stream));
             kd = tmp;
