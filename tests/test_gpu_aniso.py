@@ -228,3 +228,28 @@ def test_degenerate_grids(mp, oracle_mod, shape):
     D = torch.empty(shape, dtype=torch.float64, device="cuda")
     op.diag(D)
     np.testing.assert_allclose(host(D), o.diag(kappa, c) + o.aniso_diag(kpar, b), rtol=1e-13, atol=0)
+
+
+def test_p2p_transport_and_aniso_are_exclusive(mp):
+    """The P2P mailbox carries kernel A's sigma only: with the field-aligned
+    term on, mas_op_enable_p2p refuses, and mas_op_set_aniso refuses on a P2P
+    op (one GPU: the mailbox runs against itself)."""
+    shape = (8, 16, 64)
+    mesh = W.stretched_mesh(*shape)
+    kappa, c, kpar, b = rand_fields(shape, 31)
+    g, op = setup(mp, mesh, kappa, c, kpar, b)
+    with pytest.raises(mp.MasError) as e:
+        op.enable_p2p()
+    assert e.value.status == mp.MAS_ERR_ARG
+    g2 = mp.Grid(mesh)
+    op2 = mp.Operator(g2, 1, dev(kappa), dev(c), 0, 1)
+    op2.enable_p2p()
+    with pytest.raises(mp.MasError) as e:
+        op2.set_aniso(dev(kpar), dev(b))
+    assert e.value.status == mp.MAS_ERR_ARG
+    # both ops still solve correctly afterwards
+    f = dev(W.random_field((1,) + shape, 32))
+    for o_ in (op, op2):
+        x = torch.zeros_like(f)
+        st, it, rel, _ = o_.solve(f, x, 1e-10, 2000)
+        assert st == mp.MAS_OK and rel <= 1e-10
