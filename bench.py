@@ -294,16 +294,14 @@ def main():
     x = x0.clone()
     op = M.Operator(grid, nc, kappa, cmass, prob.bc_inner, prob.bc_outer)
     aniso = prob.kpar is not None
-    if aniso:  # NEXT-4; on r-slabs it runs the NCCL loop (no P2P mailbox for its sigma)
+    if aniso:  # NEXT-4 (r-slabs; either transport)
         if args.ptheta != 1:
             raise SystemExit("C2a (field-aligned conduction) needs r-slabs (--ptheta 1)")
         kpar = to_dev(prob.kpar[sl])
         bhat = to_dev(prob.bhat[(slice(None),) + sl])
         op.set_aniso(kpar, bhat)
     transport = "single-gpu"
-    if world > 1 and aniso:
-        transport = "nccl"
-    elif world > 1:
+    if world > 1:
         transport = "nccl"
         if args.transport != "nccl":
             try:

@@ -241,12 +241,12 @@ MAS_API mas_status_t mas_op_kernel_times(const mas_op_t* op, double* a_ms, doubl
  * iteration).  kpar == NULL switches the term off.  Synchronises the stream.
  * On an r-slab grid (mas_grid_create with a mas_dist_t) the call is
  * collective: each rank passes its local slab of kpar / bhat; the corner
- * plane above the slab comes from rank+1 and the p_k planes of the
- * neighbours are exchanged after every kernel A (NCCL loop).
- * Errors: MAS_ERR_ARG if ncomp != 1, the grid has ptheta > 1, the P2P
- * transport is on (mas_op_enable_p2p then also refuses while the term is on),
- * kpar < 0 or non-finite, b non-finite, or some D_P <= 0 (the term is then
- * off). */
+ * plane above the slab comes from rank+1.  The p_k planes of the neighbours
+ * are exchanged after every kernel A (NCCL loop) or read in place once every
+ * rank's kernel A has published (P2P transport; the term's sigma part goes
+ * through its own mailbox slot).
+ * Errors: MAS_ERR_ARG if ncomp != 1, the grid has ptheta > 1, kpar < 0 or
+ * non-finite, b non-finite, or some D_P <= 0 (the term is then off). */
 MAS_API mas_status_t mas_op_set_aniso(mas_op_t* op, const double* kpar, const double* bhat,
                                       cudaStream_t stream);
 

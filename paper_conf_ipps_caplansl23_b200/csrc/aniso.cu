@@ -224,6 +224,18 @@ __global__ void __launch_bounds__(WTHREADS, 1) k_aniso(const AnisoArgs a, const 
             cudaGraphSetConditional((cudaGraphConditionalHandle)a.cond, 0);
         return;
     }
+    const bool p2p = a.p2p.nranks > 0;
+    int kit = 0;
+    if (MODE == MODE_PCGA && p2p) {
+        // P2P: the r-neighbours' p_k edge planes are read in place; wait until
+        // every rank's kernel A(k) has published (its p_k is then complete)
+        kit = __ldcg(&a.st->k);
+        if (threadIdx.x == 0) {
+            double v[1];
+            p2p_gather_one<1>(a.p2p, MB_A, p2p_seq(__ldcg(&a.st->epoch), kit), v);
+        }
+        __syncthreads();
+    }
     const Geo& g = a.g;
     const int plane = (int)g.plane;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -459,13 +471,21 @@ __global__ void __launch_bounds__(WTHREADS, 1) k_aniso(const AnisoArgs a, const 
 
     if (MODE == MODE_PCGA) {
         double v[1] = {acc[0]};
-        if (grid_reduce<1, WTHREADS>(v, a.scr, TKT_ANISO) && threadIdx.x == 0)
-            a.st->pend_sigma = a.st->pend_sigma + v[0];  // <p,L_iso p> (kernel A) + <p,L_par p>
+        if (grid_reduce<1, WTHREADS>(v, a.scr, TKT_ANISO, p2p) && threadIdx.x == 0) {
+            if (p2p)  // kernel B(k) sums every rank's part from MB_C
+                p2p_publish(a.p2p, MB_C, p2p_seq(a.st->epoch, kit), v, 1);
+            else
+                a.st->pend_sigma = a.st->pend_sigma + v[0];  // <p,L_iso p> (kernel A) + <p,L_par p>
+        }
     } else if (MODE == MODE_RESID) {
-        if (grid_reduce<3, WTHREADS>(acc, a.scr, TKT_ANISO) && threadIdx.x == 0) {
+        if (grid_reduce<3, WTHREADS>(acc, a.scr, TKT_ANISO, p2p) && threadIdx.x == 0) {
             a.st->pend_ff = acc[0];
             a.st->pend_rr = acc[1];
             a.st->pend_rho = acc[2];
+            if (p2p) {  // the init sums (kernel A(1) reads them from MB_B)
+                const double pub[3] = {acc[2], acc[1], acc[0]};  // {rho, rr, ff}
+                p2p_publish(a.p2p, MB_B, p2p_seq(a.st->epoch, 0), pub, 3);
+            }
         }
     }
 }

@@ -374,6 +374,16 @@ static P2P p2p_args(const mas_op* op) {
     return t;
 }
 
+// p_k (= p[k & 1]) with its r-neighbour planes as the L_par kernel reads them:
+// in place from the neighbours' arrays (P2P), from the p_k seam buffers (NCCL
+// loop, exchanged after kernel A), or none (one GPU)
+static Halo aniso_p_halo(const mas_op* op, int k) {
+    const int par = k & 1;
+    if (op->p2p) return peer_halo(op, op->p[par], op->nb_p[par][0], op->nb_p[par][1]);
+    if (op->g->comm) return halo_of(op, op->p[par], op->pkg, 1);
+    return Halo{op->p[par], nullptr, nullptr, 0, 0};
+}
+
 // r-slabs: the corner plane above the slab is rank+1's plane 0 (ghost copy)
 static const double* aniso_ca_hi(const mas_op* op) {
     return (op->cag && !op->geo.glob_hi) ? op->cag + 3 * op->geo.plane : nullptr;
@@ -397,6 +407,7 @@ static AnisoArgs aniso_args(const mas_op* op, int mode, Halo u, double* out) {
     a.max_blocks = op->max_blocks;
     a.ca = op->ca;
     a.ca_hi = aniso_ca_hi(op);
+    a.p2p = p2p_args(op);
     a.ivr = op->at.ivr;
     a.u = u;
     a.out = out;
@@ -527,7 +538,7 @@ static mas_status_t loop_graph(mas_op* op, StencilArgs a, StreamArgs b, AnisoArg
                 a.tpold = pold_trows(op, kk);
                 a.pnew = op->p[kk & 1];
                 e = launch_stencil(MODE_PCGA, nc, a, op->cap_stream);
-                an.u = Halo{a.pnew, nullptr, nullptr, 0, 0};  // one GPU
+                an.u = aniso_p_halo(op, kk);
                 if (e == cudaSuccess && op->aniso) e = launch_aniso(MODE_PCGA, an, op->cap_stream);
                 if (e == cudaSuccess) e = launch_pcg_b(b, op->b_blocks, op->cap_stream);
             }
@@ -864,13 +875,11 @@ mas_status_t mas_op_radial_sums(const mas_op_t* op_c, const double* x, const dou
 mas_status_t mas_op_enable_p2p(mas_op_t* op, cudaStream_t s) {
     if (!op) return arg_error("null op");
     if (op->p2p) return MAS_OK;
-    if (op->aniso)  // the mailbox carries kernel A's sigma only; L_par runs the NCCL loop
-        return arg_error("P2P transport with the field-aligned term (mas_op_set_aniso) is not supported");
     Comm* comm = op->g->comm;
     const int P = comm_nranks(comm), rank = comm_rank(comm);
     const bool virt = comm_is_virtual(comm);
-    ST(dmalloc(&op->mbox, 2 * (size_t)P));
-    CU(cudaMemset(op->mbox, 0, 2 * (size_t)P * sizeof(Mail)));
+    ST(dmalloc(&op->mbox, MB_SLOTS * (size_t)P));
+    CU(cudaMemset(op->mbox, 0, MB_SLOTS * (size_t)P * sizeof(Mail)));
     struct Rec {
         cudaIpcMemHandle_t h[4];
         unsigned long long raw[4];
@@ -1006,7 +1015,6 @@ mas_status_t mas_op_set_aniso(mas_op_t* op, const double* kpar, const double* bh
     if (op->ncomp != 1) return arg_error("field-aligned conduction needs ncomp == 1");
     if (op->g->ptheta > 1)
         return arg_error("field-aligned conduction: r-slab decompositions only (ptheta == 1)");
-    if (op->p2p) return arg_error("field-aligned conduction runs the NCCL loop (P2P transport is on)");
     mas_grid* g = op->g;
     const int nl = g->nl, nt = g->ntl, np = g->np;
     const long long N = op->Nl;
@@ -1162,6 +1170,7 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
     a.scr = op->scr;
     a.host_flag = op->host_flag_dev;
     a.p2p = p2p_args(op);
+    a.nopub = op->aniso && p2p;  // k_aniso<RESID> publishes the corrected init sums
     CU(launch_stencil(MODE_RESID, nc, a, s));
     op->launches++;
     AnisoArgs an{};
@@ -1188,6 +1197,7 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
     b.scr = op->scr;
     b.host_flag = op->host_flag_dev;
     b.p2p = p2p_args(op);
+    b.aniso = op->aniso;
 
     // a4: iterations.  Kernel A(k) reads k, alpha, beta and the convergence
     // decision from PcgState; the host only keeps two iterations in flight
@@ -1208,7 +1218,7 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
         a.pnew = op->p[1];
         CU(launch_stencil(MODE_PCGA, nc, a, s, true));
         if (op->aniso) {
-            an.u = Halo{a.pnew, nullptr, nullptr, 0, 0};  // one GPU
+            an.u = aniso_p_halo(op, 1);
             CU(launch_aniso(MODE_PCGA, an, s));
         }
         CU(launch_pcg_b(b, op->b_blocks, s));
@@ -1275,10 +1285,11 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
         }
         if (pe) CU(cudaEventRecord(pe[1], s));
         if (op->aniso) {  // q += L_par p_k, sigma += <p_k, L_par p_k> (rank-local)
-            if (comm)  // the p_k planes of the r-neighbours (kernel A(k) just wrote them)
+            if (comm && !p2p)  // the p_k planes of the r-neighbours (kernel A(k) just wrote them)
                 ST(comm_seams(comm, pnew, 1, op->g->nl, plane, op->pkg, op->pkg + plane, s,
                               rstride(op)));
-            an.u = halo_of(op, pnew, op->pkg, 1);
+            if (p2p) ST(comm_vsync(comm, s));  // virtual P2P ranks: all A(k) done
+            an.u = aniso_p_halo(op, k);
             if (pe) CU(cudaEventRecord(pe[4], s));
             CU(launch_aniso(MODE_PCGA, an, s));
             if (pe) CU(cudaEventRecord(pe[5], s));

@@ -52,71 +52,6 @@ enum { P_NORMAL = 0, P_FINAL = 1, P_ZERO = 2 };
 enum { TKT_STENCIL = 0, TKT_B = 1, TKT_DOT = 2 };
 
 // --------------------------------------------------------------------------
-// P2P transport: one-shot allreduce through peer mailboxes (NVLink stores)
-// --------------------------------------------------------------------------
-// The reducing kernel's last block writes its rank-local partials into slot
-// [rank] of EVERY rank's mailbox, then (after a system-scope fence) the
-// sequence number.  A consumer kernel waits in thread 0 of each block until
-// all nranks entries of its own mailbox carry the expected sequence and sums
-// them in rank order: every rank obtains the same bits, so every rank takes
-// the same stop / breakdown decision and the loop needs no host handshake.
-// A publication of iteration k needs every rank past its consumer of
-// iteration k-1 (each kernel waits for all ranks' previous partials), so one
-// mailbox slot per kernel kind suffices.
-__device__ __forceinline__ unsigned long long p2p_seq(unsigned long long epoch, int k) {
-    return (epoch << 32) | (unsigned long long)(unsigned)(k + 1);
-}
-__device__ __forceinline__ unsigned long long gtimer_ns() {
-    unsigned long long t;
-    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
-    return t;
-}
-constexpr unsigned long long kP2PTimeoutNs = 60ull * 1000000000ull;
-// slow path: spin (with a 60 s limit: fail loudly rather than hang)
-__device__ __noinline__ void p2p_wait(const volatile unsigned long long* sp, unsigned long long seq,
-                                      int rank, int slot, int from) {
-    const unsigned long long t0 = gtimer_ns();
-    while (*sp != seq) {
-        __nanosleep(100);
-        if (gtimer_ns() - t0 > kP2PTimeoutNs) {
-            printf("maspcg: P2P mailbox wait timed out (rank %d, slot %d, from rank %d)\n", rank,
-                   slot, from);
-            __trap();
-        }
-    }
-}
-
-// the calling thread waits for and sums the nranks entries (rank order)
-template <int N>
-__device__ __forceinline__ void p2p_gather_one(const P2P& t, int slot, unsigned long long seq,
-                                               double (&out)[N]) {
-    const Mail* mb = t.own + slot * t.nranks;
-#pragma unroll
-    for (int n = 0; n < N; n++) out[n] = 0.0;
-    for (int q = 0; q < t.nranks; q++) {
-        const volatile unsigned long long* sp = &mb[q].seq;
-        if (*sp != seq) p2p_wait(sp, seq, t.rank, slot, q);
-        __threadfence_system();  // the values were written before the sequence
-        const volatile double* v = mb[q].v;
-#pragma unroll
-        for (int n = 0; n < N; n++) out[n] += v[n];
-    }
-}
-
-// thread 0 of the last block: publish n rank-local partials to every rank
-__device__ void p2p_publish(const P2P& t, int slot, unsigned long long seq, const double* v, int n) {
-    for (int q = 0; q < t.nranks; q++) {
-        volatile Mail* m = t.peers[q] + slot * t.nranks + t.rank;
-        for (int i = 0; i < n; i++) m->v[i] = v[i];
-    }
-    __threadfence_system();
-    for (int q = 0; q < t.nranks; q++) {
-        volatile Mail* m = t.peers[q] + slot * t.nranks + t.rank;
-        m->seq = seq;
-    }
-}
-
-// --------------------------------------------------------------------------
 // field access
 // --------------------------------------------------------------------------
 // The stencil kernels index with 32-bit offsets (the host rejects slabs with
@@ -820,7 +755,7 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
             st->pend_ff = acc[0];
             st->pend_rr = acc[1];
             st->pend_rho = acc[2];
-            if (p2p) {
+            if (p2p && !a.nopub) {  // (with the field-aligned term k_aniso<RESID> publishes)
                 const double pub[3] = {acc[2], acc[1], acc[0]};  // {rho, rr, ff}
                 p2p_publish(a.p2p, MB_B, p2p_seq(st->epoch, 0), pub, 3);
             }
@@ -868,7 +803,13 @@ __global__ void __launch_bounds__(kThreads) k_pcg_b(const StreamArgs a) {
         __shared__ double sh_sigma;
         if (threadIdx.x == 0) {
             double v[1];
-            p2p_gather_one<1>(a.p2p, MB_A, p2p_seq(__ldcg(&vst->epoch), kit), v);
+            const unsigned long long seq = p2p_seq(__ldcg(&vst->epoch), kit);
+            p2p_gather_one<1>(a.p2p, MB_A, seq, v);
+            if (a.aniso) {  // + the field-aligned part, summed over the ranks by k_aniso(k)
+                double u[1];
+                p2p_gather_one<1>(a.p2p, MB_C, seq, u);
+                v[0] = v[0] + u[0];
+            }
             sh_sigma = v[0];
         }
         __syncthreads();

@@ -72,9 +72,11 @@ struct Mail {                 // one rank's published partial sums
     unsigned long long seq;   // (epoch << 32) | (k + 1) once v is valid
     unsigned long long pad[3];
 };
-enum { MB_A = 0, MB_B = 1 };  // mailbox slots: A(k) -> B(k) (sigma); B(k)/init -> A(k+1)
+// mailbox slots: A(k) -> B(k) (sigma); B(k)/init -> A(k+1); the field-aligned
+// term's k_aniso(k) -> B(k) (its sigma part)
+enum { MB_A = 0, MB_B = 1, MB_C = 2, MB_SLOTS = 3 };
 struct P2P {
-    Mail* own;                // this rank's mailbox [2 slots][nranks]
+    Mail* own;                // this rank's mailbox [MB_SLOTS][nranks]
     Mail* const* peers;       // [nranks] every rank's mailbox (device-visible pointers)
     int nranks;               // 0: transport off
     int rank;
@@ -132,6 +134,7 @@ struct StencilArgs {
                               // (interior runs while the seams are in flight)
     unsigned long long cond;  // CUDA graph while-loop handle (0: not in a graph)
     P2P p2p;                  // RESID / PCGA: mailbox transport (nranks == 0: off)
+    int nopub;                // RESID under P2P with the field-aligned term: k_aniso publishes
 };
 
 struct StreamArgs {  // kernel B
@@ -148,6 +151,7 @@ struct StreamArgs {  // kernel B
     int* host_flag;
     unsigned long long cond;
     P2P p2p;
+    int aniso;                // the field-aligned term is on: sigma also from MB_C (P2P)
 };
 
 // ---------------------------------------------------------------------------
@@ -184,6 +188,7 @@ struct AnisoArgs {
     PcgState* st;
     Scratch scr;
     unsigned long long cond;
+    P2P p2p;               // P2P transport: waits for every rank's A(k), publishes MB_C / MB_B
 };
 
 // launchers (kernels.cu)

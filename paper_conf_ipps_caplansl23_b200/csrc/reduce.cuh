@@ -6,6 +6,8 @@
 
 #include <cuda_runtime.h>
 
+#include <cstdio>
+
 #include "mas_internal.h"
 
 namespace mas {
@@ -71,6 +73,72 @@ __device__ bool grid_reduce(double (&v)[NS], const Scratch& scr, int tkt, bool s
     }
     if (threadIdx.x == 0) scr.ticket[tkt] = 0u;
     return true;
+}
+
+
+// --------------------------------------------------------------------------
+// P2P transport: one-shot allreduce through peer mailboxes (NVLink stores)
+// --------------------------------------------------------------------------
+// The reducing kernel's last block writes its rank-local partials into slot
+// [rank] of EVERY rank's mailbox, then (after a system-scope fence) the
+// sequence number.  A consumer kernel waits in thread 0 of each block until
+// all nranks entries of its own mailbox carry the expected sequence and sums
+// them in rank order: every rank obtains the same bits, so every rank takes
+// the same stop / breakdown decision and the loop needs no host handshake.
+// A publication of iteration k needs every rank past its consumer of
+// iteration k-1 (each kernel waits for all ranks' previous partials), so one
+// mailbox slot per kernel kind suffices.
+__device__ __forceinline__ unsigned long long p2p_seq(unsigned long long epoch, int k) {
+    return (epoch << 32) | (unsigned long long)(unsigned)(k + 1);
+}
+__device__ __forceinline__ unsigned long long gtimer_ns() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+constexpr unsigned long long kP2PTimeoutNs = 60ull * 1000000000ull;
+// slow path: spin (with a 60 s limit: fail loudly rather than hang)
+static __device__ __noinline__ void p2p_wait(const volatile unsigned long long* sp, unsigned long long seq,
+                                      int rank, int slot, int from) {
+    const unsigned long long t0 = gtimer_ns();
+    while (*sp != seq) {
+        __nanosleep(100);
+        if (gtimer_ns() - t0 > kP2PTimeoutNs) {
+            printf("maspcg: P2P mailbox wait timed out (rank %d, slot %d, from rank %d)\n", rank,
+                   slot, from);
+            __trap();
+        }
+    }
+}
+
+// the calling thread waits for and sums the nranks entries (rank order)
+template <int N>
+__device__ __forceinline__ void p2p_gather_one(const P2P& t, int slot, unsigned long long seq,
+                                               double (&out)[N]) {
+    const Mail* mb = t.own + slot * t.nranks;
+#pragma unroll
+    for (int n = 0; n < N; n++) out[n] = 0.0;
+    for (int q = 0; q < t.nranks; q++) {
+        const volatile unsigned long long* sp = &mb[q].seq;
+        if (*sp != seq) p2p_wait(sp, seq, t.rank, slot, q);
+        __threadfence_system();  // the values were written before the sequence
+        const volatile double* v = mb[q].v;
+#pragma unroll
+        for (int n = 0; n < N; n++) out[n] += v[n];
+    }
+}
+
+// thread 0 of the last block: publish n rank-local partials to every rank
+static __device__ void p2p_publish(const P2P& t, int slot, unsigned long long seq, const double* v, int n) {
+    for (int q = 0; q < t.nranks; q++) {
+        volatile Mail* m = t.peers[q] + slot * t.nranks + t.rank;
+        for (int i = 0; i < n; i++) m->v[i] = v[i];
+    }
+    __threadfence_system();
+    for (int q = 0; q < t.nranks; q++) {
+        volatile Mail* m = t.peers[q] + slot * t.nranks + t.rank;
+        m->seq = seq;
+    }
 }
 
 }  // namespace mas

@@ -230,26 +230,22 @@ def test_degenerate_grids(mp, oracle_mod, shape):
     np.testing.assert_allclose(host(D), o.diag(kappa, c) + o.aniso_diag(kpar, b), rtol=1e-13, atol=0)
 
 
-def test_p2p_transport_and_aniso_are_exclusive(mp):
-    """The P2P mailbox carries kernel A's sigma only: with the field-aligned
-    term on, mas_op_enable_p2p refuses, and mas_op_set_aniso refuses on a P2P
-    op (one GPU: the mailbox runs against itself)."""
-    shape = (8, 16, 64)
-    mesh = W.stretched_mesh(*shape)
-    kappa, c, kpar, b = rand_fields(shape, 31)
-    g, op = setup(mp, mesh, kappa, c, kpar, b)
-    with pytest.raises(mp.MasError) as e:
-        op.enable_p2p()
-    assert e.value.status == mp.MAS_ERR_ARG
-    g2 = mp.Grid(mesh)
-    op2 = mp.Operator(g2, 1, dev(kappa), dev(c), 0, 1)
-    op2.enable_p2p()
-    with pytest.raises(mp.MasError) as e:
-        op2.set_aniso(dev(kpar), dev(b))
-    assert e.value.status == mp.MAS_ERR_ARG
-    # both ops still solve correctly afterwards
-    f = dev(W.random_field((1,) + shape, 32))
-    for o_ in (op, op2):
-        x = torch.zeros_like(f)
-        st, it, rel, _ = o_.solve(f, x, 1e-10, 2000)
-        assert st == mp.MAS_OK and rel <= 1e-10
+def test_aniso_on_the_p2p_mailbox_loop_one_gpu(mp, oracle_mod):
+    """The P2P transport on one GPU (the mailbox runs against itself, the loop
+    is one CUDA graph): kernel A publishes its sigma to slot A, k_aniso its
+    part to slot C, kernel B sums both; the init sums come from k_aniso<RESID>.
+    Bitwise equal to the plain single-GPU loop (both add the two parts in the
+    same order), and the oracle's iteration count."""
+    prob = W.aniso_conduction_problem(16, 24, 64)
+    a = _solve_pair(mp, oracle_mod, prob, 1e-12, 5000)
+    g = mp.Grid(prob.mesh)
+    op = mp.Operator(g, 1, dev(prob.kappa), dev(prob.c), prob.bc_inner, prob.bc_outer)
+    op.enable_p2p()
+    op.set_aniso(dev(prob.kpar), dev(prob.bhat))
+    f = dev(prob.f)
+    op.dirichlet_rhs(dev(prob.ub_inner), None, f)
+    for _ in range(2):  # repeated solves: mailbox epochs
+        x = dev(prob.x0)
+        st, it, rel, _ = op.solve(f, x, 1e-12, 5000)
+        assert st == mp.MAS_OK and it == a[1]
+        assert np.array_equal(host(x), a[2])

@@ -31,7 +31,7 @@ def mp():
     return maspcg
 
 
-def run_ranks(mp, prob, P, x_apply, tol, maxit):
+def run_ranks(mp, prob, P, x_apply, tol, maxit, p2p=False):
     _key[0] += 1
     vid = mp.virtual_ranks_id(_key[0])
     res, errs = {}, []
@@ -47,6 +47,8 @@ def run_ranks(mp, prob, P, x_apply, tol, maxit):
                 d = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()
                 op = mp.Operator(g, 1, d(prob.kappa[sl]), d(prob.c[sl]), prob.bc_inner,
                                  prob.bc_outer)
+                if p2p:  # the mailbox loop: p_k read in place from the neighbours
+                    op.enable_p2p()
                 op.set_aniso(d(prob.kpar[sl]), d(prob.bhat[:, sl]))
                 y = torch.empty((1, nl) + prob.shape[1:], dtype=torch.float64, device="cuda")
                 op.apply(d(x_apply[:, sl]), y)
@@ -77,11 +79,12 @@ def assemble(out, key, axis):
     return np.concatenate([r[key] for r in out], axis=axis)
 
 
+@pytest.mark.parametrize("p2p", [False, True])
 @pytest.mark.parametrize("P,shape", [(2, (16, 16, 64)), (3, (20, 24, 70)), (4, (33, 16, 128))])
-def test_aniso_virtual_ranks_match_oracle(mp, oracle_mod, P, shape):
+def test_aniso_virtual_ranks_match_oracle(mp, oracle_mod, P, shape, p2p):
     prob = W.aniso_conduction_problem(*shape)
     x = W.random_field((1,) + prob.shape, 42)
-    out = run_ranks(mp, prob, P, x, prob.tol, prob.maxit)
+    out = run_ranks(mp, prob, P, x, prob.tol, prob.maxit, p2p)
     o = oracle_mod.Oracle.for_problem(prob)
     V = o.volumes()[None]
     y = assemble(out, "y", 1)
