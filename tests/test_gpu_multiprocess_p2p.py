@@ -42,6 +42,8 @@ dv = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()
 op = M.Operator(g, prob.ncomp, dv(prob.kappa[sl]), dv(prob.c[sl]), prob.bc_inner, prob.bc_outer)
 if p2p:
     op.enable_p2p()
+if prob.kpar is not None:  # field-aligned conduction: neighbour p_k through the IPC mapping
+    op.set_aniso(dv(prob.kpar[sl]), dv(prob.bhat[slc]))
 f = dv(prob.f[slc])
 op.dirichlet_rhs(dv(prob.ub_inner[:, g.j0:g.j0 + g.ntl]) if prob.ub_inner is not None else None,
                  None, f)
@@ -94,7 +96,8 @@ def built():
 
 @pytest.mark.parametrize("P,kind,shape,ptheta", [(2, "viscosity", (12, 16, 64), 1),
                                                  (3, "conduction", (13, 16, 32), 1),
-                                                 (4, "viscosity", (10, 18, 64), 2)])
+                                                 (4, "viscosity", (10, 18, 64), 2),
+                                                 (2, "aniso", (12, 16, 64), 1)])
 def test_p2p_across_processes_matches_oracle(built, oracle_mod, tmp_path, P, kind, shape, ptheta):
     res, xs = run_procs(tmp_path, P, kind, shape, ptheta=ptheta)
     assert all(r["transport"] == "p2p" for r in res)
