@@ -183,8 +183,7 @@ def test_pcg_matches_oracle(mp, oracle_mod, shape):
     assert st == mp.MAS_OK and rc == oracle_mod.OK
     assert abs(it - ito) <= 1, (it, ito)
     V = oracle_mod.Oracle.for_problem(prob).volumes()
-    if it == ito:
-        assert rel_l2_V(V, x, xo) <= 1e-10
+    assert rel_l2_V(V, x, xo) <= 1e-10  # unconditional (north_star: x <= 1e-10)
     n = min(10, len(hist), len(histo))
     np.testing.assert_allclose(hist[:n], histo[:n], rtol=1e-9)
 

@@ -77,11 +77,18 @@ def test_apply_matches_oracle(mp, oracle_mod, shape, ncomp, bc):
     o = oracle_mod.Oracle(mesh, *bc)
     yo = o.apply(kappa, c, x)
     V = o.volumes()
-    assert rel_l2_V(V, host(y), yo) <= 1e-13
+    yg = host(y)
+    assert rel_l2_V(V, yg, yo) <= 1e-13
+    # elementwise: |L x| <= (c + 2 sum_f G_f / V) max|x| <= 2 D_P max|x|, so the
+    # per-cell error is bounded relative to that cell's own scale (V spans
+    # ~1e5 on these meshes, which the V-weighted norm alone would hide)
+    scale = 2.0 * o.diag(kappa, c)[None] * np.abs(x).max()
+    assert (np.abs(yg - yo) / scale).max() <= 1e-13
     # host-pointer path of the same ABI call
     yh = np.empty_like(x)
     op.apply(np.ascontiguousarray(x), yh)
     assert rel_l2_V(V, yh, yo) <= 1e-13
+    assert (np.abs(yh - yo) / scale).max() <= 1e-13
 
 
 @pytest.mark.parametrize("shape", SHAPES[:3])
@@ -155,8 +162,7 @@ def test_pcg_matches_oracle_at_tol(mp, oracle_mod, idx):
     assert abs(it - ito) <= 1, (it, ito)
     assert rel <= prob.tol
     V = oracle_mod.Oracle.for_problem(prob).volumes()
-    if it == ito:
-        assert rel_l2_V(V, x, xo) <= 1e-10
+    assert rel_l2_V(V, x, xo) <= 1e-10  # unconditional (north_star: x <= 1e-10)
     # Residual histories: CG amplifies rounding differences; the oracle run
     # against itself with a 1e-16 relative perturbation of f already differs
     # by 1e-4..3e-3 after ~20 iterations on these stiff problems (DESIGN.md
@@ -171,7 +177,6 @@ def test_pcg_matches_oracle_at_tol(mp, oracle_mod, idx):
     env = np.maximum.accumulate(np.abs(histp[:m] - histo[:m]) / histo[:m])
     dev_ = np.abs(hist[:m] - histo[:m]) / histo[:m]
     assert (dev_ <= 20.0 * env + 1e-9).all(), (dev_.max(), env.max())
-    assert op.launch_count >= 2 * it
 
 
 @pytest.mark.parametrize("k", [1, 2, 7, 40])

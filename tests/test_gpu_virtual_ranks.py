@@ -120,8 +120,7 @@ def test_virtual_ranks_apply_dot_and_pcg(mp, oracle_mod, P):
     assert all(r["st"] == mp.MAS_OK for r in out)
     assert abs(it - ito) <= 1
     xg = assemble(out, "x")
-    if it == ito:
-        assert math.sqrt((V * (xg - xo) ** 2).sum() / (V * xo ** 2).sum()) <= 1e-10
+    assert math.sqrt((V * (xg - xo) ** 2).sum() / (V * xo ** 2).sum()) <= 1e-10  # unconditional (north_star: x <= 1e-10)
 
 
 @pytest.mark.parametrize("P", [2, 3])
@@ -232,8 +231,7 @@ def test_virtual_ranks_theta_split_matches_oracle(mp, oracle_mod, P, ptheta, sha
         it = its.pop()
         assert all(r["st"] == mp.MAS_OK for r in out) and abs(it - ito) <= 1
         xg = assemble(out, "x")
-        if it == ito:
-            assert math.sqrt((V * (xg - xo) ** 2).sum() / (V * xo ** 2).sum()) <= 1e-10
+        assert math.sqrt((V * (xg - xo) ** 2).sum() / (V * xo ** 2).sum()) <= 1e-10  # unconditional (north_star: x <= 1e-10)
         res[p2p] = (it, xg)
     # both loops sum the same block partials in rank order
     assert res[False][0] == res[True][0]

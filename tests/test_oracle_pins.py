@@ -424,3 +424,56 @@ def test_block_apply_bitwise(oracle_mod, pr, pt, bc):
             xb = np.ascontiguousarray(x[:, i0:i0 + nl, j0:j0 + ntl])
             dots.append(o.dot_block(i0, nl, j0, ntl, xb, xb))
     assert abs(sum(dots) - o.dot(x, x)) <= 1e-14 * o.dot(x, x)
+
+
+# ---------------------------------------------------------------------------
+# per-cell sampler (the full-size C2/C3 checker) == the whole-field operator
+# ---------------------------------------------------------------------------
+def _boundary_class_indices(shape, ncomp, rng, n_random):
+    """Flat comp-major indices m*N + P covering every boundary class: the r
+    boundary planes (i = 0, nr-1), the pole rows (j = 0, nt-1), the phi wrap
+    columns (k = 0, np-1), the GPU tile and chunk edges (j = 7, 8, 15, 16;
+    k = 63, 64, 127, 128; i = 31, 32), all their combinations (corners), for
+    every component, plus n_random uniform cells."""
+    nr, nt, np_ = shape
+    N = nr * nt * np_
+
+    def cand(n, edges):
+        return sorted({e for e in (0, 1, n - 2, n - 1, *edges) if 0 <= e < n})
+
+    I = cand(nr, (31, 32, 33))
+    J = cand(nt, (7, 8, 15, 16))
+    K = cand(np_, (63, 64, 127, 128))
+    idx = [m * N + (i * nt + j) * np_ + k for m in range(ncomp) for i in I for j in J for k in K]
+    idx += list(rng.integers(0, ncomp * N, size=n_random))
+    return np.unique(np.asarray(idx, dtype=np.int64))
+
+
+@pytest.mark.parametrize("shape,ncomp,bc", [
+    ((5, 6, 8), 3, (0, 1)),          # every cell of a tiny grid, all 3 components
+    ((40, 20, 132), 1, (0, 0)),      # ragged tile/chunk edges, Dirichlet both ends
+    ((34, 18, 130), 3, (1, 1)),      # Neumann both ends, 3 components
+    ((33, 17, 66), 3, (0, 1)),       # odd nr / nt
+])
+def test_apply_cells_equals_apply_bitwise(oracle_mod, shape, ncomp, bc):
+    """mas_ref_op_apply_cells re-decodes flat indices (m, i, j, k) on its own;
+    it must return exactly the values of the whole-field mas_ref_op_apply
+    (itself pinned above) at every sampled cell, boundary classes included.
+    An index-decoding slip (i/j swapped, component offset, phi wrap) fails."""
+    m = W.stretched_mesh(*shape)
+    o = oracle_mod.Oracle(m, *bc)
+    kappa, c = rand_coeffs(shape, 11)
+    rng = np.random.default_rng(12)
+    x = rng.uniform(-1.0, 1.0, size=(ncomp,) + shape)
+    y = o.apply(kappa, c, x).ravel()
+    N = o.N
+    if ncomp * N <= 4096:
+        idx = np.arange(ncomp * N, dtype=np.int64)
+    else:
+        idx = _boundary_class_indices(shape, ncomp, rng, 2000)
+    assert idx.size >= min(ncomp * N, 2000)
+    got = o.apply_cells(kappa, c, x, idx)
+    assert np.array_equal(got, y[idx]), np.abs(got - y[idx]).max()
+    # and with no mass term (c = NULL), as the full-size tests may pass
+    y0 = o.apply(kappa, np.zeros(shape), x).ravel()
+    assert np.array_equal(o.apply_cells(kappa, None, x, idx), y0[idx])
