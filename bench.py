@@ -140,6 +140,17 @@ def scaling_of(cfg: str) -> str:
     return "weak" if cfg == "C4" else "strong"
 
 
+def cpu_model() -> str:
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        kv = dict(ln.split(":", 1) for ln in out.splitlines() if ":" in ln)
+        return "; ".join(f"{k.strip()}: {kv[k].strip()}" for k in
+                         ("Model name", "Socket(s)", "Core(s) per socket", "Thread(s) per core")
+                         if k in kv)
+    except Exception:
+        return "unknown"
+
+
 def cpu_cores() -> int:
     try:
         return len(os.sched_getaffinity(0))
@@ -172,8 +183,10 @@ def oracle_runner(o, prob, f):
 
 
 def host_dram_gbs(threads: int):
-    """Host DRAM copy bandwidth (tools/hostbw.c, OpenMP, 2 GiB per array),
-    the CPU roofline the oracle's time is set against."""
+    """Host DRAM bandwidth (tools/hostbw.c, OpenMP, 2 GiB per array), the CPU
+    roofline the oracle's time is set against: max of a copy
+    counted with its write-allocate traffic (24 B/element) and a read-only
+    sum (8 B/element).  Returns (max, copy, read) in GB/s."""
     import ctypes
     src = os.path.join(ROOT, "tools", "hostbw.c")
     so = os.path.join(ROOT, "tools", "libhostbw.so")
@@ -181,12 +194,15 @@ def host_dram_gbs(threads: int):
         if not os.path.exists(so) or os.path.getmtime(so) < os.path.getmtime(src):
             subprocess.check_call(["gcc", "-O2", "-fopenmp", "-shared", "-fPIC", "-o", so, src])
         lib = ctypes.CDLL(so)
-        lib.host_copy_gbs.restype = ctypes.c_double
-        lib.host_copy_gbs.argtypes = [ctypes.c_longlong, ctypes.c_int]
+        for fn in (lib.host_copy_gbs, lib.host_read_gbs):
+            fn.restype = ctypes.c_double
+            fn.argtypes = [ctypes.c_longlong, ctypes.c_int]
         os.environ.setdefault("OMP_NUM_THREADS", str(threads))
-        return float(lib.host_copy_gbs(1 << 28, 3))
+        cp = float(lib.host_copy_gbs(1 << 28, 3))
+        rd = float(lib.host_read_gbs(1 << 28, 3))
+        return max(cp, rd), cp, rd
     except Exception:
-        return None
+        return None, None, None
 
 
 # bytes per cell per iteration of the oracle's textbook (unfused) PCG, per
@@ -199,7 +215,10 @@ def oracle_bytes_per_cell(ncomp):
 
 def run_reference(args):
     """--impl reference: the CPU oracle on this box's host cores, same config,
-    metric and unit; each step = 2 fixed oracle PCG iterations on the full grid."""
+    metric and unit.  Each step is a bounded sample of the workload: 2 fixed
+    oracle PCG iterations on the full grid, timed as run(1 + 2) - run(1) so
+    the oracle's per-solve setup (diagonal, initial residual) is subtracted,
+    as in the cpu_baseline leg."""
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return 0
@@ -212,14 +231,19 @@ def run_reference(args):
     per_step_iters = 2
     run = oracle_runner(o, prob, f)
     for _ in range(args.warmup):
-        run(per_step_iters)
-    t0 = time.perf_counter()
+        run(1)
+    dt = 0.0
     for _ in range(args.steps):
-        run(per_step_iters)
-    dt = time.perf_counter() - t0
+        t0 = time.perf_counter()
+        run(1)
+        t1 = time.perf_counter()
+        run(1 + per_step_iters)
+        t2 = time.perf_counter()
+        dt += max((t2 - t1) - (t1 - t0), 1e-9)
     value = args.steps * per_step_iters / dt
     sample = (f"{args.config} full grid {prob.shape}, ncomp {prob.ncomp}: {per_step_iters} fixed "
-              f"oracle PCG iterations per step incl. its setup (diag + initial residual)")
+              f"oracle PCG iterations per step, timed as run(1+{per_step_iters}) - run(1) "
+              f"(setup subtracted)")
     line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * dt / args.steps,
             "higher_is_better": True, "scaling": scaling_of(args.config), "vs_baseline": None,
@@ -407,32 +431,35 @@ def main():
         pin = lambda a: torch.from_numpy(np.ascontiguousarray(a)).pin_memory()
         hk, hc, hf, hx0 = pin(prob.kappa[sl]), pin(prob.c[sl]), rhs.cpu().pin_memory(), \
             pin(prob.x0[slc])
-        ksteps = max(1, min(args.steps, 2))
-        # one pinned x0 per step (the solve overwrites x in place), filled
-        # before the timed region; one untimed warm-up step allocates the
-        # library's host-staging buffers
-        hxs = [hx0.clone().pin_memory() for _ in range(ksteps + 1)]
+        ksteps = args.steps
+        # the solve overwrites x in place: x0 is refilled into the pinned
+        # buffer between steps, outside the timed intervals (a host memcpy the
+        # caller does, not library work); one untimed warm-up step allocates
+        # the library's host-staging buffers
+        hx = hx0.clone().pin_memory()
         if aniso:
             hkp, hb = pin(prob.kpar[sl]), pin(prob.bhat[(slice(None),) + sl])
         op.update(hk, hc)
         if aniso:
             op.set_aniso(hkp, hb)
-        op.solve(hf, hxs[-1], args.tol, maxit)
+        op.solve(hf, hx, args.tol, maxit)
         torch.cuda.synchronize()
         if world > 1:
             dist.barrier()
+        te, e2e_iters = 0.0, 0
         h0, h1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        h0.record(stream)
-        e2e_iters = 0
         for sidx in range(ksteps):
+            hx.copy_(hx0)
+            torch.cuda.synchronize()
+            h0.record(stream)
             op.update(hk, hc)
             if aniso:
                 op.set_aniso(hkp, hb)
-            st, it, rel, _ = op.solve(hf, hxs[sidx], args.tol, maxit)
+            st, it, rel, _ = op.solve(hf, hx, args.tol, maxit)
+            h1.record(stream)
+            torch.cuda.synchronize()
+            te += h0.elapsed_time(h1)
             e2e_iters += it
-        h1.record(stream)
-        torch.cuda.synchronize()
-        te = h0.elapsed_time(h1)
         if world > 1:
             tt = torch.tensor([te], device=dev, dtype=torch.float64)
             dist.all_reduce(tt, op=dist.ReduceOp.MAX)
@@ -441,18 +468,26 @@ def main():
         e2e = {"value": e2e_iters / (te / 1e3), "unit": UNIT, "h2d_bytes_per_step": h2d,
                "d2h_bytes_per_step": nc * cells_local * 8,
                "note": "pinned host kappa, c, rhs, x0 (+ kpar, bhat for C2a) -> device inside the "
-                       "timed region; x -> host; "
-                       "1 untimed warm-up step"}
+                       "timed region; x -> host; all K steps (per-step CUDA events, x0 refilled "
+                       "between them); 1 untimed warm-up step"}
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         cores = cpu_cores()
         v, per = oracle_sample(prob, args.cpu_iters, cores)
-        hbw = host_dram_gbs(cores)
+        # the survey's single-thread point (SURVEY §8(d) timing protocol), one
+        # fixed iteration on the same grid
+        v1, per1 = oracle_sample(prob, 1, 1)
+        hbw, hcp, hrd = host_dram_gbs(cores)
         ob = oracle_bytes_per_cell(nc) * cells * v / 1e9
         cpu = {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle",
-               "host_dram_copy_gbs": hbw, "oracle_alg_gbs": ob,
+               "host_dram_gbs": hbw, "host_copy_gbs_with_write_allocate": hcp,
+               "host_read_gbs": hrd, "oracle_alg_gbs": ob,
                "oracle_frac_of_host_dram": (ob / hbw) if hbw else None,
+               "cpu_model": cpu_model(),
+               "one_thread": {"value": v1, "unit": UNIT, "cores": 1,
+                              "sample": f"{args.config} full grid, 1 fixed oracle PCG iteration "
+                                        f"(setup subtracted); {per1:.3f} s/iteration"},
                "sample": f"{args.config} full grid, {args.cpu_iters} fixed oracle PCG iterations "
                          f"(setup subtracted via a 1-iteration run); {per:.3f} s/iteration"}
 

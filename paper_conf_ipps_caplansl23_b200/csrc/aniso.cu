@@ -235,6 +235,10 @@ __global__ void __launch_bounds__(WTHREADS, 1) k_aniso(const AnisoArgs a, const 
             p2p_gather_one<1>(a.p2p, MB_A, p2p_seq(__ldcg(&a.st->epoch), kit), v);
         }
         __syncthreads();
+        // the neighbours' p_k was written through the generic proxy; the
+        // producer reads it with tensor copies (async proxy): order the two
+        // before the first cp.async.bulk.tensor of the lo / hi maps
+        asm volatile("fence.proxy.async.global;\n" ::: "memory");
     }
     const Geo& g = a.g;
     const int plane = (int)g.plane;
@@ -556,14 +560,7 @@ cudaError_t launch_aniso(int mode, const AnisoArgs& a0, cudaStream_t s) {
     a.ntj = (a.g.nt + WJ - 1) / WJ;
     a.ntk = (a.g.np + WK - 1) / WK;
     const int tiles = a.ntj * a.ntk;
-    static int sms = 0;
-    if (!sms) {
-        int dev = 0;
-        cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-        if (sms <= 0) sms = 148;
-    }
-    long long want = sms;  // one block per SM (223 KB of rings each)
+    long long want = device_sms();  // one block per SM (223 KB of rings each)
     if (const char* e = getenv("MAS_ABLOCKS")) want = std::max(1, atoi(e));  // experiment hook
     want = std::min<long long>(want, (long long)tiles * a.g.nl);
     want = std::min<long long>(want, a.max_blocks);
@@ -576,13 +573,17 @@ cudaError_t launch_aniso(int mode, const AnisoArgs& a0, cudaStream_t s) {
         set_last_error("k_aniso: cuTensorMapEncodeTiled failed");
         return cudaErrorInvalidValue;
     }
-    static bool attr = false;
-    if (!attr) {
-        cudaFuncSetAttribute(k_aniso<MODE_APPLY>, cudaFuncAttributeMaxDynamicSharedMemorySize, kAnisoSmem);
-        cudaFuncSetAttribute(k_aniso<MODE_RESID>, cudaFuncAttributeMaxDynamicSharedMemorySize, kAnisoSmem);
-        cudaFuncSetAttribute(k_aniso<MODE_PCGA>, cudaFuncAttributeMaxDynamicSharedMemorySize, kAnisoSmem);
-        attr = true;
-    }
+    static DeviceOnce attr;
+    cudaError_t e = attr.run([] {
+        cudaError_t r = cudaFuncSetAttribute(k_aniso<MODE_APPLY>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                             kAnisoSmem);
+        if (r == cudaSuccess)
+            r = cudaFuncSetAttribute(k_aniso<MODE_RESID>, cudaFuncAttributeMaxDynamicSharedMemorySize, kAnisoSmem);
+        if (r == cudaSuccess)
+            r = cudaFuncSetAttribute(k_aniso<MODE_PCGA>, cudaFuncAttributeMaxDynamicSharedMemorySize, kAnisoSmem);
+        return r;
+    });
+    if (e != cudaSuccess) return e;
     if (mode == MODE_APPLY)
         k_aniso<MODE_APPLY><<<blocks, WTHREADS, kAnisoSmem, s>>>(a, M);
     else if (mode == MODE_RESID)

@@ -122,7 +122,9 @@ struct mas_op {
     const double* g_x = nullptr;
     const double* g_hist = nullptr;
     int g_aniso = -1;
+    int g_pre = -1;
     int use_graph = 1;
+    int graph_pre = 0;                 // MAS_GRAPH_PRE: iteration 1 outside the graph
     // P2P transport (mas_op_enable_p2p): mailbox allreduce + in-place reads of
     // the r-neighbours' edge planes over NVLink instead of NCCL in the loop
     int p2p = 0;
@@ -500,28 +502,68 @@ static mas_status_t ensure_prof_events(mas_op* op, int k) {
     return MAS_OK;
 }
 
-// Build (or reuse) the graph of the iteration loop: while (!stopped) {A B A B}.
+// Build (or reuse) the graph of the whole iteration loop:
+//   A(1) [L_par(1)] B(1) -> while (!stopped) { A B A B }   (iterations 2, 3, ...)
+// Kernel A of iteration 1 is its own instantiation (FIRSTK), so it sits
+// ahead of the while node, in the same graph: one graph launch per solve.
 // Kernels read k, alpha, beta and the stop decision from PcgState; the
 // deciding kernel's last block sets the while-condition to 0.
-static mas_status_t loop_graph(mas_op* op, StencilArgs a, StreamArgs b, AnisoArgs an) {
-    if (op->gexec && op->g_x == a.x && op->g_hist == a.rho_hist && op->g_aniso == op->aniso)
+// (MAS_GRAPH_PRE=1, an experiment hook, launches iteration 1 as plain
+// kernels ahead of a graph holding only the while node, the round-1 form.)
+static mas_status_t loop_graph(mas_op* op, StencilArgs a, StreamArgs b, AnisoArgs an, bool pre_plain) {
+    if (op->gexec && op->g_x == a.x && op->g_hist == a.rho_hist && op->g_aniso == op->aniso &&
+        op->g_pre == (int)pre_plain)
         return MAS_OK;
     if (op->gexec) {
         cudaGraphExecDestroy(op->gexec);
         op->gexec = nullptr;
     }
     if (!op->cap_stream) CU(cudaStreamCreateWithFlags(&op->cap_stream, cudaStreamNonBlocking));
+    const int nc = op->ncomp;
     cudaGraph_t g;
     CU(cudaGraphCreate(&g, 0));
+    cudaError_t e = cudaSuccess;
+    std::vector<cudaGraphNode_t> deps;
+    if (!pre_plain) {  // iteration 1 into the top-level graph, as a chain of kernel nodes
+        e = cudaStreamBeginCaptureToGraph(op->cap_stream, g, nullptr, nullptr, 0,
+                                          cudaStreamCaptureModeThreadLocal);
+        if (e == cudaSuccess) {
+            StencilArgs a1 = a;
+            a1.pold = pold_halo(op, 1);  // not read in iteration 1
+            a1.tpold = pold_trows(op, 1);
+            a1.pnew = op->p[1];
+            e = launch_stencil(MODE_PCGA, nc, a1, op->cap_stream, true);
+            if (e == cudaSuccess && op->aniso) {
+                AnisoArgs an1 = an;
+                an1.u = aniso_p_halo(op, 1);
+                e = launch_aniso(MODE_PCGA, an1, op->cap_stream);
+            }
+            if (e == cudaSuccess) e = launch_pcg_b(b, op->b_blocks, op->cap_stream);
+            cudaGraph_t out = g;
+            cudaError_t e2 = cudaStreamEndCapture(op->cap_stream, &out);
+            if (e == cudaSuccess) e = e2;
+        }
+        // the chain's leaf (the node no other node depends on) precedes the loop
+        size_t n = 0;
+        if (e == cudaSuccess) e = cudaGraphGetNodes(g, nullptr, &n);
+        std::vector<cudaGraphNode_t> nodes(n);
+        if (e == cudaSuccess && n) e = cudaGraphGetNodes(g, nodes.data(), &n);
+        for (size_t i = 0; i < n && e == cudaSuccess; i++) {
+            size_t nd = 0;
+            e = cudaGraphNodeGetDependentNodes(nodes[i], nullptr, &nd);
+            if (e == cudaSuccess && nd == 0) deps.push_back(nodes[i]);
+        }
+        if (e == cudaSuccess && deps.size() != 1) e = cudaErrorInvalidValue;
+    }
     cudaGraphConditionalHandle h;
-    cudaError_t e = cudaGraphConditionalHandleCreate(&h, g, 1, cudaGraphCondAssignDefault);
+    if (e == cudaSuccess) e = cudaGraphConditionalHandleCreate(&h, g, 1, cudaGraphCondAssignDefault);
     cudaGraphNodeParams p = {};
     p.type = cudaGraphNodeTypeConditional;
     p.conditional.handle = h;
     p.conditional.type = cudaGraphCondTypeWhile;
     p.conditional.size = 1;
     cudaGraphNode_t node;
-    if (e == cudaSuccess) e = cudaGraphAddNode(&node, g, nullptr, 0, &p);
+    if (e == cudaSuccess) e = cudaGraphAddNode(&node, g, deps.data(), deps.size(), &p);
     if (e == cudaSuccess) {
         cudaGraph_t body = p.conditional.phGraph_out[0];
         e = cudaStreamBeginCaptureToGraph(op->cap_stream, body, nullptr, nullptr, 0,
@@ -530,8 +572,6 @@ static mas_status_t loop_graph(mas_op* op, StencilArgs a, StreamArgs b, AnisoArg
             a.cond = (unsigned long long)h;
             b.cond = (unsigned long long)h;
             an.cond = (unsigned long long)h;
-            const int nc = op->ncomp;
-            // iteration 1 runs before the loop (its own kernel-A instantiation);
             // the body covers an even and an odd iteration: k = 2, 3, 4, ...
             for (int kk = 2; kk <= 3 && e == cudaSuccess; kk++) {
                 a.pold = pold_halo(op, kk);
@@ -558,6 +598,7 @@ static mas_status_t loop_graph(mas_op* op, StencilArgs a, StreamArgs b, AnisoArg
     op->g_x = a.x;
     op->g_hist = a.rho_hist;
     op->g_aniso = op->aniso;
+    op->g_pre = (int)pre_plain;
     return MAS_OK;
 }
 
@@ -680,6 +721,8 @@ mas_status_t mas_op_setup(mas_grid_t* g, int ncomp, const double* kappa, const d
     G.vp = t;
     const char* g_env = getenv("MAS_NO_GRAPH");  // experiment hook: host-driven loop
     op->use_graph = !(g_env && atoi(g_env));
+    const char* gp_env = getenv("MAS_GRAPH_PRE");  // experiment hook (round-1 graph form)
+    op->graph_pre = gp_env && atoi(gp_env);
     const char* ch_env = getenv("MAS_CHUNK");  // experiment hook
     op->chunk = ch_env ? atoi(ch_env) : (nl >= 128 ? 32 : nl >= 64 ? 16 : (nl >= 16 ? 8 : 4));
     if (!ch_env && multi && nl >= 12) {
@@ -1212,16 +1255,19 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
     // (virtual P2P ranks share one GPU and need host ordering: comm_vsync)
     const bool graph = !op->prof && op->use_graph && (!comm || (p2p && !comm_is_virtual(comm)));
     if (graph) {
-        ST(loop_graph(op, a, b, an));
-        a.pold = pold_halo(op, 1);  // iteration 1 (not read)
-        a.tpold = pold_trows(op, 1);
-        a.pnew = op->p[1];
-        CU(launch_stencil(MODE_PCGA, nc, a, s, true));
-        if (op->aniso) {
-            an.u = aniso_p_halo(op, 1);
-            CU(launch_aniso(MODE_PCGA, an, s));
+        const bool pre = op->graph_pre != 0;
+        ST(loop_graph(op, a, b, an, pre));
+        if (pre) {
+            a.pold = pold_halo(op, 1);  // iteration 1 (not read)
+            a.tpold = pold_trows(op, 1);
+            a.pnew = op->p[1];
+            CU(launch_stencil(MODE_PCGA, nc, a, s, true));
+            if (op->aniso) {
+                an.u = aniso_p_halo(op, 1);
+                CU(launch_aniso(MODE_PCGA, an, s));
+            }
+            CU(launch_pcg_b(b, op->b_blocks, s));
         }
-        CU(launch_pcg_b(b, op->b_blocks, s));
         CU(cudaGraphLaunch(op->gexec, s));
     }
     int stop_seen_at = -1;

@@ -1066,13 +1066,12 @@ static cudaError_t launch_one(const StencilArgs& a0, cudaStream_t s) {
     a.ntk = (a.g.np + TK - 1) / TK;
     a.nchunk = (a.g.nl + a.chunk - 1) / a.chunk;
     const int smem = 4 * (NC + 1) * HROWS * ROW * (int)sizeof(double);
-    static bool attr_done = false;
-    if (!attr_done) {
-        cudaError_t e = cudaFuncSetAttribute(k_stencil<MODE, NC, FIRSTK>,
-                                             cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-        if (e != cudaSuccess) return e;
-        attr_done = true;
-    }
+    static DeviceOnce attr;
+    cudaError_t e = attr.run([&] {
+        return cudaFuncSetAttribute(k_stencil<MODE, NC, FIRSTK>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                    smem);
+    });
+    if (e != cudaSuccess) return e;
     const int T = a.ntj * a.ntk;
     const int blocks = a.part == 1 ? T * (a.nchunk - 2) : a.part == 2 ? 2 * T : T * a.nchunk;
     if (blocks <= 0) return cudaErrorInvalidValue;

@@ -4,6 +4,7 @@
 
 #include <cuda_runtime.h>
 
+#include <atomic>
 #include <cstdint>
 #include <string>
 
@@ -222,5 +223,35 @@ cudaError_t launch_aniso_diag(const Geo& g, const double* ca, const double* ca_h
                               double* dinv, int* bad, cudaStream_t s);
 
 void set_last_error(const std::string& msg);
+
+// Per-device one-time launch setup.  cudaFuncSetAttribute (the dynamic
+// shared-memory opt-in) is per device and virtual ranks launch from several
+// host threads: each call site keeps one bit per device in an atomic word
+// (setting the attribute twice is harmless; 64 devices per process).
+struct DeviceOnce {
+    std::atomic<unsigned long long> done{0};
+    template <class F>
+    cudaError_t run(F&& f) {
+        int dev = 0;
+        cudaError_t e = cudaGetDevice(&dev);
+        if (e != cudaSuccess) return e;
+        const unsigned long long bit = 1ull << (dev & 63);
+        if (done.load(std::memory_order_acquire) & bit) return cudaSuccess;
+        e = f();
+        if (e == cudaSuccess) done.fetch_or(bit, std::memory_order_acq_rel);
+        return e;
+    }
+};
+// SM count of the current device (cached per device, thread-safe)
+inline int device_sms() {
+    static std::atomic<int> cache[64];
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess) return 148;
+    int v = cache[dev & 63].load(std::memory_order_relaxed);
+    if (v > 0) return v;
+    if (cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || v <= 0) v = 148;
+    cache[dev & 63].store(v, std::memory_order_relaxed);
+    return v;
+}
 
 }  // namespace mas

@@ -104,19 +104,35 @@ def _check(s: int, where: str, ok=(MAS_OK,)) -> int:
 
 
 def _ptr(a) -> Optional[int]:
-    """Data pointer of a torch tensor or numpy array (must be contiguous fp64)."""
+    """Data pointer of a torch tensor or numpy array (must be contiguous fp64,
+    16-byte aligned: the kernels load double2 pairs and TMA boxes)."""
     if a is None:
         return None
     if isinstance(a, np.ndarray):
         if a.dtype != np.float64 or not a.flags.c_contiguous:
             raise TypeError("need C-contiguous float64 arrays")
-        return a.ctypes.data
-    import torch
-    if isinstance(a, torch.Tensor):
+        p = a.ctypes.data
+    else:
+        import torch
+        if not isinstance(a, torch.Tensor):
+            raise TypeError(f"unsupported array type {type(a)}")
         if a.dtype != torch.float64 or not a.is_contiguous():
             raise TypeError("need contiguous float64 tensors")
-        return a.data_ptr()
-    raise TypeError(f"unsupported array type {type(a)}")
+        p = a.data_ptr()
+    if p % 16:
+        raise ValueError("array data must be 16-byte aligned (a view with an odd element "
+                         "offset is not)")
+    return p
+
+
+def _numel(a) -> int:
+    return int(a.size) if isinstance(a, np.ndarray) else int(a.numel())
+
+
+def _expect(a, n: int, what: str) -> None:
+    """The C side reads exactly n doubles (the LOCAL block on this rank)."""
+    if a is not None and _numel(a) != n:
+        raise ValueError(f"{what}: {_numel(a)} elements, the local block needs {n}")
 
 
 def _stream(stream=None) -> Optional[int]:
@@ -269,8 +285,9 @@ def mas_op_kernel_times(op: int):
 
 
 def mas_op_set_aniso(op: int, kpar, bhat, stream=None) -> None:
-    """Field-aligned conduction term L_par (NEXT-4): kpar [nr,nt,np],
-    bhat [3,nr,nt,np] at the lower cell corners; kpar None switches it off."""
+    """Field-aligned conduction term L_par (NEXT-4): kpar [nl,nt,np] and
+    bhat [3,nl,nt,np] of the LOCAL r-slab at the lower cell corners (R25);
+    kpar None switches it off."""
     _check(lib().mas_op_set_aniso(op, _ptr(kpar), _ptr(bhat), _stream(stream)),
            "mas_op_set_aniso")
 
@@ -300,16 +317,16 @@ def mas_version() -> str:
 # ---------------------------------------------------------------------------
 class Grid:
     def __init__(self, mesh, dist=None, ptheta=1):
+        # the pole flags are the mesh's own declaration; mas_grid_create rejects
+        # a north flag with t_node[0] != 0 or a south flag with t_node[nt] != pi
+        # (MAS_ERR_ARG), nothing is dropped silently here
         flags = (MAS_POLE_NORTH if getattr(mesh, "pole_north", True) else 0) | \
                 (MAS_POLE_SOUTH if getattr(mesh, "pole_south", True) else 0)
-        if mesh.tF[0] != 0.0:
-            flags &= ~MAS_POLE_NORTH
-        if abs(mesh.tF[-1] - np.pi) > 1e-15:
-            flags &= ~MAS_POLE_SOUTH
         self.h = mas_grid_create(mesh.rF, mesh.rC, mesh.tF, mesh.tC, mesh.pF, mesh.pC, flags, 1,
                                  dist, ptheta)
         self.i0, self.nl, self.j0, self.ntl = mas_grid_local_extent_2d(self.h)
         self.shape = (len(mesh.rC), len(mesh.tC), len(mesh.pC))
+        self.local_cells = self.nl * self.ntl * self.shape[2]
 
     def close(self):
         if self.h:
@@ -324,27 +341,46 @@ class Grid:
 
 
 class Operator:
+    """Array arguments are the LOCAL block of this rank: [nl][ntl][np] for
+    per-cell coefficients, [ncomp][nl][ntl][np] for vectors."""
+
     def __init__(self, grid: Grid, ncomp, kappa, mass, bc_inner, bc_outer, stream=None):
         self.grid = grid
         self.ncomp = ncomp
+        self.N = grid.local_cells
+        _expect(kappa, self.N, "kappa")
+        _expect(mass, self.N, "mass")
         self.h = mas_op_setup(grid.h, ncomp, kappa, mass, bc_inner, bc_outer, stream)
 
     def update(self, kappa, mass, stream=None):
+        _expect(kappa, self.N, "kappa")
+        _expect(mass, self.N, "mass")
         mas_op_update(self.h, kappa, mass, stream)
 
     def apply(self, x, y, stream=None):
+        _expect(x, self.ncomp * self.N, "x")
+        _expect(y, self.ncomp * self.N, "y")
         mas_op_apply(self.h, x, y, stream)
 
     def diag(self, D, stream=None):
+        _expect(D, self.N, "D")
         mas_op_diag(self.h, D, stream)
 
     def dirichlet_rhs(self, ub_inner, ub_outer, f, stream=None):
+        nb = self.ncomp * self.grid.ntl * self.grid.shape[2]
+        _expect(ub_inner, nb, "ub_inner")
+        _expect(ub_outer, nb, "ub_outer")
+        _expect(f, self.ncomp * self.N, "f")
         mas_op_dirichlet_rhs(self.h, ub_inner, ub_outer, f, stream)
 
     def dot(self, a, b, stream=None):
+        _expect(a, self.ncomp * self.N, "a")
+        _expect(b, self.ncomp * self.N, "b")
         return mas_op_dot(self.h, a, b, stream)
 
     def solve(self, rhs, x, tol, maxit, want_hist=False, stream=None):
+        _expect(rhs, self.ncomp * self.N, "rhs")
+        _expect(x, self.ncomp * self.N, "x")
         return mas_pcg_solve(self.h, rhs, x, tol, maxit, want_hist, stream)
 
     def enable_p2p(self, stream=None):
@@ -361,12 +397,20 @@ class Operator:
         return mas_op_kernel_times(self.h)
 
     def set_aniso(self, kpar, bhat, stream=None):
+        """kpar [nl][nt][np] and bhat [3][nl][nt][np] (component-major): the
+        local r-slab, at the lower cell corners (R25)."""
+        _expect(kpar, self.N, "kpar")
+        if kpar is not None:
+            _expect(bhat, 3 * self.N, "bhat")
         mas_op_set_aniso(self.h, kpar, bhat, stream)
 
     def aniso_time(self):
         return mas_op_aniso_time(self.h)
 
     def radial_sums(self, x, w, out, stream=None):
+        _expect(x, self.ncomp * self.N, "x")
+        _expect(w, self.grid.ntl * self.grid.shape[2], "w")
+        _expect(out, self.ncomp * self.grid.nl, "out")
         mas_op_radial_sums(self.h, x, w, out, stream)
 
     @property

@@ -2,7 +2,9 @@
 """Summarise ncu output for profiles/ (run here, on the CPU box).
 
   python tools/ncu_summary.py launches <launches.csv>         # per-kernel share of the run
-  python tools/ncu_summary.py report <file.ncu-rep> [alg_bytes]  # key metrics of one capture
+  python tools/ncu_summary.py report <file.ncu-rep> [alg_bytes_per_cell cells]
+      # key metrics of one capture; traffic_over_alg = DRAM bytes of the launch
+      # / (alg_bytes_per_cell * cells of that launch)
 """
 import collections
 import csv
@@ -50,6 +52,8 @@ UNITS = {"dram__bytes_read.sum": "byte", "dram__bytes_write.sum": "byte"}
 
 
 def report(path, alg_bytes=None):
+    """alg_bytes: ALGORITHMIC bytes of the whole captured launch (per-cell
+    figure x cells), never a per-cell figure."""
     raw = subprocess.run(["ncu", "-i", path, "--page", "raw", "--csv"], capture_output=True,
                          text=True).stdout
     rows = list(csv.reader(io.StringIO(raw)))
@@ -80,8 +84,12 @@ def report(path, alg_bytes=None):
     if isinstance(rd, float) and isinstance(wr, float):
         out["dram_bytes_per_launch"] = rd + wr
         if alg_bytes:
+            ratio = (rd + wr) / alg_bytes
+            if not 0.05 < ratio < 20.0:
+                raise SystemExit(f"traffic/alg = {ratio:.3g}: alg_bytes must be per launch "
+                                 "(bytes per cell x cells), not per cell")
             out["alg_bytes_per_launch"] = alg_bytes
-            out["traffic_over_alg"] = (rd + wr) / alg_bytes
+            out["traffic_over_alg"] = ratio
     return out
 
 
@@ -89,5 +97,5 @@ if __name__ == "__main__":
     if sys.argv[1] == "launches":
         print(json.dumps(launches(sys.argv[2]), indent=1))
     else:
-        print(json.dumps(report(sys.argv[2], float(sys.argv[3]) if len(sys.argv) > 3 else None),
-                         indent=1))
+        alg = float(sys.argv[3]) * float(sys.argv[4]) if len(sys.argv) > 4 else None
+        print(json.dumps(report(sys.argv[2], alg), indent=1))
