@@ -258,6 +258,72 @@ def run_reference(args):
     return 0
 
 
+def volumes(mesh):
+    """V_P = rC^2 dr sin(tC) dt dp (the inner-product weight of R9), for the
+    bench's own x comparison."""
+    dr, dt, dp = np.diff(mesh.rF), np.diff(mesh.tF), np.diff(mesh.pF)
+    return (mesh.rC ** 2 * dr)[:, None, None] * (np.sin(mesh.tC) * dt)[None, :, None] * dp[None, None, :]
+
+
+def reference_solve(M, prob, rank, dev, tol):
+    """Rank 0: the same global problem on one GPU (no communicator)."""
+    import torch
+    g = M.Grid(prob.mesh)
+    d = lambda a: torch.from_numpy(np.ascontiguousarray(a)).to(dev)
+    o = M.Operator(g, prob.ncomp, d(prob.kappa), d(prob.c), prob.bc_inner, prob.bc_outer)
+    if prob.kpar is not None:
+        o.set_aniso(d(prob.kpar), d(prob.bhat))
+    f = d(prob.f)
+    if prob.ub_inner is not None or prob.ub_outer is not None:
+        o.dirichlet_rhs(None if prob.ub_inner is None else d(prob.ub_inner),
+                        None if prob.ub_outer is None else d(prob.ub_outer), f)
+    x = d(prob.x0)
+    st, it, rel, _ = o.solve(f, x, tol, 20000)
+    xr = x.cpu().numpy()
+    o.close()
+    g.close()
+    del x, f
+    torch.cuda.empty_cache()
+    return {"iters": it, "x": xr, "status": st}
+
+
+def check_parity(M, op, prob, x0, rhs, ref, extent, rank, world, dev, tol, dist):
+    """One solve on the multi-GPU op; gather x to rank 0 and compare with the
+    P = 1 reference (iterations +-1, x <= 1e-10 relative L2_V)."""
+    import torch
+    x = x0.clone()
+    st, it, rel, _ = op.solve(rhs, x, tol, 20000)
+    ext = [None] * world
+    dist.all_gather_object(ext, extent)
+    n = max(e[1] * e[3] for e in ext) * prob.shape[2] * prob.ncomp
+    buf = torch.zeros(n, device=dev, dtype=torch.float64)
+    buf[: x.numel()] = x.reshape(-1)
+    bufs = [torch.empty_like(buf) for _ in range(world)] if rank == 0 else None
+    dist.gather(buf, bufs, dst=0)
+    res = torch.zeros(3, device=dev, dtype=torch.float64)
+    if rank == 0:
+        xg = np.full((prob.ncomp,) + prob.shape, np.nan)
+        for b, (i0, nl, j0, ntl) in zip(bufs, ext):
+            blk = b[: prob.ncomp * nl * ntl * prob.shape[2]].cpu().numpy()
+            xg[:, i0:i0 + nl, j0:j0 + ntl] = blk.reshape(prob.ncomp, nl, ntl, prob.shape[2])
+        V = volumes(prob.mesh)[None]
+        xr = ref["x"]
+        err = float(np.sqrt((V * (xg - xr) ** 2).sum() / (V * xr ** 2).sum()))
+        res[0], res[1], res[2] = err, ref["iters"], float(np.isnan(xg).any())
+    dist.broadcast(res, src=0)
+    err, it_ref, nan = float(res[0]), int(res[1]), bool(res[2])
+    its = torch.tensor([it], device=dev, dtype=torch.float64)
+    lo, hi = its.clone(), its.clone()
+    dist.all_reduce(lo, op=dist.ReduceOp.MIN)
+    dist.all_reduce(hi, op=dist.ReduceOp.MAX)
+    ok = (st == M.MAS_OK and not nan and lo.item() == hi.item() and abs(it - it_ref) <= 1
+          and err <= 1e-10)
+    okt = torch.tensor([1.0 if ok else 0.0], device=dev, dtype=torch.float64)
+    dist.all_reduce(okt, op=dist.ReduceOp.MIN)
+    return {"ok": bool(okt.item() == 1.0), "iters": it, "iters_p1": it_ref, "x_rel_l2_V_vs_p1": err,
+            "bound": "iters +-1, x <= 1e-10 (north_star)"}
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -316,30 +382,54 @@ def main():
     f = to_dev(prob.f[slc])
     x0 = to_dev(prob.x0[slc])
     x = x0.clone()
-    op = M.Operator(grid, nc, kappa, cmass, prob.bc_inner, prob.bc_outer)
     aniso = prob.kpar is not None
     if aniso:  # NEXT-4 (r-slabs; either transport)
         if args.ptheta != 1:
             raise SystemExit("C2a (field-aligned conduction) needs r-slabs (--ptheta 1)")
         kpar = to_dev(prob.kpar[sl])
         bhat = to_dev(prob.bhat[(slice(None),) + sl])
-        op.set_aniso(kpar, bhat)
-    transport = "single-gpu"
-    if world > 1:
-        transport = "nccl"
-        if args.transport != "nccl":
-            try:
-                op.enable_p2p()
-                transport = "p2p"
-            except M.MasError as e:  # collective verdict: every rank keeps NCCL
-                if args.transport == "p2p":
-                    raise
-                transport = f"nccl (p2p unavailable: {e})"
+
+    def make_op(use_p2p):
+        o = M.Operator(grid, nc, kappa, cmass, prob.bc_inner, prob.bc_outer)
+        if aniso:
+            o.set_aniso(kpar, bhat)
+        tr = "single-gpu"
+        if world > 1:
+            tr = "nccl"
+            if use_p2p:
+                try:
+                    o.enable_p2p()
+                    tr = "p2p"
+                except M.MasError as e:  # collective verdict: every rank keeps NCCL
+                    if args.transport == "p2p":
+                        raise
+                    tr = f"nccl (p2p unavailable: {e})"
+        return o, tr
+
+    op, transport = make_op(args.transport != "nccl")
     ubi = to_dev(prob.ub_inner[:, j0:j0 + ntl]) if prob.ub_inner is not None else None
     ubo = to_dev(prob.ub_outer[:, j0:j0 + ntl]) if prob.ub_outer is not None else None
     rhs = f.clone()
     if ubi is not None or ubo is not None:
         op.dirichlet_rhs(ubi, ubo, rhs)
+
+    # N > 1: self-check before timing.  Rank 0 solves the same global problem
+    # on its own GPU (P = 1); every rank's slab of x is gathered and compared
+    # (north_star: iterations +-1, x <= 1e-10 relative L2_V).  If the P2P
+    # transport fails the check, the op falls back to NCCL and is re-checked.
+    parity = None
+    if world > 1:
+        ref = reference_solve(M, prob, rank, dev, args.tol) if rank == 0 else None
+        parity = check_parity(M, op, prob, x0, rhs, ref, (i0, nl, j0, ntl), rank, world, dev,
+                              args.tol, dist)
+        if not parity["ok"] and transport == "p2p" and args.transport == "auto":
+            op.close()
+            op, transport = make_op(False)
+            parity = check_parity(M, op, prob, x0, rhs, ref, (i0, nl, j0, ntl), rank, world, dev,
+                                  args.tol, dist)
+            parity["fallback"] = "p2p failed the P=1 check; NCCL transport used"
+        if not parity["ok"]:
+            raise SystemExit(f"multi-GPU result differs from the P=1 solve: {parity}")
     stream = torch.cuda.current_stream()
     maxit = 20000
 
@@ -399,6 +489,19 @@ def main():
     torch.cuda.synchronize()
     op.set_profiling(False)
     t_prof_ms = e2.elapsed_time(e3)
+    comm = None
+    if world > 1:  # the exchange steps of the NCCL loop, measured on this op (collective)
+        seam_us, ar_us, seam_b = op.comm_bench(20)
+        mx = torch.tensor([seam_us, ar_us, seam_b], device=dev, dtype=torch.float64)
+        dist.all_reduce(mx, op=dist.ReduceOp.MAX)
+        seam_us, ar_us, seam_b = (float(v) for v in mx.tolist())
+        comm = {"seam_bytes_per_iter_max_rank": seam_b, "seam_us": seam_us,
+                "seam_GBs": seam_b / (seam_us * 1e3) if seam_us > 0 else None,
+                "seam_frac_of_nvlink_900GBs": (seam_b / (seam_us * 1e3) / 900.0) if seam_us > 0 else None,
+                "allreduce_2dbl_us": ar_us,
+                "note": "NCCL grouped send/recv of the r and p edge planes and a 2-double "
+                        "ncclAllReduce, max over ranks (mas_op_comm_bench); the P2P transport "
+                        "reads the same planes in place inside kernel A"}
     iters_per_solve = iters_total / args.steps
     value = iters_total / (t_ms / 1e3)  # the solve is one global problem: iterations are shared
 
@@ -521,6 +624,7 @@ def main():
                         "iter_alg_GBs": iter_gbs, "iter_frac": iter_gbs / peak,
                         "alg_bytes_per_cell_iter": a_b + b_b + c_b},
             "e2e": e2e,
+            **({"parity": parity, "comm": comm} if world > 1 else {}),
             "gpu_launches": launches,
             "clocks": clk,
             "cpu_baseline": cpu,

@@ -70,7 +70,12 @@ enum { MAS_POLE_NORTH = 1, MAS_POLE_SOUTH = 2 };
 
 /* Multi-GPU description.  NULL => single GPU.  nccl_id: 128 bytes from
  * mas_comm_unique_id() on rank 0, broadcast by the caller (e.g. with
- * torch.distributed).  The current CUDA device is used. */
+ * torch.distributed).  The current CUDA device is used.  nranks == 1 with a
+ * real id creates a 1-rank NCCL communicator: the op then runs the
+ * multi-GPU (NCCL) iteration loop on one GPU (the NCCL code path's check).
+ * NCCL waits inside mas_pcg_solve poll ncclCommGetAsyncError and give up
+ * after MAS_COMM_TIMEOUT_S seconds (default 600): the communicators are
+ * aborted and MAS_ERR_NCCL returned instead of hanging. */
 typedef struct {
     int nranks;
     int rank;
@@ -208,6 +213,19 @@ MAS_API mas_status_t mas_op_enable_p2p(mas_op_t* op, cudaStream_t stream);
 
 /* Transport of the op's PCG loop: 0 NCCL (or one GPU), 1 P2P; -1 if op is NULL. */
 MAS_API int mas_op_transport(const mas_op_t* op);
+
+/* Collective measurement of the NCCL loop's exchange steps on this op
+ * (SURVEY.md §8(d) "seam bytes / seam time vs 900 GB/s; allreduce latency"):
+ * reps rounds of the per-iteration seams (the r and p edge planes to the
+ * r-neighbours, grouped ncclSend/ncclRecv) and reps 2-double ncclAllReduce,
+ * timed with CUDA events on the stream.  seam_us / allreduce_us: average per
+ * round; seam_bytes: bytes this rank sends + receives per round.  Without a
+ * communicator all three are 0.  The op's r / p contents are clobbered
+ * (call it outside a solve).  Errors: MAS_ERR_ARG (reps < 1, null pointers),
+ * MAS_ERR_NCCL, MAS_ERR_CUDA. */
+MAS_API mas_status_t mas_op_comm_bench(mas_op_t* op, int reps, double* seam_us,
+                                       double* allreduce_us, double* seam_bytes,
+                                       cudaStream_t stream);
 
 /* Kernel launches issued by the last mas_pcg_solve on this op (its CUDA path
  * evidence; includes early-exit launches after convergence). */

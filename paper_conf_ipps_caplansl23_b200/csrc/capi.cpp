@@ -239,7 +239,7 @@ mas_status_t mas_grid_create_2d(int nr, int nt, int np, const double* r_node, co
         set_last_error("cudaMemcpy tables");
         return MAS_ERR_CUDA;
     }
-    if (dist && nranks > 1) {
+    if (dist) {  // nranks == 1 with a real NCCL id: a 1-rank communicator (the NCCL loop on one GPU)
         s = comm_create(dist, &g->comm);
         if (s != MAS_OK) { cudaFree(g->d_tab); delete g; return s; }
     }
@@ -1019,6 +1019,46 @@ mas_status_t mas_op_enable_p2p(mas_op_t* op, cudaStream_t s) {
 
 int mas_op_transport(const mas_op_t* op) { return !op ? -1 : op->p2p ? 1 : 0; }
 
+mas_status_t mas_op_comm_bench(mas_op_t* op, int reps, double* seam_us, double* allreduce_us,
+                               double* seam_bytes, cudaStream_t s) {
+    if (!op || !seam_us || !allreduce_us || !seam_bytes || reps < 1) return arg_error("bad argument");
+    Comm* comm = op->g->comm;
+    const int nc = op->ncomp;
+    const long long plane = op->geo.plane;
+    const int pt = op->g->ptheta;
+    const int nb = (comm_rank(comm) - pt >= 0) + (comm_rank(comm) + pt < comm_nranks(comm));
+    *seam_bytes = comm ? 2.0 * nb * 2.0 * nc * plane * sizeof(double) : 0.0;  // r and p, sent + received
+    *seam_us = *allreduce_us = 0.0;
+    if (!comm) return MAS_OK;
+    cudaEvent_t e0, e1;
+    CU(cudaEventCreate(&e0));
+    CU(cudaEventCreate(&e1));
+    float ms = 0.f;
+    mas_status_t st = MAS_OK;
+    // the per-iteration seams of the NCCL loop: r and p_{k-1} edge planes (r-slabs)
+    ST(comm_seams(comm, op->r, nc, op->g->nl, plane, op->rg, op->rg + nc * plane, s, rstride(op)));
+    CU(cudaEventRecord(e0, s));
+    for (int i = 0; i < reps && st == MAS_OK; i++) {
+        st = comm_seams(comm, op->r, nc, op->g->nl, plane, op->rg, op->rg + nc * plane, s, rstride(op));
+        if (st == MAS_OK)
+            st = comm_seams(comm, op->p[0], nc, op->g->nl, plane, op->pg[0], op->pg[0] + nc * plane, s,
+                            rstride(op));
+    }
+    CU(cudaEventRecord(e1, s));
+    if (st == MAS_OK) st = comm_sync_stream(comm, s);
+    if (st == MAS_OK && cudaEventElapsedTime(&ms, e0, e1) == cudaSuccess) *seam_us = 1e3 * ms / reps;
+    // the 2-double allreduce of kernel B's (rho, ||r||^2)
+    CU(cudaMemsetAsync(op->scr.partials, 0, 2 * sizeof(double), s));
+    CU(cudaEventRecord(e0, s));
+    for (int i = 0; i < reps && st == MAS_OK; i++) st = comm_allreduce(comm, op->scr.partials, 2, s);
+    CU(cudaEventRecord(e1, s));
+    if (st == MAS_OK) st = comm_sync_stream(comm, s);
+    if (st == MAS_OK && cudaEventElapsedTime(&ms, e0, e1) == cudaSuccess) *allreduce_us = 1e3 * ms / reps;
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    return st;
+}
+
 long long mas_op_launch_count(const mas_op_t* op) { return op ? op->launches : -1; }
 
 mas_status_t mas_op_set_profiling(mas_op_t* op, int on) {
@@ -1355,7 +1395,7 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
             // wait for iteration k-1 to finish, then stop if the device
             // decided at or before iteration k-1 (every rank sees the same
             // decision at the same point, so the collectives stay matched)
-            CU(cudaEventSynchronize(op->ev[(k - 1) & 1]));
+            ST(comm_wait_event(comm, op->ev[(k - 1) & 1]));
             const int flag = *(volatile int*)op->host_flag;
             if (flag > 0 && flag <= k - 1) {
                 stop_seen_at = k;
@@ -1364,7 +1404,7 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
         }
     }
     (void)stop_seen_at;
-    CU(cudaStreamSynchronize(s));
+    ST(comm_sync_stream(comm, s));
     // P2P: no rank may publish the next solve's partials while another rank's
     // kernels of this solve can still read its mailbox
     if (p2p && comm) ST(comm_barrier(comm, s));

@@ -17,6 +17,7 @@
 #include <nccl.h>
 
 #include <chrono>
+#include <cstdlib>
 #include <condition_variable>
 #include <cstdio>
 #include <thread>
@@ -360,7 +361,9 @@ static mas_status_t v_allreduce(Comm* c, double* buf, int n, cudaStream_t s) {
 }
 
 mas_status_t comm_allreduce(Comm* c, double* buf, int n, cudaStream_t s) {
-    if (!c || c->nranks == 1) return MAS_OK;
+    // a 1-rank NCCL communicator still runs ncclAllReduce (the NCCL code path
+    // on one GPU, mas_grid_create with a 1-rank mas_dist_t)
+    if (!c || (c->nranks == 1 && !c->nccl)) return MAS_OK;
     if (c->vg) return v_allreduce(c, buf, n, s);
     if (!c->hdir.empty()) return h_allreduce(c, buf, n, s);
     ncclResult_t r = ncclAllReduce(buf, buf, n, ncclFloat64, ncclSum, c->nccl, s);
@@ -485,6 +488,76 @@ mas_status_t comm_exchange(Comm* c, int lo, int hi, const double* send_lo, const
 // setup-time helpers of the P2P transport
 // ---------------------------------------------------------------------------
 bool comm_is_virtual(const Comm* c) { return c && c->vg; }
+bool comm_is_nccl(const Comm* c) { return c && c->nccl; }
+
+// ---------------------------------------------------------------------------
+// waiting on the NCCL loop without hanging: poll the event, and between polls
+// the communicators' asynchronous error state (a peer that died or a network
+// error); on an error or after the timeout (MAS_COMM_TIMEOUT_S, default 600 s)
+// both communicators are aborted and MAS_ERR_NCCL is returned.
+// ---------------------------------------------------------------------------
+static double comm_timeout_s() {
+    static const double t = [] {
+        const char* e = getenv("MAS_COMM_TIMEOUT_S");
+        const double v = e ? atof(e) : 600.0;
+        return v > 0 ? v : 600.0;
+    }();
+    return t;
+}
+
+static mas_status_t comm_abort(Comm* c, const std::string& why) {
+    if (c->nccl_seam) ncclCommAbort(c->nccl_seam);
+    if (c->nccl) ncclCommAbort(c->nccl);
+    c->nccl_seam = c->nccl = nullptr;
+    set_last_error(why);
+    return MAS_ERR_NCCL;
+}
+
+mas_status_t comm_check_async(Comm* c) {
+    if (!c || !c->nccl) return MAS_OK;
+    for (ncclComm_t cm : {c->nccl, c->nccl_seam}) {
+        ncclResult_t ar = ncclSuccess;
+        if (cm && ncclCommGetAsyncError(cm, &ar) == ncclSuccess && ar != ncclSuccess && ar != ncclInProgress)
+            return comm_abort(c, std::string("NCCL asynchronous error: ") + ncclGetErrorString(ar));
+    }
+    return MAS_OK;
+}
+
+mas_status_t comm_wait_event(Comm* c, cudaEvent_t ev) {
+    if (!c || !c->nccl) {
+        cudaError_t e = cudaEventSynchronize(ev);
+        return e == cudaSuccess ? MAS_OK : cuda_fail(e, "cudaEventSynchronize");
+    }
+    const auto t0 = std::chrono::steady_clock::now();
+    for (unsigned n = 0;; n++) {
+        cudaError_t e = cudaEventQuery(ev);
+        if (e == cudaSuccess) return MAS_OK;
+        if (e != cudaErrorNotReady) return cuda_fail(e, "cudaEventQuery");
+        if ((n & 63) == 63) {
+            mas_status_t st = comm_check_async(c);
+            if (st != MAS_OK) return st;
+            const double dt = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
+            if (dt > comm_timeout_s())
+                return comm_abort(c, "NCCL loop: no progress for " + std::to_string((int)dt) +
+                                         " s (MAS_COMM_TIMEOUT_S); communicators aborted");
+        }
+        std::this_thread::yield();
+    }
+}
+
+mas_status_t comm_sync_stream(Comm* c, cudaStream_t s) {
+    if (!c || !c->nccl) {
+        cudaError_t e = cudaStreamSynchronize(s);
+        return e == cudaSuccess ? MAS_OK : cuda_fail(e, "cudaStreamSynchronize");
+    }
+    cudaEvent_t ev;
+    cudaError_t e = cudaEventCreateWithFlags(&ev, cudaEventDisableTiming);
+    if (e == cudaSuccess) e = cudaEventRecord(ev, s);
+    if (e != cudaSuccess) return cuda_fail(e, "comm_sync_stream");
+    mas_status_t st = comm_wait_event(c, ev);
+    cudaEventDestroy(ev);
+    return st;
+}
 int comm_rank(const Comm* c) { return c ? c->rank : 0; }
 int comm_nranks(const Comm* c) { return c ? c->nranks : 1; }
 

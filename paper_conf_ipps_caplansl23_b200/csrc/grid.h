@@ -57,6 +57,12 @@ mas_status_t comm_exchange(Comm* c, int lo, int hi, const double* send_lo, const
 mas_status_t comm_barrier(Comm* c, cudaStream_t s);
 // P2P transport setup helpers
 bool comm_is_virtual(const Comm* c);
+bool comm_is_nccl(const Comm* c);
+// NCCL loop waits: poll the event / stream and ncclCommGetAsyncError, abort
+// the communicators on an error or after MAS_COMM_TIMEOUT_S (default 600 s)
+mas_status_t comm_check_async(Comm* c);
+mas_status_t comm_wait_event(Comm* c, cudaEvent_t ev);
+mas_status_t comm_sync_stream(Comm* c, cudaStream_t s);
 int comm_rank(const Comm* c);
 int comm_nranks(const Comm* c);
 mas_status_t comm_allgather_bytes(Comm* c, const void* mine, void* all, size_t n, cudaStream_t s);

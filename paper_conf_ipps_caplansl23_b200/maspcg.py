@@ -28,7 +28,7 @@ ABI_SYMBOLS = ("mas_comm_unique_id", "mas_partition", "mas_grid_create", "mas_gr
                "mas_op_transport", "mas_op_launch_count", "mas_grid_create_2d",
                "mas_grid_local_extent_2d",
                "mas_op_set_profiling", "mas_op_kernel_times", "mas_op_set_aniso",
-               "mas_op_aniso_time", "mas_op_radial_sums", "mas_op_destroy", "mas_status_string", "mas_last_error", "mas_version")
+               "mas_op_aniso_time", "mas_op_radial_sums", "mas_op_comm_bench", "mas_op_destroy", "mas_status_string", "mas_last_error", "mas_version")
 
 
 class MasError(RuntimeError):
@@ -77,6 +77,7 @@ def lib() -> C.CDLL:
             "mas_op_set_aniso": (_i, [_vp, _vp, _vp, _vp]),
             "mas_op_aniso_time": (_i, [_vp, _vp]),
             "mas_op_radial_sums": (_i, [_vp, _vp, _vp, _vp, _vp]),
+            "mas_op_comm_bench": (_i, [_vp, _i, _vp, _vp, _vp, _vp]),
             "mas_op_destroy": (_i, [_vp]),
             "mas_status_string": (C.c_char_p, [_i]),
             "mas_last_error": (C.c_char_p, []),
@@ -304,6 +305,15 @@ def mas_op_radial_sums(op: int, x, w, out, stream=None) -> None:
            "mas_op_radial_sums")
 
 
+def mas_op_comm_bench(op: int, reps: int = 20, stream=None):
+    """(seam_us, allreduce_us, seam_bytes) per round of the NCCL loop's
+    exchange steps on this op (collective)."""
+    a, b, c = C.c_double(), C.c_double(), C.c_double()
+    _check(lib().mas_op_comm_bench(op, int(reps), C.byref(a), C.byref(b), C.byref(c), _stream(stream)),
+           "mas_op_comm_bench")
+    return a.value, b.value, c.value
+
+
 def mas_op_destroy(op: int) -> None:
     _check(lib().mas_op_destroy(op), "mas_op_destroy")
 
@@ -403,6 +413,9 @@ class Operator:
         if kpar is not None:
             _expect(bhat, 3 * self.N, "bhat")
         mas_op_set_aniso(self.h, kpar, bhat, stream)
+
+    def comm_bench(self, reps=20, stream=None):
+        return mas_op_comm_bench(self.h, reps, stream)
 
     def aniso_time(self):
         return mas_op_aniso_time(self.h)
