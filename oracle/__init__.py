@@ -237,16 +237,39 @@ class Oracle:
         return rc, x, iters.value, relres.value, hist[: iters.value + 1]
 
 
+    def pcg_cg1(self, kappa, c, f, x0, tol, maxit):
+        """Single-reduction (Chronopoulos-Gear) PCG, NEXT-1 / R28.
+        Returns (status, x, iters, relres, res_hist)."""
+        f = _f64(f)
+        x = _f64(x0).copy()
+        ncomp = f.size // self.N
+        kappa, c = _f64(kappa), _f64(c)
+        iters, relres = C.c_int(), C.c_double()
+        hist = np.zeros(maxit + 1)
+        rc = lib().mas_ref_pcg_solve_cg1(C.byref(self.g), ncomp, _p(kappa), _p(c), _p(f), _p(x),
+                                         C.c_double(tol), maxit, C.byref(iters), C.byref(relres),
+                                         _p(hist))
+        self._chk(rc)
+        return rc, x, iters.value, relres.value, hist[: iters.value + 1]
+
+
 def partition(nr: int, nranks: int, rank: int):
     i0, nl = C.c_int(), C.c_int()
     lib().mas_ref_partition(nr, nranks, rank, C.byref(i0), C.byref(nl))
     return i0.value, nl.value
 
 
-def solve_problem(prob, tol=None, maxit=None, x0=None, threads: int = 0, nranks: int = 0):
-    """Full oracle solve of a workloads.Problem: rhs = f + Dirichlet terms."""
+def solve_problem(prob, tol=None, maxit=None, x0=None, threads: int = 0, nranks: int = 0,
+                  cg1: bool = False):
+    """Full oracle solve of a workloads.Problem: rhs = f + Dirichlet terms.
+    cg1: the single-reduction (Chronopoulos-Gear) PCG of NEXT-1."""
     o = Oracle.for_problem(prob, threads)
     f = o.dirichlet_rhs(prob.kappa, prob.f, prob.ub_inner, prob.ub_outer)
+    if cg1:
+        if prob.kpar is not None or nranks:
+            raise ValueError("cg1: isotropic operator, one rank")
+        return o.pcg_cg1(prob.kappa, prob.c, f, prob.x0 if x0 is None else x0,
+                         prob.tol if tol is None else tol, prob.maxit if maxit is None else maxit)
     if prob.kpar is not None:  # field-aligned conduction (NEXT-4)
         return o.pcg_aniso(prob.kappa, prob.c, prob.kpar, prob.bhat, f,
                            prob.x0 if x0 is None else x0, prob.tol if tol is None else tol,

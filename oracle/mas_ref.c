@@ -978,3 +978,106 @@ int mas_ref_radial_sums(const mas_ref_grid* g, int ncomp, const double* x, const
         }
     return MAS_REF_OK;
 }
+
+/* ---------------------------------------------------------------------------
+ * Single-reduction PCG: the Chronopoulos-Gear
+ * rearrangement of the same Jacobi-PCG, in which the two inner products of
+ * an iteration (<r,z> and the curvature <Lz,z>) come from ONE reduction, so a
+ * distributed solve needs one allreduce per iteration instead of two (the
+ * paper's async / fusion lesson; its solver is
+ * "Krylov", without further detail).  Reading R28:
+ * Chronopoulos & Gear (1989), preconditioned form, with u = D^-1 r:
+ *
+ *   r0 = f - L x0;  u0 = D^-1 r0;  w0 = L u0;  g0 = <r0,u0>;  d0 = <w0,u0>
+ *   a0 = g0 / d0;  p0 = u0;  s0 = w0
+ *   for k = 1, 2, ...:
+ *       x_k = x_{k-1} + a_{k-1} p_{k-1};  r_k = r_{k-1} - a_{k-1} s_{k-1}
+ *       stop if ||r_k||_V <= tol ||f||_V   (R10; iters = k, R11: k products)
+ *       u_k = D^-1 r_k;  w_k = L u_k
+ *       g_k = <r_k,u_k>;  d_k = <w_k,u_k>          (one reduction: + ||r_k||^2)
+ *       b_k = g_k / g_{k-1};  a_k = g_k / (d_k - b_k g_k / a_{k-1})
+ *       p_k = u_k + b_k p_{k-1};  s_k = w_k + b_k s_{k-1}   (s_k = L p_k)
+ *
+ * In exact arithmetic x_k, r_k equal the standard PCG iterates (pcg_core).
+ * The denominator d_k - b_k g_k / a_{k-1} equals <p_k, L p_k>: !(> 0) is a
+ * breakdown (iters = k, x = x_k).  The residual ||r_k|| needed for the stop
+ * is the recursive one, as in pcg_core.
+ * ------------------------------------------------------------------------- */
+int mas_ref_pcg_solve_cg1(const mas_ref_grid* g, int ncomp, const double* kappa,
+                          const double* c, const double* f, double* x, double tol,
+                          int maxit, int* iters, double* relres, double* res_hist) {
+    tables T;
+    size_t N, n, e;
+    double *D, *r, *u, *w, *p, *s;
+    double bn, rn, gam, del, alpha, beta, gam_new, den;
+    int k, status = MAS_REF_NOT_CONVERGED, m;
+    if (!g || !kappa || !f || !x || !iters || !relres || ncomp < 1 || maxit < 0 ||
+        !(tol >= 0.0) || tables_make(g, &T))
+        return MAS_REF_ERR_ARG;
+    N = (size_t)g->nr * g->nt * g->np;
+    n = N * ncomp;
+    D = malloc(sizeof(double) * N);
+    r = malloc(sizeof(double) * n);
+    u = malloc(sizeof(double) * n);
+    w = malloc(sizeof(double) * n);
+    p = malloc(sizeof(double) * n);
+    s = malloc(sizeof(double) * n);
+    if (!D || !r || !u || !w || !p || !s) { status = MAS_REF_ERR_ARG; goto done; }
+    mas_ref_op_diag(g, kappa, c, D);
+
+    bn = sqrt(dot_planes(g, &T, 0, g->nr, ncomp, f, f));
+    if (bn == 0.0) {
+        for (e = 0; e < n; e++) x[e] = 0.0;
+        *iters = 0; *relres = 0.0;
+        if (res_hist) res_hist[0] = 0.0;
+        status = MAS_REF_OK; goto done;
+    }
+    mas_ref_op_apply(g, ncomp, kappa, c, x, r);                  /* r = L x       */
+#pragma omp parallel for schedule(static)
+    for (e = 0; e < n; e++) r[e] = f[e] - r[e];                  /* r0 = f - L x0 */
+    rn = sqrt(dot_planes(g, &T, 0, g->nr, ncomp, r, r));
+    if (res_hist) res_hist[0] = rn;
+    if (rn <= tol * bn) { *iters = 0; *relres = rn / bn; status = MAS_REF_OK; goto done; }
+    if (maxit == 0) { *iters = 0; *relres = rn / bn; status = MAS_REF_NOT_CONVERGED; goto done; }
+    for (m = 0; m < ncomp; m++)
+#pragma omp parallel for schedule(static)
+        for (e = 0; e < N; e++) u[m * N + e] = r[m * N + e] / D[e];   /* u0 = D^-1 r0 */
+    mas_ref_op_apply(g, ncomp, kappa, c, u, w);                  /* w0 = L u0     */
+    gam = dot_planes(g, &T, 0, g->nr, ncomp, r, u);
+    del = dot_planes(g, &T, 0, g->nr, ncomp, w, u);
+    if (!(del > 0.0) || !isfinite(del)) {
+        *iters = 1; *relres = rn / bn; status = MAS_REF_ERR_BREAKDOWN; goto done;
+    }
+    alpha = gam / del;
+    memcpy(p, u, sizeof(double) * n);                            /* p0 = u0       */
+    memcpy(s, w, sizeof(double) * n);                            /* s0 = w0       */
+
+    for (k = 1; k <= maxit; k++) {
+#pragma omp parallel for schedule(static)
+        for (e = 0; e < n; e++) { x[e] += alpha * p[e]; r[e] -= alpha * s[e]; }
+        rn = sqrt(dot_planes(g, &T, 0, g->nr, ncomp, r, r));
+        if (res_hist) res_hist[k] = rn;
+        if (rn <= tol * bn) { *iters = k; *relres = rn / bn; status = MAS_REF_OK; goto done; }
+        if (k == maxit) break;
+        for (m = 0; m < ncomp; m++)
+#pragma omp parallel for schedule(static)
+            for (e = 0; e < N; e++) u[m * N + e] = r[m * N + e] / D[e];
+        mas_ref_op_apply(g, ncomp, kappa, c, u, w);              /* w = L u       */
+        gam_new = dot_planes(g, &T, 0, g->nr, ncomp, r, u);
+        del = dot_planes(g, &T, 0, g->nr, ncomp, w, u);
+        beta = gam_new / gam;
+        gam = gam_new;
+        den = del - beta * gam / alpha;                          /* = <p, L p>    */
+        if (!(den > 0.0) || !isfinite(den)) {
+            *iters = k; *relres = rn / bn; status = MAS_REF_ERR_BREAKDOWN; goto done;
+        }
+        alpha = gam / den;
+#pragma omp parallel for schedule(static)
+        for (e = 0; e < n; e++) { p[e] = u[e] + beta * p[e]; s[e] = w[e] + beta * s[e]; }
+    }
+    *iters = maxit; *relres = rn / bn; status = MAS_REF_NOT_CONVERGED;
+done:
+    free(D); free(r); free(u); free(w); free(p); free(s);
+    tables_free(&T);
+    return status;
+}

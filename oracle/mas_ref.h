@@ -75,6 +75,14 @@ int mas_ref_pcg_solve(const mas_ref_grid* g, int ncomp, const double* kappa,
                       const double* c, const double* f, double* x, double tol,
                       int maxit, int* iters, double* relres, double* res_hist);
 
+/* Single-reduction PCG (NEXT-1, reading R28): the Chronopoulos-Gear form of
+ * the same Jacobi-PCG (one inner-product reduction per iteration); same
+ * arguments, stopping rule and counting as mas_ref_pcg_solve (iters = index
+ * of the residual that met tol = number of L products). */
+int mas_ref_pcg_solve_cg1(const mas_ref_grid* g, int ncomp, const double* kappa,
+                          const double* c, const double* f, double* x, double tol,
+                          int maxit, int* iters, double* relres, double* res_hist);
+
 /* Slab-local operator for a rank owning r-planes [i0, i0+nl) of the global
  * grid g.  kappa_ext and x_ext hold nl+2 planes per component: plane 0 is the
  * ghost copy of global plane i0-1, plane nl+1 of i0+nl (ignored at a global
