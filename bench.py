@@ -63,6 +63,12 @@ def alg_bytes_per_cell(ncomp):
     return a, b
 
 
+# single-reduction PCG (NEXT-1, --solver cg1): one kernel per iteration reads
+# r, w, s, p, x (ncomp each) + dinv, kappa, c and writes s, r, p, x, w
+def cg1_bytes_per_cell(ncomp):
+    return 8 * (5 * ncomp + 3 + 5 * ncomp)
+
+
 # the L_par kernel (NEXT-4, scalar): reads p_k and the 3 corner coefficients,
 # reads and writes q
 ANISO_BYTES_PER_CELL = 8 * (1 + 3 + 2)
@@ -335,6 +341,10 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--cpu-iters", type=int, default=3)
+    ap.add_argument("--solver", default="pcg", choices=["pcg", "cg1"],
+                    help="pcg: two fused kernels / two reductions per iteration; cg1: the "
+                         "single-reduction (Chronopoulos-Gear) loop, one kernel per iteration "
+                         "(NEXT-1, one GPU)")
     ap.add_argument("--ptheta", type=int, default=1,
                     help="(r, theta) decomposition: theta bands per r-slab (must divide --gpus)")
     ap.add_argument("--transport", default="auto", choices=["auto", "p2p", "nccl"],
@@ -393,6 +403,8 @@ def main():
         o = M.Operator(grid, nc, kappa, cmass, prob.bc_inner, prob.bc_outer)
         if aniso:
             o.set_aniso(kpar, bhat)
+        if args.solver == "cg1":
+            o.set_single_reduction(True)
         tr = "single-gpu"
         if world > 1:
             tr = "nccl"
@@ -510,6 +522,8 @@ def main():
     cells = nr * nt * np_
     cells_local = nl * ntl * np_
     a_b, b_b = alg_bytes_per_cell(nc)
+    if args.solver == "cg1":  # one kernel per iteration (kernel_times' A), no kernel B
+        a_b, b_b = cg1_bytes_per_cell(nc), 0
     a_ms = statistics.mean(ka)
     b_ms = statistics.mean(kb)
     peak, peak_src = load_peaks()
@@ -520,6 +534,7 @@ def main():
     traffic = None
     # the dominant kernel by device time: kernel A, or on C2a the L_par kernel
     dom = ("k_aniso<PCGA> (L_par)", c_b, c_ms, "kaniso") if aniso and c_ms > a_ms else \
+        ("k_stencil<CG1> (single-reduction iteration)", a_b, a_ms, "cg1") if args.solver == "cg1" else \
         ("k_stencil<PCGA> (kernel A)", a_b, a_ms, "kernelA")
     dom_achieved = dom[1] * cells_local / (dom[2] / 1e3) / 1e9
     prof_json = os.path.join(ROOT, "profiles", f"ncu_{args.config}_{dom[3]}.json")
@@ -605,6 +620,7 @@ def main():
                        "parallelism": (f"r-slab x{world}" if args.ptheta == 1 or world == 1 else
                                        f"(r,theta) {world // args.ptheta}x{args.ptheta}"),
                        "transport": transport,
+                       "solver": args.solver,
                        "l2": (f"no flush: one iteration streams {(a_b + b_b + c_b) * cells_local / 1e6:.0f}"
                               f" MB ({8 * cells_local / 1e6:.0f} MB per field) through the 126 MB L2"),
                        "step": "mas_op_update + " + ("mas_op_set_aniso + " if aniso else "") +
@@ -620,7 +636,7 @@ def main():
                         "A_GBs": achieved,
                         **({"Lpar_ms": c_ms, "Lpar_GBs": c_b * cells_local / (c_ms / 1e3) / 1e9,
                             "Lpar_alg_bytes_per_cell": c_b} if aniso and c_ms > 0 else {}),
-                        "B_GBs": b_b * cells_local / (b_ms / 1e3) / 1e9,
+                        "B_GBs": b_b * cells_local / (b_ms / 1e3) / 1e9 if b_ms > 0 else None,
                         "iter_alg_GBs": iter_gbs, "iter_frac": iter_gbs / peak,
                         "alg_bytes_per_cell_iter": a_b + b_b + c_b},
             "e2e": e2e,

@@ -211,6 +211,26 @@ MAS_API mas_status_t mas_pcg_solve(const mas_op_t* op, const double* rhs, double
  * traps the kernel (fails loudly rather than hanging). */
 MAS_API mas_status_t mas_op_enable_p2p(mas_op_t* op, cudaStream_t stream);
 
+/* Single-reduction PCG (the paper's lesson that
+ * fused, asynchronous kernels win).  on != 0: later
+ * mas_pcg_solve calls on this op run the Chronopoulos-Gear form of the same
+ * Jacobi-PCG (reading R28): ONE fused kernel and ONE
+ * reduction (<r,D^-1 r>, <L D^-1 r, D^-1 r>, <r,r>) per iteration instead of
+ * two of each:
+ *   s = w + beta s;  r -= alpha s;  p = D^-1 r_old + beta p;  x += alpha p;
+ *   w = L D^-1 r  (r, s recomputed on the halo cells, so no extra pass).
+ * Same arguments, stopping rule (R10) and counting (R11) as the standard
+ * loop; iterates equal it in exact arithmetic (rounding differs: parity band
+ * +-2 iterations, x <= 1e-9).  HBM traffic per iteration: 13 passes scalar
+ * (as the two-kernel loop), 33 passes for 3 components (31).  Allocates 3
+ * more vectors.  on == 0 restores the two-kernel loop.
+ * Errors: MAS_ERR_ARG on a grid with a mas_dist_t (one GPU only) or with
+ * the field-aligned term on; MAS_ERR_NOMEM. */
+MAS_API mas_status_t mas_op_set_single_reduction(mas_op_t* op, int on);
+
+/* 1 if the op's solve uses the single-reduction loop, 0 if not, -1 if NULL. */
+MAS_API int mas_op_single_reduction(const mas_op_t* op);
+
 /* Transport of the op's PCG loop: 0 NCCL (or one GPU), 1 P2P; -1 if op is NULL. */
 MAS_API int mas_op_transport(const mas_op_t* op);
 

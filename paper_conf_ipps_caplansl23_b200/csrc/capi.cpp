@@ -153,6 +153,12 @@ struct mas_op {
     double* rs_w = nullptr;
     double* rs_out = nullptr;
     double* astage = nullptr;                    // host kpar / b staging [4][nl][nt][np]
+    // single-reduction PCG (NEXT-1, mas_op_set_single_reduction): ping-pong r,
+    // w = L D^-1 r and s = L p (r: r / r2, w: q / w2, s: p[0] / p[1]), p in place
+    int cg1 = 0;
+    double *r2 = nullptr, *w2 = nullptr, *pcg = nullptr;
+    cudaGraphExec_t gexec1 = nullptr;
+    const double* g1_x = nullptr;
     double* atab = nullptr;                      // AnisoTab arrays (device)
     AnisoTab at{};
 };
@@ -459,8 +465,10 @@ static mas_status_t op_load(mas_op* op, const double* kappa, const double* mass,
 static void op_free(mas_op* op) {
     if (!op) return;
     for (double* p : {op->kgt, op->dgt, op->xgt, op->rgt, op->pgt[0], op->pgt[1], op->tpack, op->ca,
-                      op->atab, op->cag, op->pkg, op->rs_w, op->rs_out, op->astage})
+                      op->atab, op->cag, op->pkg, op->rs_w, op->rs_out, op->astage, op->r2, op->w2,
+                      op->pcg})
         if (p) cudaFree(p);
+    if (op->gexec1) cudaGraphExecDestroy(op->gexec1);
     for (double* p : {op->kappa, op->c, op->dinv, op->kg, op->dg, op->wR, op->r, op->p[0], op->p[1],
                       op->q, op->rg, op->pg[0], op->pg[1], op->xg, op->stage_a, op->stage_b,
                       op->hist, op->dot_out, op->scr.partials})
@@ -600,6 +608,191 @@ static mas_status_t loop_graph(mas_op* op, StencilArgs a, StreamArgs b, AnisoArg
     op->g_aniso = op->aniso;
     op->g_pre = (int)pre_plain;
     return MAS_OK;
+}
+
+// ---------------------------------------------------------------------------
+// single-reduction PCG (reading R28)
+// ---------------------------------------------------------------------------
+// kernel k >= 1 of the Chronopoulos-Gear loop: r_{k-1}, w_{k-1}, s_{k-2} in,
+// s_{k-1}, r_k, w_k out (ping-pong by parity), p and x in place
+static void cg1_args(const mas_op* op, int k, StencilArgs& a) {
+    const int nc = op->ncomp;
+    double* R[2] = {op->r, op->r2};
+    double* Wb[2] = {op->q, op->w2};
+    double* S[2] = {op->p[0], op->p[1]};
+    a.u = halo_of(op, R[(k - 1) & 1], nullptr, nc);
+    a.w = halo_of(op, Wb[(k - 1) & 1], nullptr, nc);
+    a.pold = halo_of(op, S[k & 1], nullptr, nc);
+    a.sout = S[(k - 1) & 1];
+    a.rout = R[k & 1];
+    a.out = Wb[k & 1];
+    a.pnew = op->pcg;
+}
+
+// graph: init (w0 = L D^-1 r0) -> while (!stopped) { CG1(k odd), CG1(k even) }
+static mas_status_t cg1_graph(mas_op* op, StencilArgs a) {
+    if (op->gexec1 && op->g1_x == a.x) return MAS_OK;
+    if (op->gexec1) {
+        cudaGraphExecDestroy(op->gexec1);
+        op->gexec1 = nullptr;
+    }
+    if (!op->cap_stream) CU(cudaStreamCreateWithFlags(&op->cap_stream, cudaStreamNonBlocking));
+    const int nc = op->ncomp;
+    cudaGraph_t g;
+    CU(cudaGraphCreate(&g, 0));
+    cudaError_t e = cudaStreamBeginCaptureToGraph(op->cap_stream, g, nullptr, nullptr, 0,
+                                                  cudaStreamCaptureModeThreadLocal);
+    if (e == cudaSuccess) {
+        StencilArgs a0 = a;
+        a0.u = halo_of(op, op->r, nullptr, nc);
+        a0.out = op->q;
+        e = launch_stencil(MODE_CG1, nc, a0, op->cap_stream, true);
+        cudaGraph_t out = g;
+        cudaError_t e2 = cudaStreamEndCapture(op->cap_stream, &out);
+        if (e == cudaSuccess) e = e2;
+    }
+    size_t n = 0;
+    if (e == cudaSuccess) e = cudaGraphGetNodes(g, nullptr, &n);
+    cudaGraphNode_t leaf = nullptr;
+    if (e == cudaSuccess && n == 1) e = cudaGraphGetNodes(g, &leaf, &n);
+    if (e == cudaSuccess && !leaf) e = cudaErrorInvalidValue;
+    cudaGraphConditionalHandle h;
+    if (e == cudaSuccess) e = cudaGraphConditionalHandleCreate(&h, g, 1, cudaGraphCondAssignDefault);
+    cudaGraphNodeParams p = {};
+    p.type = cudaGraphNodeTypeConditional;
+    p.conditional.handle = h;
+    p.conditional.type = cudaGraphCondTypeWhile;
+    p.conditional.size = 1;
+    cudaGraphNode_t node;
+    if (e == cudaSuccess) e = cudaGraphAddNode(&node, g, &leaf, 1, &p);
+    if (e == cudaSuccess) {
+        e = cudaStreamBeginCaptureToGraph(op->cap_stream, p.conditional.phGraph_out[0], nullptr, nullptr, 0,
+                                          cudaStreamCaptureModeThreadLocal);
+        if (e == cudaSuccess) {
+            a.cond = (unsigned long long)h;
+            for (int k = 1; k <= 2 && e == cudaSuccess; k++) {
+                cg1_args(op, k, a);
+                e = launch_stencil(MODE_CG1, nc, a, op->cap_stream);
+            }
+            cudaGraph_t out = p.conditional.phGraph_out[0];
+            cudaError_t e2 = cudaStreamEndCapture(op->cap_stream, &out);
+            if (e == cudaSuccess) e = e2;
+        }
+    }
+    if (e == cudaSuccess) e = cudaGraphInstantiate(&op->gexec1, g, 0);
+    cudaGraphDestroy(g);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        op->gexec1 = nullptr;
+        set_last_error(std::string("single-reduction loop graph: ") + cudaGetErrorString(e));
+        return MAS_ERR_CUDA;
+    }
+    op->g1_x = a.x;
+    return MAS_OK;
+}
+
+static mas_status_t cg1_solve(mas_op* op, const double* fd, double* xd, double tol, int maxit, int* iters,
+                              double* relres, double* res_hist, cudaStream_t s) {
+    const int nc = op->ncomp;
+    const size_t bytes = nc * op->Nl * sizeof(double);
+    op->launches = 0;
+    PcgState init{};
+    init.tol = tol;
+    init.maxit = maxit;
+    init.k = 0;
+    init.stopped = 0;
+    init.status = MAS_NOT_CONVERGED;
+    CU(cudaMemcpyAsync(op->st, &init, sizeof(init), cudaMemcpyHostToDevice, s));
+    *op->host_flag = 0;
+    // kernel 1 reads s_{-1} = p[1] and p_{-1} = pcg with beta_0 = 0: finite zeros
+    CU(cudaMemsetAsync(op->p[1], 0, bytes, s));
+    CU(cudaMemsetAsync(op->pcg, 0, bytes, s));
+    double* rho_h = op->hist;
+    double* sig_h = op->hist + op->hist_cap;
+    double* rr_h = op->hist + 2 * op->hist_cap;
+    StencilArgs a{};
+    a.g = op->geo;
+    a.chunk = op->chunk;
+    a.kappa = halo_of(op, op->kappa, nullptr, 1);
+    a.dinv = halo_of(op, op->dinv, nullptr, 1);
+    a.c = op->c;
+    a.st = op->st;
+    a.rho_hist = rho_h;
+    a.sigma_hist = sig_h;
+    a.rr_hist = rr_h;
+    a.scr = op->scr;
+    a.host_flag = op->host_flag_dev;
+    // a3: r0 = f - L x0 and <f,f>, <r0,r0> (k_stencil<RESID>, as the standard loop)
+    StencilArgs r0 = a;
+    r0.u = halo_of(op, xd, nullptr, nc);
+    r0.f = fd;
+    r0.out = op->r;
+    CU(launch_stencil(MODE_RESID, nc, r0, s));
+    op->launches++;
+    a.x = xd;
+    const bool graph = !op->prof && op->use_graph;
+    if (graph) {
+        ST(cg1_graph(op, a));
+        CU(cudaGraphLaunch(op->gexec1, s));
+    } else {
+        // host-driven: launch n = 1 is the init, n = k + 1 is kernel k; stop
+        // enqueueing once the device reports a decision taken by launch <= n-1
+        for (int n = 1; n <= maxit + 1; n++) {
+            cudaEvent_t* pe = nullptr;
+            if (op->prof) {
+                ST(ensure_prof_events(op, n));
+                pe = &op->pev[6 * (size_t)(n - 1)];
+                CU(cudaEventRecord(pe[0], s));
+            }
+            if (n == 1) {
+                StencilArgs a0 = a;
+                a0.u = halo_of(op, op->r, nullptr, nc);
+                a0.out = op->q;
+                CU(launch_stencil(MODE_CG1, nc, a0, s, true));
+            } else {
+                cg1_args(op, n - 1, a);
+                CU(launch_stencil(MODE_CG1, nc, a, s));
+            }
+            op->launches++;
+            if (pe) CU(cudaEventRecord(pe[1], s));
+            CU(cudaEventRecord(op->ev[n & 1], s));
+            if (n >= 2) {
+                CU(cudaEventSynchronize(op->ev[(n - 1) & 1]));
+                const int flag = *(volatile int*)op->host_flag;
+                if (flag > 0 && flag <= n - 1) break;
+            }
+        }
+    }
+    CU(cudaStreamSynchronize(s));
+    PcgState fin{};
+    CU(cudaMemcpy(&fin, op->st, sizeof(fin), cudaMemcpyDeviceToHost));
+    if (!fin.stopped) {
+        set_last_error("internal: single-reduction loop ended without a stop decision");
+        return MAS_ERR_CUDA;
+    }
+    *iters = fin.iters;
+    *relres = fin.relres;
+    if (graph) op->launches += 1 + fin.iters + (fin.iters & 1);  // init + kernels (+ an early exit)
+    if (res_hist) {
+        const int nh = (fin.status == MAS_ERR_BREAKDOWN && fin.iters == 1) ? 1 : fin.iters + 1;
+        std::vector<double> rr(nh);
+        CU(cudaMemcpy(rr.data(), rr_h, rr.size() * sizeof(double), cudaMemcpyDeviceToHost));
+        for (int k = 0; k < nh; k++) res_hist[k] = std::sqrt(rr[k]);
+    }
+    if (op->prof) {  // average device time of kernels 1..iters (the init excluded)
+        double sa = 0.0;
+        int n = 0;
+        for (int k = 2; k <= fin.iters + 1 && 6 * (size_t)k <= op->pev.size(); k++, n++) {
+            float t = 0.f;
+            CU(cudaEventElapsedTime(&t, op->pev[6 * (size_t)(k - 1)], op->pev[6 * (size_t)(k - 1) + 1]));
+            sa += t;
+        }
+        op->prof_a_ms = n ? sa / n : 0.0;
+        op->prof_b_ms = 0.0;
+        op->prof_c_ms = 0.0;
+        op->prof_n = n;
+    }
+    return (mas_status_t)fin.status;
 }
 
 static mas_status_t ensure_stage(mas_op* op) {
@@ -1019,6 +1212,24 @@ mas_status_t mas_op_enable_p2p(mas_op_t* op, cudaStream_t s) {
 
 int mas_op_transport(const mas_op_t* op) { return !op ? -1 : op->p2p ? 1 : 0; }
 
+mas_status_t mas_op_set_single_reduction(mas_op_t* op, int on) {
+    if (!op) return arg_error("null op");
+    if (!on) {
+        op->cg1 = 0;
+        return MAS_OK;
+    }
+    if (op->g->comm) return arg_error("single-reduction PCG: one GPU only (no mas_dist_t)");
+    if (op->aniso) return arg_error("single-reduction PCG: isotropic operator only (no mas_op_set_aniso)");
+    const size_t n = op->ncomp * (size_t)op->Nl;
+    if (!op->r2) ST(dmalloc(&op->r2, n));
+    if (!op->w2) ST(dmalloc(&op->w2, n));
+    if (!op->pcg) ST(dmalloc(&op->pcg, n));
+    op->cg1 = 1;
+    return MAS_OK;
+}
+
+int mas_op_single_reduction(const mas_op_t* op) { return op ? op->cg1 : -1; }
+
 mas_status_t mas_op_comm_bench(mas_op_t* op, int reps, double* seam_us, double* allreduce_us,
                                double* seam_bytes, cudaStream_t s) {
     if (!op || !seam_us || !allreduce_us || !seam_bytes || reps < 1) return arg_error("bad argument");
@@ -1095,6 +1306,7 @@ mas_status_t mas_op_set_aniso(mas_op_t* op, const double* kpar, const double* bh
         return MAS_OK;
     }
     if (!bhat) return arg_error("null bhat");
+    if (op->cg1) return arg_error("field-aligned conduction: switch the single-reduction loop off first");
     if (op->ncomp != 1) return arg_error("field-aligned conduction needs ncomp == 1");
     if (op->g->ptheta > 1)
         return arg_error("field-aligned conduction: r-slab decompositions only (ptheta == 1)");
@@ -1217,6 +1429,12 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
         xd = op->stage_b;
     }
 
+    if (op->cg1) {  // NEXT-1: single-reduction loop (one GPU, isotropic operator)
+        mas_status_t st = cg1_solve(op, fd, xd, tol, maxit, iters, relres, res_hist, s);
+        if (hx && (st == MAS_OK || st == MAS_NOT_CONVERGED || st == MAS_ERR_BREAKDOWN))
+            CU(cudaMemcpy(x, xd, bytes, cudaMemcpyDeviceToHost));
+        return st;
+    }
     const bool p2p = op->p2p;
     PcgState init{};
     if (p2p) init.epoch = ++op->epoch;

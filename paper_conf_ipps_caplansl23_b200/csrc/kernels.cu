@@ -13,6 +13,10 @@
 //   k_pcg_b               "kernel B":  r -= alpha q, z = D^-1 r, <r,z>_V, <r,r>_V
 //   k_stencil<MODE_RESID> init:  r = f - L x, <f,f>_V, <r,r>_V, <r,D^-1 r>_V
 //   k_stencil<MODE_APPLY> y = L x (mas_op_apply)
+//   k_stencil<MODE_CG1>   single-reduction PCG (NEXT-1, Chronopoulos-Gear):
+//       s = w + beta s, r -= alpha s, x += alpha p, p = D^-1 r_old + beta p
+//       (halo too for s, r), w = L D^-1 r, <r,D^-1 r>, <w,D^-1 r>, <r,r>:
+//       ONE kernel and one reduction per iteration (FIRSTK: w0 = L D^-1 r0)
 //
 // Scalars (alpha, beta, convergence, breakdown) never leave the device: each
 // reduction ends in a deterministic "last block" sum (fixed order, no fp64
@@ -95,6 +99,7 @@ struct OwnRegs {
     double2 c;      // mass term
     double2 f[NC];  // RESID: rhs
     double2 di;     // RESID: 1/D
+    double2 rn[NC]; // CG1 scalar: r_k for <r,u>, <r,r> in the stencil phase
 };
 
 // Raw inputs of one cell pair (or one cell in .x for a phi-halo column).
@@ -102,8 +107,9 @@ template <int NC>
 struct Raw {
     double2 u[NC];   // PCGA: r;  APPLY/RESID: x
     double2 po[NC];  // PCGA: p_{k-1}
-    double2 di;      // PCGA: 1/D
+    double2 di;      // PCGA, CG1: 1/D
     double2 kap;
+    double2 wv[NC];  // CG1: w_{k-1} (po holds s_{k-2})
 };
 
 template <bool SCALAR>
@@ -117,6 +123,7 @@ template <int NC>
 struct PlanePtrs {
     const double* u[NC];
     const double* po[NC];
+    const double* w[NC];
     const double* di;
     const double* kap;
 };
@@ -128,9 +135,12 @@ __device__ __forceinline__ PlanePtrs<NC> plane_ptrs(const StencilArgs& a, int i,
     P.kap = plane_ptr(a.kappa, 0, i, g);
 #pragma unroll
     for (int c = 0; c < NC; c++) P.u[c] = plane_ptr(a.u, c, i, g);
-    P.di = (MODE == MODE_PCGA) ? plane_ptr(a.dinv, 0, i, g) : nullptr;
+    constexpr bool KRY = MODE == MODE_PCGA || MODE == MODE_CG1;
+    P.di = KRY ? plane_ptr(a.dinv, 0, i, g) : nullptr;
 #pragma unroll
-    for (int c = 0; c < NC; c++) P.po[c] = (MODE == MODE_PCGA && !first) ? plane_ptr(a.pold, c, i, g) : nullptr;
+    for (int c = 0; c < NC; c++) P.po[c] = (KRY && !first) ? plane_ptr(a.pold, c, i, g) : nullptr;
+#pragma unroll
+    for (int c = 0; c < NC; c++) P.w[c] = (MODE == MODE_CG1 && !first) ? plane_ptr(a.w, c, i, g) : nullptr;
     return P;
 }
 
@@ -139,11 +149,15 @@ __device__ __forceinline__ void load_raw(const PlanePtrs<NC>& P, int off, bool f
     R.kap = ldv<SCALAR>(P.kap + off);
 #pragma unroll
     for (int c = 0; c < NC; c++) R.u[c] = ldv<SCALAR>(P.u[c] + off);
-    if (MODE == MODE_PCGA) {
+    if (MODE == MODE_PCGA || MODE == MODE_CG1) {
         R.di = ldv<SCALAR>(P.di + off);
         if (!first) {
 #pragma unroll
             for (int c = 0; c < NC; c++) R.po[c] = ldv<SCALAR>(P.po[c] + off);
+            if (MODE == MODE_CG1) {
+#pragma unroll
+                for (int c = 0; c < NC; c++) R.wv[c] = ldv<SCALAR>(P.w[c] + off);
+            }
         }
     }
 }
@@ -156,11 +170,15 @@ __device__ __forceinline__ void load_raw_in(const StencilArgs& a, int Nl, int id
     R.kap = ldv<SCALAR>(a.kappa.in + idx);
 #pragma unroll
     for (int c = 0; c < NC; c++) R.u[c] = ldv<SCALAR>(a.u.in + c * Nl + idx);
-    if (MODE == MODE_PCGA) {
+    if (MODE == MODE_PCGA || MODE == MODE_CG1) {
         R.di = ldv<SCALAR>(a.dinv.in + idx);
         if (!first) {
 #pragma unroll
             for (int c = 0; c < NC; c++) R.po[c] = ldv<SCALAR>(a.pold.in + c * Nl + idx);
+            if (MODE == MODE_CG1) {
+#pragma unroll
+                for (int c = 0; c < NC; c++) R.wv[c] = ldv<SCALAR>(a.w.in + c * Nl + idx);
+            }
         }
     }
 }
@@ -227,7 +245,8 @@ __device__ __forceinline__ HaloMeta halo_meta(const Geo& g, int j0, int k0, int 
 template <int NC>
 struct Stage {
     Raw<NC> R;                          // own double2 pair
-    double2 xv[NC];                     // own x (PCGA deferred update)
+    double2 xv[NC];                     // own x (PCGA deferred update; CG1 x_{k-1})
+    double2 pp[NC];                     // CG1: own p_{k-2}
     OwnRegs<NC> o;                      // own c (+ f, D^-1 for RESID)
 };
 
@@ -235,7 +254,8 @@ struct Stage {
 // The scalar halo items do not fit in registers next to the own pair's
 // in-flight loads (ptxas spilled them, forcing an early wait), so each halo
 // thread copies its item into a private shared-memory slot instead:
-// layout [field][kHaloSlots], fields 0 kappa, 1 1/D, 2.. u[NC], po[NC].
+// layout [field][kHaloSlots], fields 0 kappa, 1 1/D, 2.. u[NC], po[NC]
+// (+ w[NC] in MODE_CG1).
 constexpr int kHaloSlots = 2 * TK + 2 * TJ;
 __device__ __forceinline__ void cpa8(double* sdst, const double* gsrc) {
     const unsigned sa = (unsigned)__cvta_generic_to_shared(sdst);
@@ -258,7 +278,7 @@ __device__ __forceinline__ void trow_issue(const StencilArgs& a, int i, const Ha
     cpa8(h, trow_at(a.tkappa, hi, 0, i, k));
 #pragma unroll
     for (int c = 0; c < NC; c++) cpa8(h + (2 + c) * kHaloSlots, trow_at(a.tu, hi, c, i, k));
-    if (MODE == MODE_PCGA) {
+    if (MODE == MODE_PCGA || MODE == MODE_CG1) {
         cpa8(h + kHaloSlots, trow_at(a.tdinv, hi, 0, i, k));
         if (!first) {
 #pragma unroll
@@ -298,7 +318,9 @@ __device__ __forceinline__ void plane_prefetch(const StencilArgs& a, int i, int 
                                                int width, bool first, bool xupd) {
     const Geo& g = a.g;
     // fields: u[NC], po[NC] (PCGA, not first), x[NC] (xupd), dinv (PCGA), kappa, c
-    constexpr int NF = 3 * NC + 3;
+    // (+ CG1: w[NC], the own p[NC])
+    constexpr bool KRY = MODE == MODE_PCGA || MODE == MODE_CG1;
+    constexpr int NF = 3 * NC + 3 + (MODE == MODE_CG1 ? 2 * NC : 0);
     const int t = threadIdx.x;
     if (t >= NF * TJ) return;
     const int f = t / TJ, w = t - f * TJ;
@@ -307,14 +329,27 @@ __device__ __forceinline__ void plane_prefetch(const StencilArgs& a, int i, int 
     const int off = i * plane32(g) + (j0 + w) * g.np + k0;
     const double* base = nullptr;
     if (f < NC) base = a.u.in + f * Nl;
-    else if (f < 2 * NC) base = (MODE == MODE_PCGA && !first) ? a.pold.in + (f - NC) * Nl : nullptr;
-    else if (f < 3 * NC) base = (MODE == MODE_PCGA && xupd) ? a.x + (f - 2 * NC) * Nl : nullptr;
-    else if (f == 3 * NC) base = MODE == MODE_PCGA ? a.dinv.in : nullptr;
+    else if (f < 2 * NC) base = (KRY && !first) ? a.pold.in + (f - NC) * Nl : nullptr;
+    else if (f < 3 * NC) base = (KRY && xupd) ? a.x + (f - 2 * NC) * Nl : nullptr;
+    else if (f == 3 * NC) base = KRY ? a.dinv.in : nullptr;
     else if (f == 3 * NC + 1) base = a.kappa.in;
-    else base = a.c;
+    else if (f == 3 * NC + 2) base = a.c;
+    else if (f < 4 * NC + 3) base = (MODE == MODE_CG1 && !first) ? a.w.in + (f - 3 * NC - 3) * Nl : nullptr;
+    else base = (MODE == MODE_CG1 && xupd) ? a.pnew + (f - 4 * NC - 3) * Nl : nullptr;
     if (base) l2_prefetch_row(base + off, width * 8);
 }
 #endif
+
+// CG1, 3 components: the own-only x and p are loaded at commit time (L2 hits:
+// the bulk prefetch runs kPfDist planes ahead) instead of one plane ahead in
+// registers, which would spill (17 double2 of loads in flight per thread)
+template <int NC>
+constexpr bool kCg1LateOwn = (NC == 3);
+// CG1: where <r_k,u_k> and <r_k,r_k> accumulate.  3 components: at commit
+// (r_k is at hand; keeping it to the stencil phase spills); scalar: in the
+// stencil phase with r_k carried in OwnRegs (measured 5% faster at C2)
+template <int NC>
+constexpr bool kCg1DotsAtCommit = (NC == 3);
 
 template <int MODE, int NC>
 __device__ __forceinline__ void stage_issue(const StencilArgs& a, int i, int j0, int k0, int height,
@@ -337,9 +372,13 @@ __device__ __forceinline__ void stage_issue(const StencilArgs& a, int i, int j0,
         }
         if (own_work) {
             if (a.c) S.o.c = ld2(a.c + o3);
-            if (MODE == MODE_PCGA && xupd) {
+            if ((MODE == MODE_PCGA || (MODE == MODE_CG1 && !kCg1LateOwn<NC>)) && xupd) {
 #pragma unroll
                 for (int c = 0; c < NC; c++) S.xv[c] = lds2(a.x + c * Nl + o3);
+            }
+            if (MODE == MODE_CG1 && !kCg1LateOwn<NC> && xupd) {
+#pragma unroll
+                for (int c = 0; c < NC; c++) S.pp[c] = lds2(a.pnew + c * Nl + o3);
             }
             if (MODE == MODE_RESID) {
                 S.o.di = ld2(a.dinv.in + o3);
@@ -357,12 +396,17 @@ __device__ __forceinline__ void stage_issue(const StencilArgs& a, int i, int j0,
             cpa8(h, a.kappa.in + hi);
 #pragma unroll
             for (int c = 0; c < NC; c++) cpa8(h + (2 + c) * kHaloSlots, a.u.in + c * Nl + hi);
-            if (MODE == MODE_PCGA) {
+            if (MODE == MODE_PCGA || MODE == MODE_CG1) {
                 cpa8(h + kHaloSlots, a.dinv.in + hi);
                 if (!first) {
 #pragma unroll
                     for (int c = 0; c < NC; c++)
                         cpa8(h + (2 + NC + c) * kHaloSlots, a.pold.in + c * Nl + hi);
+                    if (MODE == MODE_CG1) {
+#pragma unroll
+                        for (int c = 0; c < NC; c++)
+                            cpa8(h + (2 + 2 * NC + c) * kHaloSlots, a.w.in + c * Nl + hi);
+                    }
                 }
             }
         }
@@ -375,13 +419,57 @@ __device__ __forceinline__ void stage_commit(const StencilArgs& a, int i, int j0
                                              int width, const HaloMeta& hm, bool first, double beta,
                                              double alpha_prev, bool xupd, bool halo, bool own_work,
                                              Stage<NC>& S, double* buf, double2& kown,
-                                             OwnRegs<NC>& o, const double* hst) {
+                                             OwnRegs<NC>& o, const double* hst, double (&acc)[3]) {
     const Geo& g = a.g;
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     const int kc = 2 * lane;
     const int Nl = (int)g.nl * plane32(g);
     if (w < height && kc < width) {
-        finish_raw<MODE, NC>(S.R, first, beta);
+        if constexpr (MODE == MODE_CG1) {
+            // s_{k-1} = w_{k-1} + beta s_{k-2};  r_k = r_{k-1} - alpha s_{k-1};
+            // own: p_{k-1} = D^-1 r_{k-1} + beta p_{k-2};  x_k = x_{k-1} + alpha p_{k-1}
+            // (alpha_prev = alpha_{k-1}, beta = beta_{k-1});  ring: u_k = D^-1 r_k
+            const int o3 = (int)i * plane32(g) + (int)(j0 + w) * g.np + k0 + kc;
+            double V0 = 0.0, V1 = 0.0;
+            if (kCg1DotsAtCommit<NC> && own_work) {  // <r_k, u_k>_V and <r_k, r_k>_V (own cells)
+                const double vrt = __ldg(g.vr + i) * __ldg(g.vt + j0 + w);
+                const double2 vp = ld2(g.vp + k0 + kc);
+                V0 = vrt * vp.x;
+                V1 = vrt * vp.y;
+            }
+#pragma unroll
+            for (int c = 0; c < NC; c++) {
+                double2 rk = S.R.u[c];
+                if (!first) {
+                    double2 sv;
+                    sv.x = fma(beta, S.R.po[c].x, S.R.wv[c].x);
+                    sv.y = fma(beta, S.R.po[c].y, S.R.wv[c].y);
+                    rk.x = fma(-alpha_prev, sv.x, S.R.u[c].x);
+                    rk.y = fma(-alpha_prev, sv.y, S.R.u[c].y);
+                    if (own_work) {
+                        const double2 pp = kCg1LateOwn<NC> ? lds2(a.pnew + c * Nl + o3) : S.pp[c];
+                        double2 pv;
+                        pv.x = fma(beta, pp.x, S.R.di.x * S.R.u[c].x);
+                        pv.y = fma(beta, pp.y, S.R.di.y * S.R.u[c].y);
+                        double2 xv = kCg1LateOwn<NC> ? lds2(a.x + c * Nl + o3) : S.xv[c];
+                        xv.x = fma(alpha_prev, pv.x, xv.x);
+                        xv.y = fma(alpha_prev, pv.y, xv.y);
+                        stg2a(a.sout + c * Nl + o3, sv);
+                        stg2a(a.rout + c * Nl + o3, rk);
+                        stg2a(a.pnew + c * Nl + o3, pv);
+                        stg2a(a.x + c * Nl + o3, xv);
+                    }
+                }
+                S.R.u[c] = make_double2(S.R.di.x * rk.x, S.R.di.y * rk.y);
+                if (!kCg1DotsAtCommit<NC>) S.o.rn[c] = rk;
+                if (kCg1DotsAtCommit<NC> && own_work) {
+                    acc[0] += V0 * rk.x * S.R.u[c].x + V1 * rk.y * S.R.u[c].y;
+                    acc[2] += V0 * rk.x * rk.x + V1 * rk.y * rk.y;
+                }
+            }
+        } else {
+            finish_raw<MODE, NC>(S.R, first, beta);
+        }
         const int idx = (1 + w) * ROW + OFF + kc;
 #pragma unroll
         for (int c = 0; c < NC; c++) sts2(sfield(buf, c) + idx, S.R.u[c]);
@@ -389,7 +477,7 @@ __device__ __forceinline__ void stage_commit(const StencilArgs& a, int i, int j0
         kown = S.R.kap;
         if (own_work) {
             o = S.o;
-            if (MODE == MODE_PCGA) {
+            if constexpr (MODE == MODE_PCGA) {
                 const int o3 = (int)i * plane32(g) + (int)(j0 + w) * g.np + k0 + kc;
 #pragma unroll
                 for (int c = 0; c < NC; c++) {
@@ -413,6 +501,12 @@ __device__ __forceinline__ void stage_commit(const StencilArgs& a, int i, int j0
             if (MODE == MODE_PCGA) {
                 const double z = h[kHaloSlots] * u;
                 u = first ? z : fma(beta, h[(2 + NC + c) * kHaloSlots], z);
+            } else if (MODE == MODE_CG1) {
+                if (!first) {  // r_k of the halo cell from its r, s, w of iteration k-1
+                    const double sv = fma(beta, h[(2 + NC + c) * kHaloSlots], h[(2 + 2 * NC + c) * kHaloSlots]);
+                    u = fma(-alpha_prev, sv, u);
+                }
+                u = h[kHaloSlots] * u;
             }
             sfield(buf, c)[hm.hidx] = u;
         }
@@ -517,8 +611,29 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
             pmode = P_FINAL;
         else if (!first)
             beta = rho1 / rho2;
+    } else if (MODE == MODE_CG1) {
+        // single reduction: kernel k's last block decided alpha_k, beta_k and
+        // the stop; here (k+1) everything comes from PcgState
+        const PcgState* st = a.st;
+        if (__ldcg(&st->stopped)) {
+            if (a.cond && blockIdx.x == 0 && threadIdx.x == 0)
+                cudaGraphSetConditional((cudaGraphConditionalHandle)a.cond, 0);
+            return;
+        }
+        kit = __ldcg(&st->k);
+        if (FIRSTK) {  // the init: k = 0; r0 from k_stencil<RESID>
+            const double ff = __ldcg(&st->pend_ff), rr = __ldcg(&st->pend_rr);
+            final_g[0] = ff, final_g[1] = rr, final_g[2] = 0.0;
+            if (ff == 0.0)
+                pmode = P_ZERO;
+            else if (sqrt(rr) <= __ldcg(&st->tol) * sqrt(ff) || __ldcg(&st->maxit) == 0)
+                pmode = P_FINAL;
+        } else {
+            alpha_prev = __ldcg(&st->cg_alpha);  // alpha_{k-1}
+            beta = __ldcg(&st->cg_beta);         // beta_{k-1}
+        }
     }
-    const bool xupd = (MODE == MODE_PCGA) && !FIRSTK;
+    const bool xupd = (MODE == MODE_PCGA || MODE == MODE_CG1) && !FIRSTK;
     if (MODE == MODE_PCGA && pmode == P_NORMAL && FIRSTK != first) __trap();  // host dispatch bug
 
     // ---- work item ------------------------------------------------------
@@ -542,7 +657,7 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
 
     double acc[3] = {0.0, 0.0, 0.0};
 
-    if (MODE == MODE_PCGA && pmode != P_NORMAL) {
+    if ((MODE == MODE_PCGA || MODE == MODE_CG1) && pmode != P_NORMAL) {
         // final deferred update x += alpha_{k-1} p_{k-1} (or x = 0 if f == 0)
         if (own) {
             for (int i = ia; i < ib; i++) {
@@ -551,7 +666,7 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
                     double* xp = a.x + c * Nl + (int)i * plane32(g) + off;
                     if (pmode == P_ZERO) {
                         stg2(xp, make_double2(0.0, 0.0));
-                    } else if (kit >= 2) {
+                    } else if (MODE == MODE_PCGA && kit >= 2) {
                         const double2 po = ld2(plane_ptr(a.pold, c, i, g) + off);
                         double2 xv = lds2(xp);
                         xv.x = fma(alpha_prev, po.x, xv.x);
@@ -565,8 +680,10 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
         if (grid_reduce<1, kSThreads>(v1, a.scr, TKT_STENCIL) && threadIdx.x == 0 && a.part != 1) {
             PcgState* st = a.st;
             const double ff = final_g[0], rr = final_g[1], rho1 = final_g[2];
-            a.rr_hist[kit - 1] = rr;
-            a.rho_hist[kit - 1] = rho1;
+            // PCGA: A(k) stops at iterate k-1;  CG1: only its init (k = 0) lands here
+            const int hk = MODE == MODE_CG1 ? 0 : kit - 1;
+            a.rr_hist[hk] = rr;
+            a.rho_hist[hk] = rho1;
             if (pmode == P_ZERO) {
                 st->iters = 0;
                 st->relres = 0.0;
@@ -574,7 +691,7 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
                 a.rr_hist[0] = 0.0;
             } else {
                 const bool conv = sqrt(rr) <= st->tol * sqrt(ff);
-                st->iters = kit - 1;
+                st->iters = hk;
                 st->relres = sqrt(rr) / sqrt(ff);
                 st->status = conv ? MAS_OK : MAS_NOT_CONVERGED;
             }
@@ -582,7 +699,7 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
             st->stopped = 1;
             if (a.host_flag) {
                 __threadfence_system();
-                *(volatile int*)a.host_flag = kit;
+                *(volatile int*)a.host_flag = MODE == MODE_CG1 ? kit + 1 : kit;  // CG1: launch number
             }
             if (a.cond) cudaGraphSetConditional((cudaGraphConditionalHandle)a.cond, 0);
         }
@@ -595,7 +712,7 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
     auto slot = [&](int i) { return smem + ((i - ia + 1) & 3) * BUF; };
     // private cp.async slots of the halo items: static shared memory, so the
     // shared-window address needs no runtime conversion
-    __shared__ __align__(16) double hst_arr[(2 + 2 * NC) * kHaloSlots];
+    __shared__ __align__(16) double hst_arr[(2 + (MODE == MODE_CG1 ? 3 : 2) * NC) * kHaloSlots];
     auto real_plane = [&](int p) { return !(p == g.nl && g.glob_hi); };
 
     // 1-D geometry of this work item staged in shared memory once (visible to
@@ -643,9 +760,9 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
     stage_issue<MODE, NC>(a, ia, j0, k0, height, width, hm, FIRSTK, xupd, true, true, S, hst_arr);
     if (!lo_ghost)
         stage_commit<MODE, NC>(a, ia - 1, j0, k0, height, width, hm, FIRSTK, beta, alpha_prev, false,
-                               false, false, S0, slot(ia - 1), kdummy, on, hst_arr);
+                               false, false, S0, slot(ia - 1), kdummy, on, hst_arr, acc);
     stage_commit<MODE, NC>(a, ia, j0, k0, height, width, hm, FIRSTK, beta, alpha_prev, xupd, true, true,
-                           S, slot(ia), kown, oc, hst_arr);
+                           S, slot(ia), kown, oc, hst_arr, acc);
     if (lo_ghost) ghost_plane<NC>(slot(ia - 1), height, width, kown);
     if (real_plane(ia + 1))
         stage_issue<MODE, NC>(a, ia + 1, j0, k0, height, width, hm, FIRSTK, xupd && (ia + 1 < ib),
@@ -656,7 +773,7 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
         if (real_plane(i + 1))
             stage_commit<MODE, NC>(a, i + 1, j0, k0, height, width, hm, FIRSTK, beta, alpha_prev,
                                    xupd && (i + 1 < ib), i + 1 < ib, i + 1 < ib, S, slot(i + 1),
-                                   kown, on, hst_arr);
+                                   kown, on, hst_arr, acc);
         else
             ghost_plane<NC>(slot(i + 1), height, width, kown);
         // issue plane i+2 (registers and private cp.async slots only): its
@@ -742,6 +859,15 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
                 } else {
                     stg2a(a.out + o, make_double2(L0, L1));
                     if (MODE == MODE_PCGA) acc[0] += V0 * u.x * L0 + V1 * u.y * L1;
+                    // CG1: delta = <w,u> (+ gamma = <r,u>, <r,r> unless accumulated at commit)
+                    if (MODE == MODE_CG1) {
+                        acc[1] += V0 * L0 * u.x + V1 * L1 * u.y;
+                        if (!kCg1DotsAtCommit<NC>) {
+                            const double2 rk = oc.rn[c];
+                            acc[0] += V0 * rk.x * u.x + V1 * rk.y * u.y;
+                            acc[2] += V0 * rk.x * rk.x + V1 * rk.y * rk.y;
+                        }
+                    }
                 }
             }
         }
@@ -758,6 +884,46 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
             if (p2p && !a.nopub) {  // (with the field-aligned term k_aniso<RESID> publishes)
                 const double pub[3] = {acc[2], acc[1], acc[0]};  // {rho, rr, ff}
                 p2p_publish(a.p2p, MB_B, p2p_seq(st->epoch, 0), pub, 3);
+            }
+        }
+    } else if (MODE == MODE_CG1) {
+        if (grid_reduce<3, kSThreads>(acc, a.scr, TKT_STENCIL) && threadIdx.x == 0) {
+            // the single reduction of iteration k: gamma_k, delta_k, ||r_k||^2.
+            // Decide the stop, else alpha_k and beta_k for kernel k+1 (R28).
+            PcgState* st = a.st;
+            const double gam = acc[0], del = acc[1], rr = acc[2];
+            const double ff = st->pend_ff;
+            a.rr_hist[kit] = rr;
+            a.rho_hist[kit] = gam;
+            a.sigma_hist[kit] = del;
+            int status = -1, iters = 0;
+            if (!FIRSTK && sqrt(rr) <= st->tol * sqrt(ff)) {
+                status = MAS_OK, iters = kit;
+            } else if (!FIRSTK && kit >= st->maxit) {
+                status = MAS_NOT_CONVERGED, iters = kit;
+            } else {
+                const double b = FIRSTK ? 0.0 : gam / st->cg_gamma;
+                const double den = FIRSTK ? del : del - b * gam / st->cg_alpha;  // <p_k, L p_k>
+                if (!(den > 0.0) || !isfinite(den)) {
+                    status = MAS_ERR_BREAKDOWN, iters = FIRSTK ? 1 : kit;
+                } else {
+                    st->cg_alpha = gam / den;
+                    st->cg_beta = b;
+                    st->cg_gamma = gam;
+                    st->k = kit + 1;
+                }
+            }
+            if (status >= 0) {
+                st->iters = iters;
+                st->relres = sqrt(rr) / sqrt(ff);
+                st->status = status;
+                __threadfence();
+                st->stopped = 1;
+                if (a.host_flag) {
+                    __threadfence_system();
+                    *(volatile int*)a.host_flag = kit + 1;  // launch number (init = 1)
+                }
+                if (a.cond) cudaGraphSetConditional((cudaGraphConditionalHandle)a.cond, 0);
             }
         }
     } else if (MODE == MODE_PCGA) {
@@ -1083,11 +1249,13 @@ cudaError_t launch_stencil(int mode, int ncomp, const StencilArgs& a, cudaStream
     if (ncomp == 1) {
         if (mode == MODE_APPLY) return launch_one<MODE_APPLY, 1>(a, s);
         if (mode == MODE_RESID) return launch_one<MODE_RESID, 1>(a, s);
+        if (mode == MODE_CG1) return first ? launch_one<MODE_CG1, 1, true>(a, s) : launch_one<MODE_CG1, 1>(a, s);
         return first ? launch_one<MODE_PCGA, 1, true>(a, s) : launch_one<MODE_PCGA, 1>(a, s);
     }
     if (ncomp == 3) {
         if (mode == MODE_APPLY) return launch_one<MODE_APPLY, 3>(a, s);
         if (mode == MODE_RESID) return launch_one<MODE_RESID, 3>(a, s);
+        if (mode == MODE_CG1) return first ? launch_one<MODE_CG1, 3, true>(a, s) : launch_one<MODE_CG1, 3>(a, s);
         return first ? launch_one<MODE_PCGA, 3, true>(a, s) : launch_one<MODE_PCGA, 3>(a, s);
     }
     return cudaErrorInvalidValue;

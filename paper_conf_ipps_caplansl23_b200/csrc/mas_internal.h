@@ -102,6 +102,10 @@ struct PcgState {
     int status;         // mas_status_t
     int pad;
     unsigned long long epoch;  // P2P: solve counter (mailbox sequence numbers)
+    // single-reduction PCG (MODE_CG1): decided by kernel k's last block for k+1
+    double cg_alpha;    // alpha_k
+    double cg_beta;     // beta_k
+    double cg_gamma;    // gamma_k = <r_k, D^-1 r_k>_V
 };
 
 struct Scratch {
@@ -109,22 +113,27 @@ struct Scratch {
     unsigned* ticket;    // one counter per kernel kind
 };
 
-enum { MODE_APPLY = 0, MODE_RESID = 1, MODE_PCGA = 2 };
+// MODE_CG1: the single-reduction (Chronopoulos-Gear) iteration kernel of
+// NEXT-1: its FIRSTK instantiation is the init w0 = L D^-1 r0
+enum { MODE_APPLY = 0, MODE_RESID = 1, MODE_PCGA = 2, MODE_CG1 = 3 };
 
 struct StencilArgs {
     Geo g;
     int chunk;                // r-planes per work item
     int ntj, ntk, nchunk;     // tiles in theta, phi; chunks in r
-    Halo u;                   // APPLY/RESID: x;  PCGA: r (p = D^-1 r + beta p_old)
-    Halo pold;                // PCGA: p_{k-1}
+    Halo u;                   // APPLY/RESID: x;  PCGA: r (p = D^-1 r + beta p_old);  CG1: r_{k-1}
+    Halo pold;                // PCGA: p_{k-1};  CG1: s_{k-2}
+    Halo w;                   // CG1: w_{k-1} = L u_{k-1}
+    double* sout;             // CG1: s_{k-1} = w_{k-1} + beta s_{k-2}
+    double* rout;             // CG1: r_k = r_{k-1} - alpha s_{k-1}
     Halo dinv;                // PCGA: 1/D with halo;  RESID: own only
     Halo kappa;
     TRows tu, tpold, tdinv, tkappa;  // theta-ghost rows (2-D decomposition; zero: none)
     const double* c;          // [nl][nt][np] or nullptr
     const double* f;          // RESID: rhs [ncomp][nl][nt][np]
-    double* out;              // APPLY: y;  RESID: r;  PCGA: q
-    double* pnew;             // PCGA: p_k
-    double* x;                // PCGA: x (deferred update x += alpha_{k-1} p_{k-1})
+    double* out;              // APPLY: y;  RESID: r;  PCGA: q;  CG1: w_k
+    double* pnew;             // PCGA: p_k;  CG1: p (in place: p_{k-2} in, p_{k-1} out)
+    double* x;                // PCGA: x (deferred update x += alpha_{k-1} p_{k-1});  CG1: x_k
     PcgState* st;             // RESID / PCGA
     double* rho_hist;         // [maxit+2]
     double* sigma_hist;       // [maxit+2]

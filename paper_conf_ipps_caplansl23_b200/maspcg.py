@@ -28,7 +28,8 @@ ABI_SYMBOLS = ("mas_comm_unique_id", "mas_partition", "mas_grid_create", "mas_gr
                "mas_op_transport", "mas_op_launch_count", "mas_grid_create_2d",
                "mas_grid_local_extent_2d",
                "mas_op_set_profiling", "mas_op_kernel_times", "mas_op_set_aniso",
-               "mas_op_aniso_time", "mas_op_radial_sums", "mas_op_comm_bench", "mas_op_destroy", "mas_status_string", "mas_last_error", "mas_version")
+               "mas_op_aniso_time", "mas_op_radial_sums", "mas_op_comm_bench", "mas_op_set_single_reduction",
+               "mas_op_single_reduction", "mas_op_destroy", "mas_status_string", "mas_last_error", "mas_version")
 
 
 class MasError(RuntimeError):
@@ -78,6 +79,8 @@ def lib() -> C.CDLL:
             "mas_op_aniso_time": (_i, [_vp, _vp]),
             "mas_op_radial_sums": (_i, [_vp, _vp, _vp, _vp, _vp]),
             "mas_op_comm_bench": (_i, [_vp, _i, _vp, _vp, _vp, _vp]),
+            "mas_op_set_single_reduction": (_i, [_vp, _i]),
+            "mas_op_single_reduction": (_i, [_vp]),
             "mas_op_destroy": (_i, [_vp]),
             "mas_status_string": (C.c_char_p, [_i]),
             "mas_last_error": (C.c_char_p, []),
@@ -314,6 +317,15 @@ def mas_op_comm_bench(op: int, reps: int = 20, stream=None):
     return a.value, b.value, c.value
 
 
+def mas_op_set_single_reduction(op: int, on: bool = True) -> None:
+    """NEXT-1: the single-reduction (Chronopoulos-Gear) PCG loop on this op."""
+    _check(lib().mas_op_set_single_reduction(op, int(bool(on))), "mas_op_set_single_reduction")
+
+
+def mas_op_single_reduction(op: int) -> bool:
+    return int(lib().mas_op_single_reduction(op)) == 1
+
+
 def mas_op_destroy(op: int) -> None:
     _check(lib().mas_op_destroy(op), "mas_op_destroy")
 
@@ -413,6 +425,13 @@ class Operator:
         if kpar is not None:
             _expect(bhat, 3 * self.N, "bhat")
         mas_op_set_aniso(self.h, kpar, bhat, stream)
+
+    def set_single_reduction(self, on=True):
+        mas_op_set_single_reduction(self.h, on)
+
+    @property
+    def single_reduction(self):
+        return mas_op_single_reduction(self.h)
 
     def comm_bench(self, reps=20, stream=None):
         return mas_op_comm_bench(self.h, reps, stream)
