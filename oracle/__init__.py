@@ -253,6 +253,61 @@ class Oracle:
         return rc, x, iters.value, relres.value, hist[: iters.value + 1]
 
 
+    # ---- theta-node placement with pole unknowns (NEXT-2, R29-R30) --------
+    @property
+    def tn_shape(self):
+        nr, nt, np_ = self.shape
+        return (nr, nt + 1, np_)
+
+    def tn_volumes(self):
+        V = np.empty(self.tn_shape)
+        self._chk(lib().mas_ref_tn_volumes(C.byref(self.g), _p(V)))
+        return V
+
+    def tn_apply(self, kappa, c, x):
+        x = _f64(x)
+        ncomp = x.size // int(np.prod(self.tn_shape))
+        y = np.empty_like(x)
+        kappa, c = _f64(kappa), _f64(c)
+        self._chk(lib().mas_ref_tn_apply(C.byref(self.g), ncomp, _p(kappa), _p(c), _p(x), _p(y)))
+        return y
+
+    def tn_diag(self, kappa, c):
+        D = np.empty(self.tn_shape)
+        kappa, c = _f64(kappa), _f64(c)
+        self._chk(lib().mas_ref_tn_diag(C.byref(self.g), _p(kappa), _p(c), _p(D)))
+        return D
+
+    def tn_dirichlet_rhs(self, kappa, f, ub_inner=None, ub_outer=None):
+        f = _f64(f).copy()
+        ncomp = f.size // int(np.prod(self.tn_shape))
+        kappa, ub_inner, ub_outer = _f64(kappa), _f64(ub_inner), _f64(ub_outer)
+        self._chk(lib().mas_ref_tn_dirichlet_rhs(C.byref(self.g), ncomp, _p(kappa), _p(ub_inner),
+                                                 _p(ub_outer), _p(f)))
+        return f
+
+    def tn_dot(self, a, b):
+        a, b = _f64(a), _f64(b)
+        out = C.c_double()
+        self._chk(lib().mas_ref_tn_dot(C.byref(self.g), a.size // int(np.prod(self.tn_shape)), _p(a),
+                                       _p(b), C.byref(out)))
+        return out.value
+
+    def tn_pcg(self, kappa, c, f, x0, tol, maxit):
+        """Returns (status, x, iters, relres, res_hist[:iters+1])."""
+        f = _f64(f)
+        x = _f64(x0).copy()
+        ncomp = f.size // int(np.prod(self.tn_shape))
+        kappa, c = _f64(kappa), _f64(c)
+        iters, relres = C.c_int(), C.c_double()
+        hist = np.zeros(maxit + 1)
+        rc = lib().mas_ref_tn_pcg_solve(C.byref(self.g), ncomp, _p(kappa), _p(c), _p(f), _p(x),
+                                        C.c_double(tol), maxit, C.byref(iters), C.byref(relres),
+                                        _p(hist))
+        self._chk(rc)
+        return rc, x, iters.value, relres.value, hist[: iters.value + 1]
+
+
 def partition(nr: int, nranks: int, rank: int):
     i0, nl = C.c_int(), C.c_int()
     lib().mas_ref_partition(nr, nranks, rank, C.byref(i0), C.byref(nl))

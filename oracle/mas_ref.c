@@ -1081,3 +1081,341 @@ done:
     tables_free(&T);
     return status;
 }
+
+/* ---------------------------------------------------------------------------
+ * theta-node placement with pole unknowns (readings
+ * R29-R30 in DESIGN.md §3.5).  MAS's grid is staggered: some
+ * variables live on the theta "main" mesh tF_j, j = 0..nt, whose end rows sit
+ * ON the poles.  A pole is one point per radius, so a pole row holds a single
+ * value (stored replicated over phi).  The operator is the finite-volume
+ * balance of the same L = c + (1/V) div(kappa grad):
+ *   - interior rows 1..nt-1: theta extent [tC_{j-1}, tC_j] around tF_j,
+ *       V = rC^2 dr * sin(tF_j) (tC_j - tC_{j-1}) * dp,
+ *       theta face at tC_{j-1}: g = dr sin(tC_{j-1}) dp / (tF_j - tF_{j-1}),
+ *       phi face: g = dr (tC_j - tC_{j-1}) / (sin(tF_j) hp),
+ *       r face: g = rF^2 sin(tF_j) (tC_j - tC_{j-1}) dp / hr   (R4 midpoint form);
+ *   - pole rows: the polar cap theta in [0, tC_0] (north; [tC_{nt-1}, pi]
+ *     south) of exact measure A = 1 - cos(tC_0) (1 + cos(tC_{nt-1})), split
+ *     into the np phi slices k of volume V_k = rC^2 dr A dp_k; the cap balance
+ *       V_cap (L u)_pole = sum_k [ V_k c_k u_pole + sum_{r faces} G_{R,k}(u_pole - u_N)
+ *                                  + G_{T,k} (u_pole - u_{row 1 or nt-1, k}) ]
+ *     with V_cap = sum_k V_k, G_{T,k} the theta face at tC_0 of slice k and
+ *     G_{R,k} = kappa_f rF^2 A dp_k / hr: a per-radius sum over phi -- the
+ *     paper's sum0 array reduction (Listings 3-5).
+ * kappa, c per slot as stored (kappa_f the face mean, R6); x's pole rows must
+ * be phi-constant (every slot holds the pole value); y's pole rows are
+ * written replicated.  Arrays [comp][nr][nt+1][np].  The inner product
+ * weights a pole slot with V_k (so a replicated pole row weighs V_cap).
+ * ------------------------------------------------------------------------- */
+typedef struct {
+    double* m;    /* [nt+1] theta measure of row j: sin(tF_j) dtau_j; A_N, A_S at the poles */
+    double* dtau; /* [nt+1] tC_j - tC_{j-1} (interior rows)                                  */
+    double* sT;   /* [nt+1] sin(tC_{j-1}): theta face between rows j-1 and j (j = 1..nt)      */
+    double* hT;   /* [nt+1] tF_j - tF_{j-1}                                                   */
+} tn_tables;
+
+static void tn_free(tn_tables* Q) { free(Q->m); free(Q->dtau); free(Q->sT); free(Q->hT); }
+
+static int tn_make(const mas_ref_grid* g, tn_tables* Q) {
+    int nt = g->nt, j;
+    memset(Q, 0, sizeof(*Q));
+    if (nt < 2) return MAS_REF_ERR_ARG;
+    if (g->tF[0] != 0.0 || fabs(g->tF[nt] - 3.14159265358979323846) > 1e-14) return MAS_REF_ERR_ARG;
+    Q->m = calloc(nt + 1, sizeof(double));
+    Q->dtau = calloc(nt + 1, sizeof(double));
+    Q->sT = calloc(nt + 1, sizeof(double));
+    Q->hT = calloc(nt + 1, sizeof(double));
+    if (!Q->m || !Q->dtau || !Q->sT || !Q->hT) { tn_free(Q); return MAS_REF_ERR_ARG; }
+    for (j = 1; j < nt; j++) {
+        Q->dtau[j] = g->tC[j] - g->tC[j - 1];
+        Q->m[j] = sin(g->tF[j]) * Q->dtau[j];
+    }
+    Q->m[0] = 1.0 - cos(g->tC[0]);        /* north cap measure */
+    Q->m[nt] = 1.0 + cos(g->tC[nt - 1]);  /* south cap measure */
+    for (j = 1; j <= nt; j++) {
+        Q->sT[j] = sin(g->tC[j - 1]);
+        Q->hT[j] = g->tF[j] - g->tF[j - 1];
+    }
+    return MAS_REF_OK;
+}
+
+#define TIDX(g, i, j, k) (((size_t)(i) * ((g)->nt + 1) + (size_t)(j)) * (g)->np + (size_t)(k))
+
+/* one slot (row j, slice k) of radius i: V, the face conductances and the
+ * neighbour slots (r-faces: 0 toward i-1, 1 toward i+1; theta: 2 toward j-1,
+ * 3 toward j+1; phi: 4, 5 -- none on a pole row) */
+static void tn_slot(const mas_ref_grid* g, const tables* T, const tn_tables* Q, int i, int j, int k,
+                    double* V, int kind[6], double gf[6], size_t nb[6]) {
+    int nt = g->nt, np = g->np, f;
+    const int pole = (j == 0 || j == nt);
+    for (f = 0; f < 6; f++) { kind[f] = FACE_NONE; gf[f] = 0.0; nb[f] = 0; }
+    *V = g->rC[i] * g->rC[i] * T->dr[i] * Q->m[j] * T->dp[k];
+    kind[0] = (i > 0) ? FACE_INTERIOR : (g->bc_inner == MAS_REF_DIRICHLET ? FACE_DIRICHLET : FACE_NONE);
+    kind[1] = (i < g->nr - 1) ? FACE_INTERIOR : (g->bc_outer == MAS_REF_DIRICHLET ? FACE_DIRICHLET : FACE_NONE);
+    if (kind[0]) gf[0] = g->rF[i] * g->rF[i] * Q->m[j] * T->dp[k] / T->hr[i];
+    if (kind[1]) gf[1] = g->rF[i + 1] * g->rF[i + 1] * Q->m[j] * T->dp[k] / T->hr[i + 1];
+    if (kind[0] == FACE_INTERIOR) nb[0] = TIDX(g, i - 1, j, k);
+    if (kind[1] == FACE_INTERIOR) nb[1] = TIDX(g, i + 1, j, k);
+    if (j > 0) {  /* theta face at tC_{j-1} */
+        kind[2] = FACE_INTERIOR;
+        gf[2] = T->dr[i] * Q->sT[j] * T->dp[k] / Q->hT[j];
+        nb[2] = TIDX(g, i, j - 1, k);
+    }
+    if (j < nt) { /* theta face at tC_j */
+        kind[3] = FACE_INTERIOR;
+        gf[3] = T->dr[i] * Q->sT[j + 1] * T->dp[k] / Q->hT[j + 1];
+        nb[3] = TIDX(g, i, j + 1, k);
+    }
+    if (!pole) {
+        kind[4] = kind[5] = FACE_INTERIOR;
+        gf[4] = T->dr[i] * Q->dtau[j] / (sin(g->tF[j]) * T->hp[k]);
+        gf[5] = T->dr[i] * Q->dtau[j] / (sin(g->tF[j]) * T->hp[(k + 1) % np]);
+        nb[4] = TIDX(g, i, j, (k + np - 1) % np);
+        nb[5] = TIDX(g, i, j, (k + 1) % np);
+    }
+}
+
+/* the face sum of one slot: sum_f G_f (u - u_N), G_f = kappa_f g_f (as
+ * cell_L's sum, before the division by the volume; the mass term apart) */
+static double tn_slot_flux(const int kind[6], const double gf[6], const size_t nb[6],
+                           double kP, double uP, const double* kappa, const double* u) {
+    double acc = 0.0;
+    int f;
+    for (f = 0; f < 6; f++) {
+        if (kind[f] == FACE_INTERIOR) acc += 0.5 * (kP + kappa[nb[f]]) * gf[f] * (uP - u[nb[f]]);
+        else if (kind[f] == FACE_DIRICHLET) acc += kP * gf[f] * uP;
+    }
+    return acc;
+}
+static double tn_slot_diag(const int kind[6], const double gf[6], const size_t nb[6],
+                           double kP, const double* kappa) {
+    double acc = 0.0;
+    int f;
+    for (f = 0; f < 6; f++) {
+        if (kind[f] == FACE_INTERIOR) acc += 0.5 * (kP + kappa[nb[f]]) * gf[f];
+        else if (kind[f] == FACE_DIRICHLET) acc += kP * gf[f];
+    }
+    return acc;
+}
+
+int mas_ref_tn_volumes(const mas_ref_grid* g, double* V) {
+    tables T;
+    tn_tables Q;
+    int i, j, k, kind[6];
+    double gf[6];
+    size_t nb[6];
+    if (!g || !V || tables_make(g, &T)) return MAS_REF_ERR_ARG;
+    if (tn_make(g, &Q)) { tables_free(&T); return MAS_REF_ERR_ARG; }
+    for (i = 0; i < g->nr; i++)
+        for (j = 0; j <= g->nt; j++)
+            for (k = 0; k < g->np; k++) tn_slot(g, &T, &Q, i, j, k, &V[TIDX(g, i, j, k)], kind, gf, nb);
+    tn_free(&Q);
+    tables_free(&T);
+    return MAS_REF_OK;
+}
+
+int mas_ref_tn_apply(const mas_ref_grid* g, int ncomp, const double* kappa, const double* c,
+                     const double* x, double* y) {
+    tables T;
+    tn_tables Q;
+    size_t N;
+    int i;
+    if (!g || !kappa || !x || !y || ncomp < 1 || tables_make(g, &T)) return MAS_REF_ERR_ARG;
+    if (tn_make(g, &Q)) { tables_free(&T); return MAS_REF_ERR_ARG; }
+    N = (size_t)g->nr * (g->nt + 1) * g->np;
+#pragma omp parallel for schedule(static)
+    for (i = 0; i < g->nr; i++) {
+        int j, k, m, kind[6];
+        double gf[6], V;
+        size_t nb[6];
+        for (m = 0; m < ncomp; m++) {
+            const double* u = x + (size_t)m * N;
+            double* out = y + (size_t)m * N;
+            for (j = 0; j <= g->nt; j++) {
+                if (j == 0 || j == g->nt) {
+                    /* the polar cap: sum the slices' balances over phi (sum0) */
+                    double num = 0.0, vcap = 0.0;
+                    for (k = 0; k < g->np; k++) {
+                        size_t P = TIDX(g, i, j, k);
+                        tn_slot(g, &T, &Q, i, j, k, &V, kind, gf, nb);
+                        num += V * (c ? c[P] : 0.0) * u[P] + tn_slot_flux(kind, gf, nb, kappa[P], u[P], kappa, u);
+                        vcap += V;
+                    }
+                    for (k = 0; k < g->np; k++) out[TIDX(g, i, j, k)] = num / vcap;
+                } else {
+                    for (k = 0; k < g->np; k++) {
+                        size_t P = TIDX(g, i, j, k);
+                        tn_slot(g, &T, &Q, i, j, k, &V, kind, gf, nb);
+                        out[P] = (c ? c[P] : 0.0) * u[P] + tn_slot_flux(kind, gf, nb, kappa[P], u[P], kappa, u) / V;
+                    }
+                }
+            }
+        }
+    }
+    tn_free(&Q);
+    tables_free(&T);
+    return MAS_REF_OK;
+}
+
+int mas_ref_tn_diag(const mas_ref_grid* g, const double* kappa, const double* c, double* D) {
+    tables T;
+    tn_tables Q;
+    int i;
+    if (!g || !kappa || !D || tables_make(g, &T)) return MAS_REF_ERR_ARG;
+    if (tn_make(g, &Q)) { tables_free(&T); return MAS_REF_ERR_ARG; }
+#pragma omp parallel for schedule(static)
+    for (i = 0; i < g->nr; i++) {
+        int j, k, kind[6];
+        double gf[6], V;
+        size_t nb[6];
+        for (j = 0; j <= g->nt; j++) {
+            if (j == 0 || j == g->nt) {
+                double num = 0.0, vcap = 0.0;
+                for (k = 0; k < g->np; k++) {
+                    size_t P = TIDX(g, i, j, k);
+                    tn_slot(g, &T, &Q, i, j, k, &V, kind, gf, nb);
+                    num += V * (c ? c[P] : 0.0) + tn_slot_diag(kind, gf, nb, kappa[P], kappa);
+                    vcap += V;
+                }
+                for (k = 0; k < g->np; k++) D[TIDX(g, i, j, k)] = num / vcap;
+            } else {
+                for (k = 0; k < g->np; k++) {
+                    size_t P = TIDX(g, i, j, k);
+                    tn_slot(g, &T, &Q, i, j, k, &V, kind, gf, nb);
+                    D[P] = (c ? c[P] : 0.0) + tn_slot_diag(kind, gf, nb, kappa[P], kappa) / V;
+                }
+            }
+        }
+    }
+    tn_free(&Q);
+    tables_free(&T);
+    return MAS_REF_OK;
+}
+
+/* f += (1/V) G_b u_b on the Dirichlet r-faces (pole rows: the cap sum). */
+int mas_ref_tn_dirichlet_rhs(const mas_ref_grid* g, int ncomp, const double* kappa,
+                             const double* ub_inner, const double* ub_outer, double* f) {
+    tables T;
+    tn_tables Q;
+    size_t N, plane;
+    int m, side, j, k, kind[6];
+    double gf[6], V;
+    size_t nb[6];
+    if (!g || !kappa || !f || ncomp < 1 || tables_make(g, &T)) return MAS_REF_ERR_ARG;
+    if (tn_make(g, &Q)) { tables_free(&T); return MAS_REF_ERR_ARG; }
+    N = (size_t)g->nr * (g->nt + 1) * g->np;
+    plane = (size_t)(g->nt + 1) * g->np;
+    for (m = 0; m < ncomp; m++)
+        for (side = 0; side < 2; side++) {
+            const double* ub = side ? ub_outer : ub_inner;
+            const int i = side ? g->nr - 1 : 0, face = side ? 1 : 0;
+            if (!ub || (side ? g->bc_outer : g->bc_inner) != MAS_REF_DIRICHLET) continue;
+            for (j = 0; j <= g->nt; j++) {
+                double num = 0.0, vcap = 0.0;
+                for (k = 0; k < g->np; k++) {
+                    size_t P = TIDX(g, i, j, k);
+                    tn_slot(g, &T, &Q, i, j, k, &V, kind, gf, nb);
+                    const double t = kappa[P] * gf[face] * ub[(size_t)m * plane + (size_t)j * g->np + k];
+                    if (j == 0 || j == g->nt) { num += t; vcap += V; }
+                    else f[(size_t)m * N + P] += t / V;
+                }
+                if (j == 0 || j == g->nt)
+                    for (k = 0; k < g->np; k++) f[(size_t)m * N + TIDX(g, i, j, k)] += num / vcap;
+            }
+        }
+    tn_free(&Q);
+    tables_free(&T);
+    return MAS_REF_OK;
+}
+
+/* <a,b>_V over the theta-node slots, per r-plane in (j,k) order, then planes,
+ * then components (as dot_planes). */
+static double tn_dot_raw(const mas_ref_grid* g, const double* V, int ncomp, const double* a,
+                         const double* b) {
+    size_t plane = (size_t)(g->nt + 1) * g->np, N = plane * g->nr;
+    double s = 0.0;
+    int m, i;
+    for (m = 0; m < ncomp; m++)
+        for (i = 0; i < g->nr; i++) {
+            double ps = 0.0;
+            size_t e;
+            for (e = 0; e < plane; e++) {
+                size_t P = (size_t)i * plane + e;
+                ps += V[P] * a[(size_t)m * N + P] * b[(size_t)m * N + P];
+            }
+            s += ps;
+        }
+    return s;
+}
+
+int mas_ref_tn_dot(const mas_ref_grid* g, int ncomp, const double* a, const double* b, double* out) {
+    double* V;
+    if (!g || !a || !b || !out || ncomp < 1) return MAS_REF_ERR_ARG;
+    V = malloc(sizeof(double) * (size_t)g->nr * (g->nt + 1) * g->np);
+    if (!V || mas_ref_tn_volumes(g, V)) { free(V); return MAS_REF_ERR_ARG; }
+    *out = tn_dot_raw(g, V, ncomp, a, b);
+    free(V);
+    return MAS_REF_OK;
+}
+
+/* Jacobi-PCG on the theta-node operator: the textbook loop of pcg_core
+ * (R10-R12) with mas_ref_tn_apply / _diag / the theta-node inner product. */
+int mas_ref_tn_pcg_solve(const mas_ref_grid* g, int ncomp, const double* kappa, const double* c,
+                         const double* f, double* x, double tol, int maxit, int* iters,
+                         double* relres, double* res_hist) {
+    size_t N, n, e;
+    double *V, *D, *r, *z, *p, *q;
+    double bn, rn, rho, sigma, alpha, rho_new, beta;
+    int k, m, status = MAS_REF_NOT_CONVERGED;
+    if (!g || !kappa || !f || !x || !iters || !relres || ncomp < 1 || maxit < 0 || !(tol >= 0.0))
+        return MAS_REF_ERR_ARG;
+    N = (size_t)g->nr * (g->nt + 1) * g->np;
+    n = N * ncomp;
+    V = malloc(sizeof(double) * N);
+    D = malloc(sizeof(double) * N);
+    r = malloc(sizeof(double) * n);
+    z = malloc(sizeof(double) * n);
+    p = malloc(sizeof(double) * n);
+    q = malloc(sizeof(double) * n);
+    if (!V || !D || !r || !z || !p || !q || mas_ref_tn_volumes(g, V) || mas_ref_tn_diag(g, kappa, c, D)) {
+        status = MAS_REF_ERR_ARG; goto done;
+    }
+    bn = sqrt(tn_dot_raw(g, V, ncomp, f, f));
+    if (bn == 0.0) {
+        for (e = 0; e < n; e++) x[e] = 0.0;
+        *iters = 0; *relres = 0.0;
+        if (res_hist) res_hist[0] = 0.0;
+        status = MAS_REF_OK; goto done;
+    }
+    mas_ref_tn_apply(g, ncomp, kappa, c, x, r);
+    for (e = 0; e < n; e++) r[e] = f[e] - r[e];
+    rn = sqrt(tn_dot_raw(g, V, ncomp, r, r));
+    if (res_hist) res_hist[0] = rn;
+    if (rn <= tol * bn) { *iters = 0; *relres = rn / bn; status = MAS_REF_OK; goto done; }
+    for (m = 0; m < ncomp; m++)
+        for (e = 0; e < N; e++) z[m * N + e] = r[m * N + e] / D[e];
+    memcpy(p, z, sizeof(double) * n);
+    rho = tn_dot_raw(g, V, ncomp, r, z);
+    for (k = 1; k <= maxit; k++) {
+        mas_ref_tn_apply(g, ncomp, kappa, c, p, q);
+        sigma = tn_dot_raw(g, V, ncomp, p, q);
+        if (!(sigma > 0.0) || !isfinite(sigma)) {
+            *iters = k; *relres = rn / bn; status = MAS_REF_ERR_BREAKDOWN; goto done;
+        }
+        alpha = rho / sigma;
+        for (e = 0; e < n; e++) { x[e] += alpha * p[e]; r[e] -= alpha * q[e]; }
+        rn = sqrt(tn_dot_raw(g, V, ncomp, r, r));
+        if (res_hist) res_hist[k] = rn;
+        if (rn <= tol * bn) { *iters = k; *relres = rn / bn; status = MAS_REF_OK; goto done; }
+        for (m = 0; m < ncomp; m++)
+            for (e = 0; e < N; e++) z[m * N + e] = r[m * N + e] / D[e];
+        rho_new = tn_dot_raw(g, V, ncomp, r, z);
+        beta = rho_new / rho;
+        rho = rho_new;
+        for (e = 0; e < n; e++) p[e] = z[e] + beta * p[e];
+    }
+    *iters = maxit; *relres = rn / bn; status = MAS_REF_NOT_CONVERGED;
+done:
+    free(V); free(D); free(r); free(z); free(p); free(q);
+    return status;
+}

@@ -153,4 +153,20 @@ int mas_ref_radial_sums(const mas_ref_grid* g, int ncomp, const double* x, const
 #ifdef __cplusplus
 }
 #endif
+/* theta-node placement with pole unknowns (NEXT-2, readings R29-R30,
+ * mas_ref.c): arrays [comp][nr][nt+1][np]; rows 0 and nt are the poles (one
+ * value per radius, stored replicated over phi); the grid must have tF[0] = 0
+ * and tF[nt] = pi.  volumes [nr][nt+1][np]: V of each slot (pole slots: the
+ * cap slices rC^2 dr A dp_k). */
+int mas_ref_tn_volumes(const mas_ref_grid* g, double* V);
+int mas_ref_tn_apply(const mas_ref_grid* g, int ncomp, const double* kappa, const double* c,
+                     const double* x, double* y);
+int mas_ref_tn_diag(const mas_ref_grid* g, const double* kappa, const double* c, double* D);
+int mas_ref_tn_dirichlet_rhs(const mas_ref_grid* g, int ncomp, const double* kappa,
+                             const double* ub_inner, const double* ub_outer, double* f);
+int mas_ref_tn_dot(const mas_ref_grid* g, int ncomp, const double* a, const double* b, double* out);
+int mas_ref_tn_pcg_solve(const mas_ref_grid* g, int ncomp, const double* kappa, const double* c,
+                         const double* f, double* x, double tol, int maxit, int* iters,
+                         double* relres, double* res_hist);
+
 #endif
