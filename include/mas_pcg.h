@@ -155,6 +155,31 @@ MAS_API mas_status_t mas_op_setup(mas_grid_t* g, int ncomp, const double* kappa,
                           mas_bc_t bc_r_outer, cudaStream_t stream,
                           mas_op_t** out);
 
+/* Variable placement on MAS's staggered mesh (the
+ * paper's "staggered spherical grid").  MAS_PLACE_CELL: unknowns
+ * at cell centres (rC, tC, pC) -- mas_op_setup.  MAS_PLACE_THETA_NODE:
+ * unknowns at (rC_i, tF_j, pC_k), j = 0..nt, on the theta main mesh, whose
+ * rows 0 and nt lie ON the poles (readings R29-R30): every
+ * per-cell array of the op is then [comp][nr_local][nt+1][np]; a pole row
+ * holds ONE value per radius, stored replicated over phi.  The operator is
+ * the same L = c + (1/V) div(kappa grad) on the dual theta cells
+ * [tC_{j-1}, tC_j]; a pole's equation is the balance of its polar cap
+ * (theta in [0, tC_0]), the phi sum of its slices' fluxes to row 1 -- the
+ * paper's per-radius sum0 array reduction (Listings 3-5, P:428-445,
+ * P:592-645), done on the GPU by k_pole_avg after every stencil pass.
+ * kappa and c may vary over a pole row's slots (each slot is a cap slice);
+ * rhs and x0 pole rows are taken as one value (x0's are replaced by their
+ * dp-weighted phi average; rhs must be phi-constant there).  Needs both pole
+ * flags, nt >= 2 and ptheta == 1; r-slabs run the NCCL loop (no P2P, no
+ * field-aligned term, no single-reduction loop).  Outputs of apply / diag /
+ * dirichlet_rhs / solve have phi-constant pole rows.
+ * Errors: as mas_op_setup; MAS_ERR_ARG for an unknown placement or a grid
+ * without both poles. */
+enum { MAS_PLACE_CELL = 0, MAS_PLACE_THETA_NODE = 1 };
+MAS_API mas_status_t mas_op_setup_placed(mas_grid_t* g, int ncomp, int placement, const double* kappa,
+                                         const double* mass, mas_bc_t bc_r_inner,
+                                         mas_bc_t bc_r_outer, cudaStream_t stream, mas_op_t** out);
+
 /* Replace kappa and c (e.g. kappa = T^{5/2} each implicit step); same checks. */
 MAS_API mas_status_t mas_op_update(mas_op_t* op, const double* kappa, const double* mass,
                            cudaStream_t stream);

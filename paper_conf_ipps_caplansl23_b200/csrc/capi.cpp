@@ -157,6 +157,9 @@ struct mas_op {
     // w = L D^-1 r and s = L p (r: r / r2, w: q / w2, s: p[0] / p[1]), p in place
     int cg1 = 0;
     double *r2 = nullptr, *w2 = nullptr, *pcg = nullptr;
+    // placement (NEXT-2): 0 cell centres; 1 theta nodes with pole rows (local
+    // rows 0 and nt hold one value per radius: k_pole_avg after every stencil)
+    int tnode = 0;
     cudaGraphExec_t gexec1 = nullptr;
     const double* g1_x = nullptr;
     double* atab = nullptr;                      // AnisoTab arrays (device)
@@ -245,9 +248,29 @@ mas_status_t mas_grid_create_2d(int nr, int nt, int np, const double* r_node, co
         set_last_error("cudaMemcpy tables");
         return MAS_ERR_CUDA;
     }
+    if (pole_flags == (MAS_POLE_NORTH | MAS_POLE_SOUTH) && ptheta == 1 && nt >= 2) {
+        // the theta-node placement's tables (NEXT-2): both poles on the mesh
+        const std::vector<double> tn = tnode_tables(g);
+        s = dmalloc(&g->d_tab_tn, tn.size());
+        if (s == MAS_OK && cudaMemcpy(g->d_tab_tn, tn.data(), tn.size() * sizeof(double),
+                                      cudaMemcpyHostToDevice) != cudaSuccess)
+            s = MAS_ERR_CUDA;
+        if (s != MAS_OK) {
+            cudaFree(g->d_tab);
+            if (g->d_tab_tn) cudaFree(g->d_tab_tn);
+            delete g;
+            set_last_error("theta-node tables");
+            return s;
+        }
+    }
     if (dist) {  // nranks == 1 with a real NCCL id: a 1-rank communicator (the NCCL loop on one GPU)
         s = comm_create(dist, &g->comm);
-        if (s != MAS_OK) { cudaFree(g->d_tab); delete g; return s; }
+        if (s != MAS_OK) {
+            cudaFree(g->d_tab);
+            if (g->d_tab_tn) cudaFree(g->d_tab_tn);
+            delete g;
+            return s;
+        }
     }
     *out = g;
     return MAS_OK;
@@ -281,6 +304,7 @@ mas_status_t mas_grid_local_extent_2d(const mas_grid_t* g, int* i0, int* nr_loca
 mas_status_t mas_grid_destroy(mas_grid_t* g) {
     if (!g) return MAS_OK;
     if (g->d_tab) cudaFree(g->d_tab);
+    if (g->d_tab_tn) cudaFree(g->d_tab_tn);
     comm_destroy(g->comm);
     delete g;
     return MAS_OK;
@@ -401,10 +425,19 @@ static const double* aniso_ca_hi(const mas_op* op) {
 // term's diagonal (R26) when L_par is on (D then goes through a device buffer:
 // the caller's, or q, which is free outside a solve).
 static mas_status_t op_diag(mas_op* op, double* D_out, cudaStream_t s) {
-    double* D = op->aniso && !D_out ? op->q : D_out;
+    double* D = (op->aniso || op->tnode) && !D_out ? op->q : D_out;
     CU(launch_diag(op->geo, halo_of(op, op->kappa, op->kg, 1), packed_rows(op, op->kgt, 1), op->c, D,
                    op->dinv, op->bad, s));
     if (op->aniso) CU(launch_aniso_diag(op->geo, op->ca, aniso_ca_hi(op), D, op->dinv, op->bad, s));
+    // theta nodes: a pole row's diagonal is the cap's (the phi average of its
+    // slices' diagonals), 1/D from that
+    if (op->tnode) CU(launch_pole_avg(op->geo, 1, D, op->dinv, 0, op->geo.nl, s));
+    return MAS_OK;
+}
+
+// theta nodes: the pole rows of an ncomp-field (all local planes)
+static mas_status_t pole_pass(const mas_op* op, double* y, int ncomp, cudaStream_t s) {
+    if (op->tnode) CU(launch_pole_avg(op->geo, ncomp, y, nullptr, 0, op->geo.nl, s));
     return MAS_OK;
 }
 
@@ -546,6 +579,8 @@ static mas_status_t loop_graph(mas_op* op, StencilArgs a, StreamArgs b, AnisoArg
                 an1.u = aniso_p_halo(op, 1);
                 e = launch_aniso(MODE_PCGA, an1, op->cap_stream);
             }
+            if (e == cudaSuccess && op->tnode)
+                e = launch_pole_avg(op->geo, nc, op->q, nullptr, 0, op->geo.nl, op->cap_stream);
             if (e == cudaSuccess) e = launch_pcg_b(b, op->b_blocks, op->cap_stream);
             cudaGraph_t out = g;
             cudaError_t e2 = cudaStreamEndCapture(op->cap_stream, &out);
@@ -588,6 +623,8 @@ static mas_status_t loop_graph(mas_op* op, StencilArgs a, StreamArgs b, AnisoArg
                 e = launch_stencil(MODE_PCGA, nc, a, op->cap_stream);
                 an.u = aniso_p_halo(op, kk);
                 if (e == cudaSuccess && op->aniso) e = launch_aniso(MODE_PCGA, an, op->cap_stream);
+                if (e == cudaSuccess && op->tnode)
+                    e = launch_pole_avg(op->geo, nc, op->q, nullptr, 0, op->geo.nl, op->cap_stream);
                 if (e == cudaSuccess) e = launch_pcg_b(b, op->b_blocks, op->cap_stream);
             }
             cudaGraph_t out = body;
@@ -807,11 +844,20 @@ extern "C" {
 mas_status_t mas_op_setup(mas_grid_t* g, int ncomp, const double* kappa, const double* mass,
                           mas_bc_t bc_r_inner, mas_bc_t bc_r_outer, cudaStream_t stream,
                           mas_op_t** out) {
+    return mas_op_setup_placed(g, ncomp, MAS_PLACE_CELL, kappa, mass, bc_r_inner, bc_r_outer, stream, out);
+}
+
+mas_status_t mas_op_setup_placed(mas_grid_t* g, int ncomp, int placement, const double* kappa,
+                                 const double* mass, mas_bc_t bc_r_inner, mas_bc_t bc_r_outer,
+                                 cudaStream_t stream, mas_op_t** out) {
     NvtxRange nvtx("mas_op_setup");
     if (!out) return arg_error("null out");
     *out = nullptr;
     if (!g || !kappa) return arg_error("null grid or kappa");
     if (ncomp != 1 && ncomp != 3) return arg_error("ncomp must be 1 or 3");
+    if (placement != MAS_PLACE_CELL && placement != MAS_PLACE_THETA_NODE) return arg_error("unknown placement");
+    if (placement == MAS_PLACE_THETA_NODE && !g->d_tab_tn)
+        return arg_error("theta-node placement needs both pole flags, nt >= 2 and ptheta == 1");
     if ((bc_r_inner != MAS_BC_DIRICHLET && bc_r_inner != MAS_BC_NEUMANN) ||
         (bc_r_outer != MAS_BC_DIRICHLET && bc_r_outer != MAS_BC_NEUMANN))
         return arg_error("bad boundary condition");
@@ -821,7 +867,9 @@ mas_status_t mas_op_setup(mas_grid_t* g, int ncomp, const double* kappa, const d
     op->ncomp = ncomp;
     op->bci = bc_r_inner;
     op->bco = bc_r_outer;
-    const int nl = g->nl, nt = g->ntl, np = g->np;  // local block [nl][ntl][np]
+    op->tnode = placement == MAS_PLACE_THETA_NODE;
+    // local block [nl][ntl][np]; theta nodes: [nl][nt+1][np]
+    const int nl = g->nl, nt = op->tnode ? g->nt + 1 : g->ntl, np = g->np;
     const long long plane = (long long)nt * np;
     op->Nl = (long long)nl * plane;
     if ((long long)ncomp * op->Nl >= (1LL << 31)) {  // the stencil kernels index with 32-bit offsets
@@ -905,10 +953,16 @@ mas_status_t mas_op_setup(mas_grid_t* g, int ncomp, const double* kappa, const d
     const double* t = g->d_tab;
     G.irc2 = t; t += nl;
     G.vr = t; t += nl;
-    G.wTm = t; t += nt;
-    G.wTp = t; t += nt;
-    G.isc2 = t; t += nt;
-    G.vt = t; t += nt;
+    G.wTm = t; t += g->ntl;
+    G.wTp = t; t += g->ntl;
+    G.isc2 = t; t += g->ntl;
+    G.vt = t; t += g->ntl;
+    if (op->tnode) {  // the theta part of the geometry: the theta-node rows (NEXT-2)
+        G.wTm = g->d_tab_tn;
+        G.wTp = g->d_tab_tn + nt;
+        G.isc2 = g->d_tab_tn + 2 * nt;
+        G.vt = g->d_tab_tn + 3 * nt;
+    }
     G.wPm = t; t += np;
     G.wPp = t; t += np;
     G.vp = t;
@@ -1009,6 +1063,7 @@ mas_status_t mas_op_apply(const mas_op_t* op_c, const double* x, double* y, cuda
     CU(launch_stencil(MODE_APPLY, op->ncomp, a, stream));
     if (op->aniso)
         CU(launch_aniso(MODE_APPLY, aniso_args(op, MODE_APPLY, halo_of(op, xd, op->xg, 1), yd), stream));
+    ST(pole_pass(op, yd, op->ncomp, stream));
     if (hy) {
         CU(cudaMemcpyAsync(y, yd, bytes, cudaMemcpyDeviceToHost, stream));
         CU(cudaStreamSynchronize(stream));
@@ -1040,6 +1095,8 @@ mas_status_t mas_op_dirichlet_rhs(const mas_op_t* op_c, const double* ub_inner,
             ubd = ubuf;
         }
         CU(launch_dirichlet(op->geo, op->ncomp, op->kappa, ubd, side, fd, stream));
+        if (op->tnode)  // the cap's boundary term: phi average over the pole row's slices
+            CU(launch_pole_avg(op->geo, op->ncomp, fd, nullptr, side ? op->geo.nl - 1 : 0, 1, stream));
     }
     if (hf) CU(cudaMemcpyAsync(f_inout, fd, fbytes, cudaMemcpyDeviceToHost, stream));
     if (ubuf || hf) CU(cudaStreamSynchronize(stream));
@@ -1111,6 +1168,7 @@ mas_status_t mas_op_radial_sums(const mas_op_t* op_c, const double* x, const dou
 mas_status_t mas_op_enable_p2p(mas_op_t* op, cudaStream_t s) {
     if (!op) return arg_error("null op");
     if (op->p2p) return MAS_OK;
+    if (op->tnode) return arg_error("P2P transport: cell-centred placement only (theta nodes keep NCCL)");
     Comm* comm = op->g->comm;
     const int P = comm_nranks(comm), rank = comm_rank(comm);
     const bool virt = comm_is_virtual(comm);
@@ -1220,6 +1278,7 @@ mas_status_t mas_op_set_single_reduction(mas_op_t* op, int on) {
     }
     if (op->g->comm) return arg_error("single-reduction PCG: one GPU only (no mas_dist_t)");
     if (op->aniso) return arg_error("single-reduction PCG: isotropic operator only (no mas_op_set_aniso)");
+    if (op->tnode) return arg_error("single-reduction PCG: cell-centred placement only");
     const size_t n = op->ncomp * (size_t)op->Nl;
     if (!op->r2) ST(dmalloc(&op->r2, n));
     if (!op->w2) ST(dmalloc(&op->w2, n));
@@ -1307,6 +1366,7 @@ mas_status_t mas_op_set_aniso(mas_op_t* op, const double* kpar, const double* bh
     }
     if (!bhat) return arg_error("null bhat");
     if (op->cg1) return arg_error("field-aligned conduction: switch the single-reduction loop off first");
+    if (op->tnode) return arg_error("field-aligned conduction: cell-centred placement only");
     if (op->ncomp != 1) return arg_error("field-aligned conduction needs ncomp == 1");
     if (op->g->ptheta > 1)
         return arg_error("field-aligned conduction: r-slab decompositions only (ptheta == 1)");
@@ -1450,6 +1510,7 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
     double* rr_h = op->hist + 2 * op->hist_cap;
 
     // a3: r = f - L x0 and the three initial dot products
+    ST(pole_pass(op, xd, nc, s));  // theta nodes: x0's pole rows are one value each (their average)
     if (comm) ST(comm_seams(comm, xd, nc, op->g->nl, plane, op->xg, op->xg + nc * plane, s, rstride(op)));
     ST(tseams(op, xd, nc, op->xgt, s));
     StencilArgs a{};
@@ -1482,6 +1543,11 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
         CU(launch_aniso(MODE_RESID, an, s));
         op->launches++;
         an = aniso_args(op, MODE_PCGA, Halo{}, op->q);
+    }
+    if (op->tnode) {  // the caps' residuals, then the three sums again
+        ST(pole_pass(op, op->r, nc, s));
+        CU(launch_init_dots(op->geo, nc, fd, op->r, op->dinv, op->scr, op->st, op->b_blocks, s));
+        op->launches += 2;
     }
     if (comm && !p2p) ST(comm_allreduce(comm, &op->st->pend_rho, 3, s));  // rho, rr, ff
 
@@ -1524,6 +1590,7 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
                 an.u = aniso_p_halo(op, 1);
                 CU(launch_aniso(MODE_PCGA, an, s));
             }
+            ST(pole_pass(op, op->q, nc, s));
             CU(launch_pcg_b(b, op->b_blocks, s));
         }
         CU(cudaGraphLaunch(op->gexec, s));
@@ -1602,6 +1669,10 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
         if (comm && !p2p) ST(comm_allreduce(comm, &op->st->pend_sigma, 1, s));
         if (k <= maxit) {
             if (p2p) ST(comm_vsync(comm, s));  // virtual P2P ranks: all A(k) done
+            if (op->tnode) {  // the caps of q = L p (theta nodes, NEXT-2)
+                ST(pole_pass(op, op->q, nc, s));
+                op->launches++;
+            }
             if (pe) CU(cudaEventRecord(pe[2], s));
             CU(launch_pcg_b(b, op->b_blocks, s));
             op->launches++;
@@ -1637,7 +1708,7 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
     if (graph) {  // iteration 1 + 4 kernels per executed loop body (iterations 2k, 2k+1)
         const int last_a = fin.status == MAS_ERR_BREAKDOWN ? fin.iters : fin.iters + 1;
         const int bodies = last_a <= 2 ? 1 : last_a / 2;
-        const int per = op->aniso ? 3 : 2;  // kernels per iteration
+        const int per = 2 + (op->aniso ? 1 : 0) + (op->tnode ? 1 : 0);  // kernels per iteration
         op->launches += per + 2LL * per * bodies;
     }
     if (res_hist) {

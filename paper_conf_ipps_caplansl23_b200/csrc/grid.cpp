@@ -124,4 +124,27 @@ void build_tables(mas_grid* g) {
     }
 }
 
+// theta-node placement (NEXT-2, readings R29-R30):
+// rows j = 0..nt at tF_j; interior rows span [tC_{j-1}, tC_j] (theta measure
+// m_j = sin(tF_j)(tC_j - tC_{j-1})), the pole rows are polar-cap slices of
+// measure A = 1 - cos(tC_0) (north) and 1 + cos(tC_{nt-1}) (south) without
+// phi faces.  Same layout as Tables' theta part: [wTm | wTp | isc2 | vt](nt+1).
+std::vector<double> tnode_tables(const mas_grid* g) {
+    const int nt = g->nt;
+    const double *tF = g->tF.data(), *tC = g->tC.data();
+    std::vector<double> t(4 * (size_t)(nt + 1), 0.0);
+    double *wTm = t.data(), *wTp = wTm + nt + 1, *isc2 = wTp + nt + 1, *vt = isc2 + nt + 1;
+    for (int j = 0; j <= nt; j++) {
+        double m;
+        if (j == 0) m = 1.0 - std::cos(tC[0]);
+        else if (j == nt) m = 1.0 + std::cos(tC[nt - 1]);
+        else m = std::sin(tF[j]) * (tC[j] - tC[j - 1]);
+        vt[j] = m;
+        if (j > 0) wTm[j] = std::sin(tC[j - 1]) / ((tF[j] - tF[j - 1]) * m);
+        if (j < nt) wTp[j] = std::sin(tC[j]) / ((tF[j + 1] - tF[j]) * m);
+        if (j > 0 && j < nt) isc2[j] = 1.0 / (std::sin(tF[j]) * std::sin(tF[j]));  // pole rows: no phi faces
+    }
+    return t;
+}
+
 }  // namespace mas

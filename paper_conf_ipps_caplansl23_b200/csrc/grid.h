@@ -28,6 +28,7 @@ struct mas_grid {
     std::vector<double> rF, rC, tF, tC, pF, pC;
     mas::Tables tab;
     double* d_tab = nullptr;  // device copy of the theta/phi tables + irc2/vr
+    double* d_tab_tn = nullptr;  // theta-node placement: [wTm wTp isc2 vt](nt+1) (both poles, ptheta 1)
     mas::Comm* comm = nullptr;
 };
 
@@ -38,6 +39,7 @@ int validate_mesh(int nr, int nt, int np, const double* rF, const double* rC, co
                   int periodic_phi, int pr, int ptheta, std::string* why);
 void partition(int nr, int nranks, int rank, int* i0, int* nl);
 void build_tables(mas_grid* g);
+std::vector<double> tnode_tables(const mas_grid* g);
 
 // ---- comm.cpp -------------------------------------------------------------
 mas_status_t comm_unique_id(unsigned char out[128]);

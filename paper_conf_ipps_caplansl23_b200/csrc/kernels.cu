@@ -1209,8 +1209,91 @@ __global__ void __launch_bounds__(kThreads) k_radial_sums(const Geo g, const dou
 }
 
 // --------------------------------------------------------------------------
+// theta-node placement (NEXT-2, readings R29-R30): the pole
+// rows 0 and nt (local rows 0 and g.nt-1) hold one value per radius.  The
+// stencil kernels compute each phi slot k of a pole row as its own polar-cap
+// slice (volume V_k = rC^2 dr A dp_k); the cap balance is the dp-weighted
+// phi average of the slices -- the paper's per-radius sum0 array reduction
+// (Listings 3-5) -- written back to every slot.
+// One block per (component, plane, pole); fixed-order tree (deterministic).
+// dinv != nullptr (the Jacobi diagonal, ncomp = 1): dinv = 1 / average too.
+// --------------------------------------------------------------------------
+__global__ void __launch_bounds__(kThreads) k_pole_avg(const Geo g, double* y, double* dinv, int plane_lo,
+                                                        int nplanes) {
+    __shared__ double ws[2][kThreads / 32];
+    __shared__ double avg;
+    const int pole = blockIdx.x & 1;
+    const int q = blockIdx.x >> 1;             // comp * nplanes + plane
+    const int comp = q / nplanes, il = plane_lo + q % nplanes;
+    const int row = pole ? g.nt - 1 : 0;
+    double* yr = y + ((long long)comp * g.nl + il) * g.plane + (long long)row * g.np;
+    double s = 0.0, w = 0.0;
+    for (int k = threadIdx.x; k < g.np; k += kThreads) {
+        const double dp = __ldg(g.vp + k);
+        s = fma(dp, yr[k], s);
+        w += dp;
+    }
+    s = warp_sum(s);
+    w = warp_sum(w);
+    if ((threadIdx.x & 31) == 0) ws[0][threadIdx.x >> 5] = s, ws[1][threadIdx.x >> 5] = w;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        double ts = 0.0, tw = 0.0;
+        for (int t = 0; t < kThreads / 32; t++) ts += ws[0][t], tw += ws[1][t];
+        avg = ts / tw;
+    }
+    __syncthreads();
+    const double a = avg;
+    for (int k = threadIdx.x; k < g.np; k += kThreads) {
+        yr[k] = a;
+        if (dinv) dinv[(long long)il * g.plane + (long long)row * g.np + k] = 1.0 / a;
+    }
+}
+
+// <f,f>_V, <r,r>_V, <r,D^-1 r>_V of the init (after the pole rows of r were
+// averaged) into PcgState: the values k_stencil<RESID> computed per slot are
+// replaced.  Same grid-stride row order as kernel B.
+__global__ void __launch_bounds__(kThreads) k_init_dots(const Geo g, int ncomp, const double* f, const double* r,
+                                                         const double* dinv, Scratch scr, PcgState* st) {
+    double acc[3] = {0.0, 0.0, 0.0};
+    const long long Nl = (long long)g.nl * g.plane;
+    const int rows = g.nl * g.nt;
+    for (int row = blockIdx.x; row < rows; row += gridDim.x) {
+        const int i = row / g.nt, j = row - i * g.nt;
+        const double wrow = g.vr[i] * g.vt[j];
+        const long long base = (long long)row * g.np;
+        for (int k = threadIdx.x; k < g.np; k += kThreads) {
+            const double V = wrow * g.vp[k], di = dinv[base + k];
+            for (int c = 0; c < ncomp; c++) {
+                const double fv = f[c * Nl + base + k], rv = r[c * Nl + base + k];
+                acc[0] += V * fv * fv;
+                acc[1] += V * rv * rv;
+                acc[2] += V * rv * (di * rv);
+            }
+        }
+    }
+    if (grid_reduce<3>(acc, scr, TKT_DOT) && threadIdx.x == 0) {
+        st->pend_ff = acc[0];
+        st->pend_rr = acc[1];
+        st->pend_rho = acc[2];
+    }
+}
+
+// --------------------------------------------------------------------------
 // launchers
 // --------------------------------------------------------------------------
+cudaError_t launch_pole_avg(const Geo& g, int ncomp, double* y, double* dinv, int plane_lo, int nplanes,
+                            cudaStream_t s) {
+    if (nplanes <= 0) return cudaSuccess;
+    k_pole_avg<<<2 * ncomp * nplanes, kThreads, 0, s>>>(g, y, dinv, plane_lo, nplanes);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_init_dots(const Geo& g, int ncomp, const double* f, const double* r, const double* dinv,
+                             Scratch scr, PcgState* st, int nblocks, cudaStream_t s) {
+    k_init_dots<<<nblocks, kThreads, 0, s>>>(g, ncomp, f, r, dinv, scr, st);
+    return cudaGetLastError();
+}
 cudaError_t launch_radial_sums(const Geo& g, int ncomp, const double* x, const double* w, double* out,
                                cudaStream_t s) {
     const int blocks = ncomp * g.nl;

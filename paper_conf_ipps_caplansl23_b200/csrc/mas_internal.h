@@ -207,6 +207,14 @@ int stencil_blocks(const Geo& g, int chunk);
 cudaError_t launch_stencil(int mode, int ncomp, const StencilArgs& a, cudaStream_t s,
                            bool first = false);
 cudaError_t launch_pcg_b(const StreamArgs& a, int nblocks, cudaStream_t s);
+// theta-node placement (NEXT-2): average the pole rows (local rows 0, g.nt-1)
+// of planes [plane_lo, plane_lo + nplanes) of every component over phi with
+// dp weights (dinv != nullptr: also dinv = 1 / average, ncomp = 1)
+cudaError_t launch_pole_avg(const Geo& g, int ncomp, double* y, double* dinv, int plane_lo, int nplanes,
+                            cudaStream_t s);
+// the init's <f,f>, <r,r>, <r,D^-1 r> into PcgState (after the pole average of r)
+cudaError_t launch_init_dots(const Geo& g, int ncomp, const double* f, const double* r, const double* dinv,
+                             Scratch scr, PcgState* st, int nblocks, cudaStream_t s);
 cudaError_t launch_diag(const Geo& g, Halo kappa, TRows tkappa, const double* c, double* D,
                         double* dinv, int* bad, cudaStream_t s);
 // out[side][c][i][k] = in[c][i][side ? nt-1 : 0][k]: a field's first / last theta rows

@@ -20,10 +20,11 @@ MAS_OK, MAS_NOT_CONVERGED, MAS_ERR_ARG, MAS_ERR_CUDA, MAS_ERR_NCCL, MAS_ERR_NOME
     MAS_ERR_BREAKDOWN = range(7)
 MAS_BC_DIRICHLET, MAS_BC_NEUMANN = 0, 1
 MAS_POLE_NORTH, MAS_POLE_SOUTH = 1, 2
+MAS_PLACE_CELL, MAS_PLACE_THETA_NODE = 0, 1
 
 # every symbol include/mas_pcg.h declares
 ABI_SYMBOLS = ("mas_comm_unique_id", "mas_partition", "mas_grid_create", "mas_grid_local_extent",
-               "mas_grid_destroy", "mas_op_setup", "mas_op_update", "mas_op_apply", "mas_op_diag",
+               "mas_grid_destroy", "mas_op_setup", "mas_op_setup_placed", "mas_op_update", "mas_op_apply", "mas_op_diag",
                "mas_op_dirichlet_rhs", "mas_op_dot", "mas_pcg_solve", "mas_op_enable_p2p",
                "mas_op_transport", "mas_op_launch_count", "mas_grid_create_2d",
                "mas_grid_local_extent_2d",
@@ -64,6 +65,7 @@ def lib() -> C.CDLL:
             "mas_grid_local_extent_2d": (_i, [_vp, _vp, _vp, _vp, _vp]),
             "mas_grid_destroy": (_i, [_vp]),
             "mas_op_setup": (_i, [_vp, _i, _vp, _vp, _i, _i, _vp, _vp]),
+            "mas_op_setup_placed": (_i, [_vp, _i, _i, _vp, _vp, _i, _i, _vp, _vp]),
             "mas_op_update": (_i, [_vp, _vp, _vp, _vp]),
             "mas_op_apply": (_i, [_vp, _vp, _vp, _vp]),
             "mas_op_diag": (_i, [_vp, _vp, _vp]),
@@ -225,6 +227,16 @@ def mas_op_setup(g: int, ncomp: int, kappa, mass=None, bc_r_inner=MAS_BC_DIRICHL
     return out.value
 
 
+def mas_op_setup_placed(g: int, ncomp: int, placement: int, kappa, mass=None,
+                        bc_r_inner=MAS_BC_DIRICHLET, bc_r_outer=MAS_BC_NEUMANN, stream=None) -> int:
+    """NEXT-2: placement MAS_PLACE_THETA_NODE puts the unknowns on the theta
+    nodes (rows 0 and nt on the poles): arrays [comp][nl][nt+1][np]."""
+    out = C.c_void_p()
+    _check(lib().mas_op_setup_placed(g, ncomp, placement, _ptr(kappa), _ptr(mass), bc_r_inner,
+                                     bc_r_outer, _stream(stream), C.byref(out)), "mas_op_setup_placed")
+    return out.value
+
+
 def mas_op_update(op: int, kappa, mass=None, stream=None) -> None:
     _check(lib().mas_op_update(op, _ptr(kappa), _ptr(mass), _stream(stream)), "mas_op_update")
 
@@ -366,13 +378,17 @@ class Operator:
     """Array arguments are the LOCAL block of this rank: [nl][ntl][np] for
     per-cell coefficients, [ncomp][nl][ntl][np] for vectors."""
 
-    def __init__(self, grid: Grid, ncomp, kappa, mass, bc_inner, bc_outer, stream=None):
+    def __init__(self, grid: Grid, ncomp, kappa, mass, bc_inner, bc_outer, stream=None,
+                 placement=MAS_PLACE_CELL):
         self.grid = grid
         self.ncomp = ncomp
-        self.N = grid.local_cells
+        self.placement = placement
+        # theta nodes (NEXT-2): nt + 1 rows, the first and last on the poles
+        self.rows = grid.shape[1] + 1 if placement == MAS_PLACE_THETA_NODE else grid.ntl
+        self.N = grid.nl * self.rows * grid.shape[2]
         _expect(kappa, self.N, "kappa")
         _expect(mass, self.N, "mass")
-        self.h = mas_op_setup(grid.h, ncomp, kappa, mass, bc_inner, bc_outer, stream)
+        self.h = mas_op_setup_placed(grid.h, ncomp, placement, kappa, mass, bc_inner, bc_outer, stream)
 
     def update(self, kappa, mass, stream=None):
         _expect(kappa, self.N, "kappa")
@@ -389,7 +405,7 @@ class Operator:
         mas_op_diag(self.h, D, stream)
 
     def dirichlet_rhs(self, ub_inner, ub_outer, f, stream=None):
-        nb = self.ncomp * self.grid.ntl * self.grid.shape[2]
+        nb = self.ncomp * self.rows * self.grid.shape[2]
         _expect(ub_inner, nb, "ub_inner")
         _expect(ub_outer, nb, "ub_outer")
         _expect(f, self.ncomp * self.N, "f")
@@ -441,7 +457,7 @@ class Operator:
 
     def radial_sums(self, x, w, out, stream=None):
         _expect(x, self.ncomp * self.N, "x")
-        _expect(w, self.grid.ntl * self.grid.shape[2], "w")
+        _expect(w, self.rows * self.grid.shape[2], "w")
         _expect(out, self.ncomp * self.grid.nl, "out")
         mas_op_radial_sums(self.h, x, w, out, stream)
 

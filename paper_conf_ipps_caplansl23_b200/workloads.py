@@ -296,6 +296,38 @@ def longrun_problem(nr=320, nt=300, np_=600, r0=1.0, r1=30.0, R=200.0, D_T=1000.
                    _temperature(np.float64(m.rF[0]), gT)[None].copy(), dt_T, dt_v)
 
 
+def replicate_poles(a: np.ndarray) -> np.ndarray:
+    """theta-node fields [..., nt+1, np]: every slot of a pole row (first and
+    last theta row) takes the row's first value (the pole is one point)."""
+    a = np.array(a, dtype=np.float64)
+    a[..., 0, :] = a[..., 0, :1]
+    a[..., -1, :] = a[..., -1, :1]
+    return a
+
+
+def tnode_conduction_problem(nr=128, nt=128, np_=256, r0=1.0, r1=30.0, R=200.0, D_max=1000.0,
+                             tol=1e-12, maxit=20000, warm=True) -> Problem:
+    """C2's conduction step with the temperature on the theta NODES
+    (rC_i, tF_j, pC_k), j = 0..nt (NEXT-2 placement, readings R29-R30): the
+    same T, rho fields and dt as conduction_problem, evaluated at the theta
+    nodes; the pole rows (j = 0, nt) are one value per radius (the texture is
+    smooth there: only its m = 0 term survives).  Arrays [.., nt+1, np]."""
+    base = conduction_problem(nr, nt, np_, r0, r1, R, D_max, tol, maxit, warm)
+    m = base.mesh
+    gT = texture(m.tC, m.pC, 1, at=(m.tF, m.pC))
+    grho = texture(m.tC, m.pC, 2, at=(m.tF, m.pC))
+    r = m.rC[:, None, None]
+    T = replicate_poles(np.broadcast_to(_temperature(r, gT[None]), (nr, nt + 1, np_)))
+    rho = replicate_poles(np.broadcast_to(_density(r, grho[None]), (nr, nt + 1, np_)))
+    kappa = T ** 2.5
+    c = rho / (GAMMA - 1.0) / base.extra["dt"]
+    f = (c * T)[None]
+    ub_in = replicate_poles(_temperature(np.float64(m.rF[0]), gT)[None])
+    x0 = T[None].copy() if warm else np.zeros_like(f)
+    return Problem("C2t-conduction-theta-nodes", m, 1, kappa, c, f, x0, DIRICHLET, NEUMANN, ub_in, None,
+                   tol, maxit, extra={"dt": base.extra["dt"], "placement": "theta-node"})
+
+
 def random_field(shape, seed=42) -> np.ndarray:
     """Matvec-parity input: U[-1,1] i.i.d."""
     return np.random.default_rng(seed).uniform(-1.0, 1.0, size=shape)
@@ -306,9 +338,11 @@ CONFIGS = {
     "C2": dict(kind="conduction", nr=128, nt=128, np_=256),
     "C3": dict(kind="viscosity", nr=256, nt=256, np_=512),
     "C2a": dict(kind="aniso", nr=128, nt=128, np_=256),
+    "C2t": dict(kind="tnode", nr=128, nt=128, np_=256),
 }
 
 
 def make(kind: str, **kw) -> Problem:
     return {"mms": mms_problem, "conduction": conduction_problem,
-            "viscosity": viscosity_problem, "aniso": aniso_conduction_problem}[kind](**kw)
+            "viscosity": viscosity_problem, "aniso": aniso_conduction_problem,
+            "tnode": tnode_conduction_problem}[kind](**kw)
