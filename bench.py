@@ -52,6 +52,9 @@ CONFIGS = {
     # C2 with field-aligned conduction: kernel A, the
     # L_par kernel and kernel B per iteration (one GPU)
     "C2a": ("aniso", 128, 128, 256),
+    # C2's conduction step with the temperature on the theta NODES, pole rows
+    # one value per radius: 128 x 129 x 256 unknowns
+    "C2t": ("tnode", 128, 128, 256),
     "C1": ("mms", 16, 24, 32),
 }
 # algorithmic bytes per cell per iteration: kernel A reads
@@ -170,19 +173,30 @@ def oracle_sample(prob, iters: int, threads: int):
     the setup (diagonal, initial residual).  Returns iters/s."""
     import oracle
     o = oracle.Oracle.for_problem(prob, threads)
-    f = o.dirichlet_rhs(prob.kappa, prob.f, prob.ub_inner, prob.ub_outer)
-    run = oracle_runner(o, prob, f)
+    run = oracle_runner(o, prob, oracle_rhs(o, prob))
+    run(1)  # first touch of the oracle's buffers
     t0 = time.perf_counter()
     run(1)
     t1 = time.perf_counter()
     run(1 + iters)
     t2 = time.perf_counter()
-    per_iter = max((t2 - t1) - (t1 - t0), 1e-9) / iters
+    dt = (t2 - t1) - (t1 - t0)
+    if not dt > 0.05 * (t2 - t1):  # noise above the iterations' cost: keep the setup in
+        dt = (t2 - t1) * iters / (1 + iters)
+    per_iter = dt / iters
     return 1.0 / per_iter, per_iter
+
+
+def oracle_rhs(o, prob):
+    if prob.extra.get("placement") == "theta-node":
+        return o.tn_dirichlet_rhs(prob.kappa, prob.f, prob.ub_inner, prob.ub_outer)
+    return o.dirichlet_rhs(prob.kappa, prob.f, prob.ub_inner, prob.ub_outer)
 
 
 def oracle_runner(o, prob, f):
     """k fixed oracle PCG iterations (tol = 0) on the problem's operator."""
+    if prob.extra.get("placement") == "theta-node":
+        return lambda k: o.tn_pcg(prob.kappa, prob.c, f, prob.x0, 0.0, k)
     if prob.kpar is not None:
         return lambda k: o.pcg_aniso(prob.kappa, prob.c, prob.kpar, prob.bhat, f, prob.x0, 0.0, k)
     return lambda k: o.pcg(prob.kappa, prob.c, f, prob.x0, 0.0, k)
@@ -233,23 +247,28 @@ def run_reference(args):
     prob = make_problem(args.config)
     cores = cpu_cores()
     o = oracle.Oracle.for_problem(prob, cores)
-    f = o.dirichlet_rhs(prob.kappa, prob.f, prob.ub_inner, prob.ub_outer)
+    f = oracle_rhs(o, prob)
     per_step_iters = 2
     run = oracle_runner(o, prob, f)
-    for _ in range(args.warmup):
+    for _ in range(max(1, args.warmup)):
         run(1)
-    dt = 0.0
+    t_short = t_long = 0.0
     for _ in range(args.steps):
         t0 = time.perf_counter()
         run(1)
         t1 = time.perf_counter()
         run(1 + per_step_iters)
         t2 = time.perf_counter()
-        dt += max((t2 - t1) - (t1 - t0), 1e-9)
+        t_short += t1 - t0
+        t_long += t2 - t1
+    dt = t_long - t_short
+    how = f"timed as run(1+{per_step_iters}) - run(1) (setup subtracted)"
+    if not dt > 0.05 * t_long:  # timing noise above the iterations' cost: keep the setup in
+        dt = t_long * per_step_iters / (1 + per_step_iters)
+        how = f"timed as run(1+{per_step_iters}) scaled by {per_step_iters}/{1 + per_step_iters} (setup kept)"
     value = args.steps * per_step_iters / dt
     sample = (f"{args.config} full grid {prob.shape}, ncomp {prob.ncomp}: {per_step_iters} fixed "
-              f"oracle PCG iterations per step, timed as run(1+{per_step_iters}) - run(1) "
-              f"(setup subtracted)")
+              f"oracle PCG iterations per step, {how}")
     line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * dt / args.steps,
             "higher_is_better": True, "scaling": scaling_of(args.config), "vs_baseline": None,
@@ -264,11 +283,19 @@ def run_reference(args):
     return 0
 
 
-def volumes(mesh):
+def volumes(mesh, tnode=False):
     """V_P = rC^2 dr sin(tC) dt dp (the inner-product weight of R9), for the
-    bench's own x comparison."""
+    bench's own x comparison; theta nodes: sin(tF) (tC_j - tC_{j-1}) and the
+    polar-cap measures 1 -+ cos at the pole rows (R29)."""
     dr, dt, dp = np.diff(mesh.rF), np.diff(mesh.tF), np.diff(mesh.pF)
-    return (mesh.rC ** 2 * dr)[:, None, None] * (np.sin(mesh.tC) * dt)[None, :, None] * dp[None, None, :]
+    if tnode:
+        tC, tF = mesh.tC, mesh.tF
+        mt = np.empty(len(tF))
+        mt[1:-1] = np.sin(tF[1:-1]) * np.diff(tC)
+        mt[0], mt[-1] = 1.0 - np.cos(tC[0]), 1.0 + np.cos(tC[-1])
+    else:
+        mt = np.sin(mesh.tC) * dt
+    return (mesh.rC ** 2 * dr)[:, None, None] * mt[None, :, None] * dp[None, None, :]
 
 
 def reference_solve(M, prob, rank, dev, tol):
@@ -276,7 +303,9 @@ def reference_solve(M, prob, rank, dev, tol):
     import torch
     g = M.Grid(prob.mesh)
     d = lambda a: torch.from_numpy(np.ascontiguousarray(a)).to(dev)
-    o = M.Operator(g, prob.ncomp, d(prob.kappa), d(prob.c), prob.bc_inner, prob.bc_outer)
+    tn = prob.extra.get("placement") == "theta-node"
+    o = M.Operator(g, prob.ncomp, d(prob.kappa), d(prob.c), prob.bc_inner, prob.bc_outer,
+                   placement=M.MAS_PLACE_THETA_NODE if tn else M.MAS_PLACE_CELL)
     if prob.kpar is not None:
         o.set_aniso(d(prob.kpar), d(prob.bhat))
     f = d(prob.f)
@@ -312,7 +341,7 @@ def check_parity(M, op, prob, x0, rhs, ref, extent, rank, world, dev, tol, dist)
         for b, (i0, nl, j0, ntl) in zip(bufs, ext):
             blk = b[: prob.ncomp * nl * ntl * prob.shape[2]].cpu().numpy()
             xg[:, i0:i0 + nl, j0:j0 + ntl] = blk.reshape(prob.ncomp, nl, ntl, prob.shape[2])
-        V = volumes(prob.mesh)[None]
+        V = volumes(prob.mesh, prob.extra.get("placement") == "theta-node")[None]
         xr = ref["x"]
         err = float(np.sqrt((V * (xg - xr) ** 2).sum() / (V * xr ** 2).sum()))
         res[0], res[1], res[2] = err, ref["iters"], float(np.isnan(xg).any())
@@ -380,6 +409,11 @@ def main():
         distinfo = (world, rank, obj[0])
     grid = M.Grid(prob.mesh, distinfo, ptheta=args.ptheta if world > 1 else 1)
     i0, nl, j0, ntl = grid.i0, grid.nl, grid.j0, grid.ntl
+    tnode = prob.extra.get("placement") == "theta-node"
+    if tnode:  # theta nodes: nt + 1 rows (r-slabs only)
+        if args.ptheta != 1:
+            raise SystemExit("C2t (theta-node placement) needs r-slabs (--ptheta 1)")
+        nt, j0, ntl = nt + 1, 0, nt + 1
     sl = (slice(i0, i0 + nl), slice(j0, j0 + ntl))
     slc = (slice(None),) + sl
     nc = prob.ncomp
@@ -400,7 +434,8 @@ def main():
         bhat = to_dev(prob.bhat[(slice(None),) + sl])
 
     def make_op(use_p2p):
-        o = M.Operator(grid, nc, kappa, cmass, prob.bc_inner, prob.bc_outer)
+        o = M.Operator(grid, nc, kappa, cmass, prob.bc_inner, prob.bc_outer,
+                       placement=M.MAS_PLACE_THETA_NODE if tnode else M.MAS_PLACE_CELL)
         if aniso:
             o.set_aniso(kpar, bhat)
         if args.solver == "cg1":
