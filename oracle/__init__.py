@@ -308,6 +308,27 @@ class Oracle:
         return rc, x, iters.value, relres.value, hist[: iters.value + 1]
 
 
+    # ---- vector-Laplacian curvature terms (NEXT-2, R31), ncomp = 3 ---------
+    def apply_curv(self, kappa, c, x):
+        x = _f64(x)
+        y = np.empty_like(x)
+        kappa, c = _f64(kappa), _f64(c)
+        self._chk(lib().mas_ref_op_apply_curv(C.byref(self.g), _p(kappa), _p(c), _p(x), _p(y)))
+        return y
+
+    def pcg_curv(self, kappa, c, f, x0, tol, maxit):
+        f = _f64(f)
+        x = _f64(x0).copy()
+        kappa, c = _f64(kappa), _f64(c)
+        iters, relres = C.c_int(), C.c_double()
+        hist = np.zeros(maxit + 1)
+        rc = lib().mas_ref_pcg_solve_curv(C.byref(self.g), _p(kappa), _p(c), _p(f), _p(x),
+                                          C.c_double(tol), maxit, C.byref(iters), C.byref(relres),
+                                          _p(hist))
+        self._chk(rc)
+        return rc, x, iters.value, relres.value, hist[: iters.value + 1]
+
+
 def partition(nr: int, nranks: int, rank: int):
     i0, nl = C.c_int(), C.c_int()
     lib().mas_ref_partition(nr, nranks, rank, C.byref(i0), C.byref(nl))

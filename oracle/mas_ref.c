@@ -320,10 +320,13 @@ static int aniso_add(const mas_ref_grid* g, int ncomp, const double* kpar,
                      const double* bhat, const double* x, double* y);
 static int aniso_diag_add(const mas_ref_grid* g, const double* kpar, const double* bhat,
                           double* D);
+static void curv_add(const mas_ref_grid* g, const double* kappa, const double* x, double* y);
 
-/* The PCG loop for L = L_iso (+ L_par when kpar != NULL, NEXT-4). */
+/* The PCG loop for L = L_iso (+ L_par when kpar != NULL, NEXT-4; + the
+ * vector-Laplacian curvature terms when curv, NEXT-2, R31: the Jacobi
+ * diagonal stays the 7-point one). */
 static int pcg_core(const mas_ref_grid* g, int ncomp, const double* kappa,
-                    const double* c, const double* kpar, const double* bhat,
+                    const double* c, const double* kpar, const double* bhat, int curv,
                     const double* f, double* x, double tol,
                     int maxit, int* iters, double* relres, double* res_hist) {
     tables T;
@@ -354,6 +357,7 @@ static int pcg_core(const mas_ref_grid* g, int ncomp, const double* kappa,
     }
     mas_ref_op_apply(g, ncomp, kappa, c, x, r);                  /* r = L x     */
     if (kpar) aniso_add(g, ncomp, kpar, bhat, x, r);
+    if (curv) curv_add(g, kappa, x, r);
 #pragma omp parallel for schedule(static)
     for (e = 0; e < n; e++) r[e] = f[e] - r[e];                  /* r = f - L x */
     rn = sqrt(dot_planes(g, &T, 0, g->nr, ncomp, r, r));
@@ -368,6 +372,7 @@ static int pcg_core(const mas_ref_grid* g, int ncomp, const double* kappa,
     for (k = 1; k <= maxit; k++) {
         mas_ref_op_apply(g, ncomp, kappa, c, p, q);              /* q = L p     */
         if (kpar) aniso_add(g, ncomp, kpar, bhat, p, q);
+        if (curv) curv_add(g, kappa, p, q);
         sigma = dot_planes(g, &T, 0, g->nr, ncomp, p, q);
         if (!(sigma > 0.0) || !isfinite(sigma)) {
             *iters = k; *relres = rn / bn; status = MAS_REF_ERR_BREAKDOWN; goto done;
@@ -397,7 +402,7 @@ done:
 int mas_ref_pcg_solve(const mas_ref_grid* g, int ncomp, const double* kappa,
                       const double* c, const double* f, double* x, double tol,
                       int maxit, int* iters, double* relres, double* res_hist) {
-    return pcg_core(g, ncomp, kappa, c, NULL, NULL, f, x, tol, maxit, iters, relres, res_hist);
+    return pcg_core(g, ncomp, kappa, c, NULL, NULL, 0, f, x, tol, maxit, iters, relres, res_hist);
 }
 
 /* ---------------------------------------------------------------------------
@@ -916,7 +921,7 @@ int mas_ref_pcg_solve_aniso(const mas_ref_grid* g, int ncomp, const double* kapp
                             const double* f, double* x, double tol, int maxit, int* iters,
                             double* relres, double* res_hist) {
     if (!aniso_check(g, kpar, bhat)) return MAS_REF_ERR_ARG;
-    return pcg_core(g, ncomp, kappa, c, kpar, bhat, f, x, tol, maxit, iters, relres, res_hist);
+    return pcg_core(g, ncomp, kappa, c, kpar, bhat, 0, f, x, tol, maxit, iters, relres, res_hist);
 }
 
 /* Slab-local L_par for a rank owning r-planes [i0, i0+nl) (the r-slab
@@ -1418,4 +1423,50 @@ int mas_ref_tn_pcg_solve(const mas_ref_grid* g, int ncomp, const double* kappa, 
 done:
     free(V); free(D); free(r); free(z); free(p); free(q);
     return status;
+}
+
+/* ---------------------------------------------------------------------------
+ * Vector-Laplacian curvature terms of the 3-component viscosity operator
+ * (reading R31).  The components of the
+ * viscosity unknown are the spherical components (v_r, v_theta, v_phi) (R13);
+ * the vector Laplacian in spherical coordinates adds to each component's
+ * scalar Laplacian a term in the SAME component,
+ *   (lap v)_r     = lap v_r     - 2 v_r / r^2                 - (coupling)
+ *   (lap v)_theta = lap v_theta - v_theta / (r^2 sin^2 theta) + (coupling)
+ *   (lap v)_phi   = lap v_phi   - v_phi   / (r^2 sin^2 theta) + (coupling)
+ * ("coupling": derivatives of the OTHER components, not included).  For
+ * L v = c v - div(kappa grad v) the curvature terms are
+ *   + kappa_P (2 / rC^2) v_r,  + kappa_P / (rC^2 sin^2 tC) v_theta,  + the same for v_phi,
+ * evaluated at the cell centre (all >= 0: L stays SPD).  The Jacobi
+ * preconditioner stays the shared 7-point diagonal D (R31).
+ * ------------------------------------------------------------------------- */
+static void curv_add(const mas_ref_grid* g, const double* kappa, const double* x, double* y) {
+    size_t N = (size_t)g->nr * g->nt * g->np;
+    int i;
+#pragma omp parallel for schedule(static)
+    for (i = 0; i < g->nr; i++) {
+        int j, k, m;
+        for (j = 0; j < g->nt; j++) {
+            const double s = sin(g->tC[j]);
+            const double w[3] = {2.0 / (g->rC[i] * g->rC[i]), 1.0 / (g->rC[i] * g->rC[i] * s * s),
+                                 1.0 / (g->rC[i] * g->rC[i] * s * s)};
+            for (k = 0; k < g->np; k++) {
+                size_t P = IDX(g, i, j, k);
+                for (m = 0; m < 3; m++) y[(size_t)m * N + P] += kappa[P] * w[m] * x[(size_t)m * N + P];
+            }
+        }
+    }
+}
+
+int mas_ref_op_apply_curv(const mas_ref_grid* g, const double* kappa, const double* c,
+                          const double* x, double* y) {
+    int rc = mas_ref_op_apply(g, 3, kappa, c, x, y);
+    if (rc == MAS_REF_OK) curv_add(g, kappa, x, y);
+    return rc;
+}
+
+int mas_ref_pcg_solve_curv(const mas_ref_grid* g, const double* kappa, const double* c,
+                           const double* f, double* x, double tol, int maxit, int* iters,
+                           double* relres, double* res_hist) {
+    return pcg_core(g, 3, kappa, c, NULL, NULL, 1, f, x, tol, maxit, iters, relres, res_hist);
 }

@@ -169,4 +169,13 @@ int mas_ref_tn_pcg_solve(const mas_ref_grid* g, int ncomp, const double* kappa, 
                          const double* f, double* x, double tol, int maxit, int* iters,
                          double* relres, double* res_hist);
 
+/* 3-component viscosity with the vector-Laplacian curvature terms (NEXT-2,
+ * reading R31): y = L x + kappa_P (2/rC^2 x_r, x_theta/(rC^2 sin^2 tC),
+ * x_phi/(rC^2 sin^2 tC)); PCG with the shared 7-point Jacobi diagonal. */
+int mas_ref_op_apply_curv(const mas_ref_grid* g, const double* kappa, const double* c,
+                          const double* x, double* y);
+int mas_ref_pcg_solve_curv(const mas_ref_grid* g, const double* kappa, const double* c,
+                           const double* f, double* x, double tol, int maxit, int* iters,
+                           double* relres, double* res_hist);
+
 #endif
