@@ -253,6 +253,18 @@ MAS_API mas_status_t mas_op_enable_p2p(mas_op_t* op, cudaStream_t stream);
  * the field-aligned term on; MAS_ERR_NOMEM. */
 MAS_API mas_status_t mas_op_set_single_reduction(mas_op_t* op, int on);
 
+/* Vector-Laplacian curvature terms (reading R31,
+ * DESIGN.md §3.7).  For the 3-component viscosity operator, whose components
+ * are the spherical (v_r, v_theta, v_phi) (R13), on != 0 adds the terms of the
+ * vector Laplacian in the SAME component:
+ *   (L v)_r += kappa_P 2/rC^2 v_r,  (L v)_theta += kappa_P v_theta/(rC sin tC)^2,
+ *   (L v)_phi += kappa_P v_phi/(rC sin tC)^2        (cell centres, all >= 0)
+ * in apply, the residual and every iteration (the terms coupling different
+ * components are not included).  The Jacobi preconditioner stays the shared
+ * 7-point diagonal.  Errors: MAS_ERR_ARG unless ncomp == 3 and the placement
+ * is cell-centred. */
+MAS_API mas_status_t mas_op_set_curvature(mas_op_t* op, int on);
+
 /* 1 if the op's solve uses the single-reduction loop, 0 if not, -1 if NULL. */
 MAS_API int mas_op_single_reduction(const mas_op_t* op);
 

@@ -160,6 +160,8 @@ struct mas_op {
     // placement (NEXT-2): 0 cell centres; 1 theta nodes with pole rows (local
     // rows 0 and nt hold one value per radius: k_pole_avg after every stencil)
     int tnode = 0;
+    // vector-Laplacian curvature terms of the 3-component operator (NEXT-2, R31)
+    int curv = 0;
     cudaGraphExec_t gexec1 = nullptr;
     const double* g1_x = nullptr;
     double* atab = nullptr;                      // AnisoTab arrays (device)
@@ -753,6 +755,7 @@ static mas_status_t cg1_solve(mas_op* op, const double* fd, double* xd, double t
     a.kappa = halo_of(op, op->kappa, nullptr, 1);
     a.dinv = halo_of(op, op->dinv, nullptr, 1);
     a.c = op->c;
+    a.curv = op->curv;
     a.st = op->st;
     a.rho_hist = rho_h;
     a.sigma_hist = sig_h;
@@ -1058,6 +1061,7 @@ mas_status_t mas_op_apply(const mas_op_t* op_c, const double* x, double* y, cuda
     a.tu = packed_rows(op, op->xgt, op->ncomp);
     a.tkappa = packed_rows(op, op->kgt, 1);
     a.c = op->c;
+    a.curv = op->curv;
     a.out = yd;
     a.scr = op->scr;
     CU(launch_stencil(MODE_APPLY, op->ncomp, a, stream));
@@ -1279,6 +1283,7 @@ mas_status_t mas_op_set_single_reduction(mas_op_t* op, int on) {
     if (op->g->comm) return arg_error("single-reduction PCG: one GPU only (no mas_dist_t)");
     if (op->aniso) return arg_error("single-reduction PCG: isotropic operator only (no mas_op_set_aniso)");
     if (op->tnode) return arg_error("single-reduction PCG: cell-centred placement only");
+    if (op->curv) return arg_error("single-reduction PCG: without the curvature terms");
     const size_t n = op->ncomp * (size_t)op->Nl;
     if (!op->r2) ST(dmalloc(&op->r2, n));
     if (!op->w2) ST(dmalloc(&op->w2, n));
@@ -1288,6 +1293,15 @@ mas_status_t mas_op_set_single_reduction(mas_op_t* op, int on) {
 }
 
 int mas_op_single_reduction(const mas_op_t* op) { return op ? op->cg1 : -1; }
+
+mas_status_t mas_op_set_curvature(mas_op_t* op, int on) {
+    if (!op) return arg_error("null op");
+    if (on && op->ncomp != 3) return arg_error("curvature terms: the 3-component (viscosity) operator only");
+    if (on && op->tnode) return arg_error("curvature terms: cell-centred placement only");
+    if (on && op->cg1) return arg_error("curvature terms: the two-kernel loop only (single reduction is on)");
+    op->curv = on ? 1 : 0;
+    return MAS_OK;
+}
 
 mas_status_t mas_op_comm_bench(mas_op_t* op, int reps, double* seam_us, double* allreduce_us,
                                double* seam_bytes, cudaStream_t s) {
@@ -1523,6 +1537,7 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
     a.tkappa = packed_rows(op, op->kgt, 1);
     a.tdinv = packed_rows(op, op->dgt, 1);
     a.c = op->c;
+    a.curv = op->curv;
     a.f = fd;
     a.out = op->r;
     a.st = op->st;

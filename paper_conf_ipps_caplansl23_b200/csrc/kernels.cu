@@ -827,6 +827,10 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
             const double V0 = vri * vtj * vpk[0], V1 = vri * vtj * vpk[1];
             const double2 cP = a.c ? oc.c : make_double2(0.0, 0.0);
             const int pofs = (int)i * plane32(g) + off;
+            // vector-Laplacian curvature terms (3 components, NEXT-2, R31): the
+            // mass term of component m gains kappa_P * (2/r^2 | 1/(r sin)^2)
+            const bool curv = NC == 3 && a.curv;
+            const double cmr = 2.0 * irc, cma = ic;
 #pragma unroll
             for (int c = 0; c < NC; c++) {
                 const double* s0 = sfield(const_cast<double*>(S0), c);
@@ -837,6 +841,11 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
                 const double2 uT = lds2(s0 + idx + ROW);
                 const double uL = s0[idx - 1], uR = s0[idx + 2];
                 double L0 = cP.x * u.x, L1 = cP.y * u.y;
+                if (curv) {
+                    const double cm = c == 0 ? cmr : cma;
+                    L0 = fma(kP.x * cm, u.x, L0);
+                    L1 = fma(kP.y * cm, u.y, L1);
+                }
                 L0 = fma(aRm0, u.x - uM.x, L0);
                 L1 = fma(aRm1, u.y - uM.y, L1);
                 L0 = fma(aRp0, u.x - uN.x, L0);

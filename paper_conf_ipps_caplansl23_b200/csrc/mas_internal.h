@@ -145,6 +145,7 @@ struct StencilArgs {
     unsigned long long cond;  // CUDA graph while-loop handle (0: not in a graph)
     P2P p2p;                  // RESID / PCGA: mailbox transport (nranks == 0: off)
     int nopub;                // RESID under P2P with the field-aligned term: k_aniso publishes
+    int curv;                 // NC = 3: + kappa_P (2/r^2, 1/(r sin)^2, 1/(r sin)^2) u_m (NEXT-2, R31)
 };
 
 struct StreamArgs {  // kernel B

@@ -29,7 +29,7 @@ ABI_SYMBOLS = ("mas_comm_unique_id", "mas_partition", "mas_grid_create", "mas_gr
                "mas_op_transport", "mas_op_launch_count", "mas_grid_create_2d",
                "mas_grid_local_extent_2d",
                "mas_op_set_profiling", "mas_op_kernel_times", "mas_op_set_aniso",
-               "mas_op_aniso_time", "mas_op_radial_sums", "mas_op_comm_bench", "mas_op_set_single_reduction",
+               "mas_op_aniso_time", "mas_op_radial_sums", "mas_op_comm_bench", "mas_op_set_single_reduction", "mas_op_set_curvature",
                "mas_op_single_reduction", "mas_op_destroy", "mas_status_string", "mas_last_error", "mas_version")
 
 
@@ -82,6 +82,7 @@ def lib() -> C.CDLL:
             "mas_op_radial_sums": (_i, [_vp, _vp, _vp, _vp, _vp]),
             "mas_op_comm_bench": (_i, [_vp, _i, _vp, _vp, _vp, _vp]),
             "mas_op_set_single_reduction": (_i, [_vp, _i]),
+            "mas_op_set_curvature": (_i, [_vp, _i]),
             "mas_op_single_reduction": (_i, [_vp]),
             "mas_op_destroy": (_i, [_vp]),
             "mas_status_string": (C.c_char_p, [_i]),
@@ -334,6 +335,11 @@ def mas_op_set_single_reduction(op: int, on: bool = True) -> None:
     _check(lib().mas_op_set_single_reduction(op, int(bool(on))), "mas_op_set_single_reduction")
 
 
+def mas_op_set_curvature(op: int, on: bool = True) -> None:
+    """NEXT-2: the vector-Laplacian curvature terms of the 3-component operator."""
+    _check(lib().mas_op_set_curvature(op, int(bool(on))), "mas_op_set_curvature")
+
+
 def mas_op_single_reduction(op: int) -> bool:
     return int(lib().mas_op_single_reduction(op)) == 1
 
@@ -444,6 +450,9 @@ class Operator:
 
     def set_single_reduction(self, on=True):
         mas_op_set_single_reduction(self.h, on)
+
+    def set_curvature(self, on=True):
+        mas_op_set_curvature(self.h, on)
 
     @property
     def single_reduction(self):
