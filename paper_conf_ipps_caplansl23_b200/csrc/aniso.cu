@@ -128,7 +128,15 @@ __device__ __forceinline__ double2 ld2(const double* p) { return __ldg(reinterpr
 // ring, signalled by mbarriers (full: the box bytes landed; empty: the 16
 // consumer warps are done with the slot).
 namespace {
-constexpr int WJ = 16;                 // tile rows (one consumer warp each)
+#ifndef MAS_ANISO_WJ
+#define MAS_ANISO_WJ 16
+#endif
+#ifndef MAS_ANISO_BPS
+#define MAS_ANISO_BPS 1
+#endif
+constexpr int WJ = MAS_ANISO_WJ;       // tile rows (one consumer warp each)
+constexpr int kAnisoBps = MAS_ANISO_BPS;  // resident blocks per SM (the rings must fit)
+constexpr int rup16(int x) { return (x + 15) / 16 * 16; }  // 128-byte multiples of doubles
 constexpr int WK = 64;                 // tile columns (32 lanes x 2)
 constexpr int NCW = WJ;                // consumer warps
 constexpr int WTHREADS = 32 * (NCW + 1);
@@ -138,18 +146,28 @@ constexpr int WCR = WJ + 1;            // corner rows
 constexpr int WCW = WK + 2;            // corner row: K = k0 .. k0+64 (+1)
 constexpr int WCA = WCR * WCW;         // one corner array
 // every component of a slot starts 128-byte aligned (tensor-copy destinations)
-constexpr int WP_SLOT = 1232;          // p box [18][68] (1224) + pad
-constexpr int WC_SLOT = 4496;          // coefficient box [3][17][66] + combinations array 3 (4488) + pad
-constexpr int WQ_SLOT = WJ * WK;       // out box [16][64]
-constexpr int WPL = 48, WPRT = 48;     // phi-wrap side boxes of p: [18][2] (left k0-2.., right 0..)
-constexpr int WCS = 112;               // phi-wrap side box of the coefficients: [3][17][2]
+constexpr int WP_SLOT = rup16(WPR * WPW);  // p box [WJ+2][68] + pad
+constexpr int WC_SLOT = rup16(4 * WCA);    // coefficient box [3][WJ+1][66] + combinations array 3 + pad
+#ifdef MAS_ANISO_QTMA
+constexpr int WQ_SLOT = WJ * WK;       // out box [WJ][64]
+#else
+constexpr int WQ_SLOT = 0;             // out/q is read by the consumers directly
+#endif
+constexpr int WPL = rup16(WPR * 2), WPRT = WPL;  // phi-wrap side boxes of p: [WJ+2][2]
+constexpr int WCS = rup16(3 * WCR * 2);          // phi-wrap side box of the coefficients: [3][WJ+1][2]
 constexpr int O_C = WP_SLOT, O_Q = O_C + WC_SLOT, O_PL = O_Q + WQ_SLOT, O_PR = O_PL + WPL,
               O_CS = O_PR + WPRT;
-constexpr int W_SLOT = O_CS + WCS;     // 6960 doubles
-constexpr int W_NSLOT = 4;
+constexpr int W_SLOT = O_CS + WCS;     // WJ = 16: 5936 doubles (6960 with the out box)
+#ifndef MAS_ANISO_SLOTS
+#define MAS_ANISO_SLOTS 4
+#endif
+constexpr int W_NSLOT = MAS_ANISO_SLOTS;  // ring depth (>= 2: a step reads stages n-1 and n)
 // tensor-copy transaction bytes (whole boxes, out-of-bounds elements included)
 constexpr unsigned TX_P = WPR * WPW * 8, TX_PS = WPR * 2 * 8, TX_C = 3 * WCR * WCW * 8,
-                   TX_CS = 3 * WCR * 2 * 8, TX_Q = WJ * WK * 8;
+                   TX_CS = 3 * WCR * 2 * 8;
+#ifdef MAS_ANISO_QTMA
+constexpr unsigned TX_Q = WJ * WK * 8;
+#endif
 }  // namespace
 constexpr int kAnisoSmem = W_NSLOT * W_SLOT * (int)sizeof(double) + 3 * W_NSLOT * 8;  // 222,816 B
 
@@ -216,7 +234,7 @@ __device__ __forceinline__ void consumer_sync() {  // the 16 consumer warps only
 // corners, plane i+1 (sr = -1) gives -c[-st,-sp].  sigma_par = <p, L_par p>_V
 // = sum_c s_c^2 (V L_par = G^T W K G), summed in the corner phase.
 template <int MODE>
-__global__ void __launch_bounds__(WTHREADS, 1) k_aniso(const AnisoArgs a, const __grid_constant__ AnisoMaps M) {
+__global__ void __launch_bounds__(WTHREADS, kAnisoBps) k_aniso(const AnisoArgs a, const __grid_constant__ AnisoMaps M) {
     extern __shared__ __align__(128) double sm[];
     unsigned long long* bars = reinterpret_cast<unsigned long long*>(sm + W_NSLOT * W_SLOT);
     if (MODE == MODE_PCGA && __ldcg(&a.st->stopped)) {
@@ -264,8 +282,14 @@ __global__ void __launch_bounds__(WTHREADS, 1) k_aniso(const AnisoArgs a, const 
         const int j0 = tj * WJ, k0 = tk * WK;
         const int height = min(WJ, g.nt - j0), width = min(WK, g.np - k0);  // width is even
 
-        // fresh rings (finite values in the cells no copy writes) and barriers
+        // barriers (the rings need no clearing: every value a consumer reads is
+        // written first in the same stage -- whole tensor boxes with zero-filled
+        // out-of-bounds parts, side boxes on the tiles that read them, and the
+        // corner combinations of rows <= height, columns <= width; MAS_ANISO_ZERO
+        // restores the round-1 clearing per segment)
+#ifdef MAS_ANISO_ZERO
         for (int t = threadIdx.x; t < W_NSLOT * W_SLOT; t += WTHREADS) sm[t] = 0.0;
+#endif
         if (threadIdx.x == 0) {
             for (int q = 0; q < W_NSLOT; q++) {
                 mbar_init(full0 + 8 * q, 1);    // expect_tx by the producer; the tensor bytes
@@ -274,7 +298,7 @@ __global__ void __launch_bounds__(WTHREADS, 1) k_aniso(const AnisoArgs a, const 
         }
         fence_proxy_async();
         __syncthreads();
-        // stages ia-1 .. ib; stage number n = I - (ia - 1), slot n & 3, use n >> 2
+        // stages ia-1 .. ib; stage number n = I - (ia - 1), slot n % W_NSLOT, use n / W_NSLOT
         const int nst = ib - ia + 2;
 
         if (producer) {
@@ -289,8 +313,8 @@ __global__ void __launch_bounds__(WTHREADS, 1) k_aniso(const AnisoArgs a, const 
                 return n == 0 ? 0 : (I >= 0 && I < g.nl ? 1 : (M.has_cahi ? 2 : 3));
             };
             auto issue = [&](int n) {
-                const int I = ia - 1 + n, slot = n & 3;
-                if (n >= W_NSLOT) mbar_wait(empty0 + 8 * slot, ((n >> 2) - 1) & 1);
+                const int I = ia - 1 + n, slot = n % W_NSLOT;
+                if (n >= W_NSLOT) mbar_wait(empty0 + 8 * slot, ((n / W_NSLOT) - 1) & 1);
                 const int ps = p_src(I), cs = c_src(n, I);
                 const bool ql = I - 1 >= ia && I - 1 < ib;
                 double* base = sm + slot * W_SLOT;
@@ -300,7 +324,9 @@ __global__ void __launch_bounds__(WTHREADS, 1) k_aniso(const AnisoArgs a, const 
                     unsigned bytes = 0;
                     if (ps) bytes += TX_P + (first ? TX_PS : 0u) + (last ? TX_PS : 0u);
                     if (cs) bytes += TX_C + (last ? TX_CS : 0u);
+#ifdef MAS_ANISO_QTMA
                     if (ql) bytes += TX_Q;
+#endif
                     mbar_expect_tx(full, bytes);
                     const unsigned sb = smem_u32(base);
                     const int jr = j0 - 1;
@@ -324,7 +350,11 @@ __global__ void __launch_bounds__(WTHREADS, 1) k_aniso(const AnisoArgs a, const 
                         tma3(sb + 8 * O_C, &M.cahi, k0, j0, 0, full);
                         if (last) tma3(sb + 8 * O_CS, &M.cahi_s, 0, j0, 0, full);
                     }
+#ifdef MAS_ANISO_QTMA
                     if (ql) tma3(sb + 8 * O_Q, &M.out, k0, j0, I - 1, full);
+#else
+                    (void)ql;  // out/q is read by the consumers directly (see below)
+#endif
                 }
             };
             for (int n = 0; n < nst; n++) issue(n);
@@ -370,8 +400,16 @@ __global__ void __launch_bounds__(WTHREADS, 1) k_aniso(const AnisoArgs a, const 
             double x0 = 0.0, y0 = 0.0, e0 = 0.0, e1 = 0.0, e2 = 0.0, e3 = 0.0;
             double2 x12 = make_double2(0.0, 0.0), y12 = x12;
             for (int n = 0; n < nst; n++) {
-                const int I = ia - 1 + n, slot = n & 3;
-                mbar_wait(full0 + 8 * slot, (n >> 2) & 1);
+                const int I = ia - 1 + n, slot = n % W_NSLOT;
+#ifndef MAS_ANISO_QTMA
+                // out/q of the cells of this step (plane I-1): a plain coalesced
+                // load issued before the stage wait (one register pair; no
+                // shared-memory round trip, which the MIO pipe is short of)
+                double2 qv = make_double2(0.0, 0.0);
+                if (n >= 2 && cell_ok)
+                    qv = ld2(a.out + (size_t)(I - 1) * plane + (size_t)(j0 + w) * g.np + k0 + c2);
+#endif
+                mbar_wait(full0 + 8 * slot, (n / W_NSLOT) & 1);
                 const double* p1 = P_of(slot);
                 double X0 = 0.0, Y0 = 0.0, E0 = 0.0, E1 = 0.0, E2 = 0.0, E3 = 0.0;
                 double2 X12 = make_double2(0.0, 0.0), Y12 = X12;
@@ -434,7 +472,7 @@ __global__ void __launch_bounds__(WTHREADS, 1) k_aniso(const AnisoArgs a, const 
                 // (sr = +1) and I (sr = -1); out/q plane i from this stage
                 if (n >= 2 && cell_ok) {
                     const int i = I - 1;
-                    const double* l = C_of((n - 1) & 3) + w * WCW + c2;
+                    const double* l = C_of((n - 1) % W_NSLOT) + w * WCW + c2;
                     const double* h = Cf + w * WCW + c2;
                     const double2 l0 = lds2(l), l2 = lds2(l + 2 * WCA + WCW);
                     const double2 h3 = lds2(h + 3 * WCA), h1 = lds2(h + WCA + WCW);
@@ -446,7 +484,9 @@ __global__ void __launch_bounds__(WTHREADS, 1) k_aniso(const AnisoArgs a, const 
                     const double s1 = ((l0.y + l1b) + (l2.y + l3b)) - ((h3.y + h2b) + (h1.y + h0b));
                     const double ivr = __ldg(a.ivr + i);
                     const double y0 = s0 * (ivr * cw0), y1 = s1 * (ivr * cw1);
+#ifdef MAS_ANISO_QTMA
                     const double2 qv = lds2(Q_of(slot) + w * WK + c2);
+#endif
                     double* o = a.out + (size_t)i * plane + (size_t)(j0 + w) * g.np + k0 + c2;
                     if (MODE == MODE_RESID) {
                         const double r0 = qv.x - y0, r1 = qv.y - y1;
@@ -467,7 +507,7 @@ __global__ void __launch_bounds__(WTHREADS, 1) k_aniso(const AnisoArgs a, const 
                 // proxy, the next fill of the slot is a tensor copy
                 fence_proxy_async();
                 __syncwarp();
-                if (lane == 0) mbar_arrive(empty0 + 8 * ((n - 1) & 3));
+                if (lane == 0) mbar_arrive(empty0 + 8 * ((n - 1) % W_NSLOT));
             }
         }
         __syncthreads();  // the next segment re-initialises the rings and barriers
@@ -512,6 +552,21 @@ static PFN_cuTensorMapEncodeTiled_v12000 tmap_encode_fn() {
     return fn;
 }
 
+// L2 promotion of the tensor copies (default 64 B).  The boxes are 66-68 doubles wide and
+// start 16 B off a 512 B boundary, so a 256 B promotion fetches up to 1.5x the
+// row; MAS_TMA_PROMO = 0 | 64 | 128 | 256 selects (experiment hook)
+static CUtensorMapL2promotion tma_promotion() {
+    static const CUtensorMapL2promotion p = [] {
+        const char* e = getenv("MAS_TMA_PROMO");
+        const int v = e ? atoi(e) : 64;  // 64 B measured best at C2a (r2j: 53.7 us vs 55.8 at 256 B)
+        return v == 0 ? CU_TENSOR_MAP_L2_PROMOTION_NONE
+               : v == 64 ? CU_TENSOR_MAP_L2_PROMOTION_L2_64B
+               : v == 128 ? CU_TENSOR_MAP_L2_PROMOTION_L2_128B
+                          : CU_TENSOR_MAP_L2_PROMOTION_L2_256B;
+    }();
+    return p;
+}
+
 // fp64 tiled tensor map, no swizzle, out-of-bounds elements read as zero
 static bool tmap(CUtensorMap* m, const double* base, int rank, const cuuint64_t* dims,
                  const cuuint64_t* strides, const cuuint32_t* box) {
@@ -519,8 +574,8 @@ static bool tmap(CUtensorMap* m, const double* base, int rank, const cuuint64_t*
     if (!fn || !base) return false;
     const cuuint32_t es[5] = {1, 1, 1, 1, 1};
     return fn(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, (cuuint32_t)rank, const_cast<double*>(base), dims, strides,
-              box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
-              CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+              box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, tma_promotion(),
+              CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
 static bool build_maps(const AnisoArgs& a, AnisoMaps* M) {
@@ -560,7 +615,7 @@ cudaError_t launch_aniso(int mode, const AnisoArgs& a0, cudaStream_t s) {
     a.ntj = (a.g.nt + WJ - 1) / WJ;
     a.ntk = (a.g.np + WK - 1) / WK;
     const int tiles = a.ntj * a.ntk;
-    long long want = device_sms();  // one block per SM (223 KB of rings each)
+    long long want = (long long)kAnisoBps * device_sms();  // one resident wave (the rings fill the SM)
     if (const char* e = getenv("MAS_ABLOCKS")) want = std::max(1, atoi(e));  // experiment hook
     want = std::min<long long>(want, (long long)tiles * a.g.nl);
     want = std::min<long long>(want, a.max_blocks);

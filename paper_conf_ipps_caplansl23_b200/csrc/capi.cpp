@@ -1415,9 +1415,10 @@ mas_status_t mas_op_set_aniso(mas_op_t* op, const double* kpar, const double* bh
     if (!op->ca) ST(dmalloc(&op->ca, 3 * (size_t)N));
     if (op->g->comm && !op->cag) {
         ST(dmalloc(&op->cag, 6 * (size_t)op->geo.plane));
+        // the NCCL loop's p_k seam buffers (2 planes; unused once the op runs the
+        // P2P transport, which reads the neighbours' p_k in place)
         ST(dmalloc(&op->pkg, 2 * (size_t)op->geo.plane));
     }
-    // host inputs are staged through a temporary device buffer
     const double *kd = kpar, *bd = bhat;
     // host inputs are staged through a library-owned device buffer (kept for
     // the next call: a time-stepping caller refreshes kpar and b every step)
@@ -1683,7 +1684,8 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
         }
         if (comm && !p2p) ST(comm_allreduce(comm, &op->st->pend_sigma, 1, s));
         if (k <= maxit) {
-            if (p2p) ST(comm_vsync(comm, s));  // virtual P2P ranks: all A(k) done
+            // virtual P2P ranks: all A(k) and k_aniso(k) done (B(k) reads slots A and C)
+            if (p2p) ST(comm_vsync(comm, s));
             if (op->tnode) {  // the caps of q = L p (theta nodes, NEXT-2)
                 ST(pole_pass(op, op->q, nc, s));
                 op->launches++;

@@ -1,4 +1,4 @@
-"""C5 drift check: repeated implicit steps of conduction
+"""C5 drift check: 200 repeated implicit steps of conduction
 (kappa = (T^n)^{5/2} refreshed with mas_op_update every step) followed by
 viscosity, warm-started, Delta t frozen at step 0.  GPU (C ABI) vs oracle on
 the 40x38x76 downscale (np made even): per-step iteration counts within
@@ -16,7 +16,7 @@ from paper_conf_ipps_caplansl23_b200 import workloads as W
 pytestmark = pytest.mark.gpu
 torch = pytest.importorskip("torch")
 
-NSTEPS = 60
+NSTEPS = 200  # 200 steps on the 40x38x75 downscale (np made even)
 
 
 @pytest.fixture(scope="module")
