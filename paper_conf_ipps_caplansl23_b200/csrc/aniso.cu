@@ -322,7 +322,12 @@ __global__ void __launch_bounds__(WTHREADS, kAnisoBps) k_aniso(const AnisoArgs a
                 if (lane == 0) {
                     const unsigned full = full0 + 8 * slot;
                     unsigned bytes = 0;
-                    if (ps) bytes += TX_P + (first ? TX_PS : 0u) + (last ? TX_PS : 0u);
+                    // every stage carries a p box: a dead plane (beyond a global r
+                    // boundary) is fetched from the own map at its out-of-range
+                    // plane index, i.e. as zeros (the corners there have zero
+                    // weight, but the ring slot must not hold stale or
+                    // uninitialised values: 0 * NaN)
+                    bytes += TX_P + (first ? TX_PS : 0u) + (last ? TX_PS : 0u);
                     if (cs) bytes += TX_C + (last ? TX_CS : 0u);
 #ifdef MAS_ANISO_QTMA
                     if (ql) bytes += TX_Q;
@@ -330,7 +335,7 @@ __global__ void __launch_bounds__(WTHREADS, kAnisoBps) k_aniso(const AnisoArgs a
                     mbar_expect_tx(full, bytes);
                     const unsigned sb = smem_u32(base);
                     const int jr = j0 - 1;
-                    if (ps == 1) {
+                    if (ps <= 1) {  // own plane, or a dead one (out of range: zeros)
                         tma3(sb, &M.u, k0 - 2, jr, I, full);
                         if (first) tma3(sb + 8 * O_PL, &M.u_s, g.np - 2, jr, I, full);
                         if (last) tma3(sb + 8 * O_PR, &M.u_s, 0, jr, I, full);
@@ -399,15 +404,19 @@ __global__ void __launch_bounds__(WTHREADS, kAnisoBps) k_aniso(const AnisoArgs a
             // the extra corner's 4 cells); wrap cells from the side boxes
             double x0 = 0.0, y0 = 0.0, e0 = 0.0, e1 = 0.0, e2 = 0.0, e3 = 0.0;
             double2 x12 = make_double2(0.0, 0.0), y12 = x12;
+#ifndef MAS_ANISO_QTMA
+            // out/q of the cells: plain coalesced loads (no shared-memory round
+            // trip, which the MIO pipe is short of), one step ahead of their use
+            // (step n processes the cells of plane I-1; the load of step n+1's
+            // plane I is issued at step n)
+            const size_t qoff = (size_t)(j0 + w) * g.np + k0 + c2;
+            double2 qnext = make_double2(0.0, 0.0);
+#endif
             for (int n = 0; n < nst; n++) {
                 const int I = ia - 1 + n, slot = n % W_NSLOT;
 #ifndef MAS_ANISO_QTMA
-                // out/q of the cells of this step (plane I-1): a plain coalesced
-                // load issued before the stage wait (one register pair; no
-                // shared-memory round trip, which the MIO pipe is short of)
-                double2 qv = make_double2(0.0, 0.0);
-                if (n >= 2 && cell_ok)
-                    qv = ld2(a.out + (size_t)(I - 1) * plane + (size_t)(j0 + w) * g.np + k0 + c2);
+                const double2 qv = qnext;
+                if (n + 1 >= 2 && n + 1 < nst && cell_ok) qnext = ld2(a.out + (size_t)I * plane + qoff);
 #endif
                 mbar_wait(full0 + 8 * slot, (n / W_NSLOT) & 1);
                 const double* p1 = P_of(slot);
