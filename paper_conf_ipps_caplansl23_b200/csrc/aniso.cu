@@ -128,6 +128,12 @@ __device__ __forceinline__ double2 ld2(const double* p) { return __ldg(reinterpr
 // ring, signalled by mbarriers (full: the box bytes landed; empty: the 16
 // consumer warps are done with the slot).
 namespace {
+// out/q: a TMA box per stage (default; A/B r2n: 53.7 us) or, with
+// MAS_ANISO_QLDG, plain loads by the consumers (54.0 us at the top of the
+// step, 55.4 us one step ahead)
+#ifndef MAS_ANISO_QLDG
+#define MAS_ANISO_QTMA
+#endif
 #ifndef MAS_ANISO_WJ
 #define MAS_ANISO_WJ 16
 #endif
@@ -414,9 +420,13 @@ __global__ void __launch_bounds__(WTHREADS, kAnisoBps) k_aniso(const AnisoArgs a
 #endif
             for (int n = 0; n < nst; n++) {
                 const int I = ia - 1 + n, slot = n % W_NSLOT;
-#ifndef MAS_ANISO_QTMA
+#if !defined(MAS_ANISO_QTMA) && !defined(MAS_ANISO_QNOW)
                 const double2 qv = qnext;
                 if (n + 1 >= 2 && n + 1 < nst && cell_ok) qnext = ld2(a.out + (size_t)I * plane + qoff);
+#elif !defined(MAS_ANISO_QTMA)
+                (void)qnext;  // A/B hook: the load of this step's q at the top of the step
+                double2 qv = make_double2(0.0, 0.0);
+                if (n >= 2 && cell_ok) qv = ld2(a.out + (size_t)(I - 1) * plane + qoff);
 #endif
                 mbar_wait(full0 + 8 * slot, (n / W_NSLOT) & 1);
                 const double* p1 = P_of(slot);
