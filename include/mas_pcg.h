@@ -248,9 +248,12 @@ MAS_API mas_status_t mas_op_enable_p2p(mas_op_t* op, cudaStream_t stream);
  * loop; iterates equal it in exact arithmetic (rounding differs: parity band
  * +-2 iterations, x <= 1e-9).  HBM traffic per iteration: 13 passes scalar
  * (as the two-kernel loop), 33 passes for 3 components (31).  Allocates 3
- * more vectors.  on == 0 restores the two-kernel loop.
- * Errors: MAS_ERR_ARG on a grid with a mas_dist_t (one GPU only) or with
- * the field-aligned term on; MAS_ERR_NOMEM. */
+ * more vectors.  On r-slabs the NCCL loop runs ONE 3-double allreduce per
+ * iteration (two in the two-kernel loop) plus the seams of r, w and s; kernel
+ * k+1 takes the stop / alpha / beta decision from the allreduced sums, so
+ * every rank decides alike.  on == 0 restores the two-kernel loop.
+ * Errors: MAS_ERR_ARG with the P2P transport, ptheta > 1, the field-aligned
+ * term, the theta-node placement or the curvature terms; MAS_ERR_NOMEM. */
 MAS_API mas_status_t mas_op_set_single_reduction(mas_op_t* op, int on);
 
 /* Vector-Laplacian curvature terms (reading R31,

@@ -654,14 +654,16 @@ static mas_status_t loop_graph(mas_op* op, StencilArgs a, StreamArgs b, AnisoArg
 // ---------------------------------------------------------------------------
 // kernel k >= 1 of the Chronopoulos-Gear loop: r_{k-1}, w_{k-1}, s_{k-2} in,
 // s_{k-1}, r_k, w_k out (ping-pong by parity), p and x in place
+// (r-slabs: the three halo fields come with the ghost planes exchanged just
+// before the kernel: r -> rg, w -> pg[0], s -> pg[1])
 static void cg1_args(const mas_op* op, int k, StencilArgs& a) {
     const int nc = op->ncomp;
     double* R[2] = {op->r, op->r2};
     double* Wb[2] = {op->q, op->w2};
     double* S[2] = {op->p[0], op->p[1]};
-    a.u = halo_of(op, R[(k - 1) & 1], nullptr, nc);
-    a.w = halo_of(op, Wb[(k - 1) & 1], nullptr, nc);
-    a.pold = halo_of(op, S[k & 1], nullptr, nc);
+    a.u = halo_of(op, R[(k - 1) & 1], op->rg, nc);
+    a.w = halo_of(op, Wb[(k - 1) & 1], op->pg[0], nc);
+    a.pold = halo_of(op, S[k & 1], op->pg[1], nc);
     a.sout = S[(k - 1) & 1];
     a.rout = R[k & 1];
     a.out = Wb[k & 1];
@@ -730,10 +732,27 @@ static mas_status_t cg1_graph(mas_op* op, StencilArgs a) {
     return MAS_OK;
 }
 
+// the seams kernel k >= 1 reads: r_{k-1}, w_{k-1}, s_{k-2} (NCCL loop on r-slabs)
+static mas_status_t cg1_seams(mas_op* op, int k, cudaStream_t s) {
+    Comm* comm = op->g->comm;
+    if (!comm) return MAS_OK;
+    const int nc = op->ncomp;
+    const long long plane = op->geo.plane;
+    double* R[2] = {op->r, op->r2};
+    double* Wb[2] = {op->q, op->w2};
+    double* S[2] = {op->p[0], op->p[1]};
+    ST(comm_seams(comm, R[(k - 1) & 1], nc, op->g->nl, plane, op->rg, op->rg + nc * plane, s));
+    ST(comm_seams(comm, Wb[(k - 1) & 1], nc, op->g->nl, plane, op->pg[0], op->pg[0] + nc * plane, s));
+    ST(comm_seams(comm, S[k & 1], nc, op->g->nl, plane, op->pg[1], op->pg[1] + nc * plane, s));
+    return MAS_OK;
+}
+
 static mas_status_t cg1_solve(mas_op* op, const double* fd, double* xd, double tol, int maxit, int* iters,
                               double* relres, double* res_hist, cudaStream_t s) {
     const int nc = op->ncomp;
     const size_t bytes = nc * op->Nl * sizeof(double);
+    Comm* comm = op->g->comm;
+    const long long plane = op->geo.plane;
     op->launches = 0;
     PcgState init{};
     init.tol = tol;
@@ -752,8 +771,8 @@ static mas_status_t cg1_solve(mas_op* op, const double* fd, double* xd, double t
     StencilArgs a{};
     a.g = op->geo;
     a.chunk = op->chunk;
-    a.kappa = halo_of(op, op->kappa, nullptr, 1);
-    a.dinv = halo_of(op, op->dinv, nullptr, 1);
+    a.kappa = halo_of(op, op->kappa, op->kg, 1);
+    a.dinv = halo_of(op, op->dinv, op->dg, 1);
     a.c = op->c;
     a.curv = op->curv;
     a.st = op->st;
@@ -763,14 +782,19 @@ static mas_status_t cg1_solve(mas_op* op, const double* fd, double* xd, double t
     a.scr = op->scr;
     a.host_flag = op->host_flag_dev;
     // a3: r0 = f - L x0 and <f,f>, <r0,r0> (k_stencil<RESID>, as the standard loop)
+    if (comm) ST(comm_seams(comm, xd, nc, op->g->nl, plane, op->xg, op->xg + nc * plane, s));
     StencilArgs r0 = a;
-    r0.u = halo_of(op, xd, nullptr, nc);
+    r0.u = halo_of(op, xd, op->xg, nc);
     r0.f = fd;
     r0.out = op->r;
     CU(launch_stencil(MODE_RESID, nc, r0, s));
     op->launches++;
+    if (comm) {  // the init sums over the ranks; r0's edge planes for the init kernel
+        ST(comm_allreduce(comm, &op->st->pend_rho, 3, s));  // rho, rr, ff
+        ST(comm_seams(comm, op->r, nc, op->g->nl, plane, op->rg, op->rg + nc * plane, s));
+    }
     a.x = xd;
-    const bool graph = !op->prof && op->use_graph;
+    const bool graph = !op->prof && op->use_graph && !comm;
     if (graph) {
         ST(cg1_graph(op, a));
         CU(cudaGraphLaunch(op->gexec1, s));
@@ -786,24 +810,28 @@ static mas_status_t cg1_solve(mas_op* op, const double* fd, double* xd, double t
             }
             if (n == 1) {
                 StencilArgs a0 = a;
-                a0.u = halo_of(op, op->r, nullptr, nc);
+                a0.u = halo_of(op, op->r, op->rg, nc);
                 a0.out = op->q;
                 CU(launch_stencil(MODE_CG1, nc, a0, s, true));
             } else {
+                ST(cg1_seams(op, n - 1, s));
+                if (pe) CU(cudaEventRecord(pe[0], s));
                 cg1_args(op, n - 1, a);
                 CU(launch_stencil(MODE_CG1, nc, a, s));
             }
             op->launches++;
             if (pe) CU(cudaEventRecord(pe[1], s));
+            // the one allreduce of the iteration: (gamma, delta, ||r||^2) in place
+            if (comm) ST(comm_allreduce(comm, &op->st->pend_sigma, 3, s));
             CU(cudaEventRecord(op->ev[n & 1], s));
             if (n >= 2) {
-                CU(cudaEventSynchronize(op->ev[(n - 1) & 1]));
+                ST(comm_wait_event(comm, op->ev[(n - 1) & 1]));
                 const int flag = *(volatile int*)op->host_flag;
                 if (flag > 0 && flag <= n - 1) break;
             }
         }
     }
-    CU(cudaStreamSynchronize(s));
+    ST(comm_sync_stream(comm, s));
     PcgState fin{};
     CU(cudaMemcpy(&fin, op->st, sizeof(fin), cudaMemcpyDeviceToHost));
     if (!fin.stopped) {
@@ -812,7 +840,10 @@ static mas_status_t cg1_solve(mas_op* op, const double* fd, double* xd, double t
     }
     *iters = fin.iters;
     *relres = fin.relres;
-    if (graph) op->launches += 1 + fin.iters + (fin.iters & 1);  // init + kernels (+ an early exit)
+    if (graph) {  // the init + whole bodies of 2 kernels up to the deciding kernel (iters + 1)
+        const int d = fin.status == MAS_ERR_BREAKDOWN && fin.iters == 1 ? 1 : fin.iters + 1;
+        op->launches += 1 + 2 * ((d + 1) / 2);
+    }
     if (res_hist) {
         const int nh = (fin.status == MAS_ERR_BREAKDOWN && fin.iters == 1) ? 1 : fin.iters + 1;
         std::vector<double> rr(nh);
@@ -1173,6 +1204,7 @@ mas_status_t mas_op_enable_p2p(mas_op_t* op, cudaStream_t s) {
     if (!op) return arg_error("null op");
     if (op->p2p) return MAS_OK;
     if (op->tnode) return arg_error("P2P transport: cell-centred placement only (theta nodes keep NCCL)");
+    if (op->cg1) return arg_error("P2P transport: the two-kernel loop only (single reduction is on)");
     Comm* comm = op->g->comm;
     const int P = comm_nranks(comm), rank = comm_rank(comm);
     const bool virt = comm_is_virtual(comm);
@@ -1280,7 +1312,8 @@ mas_status_t mas_op_set_single_reduction(mas_op_t* op, int on) {
         op->cg1 = 0;
         return MAS_OK;
     }
-    if (op->g->comm) return arg_error("single-reduction PCG: one GPU only (no mas_dist_t)");
+    if (op->p2p) return arg_error("single-reduction PCG: the NCCL loop on r-slabs (not the P2P transport)");
+    if (op->g->ptheta > 1) return arg_error("single-reduction PCG: r-slab decompositions only (ptheta == 1)");
     if (op->aniso) return arg_error("single-reduction PCG: isotropic operator only (no mas_op_set_aniso)");
     if (op->tnode) return arg_error("single-reduction PCG: cell-centred placement only");
     if (op->curv) return arg_error("single-reduction PCG: without the curvature terms");

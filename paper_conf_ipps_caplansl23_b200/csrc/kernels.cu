@@ -582,6 +582,9 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
     // ---- PCG scalars (all threads read the same device values) ----------
     int pmode = P_NORMAL;
     bool first = false;
+    // CG1: the global sums of kernel k-1 and, on a stop, its status / count
+    double cg_g1 = 0.0, cg_d1 = 0.0, cg_rr1 = 0.0;
+    int cg_status = -1, cg_iters = 0;
     double beta = 0.0, alpha_prev = 0.0;
     int kit = 0;
     const bool p2p = a.p2p.nranks > 0;
@@ -612,8 +615,11 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
         else if (!first)
             beta = rho1 / rho2;
     } else if (MODE == MODE_CG1) {
-        // single reduction: kernel k's last block decided alpha_k, beta_k and
-        // the stop; here (k+1) everything comes from PcgState
+        // single reduction: kernel k (k >= 1) finds in PcgState the GLOBAL sums
+        // of kernel k-1 (gamma_{k-1}, delta_{k-1}, ||r_{k-1}||^2; allreduced in
+        // place between the kernels on r-slabs) and the gamma_{k-2}, alpha_{k-2}
+        // kernel k-1 saved.  Every block takes the same decision: stop (r_{k-1}
+        // met tol, maxit reached, breakdown), else alpha_{k-1}, beta_{k-1}.
         const PcgState* st = a.st;
         if (__ldcg(&st->stopped)) {
             if (a.cond && blockIdx.x == 0 && threadIdx.x == 0)
@@ -621,16 +627,32 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
             return;
         }
         kit = __ldcg(&st->k);
+        const double ff = __ldcg(&st->pend_ff);
         if (FIRSTK) {  // the init: k = 0; r0 from k_stencil<RESID>
-            const double ff = __ldcg(&st->pend_ff), rr = __ldcg(&st->pend_rr);
+            const double rr = __ldcg(&st->pend_rr);
             final_g[0] = ff, final_g[1] = rr, final_g[2] = 0.0;
             if (ff == 0.0)
                 pmode = P_ZERO;
             else if (sqrt(rr) <= __ldcg(&st->tol) * sqrt(ff) || __ldcg(&st->maxit) == 0)
                 pmode = P_FINAL;
         } else {
-            alpha_prev = __ldcg(&st->cg_alpha);  // alpha_{k-1}
-            beta = __ldcg(&st->cg_beta);         // beta_{k-1}
+            cg_g1 = __ldcg(&st->pend_rho);
+            cg_d1 = __ldcg(&st->pend_sigma);
+            cg_rr1 = __ldcg(&st->pend_rr);
+            if (kit >= 2 && sqrt(cg_rr1) <= __ldcg(&st->tol) * sqrt(ff)) {
+                pmode = P_FINAL, cg_status = MAS_OK, cg_iters = kit - 1;
+            } else if (kit >= 2 && kit - 1 >= __ldcg(&st->maxit)) {
+                pmode = P_FINAL, cg_status = MAS_NOT_CONVERGED, cg_iters = kit - 1;
+            } else {
+                const double b = kit >= 2 ? cg_g1 / __ldcg(&st->cg_gamma) : 0.0;
+                const double den = kit >= 2 ? cg_d1 - b * cg_g1 / __ldcg(&st->cg_alpha) : cg_d1;  // <p,Lp>
+                if (!(den > 0.0) || !isfinite(den)) {
+                    pmode = P_FINAL, cg_status = MAS_ERR_BREAKDOWN, cg_iters = kit >= 2 ? kit - 1 : 1;
+                } else {
+                    beta = b;                     // beta_{k-1}
+                    alpha_prev = cg_g1 / den;     // alpha_{k-1}
+                }
+            }
         }
     }
     const bool xupd = (MODE == MODE_PCGA || MODE == MODE_CG1) && !FIRSTK;
@@ -680,11 +702,16 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
         if (grid_reduce<1, kSThreads>(v1, a.scr, TKT_STENCIL) && threadIdx.x == 0 && a.part != 1) {
             PcgState* st = a.st;
             const double ff = final_g[0], rr = final_g[1], rho1 = final_g[2];
-            // PCGA: A(k) stops at iterate k-1;  CG1: only its init (k = 0) lands here
-            const int hk = MODE == MODE_CG1 ? 0 : kit - 1;
-            a.rr_hist[hk] = rr;
-            a.rho_hist[hk] = rho1;
-            if (pmode == P_ZERO) {
+            // PCGA: A(k) stops at iterate k-1;  CG1: kernel k at iterate k-1 (its
+            // init, k = 0, at iterate 0)
+            const int hk = MODE == MODE_CG1 ? (FIRSTK ? 0 : kit - 1) : kit - 1;
+            a.rr_hist[hk] = (MODE == MODE_CG1 && !FIRSTK) ? cg_rr1 : rr;
+            a.rho_hist[hk] = (MODE == MODE_CG1 && !FIRSTK) ? cg_g1 : rho1;
+            if (MODE == MODE_CG1 && !FIRSTK) {
+                st->iters = cg_iters;
+                st->relres = sqrt(cg_rr1) / sqrt(st->pend_ff);
+                st->status = cg_status;
+            } else if (pmode == P_ZERO) {
                 st->iters = 0;
                 st->relres = 0.0;
                 st->status = MAS_OK;
@@ -897,43 +924,21 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
         }
     } else if (MODE == MODE_CG1) {
         if (grid_reduce<3, kSThreads>(acc, a.scr, TKT_STENCIL) && threadIdx.x == 0) {
-            // the single reduction of iteration k: gamma_k, delta_k, ||r_k||^2.
-            // Decide the stop, else alpha_k and beta_k for kernel k+1 (R28).
+            // the single reduction of iteration k: this rank's gamma_k, delta_k,
+            // ||r_k||^2 (summed over the ranks before kernel k+1 reads them).
+            // Kernel k+1 decides; here the values it needs besides them.
             PcgState* st = a.st;
-            const double gam = acc[0], del = acc[1], rr = acc[2];
-            const double ff = st->pend_ff;
-            a.rr_hist[kit] = rr;
-            a.rho_hist[kit] = gam;
-            a.sigma_hist[kit] = del;
-            int status = -1, iters = 0;
-            if (!FIRSTK && sqrt(rr) <= st->tol * sqrt(ff)) {
-                status = MAS_OK, iters = kit;
-            } else if (!FIRSTK && kit >= st->maxit) {
-                status = MAS_NOT_CONVERGED, iters = kit;
-            } else {
-                const double b = FIRSTK ? 0.0 : gam / st->cg_gamma;
-                const double den = FIRSTK ? del : del - b * gam / st->cg_alpha;  // <p_k, L p_k>
-                if (!(den > 0.0) || !isfinite(den)) {
-                    status = MAS_ERR_BREAKDOWN, iters = FIRSTK ? 1 : kit;
-                } else {
-                    st->cg_alpha = gam / den;
-                    st->cg_beta = b;
-                    st->cg_gamma = gam;
-                    st->k = kit + 1;
-                }
+            if (!FIRSTK) {
+                st->cg_gamma = cg_g1;        // gamma_{k-1}
+                st->cg_alpha = alpha_prev;   // alpha_{k-1}
+                a.rr_hist[kit - 1] = cg_rr1;
+                a.rho_hist[kit - 1] = cg_g1;
+                a.sigma_hist[kit - 1] = cg_d1;
             }
-            if (status >= 0) {
-                st->iters = iters;
-                st->relres = sqrt(rr) / sqrt(ff);
-                st->status = status;
-                __threadfence();
-                st->stopped = 1;
-                if (a.host_flag) {
-                    __threadfence_system();
-                    *(volatile int*)a.host_flag = kit + 1;  // launch number (init = 1)
-                }
-                if (a.cond) cudaGraphSetConditional((cudaGraphConditionalHandle)a.cond, 0);
-            }
+            st->pend_rho = acc[0];
+            st->pend_sigma = acc[1];
+            st->pend_rr = acc[2];
+            st->k = kit + 1;
         }
     } else if (MODE == MODE_PCGA) {
         double v[1] = {acc[0]};

@@ -155,8 +155,78 @@ def test_single_reduction_switch_and_refusals(mp, oracle_mod):
     oa.set_single_reduction(True)
     with pytest.raises(mp.MasError):
         oa.set_aniso(dev(pa.kpar), dev(pa.bhat))
-    # a grid with a communicator (1-rank NCCL): refused
-    gd = mp.Grid(prob.mesh, dist=(1, 0, mp.mas_comm_unique_id()))
-    od = mp.Operator(gd, prob.ncomp, dev(prob.kappa), dev(prob.c), prob.bc_inner, prob.bc_outer)
+    # the P2P transport and the single-reduction loop refuse each other
+    gp = mp.Grid(prob.mesh)
+    op2 = mp.Operator(gp, prob.ncomp, dev(prob.kappa), dev(prob.c), prob.bc_inner, prob.bc_outer)
+    op2.enable_p2p()
     with pytest.raises(mp.MasError):
-        od.set_single_reduction(True)
+        op2.set_single_reduction(True)
+    op3 = mp.Operator(gp, prob.ncomp, dev(prob.kappa), dev(prob.c), prob.bc_inner, prob.bc_outer)
+    op3.set_single_reduction(True)
+    with pytest.raises(mp.MasError):
+        op3.enable_p2p()
+
+
+@pytest.mark.parametrize("mk", ["viscosity", "conduction"])
+def test_single_reduction_one_rank_nccl(mp, oracle_mod, mk):
+    """The r-slab loop (seams of r, w, s; ONE ncclAllReduce of 3 doubles per
+    iteration; the decision in the next kernel) on a 1-rank NCCL communicator."""
+    prob = W.viscosity_problem(24, 16, 64) if mk == "viscosity" else W.conduction_problem(40, 16, 32)
+    g = mp.Grid(prob.mesh, dist=(1, 0, mp.mas_comm_unique_id()))
+    op = mp.Operator(g, prob.ncomp, dev(prob.kappa), dev(prob.c), prob.bc_inner, prob.bc_outer)
+    op.set_single_reduction(True)
+    f = dev(prob.f)
+    if prob.ub_inner is not None:
+        op.dirichlet_rhs(dev(prob.ub_inner), None, f)
+    x = dev(prob.x0)
+    st, it, rel, hist = op.solve(f, x, prob.tol, prob.maxit, True)
+    rc, xo, ito, _, histo = oracle_mod.solve_problem(prob, cg1=True)
+    V = oracle_mod.Oracle.for_problem(prob).volumes()
+    assert st == mp.MAS_OK and abs(it - ito) <= 2
+    assert rel_l2_V(V, x.cpu().numpy(), xo) <= 1e-9
+    np.testing.assert_allclose(hist[:10], histo[:10], rtol=1e-9, atol=0)
+
+
+@pytest.mark.parametrize("P", [2, 3])
+def test_single_reduction_virtual_ranks(mp, oracle_mod, P):
+    """r-slabs on P virtual ranks: every rank stops at the same iteration;
+    iterations +-2 and x <= 1e-9 against the oracle's monolithic CG1."""
+    import threading
+    prob = W.viscosity_problem(13 * P, 16, 64, warm=False)
+    vid = mp.virtual_ranks_id(7700 + P)
+    res, errs = {}, []
+
+    def rank_main(r):
+        try:
+            torch.cuda.set_device(0)
+            with torch.cuda.stream(torch.cuda.Stream()):
+                g = mp.Grid(prob.mesh, dist=(P, r, vid))
+                sl = slice(g.i0, g.i0 + g.nl)
+                op = mp.Operator(g, 3, dev(prob.kappa[sl]), dev(prob.c[sl]), prob.bc_inner,
+                                 prob.bc_outer)
+                op.set_single_reduction(True)
+                x = dev(prob.x0[:, sl])
+                st, it, rel, _ = op.solve(dev(prob.f[:, sl]), x, prob.tol, prob.maxit)
+                torch.cuda.current_stream().synchronize()
+                res[r] = (g.i0, g.nl, st, it, x.cpu().numpy())
+                op.close()
+                g.close()
+        except Exception as e:  # noqa: BLE001
+            errs.append((r, repr(e)))
+
+    th = [threading.Thread(target=rank_main, args=(r,)) for r in range(P)]
+    for t in th:
+        t.start()
+    for t in th:
+        t.join(timeout=600)
+    assert not errs, errs
+    rc, xo, ito, _, _ = oracle_mod.solve_problem(prob, cg1=True)
+    its = {res[r][3] for r in range(P)}
+    assert len(its) == 1, its
+    assert abs(its.pop() - ito) <= 2
+    xg = np.empty_like(xo)
+    for r in range(P):
+        i0, nl, st, it, x = res[r]
+        assert st == mp.MAS_OK
+        xg[:, i0:i0 + nl] = x
+    assert rel_l2_V(oracle_mod.Oracle.for_problem(prob).volumes(), xg, xo) <= 1e-9
