@@ -17,7 +17,7 @@ cap() {  # name regex skip args...
 }
 cap C3_kernelA k_stencil 2 --config C3
 cap C3_kernelB k_pcg_b 1 --config C3
-cap C2a_kaniso k_aniso 2 --config C2a
+cap C2a_kaniso k_aniso 3 --config C2a  # launches: coef, diag, RESID, PCGA
 cap C2_kernelA k_stencil 2 --config C2
 cap C2_kernelB k_pcg_b 1 --config C2
 cap C2_cg1 k_stencil 3 --config C2 --solver cg1
