@@ -370,6 +370,135 @@ __global__ void __launch_bounds__(WTHREADS, kAnisoBps) k_aniso(const AnisoArgs a
             };
             for (int n = 0; n < nst; n++) issue(n);
         } else {
+#ifdef MAS_ANISO_V2
+            // ---- consumers (V2, experiment: measured 81 us against V1's 53.7 us
+            // at C2a -- the 3x corner recomputation and register spills at the
+            // 96-register cap of a 544-thread block outweigh the saved barrier
+            // and shared-memory traffic; profiles/README.md r3d/r3e) ---------
+            // Warp w (cell row w) computes the corners of BOTH corner rows its
+            // cells touch (J = j0+w and j0+w+1) itself -- each corner twice, once
+            // per warp -- and folds them into per-cell sums held in registers:
+            //   V y_P = [sum_JK A(i,J,K) - sum_JK A(i+1,J,K)]
+            //         + [sum_IK B(I,j,K) - B(I,j+1,K)] + [sum_IJ E(I,J,k) - E(I,J,k+1)]
+            // with (A, B, E) = s_c (a, b, e).  No shared-memory stores, no
+            // consumer barrier; a stage is released as soon as its step is done.
+            const int w = warp, l2 = 2 * lane;
+            const bool first = k0 == 0, last = k0 + width == g.np;
+            const bool rows_ok = w < height;                  // this warp's row exists
+            const bool active = rows_ok && l2 < width;       // this lane's cell pair
+            const bool lfix = first && lane == 0;            // column k0-1: the left side box
+            const bool rfix = last && l2 + 2 == width;       // column k0+width: the right side box
+            double cw0 = 0.0, cw1 = 0.0;  // 1 / (vt_j vp_k) of the two cells
+            if (active) {
+                const double vt = __ldg(g.vt + j0 + w);
+                cw0 = 1.0 / (vt * __ldg(g.vp + k0 + l2));
+                cw1 = 1.0 / (vt * __ldg(g.vp + k0 + l2 + 1));
+            }
+            // p of box rows w..w+2 (cell rows j-1..j+1), columns k-1..k+2 of the
+            // previous plane; the previous plane's per-cell corner sums
+            double pp[3][4];
+#pragma unroll
+            for (int r = 0; r < 3; r++)
+#pragma unroll
+                for (int c = 0; c < 4; c++) pp[r][c] = 0.0;
+            double pA0 = 0.0, pA1 = 0.0, pB0 = 0.0, pB1 = 0.0, pE0 = 0.0, pE1 = 0.0;
+            for (int n = 0; n < nst; n++) {
+                const int I = ia - 1 + n, slot = n % W_NSLOT;
+                mbar_wait(full0 + 8 * slot, (n / W_NSLOT) & 1);
+                const double* p1 = P_of(slot);
+                double pc[3][4];
+#pragma unroll
+                for (int r = 0; r < 3; r++) {
+                    const double* b = p1 + (w + r) * WPW + l2;
+                    const double2 v = rows_ok ? lds2(b + 2) : make_double2(0.0, 0.0);
+                    pc[r][0] = rows_ok ? (lfix ? p1[O_PL + 2 * (w + r) + 1] : b[1]) : 0.0;
+                    pc[r][1] = v.x;
+                    pc[r][2] = v.y;
+                    pc[r][3] = rows_ok ? (rfix ? p1[O_PR + 2 * (w + r)] : b[4]) : 0.0;
+                }
+                if (n > 0 && rows_ok) {
+                    // corners of plane I: rows q = 0 (J = j0+w), 1; columns K = l2 + kk
+                    const double* Cf = C_of(slot);
+                    const double* CS = p1 + O_CS;
+                    double SA[3], BD[3], SE[3];
+#pragma unroll
+                    for (int q = 0; q < 2; q++) {
+                        const double* cr = Cf + (w + q) * WCW + l2;
+                        const double2 a01 = lds2(cr), b01 = lds2(cr + WCA), e01 = lds2(cr + 2 * WCA);
+                        double ca[3] = {a01.x, a01.y, cr[2]};
+                        double cb[3] = {b01.x, b01.y, cr[WCA + 2]};
+                        double ce[3] = {e01.x, e01.y, cr[2 * WCA + 2]};
+                        if (rfix) {  // corner column k0 + width = np: the side box (K = 0)
+                            ca[2] = CS[2 * (w + q)];
+                            cb[2] = CS[2 * (WCR + w + q)];
+                            ce[2] = CS[2 * (2 * WCR + w + q)];
+                        }
+#pragma unroll
+                        for (int kk = 0; kk < 3; kk++) {
+                            const double a00 = pp[q][kk], a01v = pp[q][kk + 1], a10 = pp[q + 1][kk],
+                                         a11 = pp[q + 1][kk + 1];
+                            const double b00 = pc[q][kk], b01v = pc[q][kk + 1], b10 = pc[q + 1][kk],
+                                         b11 = pc[q + 1][kk + 1];
+                            const double Dr = ((b00 - a00) + (b01v - a01v)) + ((b10 - a10) + (b11 - a11));
+                            const double Dt = ((a10 - a00) + (a11 - a01v)) + ((b10 - b00) + (b11 - b01v));
+                            const double Dp = ((a01v - a00) + (a11 - a10)) + ((b01v - b00) + (b11 - b10));
+                            const double sc = ca[kk] * Dr + cb[kk] * Dt + ce[kk] * Dp;
+                            if (q == 0) {
+                                SA[kk] = sc * ca[kk];
+                                BD[kk] = sc * cb[kk];
+                                SE[kk] = sc * ce[kk];
+                                // sigma: the tile's own corners (row < height, column <
+                                // width) of the segment's own planes
+                                if (MODE == MODE_PCGA && kk < 2 && I < ib && l2 + kk < width) acc[0] += sc * sc;
+                            } else {
+                                SA[kk] += sc * ca[kk];
+                                BD[kk] -= sc * cb[kk];
+                                SE[kk] += sc * ce[kk];
+                            }
+                        }
+                    }
+                    const double A0 = SA[0] + SA[1], A1 = SA[1] + SA[2];
+                    const double B0 = BD[0] + BD[1], B1 = BD[1] + BD[2];
+                    const double E0 = SE[0] - SE[1], E1 = SE[1] - SE[2];
+                    // ---- cells (w, l2..l2+1) of plane i = I-1: corner planes i, I
+                    if (n >= 2 && active) {
+                        const int i = I - 1;
+                        const double s0 = ((pA0 - A0) + (pB0 + B0)) + (pE0 + E0);
+                        const double s1 = ((pA1 - A1) + (pB1 + B1)) + (pE1 + E1);
+                        const double ivr = __ldg(a.ivr + i);
+                        const double y0 = s0 * (ivr * cw0), y1 = s1 * (ivr * cw1);
+#ifdef MAS_ANISO_QTMA
+                        const double2 qv = lds2(Q_of(slot) + w * WK + l2);
+#else
+                        const double2 qv = ld2(a.out + (size_t)i * plane + (size_t)(j0 + w) * g.np + k0 + l2);
+#endif
+                        double* o = a.out + (size_t)i * plane + (size_t)(j0 + w) * g.np + k0 + l2;
+                        if (MODE == MODE_RESID) {
+                            const double r0 = qv.x - y0, r1 = qv.y - y1;
+                            stg2(o, make_double2(r0, r1));
+                            const double vr = __ldg(g.vr + i);
+                            const double V0 = vr / cw0, V1 = vr / cw1;
+                            const double2 f = ld2(a.f + (o - a.out));
+                            const double2 di = ld2(a.dinv + (o - a.out));
+                            acc[0] += V0 * f.x * f.x + V1 * f.y * f.y;
+                            acc[1] += V0 * r0 * r0 + V1 * r1 * r1;
+                            acc[2] += V0 * r0 * (di.x * r0) + V1 * r1 * (di.y * r1);
+                        } else {
+                            stg2(o, make_double2(qv.x + y0, qv.y + y1));
+                        }
+                    }
+                    pA0 = A0, pA1 = A1, pB0 = B0, pB1 = B1, pE0 = E0, pE1 = E1;
+                }
+#pragma unroll
+                for (int r = 0; r < 3; r++)
+#pragma unroll
+                    for (int c = 0; c < 4; c++) pp[r][c] = pc[r][c];
+                // this stage is no longer read (its p is in registers now)
+                fence_proxy_async();
+                __syncwarp();
+                if (lane == 0) mbar_arrive(empty0 + 8 * slot);
+            }
+#else
             // ---- consumers --------------------------------------------------
             const int w = warp, c2 = 2 * lane;
             const bool first = k0 == 0, last = k0 + width == g.np;
@@ -528,6 +657,7 @@ __global__ void __launch_bounds__(WTHREADS, kAnisoBps) k_aniso(const AnisoArgs a
                 __syncwarp();
                 if (lane == 0) mbar_arrive(empty0 + 8 * ((n - 1) % W_NSLOT));
             }
+#endif
         }
         __syncthreads();  // the next segment re-initialises the rings and barriers
     }
