@@ -13,7 +13,8 @@
 // multi-rank driver, ghost-plane kernels and stop handshake can be validated
 // on a single B200 (this run has no multi-GPU box).  It is selected by a
 // mas_dist_t.nccl_id beginning with "MASVIRT\0" followed by an 8-byte group
-// key.  It is a test transport, not a performance path.
+// key.  It is a test transport, not a performance path, and is honoured only
+// with MAS_TEST_TRANSPORTS=1 in the environment.
 #include <nccl.h>
 
 #include <chrono>
@@ -263,11 +264,25 @@ static mas_status_t vgroup_join(const mas_dist_t* d, Comm* c) {
     return MAS_OK;
 }
 
+// The virtual-rank and host-exchange transports exist to validate the
+// multi-rank code on one GPU; a production run never selects them by
+// accident: their ids are honoured only with MAS_TEST_TRANSPORTS=1 set.
+static bool test_transports_enabled() {
+    const char* e = getenv("MAS_TEST_TRANSPORTS");
+    return e && atoi(e) == 1;
+}
+
 mas_status_t comm_create(const mas_dist_t* d, Comm** out) {
+    const bool host_magic = memcmp(d->nccl_id, kHostMagic, 8) == 0;
+    const bool virt_magic = memcmp(d->nccl_id, kVirtMagic, 8) == 0;
+    if ((host_magic || virt_magic) && !test_transports_enabled()) {
+        set_last_error("test transport id (virtual ranks / host exchange) without MAS_TEST_TRANSPORTS=1");
+        return MAS_ERR_ARG;
+    }
     Comm* c = new Comm();
     c->nranks = d->nranks;
     c->rank = d->rank;
-    if (memcmp(d->nccl_id, kHostMagic, 8) == 0) {
+    if (host_magic) {
         char path[121];
         memcpy(path, d->nccl_id + 8, 120);
         path[120] = 0;
@@ -282,7 +297,7 @@ mas_status_t comm_create(const mas_dist_t* d, Comm** out) {
         *out = c;
         return MAS_OK;
     }
-    if (memcmp(d->nccl_id, kVirtMagic, 8) == 0) {
+    if (virt_magic) {
         mas_status_t s = vgroup_join(d, c);
         if (s != MAS_OK) {
             delete c;

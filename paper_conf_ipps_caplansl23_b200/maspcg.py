@@ -162,7 +162,8 @@ def mas_comm_unique_id() -> bytes:
 
 def virtual_ranks_id(key: int) -> bytes:
     """mas_dist_t.nccl_id selecting the in-process "virtual ranks" transport:
-    P ranks as P host threads on one GPU (test transport, see comm.cpp)."""
+    P ranks as P host threads on one GPU (test transport, see comm.cpp; the
+    library honours it only with MAS_TEST_TRANSPORTS=1 in the environment)."""
     return b"MASVIRT\0" + int(key).to_bytes(8, "little") + bytes(112)
 
 

@@ -4,6 +4,9 @@ import sys
 import pytest
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+# the library honours its test transports (virtual ranks, host exchange) only
+# with this set (comm.cpp); spawned test processes inherit it
+os.environ.setdefault("MAS_TEST_TRANSPORTS", "1")
 if ROOT not in sys.path:
     sys.path.insert(0, ROOT)
 

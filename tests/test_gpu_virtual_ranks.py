@@ -248,3 +248,25 @@ def test_virtual_ranks_theta_split_conduction_dirichlet_fixed_iterations(mp, ora
         assert all(r["st"] == mp.MAS_NOT_CONVERGED and r["it"] == 20 for r in out)
         xg = assemble(out, "x")
         assert math.sqrt((V * (xg - xo) ** 2).sum() / (V * xo ** 2).sum()) <= 1e-10
+
+
+def test_test_transports_need_opt_in(mp):
+    """A production process (no MAS_TEST_TRANSPORTS=1) cannot select the
+    virtual-rank test transport by its id: mas_grid_create returns
+    MAS_ERR_ARG (comm.cpp)."""
+    import os
+    import subprocess
+    import sys
+    code = (
+        "import sys; sys.path.insert(0, %r)\n"
+        "import torch; torch.cuda.set_device(0)\n"
+        "from paper_conf_ipps_caplansl23_b200 import maspcg as M, workloads as W\n"
+        "m = W.stretched_mesh(4, 8, 8)\n"
+        "try:\n"
+        "    M.Grid(m, dist=(2, 0, M.virtual_ranks_id(4242)))\n"
+        "    print('created')\n"
+        "except M.MasError as e:\n"
+        "    print('status', e.status)\n" % os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    env = {k: v for k, v in os.environ.items() if k != "MAS_TEST_TRANSPORTS"}
+    out = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True, timeout=300)
+    assert ("status %d" % mp.MAS_ERR_ARG) in out.stdout, (out.stdout, out.stderr[-2000:])

@@ -13,6 +13,7 @@ import argparse
 import json
 import math
 import os
+os.environ.setdefault("MAS_TEST_TRANSPORTS", "1")  # virtual ranks (comm.cpp)
 import sys
 import threading
 import time

@@ -2,6 +2,7 @@
 scalar and 3-component, ragged tiles, one chunk boundary, host-driven loop
 and CUDA-graph loop."""
 import os
+os.environ.setdefault("MAS_TEST_TRANSPORTS", "1")  # virtual ranks (comm.cpp)
 import sys
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
