@@ -543,6 +543,16 @@ def main():
     torch.cuda.synchronize()
     op.set_profiling(False)
     t_prof_ms = e2.elapsed_time(e3)
+    # device time per launch of the iteration kernels from back-to-back CUDA
+    # graph replays (no host dispatch between launches; mas_op_kernel_bench)
+    replay = None
+    if world == 1:
+        ra, rb, rc = op.kernel_bench(20)
+        replay = {"A_ms": ra, "B_ms": rb or None, "Lpar_ms": rc or None,
+                  "note": "20 launches of each kernel in a CUDA graph on the op's stream, each "
+                          "after an L2 flush (a read sweep over 2x L2) and a PCG-state reset; the same graph without "
+                          "the kernels is subtracted (CUDA events; device time, cold L2); the op's "
+                          "vectors hold test values"}
     comm = None
     if world > 1:  # the exchange steps of the NCCL loop, measured on this op (collective)
         seam_us, ar_us, seam_b = op.comm_bench(20)
@@ -566,16 +576,20 @@ def main():
     a_b, b_b = alg_bytes_per_cell(nc)
     if args.solver == "cg1":  # one kernel per iteration (kernel_times' A), no kernel B
         a_b, b_b = cg1_bytes_per_cell(nc), 0
+    c_b = ANISO_BYTES_PER_CELL if aniso else 0
+    fused = aniso and op.aniso_fused
+    if fused:  # L_par inside kernel A: + the corner coefficients (a, b, e) per cell
+        a_b, c_b = a_b + 24, 0
     a_ms = statistics.mean(ka)
     b_ms = statistics.mean(kb)
     peak, peak_src = load_peaks()
     achieved = a_b * cells_local / (a_ms / 1e3) / 1e9
-    c_b = ANISO_BYTES_PER_CELL if aniso else 0
     c_ms = statistics.mean(kc)
     iter_gbs = (a_b + b_b + c_b) * cells / (t_ms / 1e3 / iters_total) / 1e9
     traffic = None
     # the dominant kernel by device time: kernel A, or on C2a the L_par kernel
-    dom = ("k_aniso<PCGA> (L_par)", c_b, c_ms, "kaniso") if aniso and c_ms > a_ms else \
+    dom = ("k_aniso<PCGA> (L_par)", c_b, c_ms, "kaniso") if aniso and c_b and c_ms > a_ms else \
+        ("k_stencil<PCGA> + fused L_par (kernel A)", a_b, a_ms, "kernelA_lpar") if fused else \
         ("k_stencil<CG1> (single-reduction iteration)", a_b, a_ms, "cg1") if args.solver == "cg1" else \
         ("k_stencil<PCGA> (kernel A)", a_b, a_ms, "kernelA")
     dom_achieved = dom[1] * cells_local / (dom[2] / 1e3) / 1e9
@@ -666,6 +680,8 @@ def main():
                                        f"(r,theta) {world // args.ptheta}x{args.ptheta}"),
                        "transport": transport,
                        "solver": args.solver,
+                       **({"lpar": "fused into kernel A" if fused else "separate k_aniso kernel"}
+                          if aniso else {}),
                        "l2": (f"no flush: one iteration streams {(a_b + b_b + c_b) * cells_local / 1e6:.0f}"
                               f" MB ({8 * cells_local / 1e6:.0f} MB per field) through the 126 MB L2"),
                        "step": "mas_op_update + " + ("mas_op_set_aniso + " if aniso else "") +
@@ -683,7 +699,13 @@ def main():
                             "Lpar_alg_bytes_per_cell": c_b} if aniso and c_ms > 0 else {}),
                         "B_GBs": b_b * cells_local / (b_ms / 1e3) / 1e9 if b_ms > 0 else None,
                         "iter_alg_GBs": iter_gbs, "iter_frac": iter_gbs / peak,
-                        "alg_bytes_per_cell_iter": a_b + b_b + c_b},
+                        "alg_bytes_per_cell_iter": a_b + b_b + c_b,
+                        **({"replay": {**replay,
+                                       "A_frac": a_b * cells_local / (replay["A_ms"] / 1e3) / 1e9 / peak,
+                                       "B_frac": (b_b * cells_local / (replay["B_ms"] / 1e3) / 1e9 / peak)
+                                       if replay["B_ms"] else None,
+                                       "Lpar_frac": (c_b * cells_local / (replay["Lpar_ms"] / 1e3) / 1e9 / peak)
+                                       if replay["Lpar_ms"] else None}} if replay else {})},
             "e2e": e2e,
             **({"parity": parity, "comm": comm} if world > 1 else {}),
             "gpu_launches": launches,

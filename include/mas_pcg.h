@@ -300,6 +300,20 @@ MAS_API mas_status_t mas_op_set_profiling(mas_op_t* op, int on);
  * of the last profiled solve; n = number of iterations averaged. */
 MAS_API mas_status_t mas_op_kernel_times(const mas_op_t* op, double* a_ms, double* b_ms, int* n);
 
+/* Device time of the iteration kernels, one GPU (measurement helper for
+ * bench.py; SURVEY.md §8(d) "ncu per kernel ... time"): reps launches of
+ * kernel A (or the single-reduction kernel), kernel B and the L_par kernel,
+ * each captured in a CUDA graph, each launch preceded by an L2 flush and a
+ * reset of the PCG state; the same graph without the kernels is timed too
+ * and subtracted (CUDA events on the stream);
+ * a_ms / b_ms / c_ms: average per launch (0 for a kernel the op does not
+ * run).  The op's work vectors and PCG state are overwritten with test values
+ * (call between solves); the caller's arrays are not touched.
+ * Errors: MAS_ERR_ARG (reps < 1, null pointers, a grid with a mas_dist_t),
+ * MAS_ERR_CUDA. */
+MAS_API mas_status_t mas_op_kernel_bench(mas_op_t* op, int reps, double* a_ms, double* b_ms,
+                                         double* c_ms, cudaStream_t stream);
+
 /* Field-aligned (anisotropic) thermal conduction.
  * MAS conducts heat along the magnetic field; the paper names the
  * thermodynamic model of its test problem and the implicit
@@ -328,8 +342,18 @@ MAS_API mas_status_t mas_op_kernel_times(const mas_op_t* op, double* a_ms, doubl
 MAS_API mas_status_t mas_op_set_aniso(mas_op_t* op, const double* kpar, const double* bhat,
                                       cudaStream_t stream);
 
+/* 1 if the iteration's L_par runs inside kernel A (opt-in: MAS_LPAR_FUSED=1
+ * in the environment at mas_op_setup; kernel A then stages the corner
+ * coefficients of each r-plane, computes the tile's corner products once and
+ * adds L_par p to q and <p, L_par p> to sigma, so p_k and q skip the extra
+ * round trip to HBM -- but the two extra barriers per plane make it slower
+ * than the separate kernel), 0 if the separate k_aniso kernel
+ * runs (the default, or the term is off), -1 if op is NULL.  The init
+ * residual and mas_op_apply use the separate kernel either way. */
+MAS_API int mas_op_aniso_fused(const mas_op_t* op);
+
 /* Average device time (ms) of the L_par kernel over the last profiled solve
- * (mas_op_set_profiling); 0 when the term is off. */
+ * (mas_op_set_profiling); 0 when the term is off or fused into kernel A. */
 MAS_API mas_status_t mas_op_aniso_time(const mas_op_t* op, double* ms);
 
 /* Per-radius array reduction, the paper's Listings 3-5 ("sum0(i) =

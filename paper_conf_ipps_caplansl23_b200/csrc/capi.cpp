@@ -11,6 +11,7 @@
 #include <cmath>
 #include <cstdlib>
 #include <cstring>
+#include <functional>
 #include <new>
 #include <string>
 #include <vector>
@@ -162,6 +163,9 @@ struct mas_op {
     int tnode = 0;
     // vector-Laplacian curvature terms of the 3-component operator (NEXT-2, R31)
     int curv = 0;
+    // the field-aligned term's iteration part fused into kernel A
+    // (MAS_LPAR_FUSED=1 at setup; default: the separate k_aniso<PCGA>)
+    int lpar_fused = 0;
     cudaGraphExec_t gexec1 = nullptr;
     const double* g1_x = nullptr;
     double* atab = nullptr;                      // AnisoTab arrays (device)
@@ -423,6 +427,15 @@ static const double* aniso_ca_hi(const mas_op* op) {
     return (op->cag && !op->geo.glob_hi) ? op->cag + 3 * op->geo.plane : nullptr;
 }
 
+// the iteration's L_par runs inside kernel A (k_stencil<PCGA, 1, *, LPAR>)
+static bool lpar_in_a(const mas_op* op) { return op->aniso && op->lpar_fused; }
+// kernel A's arguments for the fused term (nullptr ca: off)
+static void set_lpar_args(const mas_op* op, StencilArgs& a) {
+    a.ca = lpar_in_a(op) ? op->ca : nullptr;
+    a.ca_hi = lpar_in_a(op) ? aniso_ca_hi(op) : nullptr;
+    a.ivr = op->at.ivr;
+}
+
 // D (optional) and 1/D: the 7-point diagonal (k_diag), plus the field-aligned
 // term's diagonal (R26) when L_par is on (D then goes through a device buffer:
 // the caller's, or q, which is free outside a solve).
@@ -554,7 +567,8 @@ static mas_status_t ensure_prof_events(mas_op* op, int k) {
 // (MAS_GRAPH_PRE=1, an experiment hook, launches iteration 1 as plain
 // kernels ahead of a graph holding only the while node, the round-1 form.)
 static mas_status_t loop_graph(mas_op* op, StencilArgs a, StreamArgs b, AnisoArgs an, bool pre_plain) {
-    if (op->gexec && op->g_x == a.x && op->g_hist == a.rho_hist && op->g_aniso == op->aniso &&
+    const int aniso_key = op->aniso ? (lpar_in_a(op) ? 2 : 1) : 0;
+    if (op->gexec && op->g_x == a.x && op->g_hist == a.rho_hist && op->g_aniso == aniso_key &&
         op->g_pre == (int)pre_plain)
         return MAS_OK;
     if (op->gexec) {
@@ -576,7 +590,7 @@ static mas_status_t loop_graph(mas_op* op, StencilArgs a, StreamArgs b, AnisoArg
             a1.tpold = pold_trows(op, 1);
             a1.pnew = op->p[1];
             e = launch_stencil(MODE_PCGA, nc, a1, op->cap_stream, true);
-            if (e == cudaSuccess && op->aniso) {
+            if (e == cudaSuccess && op->aniso && !lpar_in_a(op)) {
                 AnisoArgs an1 = an;
                 an1.u = aniso_p_halo(op, 1);
                 e = launch_aniso(MODE_PCGA, an1, op->cap_stream);
@@ -624,7 +638,7 @@ static mas_status_t loop_graph(mas_op* op, StencilArgs a, StreamArgs b, AnisoArg
                 a.pnew = op->p[kk & 1];
                 e = launch_stencil(MODE_PCGA, nc, a, op->cap_stream);
                 an.u = aniso_p_halo(op, kk);
-                if (e == cudaSuccess && op->aniso) e = launch_aniso(MODE_PCGA, an, op->cap_stream);
+                if (e == cudaSuccess && op->aniso && !lpar_in_a(op)) e = launch_aniso(MODE_PCGA, an, op->cap_stream);
                 if (e == cudaSuccess && op->tnode)
                     e = launch_pole_avg(op->geo, nc, op->q, nullptr, 0, op->geo.nl, op->cap_stream);
                 if (e == cudaSuccess) e = launch_pcg_b(b, op->b_blocks, op->cap_stream);
@@ -644,7 +658,7 @@ static mas_status_t loop_graph(mas_op* op, StencilArgs a, StreamArgs b, AnisoArg
     }
     op->g_x = a.x;
     op->g_hist = a.rho_hist;
-    op->g_aniso = op->aniso;
+    op->g_aniso = aniso_key;
     op->g_pre = (int)pre_plain;
     return MAS_OK;
 }
@@ -1004,6 +1018,10 @@ mas_status_t mas_op_setup_placed(mas_grid_t* g, int ncomp, int placement, const 
     op->use_graph = !(g_env && atoi(g_env));
     const char* gp_env = getenv("MAS_GRAPH_PRE");  // experiment hook (round-1 graph form)
     op->graph_pre = gp_env && atoi(gp_env);
+    // experiment hook: the iteration's L_par inside kernel A (correct, but
+    // measured slower than the separate k_aniso: profiles/README.md r3l)
+    const char* lf_env = getenv("MAS_LPAR_FUSED");
+    op->lpar_fused = lf_env && atoi(lf_env) == 1;
     const char* ch_env = getenv("MAS_CHUNK");  // experiment hook
     op->chunk = ch_env ? atoi(ch_env) : (nl >= 128 ? 32 : nl >= 64 ? 16 : (nl >= 16 ? 8 : 4));
     if (!ch_env && multi && nl >= 12) {
@@ -1327,6 +1345,168 @@ mas_status_t mas_op_set_single_reduction(mas_op_t* op, int on) {
 
 int mas_op_single_reduction(const mas_op_t* op) { return op ? op->cg1 : -1; }
 
+int mas_op_aniso_fused(const mas_op_t* op) { return !op ? -1 : lpar_in_a(op) ? 1 : 0; }
+
+// Kernel-replay timing: reps launches of one kernel captured in a CUDA graph,
+// each preceded by an L2 flush (a read-only sweep over twice the L2 size) and a
+// reset of the PCG state to a mid-solve iteration.  A second graph holds the
+// flushes and resets alone; the time per launch is the difference of the two
+// graphs' event-timed durations over reps (device time, cold L2, no host
+// dispatch between launches).
+static mas_status_t time_graph(cudaStream_t cap, cudaStream_t s, int reps, void* flush, size_t flush_bytes,
+                               PcgState* st, const PcgState* st_init,
+                               const std::function<cudaError_t(cudaStream_t)>* launch, float* ms) {
+    cudaGraph_t g;
+    cudaError_t e = cudaStreamBeginCapture(cap, cudaStreamCaptureModeThreadLocal);
+    for (int i = 0; i < reps && e == cudaSuccess; i++) {
+        e = launch_l2_sweep(static_cast<const double*>(flush), (long long)(flush_bytes / sizeof(double)),
+                            static_cast<double*>(flush), cap);
+        if (e == cudaSuccess) e = cudaMemcpyAsync(st, st_init, sizeof(PcgState), cudaMemcpyDeviceToDevice, cap);
+        if (e == cudaSuccess && launch) e = (*launch)(cap);
+    }
+    cudaError_t e2 = cudaStreamEndCapture(cap, &g);
+    if (e != cudaSuccess || e2 != cudaSuccess) {
+        if (e2 == cudaSuccess) cudaGraphDestroy(g);
+        cudaGetLastError();
+        set_last_error(std::string("kernel replay capture: ") + cudaGetErrorString(e != cudaSuccess ? e : e2));
+        return MAS_ERR_CUDA;
+    }
+    cudaGraphExec_t ge;
+    e = cudaGraphInstantiate(&ge, g, 0);
+    cudaGraphDestroy(g);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        set_last_error(std::string("kernel replay instantiate: ") + cudaGetErrorString(e));
+        return MAS_ERR_CUDA;
+    }
+    cudaEvent_t e0 = nullptr, e1 = nullptr;
+    e = cudaEventCreate(&e0);
+    if (e == cudaSuccess) e = cudaEventCreate(&e1);
+    if (e == cudaSuccess) e = cudaGraphLaunch(ge, s);  // warm-up
+    if (e == cudaSuccess) e = cudaEventRecord(e0, s);
+    if (e == cudaSuccess) e = cudaGraphLaunch(ge, s);
+    if (e == cudaSuccess) e = cudaEventRecord(e1, s);
+    if (e == cudaSuccess) e = cudaEventSynchronize(e1);
+    if (e == cudaSuccess) e = cudaEventElapsedTime(ms, e0, e1);
+    if (e0) cudaEventDestroy(e0);
+    if (e1) cudaEventDestroy(e1);
+    cudaGraphExecDestroy(ge);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        set_last_error(std::string("kernel replay: ") + cudaGetErrorString(e));
+        return MAS_ERR_CUDA;
+    }
+    return MAS_OK;
+}
+
+static mas_status_t replay_time(cudaStream_t cap, cudaStream_t s, int reps, double* ms, void* flush,
+                                size_t flush_bytes, PcgState* st, const PcgState* st_init,
+                                const std::function<cudaError_t(cudaStream_t)>& launch) {
+    float with = 0.f, without = 0.f;
+    ST(time_graph(cap, s, reps, flush, flush_bytes, st, st_init, &launch, &with));
+    ST(time_graph(cap, s, reps, flush, flush_bytes, st, st_init, nullptr, &without));
+    *ms = (double)(with - without) / reps;
+    return MAS_OK;
+}
+
+mas_status_t mas_op_kernel_bench(mas_op_t* op, int reps, double* a_ms, double* b_ms, double* c_ms,
+                                 cudaStream_t s) {
+    if (!op || !a_ms || !b_ms || !c_ms || reps < 1) return arg_error("bad argument");
+    if (op->g->comm) return arg_error("kernel replay timing: one GPU (no mas_dist_t)");
+    *a_ms = *b_ms = *c_ms = 0.0;
+    const int nc = op->ncomp;
+    const long long n = nc * op->Nl;
+    ST(ensure_stage(op));
+    ST(ensure_hist(op, 2 * reps + 8));
+    if (op->cg1) {
+        if (!op->r2) return arg_error("single-reduction buffers missing");
+    }
+    for (double* v : {op->r, op->p[0], op->p[1], op->q}) CU(launch_fill_test(v, n, s));
+    if (op->cg1)
+        for (double* v : {op->r2, op->w2, op->pcg}) CU(launch_fill_test(v, n, s));
+    CU(cudaMemsetAsync(op->stage_b, 0, n * sizeof(double), s));
+    // the PCG state every replay starts from: iteration 2, tol 0, no stop
+    // (for the single-reduction kernel: delta - beta gamma / alpha = 2 - 1 > 0)
+    PcgState init{};
+    init.tol = 0.0;
+    init.maxit = 1 << 30;
+    init.k = 2;
+    init.pend_rho = init.rho_prev = init.sigma_prev = init.pend_rr = init.pend_ff = 1.0;
+    init.pend_sigma = 2.0;
+    init.cg_alpha = init.cg_gamma = 1.0;
+    init.status = MAS_NOT_CONVERGED;
+    PcgState* st_init = nullptr;
+    ST(dmalloc(reinterpret_cast<double**>(&st_init), (sizeof(PcgState) + 7) / 8));
+    void* flush = nullptr;
+    int l2 = 0, dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, dev);
+    const size_t flush_bytes = 2 * (size_t)(l2 > 0 ? l2 : 128 << 20);
+    if (cudaMalloc(&flush, flush_bytes) != cudaSuccess) {
+        cudaGetLastError();
+        cudaFree(st_init);
+        set_last_error("kernel replay: flush buffer");
+        return MAS_ERR_NOMEM;
+    }
+    struct Free {
+        void* a;
+        void* b;
+        ~Free() {
+            cudaFree(a);
+            cudaFree(b);
+        }
+    } free_on_exit{flush, st_init};
+    CU(cudaMemcpyAsync(st_init, &init, sizeof(init), cudaMemcpyHostToDevice, s));
+    CU(cudaMemsetAsync(flush, 0, flush_bytes, s));  // the sweep reads zeros
+    if (!op->cap_stream) CU(cudaStreamCreateWithFlags(&op->cap_stream, cudaStreamNonBlocking));
+    CU(cudaStreamSynchronize(s));
+    StencilArgs a{};
+    a.g = op->geo;
+    a.chunk = op->chunk;
+    a.kappa = halo_of(op, op->kappa, nullptr, 1);
+    a.dinv = halo_of(op, op->dinv, nullptr, 1);
+    a.c = op->c;
+    a.curv = op->curv;
+    a.st = op->st;
+    a.rho_hist = op->hist;
+    a.sigma_hist = op->hist + op->hist_cap;
+    a.rr_hist = op->hist + 2 * op->hist_cap;
+    a.scr = op->scr;
+    a.x = op->stage_b;
+    if (op->cg1) {  // the single-reduction kernel, iteration 2
+        cg1_args(op, 2, a);
+        ST(replay_time(op->cap_stream, s, reps, a_ms, flush, flush_bytes, op->st, st_init,
+                       [&](cudaStream_t cs) { return launch_stencil(MODE_CG1, nc, a, cs); }));
+        return MAS_OK;
+    }
+    a.u = halo_of(op, op->r, nullptr, nc);
+    a.pold = halo_of(op, op->p[1], nullptr, nc);
+    a.pnew = op->p[0];
+    a.out = op->q;
+    set_lpar_args(op, a);
+    ST(replay_time(op->cap_stream, s, reps, a_ms, flush, flush_bytes, op->st, st_init,
+                   [&](cudaStream_t cs) { return launch_stencil(MODE_PCGA, nc, a, cs); }));
+    if (op->aniso && !lpar_in_a(op)) {
+        AnisoArgs an = aniso_args(op, MODE_PCGA, Halo{op->p[0], nullptr, nullptr, 0, 0}, op->q);
+        ST(replay_time(op->cap_stream, s, reps, c_ms, flush, flush_bytes, op->st, st_init,
+                       [&](cudaStream_t cs) { return launch_aniso(MODE_PCGA, an, cs); }));
+    }
+    StreamArgs b{};
+    b.g = op->geo;
+    b.ncomp = nc;
+    b.r = op->r;
+    b.q = op->q;
+    b.dinv = op->dinv;
+    b.st = op->st;
+    b.rho_hist = a.rho_hist;
+    b.sigma_hist = a.sigma_hist;
+    b.rr_hist = a.rr_hist;
+    b.scr = op->scr;
+    ST(replay_time(op->cap_stream, s, reps, b_ms, flush, flush_bytes, op->st, st_init,
+                   [&](cudaStream_t cs) { return launch_pcg_b(b, op->b_blocks, cs); }));
+    return MAS_OK;
+}
+
 mas_status_t mas_op_set_curvature(mas_op_t* op, int on) {
     if (!op) return arg_error("null op");
     if (on && op->ncomp != 3) return arg_error("curvature terms: the 3-component (viscosity) operator only");
@@ -1613,7 +1793,7 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
     b.scr = op->scr;
     b.host_flag = op->host_flag_dev;
     b.p2p = p2p_args(op);
-    b.aniso = op->aniso;
+    b.aniso = op->aniso && !lpar_in_a(op);  // P2P: sigma's L_par part in its own slot (MB_C)
 
     // a4: iterations.  Kernel A(k) reads k, alpha, beta and the convergence
     // decision from PcgState; the host only keeps two iterations in flight
@@ -1624,6 +1804,7 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
     a.out = op->q;
     a.x = xd;
     a.f = nullptr;
+    set_lpar_args(op, a);  // the field-aligned term inside kernel A (fused)
     // no host involvement per iteration on one GPU and with the P2P transport
     // (virtual P2P ranks share one GPU and need host ordering: comm_vsync)
     const bool graph = !op->prof && op->use_graph && (!comm || (p2p && !comm_is_virtual(comm)));
@@ -1635,7 +1816,7 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
             a.tpold = pold_trows(op, 1);
             a.pnew = op->p[1];
             CU(launch_stencil(MODE_PCGA, nc, a, s, true));
-            if (op->aniso) {
+            if (op->aniso && !lpar_in_a(op)) {
                 an.u = aniso_p_halo(op, 1);
                 CU(launch_aniso(MODE_PCGA, an, s));
             }
@@ -1704,7 +1885,7 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
             op->launches++;
         }
         if (pe) CU(cudaEventRecord(pe[1], s));
-        if (op->aniso) {  // q += L_par p_k, sigma += <p_k, L_par p_k> (rank-local)
+        if (op->aniso && !lpar_in_a(op)) {  // q += L_par p_k, sigma += <p_k, L_par p_k> (rank-local)
             if (comm && !p2p)  // the p_k planes of the r-neighbours (kernel A(k) just wrote them)
                 ST(comm_seams(comm, pnew, 1, op->g->nl, plane, op->pkg, op->pkg + plane, s,
                               rstride(op)));
@@ -1758,7 +1939,7 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
     if (graph) {  // iteration 1 + 4 kernels per executed loop body (iterations 2k, 2k+1)
         const int last_a = fin.status == MAS_ERR_BREAKDOWN ? fin.iters : fin.iters + 1;
         const int bodies = last_a <= 2 ? 1 : last_a / 2;
-        const int per = 2 + (op->aniso ? 1 : 0) + (op->tnode ? 1 : 0);  // kernels per iteration
+        const int per = 2 + (op->aniso && !lpar_in_a(op) ? 1 : 0) + (op->tnode ? 1 : 0);  // kernels per iteration
         op->launches += per + 2LL * per * bodies;
     }
     if (res_hist) {
@@ -1776,7 +1957,7 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
             const cudaEvent_t* e = &op->pev[6 * (size_t)(k - 1)];
             CU(cudaEventElapsedTime(&ta, e[0], e[1]));
             CU(cudaEventElapsedTime(&tb, e[2], e[3]));
-            if (op->aniso) CU(cudaEventElapsedTime(&tc, e[4], e[5]));
+            if (op->aniso && !lpar_in_a(op)) CU(cudaEventElapsedTime(&tc, e[4], e[5]));
             sa += ta;
             sb += tb;
             sc += tc;

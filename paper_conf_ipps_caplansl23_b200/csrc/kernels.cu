@@ -215,7 +215,7 @@ struct HaloMeta {
 // hkind 4 / 5: the row beyond the local theta range belongs to the theta
 // neighbour (2-D decomposition): hoff is then the phi index in that row.
 __device__ __forceinline__ HaloMeta halo_meta(const Geo& g, int j0, int k0, int height, int width,
-                                              bool tnb_lo, bool tnb_hi) {
+                                              bool tnb_lo, bool tnb_hi, bool diag = false) {
     const int t = threadIdx.x;
     HaloMeta m{0, 0, 0};
     if (t < 2 * TK) {
@@ -236,6 +236,15 @@ __device__ __forceinline__ HaloMeta halo_meta(const Geo& g, int j0, int k0, int 
             m.hkind = 1;
             m.hoff = (int)(j0 + r) * g.np + k;
         }
+    } else if (diag && t < 2 * TK + 2 * TJ + 4) {
+        // the 4 diagonal halo cells (j0-1 | j0+height, k0-1 | k0+width): the
+        // corner gradients of the fused field-aligned term need them
+        const int q = t - 2 * TK - 2 * TJ, bottom = q >> 1, right = q & 1;
+        const int hr = bottom ? height + 1 : 0, j = j0 + hr - 1;
+        const int k = right ? (k0 + width) % g.np : (k0 - 1 + g.np) % g.np;
+        m.hidx = hr * ROW + (right ? OFF + width : OFF - 1);
+        m.hkind = (j >= 0 && j < g.nt) ? 1 : 3;
+        m.hoff = (int)j * g.np + k;
     }
     return m;
 }
@@ -256,7 +265,7 @@ struct Stage {
 // thread copies its item into a private shared-memory slot instead:
 // layout [field][kHaloSlots], fields 0 kappa, 1 1/D, 2.. u[NC], po[NC]
 // (+ w[NC] in MODE_CG1).
-constexpr int kHaloSlots = 2 * TK + 2 * TJ;
+constexpr int kHaloSlots = 2 * TK + 2 * TJ + 4;  // + the 4 diagonal halo cells (fused L_par)
 __device__ __forceinline__ void cpa8(double* sdst, const double* gsrc) {
     const unsigned sa = (unsigned)__cvta_generic_to_shared(sdst);
     asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"(sa), "l"(gsrc) : "memory");
@@ -409,6 +418,19 @@ __device__ __forceinline__ void stage_issue(const StencilArgs& a, int i, int j0,
                     }
                 }
             }
+        } else if (MODE == MODE_PCGA) {
+            // an r-ghost plane's halo (the fused field-aligned term's corners
+            // read it): the ghost copy, or the neighbour's own array in place
+            const PlanePtrs<NC> P = plane_ptrs<MODE, NC>(a, i, first);
+            const int hi = (int)hm.hoff;
+            cpa8(h, P.kap + hi);
+#pragma unroll
+            for (int c = 0; c < NC; c++) cpa8(h + (2 + c) * kHaloSlots, P.u[c] + hi);
+            cpa8(h + kHaloSlots, P.di + hi);
+            if (!first) {
+#pragma unroll
+                for (int c = 0; c < NC; c++) cpa8(h + (2 + NC + c) * kHaloSlots, P.po[c] + hi);
+            }
         }
     }
     cpa_commit();
@@ -521,7 +543,10 @@ __device__ __forceinline__ void stage_commit(const StencilArgs& a, int i, int j0
 // u = 0 (homogeneous Dirichlet; irrelevant under Neumann, weight 0) and
 // kappa_ghost = kappa_P so that the face kappa is kappa_P (reading R3).
 template <int NC>
-__device__ __forceinline__ void ghost_plane(double* buf, int height, int width, double2 kP) {
+__device__ __forceinline__ void ghost_plane(double* buf, int height, int width, double2 kP, bool all = false) {
+    if (all) {  // the fused L_par corners read the halo of this plane too: zeros
+        for (int t = threadIdx.x; t < HROWS * ROW; t += kSThreads) sfield(buf, 0)[t] = 0.0;
+    }
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     const int kc = 2 * lane;
     if (w < height && kc < width) {
@@ -561,6 +586,80 @@ __device__ __forceinline__ void a_globals(const StencilArgs& a, int kit, double&
 }
 
 // --------------------------------------------------------------------------
+// field-aligned term fused into kernel A (NEXT-4; readings R21-R26; DESIGN.md
+// §5.3): the corner coefficients (a, b, e) of one corner plane are staged per
+// plane, the corners of the tile computed once into the 4 sign combinations
+// c[st,sp] = s a + st s b + sp s e (s = a Dr + b Dt + e Dp), and every cell
+// gathers its 8 corners: V (L_par p)_P = sum_lower c[st,sp] - sum_upper
+// c[-st,-sp].  Same arithmetic as k_aniso (aniso.cu), one kernel less: p_k
+// and q never leave the SM for it (24 of its 48 bytes per cell).
+// --------------------------------------------------------------------------
+constexpr int LCR = TJ + 1;    // corner rows of a tile (J = j0 .. j0+TJ)
+constexpr int LCW = TK + 2;    // corner columns staged (K = k0 .. k0+65; 64 + 1 used)
+constexpr int LCA = LCR * LCW; // one corner array
+constexpr int kLparSmem = (2 * 3 + 4) * LCA;  // 2 staging buffers of (a, b, e) + 4 combinations
+
+// cp.async of corner plane c's coefficients (rows J = j0 .. j0+height,
+// columns K = k0 .. k0+width, K = np wrapping to 0) into buf [3][LCR][LCW];
+// rows beyond nt-1 and a plane beyond the slab without a ghost copy are zeros
+__device__ __forceinline__ void lpar_coef_issue(const StencilArgs& a, int c, int j0, int k0, int height,
+                                                int width, double* buf) {
+    const Geo& g = a.g;
+    const long long N = (long long)g.nl * g.plane;
+    const int pairs = width / 2 + 1;                  // pair m2 < width/2, then the single column width
+    const int items = 3 * (height + 1) * pairs;
+    for (int t = threadIdx.x; t < items; t += kSThreads) {
+        const int f = t / ((height + 1) * pairs), rem = t - f * (height + 1) * pairs;
+        const int q = rem / pairs, m2 = rem - q * pairs;
+        const int J = j0 + q;
+        double* dst = buf + f * LCA + q * LCW + 2 * m2;
+        const double* src = nullptr;
+        if (J < g.nt) {
+            if (c < g.nl) src = a.ca + f * N + (long long)c * g.plane + (long long)J * g.np;
+            else if (a.ca_hi) src = a.ca_hi + f * g.plane + (long long)J * g.np;
+        }
+        if (m2 < width / 2) {
+            if (src) {
+                const unsigned sa = (unsigned)__cvta_generic_to_shared(dst);
+                asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(sa), "l"(src + k0 + 2 * m2)
+                             : "memory");
+            } else {
+                dst[0] = 0.0, dst[1] = 0.0;
+            }
+        } else {  // column width: K = k0 + width (np -> 0)
+            const int K = (k0 + width) % g.np;
+            if (src) cpa8(dst, src + K);
+            else dst[0] = 0.0;
+        }
+    }
+    cpa_commit();
+}
+
+// corners of corner plane c (cells c-1 | c in ring slots lo | hi) into the 4
+// combination arrays cmb [4][LCR][LCW]
+__device__ __forceinline__ void lpar_corners(const double* lo, const double* hi, const double* cf, double* cmb,
+                                             int height, int width) {
+    const int cols = width + 1, n = (height + 1) * cols;
+    for (int t = threadIdx.x; t < n; t += kSThreads) {
+        const int q = t / cols, m = t - q * cols;
+        const int r0 = q * ROW + OFF + m - 1, r1 = r0 + ROW;  // cell rows J-1 | J, columns K-1 | K
+        const double a00 = lo[r0], a01 = lo[r0 + 1], a10 = lo[r1], a11 = lo[r1 + 1];
+        const double b00 = hi[r0], b01 = hi[r0 + 1], b10 = hi[r1], b11 = hi[r1 + 1];
+        const double Dr = ((b00 - a00) + (b01 - a01)) + ((b10 - a10) + (b11 - a11));
+        const double Dt = ((a10 - a00) + (a11 - a01)) + ((b10 - b00) + (b11 - b01));
+        const double Dp = ((a01 - a00) + (a11 - a10)) + ((b01 - b00) + (b11 - b10));
+        const int ci = q * LCW + m;
+        const double A0 = cf[ci], B0 = cf[LCA + ci], E0 = cf[2 * LCA + ci];
+        const double sc = A0 * Dr + B0 * Dt + E0 * Dp;
+        const double A = sc * A0, B = sc * B0, E = sc * E0;
+        cmb[ci] = (A + B) + E;            // st +, sp +
+        cmb[LCA + ci] = (A + B) - E;      // st +, sp -
+        cmb[2 * LCA + ci] = (A - B) + E;  // st -, sp +
+        cmb[3 * LCA + ci] = (A - B) - E;  // st -, sp -
+    }
+}
+
+// --------------------------------------------------------------------------
 // the fused stencil kernel
 // --------------------------------------------------------------------------
 // One block = one (TJ x TK) theta-phi tile x one chunk of r-planes.  It
@@ -572,10 +671,13 @@ __device__ __forceinline__ void a_globals(const StencilArgs& a, int kit, double&
 // FIRSTK: kernel A of iteration 1 (p = D^-1 r, no x update) is its own
 // instantiation, so the per-plane code of every other iteration carries no
 // first-iteration branches.
-template <int MODE, int NC, bool FIRSTK = false>
+// LPAR: the field-aligned term fused in (MODE_PCGA, NC = 1): q = L_iso p +
+// L_par p and <p, q> of both in one pass.
+template <int MODE, int NC, bool FIRSTK = false, bool LPAR = false>
 __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_stencil(const StencilArgs a) {
     extern __shared__ __align__(16) double smem[];
     constexpr int BUF = (NC + 1) * HROWS * ROW;
+    static_assert(!LPAR || (MODE == MODE_PCGA && NC == 1), "fused L_par: scalar kernel A only");
     const Geo& g = a.g;
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
 
@@ -779,30 +881,63 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
     double2 kown = make_double2(0.0, 0.0), kdummy;
     const bool lo_ghost = (ia == 0) && g.glob_lo;
     const HaloMeta hm = halo_meta(g, j0, k0, height, width, a.tkappa.lo != nullptr,
-                                  a.tkappa.hi != nullptr);
+                                  a.tkappa.hi != nullptr, LPAR);
+    // fused L_par: coefficient staging [2][3][LCR][LCW], combinations [4][LCR][LCW]
+    double* const lcf = smem + 4 * BUF;
+    double* const lcmb = lcf + 2 * 3 * LCA;
+    double lpart0 = 0.0, lpart1 = 0.0;  // the lower-corner (corner plane i) part of this pair's L_par p
+    double lcw0 = 0.0, lcw1 = 0.0;      // 1 / (vt_j vp_k) of the pair
+    if (LPAR && own) {
+        const double vt = __ldg(g.vt + j);
+        lcw0 = 1.0 / (vt * __ldg(g.vp + k));
+        lcw1 = 1.0 / (vt * __ldg(g.vp + k + 1));
+    }
     // planes ia-1 (own cells only) and ia: both loads in flight together
     Stage<NC> S0, S;
-    if (!lo_ghost)
-        stage_issue<MODE, NC>(a, ia - 1, j0, k0, height, width, hm, FIRSTK, false, false, false, S0, hst_arr);
+    // (fused L_par: plane ia-1's halo is a corner input too, so it is loaded
+    // in the prologue; the halo item copies of ia-1 and ia go one after the
+    // other through the same private slots)
+    if (!lo_ghost) {
+        stage_issue<MODE, NC>(a, ia - 1, j0, k0, height, width, hm, FIRSTK, false, LPAR, false, S0, hst_arr);
+        if (LPAR)
+            stage_commit<MODE, NC>(a, ia - 1, j0, k0, height, width, hm, FIRSTK, beta, alpha_prev, false,
+                                   true, false, S0, slot(ia - 1), kdummy, on, hst_arr, acc);
+    }
     stage_issue<MODE, NC>(a, ia, j0, k0, height, width, hm, FIRSTK, xupd, true, true, S, hst_arr);
-    if (!lo_ghost)
+    if (!lo_ghost && !LPAR)
         stage_commit<MODE, NC>(a, ia - 1, j0, k0, height, width, hm, FIRSTK, beta, alpha_prev, false,
                                false, false, S0, slot(ia - 1), kdummy, on, hst_arr, acc);
     stage_commit<MODE, NC>(a, ia, j0, k0, height, width, hm, FIRSTK, beta, alpha_prev, xupd, true, true,
                            S, slot(ia), kown, oc, hst_arr, acc);
-    if (lo_ghost) ghost_plane<NC>(slot(ia - 1), height, width, kown);
+    if (lo_ghost) ghost_plane<NC>(slot(ia - 1), height, width, kown, LPAR);
+    if (LPAR) {  // corner plane ia (cells ia-1 | ia): its lower-corner part for plane ia
+        lpar_coef_issue(a, ia, j0, k0, height, width, lcf + (ia & 1) * 3 * LCA);
+        cpa_wait_all();
+        __syncthreads();
+        lpar_corners(sfield(slot(ia - 1), 0), sfield(slot(ia), 0), lcf + (ia & 1) * 3 * LCA, lcmb, height,
+                     width);
+        __syncthreads();
+        if (own) {
+            const double* h = lcmb + w * LCW + kc;
+            const double2 l0 = lds2(h), l2 = lds2(h + 2 * LCA + LCW);
+            lpart0 = (l0.x + h[LCA + 1]) + (l2.x + h[3 * LCA + LCW + 1]);
+            lpart1 = (l0.y + h[LCA + 2]) + (l2.y + h[3 * LCA + LCW + 2]);
+        }
+    }
     if (real_plane(ia + 1))
         stage_issue<MODE, NC>(a, ia + 1, j0, k0, height, width, hm, FIRSTK, xupd && (ia + 1 < ib),
-                              ia + 1 < ib, ia + 1 < ib, S, hst_arr);
+                              LPAR || ia + 1 < ib, ia + 1 < ib, S, hst_arr);
+    if (LPAR) lpar_coef_issue(a, ia + 1, j0, k0, height, width, lcf + ((ia + 1) & 1) * 3 * LCA);
 
     for (int i = ia; i < ib; i++) {
         // commit plane i+1 (its loads were issued one plane earlier)
         if (real_plane(i + 1))
             stage_commit<MODE, NC>(a, i + 1, j0, k0, height, width, hm, FIRSTK, beta, alpha_prev,
-                                   xupd && (i + 1 < ib), i + 1 < ib, i + 1 < ib, S, slot(i + 1),
+                                   xupd && (i + 1 < ib), LPAR || i + 1 < ib, i + 1 < ib, S, slot(i + 1),
                                    kown, on, hst_arr, acc);
         else
-            ghost_plane<NC>(slot(i + 1), height, width, kown);
+            ghost_plane<NC>(slot(i + 1), height, width, kown, LPAR);
+        if (LPAR) cpa_wait_all();  // the coefficient copies of corner plane i+1 (every thread)
         // issue plane i+2 (registers and private cp.async slots only): its
         // latency overlaps the stencil of plane i.  Issuing it before the
         // barrier measured faster for the scalar kernel and slower for the
@@ -810,8 +945,14 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
         constexpr bool kIssueEarly = (NC == 1);
         if (kIssueEarly && i + 2 <= ib && real_plane(i + 2))
             stage_issue<MODE, NC>(a, i + 2, j0, k0, height, width, hm, FIRSTK, xupd && (i + 2 < ib),
-                                  i + 2 < ib, i + 2 < ib, S, hst_arr);
+                                  LPAR || i + 2 < ib, i + 2 < ib, S, hst_arr);
+        if (LPAR && i + 2 <= ib) lpar_coef_issue(a, i + 2, j0, k0, height, width, lcf + ((i + 2) & 1) * 3 * LCA);
         __syncthreads();
+        if (LPAR) {  // corner plane i+1 (cells i | i+1) into the combinations
+            lpar_corners(sfield(slot(i), 0), sfield(slot(i + 1), 0), lcf + ((i + 1) & 1) * 3 * LCA, lcmb,
+                         height, width);
+            __syncthreads();
+        }
 #ifndef MAS_NO_PREFETCH
         // 3-component kernels only: for the scalar kernel (C2: 256 work items,
         // under one wave) it measured slower (tools/abtest.sh)
@@ -893,6 +1034,20 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
                     acc[1] += V0 * r0 * r0 + V1 * r1 * r1;
                     acc[2] += V0 * r0 * (oc.di.x * r0) + V1 * r1 * (oc.di.y * r1);
                 } else {
+                    if constexpr (LPAR) {
+                        // upper corners (corner plane i+1) from the combinations, lower
+                        // ones (plane i) gathered one step earlier; then plane i+1's lower part
+                        const double* h = lcmb + w * LCW + kc;
+                        const double2 h3 = lds2(h + 3 * LCA), h1 = lds2(h + LCA + LCW);
+                        const double up0 = (h3.x + h[2 * LCA + 1]) + (h1.x + h[LCW + 1]);
+                        const double up1 = (h3.y + h[2 * LCA + 2]) + (h1.y + h[LCW + 2]);
+                        const double iv = __ldg(a.ivr + i);
+                        L0 += (lpart0 - up0) * (iv * lcw0);
+                        L1 += (lpart1 - up1) * (iv * lcw1);
+                        const double2 l0 = lds2(h), l2 = lds2(h + 2 * LCA + LCW);
+                        lpart0 = (l0.x + h[LCA + 1]) + (l2.x + h[3 * LCA + LCW + 1]);
+                        lpart1 = (l0.y + h[LCA + 2]) + (l2.y + h[3 * LCA + LCW + 2]);
+                    }
                     stg2a(a.out + o, make_double2(L0, L1));
                     if (MODE == MODE_PCGA) acc[0] += V0 * u.x * L0 + V1 * u.y * L1;
                     // CG1: delta = <w,u> (+ gamma = <r,u>, <r,r> unless accumulated at commit)
@@ -1293,6 +1448,37 @@ __global__ void __launch_bounds__(kThreads) k_init_dots(const Geo g, int ncomp, 
     }
 }
 
+// a[i] = 1 + 0.25 * h(i) / 1024 with h a multiplicative hash: finite,
+// positive, non-constant values (kernel-replay timing inputs; mas_op_kernel_bench)
+__global__ void k_fill_test(double* a, long long n) {
+    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n;
+         i += (long long)gridDim.x * blockDim.x)
+        a[i] = 1.0 + 0.25 * (double)(((unsigned long long)i * 2654435761ull) % 1024ull) / 1024.0;
+}
+
+// read-only sweep over a buffer larger than L2: evicts the working set and
+// leaves only clean lines behind (a memset flush would leave dirty lines whose
+// write-back the timed kernel would pay); kernel-replay timing
+__global__ void k_l2_sweep(const double* a, long long n, double* sink) {
+    double acc = 0.0;
+    for (long long i = 2 * (blockIdx.x * (long long)blockDim.x + threadIdx.x); i + 1 < n;
+         i += 2LL * gridDim.x * blockDim.x) {
+        const double2 v = __ldcg(reinterpret_cast<const double2*>(a + i));  // L2-allocating (not evict-first)
+        acc += v.x + v.y;
+    }
+    if (acc == -1.0) *sink = acc;  // keeps the loads; never true for the 0 / 1 fill
+}
+
+cudaError_t launch_l2_sweep(const double* a, long long n, double* sink, cudaStream_t s) {
+    k_l2_sweep<<<148 * 8, 256, 0, s>>>(a, n, sink);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_fill_test(double* a, long long n, cudaStream_t s) {
+    k_fill_test<<<148 * 8, 256, 0, s>>>(a, n);
+    return cudaGetLastError();
+}
+
 // --------------------------------------------------------------------------
 // launchers
 // --------------------------------------------------------------------------
@@ -1322,23 +1508,23 @@ int stencil_blocks(const Geo& g, int chunk) {
     return ntj * ntk * nch;
 }
 
-template <int MODE, int NC, bool FIRSTK = false>
+template <int MODE, int NC, bool FIRSTK = false, bool LPAR = false>
 static cudaError_t launch_one(const StencilArgs& a0, cudaStream_t s) {
     StencilArgs a = a0;
     a.ntj = (a.g.nt + TJ - 1) / TJ;
     a.ntk = (a.g.np + TK - 1) / TK;
     a.nchunk = (a.g.nl + a.chunk - 1) / a.chunk;
-    const int smem = 4 * (NC + 1) * HROWS * ROW * (int)sizeof(double);
+    const int smem = (4 * (NC + 1) * HROWS * ROW + (LPAR ? kLparSmem : 0)) * (int)sizeof(double);
     static DeviceOnce attr;
     cudaError_t e = attr.run([&] {
-        return cudaFuncSetAttribute(k_stencil<MODE, NC, FIRSTK>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+        return cudaFuncSetAttribute(k_stencil<MODE, NC, FIRSTK, LPAR>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                     smem);
     });
     if (e != cudaSuccess) return e;
     const int T = a.ntj * a.ntk;
     const int blocks = a.part == 1 ? T * (a.nchunk - 2) : a.part == 2 ? 2 * T : T * a.nchunk;
     if (blocks <= 0) return cudaErrorInvalidValue;
-    k_stencil<MODE, NC, FIRSTK><<<blocks, kSThreads, smem, s>>>(a);
+    k_stencil<MODE, NC, FIRSTK, LPAR><<<blocks, kSThreads, smem, s>>>(a);
     return cudaGetLastError();
 }
 
@@ -1347,6 +1533,8 @@ cudaError_t launch_stencil(int mode, int ncomp, const StencilArgs& a, cudaStream
         if (mode == MODE_APPLY) return launch_one<MODE_APPLY, 1>(a, s);
         if (mode == MODE_RESID) return launch_one<MODE_RESID, 1>(a, s);
         if (mode == MODE_CG1) return first ? launch_one<MODE_CG1, 1, true>(a, s) : launch_one<MODE_CG1, 1>(a, s);
+        if (a.ca)  // the field-aligned term fused into kernel A
+            return first ? launch_one<MODE_PCGA, 1, true, true>(a, s) : launch_one<MODE_PCGA, 1, false, true>(a, s);
         return first ? launch_one<MODE_PCGA, 1, true>(a, s) : launch_one<MODE_PCGA, 1>(a, s);
     }
     if (ncomp == 3) {

@@ -146,6 +146,10 @@ struct StencilArgs {
     P2P p2p;                  // RESID / PCGA: mailbox transport (nranks == 0: off)
     int nopub;                // RESID under P2P with the field-aligned term: k_aniso publishes
     int curv;                 // NC = 3: + kappa_P (2/r^2, 1/(r sin)^2, 1/(r sin)^2) u_m (NEXT-2, R31)
+    // PCGA, scalar: the field-aligned term fused into kernel A when ca != nullptr
+    const double* ca;         // corner coefficients [3][nl][nt][np] (a, b, e)
+    const double* ca_hi;      // r-slabs: corner plane nl (rank+1's plane 0) [3][plane], or nullptr
+    const double* ivr;        // [nl] 1 / (rC^2 dr)
 };
 
 struct StreamArgs {  // kernel B
@@ -213,6 +217,9 @@ cudaError_t launch_pcg_b(const StreamArgs& a, int nblocks, cudaStream_t s);
 // dp weights (dinv != nullptr: also dinv = 1 / average, ncomp = 1)
 cudaError_t launch_pole_avg(const Geo& g, int ncomp, double* y, double* dinv, int plane_lo, int nplanes,
                             cudaStream_t s);
+// finite, positive, non-constant test values (kernel-replay timing)
+cudaError_t launch_fill_test(double* a, long long n, cudaStream_t s);
+cudaError_t launch_l2_sweep(const double* a, long long n, double* sink, cudaStream_t s);
 // the init's <f,f>, <r,r>, <r,D^-1 r> into PcgState (after the pole average of r)
 cudaError_t launch_init_dots(const Geo& g, int ncomp, const double* f, const double* r, const double* dinv,
                              Scratch scr, PcgState* st, int nblocks, cudaStream_t s);

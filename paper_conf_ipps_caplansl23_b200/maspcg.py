@@ -29,7 +29,7 @@ ABI_SYMBOLS = ("mas_comm_unique_id", "mas_partition", "mas_grid_create", "mas_gr
                "mas_op_transport", "mas_op_launch_count", "mas_grid_create_2d",
                "mas_grid_local_extent_2d",
                "mas_op_set_profiling", "mas_op_kernel_times", "mas_op_set_aniso",
-               "mas_op_aniso_time", "mas_op_radial_sums", "mas_op_comm_bench", "mas_op_set_single_reduction", "mas_op_set_curvature",
+               "mas_op_aniso_time", "mas_op_radial_sums", "mas_op_comm_bench", "mas_op_set_single_reduction", "mas_op_set_curvature", "mas_op_kernel_bench", "mas_op_aniso_fused",
                "mas_op_single_reduction", "mas_op_destroy", "mas_status_string", "mas_last_error", "mas_version")
 
 
@@ -83,6 +83,8 @@ def lib() -> C.CDLL:
             "mas_op_comm_bench": (_i, [_vp, _i, _vp, _vp, _vp, _vp]),
             "mas_op_set_single_reduction": (_i, [_vp, _i]),
             "mas_op_set_curvature": (_i, [_vp, _i]),
+            "mas_op_kernel_bench": (_i, [_vp, _i, _vp, _vp, _vp, _vp]),
+            "mas_op_aniso_fused": (_i, [_vp]),
             "mas_op_single_reduction": (_i, [_vp]),
             "mas_op_destroy": (_i, [_vp]),
             "mas_status_string": (C.c_char_p, [_i]),
@@ -341,6 +343,15 @@ def mas_op_set_curvature(op: int, on: bool = True) -> None:
     _check(lib().mas_op_set_curvature(op, int(bool(on))), "mas_op_set_curvature")
 
 
+def mas_op_kernel_bench(op: int, reps: int = 20, stream=None):
+    """(kernel A or single-reduction kernel, kernel B, L_par) device ms per
+    launch from back-to-back graph replays (clobbers the op's work vectors)."""
+    a, b, c = C.c_double(), C.c_double(), C.c_double()
+    _check(lib().mas_op_kernel_bench(op, int(reps), C.byref(a), C.byref(b), C.byref(c), _stream(stream)),
+           "mas_op_kernel_bench")
+    return a.value, b.value, c.value
+
+
 def mas_op_single_reduction(op: int) -> bool:
     return int(lib().mas_op_single_reduction(op)) == 1
 
@@ -459,8 +470,16 @@ class Operator:
     def single_reduction(self):
         return mas_op_single_reduction(self.h)
 
+    def kernel_bench(self, reps=20, stream=None):
+        return mas_op_kernel_bench(self.h, reps, stream)
+
     def comm_bench(self, reps=20, stream=None):
         return mas_op_comm_bench(self.h, reps, stream)
+
+    @property
+    def aniso_fused(self):
+        """True if the iteration's L_par runs inside kernel A (mas_op_aniso_fused)."""
+        return int(lib().mas_op_aniso_fused(self.h)) == 1
 
     def aniso_time(self):
         return mas_op_aniso_time(self.h)

@@ -248,3 +248,25 @@ def test_aniso_on_the_p2p_mailbox_loop_one_gpu(mp, oracle_mod):
         st, it, rel, _ = op.solve(f, x, 1e-12, 5000)
         assert st == mp.MAS_OK and it == a[1]
         assert np.array_equal(host(x), a[2])
+
+
+@pytest.mark.parametrize("shape", [(16, 24, 64), (24, 20, 70)])
+def test_fused_lpar_kernel_matches_oracle(mp, oracle_mod, shape, monkeypatch):
+    """The opt-in fused form (MAS_LPAR_FUSED=1: the iteration's L_par inside
+    kernel A, corners staged per plane with the diagonal halo cells): PCG
+    against the oracle (+-1, x <= 1e-10), graph == host loop bitwise, and the
+    fixed-iteration iterates (k = 7) within 1e-10."""
+    monkeypatch.setenv("MAS_LPAR_FUSED", "1")
+    prob = W.aniso_conduction_problem(*shape)
+    a = _solve_pair(mp, oracle_mod, prob, 1e-12, 5000, prof=False)
+    assert a[8].aniso_fused
+    b = _solve_pair(mp, oracle_mod, prob, 1e-12, 5000, prof=True)
+    assert a[1] == b[1]
+    assert np.array_equal(a[2], b[2])
+    rc, xo, ito, _, _ = oracle_mod.solve_problem(prob)
+    V = oracle_mod.Oracle.for_problem(prob).volumes()
+    assert abs(a[1] - ito) <= 1
+    assert rel_l2_V(V, a[2], xo) <= 1e-10
+    rc, xo7, ito7, _, _ = oracle_mod.solve_problem(prob, tol=0.0, maxit=7)
+    c = _solve_pair(mp, oracle_mod, prob, 0.0, 7, prof=False)
+    assert c[1] == 7 and rel_l2_V(V, c[2], xo7) <= 1e-10
