@@ -329,6 +329,87 @@ class Oracle:
         return rc, x, iters.value, relres.value, hist[: iters.value + 1]
 
 
+    # ---- face-centred placements (NEXT-2, R32-R33) ----------------------
+    @property
+    def rn_shape(self):
+        nr, nt, np_ = self.shape
+        return (nr - 1, nt, np_)
+
+    def rn_volumes(self):
+        V = np.empty(self.rn_shape)
+        self._chk(lib().mas_ref_rn_volumes(C.byref(self.g), _p(V)))
+        return V
+
+    def rn_apply(self, kappa, c, x):
+        x = _f64(x)
+        y = np.empty_like(x)
+        kappa, c = _f64(kappa), _f64(c)
+        self._chk(lib().mas_ref_rn_apply(C.byref(self.g), x.size // int(np.prod(self.rn_shape)), _p(kappa),
+                                         _p(c), _p(x), _p(y)))
+        return y
+
+    def rn_diag(self, kappa, c):
+        D = np.empty(self.rn_shape)
+        kappa, c = _f64(kappa), _f64(c)
+        self._chk(lib().mas_ref_rn_diag(C.byref(self.g), _p(kappa), _p(c), _p(D)))
+        return D
+
+    def rn_dirichlet_rhs(self, kappa, f, ub_inner=None, ub_outer=None):
+        f = _f64(f).copy()
+        kappa, ub_inner, ub_outer = _f64(kappa), _f64(ub_inner), _f64(ub_outer)
+        self._chk(lib().mas_ref_rn_dirichlet_rhs(C.byref(self.g), f.size // int(np.prod(self.rn_shape)),
+                                                 _p(kappa), _p(ub_inner), _p(ub_outer), _p(f)))
+        return f
+
+    def rn_pcg(self, kappa, c, f, x0, tol, maxit):
+        f = _f64(f)
+        x = _f64(x0).copy()
+        kappa, c = _f64(kappa), _f64(c)
+        iters, relres = C.c_int(), C.c_double()
+        hist = np.zeros(maxit + 1)
+        rc = lib().mas_ref_rn_pcg_solve(C.byref(self.g), f.size // int(np.prod(self.rn_shape)), _p(kappa),
+                                        _p(c), _p(f), _p(x), C.c_double(tol), maxit, C.byref(iters),
+                                        C.byref(relres), _p(hist))
+        self._chk(rc)
+        return rc, x, iters.value, relres.value, hist[: iters.value + 1]
+
+    def pn_volumes(self):
+        V = np.empty(self.shape)
+        self._chk(lib().mas_ref_pn_volumes(C.byref(self.g), _p(V)))
+        return V
+
+    def pn_apply(self, kappa, c, x):
+        x = _f64(x)
+        y = np.empty_like(x)
+        kappa, c = _f64(kappa), _f64(c)
+        self._chk(lib().mas_ref_pn_apply(C.byref(self.g), x.size // self.N, _p(kappa), _p(c), _p(x), _p(y)))
+        return y
+
+    def pn_diag(self, kappa, c):
+        D = np.empty(self.shape)
+        kappa, c = _f64(kappa), _f64(c)
+        self._chk(lib().mas_ref_pn_diag(C.byref(self.g), _p(kappa), _p(c), _p(D)))
+        return D
+
+    def pn_dirichlet_rhs(self, kappa, f, ub_inner=None, ub_outer=None):
+        f = _f64(f).copy()
+        kappa, ub_inner, ub_outer = _f64(kappa), _f64(ub_inner), _f64(ub_outer)
+        self._chk(lib().mas_ref_pn_dirichlet_rhs(C.byref(self.g), f.size // self.N, _p(kappa), _p(ub_inner),
+                                                 _p(ub_outer), _p(f)))
+        return f
+
+    def pn_pcg(self, kappa, c, f, x0, tol, maxit):
+        f = _f64(f)
+        x = _f64(x0).copy()
+        kappa, c = _f64(kappa), _f64(c)
+        iters, relres = C.c_int(), C.c_double()
+        hist = np.zeros(maxit + 1)
+        rc = lib().mas_ref_pn_pcg_solve(C.byref(self.g), f.size // self.N, _p(kappa), _p(c), _p(f), _p(x),
+                                        C.c_double(tol), maxit, C.byref(iters), C.byref(relres), _p(hist))
+        self._chk(rc)
+        return rc, x, iters.value, relres.value, hist[: iters.value + 1]
+
+
 def partition(nr: int, nranks: int, rank: int):
     i0, nl = C.c_int(), C.c_int()
     lib().mas_ref_partition(nr, nranks, rank, C.byref(i0), C.byref(nl))

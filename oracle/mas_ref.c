@@ -1470,3 +1470,284 @@ int mas_ref_pcg_solve_curv(const mas_ref_grid* g, const double* kappa, const dou
                            double* relres, double* res_hist) {
     return pcg_core(g, 3, kappa, c, NULL, NULL, 1, f, x, tol, maxit, iters, relres, res_hist);
 }
+
+/* ---------------------------------------------------------------------------
+ * Face-centred placements of the staggered mesh (readings
+ * R32-R33): MAS stores a velocity component on the faces
+ * normal to it ("staggered"): v_r at the r faces, v_phi at the phi
+ * faces (v_theta at the theta faces is the theta-node placement above).  As a
+ * scalar unknown of the same operator L = c + (1/V) div(kappa grad):
+ *
+ * phi nodes (R33): unknowns at (rC_i, tC_j, pF_k), k = 0..np-1 (pF_np = pF_0 +
+ *   2 pi).  The control volume of node k is the dual phi cell [pC_{k-1}, pC_k]
+ *   (pC_{-1} = pC_{np-1} - 2 pi): it IS the cell-centred operator of R1-R16 on
+ *   the dual phi mesh (faces pC_{k-1}, centres pF_k), which is how it is
+ *   written here.
+ * r nodes (R32): unknowns at (rF_i, tC_j, pC_k), i = 1..nr-1 (the boundary
+ *   nodes rF_0, rF_nr carry the boundary values).  Node i's control volume is
+ *   the dual r cell [rC_{i-1}, rC_i]:
+ *     V = rF_i^2 (rC_i - rC_{i-1}) sin(tC) dt dp,
+ *     r face at rC_{i-1}: g = rC_{i-1}^2 sin(tC) dt dp / (rF_i - rF_{i-1})
+ *       (node i-1; for i = 1 the boundary node rF_0: Dirichlet with kappa_P
+ *        and u_b, or Neumann: no flux), likewise at rC_i (node i+1 / rF_nr),
+ *     theta / phi faces as R4 with the dual cell's r extent rC_i - rC_{i-1}.
+ *   Arrays [comp][nr-1][nt][np].
+ * ------------------------------------------------------------------------- */
+static int pn_dual_grid(const mas_ref_grid* g, mas_ref_grid* d, double** pF, double** pC) {
+    int np = g->np, k;
+    *pF = malloc(sizeof(double) * (np + 1));
+    *pC = malloc(sizeof(double) * np);
+    if (!*pF || !*pC) { free(*pF); free(*pC); return MAS_REF_ERR_ARG; }
+    (*pF)[0] = g->pC[np - 1] - TWO_PI;
+    for (k = 1; k <= np; k++) (*pF)[k] = g->pC[k - 1];
+    for (k = 0; k < np; k++) (*pC)[k] = g->pF[k];
+    *d = *g;
+    d->pF = *pF;
+    d->pC = *pC;
+    return MAS_REF_OK;
+}
+
+int mas_ref_pn_apply(const mas_ref_grid* g, int ncomp, const double* kappa, const double* c,
+                     const double* x, double* y) {
+    mas_ref_grid d;
+    double *pF, *pC;
+    int rc;
+    if (!g || pn_dual_grid(g, &d, &pF, &pC)) return MAS_REF_ERR_ARG;
+    rc = mas_ref_op_apply(&d, ncomp, kappa, c, x, y);
+    free(pF); free(pC);
+    return rc;
+}
+
+int mas_ref_pn_volumes(const mas_ref_grid* g, double* V) {
+    mas_ref_grid d;
+    double *pF, *pC;
+    int rc;
+    if (!g || pn_dual_grid(g, &d, &pF, &pC)) return MAS_REF_ERR_ARG;
+    rc = mas_ref_volumes(&d, V);
+    free(pF); free(pC);
+    return rc;
+}
+
+int mas_ref_pn_pcg_solve(const mas_ref_grid* g, int ncomp, const double* kappa, const double* c,
+                         const double* f, double* x, double tol, int maxit, int* iters,
+                         double* relres, double* res_hist) {
+    mas_ref_grid d;
+    double *pF, *pC;
+    int rc;
+    if (!g || pn_dual_grid(g, &d, &pF, &pC)) return MAS_REF_ERR_ARG;
+    rc = mas_ref_pcg_solve(&d, ncomp, kappa, c, f, x, tol, maxit, iters, relres, res_hist);
+    free(pF); free(pC);
+    return rc;
+}
+
+/* r nodes: the slot of node i (1..nr-1) at (j, k): volume, face kinds /
+ * conductances, neighbours (flat indices of [nr-1][nt][np]) */
+#define RIDX(g, i, j, k) ((((size_t)(i) - 1) * (g)->nt + (size_t)(j)) * (g)->np + (size_t)(k))
+static void rn_slot(const mas_ref_grid* g, const tables* T, int i, int j, int k, double* V, int kind[6],
+                    double gf[6], size_t nb[6]) {
+    const int nr = g->nr, np = g->np;
+    const double drd = g->rC[i] - g->rC[i - 1];   /* the dual cell's r extent */
+    int f;
+    for (f = 0; f < 6; f++) { kind[f] = FACE_NONE; gf[f] = 0.0; nb[f] = 0; }
+    *V = g->rF[i] * g->rF[i] * drd * T->sC[j] * T->dt[j] * T->dp[k];
+    kind[0] = (i > 1) ? FACE_INTERIOR : (g->bc_inner == MAS_REF_DIRICHLET ? FACE_DIRICHLET : FACE_NONE);
+    kind[1] = (i < nr - 1) ? FACE_INTERIOR : (g->bc_outer == MAS_REF_DIRICHLET ? FACE_DIRICHLET : FACE_NONE);
+    if (kind[0]) gf[0] = g->rC[i - 1] * g->rC[i - 1] * T->sC[j] * T->dt[j] * T->dp[k] / (g->rF[i] - g->rF[i - 1]);
+    if (kind[1]) gf[1] = g->rC[i] * g->rC[i] * T->sC[j] * T->dt[j] * T->dp[k] / (g->rF[i + 1] - g->rF[i]);
+    if (kind[0] == FACE_INTERIOR) nb[0] = RIDX(g, i - 1, j, k);
+    if (kind[1] == FACE_INTERIOR) nb[1] = RIDX(g, i + 1, j, k);
+    if (j > 0) {
+        kind[2] = FACE_INTERIOR;
+        gf[2] = drd * T->sF[j] * T->dp[k] / T->ht[j];
+        nb[2] = RIDX(g, i, j - 1, k);
+    }
+    if (j < g->nt - 1) {
+        kind[3] = FACE_INTERIOR;
+        gf[3] = drd * T->sF[j + 1] * T->dp[k] / T->ht[j + 1];
+        nb[3] = RIDX(g, i, j + 1, k);
+    }
+    kind[4] = kind[5] = FACE_INTERIOR;
+    gf[4] = drd * T->dt[j] / (T->sC[j] * T->hp[k]);
+    gf[5] = drd * T->dt[j] / (T->sC[j] * T->hp[(k + 1) % np]);
+    nb[4] = RIDX(g, i, j, (k + np - 1) % np);
+    nb[5] = RIDX(g, i, j, (k + 1) % np);
+}
+
+int mas_ref_rn_volumes(const mas_ref_grid* g, double* V) {
+    tables T;
+    int i, j, k, kind[6];
+    double gf[6];
+    size_t nb[6];
+    if (!g || !V || g->nr < 2 || tables_make(g, &T)) return MAS_REF_ERR_ARG;
+    for (i = 1; i < g->nr; i++)
+        for (j = 0; j < g->nt; j++)
+            for (k = 0; k < g->np; k++) rn_slot(g, &T, i, j, k, &V[RIDX(g, i, j, k)], kind, gf, nb);
+    tables_free(&T);
+    return MAS_REF_OK;
+}
+
+int mas_ref_rn_apply(const mas_ref_grid* g, int ncomp, const double* kappa, const double* c,
+                     const double* x, double* y) {
+    tables T;
+    size_t N;
+    int i;
+    if (!g || !kappa || !x || !y || ncomp < 1 || g->nr < 2 || tables_make(g, &T)) return MAS_REF_ERR_ARG;
+    N = (size_t)(g->nr - 1) * g->nt * g->np;
+#pragma omp parallel for schedule(static)
+    for (i = 1; i < g->nr; i++) {
+        int j, k, m, kind[6];
+        double gf[6], V;
+        size_t nb[6];
+        for (j = 0; j < g->nt; j++)
+            for (k = 0; k < g->np; k++) {
+                const size_t P = RIDX(g, i, j, k);
+                rn_slot(g, &T, i, j, k, &V, kind, gf, nb);
+                for (m = 0; m < ncomp; m++) {
+                    const double* u = x + (size_t)m * N;
+                    y[(size_t)m * N + P] = (c ? c[P] : 0.0) * u[P] +
+                                           tn_slot_flux(kind, gf, nb, kappa[P], u[P], kappa, u) / V;
+                }
+            }
+    }
+    tables_free(&T);
+    return MAS_REF_OK;
+}
+
+int mas_ref_rn_diag(const mas_ref_grid* g, const double* kappa, const double* c, double* D) {
+    tables T;
+    int i;
+    if (!g || !kappa || !D || g->nr < 2 || tables_make(g, &T)) return MAS_REF_ERR_ARG;
+#pragma omp parallel for schedule(static)
+    for (i = 1; i < g->nr; i++) {
+        int j, k, kind[6];
+        double gf[6], V;
+        size_t nb[6];
+        for (j = 0; j < g->nt; j++)
+            for (k = 0; k < g->np; k++) {
+                const size_t P = RIDX(g, i, j, k);
+                rn_slot(g, &T, i, j, k, &V, kind, gf, nb);
+                D[P] = (c ? c[P] : 0.0) + tn_slot_diag(kind, gf, nb, kappa[P], kappa) / V;
+            }
+    }
+    tables_free(&T);
+    return MAS_REF_OK;
+}
+
+/* f += (1/V) G_b u_b at the boundary nodes' faces; ub [ncomp][nt][np] */
+int mas_ref_rn_dirichlet_rhs(const mas_ref_grid* g, int ncomp, const double* kappa,
+                             const double* ub_inner, const double* ub_outer, double* f) {
+    tables T;
+    size_t N, plane;
+    int m, side, j, k, kind[6];
+    double gf[6], V;
+    size_t nb[6];
+    if (!g || !kappa || !f || ncomp < 1 || g->nr < 2 || tables_make(g, &T)) return MAS_REF_ERR_ARG;
+    N = (size_t)(g->nr - 1) * g->nt * g->np;
+    plane = (size_t)g->nt * g->np;
+    for (m = 0; m < ncomp; m++)
+        for (side = 0; side < 2; side++) {
+            const double* ub = side ? ub_outer : ub_inner;
+            const int i = side ? g->nr - 1 : 1, face = side ? 1 : 0;
+            if (!ub || (side ? g->bc_outer : g->bc_inner) != MAS_REF_DIRICHLET) continue;
+            for (j = 0; j < g->nt; j++)
+                for (k = 0; k < g->np; k++) {
+                    const size_t P = RIDX(g, i, j, k);
+                    rn_slot(g, &T, i, j, k, &V, kind, gf, nb);
+                    f[(size_t)m * N + P] += kappa[P] * gf[face] * ub[(size_t)m * plane + (size_t)j * g->np + k] / V;
+                }
+        }
+    tables_free(&T);
+    return MAS_REF_OK;
+}
+
+/* Jacobi-PCG on the r-node operator (the textbook loop of pcg_core). */
+int mas_ref_rn_pcg_solve(const mas_ref_grid* g, int ncomp, const double* kappa, const double* c,
+                         const double* f, double* x, double tol, int maxit, int* iters,
+                         double* relres, double* res_hist) {
+    size_t N, n, e;
+    double *V, *D, *r, *z, *p, *q;
+    double bn, rn, rho, sigma, alpha, rho_new, beta;
+    int k, m, status = MAS_REF_NOT_CONVERGED;
+    if (!g || !kappa || !f || !x || !iters || !relres || ncomp < 1 || maxit < 0 || !(tol >= 0.0) || g->nr < 2)
+        return MAS_REF_ERR_ARG;
+    N = (size_t)(g->nr - 1) * g->nt * g->np;
+    n = N * ncomp;
+    V = malloc(sizeof(double) * N);
+    D = malloc(sizeof(double) * N);
+    r = malloc(sizeof(double) * n);
+    z = malloc(sizeof(double) * n);
+    p = malloc(sizeof(double) * n);
+    q = malloc(sizeof(double) * n);
+    if (!V || !D || !r || !z || !p || !q || mas_ref_rn_volumes(g, V) || mas_ref_rn_diag(g, kappa, c, D)) {
+        status = MAS_REF_ERR_ARG; goto done;
+    }
+    /* the V-weighted dot, per node plane in (j,k) order, then planes, then components */
+#define RDOT(a, b, out) do { size_t pl = (size_t)g->nt * g->np; int mm, ii; double s_ = 0.0; \
+        for (mm = 0; mm < ncomp; mm++) for (ii = 0; ii < g->nr - 1; ii++) { double ps = 0.0; size_t ee; \
+            for (ee = 0; ee < pl; ee++) { size_t P_ = (size_t)ii * pl + ee; \
+                ps += V[P_] * (a)[(size_t)mm * N + P_] * (b)[(size_t)mm * N + P_]; } s_ += ps; } \
+        (out) = s_; } while (0)
+    RDOT(f, f, bn);
+    bn = sqrt(bn);
+    if (bn == 0.0) {
+        for (e = 0; e < n; e++) x[e] = 0.0;
+        *iters = 0; *relres = 0.0;
+        if (res_hist) res_hist[0] = 0.0;
+        status = MAS_REF_OK; goto done;
+    }
+    mas_ref_rn_apply(g, ncomp, kappa, c, x, r);
+    for (e = 0; e < n; e++) r[e] = f[e] - r[e];
+    RDOT(r, r, rn);
+    rn = sqrt(rn);
+    if (res_hist) res_hist[0] = rn;
+    if (rn <= tol * bn) { *iters = 0; *relres = rn / bn; status = MAS_REF_OK; goto done; }
+    for (m = 0; m < ncomp; m++)
+        for (e = 0; e < N; e++) z[m * N + e] = r[m * N + e] / D[e];
+    memcpy(p, z, sizeof(double) * n);
+    RDOT(r, z, rho);
+    for (k = 1; k <= maxit; k++) {
+        mas_ref_rn_apply(g, ncomp, kappa, c, p, q);
+        RDOT(p, q, sigma);
+        if (!(sigma > 0.0) || !isfinite(sigma)) {
+            *iters = k; *relres = rn / bn; status = MAS_REF_ERR_BREAKDOWN; goto done;
+        }
+        alpha = rho / sigma;
+        for (e = 0; e < n; e++) { x[e] += alpha * p[e]; r[e] -= alpha * q[e]; }
+        RDOT(r, r, rn);
+        rn = sqrt(rn);
+        if (res_hist) res_hist[k] = rn;
+        if (rn <= tol * bn) { *iters = k; *relres = rn / bn; status = MAS_REF_OK; goto done; }
+        for (m = 0; m < ncomp; m++)
+            for (e = 0; e < N; e++) z[m * N + e] = r[m * N + e] / D[e];
+        RDOT(r, z, rho_new);
+        beta = rho_new / rho;
+        rho = rho_new;
+        for (e = 0; e < n; e++) p[e] = z[e] + beta * p[e];
+    }
+#undef RDOT
+    *iters = maxit; *relres = rn / bn; status = MAS_REF_NOT_CONVERGED;
+done:
+    free(V); free(D); free(r); free(z); free(p); free(q);
+    return status;
+}
+
+int mas_ref_pn_diag(const mas_ref_grid* g, const double* kappa, const double* c, double* D) {
+    mas_ref_grid d;
+    double *pF, *pC;
+    int rc;
+    if (!g || pn_dual_grid(g, &d, &pF, &pC)) return MAS_REF_ERR_ARG;
+    rc = mas_ref_op_diag(&d, kappa, c, D);
+    free(pF); free(pC);
+    return rc;
+}
+
+int mas_ref_pn_dirichlet_rhs(const mas_ref_grid* g, int ncomp, const double* kappa,
+                             const double* ub_inner, const double* ub_outer, double* f) {
+    mas_ref_grid d;
+    double *pF, *pC;
+    int rc;
+    if (!g || pn_dual_grid(g, &d, &pF, &pC)) return MAS_REF_ERR_ARG;
+    rc = mas_ref_dirichlet_rhs(&d, ncomp, kappa, ub_inner, ub_outer, f);
+    free(pF); free(pC);
+    return rc;
+}

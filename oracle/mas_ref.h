@@ -178,4 +178,28 @@ int mas_ref_pcg_solve_curv(const mas_ref_grid* g, const double* kappa, const dou
                            const double* f, double* x, double tol, int maxit, int* iters,
                            double* relres, double* res_hist);
 
+/* Face-centred placements (NEXT-2, readings R32-R33, mas_ref.c):
+ * phi nodes: unknowns at (rC, tC, pF_k), k = 0..np-1: the cell-centred
+ * operator on the dual phi mesh (faces pC_{k-1}, centres pF_k);
+ * r nodes: unknowns at (rF_i, tC, pC), i = 1..nr-1, arrays [comp][nr-1][nt][np];
+ * the boundary nodes rF_0 / rF_nr carry the Dirichlet values (or no flux). */
+int mas_ref_pn_apply(const mas_ref_grid* g, int ncomp, const double* kappa, const double* c,
+                     const double* x, double* y);
+int mas_ref_pn_volumes(const mas_ref_grid* g, double* V);
+int mas_ref_pn_diag(const mas_ref_grid* g, const double* kappa, const double* c, double* D);
+int mas_ref_pn_dirichlet_rhs(const mas_ref_grid* g, int ncomp, const double* kappa,
+                             const double* ub_inner, const double* ub_outer, double* f);
+int mas_ref_pn_pcg_solve(const mas_ref_grid* g, int ncomp, const double* kappa, const double* c,
+                         const double* f, double* x, double tol, int maxit, int* iters,
+                         double* relres, double* res_hist);
+int mas_ref_rn_volumes(const mas_ref_grid* g, double* V);
+int mas_ref_rn_apply(const mas_ref_grid* g, int ncomp, const double* kappa, const double* c,
+                     const double* x, double* y);
+int mas_ref_rn_diag(const mas_ref_grid* g, const double* kappa, const double* c, double* D);
+int mas_ref_rn_dirichlet_rhs(const mas_ref_grid* g, int ncomp, const double* kappa,
+                             const double* ub_inner, const double* ub_outer, double* f);
+int mas_ref_rn_pcg_solve(const mas_ref_grid* g, int ncomp, const double* kappa, const double* c,
+                         const double* f, double* x, double tol, int maxit, int* iters,
+                         double* relres, double* res_hist);
+
 #endif
