@@ -175,7 +175,17 @@ MAS_API mas_status_t mas_op_setup(mas_grid_t* g, int ncomp, const double* kappa,
  * dirichlet_rhs / solve have phi-constant pole rows.
  * Errors: as mas_op_setup; MAS_ERR_ARG for an unknown placement or a grid
  * without both poles. */
-enum { MAS_PLACE_CELL = 0, MAS_PLACE_THETA_NODE = 1 };
+/* MAS_PLACE_R_NODE / MAS_PLACE_PHI_NODE (readings R32-R33):
+ * the face-centred locations of MAS's staggered velocity components, as a
+ * scalar unknown of the same operator.  r nodes: unknowns at (rF_i, tC, pC),
+ * i = 1..nr-1, control volume the dual r cell [rC_{i-1}, rC_i], the boundary
+ * nodes rF_0 / rF_nr carrying the Dirichlet values (ub of the Dirichlet
+ * helper) or no flux; arrays [comp][nr-1][nt][np]; one rank only.  phi nodes:
+ * unknowns at (rC, tC, pF_k), k = 0..np-1, control volume the dual phi cell
+ * [pC_{k-1}, pC_k] (periodic); arrays [comp][nl][ntl][np]; any r-slab / (r,
+ * theta) decomposition on the NCCL loop.  Both: no P2P, L_par, single-
+ * reduction loop or curvature terms. */
+enum { MAS_PLACE_CELL = 0, MAS_PLACE_THETA_NODE = 1, MAS_PLACE_R_NODE = 2, MAS_PLACE_PHI_NODE = 3 };
 MAS_API mas_status_t mas_op_setup_placed(mas_grid_t* g, int ncomp, int placement, const double* kappa,
                                          const double* mass, mas_bc_t bc_r_inner,
                                          mas_bc_t bc_r_outer, cudaStream_t stream, mas_op_t** out);

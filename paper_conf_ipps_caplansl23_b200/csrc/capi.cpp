@@ -159,8 +159,10 @@ struct mas_op {
     int cg1 = 0;
     double *r2 = nullptr, *w2 = nullptr, *pcg = nullptr;
     // placement (NEXT-2): 0 cell centres; 1 theta nodes with pole rows (local
-    // rows 0 and nt hold one value per radius: k_pole_avg after every stencil)
+    // rows 0 and nt hold one value per radius: k_pole_avg after every stencil);
+    // 2 r nodes, 3 phi nodes (face-centred: other 1-D tables only)
     int tnode = 0;
+    int placement = MAS_PLACE_CELL;
     // vector-Laplacian curvature terms of the 3-component operator (NEXT-2, R31)
     int curv = 0;
     // the field-aligned term's iteration part fused into kernel A
@@ -269,11 +271,32 @@ mas_status_t mas_grid_create_2d(int nr, int nt, int np, const double* r_node, co
             return s;
         }
     }
+    {  // the face-centred placements' tables (NEXT-2): phi nodes always, r nodes on one rank
+        const std::vector<double> pn = pnode_tables(g);
+        s = dmalloc(&g->d_tab_pn, pn.size());
+        if (s == MAS_OK && cudaMemcpy(g->d_tab_pn, pn.data(), pn.size() * sizeof(double),
+                                      cudaMemcpyHostToDevice) != cudaSuccess)
+            s = MAS_ERR_CUDA;
+        if (s == MAS_OK && nranks == 1 && nr >= 2) {
+            g->rn_host = rnode_tables(g);
+            s = dmalloc(&g->d_tab_rn, g->rn_host.size());
+            if (s == MAS_OK && cudaMemcpy(g->d_tab_rn, g->rn_host.data(), g->rn_host.size() * sizeof(double),
+                                          cudaMemcpyHostToDevice) != cudaSuccess)
+                s = MAS_ERR_CUDA;
+        }
+        if (s != MAS_OK) {
+            for (double* p : {g->d_tab, g->d_tab_tn, g->d_tab_pn, g->d_tab_rn})
+                if (p) cudaFree(p);
+            delete g;
+            set_last_error("face-placement tables");
+            return s;
+        }
+    }
     if (dist) {  // nranks == 1 with a real NCCL id: a 1-rank communicator (the NCCL loop on one GPU)
         s = comm_create(dist, &g->comm);
         if (s != MAS_OK) {
-            cudaFree(g->d_tab);
-            if (g->d_tab_tn) cudaFree(g->d_tab_tn);
+            for (double* p : {g->d_tab, g->d_tab_tn, g->d_tab_pn, g->d_tab_rn})
+                if (p) cudaFree(p);
             delete g;
             return s;
         }
@@ -309,8 +332,8 @@ mas_status_t mas_grid_local_extent_2d(const mas_grid_t* g, int* i0, int* nr_loca
 
 mas_status_t mas_grid_destroy(mas_grid_t* g) {
     if (!g) return MAS_OK;
-    if (g->d_tab) cudaFree(g->d_tab);
-    if (g->d_tab_tn) cudaFree(g->d_tab_tn);
+    for (double* p : {g->d_tab, g->d_tab_tn, g->d_tab_pn, g->d_tab_rn})
+        if (p) cudaFree(p);
     comm_destroy(g->comm);
     delete g;
     return MAS_OK;
@@ -903,9 +926,11 @@ mas_status_t mas_op_setup_placed(mas_grid_t* g, int ncomp, int placement, const 
     *out = nullptr;
     if (!g || !kappa) return arg_error("null grid or kappa");
     if (ncomp != 1 && ncomp != 3) return arg_error("ncomp must be 1 or 3");
-    if (placement != MAS_PLACE_CELL && placement != MAS_PLACE_THETA_NODE) return arg_error("unknown placement");
+    if (placement < MAS_PLACE_CELL || placement > MAS_PLACE_PHI_NODE) return arg_error("unknown placement");
     if (placement == MAS_PLACE_THETA_NODE && !g->d_tab_tn)
         return arg_error("theta-node placement needs both pole flags, nt >= 2 and ptheta == 1");
+    if (placement == MAS_PLACE_R_NODE && !g->d_tab_rn)
+        return arg_error("r-node placement needs one rank and nr >= 2");
     if ((bc_r_inner != MAS_BC_DIRICHLET && bc_r_inner != MAS_BC_NEUMANN) ||
         (bc_r_outer != MAS_BC_DIRICHLET && bc_r_outer != MAS_BC_NEUMANN))
         return arg_error("bad boundary condition");
@@ -916,8 +941,12 @@ mas_status_t mas_op_setup_placed(mas_grid_t* g, int ncomp, int placement, const 
     op->bci = bc_r_inner;
     op->bco = bc_r_outer;
     op->tnode = placement == MAS_PLACE_THETA_NODE;
-    // local block [nl][ntl][np]; theta nodes: [nl][nt+1][np]
-    const int nl = g->nl, nt = op->tnode ? g->nt + 1 : g->ntl, np = g->np;
+    op->placement = placement;
+    // local block [nl][ntl][np]; theta nodes: [nl][nt+1][np]; r nodes: [nr-1][nt][np]
+    const int nl = placement == MAS_PLACE_R_NODE ? g->nr - 1 : g->nl;
+    const int nt = op->tnode ? g->nt + 1 : g->ntl, np = g->np;
+    // this block holds the global outer r-boundary (r nodes: one rank, always)
+    const bool owns_top = placement == MAS_PLACE_R_NODE || g->i0 + g->nl == g->nr;
     const long long plane = (long long)nt * np;
     op->Nl = (long long)nl * plane;
     if ((long long)ncomp * op->Nl >= (1LL << 31)) {  // the stencil kernels index with 32-bit offsets
@@ -979,12 +1008,13 @@ mas_status_t mas_op_setup_placed(mas_grid_t* g, int ncomp, int placement, const 
     // kernels use kappa_ghost = kappa_P, u_ghost = 0 (R3).
     {
         std::vector<double> w(2 * nl);
+        const bool rn = placement == MAS_PLACE_R_NODE;  // r nodes: the rnode_tables weights
         for (int il = 0; il < nl; il++) {
-            w[il] = g->tab.wRm[il];
-            w[nl + il] = g->tab.wRp[il];
+            w[il] = rn ? g->rn_host[il] : g->tab.wRm[il];
+            w[nl + il] = rn ? g->rn_host[nl + il] : g->tab.wRp[il];
         }
         if (g->i0 == 0 && bc_r_inner == MAS_BC_NEUMANN) w[0] = 0.0;
-        if (g->i0 + nl == g->nr && bc_r_outer == MAS_BC_NEUMANN) w[2 * nl - 1] = 0.0;
+        if (owns_top && bc_r_outer == MAS_BC_NEUMANN) w[2 * nl - 1] = 0.0;
         if (cudaMemcpy(op->wR, w.data(), w.size() * sizeof(double), cudaMemcpyHostToDevice) !=
             cudaSuccess) {
             op_free(op);
@@ -995,12 +1025,12 @@ mas_status_t mas_op_setup_placed(mas_grid_t* g, int ncomp, int placement, const 
     Geo& G = op->geo;
     G.nl = nl; G.nt = nt; G.np = np; G.plane = plane;
     G.glob_lo = g->i0 == 0;
-    G.glob_hi = g->i0 + nl == g->nr;
+    G.glob_hi = owns_top;
     G.wRm = op->wR;
     G.wRp = op->wR + nl;
-    const double* t = g->d_tab;
-    G.irc2 = t; t += nl;
-    G.vr = t; t += nl;
+    const double* t = g->d_tab;  // the grid's (cell-centred) tables: [irc2 vr](g->nl) [theta](ntl) [phi](np)
+    G.irc2 = t; t += g->nl;
+    G.vr = t; t += g->nl;
     G.wTm = t; t += g->ntl;
     G.wTp = t; t += g->ntl;
     G.isc2 = t; t += g->ntl;
@@ -1010,6 +1040,15 @@ mas_status_t mas_op_setup_placed(mas_grid_t* g, int ncomp, int placement, const 
         G.wTp = g->d_tab_tn + nt;
         G.isc2 = g->d_tab_tn + 2 * nt;
         G.vt = g->d_tab_tn + 3 * nt;
+    }
+    if (placement == MAS_PLACE_PHI_NODE) {  // the dual phi cells (NEXT-2, R33)
+        G.wPm = g->d_tab_pn;
+        G.wPp = g->d_tab_pn + np;
+        G.vp = g->d_tab_pn + 2 * np;
+    }
+    if (placement == MAS_PLACE_R_NODE) {  // the dual r cells (NEXT-2, R32); wR above
+        G.irc2 = g->d_tab_rn + 2 * nl;
+        G.vr = g->d_tab_rn + 3 * nl;
     }
     G.wPm = t; t += np;
     G.wPp = t; t += np;
@@ -1221,7 +1260,8 @@ mas_status_t mas_op_radial_sums(const mas_op_t* op_c, const double* x, const dou
 mas_status_t mas_op_enable_p2p(mas_op_t* op, cudaStream_t s) {
     if (!op) return arg_error("null op");
     if (op->p2p) return MAS_OK;
-    if (op->tnode) return arg_error("P2P transport: cell-centred placement only (theta nodes keep NCCL)");
+    if (op->placement != MAS_PLACE_CELL)
+        return arg_error("P2P transport: cell-centred placement only (the other placements keep NCCL)");
     if (op->cg1) return arg_error("P2P transport: the two-kernel loop only (single reduction is on)");
     Comm* comm = op->g->comm;
     const int P = comm_nranks(comm), rank = comm_rank(comm);
@@ -1333,7 +1373,7 @@ mas_status_t mas_op_set_single_reduction(mas_op_t* op, int on) {
     if (op->p2p) return arg_error("single-reduction PCG: the NCCL loop on r-slabs (not the P2P transport)");
     if (op->g->ptheta > 1) return arg_error("single-reduction PCG: r-slab decompositions only (ptheta == 1)");
     if (op->aniso) return arg_error("single-reduction PCG: isotropic operator only (no mas_op_set_aniso)");
-    if (op->tnode) return arg_error("single-reduction PCG: cell-centred placement only");
+    if (op->placement != MAS_PLACE_CELL) return arg_error("single-reduction PCG: cell-centred placement only");
     if (op->curv) return arg_error("single-reduction PCG: without the curvature terms");
     const size_t n = op->ncomp * (size_t)op->Nl;
     if (!op->r2) ST(dmalloc(&op->r2, n));
@@ -1510,7 +1550,7 @@ mas_status_t mas_op_kernel_bench(mas_op_t* op, int reps, double* a_ms, double* b
 mas_status_t mas_op_set_curvature(mas_op_t* op, int on) {
     if (!op) return arg_error("null op");
     if (on && op->ncomp != 3) return arg_error("curvature terms: the 3-component (viscosity) operator only");
-    if (on && op->tnode) return arg_error("curvature terms: cell-centred placement only");
+    if (on && op->placement != MAS_PLACE_CELL) return arg_error("curvature terms: cell-centred placement only");
     if (on && op->cg1) return arg_error("curvature terms: the two-kernel loop only (single reduction is on)");
     op->curv = on ? 1 : 0;
     return MAS_OK;
@@ -1593,7 +1633,7 @@ mas_status_t mas_op_set_aniso(mas_op_t* op, const double* kpar, const double* bh
     }
     if (!bhat) return arg_error("null bhat");
     if (op->cg1) return arg_error("field-aligned conduction: switch the single-reduction loop off first");
-    if (op->tnode) return arg_error("field-aligned conduction: cell-centred placement only");
+    if (op->placement != MAS_PLACE_CELL) return arg_error("field-aligned conduction: cell-centred placement only");
     if (op->ncomp != 1) return arg_error("field-aligned conduction needs ncomp == 1");
     if (op->g->ptheta > 1)
         return arg_error("field-aligned conduction: r-slab decompositions only (ptheta == 1)");

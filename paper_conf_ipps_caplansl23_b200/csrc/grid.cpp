@@ -147,4 +147,43 @@ std::vector<double> tnode_tables(const mas_grid* g) {
     return t;
 }
 
+// phi-node placement (NEXT-2, R33): unknowns at pF_k; the dual phi cells
+// [pC_{k-1}, pC_k] (width hp_k) with node distances pF_k - pF_{k-1} (dp_{k-1},
+// periodic).  Same layout as Tables' phi part: [wPm | wPp | vp](np).
+std::vector<double> pnode_tables(const mas_grid* g) {
+    const int np = g->np;
+    const double *pF = g->pF.data(), *pC = g->pC.data();
+    std::vector<double> t(3 * (size_t)np);
+    double *wPm = t.data(), *wPp = wPm + np, *vp = wPp + np;
+    auto width = [&](int k) { return k == 0 ? pC[0] + kTwoPi - pC[np - 1] : pC[k] - pC[k - 1]; };
+    auto dist = [&](int k) { k = (k + np) % np; return pF[k == 0 ? np : k] - pF[k == 0 ? np - 1 : k - 1]; };
+    for (int k = 0; k < np; k++) {
+        const double w = width(k);
+        wPm[k] = 1.0 / (dist(k) * w);
+        wPp[k] = 1.0 / (dist(k + 1) * w);
+        vp[k] = w;
+    }
+    return t;
+}
+
+// r-node placement (NEXT-2, R32): unknowns at rF_i, i = 1..nr-1 (one rank);
+// the dual r cells [rC_{i-1}, rC_i] with node distances rF_i - rF_{i-1}; the
+// boundary nodes rF_0 / rF_nr are the Dirichlet faces' values.
+// [wRm | wRp | irc2 | vr](nr-1)
+std::vector<double> rnode_tables(const mas_grid* g) {
+    const int n = g->nr - 1;
+    const double *rF = g->rF.data(), *rC = g->rC.data();
+    std::vector<double> t(4 * (size_t)(n > 0 ? n : 0));
+    double *wRm = t.data(), *wRp = wRm + n, *irc2 = wRp + n, *vr = irc2 + n;
+    for (int l = 0; l < n; l++) {
+        const int i = l + 1;
+        const double drd = rC[i] - rC[i - 1], rf2 = rF[i] * rF[i];
+        wRm[l] = rC[i - 1] * rC[i - 1] / ((rF[i] - rF[i - 1]) * rf2 * drd);
+        wRp[l] = rC[i] * rC[i] / ((rF[i + 1] - rF[i]) * rf2 * drd);
+        irc2[l] = 1.0 / rf2;
+        vr[l] = rf2 * drd;
+    }
+    return t;
+}
+
 }  // namespace mas

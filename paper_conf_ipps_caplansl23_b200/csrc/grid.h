@@ -29,6 +29,9 @@ struct mas_grid {
     mas::Tables tab;
     double* d_tab = nullptr;  // device copy of the theta/phi tables + irc2/vr
     double* d_tab_tn = nullptr;  // theta-node placement: [wTm wTp isc2 vt](nt+1) (both poles, ptheta 1)
+    double* d_tab_pn = nullptr;  // phi-node placement: [wPm wPp vp](np)
+    double* d_tab_rn = nullptr;  // r-node placement (one rank): [wRm wRp irc2 vr](nr-1)
+    std::vector<double> rn_host; // the same, host copy (the op folds the boundary conditions into wR)
     mas::Comm* comm = nullptr;
 };
 
@@ -40,6 +43,8 @@ int validate_mesh(int nr, int nt, int np, const double* rF, const double* rC, co
 void partition(int nr, int nranks, int rank, int* i0, int* nl);
 void build_tables(mas_grid* g);
 std::vector<double> tnode_tables(const mas_grid* g);
+std::vector<double> pnode_tables(const mas_grid* g);
+std::vector<double> rnode_tables(const mas_grid* g);
 
 // ---- comm.cpp -------------------------------------------------------------
 mas_status_t comm_unique_id(unsigned char out[128]);

@@ -20,7 +20,7 @@ MAS_OK, MAS_NOT_CONVERGED, MAS_ERR_ARG, MAS_ERR_CUDA, MAS_ERR_NCCL, MAS_ERR_NOME
     MAS_ERR_BREAKDOWN = range(7)
 MAS_BC_DIRICHLET, MAS_BC_NEUMANN = 0, 1
 MAS_POLE_NORTH, MAS_POLE_SOUTH = 1, 2
-MAS_PLACE_CELL, MAS_PLACE_THETA_NODE = 0, 1
+MAS_PLACE_CELL, MAS_PLACE_THETA_NODE, MAS_PLACE_R_NODE, MAS_PLACE_PHI_NODE = 0, 1, 2, 3
 
 # every symbol include/mas_pcg.h declares
 ABI_SYMBOLS = ("mas_comm_unique_id", "mas_partition", "mas_grid_create", "mas_grid_local_extent",
@@ -401,9 +401,11 @@ class Operator:
         self.grid = grid
         self.ncomp = ncomp
         self.placement = placement
-        # theta nodes (NEXT-2): nt + 1 rows, the first and last on the poles
+        # theta nodes (NEXT-2): nt + 1 rows, the first and last on the poles;
+        # r nodes: nr - 1 planes (one rank)
         self.rows = grid.shape[1] + 1 if placement == MAS_PLACE_THETA_NODE else grid.ntl
-        self.N = grid.nl * self.rows * grid.shape[2]
+        self.planes = grid.shape[0] - 1 if placement == MAS_PLACE_R_NODE else grid.nl
+        self.N = self.planes * self.rows * grid.shape[2]
         _expect(kappa, self.N, "kappa")
         _expect(mass, self.N, "mass")
         self.h = mas_op_setup_placed(grid.h, ncomp, placement, kappa, mass, bc_inner, bc_outer, stream)
@@ -487,7 +489,7 @@ class Operator:
     def radial_sums(self, x, w, out, stream=None):
         _expect(x, self.ncomp * self.N, "x")
         _expect(w, self.rows * self.grid.shape[2], "w")
-        _expect(out, self.ncomp * self.grid.nl, "out")
+        _expect(out, self.ncomp * self.planes, "out")
         mas_op_radial_sums(self.h, x, w, out, stream)
 
     @property
