@@ -142,3 +142,57 @@ def test_fullsize_c2a_apply_and_solve(mp, oracle_mod):
     assert abs(it - ito) <= 1, (it, ito)
     xg = xs.cpu().numpy()
     assert math.sqrt((V * (xg - xo) ** 2).sum() / (V * xo ** 2).sum()) <= 1e-10  # unconditional (north_star: x <= 1e-10)
+
+
+# ---------------------------------------------------------------------------
+# the round-2 bench configurations at full size: the single-reduction loop
+# (bench --solver cg1) on C2 and C3, and C2t (theta nodes with pole rows)
+# ---------------------------------------------------------------------------
+@pytest.mark.parametrize("cfg", ["C2", "C3"])
+def test_fullsize_single_reduction_vs_oracle(mp, oracle_mod, cfg):
+    kind, nr, nt, np_ = {"C2": ("conduction", 128, 128, 256), "C3": ("viscosity", 256, 256, 512)}[cfg]
+    prob = W.make(kind, nr=nr, nt=nt, np_=np_)
+    d = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()
+    g = mp.Grid(prob.mesh)
+    op = mp.Operator(g, prob.ncomp, d(prob.kappa), d(prob.c), prob.bc_inner, prob.bc_outer)
+    op.set_single_reduction(True)
+    f = d(prob.f)
+    if prob.ub_inner is not None:
+        op.dirichlet_rhs(d(prob.ub_inner), None, f)
+    x = d(prob.x0)
+    st, it, rel, _ = op.solve(f, x, prob.tol, prob.maxit)
+    assert st == mp.MAS_OK and rel <= prob.tol
+    xg = x.cpu().numpy()
+    rc, xo, ito, _, _ = oracle_mod.solve_problem(prob, cg1=True)
+    assert rc == oracle_mod.OK
+    # NEXT-1's band: +-2 iterations, x <= 1e-9
+    assert abs(it - ito) <= 2, (it, ito)
+    V = oracle_mod.Oracle.for_problem(prob).volumes()[None]
+    assert math.sqrt((V * (xg - xo) ** 2).sum() / (V * xo ** 2).sum()) <= 1e-9
+
+
+def test_fullsize_theta_nodes_vs_oracle(mp, oracle_mod):
+    prob = W.tnode_conduction_problem(128, 128, 256)
+    d = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()
+    g = mp.Grid(prob.mesh)
+    op = mp.Operator(g, 1, d(prob.kappa), d(prob.c), prob.bc_inner, prob.bc_outer,
+                     placement=mp.MAS_PLACE_THETA_NODE)
+    f = d(prob.f)
+    op.dirichlet_rhs(d(prob.ub_inner), None, f)
+    x = d(prob.x0)
+    st, it, rel, _ = op.solve(f, x, prob.tol, prob.maxit)
+    assert st == mp.MAS_OK
+    o = oracle_mod.Oracle.for_problem(prob)
+    fo = o.tn_dirichlet_rhs(prob.kappa, prob.f, prob.ub_inner, None)
+    rc, xo, ito, _, _ = o.tn_pcg(prob.kappa, prob.c, fo, prob.x0, prob.tol, prob.maxit)
+    env = 0  # the oracle's own 1-ulp sensitivity (R20)
+    for sd in range(2):
+        fp = fo * (1.0 + 1e-16 * np.random.default_rng(sd).standard_normal(fo.shape))
+        _, _, itp, _, _ = o.tn_pcg(prob.kappa, prob.c, fp, prob.x0, prob.tol, prob.maxit)
+        env = max(env, abs(itp - ito))
+    assert abs(it - ito) <= max(1, env), (it, ito, env)
+    V = o.tn_volumes()[None]
+    xg = x.cpu().numpy()
+    assert math.sqrt((V * (xg - xo) ** 2).sum() / (V * xo ** 2).sum()) <= 1e-10
+    for row in (0, -1):  # one value per pole and radius
+        assert np.array_equal(xg[0, :, row, :], np.broadcast_to(xg[0, :, row, :1], xg[0, :, row, :].shape))
