@@ -1041,11 +1041,6 @@ mas_status_t mas_op_setup_placed(mas_grid_t* g, int ncomp, int placement, const 
         G.isc2 = g->d_tab_tn + 2 * nt;
         G.vt = g->d_tab_tn + 3 * nt;
     }
-    if (placement == MAS_PLACE_PHI_NODE) {  // the dual phi cells (NEXT-2, R33)
-        G.wPm = g->d_tab_pn;
-        G.wPp = g->d_tab_pn + np;
-        G.vp = g->d_tab_pn + 2 * np;
-    }
     if (placement == MAS_PLACE_R_NODE) {  // the dual r cells (NEXT-2, R32); wR above
         G.irc2 = g->d_tab_rn + 2 * nl;
         G.vr = g->d_tab_rn + 3 * nl;
@@ -1053,6 +1048,11 @@ mas_status_t mas_op_setup_placed(mas_grid_t* g, int ncomp, int placement, const 
     G.wPm = t; t += np;
     G.wPp = t; t += np;
     G.vp = t;
+    if (placement == MAS_PLACE_PHI_NODE) {  // the dual phi cells (NEXT-2, R33)
+        G.wPm = g->d_tab_pn;
+        G.wPp = g->d_tab_pn + np;
+        G.vp = g->d_tab_pn + 2 * np;
+    }
     const char* g_env = getenv("MAS_NO_GRAPH");  // experiment hook: host-driven loop
     op->use_graph = !(g_env && atoi(g_env));
     const char* gp_env = getenv("MAS_GRAPH_PRE");  // experiment hook (round-1 graph form)

@@ -263,9 +263,12 @@ struct Stage {
 // The scalar halo items do not fit in registers next to the own pair's
 // in-flight loads (ptxas spilled them, forcing an early wait), so each halo
 // thread copies its item into a private shared-memory slot instead:
-// layout [field][kHaloSlots], fields 0 kappa, 1 1/D, 2.. u[NC], po[NC]
+// layout [field][kHS], fields 0 kappa, 1 1/D, 2.. u[NC], po[NC]
 // (+ w[NC] in MODE_CG1).
-constexpr int kHaloSlots = 2 * TK + 2 * TJ + 4;  // + the 4 diagonal halo cells (fused L_par)
+// (+ the 4 diagonal halo cells for the fused L_par only: the slot stride and
+// the extra ghost-plane halo branch cost the 3-component kernel A ~20%)
+template <bool LPAR>
+constexpr int kHS = 2 * TK + 2 * TJ + (LPAR ? 4 : 0);
 __device__ __forceinline__ void cpa8(double* sdst, const double* gsrc) {
     const unsigned sa = (unsigned)__cvta_generic_to_shared(sdst);
     asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"(sa), "l"(gsrc) : "memory");
@@ -279,19 +282,19 @@ __device__ __forceinline__ void cpa_wait_all() { asm volatile("cp.async.wait_gro
 __device__ __forceinline__ const double* trow_at(const TRows& T, bool hi, int comp, int i, int k) {
     return hi ? T.hi + comp * T.cs_hi + i * T.ps_hi + k : T.lo + comp * T.cs_lo + i * T.ps_lo + k;
 }
-template <int MODE, int NC>
+template <int MODE, int NC, bool LPAR = false>
 __device__ __forceinline__ void trow_issue(const StencilArgs& a, int i, const HaloMeta& hm, bool first,
                                         double* h) {
     const bool hi = hm.hkind == 5;
     const int k = hm.hoff;
     cpa8(h, trow_at(a.tkappa, hi, 0, i, k));
 #pragma unroll
-    for (int c = 0; c < NC; c++) cpa8(h + (2 + c) * kHaloSlots, trow_at(a.tu, hi, c, i, k));
+    for (int c = 0; c < NC; c++) cpa8(h + (2 + c) * kHS<LPAR>, trow_at(a.tu, hi, c, i, k));
     if (MODE == MODE_PCGA || MODE == MODE_CG1) {
-        cpa8(h + kHaloSlots, trow_at(a.tdinv, hi, 0, i, k));
+        cpa8(h + kHS<LPAR>, trow_at(a.tdinv, hi, 0, i, k));
         if (!first) {
 #pragma unroll
-            for (int c = 0; c < NC; c++) cpa8(h + (2 + NC + c) * kHaloSlots, trow_at(a.tpold, hi, c, i, k));
+            for (int c = 0; c < NC; c++) cpa8(h + (2 + NC + c) * kHS<LPAR>, trow_at(a.tpold, hi, c, i, k));
         }
     }
 }
@@ -360,7 +363,7 @@ constexpr bool kCg1LateOwn = (NC == 3);
 template <int NC>
 constexpr bool kCg1DotsAtCommit = (NC == 3);
 
-template <int MODE, int NC>
+template <int MODE, int NC, bool LPAR = false>
 __device__ __forceinline__ void stage_issue(const StencilArgs& a, int i, int j0, int k0, int height,
                                             int width, const HaloMeta& hm, bool first, bool xupd,
                                             bool halo, bool own_work, Stage<NC>& S, double* hst) {
@@ -397,46 +400,46 @@ __device__ __forceinline__ void stage_issue(const StencilArgs& a, int i, int j0,
         }
     }
     if (halo && hm.hkind >= 4 && interior) {
-        trow_issue<MODE, NC>(a, i, hm, first, hst + threadIdx.x);
+        trow_issue<MODE, NC, LPAR>(a, i, hm, first, hst + threadIdx.x);
     } else if (halo && hm.hkind == 1) {
         double* h = hst + threadIdx.x;
         if (interior) {  // halo planes are stencil planes: always interior here
             const int hi = ipl + (int)hm.hoff;
             cpa8(h, a.kappa.in + hi);
 #pragma unroll
-            for (int c = 0; c < NC; c++) cpa8(h + (2 + c) * kHaloSlots, a.u.in + c * Nl + hi);
+            for (int c = 0; c < NC; c++) cpa8(h + (2 + c) * kHS<LPAR>, a.u.in + c * Nl + hi);
             if (MODE == MODE_PCGA || MODE == MODE_CG1) {
-                cpa8(h + kHaloSlots, a.dinv.in + hi);
+                cpa8(h + kHS<LPAR>, a.dinv.in + hi);
                 if (!first) {
 #pragma unroll
                     for (int c = 0; c < NC; c++)
-                        cpa8(h + (2 + NC + c) * kHaloSlots, a.pold.in + c * Nl + hi);
+                        cpa8(h + (2 + NC + c) * kHS<LPAR>, a.pold.in + c * Nl + hi);
                     if (MODE == MODE_CG1) {
 #pragma unroll
                         for (int c = 0; c < NC; c++)
-                            cpa8(h + (2 + 2 * NC + c) * kHaloSlots, a.w.in + c * Nl + hi);
+                            cpa8(h + (2 + 2 * NC + c) * kHS<LPAR>, a.w.in + c * Nl + hi);
                     }
                 }
             }
-        } else if (MODE == MODE_PCGA) {
+        } else if (LPAR && MODE == MODE_PCGA) {
             // an r-ghost plane's halo (the fused field-aligned term's corners
             // read it): the ghost copy, or the neighbour's own array in place
             const PlanePtrs<NC> P = plane_ptrs<MODE, NC>(a, i, first);
             const int hi = (int)hm.hoff;
             cpa8(h, P.kap + hi);
 #pragma unroll
-            for (int c = 0; c < NC; c++) cpa8(h + (2 + c) * kHaloSlots, P.u[c] + hi);
-            cpa8(h + kHaloSlots, P.di + hi);
+            for (int c = 0; c < NC; c++) cpa8(h + (2 + c) * kHS<LPAR>, P.u[c] + hi);
+            cpa8(h + kHS<LPAR>, P.di + hi);
             if (!first) {
 #pragma unroll
-                for (int c = 0; c < NC; c++) cpa8(h + (2 + NC + c) * kHaloSlots, P.po[c] + hi);
+                for (int c = 0; c < NC; c++) cpa8(h + (2 + NC + c) * kHS<LPAR>, P.po[c] + hi);
             }
         }
     }
     cpa_commit();
 }
 
-template <int MODE, int NC>
+template <int MODE, int NC, bool LPAR = false>
 __device__ __forceinline__ void stage_commit(const StencilArgs& a, int i, int j0, int k0, int height,
                                              int width, const HaloMeta& hm, bool first, double beta,
                                              double alpha_prev, bool xupd, bool halo, bool own_work,
@@ -519,16 +522,16 @@ __device__ __forceinline__ void stage_commit(const StencilArgs& a, int i, int j0
         const double* h = hst + threadIdx.x;
 #pragma unroll
         for (int c = 0; c < NC; c++) {
-            double u = h[(2 + c) * kHaloSlots];
+            double u = h[(2 + c) * kHS<LPAR>];
             if (MODE == MODE_PCGA) {
-                const double z = h[kHaloSlots] * u;
-                u = first ? z : fma(beta, h[(2 + NC + c) * kHaloSlots], z);
+                const double z = h[kHS<LPAR>] * u;
+                u = first ? z : fma(beta, h[(2 + NC + c) * kHS<LPAR>], z);
             } else if (MODE == MODE_CG1) {
                 if (!first) {  // r_k of the halo cell from its r, s, w of iteration k-1
-                    const double sv = fma(beta, h[(2 + NC + c) * kHaloSlots], h[(2 + 2 * NC + c) * kHaloSlots]);
+                    const double sv = fma(beta, h[(2 + NC + c) * kHS<LPAR>], h[(2 + 2 * NC + c) * kHS<LPAR>]);
                     u = fma(-alpha_prev, sv, u);
                 }
-                u = h[kHaloSlots] * u;
+                u = h[kHS<LPAR>] * u;
             }
             sfield(buf, c)[hm.hidx] = u;
         }
@@ -841,7 +844,7 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
     auto slot = [&](int i) { return smem + ((i - ia + 1) & 3) * BUF; };
     // private cp.async slots of the halo items: static shared memory, so the
     // shared-window address needs no runtime conversion
-    __shared__ __align__(16) double hst_arr[(2 + (MODE == MODE_CG1 ? 3 : 2) * NC) * kHaloSlots];
+    __shared__ __align__(16) double hst_arr[(2 + (MODE == MODE_CG1 ? 3 : 2) * NC) * kHS<LPAR>];
     auto real_plane = [&](int p) { return !(p == g.nl && g.glob_hi); };
 
     // 1-D geometry of this work item staged in shared memory once (visible to
@@ -898,16 +901,16 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
     // in the prologue; the halo item copies of ia-1 and ia go one after the
     // other through the same private slots)
     if (!lo_ghost) {
-        stage_issue<MODE, NC>(a, ia - 1, j0, k0, height, width, hm, FIRSTK, false, LPAR, false, S0, hst_arr);
+        stage_issue<MODE, NC, LPAR>(a, ia - 1, j0, k0, height, width, hm, FIRSTK, false, LPAR, false, S0, hst_arr);
         if (LPAR)
-            stage_commit<MODE, NC>(a, ia - 1, j0, k0, height, width, hm, FIRSTK, beta, alpha_prev, false,
+            stage_commit<MODE, NC, LPAR>(a, ia - 1, j0, k0, height, width, hm, FIRSTK, beta, alpha_prev, false,
                                    true, false, S0, slot(ia - 1), kdummy, on, hst_arr, acc);
     }
-    stage_issue<MODE, NC>(a, ia, j0, k0, height, width, hm, FIRSTK, xupd, true, true, S, hst_arr);
+    stage_issue<MODE, NC, LPAR>(a, ia, j0, k0, height, width, hm, FIRSTK, xupd, true, true, S, hst_arr);
     if (!lo_ghost && !LPAR)
-        stage_commit<MODE, NC>(a, ia - 1, j0, k0, height, width, hm, FIRSTK, beta, alpha_prev, false,
+        stage_commit<MODE, NC, LPAR>(a, ia - 1, j0, k0, height, width, hm, FIRSTK, beta, alpha_prev, false,
                                false, false, S0, slot(ia - 1), kdummy, on, hst_arr, acc);
-    stage_commit<MODE, NC>(a, ia, j0, k0, height, width, hm, FIRSTK, beta, alpha_prev, xupd, true, true,
+    stage_commit<MODE, NC, LPAR>(a, ia, j0, k0, height, width, hm, FIRSTK, beta, alpha_prev, xupd, true, true,
                            S, slot(ia), kown, oc, hst_arr, acc);
     if (lo_ghost) ghost_plane<NC>(slot(ia - 1), height, width, kown, LPAR);
     if (LPAR) {  // corner plane ia (cells ia-1 | ia): its lower-corner part for plane ia
@@ -925,14 +928,14 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
         }
     }
     if (real_plane(ia + 1))
-        stage_issue<MODE, NC>(a, ia + 1, j0, k0, height, width, hm, FIRSTK, xupd && (ia + 1 < ib),
+        stage_issue<MODE, NC, LPAR>(a, ia + 1, j0, k0, height, width, hm, FIRSTK, xupd && (ia + 1 < ib),
                               LPAR || ia + 1 < ib, ia + 1 < ib, S, hst_arr);
     if (LPAR) lpar_coef_issue(a, ia + 1, j0, k0, height, width, lcf + ((ia + 1) & 1) * 3 * LCA);
 
     for (int i = ia; i < ib; i++) {
         // commit plane i+1 (its loads were issued one plane earlier)
         if (real_plane(i + 1))
-            stage_commit<MODE, NC>(a, i + 1, j0, k0, height, width, hm, FIRSTK, beta, alpha_prev,
+            stage_commit<MODE, NC, LPAR>(a, i + 1, j0, k0, height, width, hm, FIRSTK, beta, alpha_prev,
                                    xupd && (i + 1 < ib), LPAR || i + 1 < ib, i + 1 < ib, S, slot(i + 1),
                                    kown, on, hst_arr, acc);
         else
@@ -944,7 +947,7 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
         // 3-component one (tools/abtest.sh), hence the split.
         constexpr bool kIssueEarly = (NC == 1);
         if (kIssueEarly && i + 2 <= ib && real_plane(i + 2))
-            stage_issue<MODE, NC>(a, i + 2, j0, k0, height, width, hm, FIRSTK, xupd && (i + 2 < ib),
+            stage_issue<MODE, NC, LPAR>(a, i + 2, j0, k0, height, width, hm, FIRSTK, xupd && (i + 2 < ib),
                                   LPAR || i + 2 < ib, i + 2 < ib, S, hst_arr);
         if (LPAR && i + 2 <= ib) lpar_coef_issue(a, i + 2, j0, k0, height, width, lcf + ((i + 2) & 1) * 3 * LCA);
         __syncthreads();
@@ -960,7 +963,7 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
             plane_prefetch<MODE, NC>(a, i + kPfDist, j0, k0, height, width, FIRSTK, xupd);
 #endif
         if (!kIssueEarly && i + 2 <= ib && real_plane(i + 2))
-            stage_issue<MODE, NC>(a, i + 2, j0, k0, height, width, hm, FIRSTK, xupd && (i + 2 < ib),
+            stage_issue<MODE, NC, LPAR>(a, i + 2, j0, k0, height, width, hm, FIRSTK, xupd && (i + 2 < ib),
                                   i + 2 < ib, i + 2 < ib, S, hst_arr);
 
         if (own) {

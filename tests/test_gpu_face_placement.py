@@ -80,6 +80,35 @@ def test_face_apply_diag_rhs(mp, oracle_mod, shape, ncomp, bc, which):
     g.close()
 
 
+@pytest.mark.parametrize("ncomp", [1, 3])
+def test_phi_nodes_nonuniform_phi(mp, oracle_mod, ncomp):
+    """A non-uniform periodic phi mesh: the dual phi cells differ from the
+    cell-centred ones (on a uniform mesh they coincide, so only this case
+    tells the phi-node tables from the cell tables)."""
+    import dataclasses
+    m0 = W.stretched_mesh(12, 10, 48)
+    s = np.arange(49, dtype=np.float64) / 48
+    pF = 2.0 * math.pi * s + 0.6 * np.sin(2.0 * math.pi * s)
+    pF[0], pF[-1] = 0.0, 2.0 * math.pi
+    mesh = dataclasses.replace(m0, pF=pF, pC=0.5 * (pF[1:] + pF[:-1]))
+    for which in ("pn", "cell"):
+        o = oracle_mod.Oracle(mesh, 0, 1)
+        sh = o.shape
+        rng = np.random.default_rng(3)
+        kappa, c = rng.uniform(0.5, 2.0, size=sh), rng.uniform(0.1, 1.0, size=sh)
+        x = W.random_field((ncomp,) + sh, 7)
+        pl = mp.MAS_PLACE_PHI_NODE if which == "pn" else mp.MAS_PLACE_CELL
+        g = mp.Grid(mesh)
+        op = mp.Operator(g, ncomp, dev(kappa), dev(c), 0, 1, placement=pl)
+        y = torch.empty((ncomp,) + sh, dtype=torch.float64, device="cuda")
+        op.apply(dev(x), y)
+        yo = (o.pn_apply if which == "pn" else o.apply)(kappa, c, x)
+        V = o.pn_volumes() if which == "pn" else o.volumes()
+        assert rel_l2_V(V, host(y), yo) <= 1e-13, which
+        op.close()
+        g.close()
+
+
 def mms_at(mesh, which):
     """C1's manufactured problem at the nodes of the placement."""
     r = mesh.rF[1:-1] if which == "rn" else mesh.rC

@@ -21,6 +21,18 @@ def mesh(nr, nt, np_, R=3.0):
     return W.stretched_mesh(nr, nt, np_, 1.0, 2.0, R)
 
 
+def phi_stretched(m, b=0.6):
+    """the same mesh with a smooth non-uniform periodic phi mesh
+    (pF = 2 pi s + b sin 2 pi s): the phi nodes are then off the dual cells'
+    midpoints by O(h^2), and the dual tables differ from the cell ones"""
+    import dataclasses
+    n = len(m.pF) - 1
+    s = np.arange(n + 1, dtype=np.float64) / n
+    pF = 2.0 * math.pi * s + b * np.sin(2.0 * math.pi * s)
+    pF[0], pF[-1] = 0.0, 2.0 * math.pi
+    return dataclasses.replace(m, pF=pF, pC=0.5 * (pF[1:] + pF[:-1]))
+
+
 def rand(shape, seed):
     rng = np.random.default_rng(seed)
     return rng.uniform(0.5, 2.0, size=shape), rng.uniform(0.1, 1.0, size=shape)
@@ -40,15 +52,17 @@ def test_rn_volumes_fill_the_node_shell(oracle_mod):
     assert min(orders(errs)) > 1.8, errs
 
 
-def test_pn_volumes_fill_the_shell(oracle_mod):
-    m = mesh(6, 8, 12)
+@pytest.mark.parametrize("stretch", [False, True])
+def test_pn_volumes_fill_the_shell(oracle_mod, stretch):
+    m = phi_stretched(mesh(6, 8, 12)) if stretch else mesh(6, 8, 12)
     o = oracle_mod.Oracle(m, 0, 0)
     np.testing.assert_allclose(o.pn_volumes().sum(), o.volumes().sum(), rtol=1e-14)
 
 
-@pytest.mark.parametrize("which", ["rn", "pn"])
+@pytest.mark.parametrize("which", ["rn", "pn", "pn-stretched"])
 def test_constant_symmetry_conservation(oracle_mod, which):
-    m = mesh(7, 8, 10)
+    m = phi_stretched(mesh(7, 8, 10)) if which == "pn-stretched" else mesh(7, 8, 10)
+    which = which[:2]
     o = oracle_mod.Oracle(m, 1, 1)
     sh = o.rn_shape if which == "rn" else o.shape
     ap = o.rn_apply if which == "rn" else o.pn_apply
@@ -113,11 +127,14 @@ def test_rn_mms_second_order(oracle_mod):
     assert min(orders(e2)) > 1.8 and min(orders(em)) > 1.7, (e2, em)
 
 
-def test_pn_mms_second_order(oracle_mod):
-    """C1's manufactured solution at the phi nodes (rC, tC, pF_k)."""
+@pytest.mark.parametrize("stretch", [False, True])
+def test_pn_mms_second_order(oracle_mod, stretch):
+    """C1's manufactured solution at the phi nodes (rC, tC, pF_k); also on a
+    non-uniform phi mesh"""
     e2 = []
     for n in (8, 16, 32):
         m = mesh(n, n + n // 2, 2 * n, R=4.0)
+        m = phi_stretched(m) if stretch else m
         o = oracle_mod.Oracle(m, 0, 0)
         R, T, P = np.meshgrid(m.rC, m.tC, m.pF[:-1], indexing="ij")
         f = W.mms_forcing(R, T, P)[None]
