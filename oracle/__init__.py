@@ -410,6 +410,38 @@ class Oracle:
         return rc, x, iters.value, relres.value, hist[: iters.value + 1]
 
 
+PLACE_CELL, PLACE_THETA_NODE, PLACE_R_NODE, PLACE_PHI_NODE = 0, 1, 2, 3
+
+
+def stacked_pcg(blocks, tol, maxit):
+    """ONE Jacobi-PCG on the stacked vector of several placed operators
+    (NEXT-2, reading R34: MAS's viscosity step with v_r at r nodes, v_theta at
+    theta nodes, v_phi at phi nodes; mas_ref_stacked_pcg_solve).  blocks: a
+    list of (Oracle, placement, kappa, c, f, x0), c may be None; f and x0 of
+    shape (ncomp,) + the placement's shape.  Returns (status, [x_b],
+    iters, relres, res_hist[:iters+1])."""
+    n = len(blocks)
+    grids = (C.POINTER(_Grid) * n)(*[C.pointer(b[0].g) for b in blocks])
+    pl = (C.c_int * n)(*[int(b[1]) for b in blocks])
+    keep = []
+    ncomp, kap, cc, ff, xx = [], [], [], [], []
+    for o, place, kappa, c, f, x0 in blocks:
+        kappa, c, f = _f64(kappa), _f64(c), _f64(f)
+        x = _f64(x0).copy()
+        keep += [kappa, c, f, x]
+        ncomp.append(f.size // kappa.size)
+        kap.append(_p(kappa)); cc.append(_p(c)); ff.append(_p(f)); xx.append(x)
+    iters, relres = C.c_int(), C.c_double()
+    hist = np.zeros(maxit + 1)
+    VP = C.c_void_p * n
+    rc = lib().mas_ref_stacked_pcg_solve(
+        n, grids, pl, (C.c_int * n)(*ncomp), VP(*kap), VP(*cc), VP(*ff), VP(*[_p(x) for x in xx]),
+        C.c_double(tol), maxit, C.byref(iters), C.byref(relres), _p(hist))
+    if rc not in (OK, NOT_CONVERGED, ERR_BREAKDOWN):
+        raise RuntimeError(f"oracle returned {rc}")
+    return rc, xx, iters.value, relres.value, hist[: iters.value + 1]
+
+
 def partition(nr: int, nranks: int, rank: int):
     i0, nl = C.c_int(), C.c_int()
     lib().mas_ref_partition(nr, nranks, rank, C.byref(i0), C.byref(nl))

@@ -1751,3 +1751,157 @@ int mas_ref_pn_dirichlet_rhs(const mas_ref_grid* g, int ncomp, const double* kap
     free(pF); free(pC);
     return rc;
 }
+
+/* ---------------------------------------------------------------------------
+ * Stacked PCG over several placed operators (NEXT-2, reading R34).
+ * MAS solves the viscous step for the velocity VECTOR, each component at its
+ * staggered location ("staggered spherical grid"; the survey's R13
+ * takes one PCG on the stacked vector with the summed inner product).  With
+ * the components at different locations the operator is block-diagonal: block
+ * b is the placed operator of its location (R1-R16 on the cell centres, R29
+ * theta nodes, R32 r nodes, R33 phi nodes) with its own D, V and arrays.  The
+ * loop is pcg_core's, line for line; every inner product is the sum over the
+ * blocks (in block order) of the block's V-weighted one.
+ * ------------------------------------------------------------------------- */
+static size_t stk_cells(const mas_ref_grid* g, int pl) {
+    switch (pl) {
+    case MAS_REF_PLACE_THETA_NODE: return (size_t)g->nr * (g->nt + 1) * g->np;
+    case MAS_REF_PLACE_R_NODE: return (size_t)(g->nr - 1) * g->nt * g->np;
+    default: return (size_t)g->nr * g->nt * g->np;
+    }
+}
+static int stk_apply(const mas_ref_grid* g, int pl, int ncomp, const double* kappa, const double* c,
+                     const double* x, double* y) {
+    switch (pl) {
+    case MAS_REF_PLACE_CELL: return mas_ref_op_apply(g, ncomp, kappa, c, x, y);
+    case MAS_REF_PLACE_THETA_NODE: return mas_ref_tn_apply(g, ncomp, kappa, c, x, y);
+    case MAS_REF_PLACE_R_NODE: return mas_ref_rn_apply(g, ncomp, kappa, c, x, y);
+    case MAS_REF_PLACE_PHI_NODE: return mas_ref_pn_apply(g, ncomp, kappa, c, x, y);
+    default: return MAS_REF_ERR_ARG;
+    }
+}
+static int stk_diag(const mas_ref_grid* g, int pl, const double* kappa, const double* c, double* D) {
+    switch (pl) {
+    case MAS_REF_PLACE_CELL: return mas_ref_op_diag(g, kappa, c, D);
+    case MAS_REF_PLACE_THETA_NODE: return mas_ref_tn_diag(g, kappa, c, D);
+    case MAS_REF_PLACE_R_NODE: return mas_ref_rn_diag(g, kappa, c, D);
+    case MAS_REF_PLACE_PHI_NODE: return mas_ref_pn_diag(g, kappa, c, D);
+    default: return MAS_REF_ERR_ARG;
+    }
+}
+static int stk_volumes(const mas_ref_grid* g, int pl, double* V) {
+    switch (pl) {
+    case MAS_REF_PLACE_CELL: return mas_ref_volumes(g, V);
+    case MAS_REF_PLACE_THETA_NODE: return mas_ref_tn_volumes(g, V);
+    case MAS_REF_PLACE_R_NODE: return mas_ref_rn_volumes(g, V);
+    case MAS_REF_PLACE_PHI_NODE: return mas_ref_pn_volumes(g, V);
+    default: return MAS_REF_ERR_ARG;
+    }
+}
+/* sum over the blocks of sum_m sum_P V_P a_m,P b_m,P (per block: per
+ * component, per r-plane partial sums, as dot_planes) */
+static double stk_dot(int nblk, const mas_ref_grid* const* g, const int* pl, const int* ncomp,
+                      double* const* V, double* const* a, double* const* b) {
+    double s = 0.0;
+    int q, m, i;
+    for (q = 0; q < nblk; q++) {
+        const size_t N = stk_cells(g[q], pl[q]);
+        const int nplanes = pl[q] == MAS_REF_PLACE_R_NODE ? g[q]->nr - 1 : g[q]->nr;
+        const size_t plane = N / (size_t)nplanes;
+        double sb = 0.0;
+        for (m = 0; m < ncomp[q]; m++)
+            for (i = 0; i < nplanes; i++) {
+                double ps = 0.0;
+                size_t e;
+                for (e = 0; e < plane; e++) {
+                    const size_t P = (size_t)i * plane + e;
+                    ps += V[q][P] * a[q][(size_t)m * N + P] * b[q][(size_t)m * N + P];
+                }
+                sb += ps;
+            }
+        s += sb;
+    }
+    return s;
+}
+
+int mas_ref_stacked_pcg_solve(int nblk, const mas_ref_grid* const* g, const int* pl,
+                              const int* ncomp, const double* const* kappa, const double* const* c,
+                              const double* const* f, double* const* x, double tol, int maxit,
+                              int* iters, double* relres, double* res_hist) {
+    double *V[MAS_REF_MAX_STACK] = {0}, *D[MAS_REF_MAX_STACK] = {0}, *r[MAS_REF_MAX_STACK] = {0},
+           *z[MAS_REF_MAX_STACK] = {0}, *p[MAS_REF_MAX_STACK] = {0}, *q[MAS_REF_MAX_STACK] = {0};
+    double* fc[MAS_REF_MAX_STACK];
+    size_t N[MAS_REF_MAX_STACK];
+    double bn, rn, rho, sigma, alpha, rho_new, beta;
+    int k, b, m, status = MAS_REF_NOT_CONVERGED;
+    size_t e;
+    if (nblk < 1 || nblk > MAS_REF_MAX_STACK || !g || !pl || !ncomp || !kappa || !c || !f || !x ||
+        !iters || !relres || maxit < 0 || !(tol >= 0.0))
+        return MAS_REF_ERR_ARG;
+    for (b = 0; b < nblk; b++) {
+        if (!g[b] || !kappa[b] || !f[b] || !x[b] || ncomp[b] < 1 || pl[b] < MAS_REF_PLACE_CELL ||
+            pl[b] > MAS_REF_PLACE_PHI_NODE || (pl[b] == MAS_REF_PLACE_R_NODE && g[b]->nr < 2))
+            return MAS_REF_ERR_ARG;
+        N[b] = stk_cells(g[b], pl[b]);
+        fc[b] = (double*)f[b];
+    }
+    for (b = 0; b < nblk; b++) {
+        const size_t n = N[b] * ncomp[b];
+        V[b] = malloc(sizeof(double) * N[b]);
+        D[b] = malloc(sizeof(double) * N[b]);
+        r[b] = malloc(sizeof(double) * n);
+        z[b] = malloc(sizeof(double) * n);
+        p[b] = malloc(sizeof(double) * n);
+        q[b] = malloc(sizeof(double) * n);
+        if (!V[b] || !D[b] || !r[b] || !z[b] || !p[b] || !q[b] || stk_volumes(g[b], pl[b], V[b]) ||
+            stk_diag(g[b], pl[b], kappa[b], c[b], D[b])) {
+            status = MAS_REF_ERR_ARG; goto done;
+        }
+    }
+    bn = sqrt(stk_dot(nblk, g, pl, ncomp, V, fc, fc));
+    if (bn == 0.0) {
+        for (b = 0; b < nblk; b++)
+            for (e = 0; e < N[b] * ncomp[b]; e++) x[b][e] = 0.0;
+        *iters = 0; *relres = 0.0;
+        if (res_hist) res_hist[0] = 0.0;
+        status = MAS_REF_OK; goto done;
+    }
+    for (b = 0; b < nblk; b++) {                                 /* r = f - L x */
+        stk_apply(g[b], pl[b], ncomp[b], kappa[b], c[b], x[b], r[b]);
+        for (e = 0; e < N[b] * ncomp[b]; e++) r[b][e] = f[b][e] - r[b][e];
+    }
+    rn = sqrt(stk_dot(nblk, g, pl, ncomp, V, r, r));
+    if (res_hist) res_hist[0] = rn;
+    if (rn <= tol * bn) { *iters = 0; *relres = rn / bn; status = MAS_REF_OK; goto done; }
+    for (b = 0; b < nblk; b++) {                                 /* z = D^-1 r, p = z */
+        for (m = 0; m < ncomp[b]; m++)
+            for (e = 0; e < N[b]; e++) z[b][m * N[b] + e] = r[b][m * N[b] + e] / D[b][e];
+        memcpy(p[b], z[b], sizeof(double) * N[b] * ncomp[b]);
+    }
+    rho = stk_dot(nblk, g, pl, ncomp, V, r, z);
+    for (k = 1; k <= maxit; k++) {
+        for (b = 0; b < nblk; b++) stk_apply(g[b], pl[b], ncomp[b], kappa[b], c[b], p[b], q[b]);
+        sigma = stk_dot(nblk, g, pl, ncomp, V, p, q);
+        if (!(sigma > 0.0) || !isfinite(sigma)) {
+            *iters = k; *relres = rn / bn; status = MAS_REF_ERR_BREAKDOWN; goto done;
+        }
+        alpha = rho / sigma;
+        for (b = 0; b < nblk; b++)
+            for (e = 0; e < N[b] * ncomp[b]; e++) { x[b][e] += alpha * p[b][e]; r[b][e] -= alpha * q[b][e]; }
+        rn = sqrt(stk_dot(nblk, g, pl, ncomp, V, r, r));
+        if (res_hist) res_hist[k] = rn;
+        if (rn <= tol * bn) { *iters = k; *relres = rn / bn; status = MAS_REF_OK; goto done; }
+        for (b = 0; b < nblk; b++)
+            for (m = 0; m < ncomp[b]; m++)
+                for (e = 0; e < N[b]; e++) z[b][m * N[b] + e] = r[b][m * N[b] + e] / D[b][e];
+        rho_new = stk_dot(nblk, g, pl, ncomp, V, r, z);
+        beta = rho_new / rho;
+        rho = rho_new;
+        for (b = 0; b < nblk; b++)
+            for (e = 0; e < N[b] * ncomp[b]; e++) p[b][e] = z[b][e] + beta * p[b][e];
+    }
+    *iters = maxit; *relres = rn / bn; status = MAS_REF_NOT_CONVERGED;
+done:
+    for (b = 0; b < nblk; b++) { free(V[b]); free(D[b]); free(r[b]); free(z[b]); free(p[b]); free(q[b]); }
+    return status;
+}

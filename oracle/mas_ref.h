@@ -202,4 +202,21 @@ int mas_ref_rn_pcg_solve(const mas_ref_grid* g, int ncomp, const double* kappa, 
                          const double* f, double* x, double tol, int maxit, int* iters,
                          double* relres, double* res_hist);
 
+/* Stacked PCG over several placed operators (NEXT-2, reading R34,
+ * mas_ref.c): MAS's viscosity solve on the staggered mesh -- v_r at r nodes,
+ * v_theta at theta nodes, v_phi at phi nodes -- as ONE Jacobi-PCG on the
+ * stacked vector (block-diagonal operator, the sum of the blocks' V-weighted
+ * inner products).  Block b: grid g[b] (its mesh and r-boundary conditions),
+ * placement[b] (MAS_REF_PLACE_*), ncomp[b], kappa[b], c[b] (may be NULL),
+ * f[b], x[b] (in: x0, out: the solution). */
+#define MAS_REF_PLACE_CELL 0
+#define MAS_REF_PLACE_THETA_NODE 1
+#define MAS_REF_PLACE_R_NODE 2
+#define MAS_REF_PLACE_PHI_NODE 3
+#define MAS_REF_MAX_STACK 8
+int mas_ref_stacked_pcg_solve(int nblk, const mas_ref_grid* const* g, const int* placement,
+                              const int* ncomp, const double* const* kappa, const double* const* c,
+                              const double* const* f, double* const* x, double tol, int maxit,
+                              int* iters, double* relres, double* res_hist);
+
 #endif
