@@ -54,6 +54,7 @@ extern "C" {
 
 typedef struct mas_grid mas_grid_t;
 typedef struct mas_op mas_op_t;
+typedef struct mas_stack mas_stack_t;
 
 typedef enum {
     MAS_OK = 0,
@@ -380,6 +381,32 @@ MAS_API mas_status_t mas_op_aniso_time(const mas_op_t* op, double* ms);
  * Errors: MAS_ERR_ARG on a null pointer or a grid with ptheta > 1. */
 MAS_API mas_status_t mas_op_radial_sums(const mas_op_t* op, const double* x, const double* w,
                                         double* out, cudaStream_t stream);
+
+/* Stacked solve (reading R34 in DESIGN.md §3.9):
+ * ONE Jacobi-PCG on the stacked vector of several operators, the block-
+ * diagonal operator diag(L_1, .., L_n) with the summed inner product
+ * <a,b> = sum_b <a_b, b_b>_V of the blocks.  MAS solves its viscous step for
+ * the velocity vector with each component at its own staggered location
+ * (P:208-209): v_r at r nodes (MAS_PLACE_R_NODE), v_theta at theta nodes
+ * (MAS_PLACE_THETA_NODE), v_phi at phi nodes (MAS_PLACE_PHI_NODE), each its
+ * own mas_op_t (own kappa, c, boundary conditions and array shape); the
+ * curvature terms of R31 go into each block's c.  alpha, beta and the stop
+ * test ||r||_V <= tol ||rhs||_V are those of the stacked vector.
+ *   mas_stack_create: ops[0..nops-1], 1 <= nops <= 8, distinct, each on one
+ *     GPU without a mas_dist_t, no P2P, no single-reduction loop, no
+ *     field-aligned term (MAS_ERR_ARG otherwise).  The stack keeps the op
+ *     pointers (not the ops): destroy the stack before its ops.
+ *   mas_stack_solve: rhs[b], x[b] DEVICE arrays of op b's shape
+ *     ([comp][nl][nt][np] of its placement); x in = x0, out = solution;
+ *     tol, maxit, iters, relres, res_hist as mas_pcg_solve (the stacked
+ *     residual).  Runs on `stream` (every op's work goes there; the single-GPU
+ *     CUDA-graph loop with one k_stack_sum node after each kernel round).
+ *     Blocks until done.  The ops' own solve state is overwritten. */
+MAS_API mas_status_t mas_stack_create(mas_op_t* const* ops, int nops, mas_stack_t** out);
+MAS_API mas_status_t mas_stack_solve(mas_stack_t* stack, const double* const* rhs, double* const* x,
+                                     double tol, int maxit, int* iters, double* relres,
+                                     double* res_hist, cudaStream_t stream);
+MAS_API mas_status_t mas_stack_destroy(mas_stack_t* stack);
 
 MAS_API mas_status_t mas_op_destroy(mas_op_t* op);
 

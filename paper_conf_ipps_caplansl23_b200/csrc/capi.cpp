@@ -9,6 +9,7 @@
 #include <cuda_runtime.h>
 
 #include <cmath>
+#include <cstddef>
 #include <cstdlib>
 #include <cstring>
 #include <functional>
@@ -2008,6 +2009,284 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
         op->prof_b_ms = n ? sb / n : 0.0;
     }
     if (hx) CU(cudaMemcpy(x, xd, bytes, cudaMemcpyDeviceToHost));
+    return (mas_status_t)fin.status;
+}
+
+// ---------------------------------------------------------------------------
+// stacked solve: one PCG on the stacked vector of several operators (NEXT-2,
+// reading R34).  Each block runs its own kernels A and B on
+// its own PcgState exactly as a rank of the r-slab NCCL loop does; where that
+// loop allreduces the partial sums over the ranks, k_stack_sum sums them over
+// the blocks (in block order) and writes the sum back to every block's state.
+// Every block then takes the same alpha, beta and stop decision.
+// ---------------------------------------------------------------------------
+static_assert(offsetof(PcgState, pend_sigma) == 0 && offsetof(PcgState, pend_rho) == 8 &&
+                  offsetof(PcgState, pend_rr) == 16 && offsetof(PcgState, pend_ff) == 24,
+              "k_stack_sum offsets (0 sigma; 1 rho, 2 rr, 3 ff)");
+}  // extern "C"
+
+struct mas_stack {
+    std::vector<mas_op*> ops;
+    cudaGraphExec_t gexec = nullptr;   // the loop graph (iteration 1, then the while node)
+    std::vector<const double*> g_x, g_hist;
+    cudaStream_t cap = nullptr;
+    cudaEvent_t ev[2] = {nullptr, nullptr};
+};
+
+extern "C" {
+
+static StackStates stack_states(const mas_stack* sk) {
+    StackStates ss{};
+    ss.n = (int)sk->ops.size();
+    for (int m = 0; m < ss.n; m++) ss.st[m] = sk->ops[m]->st;
+    return ss;
+}
+
+// iteration k of every block: kernels A, the sigma sum, [q's pole rows,]
+// kernels B, the rho / ||r||^2 sum
+static cudaError_t stack_iteration(const mas_stack* sk, std::vector<StencilArgs>& a,
+                                   std::vector<StreamArgs>& b, int k, bool first, bool with_b,
+                                   cudaStream_t s) {
+    const StackStates ss = stack_states(sk);
+    cudaError_t e = cudaSuccess;
+    for (size_t m = 0; m < sk->ops.size() && e == cudaSuccess; m++) {
+        const mas_op* op = sk->ops[m];
+        a[m].pold = pold_halo(op, k);
+        a[m].tpold = pold_trows(op, k);
+        a[m].pnew = op->p[k & 1];
+        e = launch_stencil(MODE_PCGA, op->ncomp, a[m], s, first);
+    }
+    if (e == cudaSuccess) e = launch_stack_sum(ss, 0, 1, s);  // sigma_k
+    if (!with_b) return e;
+    for (size_t m = 0; m < sk->ops.size() && e == cudaSuccess; m++) {
+        const mas_op* op = sk->ops[m];
+        if (op->tnode) e = launch_pole_avg(op->geo, op->ncomp, op->q, nullptr, 0, op->geo.nl, s);
+        if (e == cudaSuccess) e = launch_pcg_b(b[m], op->b_blocks, s);
+    }
+    if (e == cudaSuccess) e = launch_stack_sum(ss, 1, 2, s);  // rho_k, ||r_k||^2
+    return e;
+}
+
+// the single-GPU loop graph of a stack (loop_graph's structure): iteration 1
+// as a chain of kernel nodes, then a device-side while node whose body runs
+// iterations 2k and 2k+1; rebuilt when an x or history buffer moves
+static mas_status_t stack_graph(mas_stack* sk, std::vector<StencilArgs> a, std::vector<StreamArgs> b) {
+    const size_t n = sk->ops.size();
+    bool same = sk->gexec && sk->g_x.size() == n;
+    for (size_t m = 0; same && m < n; m++) same = sk->g_x[m] == a[m].x && sk->g_hist[m] == a[m].rho_hist;
+    if (same) return MAS_OK;
+    if (sk->gexec) {
+        cudaGraphExecDestroy(sk->gexec);
+        sk->gexec = nullptr;
+    }
+    if (!sk->cap) CU(cudaStreamCreateWithFlags(&sk->cap, cudaStreamNonBlocking));
+    cudaGraph_t g;
+    CU(cudaGraphCreate(&g, 0));
+    cudaError_t e = cudaStreamBeginCaptureToGraph(sk->cap, g, nullptr, nullptr, 0, cudaStreamCaptureModeThreadLocal);
+    if (e == cudaSuccess) {
+        e = stack_iteration(sk, a, b, 1, true, true, sk->cap);
+        cudaGraph_t out = g;
+        const cudaError_t e2 = cudaStreamEndCapture(sk->cap, &out);
+        if (e == cudaSuccess) e = e2;
+    }
+    std::vector<cudaGraphNode_t> deps;
+    size_t nn = 0;
+    if (e == cudaSuccess) e = cudaGraphGetNodes(g, nullptr, &nn);
+    std::vector<cudaGraphNode_t> nodes(nn);
+    if (e == cudaSuccess && nn) e = cudaGraphGetNodes(g, nodes.data(), &nn);
+    for (size_t i = 0; i < nn && e == cudaSuccess; i++) {
+        size_t nd = 0;
+        e = cudaGraphNodeGetDependentNodes(nodes[i], nullptr, &nd);
+        if (e == cudaSuccess && nd == 0) deps.push_back(nodes[i]);
+    }
+    if (e == cudaSuccess && deps.size() != 1) e = cudaErrorInvalidValue;
+    cudaGraphConditionalHandle h;
+    if (e == cudaSuccess) e = cudaGraphConditionalHandleCreate(&h, g, 1, cudaGraphCondAssignDefault);
+    cudaGraphNodeParams p = {};
+    p.type = cudaGraphNodeTypeConditional;
+    p.conditional.handle = h;
+    p.conditional.type = cudaGraphCondTypeWhile;
+    p.conditional.size = 1;
+    cudaGraphNode_t node;
+    if (e == cudaSuccess) e = cudaGraphAddNode(&node, g, deps.data(), deps.size(), &p);
+    if (e == cudaSuccess) {
+        cudaGraph_t body = p.conditional.phGraph_out[0];
+        e = cudaStreamBeginCaptureToGraph(sk->cap, body, nullptr, nullptr, 0, cudaStreamCaptureModeThreadLocal);
+        if (e == cudaSuccess) {
+            for (size_t m = 0; m < n; m++) a[m].cond = b[m].cond = (unsigned long long)h;
+            for (int kk = 2; kk <= 3 && e == cudaSuccess; kk++) e = stack_iteration(sk, a, b, kk, false, true, sk->cap);
+            cudaGraph_t out = body;
+            const cudaError_t e2 = cudaStreamEndCapture(sk->cap, &out);
+            if (e == cudaSuccess) e = e2;
+        }
+    }
+    if (e == cudaSuccess) e = cudaGraphInstantiate(&sk->gexec, g, 0);
+    cudaGraphDestroy(g);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        sk->gexec = nullptr;
+        set_last_error(std::string("stack loop graph: ") + cudaGetErrorString(e));
+        return MAS_ERR_CUDA;
+    }
+    sk->g_x.resize(n);
+    sk->g_hist.resize(n);
+    for (size_t m = 0; m < n; m++) {
+        sk->g_x[m] = a[m].x;
+        sk->g_hist[m] = a[m].rho_hist;
+    }
+    return MAS_OK;
+}
+
+mas_status_t mas_stack_create(mas_op_t* const* ops, int nops, mas_stack_t** out) {
+    if (!out) return arg_error("null out");
+    *out = nullptr;
+    if (!ops || nops < 1 || nops > kMaxStack) return arg_error("need 1 <= nops <= 8 operators");
+    for (int m = 0; m < nops; m++) {
+        const mas_op* op = ops[m];
+        if (!op) return arg_error("null operator");
+        for (int q = 0; q < m; q++)
+            if (ops[q] == op) return arg_error("the same operator twice in a stack");
+        if (op->g->comm) return arg_error("stacked solve: one GPU without a mas_dist_t");
+        if (op->p2p) return arg_error("stacked solve: no P2P transport");
+        if (op->cg1) return arg_error("stacked solve: the two-kernel loop (single reduction is on)");
+        if (op->aniso) return arg_error("stacked solve: isotropic operators (no mas_op_set_aniso)");
+    }
+    mas_stack* sk = new mas_stack;
+    sk->ops.assign(ops, ops + nops);
+    for (int q = 0; q < 2; q++)
+        if (cudaEventCreateWithFlags(&sk->ev[q], cudaEventDisableTiming) != cudaSuccess) {
+            cudaGetLastError();
+            mas_stack_destroy(sk);
+            set_last_error("stack events");
+            return MAS_ERR_CUDA;
+        }
+    *out = sk;
+    return MAS_OK;
+}
+
+mas_status_t mas_stack_destroy(mas_stack_t* sk) {
+    if (!sk) return MAS_OK;
+    if (sk->gexec) cudaGraphExecDestroy(sk->gexec);
+    if (sk->cap) cudaStreamDestroy(sk->cap);
+    for (cudaEvent_t e : sk->ev)
+        if (e) cudaEventDestroy(e);
+    delete sk;
+    return MAS_OK;
+}
+
+mas_status_t mas_stack_solve(mas_stack_t* sk, const double* const* rhs, double* const* x, double tol,
+                             int maxit, int* iters, double* relres, double* res_hist, cudaStream_t s) {
+    NvtxRange nvtx("mas_stack_solve");
+    if (!sk || !rhs || !x || !iters || !relres) return arg_error("null argument");
+    if (!(tol >= 0.0) || maxit < 0) return arg_error("need tol >= 0 and maxit >= 0");
+    const size_t n = sk->ops.size();
+    for (size_t m = 0; m < n; m++) {
+        if (!rhs[m] || !x[m]) return arg_error("null rhs or x");
+        if (!is_device_ptr(rhs[m]) || !is_device_ptr(x[m])) return arg_error("stacked solve: device arrays");
+    }
+    const StackStates ss = stack_states(sk);
+    std::vector<StencilArgs> a(n);
+    std::vector<StreamArgs> b(n);
+    // init: every block's state, r = f - L x0 and its three partial sums
+    for (size_t m = 0; m < n; m++) {
+        mas_op* op = sk->ops[m];
+        ST(ensure_hist(op, maxit));
+        op->launches = 0;
+        PcgState init{};
+        init.tol = tol;
+        init.maxit = maxit;
+        init.k = 1;
+        init.status = MAS_NOT_CONVERGED;
+        CU(cudaMemcpyAsync(op->st, &init, sizeof(init), cudaMemcpyHostToDevice, s));
+        *op->host_flag = 0;
+        const int nc = op->ncomp;
+        double* xd = x[m];
+        ST(pole_pass(op, xd, nc, s));
+        StencilArgs& A = a[m];
+        A.g = op->geo;
+        A.chunk = op->chunk;
+        A.u = halo_of(op, xd, op->xg, nc);
+        A.kappa = halo_of(op, op->kappa, op->kg, 1);
+        A.dinv = halo_of(op, op->dinv, op->dg, 1);
+        A.tu = packed_rows(op, op->xgt, nc);
+        A.tkappa = packed_rows(op, op->kgt, 1);
+        A.tdinv = packed_rows(op, op->dgt, 1);
+        A.c = op->c;
+        A.curv = op->curv;
+        A.f = rhs[m];
+        A.out = op->r;
+        A.st = op->st;
+        A.rho_hist = op->hist;
+        A.sigma_hist = op->hist + op->hist_cap;
+        A.rr_hist = op->hist + 2 * op->hist_cap;
+        A.scr = op->scr;
+        A.host_flag = op->host_flag_dev;
+        CU(launch_stencil(MODE_RESID, nc, A, s));
+        if (op->tnode) {  // the caps' residuals, then the three sums again
+            ST(pole_pass(op, op->r, nc, s));
+            CU(launch_init_dots(op->geo, nc, rhs[m], op->r, op->dinv, op->scr, op->st, op->b_blocks, s));
+        }
+        // the iteration arguments (kernel A: p from r; kernel B)
+        A.u = r_halo(op);
+        A.tu = r_trows(op);
+        A.out = op->q;
+        A.x = xd;
+        A.f = nullptr;
+        StreamArgs& B = b[m];
+        B.g = op->geo;
+        B.ncomp = nc;
+        B.r = op->r;
+        B.q = op->q;
+        B.dinv = op->dinv;
+        B.st = op->st;
+        B.rho_hist = A.rho_hist;
+        B.sigma_hist = A.sigma_hist;
+        B.rr_hist = A.rr_hist;
+        B.scr = op->scr;
+        B.host_flag = op->host_flag_dev;
+    }
+    CU(launch_stack_sum(ss, 1, 3, s));  // rho_0, ||r_0||^2, ||f||^2 of the stacked vector
+    bool graph = true;
+    for (const mas_op* op : sk->ops) graph = graph && op->use_graph && !op->prof;
+    if (graph) {
+        ST(stack_graph(sk, a, b));
+        CU(cudaGraphLaunch(sk->gexec, s));
+    }
+    for (int k = 1; !graph && k <= maxit + 1; k++) {
+        CU(stack_iteration(sk, a, b, k, k == 1, k <= maxit, s));
+        CU(cudaEventRecord(sk->ev[k & 1], s));
+        if (k >= 2) {  // stop once block 0 reports a decision at or before iteration k-1
+            CU(cudaEventSynchronize(sk->ev[(k - 1) & 1]));
+            const int flag = *(volatile int*)sk->ops[0]->host_flag;
+            if (flag > 0 && flag <= k - 1) break;
+        }
+    }
+    CU(cudaStreamSynchronize(s));
+    PcgState fin{};
+    for (size_t m = 0; m < n; m++) {
+        PcgState f{};
+        CU(cudaMemcpy(&f, sk->ops[m]->st, sizeof(f), cudaMemcpyDeviceToHost));
+        if (!f.stopped) {
+            set_last_error("internal: stacked loop ended without a stop decision");
+            return MAS_ERR_CUDA;
+        }
+        if (m == 0) {
+            fin = f;
+        } else if (f.iters != fin.iters || f.status != fin.status) {
+            set_last_error("internal: the blocks of a stack took different stop decisions");
+            return MAS_ERR_CUDA;
+        }
+    }
+    *iters = fin.iters;
+    *relres = fin.relres;
+    if (res_hist) {
+        const int nh = fin.status == MAS_ERR_BREAKDOWN ? fin.iters : fin.iters + 1;
+        std::vector<double> rr(nh);
+        const mas_op* op0 = sk->ops[0];
+        CU(cudaMemcpy(rr.data(), op0->hist + 2 * op0->hist_cap, rr.size() * sizeof(double),
+                      cudaMemcpyDeviceToHost));
+        for (int k = 0; k < nh; k++) res_hist[k] = std::sqrt(rr[k]);
+    }
     return (mas_status_t)fin.status;
 }
 

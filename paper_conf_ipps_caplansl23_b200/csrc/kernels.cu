@@ -1549,6 +1549,24 @@ cudaError_t launch_stencil(int mode, int ncomp, const StencilArgs& a, cudaStream
     return cudaErrorInvalidValue;
 }
 
+// the per-block partial sums of a stacked solve (mas_stack_solve) into their
+// sum, written back to every block's PcgState: the "allreduce" over the blocks
+// of the stacked vector (R34).  Offsets in doubles: 0 sigma;
+// 1..3 rho, rr, ff (PcgState layout)
+__global__ void k_stack_sum(const StackStates s, int off, int cnt) {
+    const int t = threadIdx.x;
+    if (t >= cnt) return;
+    double v = 0.0;
+    for (int m = 0; m < s.n; m++) v += __ldcg(reinterpret_cast<const double*>(s.st[m]) + off + t);
+    for (int m = 0; m < s.n; m++) reinterpret_cast<double*>(s.st[m])[off + t] = v;
+}
+
+cudaError_t launch_stack_sum(const StackStates& s, int off, int cnt, cudaStream_t stream) {
+    if (s.n < 1 || s.n > kMaxStack || cnt < 1 || cnt > 32) return cudaErrorInvalidValue;
+    k_stack_sum<<<1, 32, 0, stream>>>(s, off, cnt);
+    return cudaGetLastError();
+}
+
 cudaError_t launch_pcg_b(const StreamArgs& a, int nblocks, cudaStream_t s) {
     if (a.ncomp == 1)
         k_pcg_b<1><<<nblocks, kThreads, 0, s>>>(a);

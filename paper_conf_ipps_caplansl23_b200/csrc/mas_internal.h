@@ -212,6 +212,15 @@ int stencil_blocks(const Geo& g, int chunk);
 cudaError_t launch_stencil(int mode, int ncomp, const StencilArgs& a, cudaStream_t s,
                            bool first = false);
 cudaError_t launch_pcg_b(const StreamArgs& a, int nblocks, cudaStream_t s);
+// stacked PCG over several operators (mas_stack_solve, NEXT-2 R34): the
+// PcgState of every block; k_stack_sum replaces the doubles [off, off+cnt) of
+// each by their sum over the blocks (block order: deterministic)
+constexpr int kMaxStack = 8;
+struct StackStates {
+    PcgState* st[kMaxStack];
+    int n;
+};
+cudaError_t launch_stack_sum(const StackStates& s, int off, int cnt, cudaStream_t stream);
 // theta-node placement (NEXT-2): average the pole rows (local rows 0, g.nt-1)
 // of planes [plane_lo, plane_lo + nplanes) of every component over phi with
 // dp weights (dinv != nullptr: also dinv = 1 / average, ncomp = 1)

@@ -30,7 +30,8 @@ ABI_SYMBOLS = ("mas_comm_unique_id", "mas_partition", "mas_grid_create", "mas_gr
                "mas_grid_local_extent_2d",
                "mas_op_set_profiling", "mas_op_kernel_times", "mas_op_set_aniso",
                "mas_op_aniso_time", "mas_op_radial_sums", "mas_op_comm_bench", "mas_op_set_single_reduction", "mas_op_set_curvature", "mas_op_kernel_bench", "mas_op_aniso_fused",
-               "mas_op_single_reduction", "mas_op_destroy", "mas_status_string", "mas_last_error", "mas_version")
+               "mas_op_single_reduction", "mas_stack_create", "mas_stack_solve", "mas_stack_destroy",
+               "mas_op_destroy", "mas_status_string", "mas_last_error", "mas_version")
 
 
 class MasError(RuntimeError):
@@ -86,6 +87,9 @@ def lib() -> C.CDLL:
             "mas_op_kernel_bench": (_i, [_vp, _i, _vp, _vp, _vp, _vp]),
             "mas_op_aniso_fused": (_i, [_vp]),
             "mas_op_single_reduction": (_i, [_vp]),
+            "mas_stack_create": (_i, [_vp, _i, _vp]),
+            "mas_stack_solve": (_i, [_vp, _vp, _vp, _d, _i, _vp, _vp, _vp, _vp]),
+            "mas_stack_destroy": (_i, [_vp]),
             "mas_op_destroy": (_i, [_vp]),
             "mas_status_string": (C.c_char_p, [_i]),
             "mas_last_error": (C.c_char_p, []),
@@ -277,6 +281,34 @@ def mas_pcg_solve(op: int, rhs, x, tol: float, maxit: int, want_hist: bool = Fal
         n = it.value if s == MAS_ERR_BREAKDOWN else it.value + 1
         hist = hist[:n]
     return s, it.value, rel.value, hist
+
+
+def mas_stack_create(ops) -> int:
+    arr = (C.c_void_p * len(ops))(*ops)
+    h = C.c_void_p()
+    _check(lib().mas_stack_create(arr, len(ops), C.byref(h)), "mas_stack_create")
+    return h.value
+
+
+def mas_stack_solve(stack: int, rhs, x, tol: float, maxit: int, want_hist: bool = False, stream=None):
+    """rhs, x: one device array per block.  Returns (status, iters, relres,
+    res_hist or None) of the stacked vector."""
+    if len(rhs) != len(x):
+        raise ValueError("one rhs and one x per block")
+    R = (C.c_void_p * len(rhs))(*[_ptr(a) for a in rhs])
+    X = (C.c_void_p * len(x))(*[_ptr(a) for a in x])
+    it, rel = C.c_int(), C.c_double()
+    hist = np.zeros(maxit + 1) if want_hist else None
+    s = lib().mas_stack_solve(stack, R, X, float(tol), int(maxit), C.byref(it), C.byref(rel),
+                              hist.ctypes.data if want_hist else None, _stream(stream))
+    _check(s, "mas_stack_solve", ok=(MAS_OK, MAS_NOT_CONVERGED, MAS_ERR_BREAKDOWN))
+    if hist is not None:
+        hist = hist[:it.value if s == MAS_ERR_BREAKDOWN else it.value + 1]
+    return s, it.value, rel.value, hist
+
+
+def mas_stack_destroy(stack: int) -> None:
+    _check(lib().mas_stack_destroy(stack), "mas_stack_destroy")
 
 
 def mas_op_enable_p2p(op: int, stream=None) -> None:
@@ -499,6 +531,30 @@ class Operator:
     def close(self):
         if self.h:
             mas_op_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+class Stack:
+    """One PCG on the stacked vector of several operators (mas_stack_*; NEXT-2,
+    reading R34): e.g. MAS's viscous step with v_r, v_theta, v_phi each at its
+    staggered location.  Keeps the Operators alive; close() before them."""
+
+    def __init__(self, ops):
+        self.ops = list(ops)
+        self.h = mas_stack_create([o.h for o in self.ops])
+
+    def solve(self, rhs, x, tol, maxit, want_hist=False, stream=None):
+        return mas_stack_solve(self.h, rhs, x, tol, maxit, want_hist, stream)
+
+    def close(self):
+        if self.h:
+            mas_stack_destroy(self.h)
             self.h = None
 
     def __del__(self):
