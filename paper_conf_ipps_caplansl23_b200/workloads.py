@@ -328,6 +328,44 @@ def tnode_conduction_problem(nr=128, nt=128, np_=256, r0=1.0, r1=30.0, R=200.0, 
                    tol, maxit, extra={"dt": base.extra["dt"], "placement": "theta-node"})
 
 
+def staggered_viscosity_blocks(nr=256, nt=256, np_=512, r0=1.0, r1=30.0, R=200.0, D_max=100.0,
+                               warm=True):
+    """C3's viscosity step on the staggered mesh (NEXT-2, reading R34): v_r at
+    the r nodes (rF_i, tC, pC), i = 1..nr-1; v_theta at the theta nodes (rC,
+    tF_j, pC), j = 0..nt (pole rows one value per radius); v_phi at the phi
+    nodes (rC, tC, pF_k).  The same rho texture, nu = 1, dt and velocity
+    profile as viscosity_problem, evaluated at each component's location.
+    Returns (mesh, dt, [(placement, kappa, c, f[None], x0[None])]) with
+    placements 2 (r nodes), 1 (theta nodes), 3 (phi nodes); boundary
+    conditions DIRICHLET inner, NEUMANN outer for every block."""
+    m = stretched_mesh(nr, nt, np_, r0, r1, R)
+    grho_c = texture(m.tC, m.pC, 2)
+    rho_c = np.ascontiguousarray(np.broadcast_to(_density(m.rC[:, None, None], grho_c[None]), (nr, nt, np_)))
+    dt = D_max / _diffusion_number_scale(m, rho_c, rho_c)
+    pF = m.pF[:-1]
+    locs = [  # placement, r points, (theta, phi) points of the texture, velocity texture seed
+        (2, m.rF[1:-1], (m.tC, m.pC), 10),
+        (1, m.rC, (m.tF, m.pC), 11),
+        (3, m.rC, (m.tC, pF), 12),
+    ]
+    out = []
+    for pl, rr, (tt, pp), seed in locs:
+        g_rho = texture(m.tC, m.pC, 2, at=(tt, pp))
+        rho = _density(rr[:, None, None], g_rho[None])
+        prof = np.sin(math.pi * (rr - r0) / (r1 - r0))[:, None, None]
+        v = prof * texture(m.tC, m.pC, seed, at=(tt, pp))[None]
+        shape = (len(rr), len(tt), len(pp))
+        rho = np.ascontiguousarray(np.broadcast_to(rho, shape))
+        v = np.ascontiguousarray(np.broadcast_to(v, shape))
+        if pl == 1:
+            rho, v = replicate_poles(rho), replicate_poles(v)
+        c = rho / dt
+        f = (c * v)[None]
+        x0 = v[None].copy() if warm else np.zeros_like(f)
+        out.append((pl, rho, c, f, x0))
+    return m, dt, out
+
+
 def random_field(shape, seed=42) -> np.ndarray:
     """Matvec-parity input: U[-1,1] i.i.d."""
     return np.random.default_rng(seed).uniform(-1.0, 1.0, size=shape)
