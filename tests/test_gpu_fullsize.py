@@ -196,3 +196,38 @@ def test_fullsize_theta_nodes_vs_oracle(mp, oracle_mod):
     assert math.sqrt((V * (xg - xo) ** 2).sum() / (V * xo ** 2).sum()) <= 1e-10
     for row in (0, -1):  # one value per pole and radius
         assert np.array_equal(xg[0, :, row, :], np.broadcast_to(xg[0, :, row, :1], xg[0, :, row, :].shape))
+
+
+def test_fullsize_staggered_stack_vs_oracle(mp, oracle_mod):
+    """NEXT-2 R34 at C2's grid: C3's viscous fields on the staggered mesh
+    (v_r r nodes, v_theta theta nodes, v_phi phi nodes), one PCG on the
+    stacked vector: iterations within max(1, the oracle's envelope), x <= 1e-10
+    in the stacked V-norm."""
+    mesh, dt, blocks = W.staggered_viscosity_blocks(128, 128, 256)
+    d = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()
+    g = mp.Grid(mesh)
+    ops = [mp.Operator(g, 1, d(k), d(c), W.DIRICHLET, W.NEUMANN, placement=pl) for pl, k, c, f, x0 in blocks]
+    sk = mp.Stack(ops)
+    xs = [d(b[4]) for b in blocks]
+    tol = 1e-12
+    st, it, rel, _ = sk.solve([d(b[3]) for b in blocks], xs, tol, 20000)
+    assert st == mp.MAS_OK and rel <= tol
+    xg = [x.cpu().numpy() for x in xs]
+    o = oracle_mod.Oracle(mesh, W.DIRICHLET, W.NEUMANN)
+
+    def run(scale):
+        return oracle_mod.stacked_pcg([(o, pl, k, c, f * scale, x0) for pl, k, c, f, x0 in blocks], tol, 20000)
+
+    rc, xo, ito, _, _ = run(1.0)
+    assert rc == oracle_mod.OK
+    _, _, itp, _, _ = run(1.0 + 2.2e-16)
+    env = abs(itp - ito)
+    assert abs(it - ito) <= max(1, env), (it, ito, env)
+    V = [{1: o.tn_volumes, 2: o.rn_volumes, 3: o.pn_volumes}[b[0]]()[None] for b in blocks]
+    num = sum((v * (a - b) ** 2).sum() for v, a, b in zip(V, xg, xo))
+    den = sum((v * b ** 2).sum() for v, b in zip(V, xo))
+    assert math.sqrt(num / den) <= 1e-10
+    sk.close()
+    for op in ops:
+        op.close()
+    g.close()
