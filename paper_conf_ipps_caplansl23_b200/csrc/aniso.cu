@@ -547,8 +547,13 @@ __global__ void __launch_bounds__(WTHREADS, kAnisoBps) k_aniso(const AnisoArgs a
             const size_t qoff = (size_t)(j0 + w) * g.np + k0 + c2;
             double2 qnext = make_double2(0.0, 0.0);
 #endif
+            // 1/vr of the cell plane of the next step, loaded one step ahead
+            // (its latency sat on the cell phase's dependency chain)
+            double ivr_cur = 0.0;
             for (int n = 0; n < nst; n++) {
                 const int I = ia - 1 + n, slot = n % W_NSLOT;
+                const double ivr_here = ivr_cur;
+                if (cell_ok && n + 1 >= 2 && n + 1 < nst) ivr_cur = __ldg(a.ivr + I);
 #if !defined(MAS_ANISO_QTMA) && !defined(MAS_ANISO_QNOW)
                 const double2 qv = qnext;
                 if (n + 1 >= 2 && n + 1 < nst && cell_ok) qnext = ld2(a.out + (size_t)I * plane + qoff);
@@ -630,7 +635,7 @@ __global__ void __launch_bounds__(WTHREADS, kAnisoBps) k_aniso(const AnisoArgs a
                     const double h0a = h[WCW + 1], h0b = h[WCW + 2];
                     const double s0 = ((l0.x + l1a) + (l2.x + l3a)) - ((h3.x + h2a) + (h1.x + h0a));
                     const double s1 = ((l0.y + l1b) + (l2.y + l3b)) - ((h3.y + h2b) + (h1.y + h0b));
-                    const double ivr = __ldg(a.ivr + i);
+                    const double ivr = ivr_here;  // 1/vr of plane i = I-1
                     const double y0 = s0 * (ivr * cw0), y1 = s1 * (ivr * cw1);
 #ifdef MAS_ANISO_QTMA
                     const double2 qv = lds2(Q_of(slot) + w * WK + c2);

@@ -550,6 +550,11 @@ class Stack:
         self.h = mas_stack_create([o.h for o in self.ops])
 
     def solve(self, rhs, x, tol, maxit, want_hist=False, stream=None):
+        if len(rhs) != len(self.ops) or len(x) != len(self.ops):
+            raise ValueError("one rhs and one x per operator of the stack")
+        for o, r, xx in zip(self.ops, rhs, x):
+            _expect(r, o.ncomp * o.N, "rhs")
+            _expect(xx, o.ncomp * o.N, "x")
         return mas_stack_solve(self.h, rhs, x, tol, maxit, want_hist, stream)
 
     def close(self):
