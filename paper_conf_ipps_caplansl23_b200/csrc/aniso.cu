@@ -140,11 +140,16 @@ namespace {
 #ifndef MAS_ANISO_BPS
 #define MAS_ANISO_BPS 1
 #endif
-constexpr int WJ = MAS_ANISO_WJ;       // tile rows (one consumer warp each)
+#ifndef MAS_ANISO_RPW
+#define MAS_ANISO_RPW 1
+#endif
+constexpr int WJ = MAS_ANISO_WJ;       // tile rows
+constexpr int RPW = MAS_ANISO_RPW;     // tile rows per consumer warp (rows w + r * NCW)
 constexpr int kAnisoBps = MAS_ANISO_BPS;  // resident blocks per SM (the rings must fit)
 constexpr int rup16(int x) { return (x + 15) / 16 * 16; }  // 128-byte multiples of doubles
 constexpr int WK = 64;                 // tile columns (32 lanes x 2)
-constexpr int NCW = WJ;                // consumer warps
+constexpr int NCW = WJ / RPW;          // consumer warps
+static_assert(WJ % RPW == 0, "MAS_ANISO_RPW must divide MAS_ANISO_WJ");
 constexpr int WTHREADS = 32 * (NCW + 1);
 constexpr int WPR = WJ + 2;            // p rows: j0-1 .. j0+16
 constexpr int WPW = WK + 4;            // p row: [k0-2][k0-1][64 cells][k0+64][k0+65]
@@ -497,6 +502,166 @@ __global__ void __launch_bounds__(WTHREADS, kAnisoBps) k_aniso(const AnisoArgs a
                 fence_proxy_async();
                 __syncwarp();
                 if (lane == 0) mbar_arrive(empty0 + 8 * slot);
+            }
+#elif MAS_ANISO_RPW > 1
+            // ---- consumers, RPW rows per warp (experiment: fewer warps, RPW
+            // independent row chains per thread; V1's arithmetic row by row)
+            static_assert(WQ_SLOT > 0, "MAS_ANISO_RPW > 1 needs the out/q TMA box");
+            const int c2 = 2 * lane;
+            const bool first = k0 == 0, last = k0 + width == g.np;
+            const bool lfix = first && c2 == 0, rfix = last && c2 == width;
+            bool crow_ok[RPW], cell_ok[RPW];
+            double cw0[RPW], cw1[RPW];
+#pragma unroll
+            for (int r = 0; r < RPW; r++) {
+                const int w = warp + r * NCW;
+                crow_ok[r] = w <= height && c2 <= width;
+                cell_ok[r] = w < height && c2 < width;
+                cw0[r] = cw1[r] = 0.0;
+                if (cell_ok[r]) {
+                    const double vt = __ldg(g.vt + j0 + w);
+                    cw0[r] = 1.0 / (vt * __ldg(g.vp + k0 + c2));
+                    cw1[r] = 1.0 / (vt * __ldg(g.vp + k0 + c2 + 1));
+                }
+            }
+            int xr = -1, xc = 0;  // extra corner: row WJ / column 64
+            {
+                const int t = threadIdx.x;
+                if (height == WJ && t <= width) {
+                    xr = WJ, xc = t;
+                } else if (width == WK && t >= WK + 1 && t - (WK + 1) < min(height + 1, WJ)) {
+                    xr = t - (WK + 1), xc = WK;
+                }
+            }
+            auto corner_math = [&](double a00, double a01, double a10, double a11, double b00, double b01,
+                                   double b10, double b11, double A0, double B0, double E0, double& o0,
+                                   double& o1, double& o2, double& o3) -> double {
+                const double Dr = ((b00 - a00) + (b01 - a01)) + ((b10 - a10) + (b11 - a11));
+                const double Dt = ((a10 - a00) + (a11 - a01)) + ((b10 - b00) + (b11 - b01));
+                const double Dp = ((a01 - a00) + (a11 - a10)) + ((b01 - b00) + (b11 - b10));
+                const double sc = A0 * Dr + B0 * Dt + E0 * Dp;
+                const double A = sc * A0, B = sc * B0, E = sc * E0;
+                o0 = (A + B) + E;
+                o1 = (A + B) - E;
+                o2 = (A - B) + E;
+                o3 = (A - B) - E;
+                return sc;
+            };
+            double x0[RPW], y0[RPW], e0 = 0.0, e1 = 0.0, e2 = 0.0, e3 = 0.0;
+            double2 x12[RPW], y12[RPW];
+#pragma unroll
+            for (int r = 0; r < RPW; r++) x0[r] = y0[r] = 0.0, x12[r] = y12[r] = make_double2(0.0, 0.0);
+            double ivr_cur = 0.0;
+            for (int n = 0; n < nst; n++) {
+                const int I = ia - 1 + n, slot = n % W_NSLOT;
+                const double ivr_here = ivr_cur;
+                if (cell_ok[0] && n + 1 >= 2 && n + 1 < nst) ivr_cur = __ldg(a.ivr + I);
+                mbar_wait(full0 + 8 * slot, (n / W_NSLOT) & 1);
+                const double* p1 = P_of(slot);
+                double X0[RPW], Y0[RPW], E0 = 0.0, E1 = 0.0, E2 = 0.0, E3 = 0.0;
+                double2 X12[RPW], Y12[RPW];
+#pragma unroll
+                for (int r = 0; r < RPW; r++) {
+                    const int w = warp + r * NCW;
+                    X0[r] = Y0[r] = 0.0;
+                    X12[r] = Y12[r] = make_double2(0.0, 0.0);
+                    if (crow_ok[r]) {
+                        const double* q1 = p1 + w * WPW + c2;
+                        X0[r] = q1[1], Y0[r] = q1[WPW + 1];
+                        X12[r] = lds2(q1 + 2), Y12[r] = lds2(q1 + WPW + 2);
+                        if (lfix) X0[r] = p1[O_PL + 2 * w + 1], Y0[r] = p1[O_PL + 2 * w + 3];
+                        if (rfix) X12[r].x = p1[O_PR + 2 * w], Y12[r].x = p1[O_PR + 2 * w + 2];
+                    }
+                }
+                if (xr >= 0) {
+                    const double* q1 = p1 + xr * WPW + xc + 1;
+                    E0 = q1[0], E1 = q1[1], E2 = q1[WPW], E3 = q1[WPW + 1];
+                    if (first && xc == 0) E0 = p1[O_PL + 2 * xr + 1], E2 = p1[O_PL + 2 * xr + 3];
+                    if (last && xc == width) E1 = p1[O_PR + 2 * xr], E3 = p1[O_PR + 2 * xr + 2];
+                }
+                if (n == 0) {
+#pragma unroll
+                    for (int r = 0; r < RPW; r++) x0[r] = X0[r], y0[r] = Y0[r], x12[r] = X12[r], y12[r] = Y12[r];
+                    e0 = E0, e1 = E1, e2 = E2, e3 = E3;
+                    continue;
+                }
+                double* Cf = C_of(slot);
+#pragma unroll
+                for (int r = 0; r < RPW; r++) {
+                    const int w = warp + r * NCW;
+                    if (crow_ok[r]) {
+                        double* c0 = Cf + w * WCW + c2;
+                        double2 A0 = lds2(c0), B0 = lds2(c0 + WCA), C0 = lds2(c0 + 2 * WCA);
+                        if (rfix) {
+                            const double* CS = p1 + O_CS;
+                            A0.x = CS[2 * w], B0.x = CS[2 * (WCR + w)], C0.x = CS[2 * (2 * WCR + w)];
+                        }
+                        double o[2][4];
+                        const double s0 = corner_math(x0[r], x12[r].x, y0[r], y12[r].x, X0[r], X12[r].x, Y0[r],
+                                                      Y12[r].x, A0.x, B0.x, C0.x, o[0][0], o[0][1], o[0][2], o[0][3]);
+                        const double s1 = corner_math(x12[r].x, x12[r].y, y12[r].x, y12[r].y, X12[r].x, X12[r].y,
+                                                      Y12[r].x, Y12[r].y, A0.y, B0.y, C0.y, o[1][0], o[1][1],
+                                                      o[1][2], o[1][3]);
+#pragma unroll
+                        for (int q = 0; q < 4; q++) sts2(c0 + q * WCA, make_double2(o[0][q], o[1][q]));
+                        if (MODE == MODE_PCGA && I < ib && w < height && c2 < width) acc[0] += s0 * s0 + s1 * s1;
+                    }
+                }
+                if (xr >= 0) {
+                    double* c0 = Cf + xr * WCW + xc;
+                    double A = c0[0], B = c0[WCA], E = c0[2 * WCA];
+                    if (last && xc == width) {
+                        const double* CS = p1 + O_CS;
+                        A = CS[2 * xr], B = CS[2 * (WCR + xr)], E = CS[2 * (2 * WCR + xr)];
+                    }
+                    double o0, o1, o2, o3;
+                    corner_math(e0, e1, e2, e3, E0, E1, E2, E3, A, B, E, o0, o1, o2, o3);
+                    c0[0] = o0;
+                    c0[WCA] = o1;
+                    c0[2 * WCA] = o2;
+                    c0[3 * WCA] = o3;
+                }
+#pragma unroll
+                for (int r = 0; r < RPW; r++) x0[r] = X0[r], y0[r] = Y0[r], x12[r] = X12[r], y12[r] = Y12[r];
+                e0 = E0, e1 = E1, e2 = E2, e3 = E3;
+                consumer_sync();
+                if (n >= 2) {
+                    const int i = I - 1;
+#pragma unroll
+                    for (int r = 0; r < RPW; r++) {
+                        const int w = warp + r * NCW;
+                        if (!cell_ok[r]) continue;
+                        const double* l = C_of((n - 1) % W_NSLOT) + w * WCW + c2;
+                        const double* h = Cf + w * WCW + c2;
+                        const double2 l0 = lds2(l), l2 = lds2(l + 2 * WCA + WCW);
+                        const double2 h3 = lds2(h + 3 * WCA), h1 = lds2(h + WCA + WCW);
+                        const double l1a = l[WCA + 1], l1b = l[WCA + 2];
+                        const double l3a = l[3 * WCA + WCW + 1], l3b = l[3 * WCA + WCW + 2];
+                        const double h2a = h[2 * WCA + 1], h2b = h[2 * WCA + 2];
+                        const double h0a = h[WCW + 1], h0b = h[WCW + 2];
+                        const double s0 = ((l0.x + l1a) + (l2.x + l3a)) - ((h3.x + h2a) + (h1.x + h0a));
+                        const double s1 = ((l0.y + l1b) + (l2.y + l3b)) - ((h3.y + h2b) + (h1.y + h0b));
+                        const double yy0 = s0 * (ivr_here * cw0[r]), yy1 = s1 * (ivr_here * cw1[r]);
+                        const double2 qv = lds2(Q_of(slot) + w * WK + c2);
+                        double* o = a.out + (size_t)i * plane + (size_t)(j0 + w) * g.np + k0 + c2;
+                        if (MODE == MODE_RESID) {
+                            const double r0 = qv.x - yy0, r1 = qv.y - yy1;
+                            stg2(o, make_double2(r0, r1));
+                            const double vr = __ldg(g.vr + i);
+                            const double V0 = vr / cw0[r], V1 = vr / cw1[r];
+                            const double2 f = ld2(a.f + (o - a.out));
+                            const double2 di = ld2(a.dinv + (o - a.out));
+                            acc[0] += V0 * f.x * f.x + V1 * f.y * f.y;
+                            acc[1] += V0 * r0 * r0 + V1 * r1 * r1;
+                            acc[2] += V0 * r0 * (di.x * r0) + V1 * r1 * (di.y * r1);
+                        } else {
+                            stg2(o, make_double2(qv.x + yy0, qv.y + yy1));
+                        }
+                    }
+                }
+                fence_proxy_async();
+                __syncwarp();
+                if (lane == 0) mbar_arrive(empty0 + 8 * ((n - 1) % W_NSLOT));
             }
 #else
             // ---- consumers --------------------------------------------------
