@@ -141,7 +141,11 @@ namespace {
 #define MAS_ANISO_BPS 1
 #endif
 #ifndef MAS_ANISO_RPW
+#ifdef MAS_ANISO_V3
+#define MAS_ANISO_RPW 2
+#else
 #define MAS_ANISO_RPW 1
+#endif
 #endif
 constexpr int WJ = MAS_ANISO_WJ;       // tile rows
 constexpr int RPW = MAS_ANISO_RPW;     // tile rows per consumer warp (rows w + r * NCW)
@@ -502,6 +506,173 @@ __global__ void __launch_bounds__(WTHREADS, kAnisoBps) k_aniso(const AnisoArgs a
                 fence_proxy_async();
                 __syncwarp();
                 if (lane == 0) mbar_arrive(empty0 + 8 * slot);
+            }
+#elif defined(MAS_ANISO_V3)
+            // ---- consumers V3: pair sums ------------------------------------
+            // Warp q owns the corner rows J = q + r * NCW (r < RPW) and warp 0
+            // also the tile's bottom corner row WJ.  Per corner row each lane
+            // computes its corners (J, c2), (J, c2+1), lane 31 also (J, 64); the
+            // column neighbour's combinations come by shuffle, and the lane forms
+            //   P1 = o0(c) + o1(c+1)   lower part of cell (J, c) from row J
+            //   P2 = o2(c) + o3(c+1)   lower part of cell (J-1, c) from row J
+            //   P3 = o3(c) + o2(c+1)   upper part of cell (J, c) from row J
+            //   P4 = o1(c) + o0(c+1)   upper part of cell (J-1, c) from row J
+            // It keeps P1 (for the next step) and P3 in registers and stores P2,
+            // P4 for the warp of row J-1, into arrays 0 and 1 of the slot's
+            // corner region in place of the coefficients it read.  A cell then
+            // reads 2 aligned double2 instead of 12 values of the 4 combination
+            // arrays; the sums are V1's, in V1's order (bitwise equal).
+            static_assert(WQ_SLOT > 0, "MAS_ANISO_V3 needs the out/q TMA box");
+            constexpr int NR = RPW + 1;
+            const int c2 = 2 * lane;
+            const bool first = k0 == 0, last = k0 + width == g.np;
+            const bool lfix = first && c2 == 0, rfix = last && c2 == width;
+            const bool xcol = lane == 31 && width == WK;  // the extra corner (J, 64)
+            int rowJ[NR];
+            bool rok[NR], cok[NR];
+            double cw0[NR], cw1[NR];
+#pragma unroll
+            for (int r = 0; r < NR; r++) {
+                const int J = r < RPW ? warp + r * NCW : (warp == 0 && height == WJ ? WJ : -1);
+                rowJ[r] = J;
+                rok[r] = J >= 0 && J <= height && c2 <= width;
+                cok[r] = r < RPW && J < height && c2 < width;
+                cw0[r] = cw1[r] = 0.0;
+                if (cok[r]) {
+                    const double vt = __ldg(g.vt + j0 + J);
+                    cw0[r] = 1.0 / (vt * __ldg(g.vp + k0 + c2));
+                    cw1[r] = 1.0 / (vt * __ldg(g.vp + k0 + c2 + 1));
+                }
+            }
+            auto corner_math = [&](double a00, double a01, double a10, double a11, double b00, double b01,
+                                   double b10, double b11, double A0, double B0, double E0, double& o0,
+                                   double& o1, double& o2, double& o3) -> double {
+                const double Dr = ((b00 - a00) + (b01 - a01)) + ((b10 - a10) + (b11 - a11));
+                const double Dt = ((a10 - a00) + (a11 - a01)) + ((b10 - b00) + (b11 - b01));
+                const double Dp = ((a01 - a00) + (a11 - a10)) + ((b01 - b00) + (b11 - b10));
+                const double sc = A0 * Dr + B0 * Dt + E0 * Dp;
+                const double A = sc * A0, B = sc * B0, E = sc * E0;
+                o0 = (A + B) + E;
+                o1 = (A + B) - E;
+                o2 = (A - B) + E;
+                o3 = (A - B) - E;
+                return sc;
+            };
+            // p of a plane for row J's corners: the pair (X0 / Y0: column c2-1 of
+            // rows J-1 / J; X12 / Y12: columns c2, c2+1) and the extra corner's
+            // cells 63, 64 (EX); wrap cells from the side boxes.  Both planes of a
+            // corner come from the ring (stage n-1 is released after step n), so
+            // no p is carried in registers (a 9-warp block gets 168 registers).
+            auto load_p = [&](const double* pb, int J, double& X0, double& Y0, double2& X12, double2& Y12,
+                              double (&EX)[4]) {
+                const double* q1 = pb + J * WPW + c2;
+                X0 = q1[1], Y0 = q1[WPW + 1];
+                X12 = lds2(q1 + 2), Y12 = lds2(q1 + WPW + 2);
+                if (lfix) X0 = pb[O_PL + 2 * J + 1], Y0 = pb[O_PL + 2 * J + 3];
+                if (rfix) X12.x = pb[O_PR + 2 * J], Y12.x = pb[O_PR + 2 * J + 2];
+                EX[0] = EX[1] = EX[2] = EX[3] = 0.0;
+                if (xcol) {  // cells 63, 64 of rows J-1, J (box columns 65, 66)
+                    const double* e = pb + J * WPW + WK + 1;
+                    EX[0] = e[0], EX[1] = e[1], EX[2] = e[WPW], EX[3] = e[WPW + 1];
+                    if (last) EX[1] = pb[O_PR + 2 * J], EX[3] = pb[O_PR + 2 * J + 2];
+                }
+            };
+            double2 p1prev[NR];  // P1 of the previous corner plane
+#pragma unroll
+            for (int r = 0; r < NR; r++) p1prev[r] = make_double2(0.0, 0.0);
+            double ivr_cur = 0.0;
+            for (int n = 0; n < nst; n++) {
+                const int I = ia - 1 + n, slot = n % W_NSLOT;
+                const double ivr_here = ivr_cur;
+                if (cok[0] && n + 1 >= 2 && n + 1 < nst) ivr_cur = __ldg(a.ivr + I);
+                mbar_wait(full0 + 8 * slot, (n / W_NSLOT) & 1);
+                const double* p1 = P_of(slot);
+                if (n == 0) continue;  // stage ia-1: p plane ia-1 only (read at step 1)
+                const double* p0 = P_of((n - 1) % W_NSLOT);
+                double* Cf = C_of(slot);
+                double2 p1now[NR], p3now[NR];
+#pragma unroll
+                for (int r = 0; r < NR; r++) {
+                    const int J = rowJ[r];
+                    double o[2][4] = {{0.0, 0.0, 0.0, 0.0}, {0.0, 0.0, 0.0, 0.0}};
+                    double ox[4] = {0.0, 0.0, 0.0, 0.0};
+                    if (rok[r]) {
+                        double x0, y0, X0, Y0, ex[4], EX[4];
+                        double2 x12, y12, X12, Y12;
+                        load_p(p0, J, x0, y0, x12, y12, ex);
+                        load_p(p1, J, X0, Y0, X12, Y12, EX);
+                        const double* c0 = Cf + J * WCW + c2;
+                        double2 A0 = lds2(c0), B0 = lds2(c0 + WCA), C0 = lds2(c0 + 2 * WCA);
+                        if (rfix) {
+                            const double* CS = p1 + O_CS;
+                            A0.x = CS[2 * J], B0.x = CS[2 * (WCR + J)], C0.x = CS[2 * (2 * WCR + J)];
+                        }
+                        const double s0 = corner_math(x0, x12.x, y0, y12.x, X0, X12.x, Y0, Y12.x, A0.x, B0.x,
+                                                      C0.x, o[0][0], o[0][1], o[0][2], o[0][3]);
+                        const double s1 = corner_math(x12.x, x12.y, y12.x, y12.y, X12.x, X12.y, Y12.x, Y12.y,
+                                                      A0.y, B0.y, C0.y, o[1][0], o[1][1], o[1][2], o[1][3]);
+                        if (MODE == MODE_PCGA && I < ib && J < height && c2 < width) acc[0] += s0 * s0 + s1 * s1;
+                        if (xcol) {
+                            const double* cx = Cf + J * WCW + WK;
+                            double A = cx[0], B = cx[WCA], E = cx[2 * WCA];
+                            if (last) {
+                                const double* CS = p1 + O_CS;
+                                A = CS[2 * J], B = CS[2 * (WCR + J)], E = CS[2 * (2 * WCR + J)];
+                            }
+                            corner_math(ex[0], ex[1], ex[2], ex[3], EX[0], EX[1], EX[2], EX[3], A, B, E, ox[0],
+                                        ox[1], ox[2], ox[3]);
+                        }
+                    }
+                    // the combinations of corner (J, c2+2): lane+1's first corner, or the extra one
+                    double nb[4];
+#pragma unroll
+                    for (int q = 0; q < 4; q++) {
+                        nb[q] = __shfl_down_sync(0xffffffffu, o[0][q], 1);
+                        if (lane == 31) nb[q] = ox[q];
+                    }
+                    p1now[r] = make_double2(o[0][0] + o[1][1], o[1][0] + nb[1]);
+                    p3now[r] = make_double2(o[0][3] + o[1][2], o[1][3] + nb[2]);
+                    if (rok[r]) {
+                        double* c0 = Cf + J * WCW + c2;  // its own coefficient positions (read above)
+                        sts2(c0, make_double2(o[0][2] + o[1][3], o[1][2] + nb[3]));        // P2
+                        sts2(c0 + WCA, make_double2(o[0][1] + o[1][0], o[1][1] + nb[0]));  // P4
+                    }
+                }
+                consumer_sync();
+                if (n >= 2) {
+                    const int i = I - 1;
+                    const double* Cp = C_of((n - 1) % W_NSLOT);
+#pragma unroll
+                    for (int r = 0; r < RPW; r++) {
+                        if (!cok[r]) continue;
+                        const int J = rowJ[r];
+                        const double2 s2 = lds2(Cp + (J + 1) * WCW + c2);       // P2 of row J+1, plane I-1
+                        const double2 s4 = lds2(Cf + WCA + (J + 1) * WCW + c2); // P4 of row J+1, plane I
+                        const double s0 = (p1prev[r].x + s2.x) - (p3now[r].x + s4.x);
+                        const double s1 = (p1prev[r].y + s2.y) - (p3now[r].y + s4.y);
+                        const double yy0 = s0 * (ivr_here * cw0[r]), yy1 = s1 * (ivr_here * cw1[r]);
+                        const double2 qv = lds2(Q_of(slot) + J * WK + c2);
+                        double* o = a.out + (size_t)i * plane + (size_t)(j0 + J) * g.np + k0 + c2;
+                        if (MODE == MODE_RESID) {
+                            const double r0 = qv.x - yy0, r1 = qv.y - yy1;
+                            stg2(o, make_double2(r0, r1));
+                            const double vr = __ldg(g.vr + i);
+                            const double V0 = vr / cw0[r], V1 = vr / cw1[r];
+                            const double2 f = ld2(a.f + (o - a.out));
+                            const double2 di = ld2(a.dinv + (o - a.out));
+                            acc[0] += V0 * f.x * f.x + V1 * f.y * f.y;
+                            acc[1] += V0 * r0 * r0 + V1 * r1 * r1;
+                            acc[2] += V0 * r0 * (di.x * r0) + V1 * r1 * (di.y * r1);
+                        } else {
+                            stg2(o, make_double2(qv.x + yy0, qv.y + yy1));
+                        }
+                    }
+                }
+#pragma unroll
+                for (int r = 0; r < NR; r++) p1prev[r] = p1now[r];
+                fence_proxy_async();
+                __syncwarp();
+                if (lane == 0) mbar_arrive(empty0 + 8 * ((n - 1) % W_NSLOT));
             }
 #elif MAS_ANISO_RPW > 1
             // ---- consumers, RPW rows per warp (experiment: fewer warps, RPW
