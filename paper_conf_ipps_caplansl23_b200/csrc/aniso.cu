@@ -141,18 +141,19 @@ namespace {
 #define MAS_ANISO_BPS 1
 #endif
 #ifndef MAS_ANISO_RPW
-#ifdef MAS_ANISO_V3
-#define MAS_ANISO_RPW 2
-#else
 #define MAS_ANISO_RPW 1
-#endif
 #endif
 constexpr int WJ = MAS_ANISO_WJ;       // tile rows
 constexpr int RPW = MAS_ANISO_RPW;     // tile rows per consumer warp (rows w + r * NCW)
 constexpr int kAnisoBps = MAS_ANISO_BPS;  // resident blocks per SM (the rings must fit)
 constexpr int rup16(int x) { return (x + 15) / 16 * 16; }  // 128-byte multiples of doubles
 constexpr int WK = 64;                 // tile columns (32 lanes x 2)
+#ifdef MAS_ANISO_V3
+constexpr int NCW = WJ + 1;            // consumer warps: one per corner row J = 0..WJ
+static_assert(RPW == 1, "MAS_ANISO_V3: one corner row per warp");
+#else
 constexpr int NCW = WJ / RPW;          // consumer warps
+#endif
 static_assert(WJ % RPW == 0, "MAS_ANISO_RPW must divide MAS_ANISO_WJ");
 constexpr int WTHREADS = 32 * (NCW + 1);
 constexpr int WPR = WJ + 2;            // p rows: j0-1 .. j0+16
@@ -317,6 +318,15 @@ __global__ void __launch_bounds__(WTHREADS, kAnisoBps) k_aniso(const AnisoArgs a
         const int nst = ib - ia + 2;
 
         if (producer) {
+#ifdef MAS_ANISO_TMAP_PREFETCH
+            if (lane == 0) {  // the tensor-map descriptors into the descriptor cache
+                const CUtensorMap* maps[] = {&M.u, &M.u_s, &M.lo, &M.lo_s, &M.hi, &M.hi_s, &M.ca, &M.ca_s,
+                                             &M.cahi, &M.cahi_s, &M.out};
+                for (const CUtensorMap* m : maps)
+                    asm volatile("prefetch.tensormap [%0];\n" ::"l"(reinterpret_cast<unsigned long long>(m))
+                                 : "memory");
+            }
+#endif
             // one lane issues the stage's tensor copies: one box per field, plus
             // the 2-wide phi-wrap side boxes on the first / last phi tile (the
             // consumers read the wrap cells from those)
@@ -509,8 +519,7 @@ __global__ void __launch_bounds__(WTHREADS, kAnisoBps) k_aniso(const AnisoArgs a
             }
 #elif defined(MAS_ANISO_V3)
             // ---- consumers V3: pair sums ------------------------------------
-            // Warp q owns the corner rows J = q + r * NCW (r < RPW) and warp 0
-            // also the tile's bottom corner row WJ.  Per corner row each lane
+            // Warp J owns corner row J (J = 0..WJ: 17 consumer warps).  Each lane
             // computes its corners (J, c2), (J, c2+1), lane 31 also (J, 64); the
             // column neighbour's combinations come by shuffle, and the lane forms
             //   P1 = o0(c) + o1(c+1)   lower part of cell (J, c) from row J
@@ -523,7 +532,7 @@ __global__ void __launch_bounds__(WTHREADS, kAnisoBps) k_aniso(const AnisoArgs a
             // reads 2 aligned double2 instead of 12 values of the 4 combination
             // arrays; the sums are V1's, in V1's order (bitwise equal).
             static_assert(WQ_SLOT > 0, "MAS_ANISO_V3 needs the out/q TMA box");
-            constexpr int NR = RPW + 1;
+            constexpr int NR = 1;
             const int c2 = 2 * lane;
             const bool first = k0 == 0, last = k0 + width == g.np;
             const bool lfix = first && c2 == 0, rfix = last && c2 == width;
@@ -533,10 +542,10 @@ __global__ void __launch_bounds__(WTHREADS, kAnisoBps) k_aniso(const AnisoArgs a
             double cw0[NR], cw1[NR];
 #pragma unroll
             for (int r = 0; r < NR; r++) {
-                const int J = r < RPW ? warp + r * NCW : (warp == 0 && height == WJ ? WJ : -1);
+                const int J = warp;
                 rowJ[r] = J;
-                rok[r] = J >= 0 && J <= height && c2 <= width;
-                cok[r] = r < RPW && J < height && c2 < width;
+                rok[r] = J <= height && c2 <= width;
+                cok[r] = J < height && c2 < width;
                 cw0[r] = cw1[r] = 0.0;
                 if (cok[r]) {
                     const double vt = __ldg(g.vt + j0 + J);
@@ -643,7 +652,7 @@ __global__ void __launch_bounds__(WTHREADS, kAnisoBps) k_aniso(const AnisoArgs a
                     const int i = I - 1;
                     const double* Cp = C_of((n - 1) % W_NSLOT);
 #pragma unroll
-                    for (int r = 0; r < RPW; r++) {
+                    for (int r = 0; r < NR; r++) {
                         if (!cok[r]) continue;
                         const int J = rowJ[r];
                         const double2 s2 = lds2(Cp + (J + 1) * WCW + c2);       // P2 of row J+1, plane I-1
@@ -899,6 +908,15 @@ __global__ void __launch_bounds__(WTHREADS, kAnisoBps) k_aniso(const AnisoArgs a
                 if (n >= 2 && cell_ok) qv = ld2(a.out + (size_t)(I - 1) * plane + qoff);
 #endif
                 mbar_wait(full0 + 8 * slot, (n / W_NSLOT) & 1);
+#ifdef MAS_ANISO_DIAG_NOCOMPUTE
+                // diagnostic build (wrong results): the consumers only wait for
+                // each stage and release it -- the producer / TMA pipeline alone
+                if (n >= 1) {
+                    __syncwarp();
+                    if (lane == 0) mbar_arrive(empty0 + 8 * ((n - 1) % W_NSLOT));
+                }
+                continue;
+#endif
                 const double* p1 = P_of(slot);
                 double X0 = 0.0, Y0 = 0.0, E0 = 0.0, E1 = 0.0, E2 = 0.0, E3 = 0.0;
                 double2 X12 = make_double2(0.0, 0.0), Y12 = X12;
