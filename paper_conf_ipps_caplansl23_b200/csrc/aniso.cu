@@ -236,6 +236,16 @@ __device__ __forceinline__ void tma4(unsigned dst, const CUtensorMap* m, int c0,
 __device__ __forceinline__ void fence_proxy_async() {
     asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
 }
+// tensor store (TMA) of a shared-memory box into global memory, bulk-group
+// completion (MAS_ANISO_QST: the updated out/q box leaves through the TMA
+// engine instead of per-thread stores)
+__device__ __forceinline__ void tma_store3(const CUtensorMap* m, int c0, int c1, int c2, unsigned src) {
+    asm volatile("cp.async.bulk.tensor.3d.global.shared::cta.bulk_group [%0, {%1, %2, %3}], [%4];\n"
+                 ::"l"(m), "r"(c0), "r"(c1), "r"(c2), "r"(src) : "memory");
+}
+__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;\n" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_read0() { asm volatile("cp.async.bulk.wait_group.read 0;\n" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait0() { asm volatile("cp.async.bulk.wait_group 0;\n" ::: "memory"); }
 __device__ __forceinline__ void consumer_sync() {  // the 16 consumer warps only
     asm volatile("bar.sync 1, %0;\n" ::"n"(32 * NCW) : "memory");
 }
@@ -895,10 +905,48 @@ __global__ void __launch_bounds__(WTHREADS, kAnisoBps) k_aniso(const AnisoArgs a
             // 1/vr of the cell plane of the next step, loaded one step ahead
             // (its latency sat on the cell phase's dependency chain)
             double ivr_cur = 0.0;
+#ifdef MAS_ANISO_LAG
+            static_assert(WQ_SLOT > 0, "MAS_ANISO_LAG needs the out/q TMA box");
+            // cells (w, c2..c2+1) of plane i: corner planes i (slot sl, sr = +1)
+            // and i+1 (slot sh, sr = -1); out/q plane i from slot sh's box
+            auto gather = [&](int i, int sl, int sh, double ivr) {
+                if (!cell_ok) return;
+                const double* l = C_of(sl) + w * WCW + c2;
+                const double* h = C_of(sh) + w * WCW + c2;
+                const double2 l0 = lds2(l), l2 = lds2(l + 2 * WCA + WCW);
+                const double2 h3 = lds2(h + 3 * WCA), h1 = lds2(h + WCA + WCW);
+                const double l1a = l[WCA + 1], l1b = l[WCA + 2];
+                const double l3a = l[3 * WCA + WCW + 1], l3b = l[3 * WCA + WCW + 2];
+                const double h2a = h[2 * WCA + 1], h2b = h[2 * WCA + 2];
+                const double h0a = h[WCW + 1], h0b = h[WCW + 2];
+                const double s0 = ((l0.x + l1a) + (l2.x + l3a)) - ((h3.x + h2a) + (h1.x + h0a));
+                const double s1 = ((l0.y + l1b) + (l2.y + l3b)) - ((h3.y + h2b) + (h1.y + h0b));
+                const double yy0 = s0 * (ivr * cw0), yy1 = s1 * (ivr * cw1);
+                const double2 qv = lds2(Q_of(sh) + w * WK + c2);
+                double* o = a.out + (size_t)i * plane + (size_t)(j0 + w) * g.np + k0 + c2;
+                if (MODE == MODE_RESID) {
+                    const double r0 = qv.x - yy0, r1 = qv.y - yy1;
+                    stg2(o, make_double2(r0, r1));
+                    const double vr = __ldg(g.vr + i);
+                    const double V0 = vr / cw0, V1 = vr / cw1;
+                    const double2 f = ld2(a.f + (o - a.out));
+                    const double2 di = ld2(a.dinv + (o - a.out));
+                    acc[0] += V0 * f.x * f.x + V1 * f.y * f.y;
+                    acc[1] += V0 * r0 * r0 + V1 * r1 * r1;
+                    acc[2] += V0 * r0 * (di.x * r0) + V1 * r1 * (di.y * r1);
+                } else {
+                    stg2(o, make_double2(qv.x + yy0, qv.y + yy1));
+                }
+            };
+#endif
             for (int n = 0; n < nst; n++) {
                 const int I = ia - 1 + n, slot = n % W_NSLOT;
                 const double ivr_here = ivr_cur;
+#ifdef MAS_ANISO_LAG
+                if (cell_ok && n >= 2) ivr_cur = __ldg(a.ivr + I - 1);  // the gather of step n+1 / the epilogue
+#else
                 if (cell_ok && n + 1 >= 2 && n + 1 < nst) ivr_cur = __ldg(a.ivr + I);
+#endif
 #if !defined(MAS_ANISO_QTMA) && !defined(MAS_ANISO_QNOW)
                 const double2 qv = qnext;
                 if (n + 1 >= 2 && n + 1 < nst && cell_ok) qnext = ld2(a.out + (size_t)I * plane + qoff);
@@ -911,6 +959,13 @@ __global__ void __launch_bounds__(WTHREADS, kAnisoBps) k_aniso(const AnisoArgs a
 #ifdef MAS_ANISO_DIAG_NOCOMPUTE
                 // diagnostic build (wrong results): the consumers only wait for
                 // each stage and release it -- the producer / TMA pipeline alone
+                // (MAS_ANISO_DIAG_STORE: plus the q store of the cells)
+#ifdef MAS_ANISO_DIAG_STORE
+                if (n >= 2 && cell_ok) {
+                    const double2 qv = lds2(Q_of(slot) + w * WK + c2);
+                    stg2(a.out + (size_t)(I - 1) * plane + (size_t)(j0 + w) * g.np + k0 + c2, qv);
+                }
+#endif
                 if (n >= 1) {
                     __syncwarp();
                     if (lane == 0) mbar_arrive(empty0 + 8 * ((n - 1) % W_NSLOT));
@@ -974,7 +1029,33 @@ __global__ void __launch_bounds__(WTHREADS, kAnisoBps) k_aniso(const AnisoArgs a
                     c0[3 * WCA] = o3;
                 }
                 x0 = X0, y0 = Y0, x12 = X12, y12 = Y12, e0 = E0, e1 = E1, e2 = E2, e3 = E3;
+#ifdef MAS_ANISO_QST
+                // every warp has finished step n-1's cells (written into stage
+                // n-1's out box): one thread stores that box with the TMA engine
+                // (plane I-2); its warp waits until the box is read before the
+                // stage is released below
                 consumer_sync();
+                if (threadIdx.x == 0 && n >= 3) {
+                    tma_store3(&M.out, k0, j0, I - 2, smem_u32(Q_of((n - 1) % W_NSLOT)));
+                    bulk_commit();
+                }
+#endif
+#ifdef MAS_ANISO_LAG
+                // software pipeline: the cells of plane I-2 (corner planes I-2, I-1,
+                // complete since the last barrier) next to the corners of plane I,
+                // one barrier per step; stage n-2 is released after it
+                if (n >= 3) gather(I - 2, (n - 2) % W_NSLOT, (n - 1) % W_NSLOT, ivr_here);
+                consumer_sync();
+                if (n >= 2) {
+                    fence_proxy_async();
+                    __syncwarp();
+                    if (lane == 0) mbar_arrive(empty0 + 8 * ((n - 2) % W_NSLOT));
+                }
+                continue;
+#endif
+#ifndef MAS_ANISO_QST
+                consumer_sync();
+#endif
                 // ---- cells (w, c2..c2+1) of plane i = I-1: corner planes i
                 // (sr = +1) and I (sr = -1); out/q plane i from this stage
                 if (n >= 2 && cell_ok) {
@@ -995,9 +1076,17 @@ __global__ void __launch_bounds__(WTHREADS, kAnisoBps) k_aniso(const AnisoArgs a
                     const double2 qv = lds2(Q_of(slot) + w * WK + c2);
 #endif
                     double* o = a.out + (size_t)i * plane + (size_t)(j0 + w) * g.np + k0 + c2;
+#ifdef MAS_ANISO_QST
+                    double* qs = Q_of(slot) + w * WK + c2;  // the result goes back into the out box
+                    (void)o;
+#endif
                     if (MODE == MODE_RESID) {
                         const double r0 = qv.x - y0, r1 = qv.y - y1;
+#ifdef MAS_ANISO_QST
+                        sts2(qs, make_double2(r0, r1));
+#else
                         stg2(o, make_double2(r0, r1));
+#endif
                         const double vr = __ldg(g.vr + i);
                         const double V0 = vr / cw0, V1 = vr / cw1;
                         const double2 f = ld2(a.f + (o - a.out));
@@ -1006,16 +1095,38 @@ __global__ void __launch_bounds__(WTHREADS, kAnisoBps) k_aniso(const AnisoArgs a
                         acc[1] += V0 * r0 * r0 + V1 * r1 * r1;
                         acc[2] += V0 * r0 * (di.x * r0) + V1 * r1 * (di.y * r1);
                     } else {
+#if defined(MAS_ANISO_QST)
+                        sts2(qs, make_double2(qv.x + y0, qv.y + y1));
+#elif !defined(MAS_ANISO_DIAG_NOSTORE)  // diagnostic build (wrong results): no q store
                         stg2(o, make_double2(qv.x + y0, qv.y + y1));
+#else
+                        if (qv.x + y0 == 1.2345e-300) stg2(o, make_double2(qv.x + y0, qv.y + y1));
+#endif
                     }
                 }
                 // stage n-1 is no longer read (p by corners(I), products by
                 // cells(I-1)); the combination writes went through the generic
                 // proxy, the next fill of the slot is a tensor copy
                 fence_proxy_async();
+#ifdef MAS_ANISO_QST
+                if (threadIdx.x == 0 && n >= 3) bulk_wait_read0();  // stage n-1's out box has left
+#endif
                 __syncwarp();
                 if (lane == 0) mbar_arrive(empty0 + 8 * ((n - 1) % W_NSLOT));
             }
+#ifdef MAS_ANISO_LAG
+            // the last cell plane ib-1 (corner planes ib-1, ib: the last two stages)
+            if (nst >= 3) gather(ib - 1, (nst - 2) % W_NSLOT, (nst - 1) % W_NSLOT, ivr_cur);
+#endif
+#ifdef MAS_ANISO_QST
+            // the segment's last out box (plane ib-1), after every warp's cells
+            consumer_sync();
+            if (threadIdx.x == 0 && nst >= 3) {
+                tma_store3(&M.out, k0, j0, ib - 1, smem_u32(Q_of((nst - 1) % W_NSLOT)));
+                bulk_commit();
+                bulk_wait0();  // complete before the next segment reuses the ring / the kernel ends
+            }
+#endif
 #endif
         }
         __syncthreads();  // the next segment re-initialises the rings and barriers
