@@ -128,33 +128,20 @@ __device__ __forceinline__ double2 ld2(const double* p) { return __ldg(reinterpr
 // ring, signalled by mbarriers (full: the box bytes landed; empty: the 16
 // consumer warps are done with the slot).
 namespace {
-// out/q: a TMA box per stage (default; A/B r2n: 53.7 us) or, with
-// MAS_ANISO_QLDG, plain loads by the consumers (54.0 us at the top of the
-// step, 55.4 us one step ahead)
-#ifndef MAS_ANISO_QLDG
-#define MAS_ANISO_QTMA
-#endif
+// out/q arrives as a TMA box per stage (plain loads by the consumers measured
+// slower; the other consumer designs tried are listed in profiles/README.md,
+// "k_aniso A/B", and kept in the history up to c1ffbea)
 #ifndef MAS_ANISO_WJ
 #define MAS_ANISO_WJ 16
 #endif
 #ifndef MAS_ANISO_BPS
 #define MAS_ANISO_BPS 1
 #endif
-#ifndef MAS_ANISO_RPW
-#define MAS_ANISO_RPW 1
-#endif
-constexpr int WJ = MAS_ANISO_WJ;       // tile rows
-constexpr int RPW = MAS_ANISO_RPW;     // tile rows per consumer warp (rows w + r * NCW)
+constexpr int WJ = MAS_ANISO_WJ;       // tile rows (one consumer warp each)
 constexpr int kAnisoBps = MAS_ANISO_BPS;  // resident blocks per SM (the rings must fit)
 constexpr int rup16(int x) { return (x + 15) / 16 * 16; }  // 128-byte multiples of doubles
 constexpr int WK = 64;                 // tile columns (32 lanes x 2)
-#ifdef MAS_ANISO_V3
-constexpr int NCW = WJ + 1;            // consumer warps: one per corner row J = 0..WJ
-static_assert(RPW == 1, "MAS_ANISO_V3: one corner row per warp");
-#else
-constexpr int NCW = WJ / RPW;          // consumer warps
-#endif
-static_assert(WJ % RPW == 0, "MAS_ANISO_RPW must divide MAS_ANISO_WJ");
+constexpr int NCW = WJ;                // consumer warps
 constexpr int WTHREADS = 32 * (NCW + 1);
 constexpr int WPR = WJ + 2;            // p rows: j0-1 .. j0+16
 constexpr int WPW = WK + 4;            // p row: [k0-2][k0-1][64 cells][k0+64][k0+65]
@@ -164,11 +151,7 @@ constexpr int WCA = WCR * WCW;         // one corner array
 // every component of a slot starts 128-byte aligned (tensor-copy destinations)
 constexpr int WP_SLOT = rup16(WPR * WPW);  // p box [WJ+2][68] + pad
 constexpr int WC_SLOT = rup16(4 * WCA);    // coefficient box [3][WJ+1][66] + combinations array 3 + pad
-#ifdef MAS_ANISO_QTMA
 constexpr int WQ_SLOT = WJ * WK;       // out box [WJ][64]
-#else
-constexpr int WQ_SLOT = 0;             // out/q is read by the consumers directly
-#endif
 constexpr int WPL = rup16(WPR * 2), WPRT = WPL;  // phi-wrap side boxes of p: [WJ+2][2]
 constexpr int WCS = rup16(3 * WCR * 2);          // phi-wrap side box of the coefficients: [3][WJ+1][2]
 constexpr int O_C = WP_SLOT, O_Q = O_C + WC_SLOT, O_PL = O_Q + WQ_SLOT, O_PR = O_PL + WPL,
@@ -181,9 +164,7 @@ constexpr int W_NSLOT = MAS_ANISO_SLOTS;  // ring depth (>= 2: a step reads stag
 // tensor-copy transaction bytes (whole boxes, out-of-bounds elements included)
 constexpr unsigned TX_P = WPR * WPW * 8, TX_PS = WPR * 2 * 8, TX_C = 3 * WCR * WCW * 8,
                    TX_CS = 3 * WCR * 2 * 8;
-#ifdef MAS_ANISO_QTMA
 constexpr unsigned TX_Q = WJ * WK * 8;
-#endif
 }  // namespace
 constexpr int kAnisoSmem = W_NSLOT * W_SLOT * (int)sizeof(double) + 3 * W_NSLOT * 8;  // 222,816 B
 
@@ -236,16 +217,6 @@ __device__ __forceinline__ void tma4(unsigned dst, const CUtensorMap* m, int c0,
 __device__ __forceinline__ void fence_proxy_async() {
     asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
 }
-// tensor store (TMA) of a shared-memory box into global memory, bulk-group
-// completion (MAS_ANISO_QST: the updated out/q box leaves through the TMA
-// engine instead of per-thread stores)
-__device__ __forceinline__ void tma_store3(const CUtensorMap* m, int c0, int c1, int c2, unsigned src) {
-    asm volatile("cp.async.bulk.tensor.3d.global.shared::cta.bulk_group [%0, {%1, %2, %3}], [%4];\n"
-                 ::"l"(m), "r"(c0), "r"(c1), "r"(c2), "r"(src) : "memory");
-}
-__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;\n" ::: "memory"); }
-__device__ __forceinline__ void bulk_wait_read0() { asm volatile("cp.async.bulk.wait_group.read 0;\n" ::: "memory"); }
-__device__ __forceinline__ void bulk_wait0() { asm volatile("cp.async.bulk.wait_group 0;\n" ::: "memory"); }
 __device__ __forceinline__ void consumer_sync() {  // the 16 consumer warps only
     asm volatile("bar.sync 1, %0;\n" ::"n"(32 * NCW) : "memory");
 }
@@ -328,15 +299,6 @@ __global__ void __launch_bounds__(WTHREADS, kAnisoBps) k_aniso(const AnisoArgs a
         const int nst = ib - ia + 2;
 
         if (producer) {
-#ifdef MAS_ANISO_TMAP_PREFETCH
-            if (lane == 0) {  // the tensor-map descriptors into the descriptor cache
-                const CUtensorMap* maps[] = {&M.u, &M.u_s, &M.lo, &M.lo_s, &M.hi, &M.hi_s, &M.ca, &M.ca_s,
-                                             &M.cahi, &M.cahi_s, &M.out};
-                for (const CUtensorMap* m : maps)
-                    asm volatile("prefetch.tensormap [%0];\n" ::"l"(reinterpret_cast<unsigned long long>(m))
-                                 : "memory");
-            }
-#endif
             // one lane issues the stage's tensor copies: one box per field, plus
             // the 2-wide phi-wrap side boxes on the first / last phi tile (the
             // consumers read the wrap cells from those)
@@ -364,9 +326,7 @@ __global__ void __launch_bounds__(WTHREADS, kAnisoBps) k_aniso(const AnisoArgs a
                     // uninitialised values: 0 * NaN)
                     bytes += TX_P + (first ? TX_PS : 0u) + (last ? TX_PS : 0u);
                     if (cs) bytes += TX_C + (last ? TX_CS : 0u);
-#ifdef MAS_ANISO_QTMA
                     if (ql) bytes += TX_Q;
-#endif
                     mbar_expect_tx(full, bytes);
                     const unsigned sb = smem_u32(base);
                     const int jr = j0 - 1;
@@ -390,470 +350,11 @@ __global__ void __launch_bounds__(WTHREADS, kAnisoBps) k_aniso(const AnisoArgs a
                         tma3(sb + 8 * O_C, &M.cahi, k0, j0, 0, full);
                         if (last) tma3(sb + 8 * O_CS, &M.cahi_s, 0, j0, 0, full);
                     }
-#ifdef MAS_ANISO_QTMA
                     if (ql) tma3(sb + 8 * O_Q, &M.out, k0, j0, I - 1, full);
-#else
-                    (void)ql;  // out/q is read by the consumers directly (see below)
-#endif
                 }
             };
             for (int n = 0; n < nst; n++) issue(n);
         } else {
-#ifdef MAS_ANISO_V2
-            // ---- consumers (V2, experiment: measured 81 us against V1's 53.7 us
-            // at C2a -- the 3x corner recomputation and register spills at the
-            // 96-register cap of a 544-thread block outweigh the saved barrier
-            // and shared-memory traffic; profiles/README.md r3d/r3e) ---------
-            // Warp w (cell row w) computes the corners of BOTH corner rows its
-            // cells touch (J = j0+w and j0+w+1) itself -- each corner twice, once
-            // per warp -- and folds them into per-cell sums held in registers:
-            //   V y_P = [sum_JK A(i,J,K) - sum_JK A(i+1,J,K)]
-            //         + [sum_IK B(I,j,K) - B(I,j+1,K)] + [sum_IJ E(I,J,k) - E(I,J,k+1)]
-            // with (A, B, E) = s_c (a, b, e).  No shared-memory stores, no
-            // consumer barrier; a stage is released as soon as its step is done.
-            const int w = warp, l2 = 2 * lane;
-            const bool first = k0 == 0, last = k0 + width == g.np;
-            const bool rows_ok = w < height;                  // this warp's row exists
-            const bool active = rows_ok && l2 < width;       // this lane's cell pair
-            const bool lfix = first && lane == 0;            // column k0-1: the left side box
-            const bool rfix = last && l2 + 2 == width;       // column k0+width: the right side box
-            double cw0 = 0.0, cw1 = 0.0;  // 1 / (vt_j vp_k) of the two cells
-            if (active) {
-                const double vt = __ldg(g.vt + j0 + w);
-                cw0 = 1.0 / (vt * __ldg(g.vp + k0 + l2));
-                cw1 = 1.0 / (vt * __ldg(g.vp + k0 + l2 + 1));
-            }
-            // p of box rows w..w+2 (cell rows j-1..j+1), columns k-1..k+2 of the
-            // previous plane; the previous plane's per-cell corner sums
-            double pp[3][4];
-#pragma unroll
-            for (int r = 0; r < 3; r++)
-#pragma unroll
-                for (int c = 0; c < 4; c++) pp[r][c] = 0.0;
-            double pA0 = 0.0, pA1 = 0.0, pB0 = 0.0, pB1 = 0.0, pE0 = 0.0, pE1 = 0.0;
-            for (int n = 0; n < nst; n++) {
-                const int I = ia - 1 + n, slot = n % W_NSLOT;
-                mbar_wait(full0 + 8 * slot, (n / W_NSLOT) & 1);
-                const double* p1 = P_of(slot);
-                double pc[3][4];
-#pragma unroll
-                for (int r = 0; r < 3; r++) {
-                    const double* b = p1 + (w + r) * WPW + l2;
-                    const double2 v = rows_ok ? lds2(b + 2) : make_double2(0.0, 0.0);
-                    pc[r][0] = rows_ok ? (lfix ? p1[O_PL + 2 * (w + r) + 1] : b[1]) : 0.0;
-                    pc[r][1] = v.x;
-                    pc[r][2] = v.y;
-                    pc[r][3] = rows_ok ? (rfix ? p1[O_PR + 2 * (w + r)] : b[4]) : 0.0;
-                }
-                if (n > 0 && rows_ok) {
-                    // corners of plane I: rows q = 0 (J = j0+w), 1; columns K = l2 + kk
-                    const double* Cf = C_of(slot);
-                    const double* CS = p1 + O_CS;
-                    double SA[3], BD[3], SE[3];
-#pragma unroll
-                    for (int q = 0; q < 2; q++) {
-                        const double* cr = Cf + (w + q) * WCW + l2;
-                        const double2 a01 = lds2(cr), b01 = lds2(cr + WCA), e01 = lds2(cr + 2 * WCA);
-                        double ca[3] = {a01.x, a01.y, cr[2]};
-                        double cb[3] = {b01.x, b01.y, cr[WCA + 2]};
-                        double ce[3] = {e01.x, e01.y, cr[2 * WCA + 2]};
-                        if (rfix) {  // corner column k0 + width = np: the side box (K = 0)
-                            ca[2] = CS[2 * (w + q)];
-                            cb[2] = CS[2 * (WCR + w + q)];
-                            ce[2] = CS[2 * (2 * WCR + w + q)];
-                        }
-#pragma unroll
-                        for (int kk = 0; kk < 3; kk++) {
-                            const double a00 = pp[q][kk], a01v = pp[q][kk + 1], a10 = pp[q + 1][kk],
-                                         a11 = pp[q + 1][kk + 1];
-                            const double b00 = pc[q][kk], b01v = pc[q][kk + 1], b10 = pc[q + 1][kk],
-                                         b11 = pc[q + 1][kk + 1];
-                            const double Dr = ((b00 - a00) + (b01v - a01v)) + ((b10 - a10) + (b11 - a11));
-                            const double Dt = ((a10 - a00) + (a11 - a01v)) + ((b10 - b00) + (b11 - b01v));
-                            const double Dp = ((a01v - a00) + (a11 - a10)) + ((b01v - b00) + (b11 - b10));
-                            const double sc = ca[kk] * Dr + cb[kk] * Dt + ce[kk] * Dp;
-                            if (q == 0) {
-                                SA[kk] = sc * ca[kk];
-                                BD[kk] = sc * cb[kk];
-                                SE[kk] = sc * ce[kk];
-                                // sigma: the tile's own corners (row < height, column <
-                                // width) of the segment's own planes
-                                if (MODE == MODE_PCGA && kk < 2 && I < ib && l2 + kk < width) acc[0] += sc * sc;
-                            } else {
-                                SA[kk] += sc * ca[kk];
-                                BD[kk] -= sc * cb[kk];
-                                SE[kk] += sc * ce[kk];
-                            }
-                        }
-                    }
-                    const double A0 = SA[0] + SA[1], A1 = SA[1] + SA[2];
-                    const double B0 = BD[0] + BD[1], B1 = BD[1] + BD[2];
-                    const double E0 = SE[0] - SE[1], E1 = SE[1] - SE[2];
-                    // ---- cells (w, l2..l2+1) of plane i = I-1: corner planes i, I
-                    if (n >= 2 && active) {
-                        const int i = I - 1;
-                        const double s0 = ((pA0 - A0) + (pB0 + B0)) + (pE0 + E0);
-                        const double s1 = ((pA1 - A1) + (pB1 + B1)) + (pE1 + E1);
-                        const double ivr = __ldg(a.ivr + i);
-                        const double y0 = s0 * (ivr * cw0), y1 = s1 * (ivr * cw1);
-#ifdef MAS_ANISO_QTMA
-                        const double2 qv = lds2(Q_of(slot) + w * WK + l2);
-#else
-                        const double2 qv = ld2(a.out + (size_t)i * plane + (size_t)(j0 + w) * g.np + k0 + l2);
-#endif
-                        double* o = a.out + (size_t)i * plane + (size_t)(j0 + w) * g.np + k0 + l2;
-                        if (MODE == MODE_RESID) {
-                            const double r0 = qv.x - y0, r1 = qv.y - y1;
-                            stg2(o, make_double2(r0, r1));
-                            const double vr = __ldg(g.vr + i);
-                            const double V0 = vr / cw0, V1 = vr / cw1;
-                            const double2 f = ld2(a.f + (o - a.out));
-                            const double2 di = ld2(a.dinv + (o - a.out));
-                            acc[0] += V0 * f.x * f.x + V1 * f.y * f.y;
-                            acc[1] += V0 * r0 * r0 + V1 * r1 * r1;
-                            acc[2] += V0 * r0 * (di.x * r0) + V1 * r1 * (di.y * r1);
-                        } else {
-                            stg2(o, make_double2(qv.x + y0, qv.y + y1));
-                        }
-                    }
-                    pA0 = A0, pA1 = A1, pB0 = B0, pB1 = B1, pE0 = E0, pE1 = E1;
-                }
-#pragma unroll
-                for (int r = 0; r < 3; r++)
-#pragma unroll
-                    for (int c = 0; c < 4; c++) pp[r][c] = pc[r][c];
-                // this stage is no longer read (its p is in registers now)
-                fence_proxy_async();
-                __syncwarp();
-                if (lane == 0) mbar_arrive(empty0 + 8 * slot);
-            }
-#elif defined(MAS_ANISO_V3)
-            // ---- consumers V3: pair sums ------------------------------------
-            // Warp J owns corner row J (J = 0..WJ: 17 consumer warps).  Each lane
-            // computes its corners (J, c2), (J, c2+1), lane 31 also (J, 64); the
-            // column neighbour's combinations come by shuffle, and the lane forms
-            //   P1 = o0(c) + o1(c+1)   lower part of cell (J, c) from row J
-            //   P2 = o2(c) + o3(c+1)   lower part of cell (J-1, c) from row J
-            //   P3 = o3(c) + o2(c+1)   upper part of cell (J, c) from row J
-            //   P4 = o1(c) + o0(c+1)   upper part of cell (J-1, c) from row J
-            // It keeps P1 (for the next step) and P3 in registers and stores P2,
-            // P4 for the warp of row J-1, into arrays 0 and 1 of the slot's
-            // corner region in place of the coefficients it read.  A cell then
-            // reads 2 aligned double2 instead of 12 values of the 4 combination
-            // arrays; the sums are V1's, in V1's order (bitwise equal).
-            static_assert(WQ_SLOT > 0, "MAS_ANISO_V3 needs the out/q TMA box");
-            constexpr int NR = 1;
-            const int c2 = 2 * lane;
-            const bool first = k0 == 0, last = k0 + width == g.np;
-            const bool lfix = first && c2 == 0, rfix = last && c2 == width;
-            const bool xcol = lane == 31 && width == WK;  // the extra corner (J, 64)
-            int rowJ[NR];
-            bool rok[NR], cok[NR];
-            double cw0[NR], cw1[NR];
-#pragma unroll
-            for (int r = 0; r < NR; r++) {
-                const int J = warp;
-                rowJ[r] = J;
-                rok[r] = J <= height && c2 <= width;
-                cok[r] = J < height && c2 < width;
-                cw0[r] = cw1[r] = 0.0;
-                if (cok[r]) {
-                    const double vt = __ldg(g.vt + j0 + J);
-                    cw0[r] = 1.0 / (vt * __ldg(g.vp + k0 + c2));
-                    cw1[r] = 1.0 / (vt * __ldg(g.vp + k0 + c2 + 1));
-                }
-            }
-            auto corner_math = [&](double a00, double a01, double a10, double a11, double b00, double b01,
-                                   double b10, double b11, double A0, double B0, double E0, double& o0,
-                                   double& o1, double& o2, double& o3) -> double {
-                const double Dr = ((b00 - a00) + (b01 - a01)) + ((b10 - a10) + (b11 - a11));
-                const double Dt = ((a10 - a00) + (a11 - a01)) + ((b10 - b00) + (b11 - b01));
-                const double Dp = ((a01 - a00) + (a11 - a10)) + ((b01 - b00) + (b11 - b10));
-                const double sc = A0 * Dr + B0 * Dt + E0 * Dp;
-                const double A = sc * A0, B = sc * B0, E = sc * E0;
-                o0 = (A + B) + E;
-                o1 = (A + B) - E;
-                o2 = (A - B) + E;
-                o3 = (A - B) - E;
-                return sc;
-            };
-            // p of a plane for row J's corners: the pair (X0 / Y0: column c2-1 of
-            // rows J-1 / J; X12 / Y12: columns c2, c2+1) and the extra corner's
-            // cells 63, 64 (EX); wrap cells from the side boxes.  Both planes of a
-            // corner come from the ring (stage n-1 is released after step n), so
-            // no p is carried in registers (a 9-warp block gets 168 registers).
-            auto load_p = [&](const double* pb, int J, double& X0, double& Y0, double2& X12, double2& Y12,
-                              double (&EX)[4]) {
-                const double* q1 = pb + J * WPW + c2;
-                X0 = q1[1], Y0 = q1[WPW + 1];
-                X12 = lds2(q1 + 2), Y12 = lds2(q1 + WPW + 2);
-                if (lfix) X0 = pb[O_PL + 2 * J + 1], Y0 = pb[O_PL + 2 * J + 3];
-                if (rfix) X12.x = pb[O_PR + 2 * J], Y12.x = pb[O_PR + 2 * J + 2];
-                EX[0] = EX[1] = EX[2] = EX[3] = 0.0;
-                if (xcol) {  // cells 63, 64 of rows J-1, J (box columns 65, 66)
-                    const double* e = pb + J * WPW + WK + 1;
-                    EX[0] = e[0], EX[1] = e[1], EX[2] = e[WPW], EX[3] = e[WPW + 1];
-                    if (last) EX[1] = pb[O_PR + 2 * J], EX[3] = pb[O_PR + 2 * J + 2];
-                }
-            };
-            double2 p1prev[NR];  // P1 of the previous corner plane
-#pragma unroll
-            for (int r = 0; r < NR; r++) p1prev[r] = make_double2(0.0, 0.0);
-            double ivr_cur = 0.0;
-            for (int n = 0; n < nst; n++) {
-                const int I = ia - 1 + n, slot = n % W_NSLOT;
-                const double ivr_here = ivr_cur;
-                if (cok[0] && n + 1 >= 2 && n + 1 < nst) ivr_cur = __ldg(a.ivr + I);
-                mbar_wait(full0 + 8 * slot, (n / W_NSLOT) & 1);
-                const double* p1 = P_of(slot);
-                if (n == 0) continue;  // stage ia-1: p plane ia-1 only (read at step 1)
-                const double* p0 = P_of((n - 1) % W_NSLOT);
-                double* Cf = C_of(slot);
-                double2 p1now[NR], p3now[NR];
-#pragma unroll
-                for (int r = 0; r < NR; r++) {
-                    const int J = rowJ[r];
-                    double o[2][4] = {{0.0, 0.0, 0.0, 0.0}, {0.0, 0.0, 0.0, 0.0}};
-                    double ox[4] = {0.0, 0.0, 0.0, 0.0};
-                    if (rok[r]) {
-                        double x0, y0, X0, Y0, ex[4], EX[4];
-                        double2 x12, y12, X12, Y12;
-                        load_p(p0, J, x0, y0, x12, y12, ex);
-                        load_p(p1, J, X0, Y0, X12, Y12, EX);
-                        const double* c0 = Cf + J * WCW + c2;
-                        double2 A0 = lds2(c0), B0 = lds2(c0 + WCA), C0 = lds2(c0 + 2 * WCA);
-                        if (rfix) {
-                            const double* CS = p1 + O_CS;
-                            A0.x = CS[2 * J], B0.x = CS[2 * (WCR + J)], C0.x = CS[2 * (2 * WCR + J)];
-                        }
-                        const double s0 = corner_math(x0, x12.x, y0, y12.x, X0, X12.x, Y0, Y12.x, A0.x, B0.x,
-                                                      C0.x, o[0][0], o[0][1], o[0][2], o[0][3]);
-                        const double s1 = corner_math(x12.x, x12.y, y12.x, y12.y, X12.x, X12.y, Y12.x, Y12.y,
-                                                      A0.y, B0.y, C0.y, o[1][0], o[1][1], o[1][2], o[1][3]);
-                        if (MODE == MODE_PCGA && I < ib && J < height && c2 < width) acc[0] += s0 * s0 + s1 * s1;
-                        if (xcol) {
-                            const double* cx = Cf + J * WCW + WK;
-                            double A = cx[0], B = cx[WCA], E = cx[2 * WCA];
-                            if (last) {
-                                const double* CS = p1 + O_CS;
-                                A = CS[2 * J], B = CS[2 * (WCR + J)], E = CS[2 * (2 * WCR + J)];
-                            }
-                            corner_math(ex[0], ex[1], ex[2], ex[3], EX[0], EX[1], EX[2], EX[3], A, B, E, ox[0],
-                                        ox[1], ox[2], ox[3]);
-                        }
-                    }
-                    // the combinations of corner (J, c2+2): lane+1's first corner, or the extra one
-                    double nb[4];
-#pragma unroll
-                    for (int q = 0; q < 4; q++) {
-                        nb[q] = __shfl_down_sync(0xffffffffu, o[0][q], 1);
-                        if (lane == 31) nb[q] = ox[q];
-                    }
-                    p1now[r] = make_double2(o[0][0] + o[1][1], o[1][0] + nb[1]);
-                    p3now[r] = make_double2(o[0][3] + o[1][2], o[1][3] + nb[2]);
-                    if (rok[r]) {
-                        double* c0 = Cf + J * WCW + c2;  // its own coefficient positions (read above)
-                        sts2(c0, make_double2(o[0][2] + o[1][3], o[1][2] + nb[3]));        // P2
-                        sts2(c0 + WCA, make_double2(o[0][1] + o[1][0], o[1][1] + nb[0]));  // P4
-                    }
-                }
-                consumer_sync();
-                if (n >= 2) {
-                    const int i = I - 1;
-                    const double* Cp = C_of((n - 1) % W_NSLOT);
-#pragma unroll
-                    for (int r = 0; r < NR; r++) {
-                        if (!cok[r]) continue;
-                        const int J = rowJ[r];
-                        const double2 s2 = lds2(Cp + (J + 1) * WCW + c2);       // P2 of row J+1, plane I-1
-                        const double2 s4 = lds2(Cf + WCA + (J + 1) * WCW + c2); // P4 of row J+1, plane I
-                        const double s0 = (p1prev[r].x + s2.x) - (p3now[r].x + s4.x);
-                        const double s1 = (p1prev[r].y + s2.y) - (p3now[r].y + s4.y);
-                        const double yy0 = s0 * (ivr_here * cw0[r]), yy1 = s1 * (ivr_here * cw1[r]);
-                        const double2 qv = lds2(Q_of(slot) + J * WK + c2);
-                        double* o = a.out + (size_t)i * plane + (size_t)(j0 + J) * g.np + k0 + c2;
-                        if (MODE == MODE_RESID) {
-                            const double r0 = qv.x - yy0, r1 = qv.y - yy1;
-                            stg2(o, make_double2(r0, r1));
-                            const double vr = __ldg(g.vr + i);
-                            const double V0 = vr / cw0[r], V1 = vr / cw1[r];
-                            const double2 f = ld2(a.f + (o - a.out));
-                            const double2 di = ld2(a.dinv + (o - a.out));
-                            acc[0] += V0 * f.x * f.x + V1 * f.y * f.y;
-                            acc[1] += V0 * r0 * r0 + V1 * r1 * r1;
-                            acc[2] += V0 * r0 * (di.x * r0) + V1 * r1 * (di.y * r1);
-                        } else {
-                            stg2(o, make_double2(qv.x + yy0, qv.y + yy1));
-                        }
-                    }
-                }
-#pragma unroll
-                for (int r = 0; r < NR; r++) p1prev[r] = p1now[r];
-                fence_proxy_async();
-                __syncwarp();
-                if (lane == 0) mbar_arrive(empty0 + 8 * ((n - 1) % W_NSLOT));
-            }
-#elif MAS_ANISO_RPW > 1
-            // ---- consumers, RPW rows per warp (experiment: fewer warps, RPW
-            // independent row chains per thread; V1's arithmetic row by row)
-            static_assert(WQ_SLOT > 0, "MAS_ANISO_RPW > 1 needs the out/q TMA box");
-            const int c2 = 2 * lane;
-            const bool first = k0 == 0, last = k0 + width == g.np;
-            const bool lfix = first && c2 == 0, rfix = last && c2 == width;
-            bool crow_ok[RPW], cell_ok[RPW];
-            double cw0[RPW], cw1[RPW];
-#pragma unroll
-            for (int r = 0; r < RPW; r++) {
-                const int w = warp + r * NCW;
-                crow_ok[r] = w <= height && c2 <= width;
-                cell_ok[r] = w < height && c2 < width;
-                cw0[r] = cw1[r] = 0.0;
-                if (cell_ok[r]) {
-                    const double vt = __ldg(g.vt + j0 + w);
-                    cw0[r] = 1.0 / (vt * __ldg(g.vp + k0 + c2));
-                    cw1[r] = 1.0 / (vt * __ldg(g.vp + k0 + c2 + 1));
-                }
-            }
-            int xr = -1, xc = 0;  // extra corner: row WJ / column 64
-            {
-                const int t = threadIdx.x;
-                if (height == WJ && t <= width) {
-                    xr = WJ, xc = t;
-                } else if (width == WK && t >= WK + 1 && t - (WK + 1) < min(height + 1, WJ)) {
-                    xr = t - (WK + 1), xc = WK;
-                }
-            }
-            auto corner_math = [&](double a00, double a01, double a10, double a11, double b00, double b01,
-                                   double b10, double b11, double A0, double B0, double E0, double& o0,
-                                   double& o1, double& o2, double& o3) -> double {
-                const double Dr = ((b00 - a00) + (b01 - a01)) + ((b10 - a10) + (b11 - a11));
-                const double Dt = ((a10 - a00) + (a11 - a01)) + ((b10 - b00) + (b11 - b01));
-                const double Dp = ((a01 - a00) + (a11 - a10)) + ((b01 - b00) + (b11 - b10));
-                const double sc = A0 * Dr + B0 * Dt + E0 * Dp;
-                const double A = sc * A0, B = sc * B0, E = sc * E0;
-                o0 = (A + B) + E;
-                o1 = (A + B) - E;
-                o2 = (A - B) + E;
-                o3 = (A - B) - E;
-                return sc;
-            };
-            double x0[RPW], y0[RPW], e0 = 0.0, e1 = 0.0, e2 = 0.0, e3 = 0.0;
-            double2 x12[RPW], y12[RPW];
-#pragma unroll
-            for (int r = 0; r < RPW; r++) x0[r] = y0[r] = 0.0, x12[r] = y12[r] = make_double2(0.0, 0.0);
-            double ivr_cur = 0.0;
-            for (int n = 0; n < nst; n++) {
-                const int I = ia - 1 + n, slot = n % W_NSLOT;
-                const double ivr_here = ivr_cur;
-                if (cell_ok[0] && n + 1 >= 2 && n + 1 < nst) ivr_cur = __ldg(a.ivr + I);
-                mbar_wait(full0 + 8 * slot, (n / W_NSLOT) & 1);
-                const double* p1 = P_of(slot);
-                double X0[RPW], Y0[RPW], E0 = 0.0, E1 = 0.0, E2 = 0.0, E3 = 0.0;
-                double2 X12[RPW], Y12[RPW];
-#pragma unroll
-                for (int r = 0; r < RPW; r++) {
-                    const int w = warp + r * NCW;
-                    X0[r] = Y0[r] = 0.0;
-                    X12[r] = Y12[r] = make_double2(0.0, 0.0);
-                    if (crow_ok[r]) {
-                        const double* q1 = p1 + w * WPW + c2;
-                        X0[r] = q1[1], Y0[r] = q1[WPW + 1];
-                        X12[r] = lds2(q1 + 2), Y12[r] = lds2(q1 + WPW + 2);
-                        if (lfix) X0[r] = p1[O_PL + 2 * w + 1], Y0[r] = p1[O_PL + 2 * w + 3];
-                        if (rfix) X12[r].x = p1[O_PR + 2 * w], Y12[r].x = p1[O_PR + 2 * w + 2];
-                    }
-                }
-                if (xr >= 0) {
-                    const double* q1 = p1 + xr * WPW + xc + 1;
-                    E0 = q1[0], E1 = q1[1], E2 = q1[WPW], E3 = q1[WPW + 1];
-                    if (first && xc == 0) E0 = p1[O_PL + 2 * xr + 1], E2 = p1[O_PL + 2 * xr + 3];
-                    if (last && xc == width) E1 = p1[O_PR + 2 * xr], E3 = p1[O_PR + 2 * xr + 2];
-                }
-                if (n == 0) {
-#pragma unroll
-                    for (int r = 0; r < RPW; r++) x0[r] = X0[r], y0[r] = Y0[r], x12[r] = X12[r], y12[r] = Y12[r];
-                    e0 = E0, e1 = E1, e2 = E2, e3 = E3;
-                    continue;
-                }
-                double* Cf = C_of(slot);
-#pragma unroll
-                for (int r = 0; r < RPW; r++) {
-                    const int w = warp + r * NCW;
-                    if (crow_ok[r]) {
-                        double* c0 = Cf + w * WCW + c2;
-                        double2 A0 = lds2(c0), B0 = lds2(c0 + WCA), C0 = lds2(c0 + 2 * WCA);
-                        if (rfix) {
-                            const double* CS = p1 + O_CS;
-                            A0.x = CS[2 * w], B0.x = CS[2 * (WCR + w)], C0.x = CS[2 * (2 * WCR + w)];
-                        }
-                        double o[2][4];
-                        const double s0 = corner_math(x0[r], x12[r].x, y0[r], y12[r].x, X0[r], X12[r].x, Y0[r],
-                                                      Y12[r].x, A0.x, B0.x, C0.x, o[0][0], o[0][1], o[0][2], o[0][3]);
-                        const double s1 = corner_math(x12[r].x, x12[r].y, y12[r].x, y12[r].y, X12[r].x, X12[r].y,
-                                                      Y12[r].x, Y12[r].y, A0.y, B0.y, C0.y, o[1][0], o[1][1],
-                                                      o[1][2], o[1][3]);
-#pragma unroll
-                        for (int q = 0; q < 4; q++) sts2(c0 + q * WCA, make_double2(o[0][q], o[1][q]));
-                        if (MODE == MODE_PCGA && I < ib && w < height && c2 < width) acc[0] += s0 * s0 + s1 * s1;
-                    }
-                }
-                if (xr >= 0) {
-                    double* c0 = Cf + xr * WCW + xc;
-                    double A = c0[0], B = c0[WCA], E = c0[2 * WCA];
-                    if (last && xc == width) {
-                        const double* CS = p1 + O_CS;
-                        A = CS[2 * xr], B = CS[2 * (WCR + xr)], E = CS[2 * (2 * WCR + xr)];
-                    }
-                    double o0, o1, o2, o3;
-                    corner_math(e0, e1, e2, e3, E0, E1, E2, E3, A, B, E, o0, o1, o2, o3);
-                    c0[0] = o0;
-                    c0[WCA] = o1;
-                    c0[2 * WCA] = o2;
-                    c0[3 * WCA] = o3;
-                }
-#pragma unroll
-                for (int r = 0; r < RPW; r++) x0[r] = X0[r], y0[r] = Y0[r], x12[r] = X12[r], y12[r] = Y12[r];
-                e0 = E0, e1 = E1, e2 = E2, e3 = E3;
-                consumer_sync();
-                if (n >= 2) {
-                    const int i = I - 1;
-#pragma unroll
-                    for (int r = 0; r < RPW; r++) {
-                        const int w = warp + r * NCW;
-                        if (!cell_ok[r]) continue;
-                        const double* l = C_of((n - 1) % W_NSLOT) + w * WCW + c2;
-                        const double* h = Cf + w * WCW + c2;
-                        const double2 l0 = lds2(l), l2 = lds2(l + 2 * WCA + WCW);
-                        const double2 h3 = lds2(h + 3 * WCA), h1 = lds2(h + WCA + WCW);
-                        const double l1a = l[WCA + 1], l1b = l[WCA + 2];
-                        const double l3a = l[3 * WCA + WCW + 1], l3b = l[3 * WCA + WCW + 2];
-                        const double h2a = h[2 * WCA + 1], h2b = h[2 * WCA + 2];
-                        const double h0a = h[WCW + 1], h0b = h[WCW + 2];
-                        const double s0 = ((l0.x + l1a) + (l2.x + l3a)) - ((h3.x + h2a) + (h1.x + h0a));
-                        const double s1 = ((l0.y + l1b) + (l2.y + l3b)) - ((h3.y + h2b) + (h1.y + h0b));
-                        const double yy0 = s0 * (ivr_here * cw0[r]), yy1 = s1 * (ivr_here * cw1[r]);
-                        const double2 qv = lds2(Q_of(slot) + w * WK + c2);
-                        double* o = a.out + (size_t)i * plane + (size_t)(j0 + w) * g.np + k0 + c2;
-                        if (MODE == MODE_RESID) {
-                            const double r0 = qv.x - yy0, r1 = qv.y - yy1;
-                            stg2(o, make_double2(r0, r1));
-                            const double vr = __ldg(g.vr + i);
-                            const double V0 = vr / cw0[r], V1 = vr / cw1[r];
-                            const double2 f = ld2(a.f + (o - a.out));
-                            const double2 di = ld2(a.dinv + (o - a.out));
-                            acc[0] += V0 * f.x * f.x + V1 * f.y * f.y;
-                            acc[1] += V0 * r0 * r0 + V1 * r1 * r1;
-                            acc[2] += V0 * r0 * (di.x * r0) + V1 * r1 * (di.y * r1);
-                        } else {
-                            stg2(o, make_double2(qv.x + yy0, qv.y + yy1));
-                        }
-                    }
-                }
-                fence_proxy_async();
-                __syncwarp();
-                if (lane == 0) mbar_arrive(empty0 + 8 * ((n - 1) % W_NSLOT));
-            }
-#else
             // ---- consumers --------------------------------------------------
             const int w = warp, c2 = 2 * lane;
             const bool first = k0 == 0, last = k0 + width == g.np;
@@ -894,78 +395,17 @@ __global__ void __launch_bounds__(WTHREADS, kAnisoBps) k_aniso(const AnisoArgs a
             // the extra corner's 4 cells); wrap cells from the side boxes
             double x0 = 0.0, y0 = 0.0, e0 = 0.0, e1 = 0.0, e2 = 0.0, e3 = 0.0;
             double2 x12 = make_double2(0.0, 0.0), y12 = x12;
-#ifndef MAS_ANISO_QTMA
-            // out/q of the cells: plain coalesced loads (no shared-memory round
-            // trip, which the MIO pipe is short of), one step ahead of their use
-            // (step n processes the cells of plane I-1; the load of step n+1's
-            // plane I is issued at step n)
-            const size_t qoff = (size_t)(j0 + w) * g.np + k0 + c2;
-            double2 qnext = make_double2(0.0, 0.0);
-#endif
             // 1/vr of the cell plane of the next step, loaded one step ahead
             // (its latency sat on the cell phase's dependency chain)
             double ivr_cur = 0.0;
-#ifdef MAS_ANISO_LAG
-            static_assert(WQ_SLOT > 0, "MAS_ANISO_LAG needs the out/q TMA box");
-            // cells (w, c2..c2+1) of plane i: corner planes i (slot sl, sr = +1)
-            // and i+1 (slot sh, sr = -1); out/q plane i from slot sh's box
-            auto gather = [&](int i, int sl, int sh, double ivr) {
-                if (!cell_ok) return;
-                const double* l = C_of(sl) + w * WCW + c2;
-                const double* h = C_of(sh) + w * WCW + c2;
-                const double2 l0 = lds2(l), l2 = lds2(l + 2 * WCA + WCW);
-                const double2 h3 = lds2(h + 3 * WCA), h1 = lds2(h + WCA + WCW);
-                const double l1a = l[WCA + 1], l1b = l[WCA + 2];
-                const double l3a = l[3 * WCA + WCW + 1], l3b = l[3 * WCA + WCW + 2];
-                const double h2a = h[2 * WCA + 1], h2b = h[2 * WCA + 2];
-                const double h0a = h[WCW + 1], h0b = h[WCW + 2];
-                const double s0 = ((l0.x + l1a) + (l2.x + l3a)) - ((h3.x + h2a) + (h1.x + h0a));
-                const double s1 = ((l0.y + l1b) + (l2.y + l3b)) - ((h3.y + h2b) + (h1.y + h0b));
-                const double yy0 = s0 * (ivr * cw0), yy1 = s1 * (ivr * cw1);
-                const double2 qv = lds2(Q_of(sh) + w * WK + c2);
-                double* o = a.out + (size_t)i * plane + (size_t)(j0 + w) * g.np + k0 + c2;
-                if (MODE == MODE_RESID) {
-                    const double r0 = qv.x - yy0, r1 = qv.y - yy1;
-                    stg2(o, make_double2(r0, r1));
-                    const double vr = __ldg(g.vr + i);
-                    const double V0 = vr / cw0, V1 = vr / cw1;
-                    const double2 f = ld2(a.f + (o - a.out));
-                    const double2 di = ld2(a.dinv + (o - a.out));
-                    acc[0] += V0 * f.x * f.x + V1 * f.y * f.y;
-                    acc[1] += V0 * r0 * r0 + V1 * r1 * r1;
-                    acc[2] += V0 * r0 * (di.x * r0) + V1 * r1 * (di.y * r1);
-                } else {
-                    stg2(o, make_double2(qv.x + yy0, qv.y + yy1));
-                }
-            };
-#endif
             for (int n = 0; n < nst; n++) {
                 const int I = ia - 1 + n, slot = n % W_NSLOT;
                 const double ivr_here = ivr_cur;
-#ifdef MAS_ANISO_LAG
-                if (cell_ok && n >= 2) ivr_cur = __ldg(a.ivr + I - 1);  // the gather of step n+1 / the epilogue
-#else
                 if (cell_ok && n + 1 >= 2 && n + 1 < nst) ivr_cur = __ldg(a.ivr + I);
-#endif
-#if !defined(MAS_ANISO_QTMA) && !defined(MAS_ANISO_QNOW)
-                const double2 qv = qnext;
-                if (n + 1 >= 2 && n + 1 < nst && cell_ok) qnext = ld2(a.out + (size_t)I * plane + qoff);
-#elif !defined(MAS_ANISO_QTMA)
-                (void)qnext;  // A/B hook: the load of this step's q at the top of the step
-                double2 qv = make_double2(0.0, 0.0);
-                if (n >= 2 && cell_ok) qv = ld2(a.out + (size_t)(I - 1) * plane + qoff);
-#endif
                 mbar_wait(full0 + 8 * slot, (n / W_NSLOT) & 1);
 #ifdef MAS_ANISO_DIAG_NOCOMPUTE
                 // diagnostic build (wrong results): the consumers only wait for
                 // each stage and release it -- the producer / TMA pipeline alone
-                // (MAS_ANISO_DIAG_STORE: plus the q store of the cells)
-#ifdef MAS_ANISO_DIAG_STORE
-                if (n >= 2 && cell_ok) {
-                    const double2 qv = lds2(Q_of(slot) + w * WK + c2);
-                    stg2(a.out + (size_t)(I - 1) * plane + (size_t)(j0 + w) * g.np + k0 + c2, qv);
-                }
-#endif
                 if (n >= 1) {
                     __syncwarp();
                     if (lane == 0) mbar_arrive(empty0 + 8 * ((n - 1) % W_NSLOT));
@@ -1029,33 +469,7 @@ __global__ void __launch_bounds__(WTHREADS, kAnisoBps) k_aniso(const AnisoArgs a
                     c0[3 * WCA] = o3;
                 }
                 x0 = X0, y0 = Y0, x12 = X12, y12 = Y12, e0 = E0, e1 = E1, e2 = E2, e3 = E3;
-#ifdef MAS_ANISO_QST
-                // every warp has finished step n-1's cells (written into stage
-                // n-1's out box): one thread stores that box with the TMA engine
-                // (plane I-2); its warp waits until the box is read before the
-                // stage is released below
                 consumer_sync();
-                if (threadIdx.x == 0 && n >= 3) {
-                    tma_store3(&M.out, k0, j0, I - 2, smem_u32(Q_of((n - 1) % W_NSLOT)));
-                    bulk_commit();
-                }
-#endif
-#ifdef MAS_ANISO_LAG
-                // software pipeline: the cells of plane I-2 (corner planes I-2, I-1,
-                // complete since the last barrier) next to the corners of plane I,
-                // one barrier per step; stage n-2 is released after it
-                if (n >= 3) gather(I - 2, (n - 2) % W_NSLOT, (n - 1) % W_NSLOT, ivr_here);
-                consumer_sync();
-                if (n >= 2) {
-                    fence_proxy_async();
-                    __syncwarp();
-                    if (lane == 0) mbar_arrive(empty0 + 8 * ((n - 2) % W_NSLOT));
-                }
-                continue;
-#endif
-#ifndef MAS_ANISO_QST
-                consumer_sync();
-#endif
                 // ---- cells (w, c2..c2+1) of plane i = I-1: corner planes i
                 // (sr = +1) and I (sr = -1); out/q plane i from this stage
                 if (n >= 2 && cell_ok) {
@@ -1072,21 +486,11 @@ __global__ void __launch_bounds__(WTHREADS, kAnisoBps) k_aniso(const AnisoArgs a
                     const double s1 = ((l0.y + l1b) + (l2.y + l3b)) - ((h3.y + h2b) + (h1.y + h0b));
                     const double ivr = ivr_here;  // 1/vr of plane i = I-1
                     const double y0 = s0 * (ivr * cw0), y1 = s1 * (ivr * cw1);
-#ifdef MAS_ANISO_QTMA
                     const double2 qv = lds2(Q_of(slot) + w * WK + c2);
-#endif
                     double* o = a.out + (size_t)i * plane + (size_t)(j0 + w) * g.np + k0 + c2;
-#ifdef MAS_ANISO_QST
-                    double* qs = Q_of(slot) + w * WK + c2;  // the result goes back into the out box
-                    (void)o;
-#endif
                     if (MODE == MODE_RESID) {
                         const double r0 = qv.x - y0, r1 = qv.y - y1;
-#ifdef MAS_ANISO_QST
-                        sts2(qs, make_double2(r0, r1));
-#else
                         stg2(o, make_double2(r0, r1));
-#endif
                         const double vr = __ldg(g.vr + i);
                         const double V0 = vr / cw0, V1 = vr / cw1;
                         const double2 f = ld2(a.f + (o - a.out));
@@ -1095,39 +499,16 @@ __global__ void __launch_bounds__(WTHREADS, kAnisoBps) k_aniso(const AnisoArgs a
                         acc[1] += V0 * r0 * r0 + V1 * r1 * r1;
                         acc[2] += V0 * r0 * (di.x * r0) + V1 * r1 * (di.y * r1);
                     } else {
-#if defined(MAS_ANISO_QST)
-                        sts2(qs, make_double2(qv.x + y0, qv.y + y1));
-#elif !defined(MAS_ANISO_DIAG_NOSTORE)  // diagnostic build (wrong results): no q store
                         stg2(o, make_double2(qv.x + y0, qv.y + y1));
-#else
-                        if (qv.x + y0 == 1.2345e-300) stg2(o, make_double2(qv.x + y0, qv.y + y1));
-#endif
                     }
                 }
                 // stage n-1 is no longer read (p by corners(I), products by
                 // cells(I-1)); the combination writes went through the generic
                 // proxy, the next fill of the slot is a tensor copy
                 fence_proxy_async();
-#ifdef MAS_ANISO_QST
-                if (threadIdx.x == 0 && n >= 3) bulk_wait_read0();  // stage n-1's out box has left
-#endif
                 __syncwarp();
                 if (lane == 0) mbar_arrive(empty0 + 8 * ((n - 1) % W_NSLOT));
             }
-#ifdef MAS_ANISO_LAG
-            // the last cell plane ib-1 (corner planes ib-1, ib: the last two stages)
-            if (nst >= 3) gather(ib - 1, (nst - 2) % W_NSLOT, (nst - 1) % W_NSLOT, ivr_cur);
-#endif
-#ifdef MAS_ANISO_QST
-            // the segment's last out box (plane ib-1), after every warp's cells
-            consumer_sync();
-            if (threadIdx.x == 0 && nst >= 3) {
-                tma_store3(&M.out, k0, j0, ib - 1, smem_u32(Q_of((nst - 1) % W_NSLOT)));
-                bulk_commit();
-                bulk_wait0();  // complete before the next segment reuses the ring / the kernel ends
-            }
-#endif
-#endif
         }
         __syncthreads();  // the next segment re-initialises the rings and barriers
     }
