@@ -376,6 +376,8 @@ def main():
     ap.add_argument("--tol", type=float, default=1e-12)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-replay", action="store_true",
+                    help="skip the kernel-replay timing (e.g. for an ncu launch list of the timed steps only)")
     ap.add_argument("--cpu-iters", type=int, default=6)
     ap.add_argument("--solver", default="pcg", choices=["pcg", "cg1"],
                     help="pcg: two fused kernels / two reductions per iteration; cg1: the "
@@ -546,7 +548,7 @@ def main():
     # device time per launch of the iteration kernels from back-to-back CUDA
     # graph replays (no host dispatch between launches; mas_op_kernel_bench)
     replay = None
-    if world == 1:
+    if world == 1 and not args.no_replay:
         ra, rb, rc = op.kernel_bench(20)
         replay = {"A_ms": ra, "B_ms": rb or None, "Lpar_ms": rc or None,
                   "note": "20 launches of each kernel in a CUDA graph on the op's stream, each "

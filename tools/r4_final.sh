@@ -1,0 +1,29 @@
+#!/bin/bash
+# Closing session of round 2 (second half): full GPU suite, smoke, every bench
+# line, the staggered stack bench, launch lists and fresh ncu --set full
+# captures of C3 kernel A and k_aniso<PCGA>.  Outputs gpurun_out/${TAG}_*.
+cd "$(dirname "$0")/.."
+O=gpurun_out; TAG=${TAG:-r4z}; NCU=/usr/local/cuda/bin/ncu
+python -c "import __graft_entry__ as g; g.build()" > $O/${TAG}_build.log 2>&1 || exit 1
+timeout 1500 python -m pytest tests -m gpu -q > $O/${TAG}_gputest.log 2>&1
+echo "gpu suite rc=$?: $(tail -1 $O/${TAG}_gputest.log)"
+python -c "import __graft_entry__ as g; g.smoke()" > $O/${TAG}_smoke.log 2>&1; echo "smoke rc=$?"
+python bench.py > $O/${TAG}_bench_C3.log 2>&1
+python bench.py --impl reference > $O/${TAG}_bench_C3_reference.log 2>&1
+for cfg in C2 C2a C2t C1; do python bench.py --config $cfg > $O/${TAG}_bench_$cfg.log 2>&1; done
+python bench.py --config C2 --solver cg1 --no-cpu-baseline > $O/${TAG}_bench_C2_cg1.log 2>&1
+python bench.py --config C1 --solver cg1 --no-cpu-baseline > $O/${TAG}_bench_C1_cg1.log 2>&1
+python bench.py --solver cg1 --no-cpu-baseline --no-e2e > $O/${TAG}_bench_C3_cg1.log 2>&1
+python bench.py --config C3s8 --no-cpu-baseline --no-e2e > $O/${TAG}_bench_C3s8.log 2>&1
+python tools/stack_bench.py > $O/${TAG}_stack_bench.json 2> $O/${TAG}_stack_bench.err
+for f in $O/${TAG}_bench_*.log; do echo "$f: $(tail -1 $f | cut -c1-160)"; done
+$NCU --metrics gpu__time_duration.sum --clock-control none -c 400 --csv --log-file $O/${TAG}_launches_C3.csv \
+  python bench.py --steps 2 --warmup 1 --no-cpu-baseline --no-e2e --no-replay > /dev/null 2>&1
+$NCU --metrics gpu__time_duration.sum --clock-control none -c 600 --csv --log-file $O/${TAG}_launches_C2a.csv \
+  python bench.py --config C2a --steps 2 --warmup 1 --no-cpu-baseline --no-e2e --no-replay > /dev/null 2>&1
+MAS_NO_GRAPH=1 $NCU --set full --clock-control none --import-source on -k regex:k_stencil --launch-skip 2 --launch-count 1 \
+  -f -o $O/${TAG}_C3_kernelA python tools/prof_driver.py --config C3 > /dev/null 2>&1
+MAS_NO_GRAPH=1 $NCU --set full --clock-control none --import-source on -k regex:k_aniso --launch-skip 3 --launch-count 1 \
+  -f -o $O/${TAG}_C2a_kaniso python tools/prof_driver.py --config C2a > /dev/null 2>&1
+grep -E "FAILED" $O/${TAG}_gputest.log | head
+ls -la $O/${TAG}_*.ncu-rep
