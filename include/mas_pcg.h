@@ -396,8 +396,9 @@ MAS_API mas_status_t mas_op_radial_sums(const mas_op_t* op, const double* x, con
  *     GPU without a mas_dist_t, no P2P, no single-reduction loop, no
  *     field-aligned term (MAS_ERR_ARG otherwise).  The stack keeps the op
  *     pointers (not the ops): destroy the stack before its ops.
- *   mas_stack_solve: rhs[b], x[b] DEVICE arrays of op b's shape
- *     ([comp][nl][nt][np] of its placement); x in = x0, out = solution;
+ *   mas_stack_solve: rhs[b], x[b] arrays of op b's shape ([comp][nl][nt][np]
+ *     of its placement), device or host (staged like mas_pcg_solve); x in =
+ *     x0, out = solution;
  *     tol, maxit, iters, relres, res_hist as mas_pcg_solve (the stacked
  *     residual).  Runs on `stream` (every op's work goes there; the single-GPU
  *     CUDA-graph loop with one k_stack_sum node after each kernel round).

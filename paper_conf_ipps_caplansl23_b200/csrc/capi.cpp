@@ -2180,9 +2180,28 @@ mas_status_t mas_stack_solve(mas_stack_t* sk, const double* const* rhs, double* 
     if (!sk || !rhs || !x || !iters || !relres) return arg_error("null argument");
     if (!(tol >= 0.0) || maxit < 0) return arg_error("need tol >= 0 and maxit >= 0");
     const size_t n = sk->ops.size();
+    // host arrays are staged through each op's library-owned device buffers
+    // (as mas_pcg_solve does); device arrays are used in place
+    std::vector<const double*> fd(n);
+    std::vector<double*> xd(n);
+    std::vector<bool> hx(n, false);
     for (size_t m = 0; m < n; m++) {
         if (!rhs[m] || !x[m]) return arg_error("null rhs or x");
-        if (!is_device_ptr(rhs[m]) || !is_device_ptr(x[m])) return arg_error("stacked solve: device arrays");
+        mas_op* op = sk->ops[m];
+        const size_t bytes = op->ncomp * op->Nl * sizeof(double);
+        fd[m] = rhs[m];
+        xd[m] = x[m];
+        const bool hf = !is_device_ptr(rhs[m]);
+        hx[m] = !is_device_ptr(x[m]);
+        if (hf || hx[m]) ST(ensure_stage(op));
+        if (hf) {
+            CU(cudaMemcpyAsync(op->stage_a, rhs[m], bytes, cudaMemcpyHostToDevice, s));
+            fd[m] = op->stage_a;
+        }
+        if (hx[m]) {
+            CU(cudaMemcpyAsync(op->stage_b, x[m], bytes, cudaMemcpyHostToDevice, s));
+            xd[m] = op->stage_b;
+        }
     }
     const StackStates ss = stack_states(sk);
     std::vector<StencilArgs> a(n);
@@ -2200,12 +2219,11 @@ mas_status_t mas_stack_solve(mas_stack_t* sk, const double* const* rhs, double* 
         CU(cudaMemcpyAsync(op->st, &init, sizeof(init), cudaMemcpyHostToDevice, s));
         *op->host_flag = 0;
         const int nc = op->ncomp;
-        double* xd = x[m];
-        ST(pole_pass(op, xd, nc, s));
+        ST(pole_pass(op, xd[m], nc, s));
         StencilArgs& A = a[m];
         A.g = op->geo;
         A.chunk = op->chunk;
-        A.u = halo_of(op, xd, op->xg, nc);
+        A.u = halo_of(op, xd[m], op->xg, nc);
         A.kappa = halo_of(op, op->kappa, op->kg, 1);
         A.dinv = halo_of(op, op->dinv, op->dg, 1);
         A.tu = packed_rows(op, op->xgt, nc);
@@ -2213,7 +2231,7 @@ mas_status_t mas_stack_solve(mas_stack_t* sk, const double* const* rhs, double* 
         A.tdinv = packed_rows(op, op->dgt, 1);
         A.c = op->c;
         A.curv = op->curv;
-        A.f = rhs[m];
+        A.f = fd[m];
         A.out = op->r;
         A.st = op->st;
         A.rho_hist = op->hist;
@@ -2224,13 +2242,13 @@ mas_status_t mas_stack_solve(mas_stack_t* sk, const double* const* rhs, double* 
         CU(launch_stencil(MODE_RESID, nc, A, s));
         if (op->tnode) {  // the caps' residuals, then the three sums again
             ST(pole_pass(op, op->r, nc, s));
-            CU(launch_init_dots(op->geo, nc, rhs[m], op->r, op->dinv, op->scr, op->st, op->b_blocks, s));
+            CU(launch_init_dots(op->geo, nc, fd[m], op->r, op->dinv, op->scr, op->st, op->b_blocks, s));
         }
         // the iteration arguments (kernel A: p from r; kernel B)
         A.u = r_halo(op);
         A.tu = r_trows(op);
         A.out = op->q;
-        A.x = xd;
+        A.x = xd[m];
         A.f = nullptr;
         StreamArgs& B = b[m];
         B.g = op->geo;
@@ -2287,6 +2305,9 @@ mas_status_t mas_stack_solve(mas_stack_t* sk, const double* const* rhs, double* 
                       cudaMemcpyDeviceToHost));
         for (int k = 0; k < nh; k++) res_hist[k] = std::sqrt(rr[k]);
     }
+    for (size_t m = 0; m < n; m++)
+        if (hx[m])
+            CU(cudaMemcpy(x[m], xd[m], sk->ops[m]->ncomp * sk->ops[m]->Nl * sizeof(double), cudaMemcpyDeviceToHost));
     return (mas_status_t)fin.status;
 }
 

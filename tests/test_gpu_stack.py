@@ -207,8 +207,13 @@ def test_zero_rhs_and_refusals(mp):
     with pytest.raises(mp.MasError):
         mp.Stack([])
     sk = mp.Stack([op, op2])
-    with pytest.raises(mp.MasError):            # host arrays
-        sk.solve([f, f], [x0.copy(), x0.copy()], 1e-10, 10)
+    # host arrays: staged through the ops' device buffers, same result as device arrays
+    xh = [x0.copy(), x0.copy()]
+    st_h, it_h, rel_h, _ = sk.solve([f, f], xh, 1e-10, 500)
+    xd = [dev(x0), dev(x0)]
+    st_d, it_d, rel_d, _ = sk.solve([dev(f), dev(f)], xd, 1e-10, 500)
+    assert (st_h, it_h, rel_h) == (st_d, it_d, rel_d) and st_h == mp.MAS_OK
+    assert np.array_equal(xh[0], host(xd[0])) and np.array_equal(xh[1], host(xd[1]))
     sk.close()
     op2.close()
     c1 = make_blocks(shape, [(0, 1, (0, 1))], seed=1)[0]
