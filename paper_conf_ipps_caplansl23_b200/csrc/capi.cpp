@@ -1835,6 +1835,9 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
     b.host_flag = op->host_flag_dev;
     b.p2p = p2p_args(op);
     b.aniso = op->aniso && !lpar_in_a(op);  // P2P: sigma's L_par part in its own slot (MB_C)
+    b.x = xd;  // a breakdown at an even k completes x's two-iteration update
+    b.p[0] = op->p[0];
+    b.p[1] = op->p[1];
 
     // a4: iterations.  Kernel A(k) reads k, alpha, beta and the convergence
     // decision from PcgState; the host only keeps two iterations in flight
@@ -2262,6 +2265,9 @@ mas_status_t mas_stack_solve(mas_stack_t* sk, const double* const* rhs, double* 
         B.rr_hist = A.rr_hist;
         B.scr = op->scr;
         B.host_flag = op->host_flag_dev;
+        B.x = xd[m];
+        B.p[0] = op->p[0];
+        B.p[1] = op->p[1];
     }
     CU(launch_stack_sum(ss, 1, 3, s));  // rho_0, ||r_0||^2, ||f||^2 of the stacked vector
     bool graph = true;

@@ -299,6 +299,13 @@ __device__ __forceinline__ void trow_issue(const StencilArgs& a, int i, const Ha
     }
 }
 
+// PCGA: the two-iteration x update (x read and written by every second kernel
+// A, which also reads p_{k-2}) for the scalar operator.  The 3-component kernel
+// keeps the one-step update: with p_{k-2} in registers it spills, and loaded
+// at commit time it measured 4% slower at C3 (profiles/README.md)
+template <int NC>
+constexpr bool kX2 = (NC == 1);
+
 // --- L2 prefetch one plane ahead of the register pipeline -----------------
 // The own-tile loads of plane i+2 are issued (into registers) before the
 // stencil of plane i.  Before that, plane i+3's tile rows are prefetched into
@@ -332,7 +339,8 @@ __device__ __forceinline__ void plane_prefetch(const StencilArgs& a, int i, int 
     // fields: u[NC], po[NC] (PCGA, not first), x[NC] (xupd), dinv (PCGA), kappa, c
     // (+ CG1: w[NC], the own p[NC])
     constexpr bool KRY = MODE == MODE_PCGA || MODE == MODE_CG1;
-    constexpr int NF = 3 * NC + 3 + (MODE == MODE_CG1 ? 2 * NC : 0);
+    // (+ PCGA, kX2, with the x update: p_{k-2} from the p_k buffer, fields 3NC+3..)
+    constexpr int NF = 3 * NC + 3 + (MODE == MODE_CG1 ? 2 * NC : (MODE == MODE_PCGA && kX2<NC> ? NC : 0));
     const int t = threadIdx.x;
     if (t >= NF * TJ) return;
     const int f = t / TJ, w = t - f * TJ;
@@ -346,6 +354,7 @@ __device__ __forceinline__ void plane_prefetch(const StencilArgs& a, int i, int 
     else if (f == 3 * NC) base = KRY ? a.dinv.in : nullptr;
     else if (f == 3 * NC + 1) base = a.kappa.in;
     else if (f == 3 * NC + 2) base = a.c;
+    else if (MODE == MODE_PCGA) base = (kX2<NC> && xupd) ? a.pnew + (f - 3 * NC - 3) * Nl : nullptr;
     else if (f < 4 * NC + 3) base = (MODE == MODE_CG1 && !first) ? a.w.in + (f - 3 * NC - 3) * Nl : nullptr;
     else base = (MODE == MODE_CG1 && xupd) ? a.pnew + (f - 4 * NC - 3) * Nl : nullptr;
     if (base) l2_prefetch_row(base + off, width * 8);
@@ -388,7 +397,7 @@ __device__ __forceinline__ void stage_issue(const StencilArgs& a, int i, int j0,
 #pragma unroll
                 for (int c = 0; c < NC; c++) S.xv[c] = lds2(a.x + c * Nl + o3);
             }
-            if (MODE == MODE_CG1 && !kCg1LateOwn<NC> && xupd) {
+            if (((MODE == MODE_CG1 && !kCg1LateOwn<NC>) || (MODE == MODE_PCGA && kX2<NC>)) && xupd) {
 #pragma unroll
                 for (int c = 0; c < NC; c++) S.pp[c] = lds2(a.pnew + c * Nl + o3);
             }
@@ -442,7 +451,8 @@ __device__ __forceinline__ void stage_issue(const StencilArgs& a, int i, int j0,
 template <int MODE, int NC, bool LPAR = false>
 __device__ __forceinline__ void stage_commit(const StencilArgs& a, int i, int j0, int k0, int height,
                                              int width, const HaloMeta& hm, bool first, double beta,
-                                             double alpha_prev, bool xupd, bool halo, bool own_work,
+                                             double alpha_prev, double alpha_km2, bool xupd, bool halo,
+                                             bool own_work,
                                              Stage<NC>& S, double* buf, double2& kown,
                                              OwnRegs<NC>& o, const double* hst, double (&acc)[3]) {
     const Geo& g = a.g;
@@ -506,13 +516,20 @@ __device__ __forceinline__ void stage_commit(const StencilArgs& a, int i, int j0
                 const int o3 = (int)i * plane32(g) + (int)(j0 + w) * g.np + k0 + kc;
 #pragma unroll
                 for (int c = 0; c < NC; c++) {
-                    stg2a(a.pnew + c * Nl + o3, S.R.u[c]);
                     if (xupd) {
                         double2 xv = S.xv[c];
+                        if constexpr (kX2<NC>) {
+                            // odd k >= 3: x += alpha_{k-2} p_{k-2} + alpha_{k-1} p_{k-1},
+                            // the two fmas of two one-step updates (p_{k-2} was loaded
+                            // one plane ahead, before p_k overwrites it)
+                            xv.x = fma(alpha_km2, S.pp[c].x, xv.x);
+                            xv.y = fma(alpha_km2, S.pp[c].y, xv.y);
+                        }
                         xv.x = fma(alpha_prev, S.R.po[c].x, xv.x);
                         xv.y = fma(alpha_prev, S.R.po[c].y, xv.y);
                         stg2a(a.x + c * Nl + o3, xv);
                     }
+                    stg2a(a.pnew + c * Nl + o3, S.R.u[c]);
                 }
             }
         }
@@ -691,6 +708,7 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
     double cg_g1 = 0.0, cg_d1 = 0.0, cg_rr1 = 0.0;
     int cg_status = -1, cg_iters = 0;
     double beta = 0.0, alpha_prev = 0.0;
+    double alpha_km2 = 0.0;  // PCGA: alpha_{k-2} (saved by A(k-1))
     int kit = 0;
     const bool p2p = a.p2p.nranks > 0;
     __shared__ double final_g[3];
@@ -713,6 +731,7 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
         const double sig1 = __ldcg(&st->sigma_prev);
         first = (kit == 1);
         if (kit >= 2) alpha_prev = rho2 / sig1;
+        if (kit >= 3) alpha_km2 = __ldcg(&st->alpha_save);
         if (first && ff == 0.0)
             pmode = P_ZERO;
         else if (sqrt(rr) <= __ldcg(&st->tol) * sqrt(ff) || kit > __ldcg(&st->maxit))
@@ -760,7 +779,13 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
             }
         }
     }
-    const bool xupd = (MODE == MODE_PCGA || MODE == MODE_CG1) && !FIRSTK;
+    // the deferred x update.  PCGA, scalar (kX2): every other kernel A, odd
+    // k >= 3, applies the last two steps, x += alpha_{k-2} p_{k-2} + alpha_{k-1}
+    // p_{k-1} (the same two fmas as two one-step updates; x read and written
+    // every second iteration only, p_{k-2} read then).  PCGA,
+    // 3 components: every kernel A, x += alpha_{k-1} p_{k-1}.  CG1: every kernel.
+    const bool xupd = MODE == MODE_PCGA ? (!FIRSTK && (!kX2<NC> || ((kit & 1) && kit >= 3)))
+                                        : (MODE == MODE_CG1 && !FIRSTK);
     if (MODE == MODE_PCGA && pmode == P_NORMAL && FIRSTK != first) __trap();  // host dispatch bug
 
     // ---- work item ------------------------------------------------------
@@ -794,8 +819,16 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
                     if (pmode == P_ZERO) {
                         stg2(xp, make_double2(0.0, 0.0));
                     } else if (MODE == MODE_PCGA && kit >= 2) {
+                        // the pending steps of the two-iteration update: alpha_{k-1}
+                        // p_{k-1}, and for odd k also alpha_{k-2} p_{k-2} (still in
+                        // the p_k buffer: this kernel writes no p_k)
                         const double2 po = ld2(plane_ptr(a.pold, c, i, g) + off);
                         double2 xv = lds2(xp);
+                        if (kX2<NC> && (kit & 1)) {
+                            const double2 pp = lds2(a.pnew + c * Nl + (int)i * plane32(g) + off);
+                            xv.x = fma(alpha_km2, pp.x, xv.x);
+                            xv.y = fma(alpha_km2, pp.y, xv.y);
+                        }
                         xv.x = fma(alpha_prev, po.x, xv.x);
                         xv.y = fma(alpha_prev, po.y, xv.y);
                         stg2(xp, xv);
@@ -903,14 +936,14 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
     if (!lo_ghost) {
         stage_issue<MODE, NC, LPAR>(a, ia - 1, j0, k0, height, width, hm, FIRSTK, false, LPAR, false, S0, hst_arr);
         if (LPAR)
-            stage_commit<MODE, NC, LPAR>(a, ia - 1, j0, k0, height, width, hm, FIRSTK, beta, alpha_prev, false,
+            stage_commit<MODE, NC, LPAR>(a, ia - 1, j0, k0, height, width, hm, FIRSTK, beta, alpha_prev, alpha_km2, false,
                                    true, false, S0, slot(ia - 1), kdummy, on, hst_arr, acc);
     }
     stage_issue<MODE, NC, LPAR>(a, ia, j0, k0, height, width, hm, FIRSTK, xupd, true, true, S, hst_arr);
     if (!lo_ghost && !LPAR)
-        stage_commit<MODE, NC, LPAR>(a, ia - 1, j0, k0, height, width, hm, FIRSTK, beta, alpha_prev, false,
+        stage_commit<MODE, NC, LPAR>(a, ia - 1, j0, k0, height, width, hm, FIRSTK, beta, alpha_prev, alpha_km2, false,
                                false, false, S0, slot(ia - 1), kdummy, on, hst_arr, acc);
-    stage_commit<MODE, NC, LPAR>(a, ia, j0, k0, height, width, hm, FIRSTK, beta, alpha_prev, xupd, true, true,
+    stage_commit<MODE, NC, LPAR>(a, ia, j0, k0, height, width, hm, FIRSTK, beta, alpha_prev, alpha_km2, xupd, true, true,
                            S, slot(ia), kown, oc, hst_arr, acc);
     if (lo_ghost) ghost_plane<NC>(slot(ia - 1), height, width, kown, LPAR);
     if (LPAR) {  // corner plane ia (cells ia-1 | ia): its lower-corner part for plane ia
@@ -936,7 +969,7 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
         // commit plane i+1 (its loads were issued one plane earlier)
         if (real_plane(i + 1))
             stage_commit<MODE, NC, LPAR>(a, i + 1, j0, k0, height, width, hm, FIRSTK, beta, alpha_prev,
-                                   xupd && (i + 1 < ib), LPAR || i + 1 < ib, i + 1 < ib, S, slot(i + 1),
+                                   alpha_km2, xupd && (i + 1 < ib), LPAR || i + 1 < ib, i + 1 < ib, S, slot(i + 1),
                                    kown, on, hst_arr, acc);
         else
             ghost_plane<NC>(slot(i + 1), height, width, kown, LPAR);
@@ -1111,6 +1144,7 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
                 a.rr_hist[kit - 1] = rr;
                 a.rho_hist[kit - 1] = rho1;
                 st->rho_prev = rho1;  // rho_{k-1}, read as rho_{(k+1)-2} by A(k+1)
+                st->alpha_save = alpha_prev;  // alpha_{k-1}: A(k+1)'s alpha_{k-2}, B(k)'s fix-up
                 if (p2p) {
                     // globals for B(k) (alpha, breakdown report) and later A's
                     st->pend_rho = rho1;
@@ -1156,6 +1190,16 @@ __global__ void __launch_bounds__(kThreads) k_pcg_b(const StreamArgs a) {
     const bool brk = !(sigma > 0.0) || !isfinite(sigma);
     const double alpha = __ldcg(&vst->pend_rho) / sigma;  // rho_{k-1} / sigma_k
     double acc[2] = {0.0, 0.0};
+    if (kX2<NC> && brk && a.x && kit >= 2 && !(kit & 1)) {
+        // breakdown at an even k: A(k) left x at x_{k-2} (two-iteration
+        // update); the solve reports x_{k-1} = x_{k-2} + alpha_{k-1} p_{k-1}
+        const double am1 = __ldcg(&vst->alpha_save);
+        const double* pk1 = a.p[(kit - 1) & 1];
+        const long long n = (long long)a.ncomp * g.nl * g.plane;
+        for (long long e = blockIdx.x * (long long)blockDim.x + threadIdx.x; e < n;
+             e += (long long)gridDim.x * blockDim.x)
+            a.x[e] = fma(am1, pk1[e], a.x[e]);
+    }
     if (!brk) {
         const long long Nl = (long long)g.nl * g.plane;
         const int rows = g.nl * g.nt;

@@ -106,6 +106,9 @@ struct PcgState {
     double cg_alpha;    // alpha_k
     double cg_beta;     // beta_k
     double cg_gamma;    // gamma_k = <r_k, D^-1 r_k>_V
+    // the two-iteration x update: alpha_{k-1} as A(k) used
+    // it, saved by A(k)'s last block for A(k+1) and for B(k)'s breakdown fix-up
+    double alpha_save;
 };
 
 struct Scratch {
@@ -167,6 +170,10 @@ struct StreamArgs {  // kernel B
     unsigned long long cond;
     P2P p2p;
     int aniso;                // the field-aligned term is on: sigma also from MB_C (P2P)
+    // the two-iteration x update: on a breakdown in B(k), k even, the pending
+    // x += alpha_{k-1} p_{k-1} (p_j lives in p[j & 1]); x == nullptr: none
+    double* x;
+    const double* p[2];
 };
 
 // ---------------------------------------------------------------------------
