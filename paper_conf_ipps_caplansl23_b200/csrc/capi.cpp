@@ -1838,6 +1838,11 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
     b.x = xd;  // a breakdown at an even k completes x's two-iteration update
     b.p[0] = op->p[0];
     b.p[1] = op->p[1];
+    {  // test hook: a breakdown forced in B(k) (tests of the breakdown paths)
+        const char* t = getenv("MAS_TEST_TRANSPORTS");
+        const char* k = getenv("MAS_TEST_BREAKDOWN_AT");
+        b.brk_at = (t && atoi(t) == 1 && k) ? atoi(k) : 0;
+    }
 
     // a4: iterations.  Kernel A(k) reads k, alpha, beta and the convergence
     // decision from PcgState; the host only keeps two iterations in flight

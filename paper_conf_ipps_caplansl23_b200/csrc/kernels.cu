@@ -1187,7 +1187,7 @@ __global__ void __launch_bounds__(kThreads) k_pcg_b(const StreamArgs a) {
         __syncthreads();
         sigma = sh_sigma;
     }
-    const bool brk = !(sigma > 0.0) || !isfinite(sigma);
+    const bool brk = !(sigma > 0.0) || !isfinite(sigma) || (a.brk_at > 0 && kit == a.brk_at);
     const double alpha = __ldcg(&vst->pend_rho) / sigma;  // rho_{k-1} / sigma_k
     double acc[2] = {0.0, 0.0};
     if (kX2<NC> && brk && a.x && kit >= 2 && !(kit & 1)) {

@@ -174,6 +174,7 @@ struct StreamArgs {  // kernel B
     // x += alpha_{k-1} p_{k-1} (p_j lives in p[j & 1]); x == nullptr: none
     double* x;
     const double* p[2];
+    int brk_at;               // test hook (MAS_TEST_TRANSPORTS=1 + MAS_TEST_BREAKDOWN_AT=k): B(k) breaks down
 };
 
 // ---------------------------------------------------------------------------
