@@ -65,8 +65,8 @@ def alg_bytes_per_cell(ncomp):
     if ncomp == 1:
         # scalar operator: x is read and written by every second kernel A (the
         # two-iteration x update), which then also reads p_{k-2}; per launch on
-        # average 2 doubles less and half a double more (72 -> 68 B)
-        a += -16 + 4
+        # average one double less and half a double more (72 -> 68 B)
+        a += -8 + 4
     b = 8 * (2 * ncomp + 1 + ncomp)
     return a, b
 
