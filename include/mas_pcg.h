@@ -242,6 +242,10 @@ MAS_API mas_status_t mas_pcg_solve(const mas_op_t* op, const double* rhs, double
  * library-owned r, p and mailbox buffers, with the handles all-gathered over
  * the grid's NCCL communicator; the init residual, op setup/update seams and
  * mas_op_dot keep NCCL.  With one rank the mailbox path runs against itself.
+ * With the single-reduction loop switched on BEFORE this call, its ping-pong
+ * buffers are mapped too: each of its kernels publishes its 3 partial sums
+ * to every rank's mailbox (two slots alternating by parity) and the next
+ * kernel sums them there -- NEXT-1's allreduce fused into the kernels.
  * Errors: MAS_ERR_CUDA on every rank if any rank cannot map its peers (the op
  * then keeps the NCCL loop); MAS_ERR_NCCL.  A mailbox wait longer than 60 s
  * traps the kernel (fails loudly rather than hanging). */
@@ -262,9 +266,13 @@ MAS_API mas_status_t mas_op_enable_p2p(mas_op_t* op, cudaStream_t stream);
  * more vectors.  On r-slabs the NCCL loop runs ONE 3-double allreduce per
  * iteration (two in the two-kernel loop) plus the seams of r, w and s; kernel
  * k+1 takes the stop / alpha / beta decision from the allreduced sums, so
- * every rank decides alike.  on == 0 restores the two-kernel loop.
- * Errors: MAS_ERR_ARG with the P2P transport, ptheta > 1, the field-aligned
- * term, the theta-node placement or the curvature terms; MAS_ERR_NOMEM. */
+ * every rank decides alike.  Over the P2P transport (mas_op_enable_p2p
+ * called after this) the reduction happens in the kernels through the
+ * mailbox, and the r, w, s halos are read in place.  on == 0 restores the
+ * two-kernel loop.
+ * Errors: MAS_ERR_ARG after mas_op_enable_p2p of an op without the loop on,
+ * ptheta > 1, the field-aligned term, the theta-node placement or the
+ * curvature terms; MAS_ERR_NOMEM. */
 MAS_API mas_status_t mas_op_set_single_reduction(mas_op_t* op, int on);
 
 /* Vector-Laplacian curvature terms (reading R31,

@@ -134,6 +134,10 @@ struct mas_op {
     Mail** d_peers = nullptr;          // device array [nranks] of every rank's mailbox
     std::vector<void*> ipc_opened;     // cudaIpcOpenMemHandle mappings (closed at destroy)
     const double* nb_r[2] = {nullptr, nullptr};  // rank-1 / rank+1 r arrays
+    // the single-reduction loop's other ping-pong buffers of the r-neighbours
+    // (r2, w = q, w2), mapped when the loop was on before mas_op_enable_p2p
+    const double* nb_cg[3][2] = {{nullptr, nullptr}, {nullptr, nullptr}, {nullptr, nullptr}};
+    int p2p_cg1 = 0;
     const double* nb_p[2][2] = {{nullptr, nullptr}, {nullptr, nullptr}};  // [parity][lo/hi]
     int nb_nl[2] = {0, 0};             // their slab sizes
     unsigned long long epoch = 0;      // solves so far (mailbox sequence numbers)
@@ -699,9 +703,18 @@ static void cg1_args(const mas_op* op, int k, StencilArgs& a) {
     double* R[2] = {op->r, op->r2};
     double* Wb[2] = {op->q, op->w2};
     double* S[2] = {op->p[0], op->p[1]};
-    a.u = halo_of(op, R[(k - 1) & 1], op->rg, nc);
-    a.w = halo_of(op, Wb[(k - 1) & 1], op->pg[0], nc);
-    a.pold = halo_of(op, S[k & 1], op->pg[1], nc);
+    if (op->p2p) {  // the r-neighbours' buffers of the same parity, read in place
+        const double* const* nR[2] = {op->nb_r, op->nb_cg[0]};
+        const double* const* nW[2] = {op->nb_cg[1], op->nb_cg[2]};
+        const int ru = (k - 1) & 1, rs = k & 1;
+        a.u = peer_halo(op, R[ru], nR[ru][0], nR[ru][1]);
+        a.w = peer_halo(op, Wb[ru], nW[ru][0], nW[ru][1]);
+        a.pold = peer_halo(op, S[rs], op->nb_p[rs][0], op->nb_p[rs][1]);
+    } else {
+        a.u = halo_of(op, R[(k - 1) & 1], op->rg, nc);
+        a.w = halo_of(op, Wb[(k - 1) & 1], op->pg[0], nc);
+        a.pold = halo_of(op, S[k & 1], op->pg[1], nc);
+    }
     a.sout = S[(k - 1) & 1];
     a.rout = R[k & 1];
     a.out = Wb[k & 1];
@@ -723,7 +736,7 @@ static mas_status_t cg1_graph(mas_op* op, StencilArgs a) {
                                                   cudaStreamCaptureModeThreadLocal);
     if (e == cudaSuccess) {
         StencilArgs a0 = a;
-        a0.u = halo_of(op, op->r, nullptr, nc);
+        a0.u = op->p2p ? peer_halo(op, op->r, op->nb_r[0], op->nb_r[1]) : halo_of(op, op->r, nullptr, nc);
         a0.out = op->q;
         e = launch_stencil(MODE_CG1, nc, a0, op->cap_stream, true);
         cudaGraph_t out = g;
@@ -792,7 +805,9 @@ static mas_status_t cg1_solve(mas_op* op, const double* fd, double* xd, double t
     Comm* comm = op->g->comm;
     const long long plane = op->geo.plane;
     op->launches = 0;
+    const bool p2p = op->p2p != 0;
     PcgState init{};
+    if (p2p) init.epoch = ++op->epoch;
     init.tol = tol;
     init.maxit = maxit;
     init.k = 0;
@@ -819,20 +834,24 @@ static mas_status_t cg1_solve(mas_op* op, const double* fd, double* xd, double t
     a.rr_hist = rr_h;
     a.scr = op->scr;
     a.host_flag = op->host_flag_dev;
+    // P2P transport: every kernel publishes its 3 partial sums to every rank's
+    // mailbox and the next one sums them there (no host-side allreduce)
+    a.p2p = p2p_args(op);
     // a3: r0 = f - L x0 and <f,f>, <r0,r0> (k_stencil<RESID>, as the standard loop)
     if (comm) ST(comm_seams(comm, xd, nc, op->g->nl, plane, op->xg, op->xg + nc * plane, s));
     StencilArgs r0 = a;
     r0.u = halo_of(op, xd, op->xg, nc);
     r0.f = fd;
     r0.out = op->r;
-    CU(launch_stencil(MODE_RESID, nc, r0, s));
+    if (p2p) ST(comm_vsync(comm, s));  // virtual P2P ranks: every rank's previous solve done
+    CU(launch_stencil(MODE_RESID, nc, r0, s));  // (P2P: publishes rho, rr, ff to slot B)
     op->launches++;
-    if (comm) {  // the init sums over the ranks; r0's edge planes for the init kernel
+    if (comm && !p2p) {  // the init sums over the ranks; r0's edge planes for the init kernel
         ST(comm_allreduce(comm, &op->st->pend_rho, 3, s));  // rho, rr, ff
         ST(comm_seams(comm, op->r, nc, op->g->nl, plane, op->rg, op->rg + nc * plane, s));
     }
     a.x = xd;
-    const bool graph = !op->prof && op->use_graph && !comm;
+    const bool graph = !op->prof && op->use_graph && (!comm || (p2p && !comm_is_virtual(comm)));
     if (graph) {
         ST(cg1_graph(op, a));
         CU(cudaGraphLaunch(op->gexec1, s));
@@ -846,13 +865,16 @@ static mas_status_t cg1_solve(mas_op* op, const double* fd, double* xd, double t
                 pe = &op->pev[6 * (size_t)(n - 1)];
                 CU(cudaEventRecord(pe[0], s));
             }
+            // virtual P2P ranks share one GPU: every rank's previous kernel done
+            // before a kernel that waits on their mailbox entries is launched
+            if (p2p) ST(comm_vsync(comm, s));
             if (n == 1) {
                 StencilArgs a0 = a;
-                a0.u = halo_of(op, op->r, op->rg, nc);
+                a0.u = p2p ? peer_halo(op, op->r, op->nb_r[0], op->nb_r[1]) : halo_of(op, op->r, op->rg, nc);
                 a0.out = op->q;
                 CU(launch_stencil(MODE_CG1, nc, a0, s, true));
             } else {
-                ST(cg1_seams(op, n - 1, s));
+                if (!p2p) ST(cg1_seams(op, n - 1, s));
                 if (pe) CU(cudaEventRecord(pe[0], s));
                 cg1_args(op, n - 1, a);
                 CU(launch_stencil(MODE_CG1, nc, a, s));
@@ -860,7 +882,7 @@ static mas_status_t cg1_solve(mas_op* op, const double* fd, double* xd, double t
             op->launches++;
             if (pe) CU(cudaEventRecord(pe[1], s));
             // the one allreduce of the iteration: (gamma, delta, ||r||^2) in place
-            if (comm) ST(comm_allreduce(comm, &op->st->pend_sigma, 3, s));
+            if (comm && !p2p) ST(comm_allreduce(comm, &op->st->pend_sigma, 3, s));
             CU(cudaEventRecord(op->ev[n & 1], s));
             if (n >= 2) {
                 ST(comm_wait_event(comm, op->ev[(n - 1) & 1]));
@@ -870,6 +892,9 @@ static mas_status_t cg1_solve(mas_op* op, const double* fd, double* xd, double t
         }
     }
     ST(comm_sync_stream(comm, s));
+    // P2P: no rank may publish the next solve's partials while another rank's
+    // kernels of this solve can still read its mailbox
+    if (p2p && comm) ST(comm_barrier(comm, s));
     PcgState fin{};
     CU(cudaMemcpy(&fin, op->st, sizeof(fin), cudaMemcpyDeviceToHost));
     if (!fin.stopped) {
@@ -1263,25 +1288,30 @@ mas_status_t mas_op_enable_p2p(mas_op_t* op, cudaStream_t s) {
     if (op->p2p) return MAS_OK;
     if (op->placement != MAS_PLACE_CELL)
         return arg_error("P2P transport: cell-centred placement only (the other placements keep NCCL)");
-    if (op->cg1) return arg_error("P2P transport: the two-kernel loop only (single reduction is on)");
+    if (op->cg1 && op->g->ptheta > 1) return arg_error("P2P transport with single reduction: r-slabs only");
     Comm* comm = op->g->comm;
     const int P = comm_nranks(comm), rank = comm_rank(comm);
     const bool virt = comm_is_virtual(comm);
     ST(dmalloc(&op->mbox, MB_SLOTS * (size_t)P));
     CU(cudaMemset(op->mbox, 0, MB_SLOTS * (size_t)P * sizeof(Mail)));
     struct Rec {
-        cudaIpcMemHandle_t h[4];
-        unsigned long long raw[4];
+        cudaIpcMemHandle_t h[7];
+        unsigned long long raw[7];
         int nl, ntl;
         int ok;
     };
     Rec mine;
     memset(&mine, 0, sizeof(mine));
-    const void* bufs[4] = {op->r, op->p[0], op->p[1], op->mbox};
+    // r, p[0], p[1], the mailbox; with the single-reduction loop on also its
+    // ping-pong buffers r2, w = q, w2 (r-neighbours' halos read in place)
+    const bool cg = op->cg1 != 0;
+    const void* bufs[7] = {op->r, op->p[0], op->p[1], op->mbox, cg ? op->r2 : nullptr, cg ? op->q : nullptr,
+                           cg ? op->w2 : nullptr};
     mine.nl = op->g->nl;
     mine.ntl = op->g->ntl;
     mine.ok = 1;
-    for (int b = 0; b < 4; b++) {
+    for (int b = 0; b < 7; b++) {
+        if (!bufs[b]) continue;
         mine.raw[b] = (unsigned long long)(uintptr_t)bufs[b];
         if (P > 1 && !virt && cudaIpcGetMemHandle(&mine.h[b], const_cast<void*>(bufs[b])) != cudaSuccess) {
             cudaGetLastError();
@@ -1314,6 +1344,7 @@ mas_status_t mas_op_enable_p2p(mas_op_t* op, cudaStream_t s) {
         op->nb_p[0][side] = (const double*)map(q, 1);
         op->nb_p[1][side] = (const double*)map(q, 2);
         op->nb_nl[side] = all[q].nl;
+        for (int b = 0; b < 3 && cg && ok; b++) op->nb_cg[b][side] = (const double*)map(q, 4 + b);
     }
     for (int side = 0; side < 2 && ok; side++) {  // theta neighbours (same r-slab)
         const int q = side == 0 ? op->tlo : op->thi;
@@ -1352,13 +1383,19 @@ mas_status_t mas_op_enable_p2p(mas_op_t* op, cudaStream_t s) {
         op->nbt_r[0] = op->nbt_r[1] = nullptr;
         op->nbt_p[0][0] = op->nbt_p[0][1] = op->nbt_p[1][0] = op->nbt_p[1][1] = nullptr;
         op->nb_p[0][0] = op->nb_p[0][1] = op->nb_p[1][0] = op->nb_p[1][1] = nullptr;
+        for (auto& v : op->nb_cg) v[0] = v[1] = nullptr;
         set_last_error("P2P transport unavailable: " + why);
         return MAS_ERR_CUDA;
     }
     op->p2p = 1;
+    op->p2p_cg1 = cg ? 1 : 0;
     if (op->gexec) {  // the loop graph reads the ghost planes differently now
         cudaGraphExecDestroy(op->gexec);
         op->gexec = nullptr;
+    }
+    if (op->gexec1) {
+        cudaGraphExecDestroy(op->gexec1);
+        op->gexec1 = nullptr;
     }
     return MAS_OK;
 }
@@ -1371,7 +1408,8 @@ mas_status_t mas_op_set_single_reduction(mas_op_t* op, int on) {
         op->cg1 = 0;
         return MAS_OK;
     }
-    if (op->p2p) return arg_error("single-reduction PCG: the NCCL loop on r-slabs (not the P2P transport)");
+    if (op->p2p && !op->p2p_cg1)
+        return arg_error("single-reduction PCG over the P2P transport: switch it on before mas_op_enable_p2p");
     if (op->g->ptheta > 1) return arg_error("single-reduction PCG: r-slab decompositions only (ptheta == 1)");
     if (op->aniso) return arg_error("single-reduction PCG: isotropic operator only (no mas_op_set_aniso)");
     if (op->placement != MAS_PLACE_CELL) return arg_error("single-reduction PCG: cell-centred placement only");

@@ -751,18 +751,34 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
             return;
         }
         kit = __ldcg(&st->k);
-        const double ff = __ldcg(&st->pend_ff);
+        double ff = __ldcg(&st->pend_ff);
+        // P2P transport: the global sums come from the mailbox, summed in rank
+        // order (the init's from k_stencil<RESID>'s slot B {rho, rr, ff};
+        // kernel k-1's {gamma, delta, ||r||^2} from slot A / C by its parity)
+        double pv[3] = {0.0, 0.0, 0.0};
+        if (p2p) {
+            __shared__ double sh_pv[3];
+            if (threadIdx.x == 0) {
+                const unsigned long long ep = __ldcg(&st->epoch);
+                if (FIRSTK) p2p_gather_one<3>(a.p2p, MB_B, p2p_seq(ep, 0), pv);
+                else p2p_gather_one<3>(a.p2p, ((kit - 1) & 1) ? MB_C : MB_A, p2p_seq(ep, kit - 1), pv);
+                sh_pv[0] = pv[0], sh_pv[1] = pv[1], sh_pv[2] = pv[2];
+            }
+            __syncthreads();
+            pv[0] = sh_pv[0], pv[1] = sh_pv[1], pv[2] = sh_pv[2];
+            if (FIRSTK) ff = pv[2];
+        }
         if (FIRSTK) {  // the init: k = 0; r0 from k_stencil<RESID>
-            const double rr = __ldcg(&st->pend_rr);
+            const double rr = p2p ? pv[1] : __ldcg(&st->pend_rr);
             final_g[0] = ff, final_g[1] = rr, final_g[2] = 0.0;
             if (ff == 0.0)
                 pmode = P_ZERO;
             else if (sqrt(rr) <= __ldcg(&st->tol) * sqrt(ff) || __ldcg(&st->maxit) == 0)
                 pmode = P_FINAL;
         } else {
-            cg_g1 = __ldcg(&st->pend_rho);
-            cg_d1 = __ldcg(&st->pend_sigma);
-            cg_rr1 = __ldcg(&st->pend_rr);
+            cg_g1 = p2p ? pv[0] : __ldcg(&st->pend_rho);
+            cg_d1 = p2p ? pv[1] : __ldcg(&st->pend_sigma);
+            cg_rr1 = p2p ? pv[2] : __ldcg(&st->pend_rr);
             if (kit >= 2 && sqrt(cg_rr1) <= __ldcg(&st->tol) * sqrt(ff)) {
                 pmode = P_FINAL, cg_status = MAS_OK, cg_iters = kit - 1;
             } else if (kit >= 2 && kit - 1 >= __ldcg(&st->maxit)) {
@@ -1114,7 +1130,7 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
             }
         }
     } else if (MODE == MODE_CG1) {
-        if (grid_reduce<3, kSThreads>(acc, a.scr, TKT_STENCIL) && threadIdx.x == 0) {
+        if (grid_reduce<3, kSThreads>(acc, a.scr, TKT_STENCIL, p2p) && threadIdx.x == 0) {
             // the single reduction of iteration k: this rank's gamma_k, delta_k,
             // ||r_k||^2 (summed over the ranks before kernel k+1 reads them).
             // Kernel k+1 decides; here the values it needs besides them.
@@ -1130,6 +1146,14 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
             st->pend_sigma = acc[1];
             st->pend_rr = acc[2];
             st->k = kit + 1;
+            if (p2p) {
+                if (FIRSTK) st->pend_ff = final_g[0];  // the global ||f||^2 for every later kernel
+                // the single reduction of iteration k: this rank's partials to
+                // every rank's mailbox (slots alternate by parity: a rank publishes
+                // k+2 only after every rank has consumed k)
+                const double pub[3] = {acc[0], acc[1], acc[2]};
+                p2p_publish(a.p2p, (kit & 1) ? MB_C : MB_A, p2p_seq(st->epoch, kit), pub, 3);
+            }
         }
     } else if (MODE == MODE_PCGA) {
         double v[1] = {acc[0]};

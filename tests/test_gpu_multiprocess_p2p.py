@@ -31,8 +31,8 @@ import json, sys
 import numpy as np, torch
 sys.path.insert(0, {root!r})
 from paper_conf_ipps_caplansl23_b200 import maspcg as M, workloads as W
-P, rank, d, kind, nr, nt, np_, p2p, pt = ({P}, int(sys.argv[1]), {d!r}, {kind!r}, {nr}, {nt}, {np_},
-                                          {p2p}, {ptheta})
+P, rank, d, kind, nr, nt, np_, p2p, pt, cg1 = ({P}, int(sys.argv[1]), {d!r}, {kind!r}, {nr}, {nt}, {np_},
+                                               {p2p}, {ptheta}, {cg1})
 torch.cuda.set_device(0)
 prob = W.make(kind, nr=nr, nt=nt, np_=np_, warm=False)
 g = M.Grid(prob.mesh, dist=(P, rank, M.host_exchange_id(d)), ptheta=pt)
@@ -40,6 +40,8 @@ sl = (slice(g.i0, g.i0 + g.nl), slice(g.j0, g.j0 + g.ntl))
 slc = (slice(None),) + sl
 dv = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()
 op = M.Operator(g, prob.ncomp, dv(prob.kappa[sl]), dv(prob.c[sl]), prob.bc_inner, prob.bc_outer)
+if cg1:  # the single-reduction loop first: enable_p2p then maps its buffers too
+    op.set_single_reduction(True)
 if p2p:
     op.enable_p2p()
 if prob.kpar is not None:  # field-aligned conduction: neighbour p_k through the IPC mapping
@@ -61,10 +63,10 @@ op.close(); g.close()
 """
 
 
-def run_procs(tmp_path, P, kind, shape, p2p=True, timeout=600, ptheta=1):
+def run_procs(tmp_path, P, kind, shape, p2p=True, timeout=600, ptheta=1, cg1=False):
     d = str(tmp_path)
     src = WORKER.format(root=ROOT, P=P, d=d, kind=kind, nr=shape[0], nt=shape[1], np_=shape[2],
-                        p2p=p2p, ptheta=ptheta)
+                        p2p=p2p, ptheta=ptheta, cg1=cg1)
     script = os.path.join(d, "worker.py")
     with open(script, "w") as fh:
         fh.write(src)
@@ -113,3 +115,25 @@ def test_p2p_across_processes_matches_oracle(built, oracle_mod, tmp_path, P, kin
         xg[:, r["i0"]:r["i0"] + r["nl"], r["j0"]:r["j0"] + r["ntl"]] = xl
     assert not np.isnan(xg).any()
     assert math.sqrt((V * (xg - xo) ** 2).sum() / (V * xo ** 2).sum()) <= 1e-10
+
+
+@pytest.mark.parametrize("P,kind,shape", [(2, "viscosity", (12, 16, 64)), (3, "conduction", (13, 16, 32))])
+def test_single_reduction_p2p_across_processes(built, oracle_mod, tmp_path, P, kind, shape):
+    """NEXT-1 over the P2P transport: each single-reduction kernel publishes its
+    3 partial sums to every process's mailbox and the next kernel sums them
+    there; the r, w, s halos come through the IPC mappings.  Against the
+    oracle's CG1: +-2 iterations, x <= 1e-9 (SURVEY §8(f) NEXT-1 band)."""
+    res, xs = run_procs(tmp_path, P, kind, shape, cg1=True)
+    assert all(r["transport"] == "p2p" for r in res)
+    prob = W.make(kind, nr=shape[0], nt=shape[1], np_=shape[2], warm=False)
+    rc, xo, ito, _, _ = oracle_mod.solve_problem(prob, cg1=True)
+    its = {tuple(map(tuple, r["res"])) for r in res}
+    assert len(its) == 1, its
+    (st1, it1), (st2, it2) = its.pop()
+    assert st1 == st2 == 0 and it1 == it2 and abs(it1 - ito) <= 2
+    V = oracle_mod.Oracle.for_problem(prob).volumes()[None]
+    xg = np.full(xo.shape, np.nan)
+    for r, xl in zip(res, xs):
+        xg[:, r["i0"]:r["i0"] + r["nl"], r["j0"]:r["j0"] + r["ntl"]] = xl
+    assert not np.isnan(xg).any()
+    assert math.sqrt((V * (xg - xo) ** 2).sum() / (V * xo ** 2).sum()) <= 1e-9

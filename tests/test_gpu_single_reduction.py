@@ -155,7 +155,8 @@ def test_single_reduction_switch_and_refusals(mp, oracle_mod):
     oa.set_single_reduction(True)
     with pytest.raises(mp.MasError):
         oa.set_aniso(dev(pa.kpar), dev(pa.bhat))
-    # the P2P transport and the single-reduction loop refuse each other
+    # the single-reduction loop over the P2P transport: switched on before
+    # mas_op_enable_p2p (which then maps its buffers), refused after it
     gp = mp.Grid(prob.mesh)
     op2 = mp.Operator(gp, prob.ncomp, dev(prob.kappa), dev(prob.c), prob.bc_inner, prob.bc_outer)
     op2.enable_p2p()
@@ -163,8 +164,8 @@ def test_single_reduction_switch_and_refusals(mp, oracle_mod):
         op2.set_single_reduction(True)
     op3 = mp.Operator(gp, prob.ncomp, dev(prob.kappa), dev(prob.c), prob.bc_inner, prob.bc_outer)
     op3.set_single_reduction(True)
-    with pytest.raises(mp.MasError):
-        op3.enable_p2p()
+    op3.enable_p2p()
+    assert op3.transport == "p2p" and op3.single_reduction
 
 
 @pytest.mark.parametrize("mk", ["viscosity", "conduction"])
@@ -230,3 +231,82 @@ def test_single_reduction_virtual_ranks(mp, oracle_mod, P):
         assert st == mp.MAS_OK
         xg[:, i0:i0 + nl] = x
     assert rel_l2_V(oracle_mod.Oracle.for_problem(prob).volumes(), xg, xo) <= 1e-9
+
+
+@pytest.mark.parametrize("mk", ["viscosity", "conduction"])
+def test_single_reduction_p2p_one_rank_bitwise(mp, mk):
+    """The mailbox reduction against the rank itself (0 + v = v): the P2P
+    single-reduction loop equals the plain one bit for bit, over repeated
+    solves (epochs), in the CUDA-graph loop."""
+    prob = W.viscosity_problem(12, 16, 64) if mk == "viscosity" else W.conduction_problem(10, 16, 32)
+    st, x, it, rel, hist, op, g = gsolve(mp, prob)
+    op2 = mp.Operator(g, prob.ncomp, dev(prob.kappa), dev(prob.c), prob.bc_inner, prob.bc_outer)
+    op2.set_single_reduction(True)
+    op2.enable_p2p()
+    f = dev(prob.f)
+    if prob.ub_inner is not None:
+        op2.dirichlet_rhs(dev(prob.ub_inner), None, f)
+    for _ in range(3):
+        x2 = dev(prob.x0)
+        st2, it2, rel2, hist2 = op2.solve(f, x2, prob.tol, prob.maxit, True)
+        assert (st2, it2, rel2) == (st, it, rel)
+        np.testing.assert_array_equal(x2.cpu().numpy(), x)
+        np.testing.assert_array_equal(np.asarray(hist2), np.asarray(hist))
+
+
+@pytest.mark.parametrize("P", [2, 3])
+def test_single_reduction_p2p_virtual_ranks(mp, oracle_mod, P):
+    """r-slabs on P virtual ranks with the P2P transport: the kernels sum the
+    3 partials in the mailbox (rank order), the halos are read in place; the
+    same bits as the NCCL loop of the virtual ranks (its allreduce also sums
+    in rank order), and the oracle's CG1 band."""
+    import threading
+    prob = W.viscosity_problem(13 * P, 16, 64, warm=False)
+    out = {}
+    for p2p in (False, True):
+        vid = mp.virtual_ranks_id(7800 + 10 * P + int(p2p))
+        res, errs = {}, []
+
+        def rank_main(r):
+            try:
+                torch.cuda.set_device(0)
+                with torch.cuda.stream(torch.cuda.Stream()):
+                    g = mp.Grid(prob.mesh, dist=(P, r, vid))
+                    sl = slice(g.i0, g.i0 + g.nl)
+                    op = mp.Operator(g, 3, dev(prob.kappa[sl]), dev(prob.c[sl]), prob.bc_inner,
+                                     prob.bc_outer)
+                    op.set_single_reduction(True)
+                    if p2p:
+                        op.enable_p2p()
+                    x = dev(prob.x0[:, sl])
+                    st, it, rel, _ = op.solve(dev(prob.f[:, sl]), x, prob.tol, prob.maxit)
+                    torch.cuda.current_stream().synchronize()
+                    res[r] = (g.i0, g.nl, st, it, x.cpu().numpy(), op.transport)
+                    op.close()
+                    g.close()
+            except Exception as e:  # noqa: BLE001
+                errs.append((r, repr(e)))
+
+        th = [threading.Thread(target=rank_main, args=(r,)) for r in range(P)]
+        for t in th:
+            t.start()
+        for t in th:
+            t.join(timeout=600)
+        assert not errs, errs
+        assert {res[r][5] for r in range(P)} == {"p2p" if p2p else "nccl"}
+        out[p2p] = res
+    rc, xo, ito, _, _ = oracle_mod.solve_problem(prob, cg1=True)
+    for p2p in (False, True):
+        its = {out[p2p][r][3] for r in range(P)}
+        assert len(its) == 1 and abs(next(iter(its)) - ito) <= 2
+    xs = {}
+    for p2p in (False, True):
+        xg = np.empty_like(xo)
+        for r in range(P):
+            i0, nl, st, it, x, _ = out[p2p][r]
+            assert st == mp.MAS_OK
+            xg[:, i0:i0 + nl] = x
+        xs[p2p] = xg
+    assert out[True][0][3] == out[False][0][3]
+    np.testing.assert_array_equal(xs[True], xs[False])
+    assert rel_l2_V(oracle_mod.Oracle.for_problem(prob).volumes(), xs[True], xo) <= 1e-9
