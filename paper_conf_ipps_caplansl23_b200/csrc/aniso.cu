@@ -122,15 +122,16 @@ __device__ __forceinline__ void stg2(double* p, double2 v) { *reinterpret_cast<d
 __device__ __forceinline__ double2 ld2(const double* p) { return __ldg(reinterpret_cast<const double2*>(p)); }
 
 // ---- warp-specialised pipeline ---------------------------------------------
-// One block per SM: 16 consumer warps (warp w = tile row w, lane l = the
-// column pair 2l, 2l+1) and one producer warp whose lane 0 streams the stages
-// with tensor copies (cp.async.bulk.tensor, the TMA engine) into a 4-slot
-// ring, signalled by mbarriers (full: the box bytes landed; empty: the 16
-// consumer warps are done with the slot).
+// One block per SM: 16 cell warps (warp w = tile row w, lane l = the column
+// pair 2l, 2l+1), a halo warp (the corner row below the tile and the extra
+// corner column) and one producer warp whose lane 0 streams the stages with
+// tensor copies (cp.async.bulk.tensor, the TMA engine) into a 4-slot ring,
+// signalled by mbarriers (full: the box bytes landed; empty: the 17 consumer
+// warps are done with the slot).
 namespace {
-// out/q arrives as a TMA box per stage (plain loads by the consumers measured
-// slower; the other consumer designs tried are listed in profiles/README.md,
-// "k_aniso A/B", and kept in the history up to c1ffbea)
+// out/q arrives as a TMA box per stage (MAS_ANISO_QREG: plain loads by the
+// consumers, a tie; the other consumer designs tried are listed in
+// profiles/README.md, "k_aniso A/B", and kept in the history up to c1ffbea)
 #ifndef MAS_ANISO_WJ
 #define MAS_ANISO_WJ 16
 #endif
@@ -141,8 +142,9 @@ constexpr int WJ = MAS_ANISO_WJ;       // tile rows (one consumer warp each)
 constexpr int kAnisoBps = MAS_ANISO_BPS;  // resident blocks per SM (the rings must fit)
 constexpr int rup16(int x) { return (x + 15) / 16 * 16; }  // 128-byte multiples of doubles
 constexpr int WK = 64;                 // tile columns (32 lanes x 2)
-constexpr int NCW = WJ;                // consumer warps
-constexpr int WTHREADS = 32 * (NCW + 1);
+constexpr int NCW = WJ;                // cell warps (warp w: cell row w and corner row w)
+constexpr int NXW = NCW + 1;           // consumer warps: + the halo warp (corner row WJ, extra column)
+constexpr int WTHREADS = 32 * (NXW + 1);
 constexpr int WPR = WJ + 2;            // p rows: j0-1 .. j0+16
 constexpr int WPW = WK + 4;            // p row: [k0-2][k0-1][64 cells][k0+64][k0+65]
 constexpr int WCR = WJ + 1;            // corner rows
@@ -150,23 +152,34 @@ constexpr int WCW = WK + 2;            // corner row: K = k0 .. k0+64 (+1)
 constexpr int WCA = WCR * WCW;         // one corner array
 // every component of a slot starts 128-byte aligned (tensor-copy destinations)
 constexpr int WP_SLOT = rup16(WPR * WPW);  // p box [WJ+2][68] + pad
-constexpr int WC_SLOT = rup16(4 * WCA);    // coefficient box [3][WJ+1][66] + combinations array 3 + pad
+constexpr int WC_SLOT = rup16(3 * WCA);    // coefficient box [3][WJ+1][66] + pad
+#ifdef MAS_ANISO_QREG
+constexpr int WQ_SLOT = 0;             // out/q loaded by the consumers (experiment hook)
+#else
 constexpr int WQ_SLOT = WJ * WK;       // out box [WJ][64]
+#endif
 constexpr int WPL = rup16(WPR * 2), WPRT = WPL;  // phi-wrap side boxes of p: [WJ+2][2]
 constexpr int WCS = rup16(3 * WCR * 2);          // phi-wrap side box of the coefficients: [3][WJ+1][2]
 constexpr int O_C = WP_SLOT, O_Q = O_C + WC_SLOT, O_PL = O_Q + WQ_SLOT, O_PR = O_PL + WPL,
               O_CS = O_PR + WPRT;
-constexpr int W_SLOT = O_CS + WCS;     // WJ = 16: 5936 doubles (6960 with the out box)
+constexpr int W_SLOT = O_CS + WCS;     // WJ = 16: 5840 doubles
 #ifndef MAS_ANISO_SLOTS
 #define MAS_ANISO_SLOTS 4
 #endif
-constexpr int W_NSLOT = MAS_ANISO_SLOTS;  // ring depth (>= 2: a step reads stages n-1 and n)
+constexpr int W_NSLOT = MAS_ANISO_SLOTS;  // ring depth (>= 2)
+// corner-row exchange between the consumer warps (outside the ring, two
+// parities): per corner row and cell column the K-combined A2 and Y (XA, XY),
+// and the extra column's (A, B, E) per corner row (XC, padded to 4)
+constexpr int XSZ = WCR * WK;          // one parity of XA / XY
+constexpr int XCS = WCR * 4;           // one parity of XC
+constexpr int O_XA = W_NSLOT * W_SLOT, O_XY = O_XA + 2 * XSZ, O_XC = O_XY + 2 * XSZ;
+constexpr int W_SMEM_D = O_XC + 2 * XCS;
 // tensor-copy transaction bytes (whole boxes, out-of-bounds elements included)
 constexpr unsigned TX_P = WPR * WPW * 8, TX_PS = WPR * 2 * 8, TX_C = 3 * WCR * WCW * 8,
                    TX_CS = 3 * WCR * 2 * 8;
 constexpr unsigned TX_Q = WJ * WK * 8;
 }  // namespace
-constexpr int kAnisoSmem = W_NSLOT * W_SLOT * (int)sizeof(double) + 3 * W_NSLOT * 8;  // 222,816 B
+constexpr int kAnisoSmem = W_SMEM_D * (int)sizeof(double) + 3 * W_NSLOT * 8;  // 222,880 B
 
 // Tensor maps of one launch (host-encoded, cuTensorMapEncodeTiled): boxes of
 // the field u, of its r-slab ghost planes, of the corner coefficients (all 3
@@ -217,23 +230,27 @@ __device__ __forceinline__ void tma4(unsigned dst, const CUtensorMap* m, int c0,
 __device__ __forceinline__ void fence_proxy_async() {
     asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
 }
-__device__ __forceinline__ void consumer_sync() {  // the 16 consumer warps only
-    asm volatile("bar.sync 1, %0;\n" ::"n"(32 * NCW) : "memory");
+__device__ __forceinline__ void consumer_sync() {  // the 17 consumer warps only
+    asm volatile("bar.sync 1, %0;\n" ::"n"(32 * NXW) : "memory");
 }
 
 // Per step I (corner plane I, cells of plane I-1), consumer side:
-//   wait full(stage I) -> corners(I) -> consumer barrier -> cells(I-1) ->
-//   release stage I-1 (every read of its p, coefficients and out rows done).
+//   wait full(stage I) -> corners(I) -> publish the corner row -> release
+//   stage I -> consumer barrier -> cells(I-1).
 // A stage I is {p plane I, corner coefficients of corner plane I, out/q plane
-// I-1}.  The corner thread replaces the raw (a, b, e) of its corner by the 4
-// sign combinations c[st,sp] = s a + st s b + sp s e, so that a cell reads
-// one value per corner: corner plane i (sr = +1) gives c[st,sp] of its 4
-// corners, plane i+1 (sr = -1) gives -c[-st,-sp].  sigma_par = <p, L_par p>_V
-// = sum_c s_c^2 (V L_par = G^T W K G), summed in the corner phase.
+// I-1}.  With the corner fluxes (A, B, E) = s_c (a, b, e), a cell sums over
+// its 8 corners sr A + st B + sp E (sr, st, sp = +1 where the corner is on
+// the cell's low r / theta / phi side, -1 on the high side), so the sum
+// separates by direction: the thread combines its corners along K with the
+// right lane (shuffle), keeps its own row's B2 + Ed, and publishes A2 and
+// Ed - B2 to the warp of the row above through a small two-parity shared
+// array; along r the cell carries G+ of its lower corner plane in registers
+// from the previous step.  sigma_par = <p, L_par p>_V = sum_c s_c^2
+// (V L_par = G^T W K G), summed in the corner phase.
 template <int MODE>
 __global__ void __launch_bounds__(WTHREADS, kAnisoBps) k_aniso(const AnisoArgs a, const __grid_constant__ AnisoMaps M) {
     extern __shared__ __align__(128) double sm[];
-    unsigned long long* bars = reinterpret_cast<unsigned long long*>(sm + W_NSLOT * W_SLOT);
+    unsigned long long* bars = reinterpret_cast<unsigned long long*>(sm + W_SMEM_D);
     if (MODE == MODE_PCGA && __ldcg(&a.st->stopped)) {
         if (a.cond && blockIdx.x == 0 && threadIdx.x == 0)
             cudaGraphSetConditional((cudaGraphConditionalHandle)a.cond, 0);
@@ -258,13 +275,14 @@ __global__ void __launch_bounds__(WTHREADS, kAnisoBps) k_aniso(const AnisoArgs a
     const Geo& g = a.g;
     const int plane = (int)g.plane;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const bool producer = warp == NCW;
+    const bool producer = warp == NXW;
     double acc[3] = {0.0, 0.0, 0.0};
     auto P_of = [&](int slot) { return sm + slot * W_SLOT; };
     auto C_of = [&](int slot) { return sm + slot * W_SLOT + O_C; };
     auto Q_of = [&](int slot) { return sm + slot * W_SLOT + O_Q; };
     const unsigned full0 = smem_u32(bars), empty0 = smem_u32(bars + W_NSLOT);
 
+    int par = 0;  // parity of the consumers' corner-row exchange (toggled per barrier step)
     // balanced partition of the (tile, r-plane) units, tile-major (one or two
     // segments per block)
     const long long units = (long long)a.ntj * a.ntk * g.nl;
@@ -281,16 +299,11 @@ __global__ void __launch_bounds__(WTHREADS, kAnisoBps) k_aniso(const AnisoArgs a
 
         // barriers (the rings need no clearing: every value a consumer reads is
         // written first in the same stage -- whole tensor boxes with zero-filled
-        // out-of-bounds parts, side boxes on the tiles that read them, and the
-        // corner combinations of rows <= height, columns <= width; MAS_ANISO_ZERO
-        // restores the round-1 clearing per segment)
-#ifdef MAS_ANISO_ZERO
-        for (int t = threadIdx.x; t < W_NSLOT * W_SLOT; t += WTHREADS) sm[t] = 0.0;
-#endif
+        // out-of-bounds parts, side boxes on the tiles that read them)
         if (threadIdx.x == 0) {
             for (int q = 0; q < W_NSLOT; q++) {
                 mbar_init(full0 + 8 * q, 1);    // expect_tx by the producer; the tensor bytes
-                mbar_init(empty0 + 8 * q, NCW);
+                mbar_init(empty0 + 8 * q, NXW);
             }
         }
         fence_proxy_async();
@@ -326,7 +339,9 @@ __global__ void __launch_bounds__(WTHREADS, kAnisoBps) k_aniso(const AnisoArgs a
                     // uninitialised values: 0 * NaN)
                     bytes += TX_P + (first ? TX_PS : 0u) + (last ? TX_PS : 0u);
                     if (cs) bytes += TX_C + (last ? TX_CS : 0u);
+#ifndef MAS_ANISO_QREG
                     if (ql) bytes += TX_Q;
+#endif
                     mbar_expect_tx(full, bytes);
                     const unsigned sb = smem_u32(base);
                     const int jr = j0 - 1;
@@ -350,164 +365,178 @@ __global__ void __launch_bounds__(WTHREADS, kAnisoBps) k_aniso(const AnisoArgs a
                         tma3(sb + 8 * O_C, &M.cahi, k0, j0, 0, full);
                         if (last) tma3(sb + 8 * O_CS, &M.cahi_s, 0, j0, 0, full);
                     }
+#ifndef MAS_ANISO_QREG
                     if (ql) tma3(sb + 8 * O_Q, &M.out, k0, j0, I - 1, full);
+#endif
                 }
             };
             for (int n = 0; n < nst; n++) issue(n);
         } else {
-            // ---- consumers --------------------------------------------------
+            // ---- consumers: warp w < WJ owns corner row w and cell row w; the
+            // halo warp (w = WJ) owns corner row WJ and the extra corner column
+            // (K = k0 + width, one corner per lane = row) ----------------------
             const int w = warp, c2 = 2 * lane;
             const bool first = k0 == 0, last = k0 + width == g.np;
-            const bool lfix = first && c2 == 0, rfix = last && c2 == width;
-            const bool crow_ok = w <= height && c2 <= width;  // corner pair in use
-            const bool cell_ok = w < height && c2 < width;    // cell pair in use
-            int xr = -1, xc = 0;  // extra corner: row 16 / column 64
-            {
-                const int t = threadIdx.x;
-                if (height == WJ && t <= width) {
-                    xr = WJ, xc = t;
-                } else if (width == WK && t >= WK + 1 && t - (WK + 1) < min(height + 1, WJ)) {
-                    xr = t - (WK + 1), xc = WK;
-                }
-            }
+            const bool halo = w == NCW;
+            const bool crow = w <= height && c2 < width;     // corner pair in use
+            const bool cell_ok = w < height && c2 < width;   // cell pair in use
+            const bool edge = c2 + 2 == width;               // right neighbour corner: the extra column
+            const bool xlane = halo && lane <= height;       // extra-column corner (row lane, col width)
             double cw0 = 0.0, cw1 = 0.0;  // 1 / (vt_j vp_k) of the two cells
             if (cell_ok) {
                 const double vt = __ldg(g.vt + j0 + w);
                 cw0 = 1.0 / (vt * __ldg(g.vp + k0 + c2));
                 cw1 = 1.0 / (vt * __ldg(g.vp + k0 + c2 + 1));
             }
-            auto corner_math = [&](double a00, double a01, double a10, double a11, double b00, double b01,
-                                   double b10, double b11, double A0, double B0, double E0, double& o0,
-                                   double& o1, double& o2, double& o3) -> double {
+            // s_c = a Dr + b Dt + e Dp of a corner from its 8 cells (a: plane
+            // I-1, b: plane I; [row J-1 / J][column K-1 / K])
+            auto corner_s = [&](double a00, double a01, double a10, double a11, double b00, double b01,
+                                double b10, double b11, double A0, double B0, double E0) -> double {
                 const double Dr = ((b00 - a00) + (b01 - a01)) + ((b10 - a10) + (b11 - a11));
                 const double Dt = ((a10 - a00) + (a11 - a01)) + ((b10 - b00) + (b11 - b01));
                 const double Dp = ((a01 - a00) + (a11 - a10)) + ((b01 - b00) + (b11 - b10));
-                const double sc = A0 * Dr + B0 * Dt + E0 * Dp;
-                const double A = sc * A0, B = sc * B0, E = sc * E0;
-                o0 = (A + B) + E;  // st +, sp +
-                o1 = (A + B) - E;  // st +, sp -
-                o2 = (A - B) + E;  // st -, sp +
-                o3 = (A - B) - E;  // st -, sp -
-                return sc;
+                return A0 * Dr + B0 * Dt + E0 * Dp;
             };
-            // p of the previous plane for this thread's corners, carried in
-            // registers from one step to the next (rows w, w+1 of the pair;
-            // the extra corner's 4 cells); wrap cells from the side boxes
+            // p of the previous plane carried in registers: rows w, w+1 of the
+            // box at columns c2+1 .. c2+3; the extra-column corner's 4 cells
             double x0 = 0.0, y0 = 0.0, e0 = 0.0, e1 = 0.0, e2 = 0.0, e3 = 0.0;
             double2 x12 = make_double2(0.0, 0.0), y12 = x12;
-            // 1/vr of the cell plane of the next step, loaded one step ahead
-            // (its latency sat on the cell phase's dependency chain)
-            double ivr_cur = 0.0;
+            // G+ of the previous corner plane (the cells' lower-r face), carried
+            double2 carry = make_double2(0.0, 0.0);
+            double ivr_cur = 0.0;  // 1/vr of the next step's cell plane, loaded one step ahead
+            double* XA = sm + O_XA;
+            double* XY = sm + O_XY;
+            double* XC = sm + O_XC;
             for (int n = 0; n < nst; n++) {
                 const int I = ia - 1 + n, slot = n % W_NSLOT;
                 const double ivr_here = ivr_cur;
                 if (cell_ok && n + 1 >= 2 && n + 1 < nst) ivr_cur = __ldg(a.ivr + I);
+                // q / out of plane I-1 (the cells of this step)
+                double2 qv = make_double2(0.0, 0.0);
+#ifdef MAS_ANISO_QREG
+                if (n >= 2 && cell_ok)
+                    qv = ld2(a.out + (size_t)(I - 1) * plane + (size_t)(j0 + w) * g.np + k0 + c2);
+#endif
                 mbar_wait(full0 + 8 * slot, (n / W_NSLOT) & 1);
 #ifdef MAS_ANISO_DIAG_NOCOMPUTE
                 // diagnostic build (wrong results): the consumers only wait for
                 // each stage and release it -- the producer / TMA pipeline alone
-                if (n >= 1) {
-                    __syncwarp();
-                    if (lane == 0) mbar_arrive(empty0 + 8 * ((n - 1) % W_NSLOT));
-                }
+                __syncwarp();
+                if (lane == 0) mbar_arrive(empty0 + 8 * slot);
                 continue;
 #endif
                 const double* p1 = P_of(slot);
-                double X0 = 0.0, Y0 = 0.0, E0 = 0.0, E1 = 0.0, E2 = 0.0, E3 = 0.0;
-                double2 X12 = make_double2(0.0, 0.0), Y12 = X12;
-                if (crow_ok) {
-                    const double* q1 = p1 + w * WPW + c2;
-                    X0 = q1[1], Y0 = q1[WPW + 1];
-                    X12 = lds2(q1 + 2), Y12 = lds2(q1 + WPW + 2);
-                    if (lfix) X0 = p1[O_PL + 2 * w + 1], Y0 = p1[O_PL + 2 * w + 3];
-                    if (rfix) X12.x = p1[O_PR + 2 * w], Y12.x = p1[O_PR + 2 * w + 2];
+                // p rows w, w+1 (cell rows J-1, J) at cells k0+c2, k0+c2+1; the
+                // cell k0+c2-1 from the left lane (lane 0: the box or the wrap box)
+                const double* q1 = p1 + w * WPW + c2;
+                const double2 X12 = lds2(q1 + 2), Y12 = lds2(q1 + WPW + 2);
+                double X0 = __shfl_up_sync(0xffffffffu, X12.y, 1);
+                double Y0 = __shfl_up_sync(0xffffffffu, Y12.y, 1);
+                if (lane == 0) {
+                    X0 = first ? p1[O_PL + 2 * w + 1] : q1[1];
+                    Y0 = first ? p1[O_PL + 2 * w + 3] : q1[WPW + 1];
                 }
-                if (xr >= 0) {
-                    const double* q1 = p1 + xr * WPW + xc + 1;
-                    E0 = q1[0], E1 = q1[1], E2 = q1[WPW], E3 = q1[WPW + 1];
-                    if (first && xc == 0) E0 = p1[O_PL + 2 * xr + 1], E2 = p1[O_PL + 2 * xr + 3];
-                    if (last && xc == width) E1 = p1[O_PR + 2 * xr], E3 = p1[O_PR + 2 * xr + 2];
+                double E0 = 0.0, E1 = 0.0, E2 = 0.0, E3 = 0.0;
+                if (xlane) {  // cells k0+width-1, k0+width (the latter wraps on the last tile)
+                    const double* q2 = p1 + lane * WPW + width + 1;
+                    E0 = q2[0], E2 = q2[WPW];
+                    E1 = last ? p1[O_PR + 2 * lane] : q2[1];
+                    E3 = last ? p1[O_PR + 2 * lane + 2] : q2[WPW + 1];
                 }
                 if (n == 0) {  // stage ia-1: p plane ia-1 only
                     x0 = X0, y0 = Y0, x12 = X12, y12 = Y12, e0 = E0, e1 = E1, e2 = E2, e3 = E3;
+                    __syncwarp();
+                    if (lane == 0) mbar_arrive(empty0 + 8 * slot);
                     continue;
                 }
-                // ---- corners of plane I: p(I-1) rows w, w+1 (cell rows J-1, J)
-                // from registers, p(I) from the stage
-                double* Cf = C_of(slot);
-                if (crow_ok) {
-                    double* c0 = Cf + w * WCW + c2;
-                    double2 A0 = lds2(c0), B0 = lds2(c0 + WCA), C0 = lds2(c0 + 2 * WCA);
-                    if (rfix) {  // corner column width = k0 + width: the right box
-                        const double* CS = p1 + O_CS;
-                        A0.x = CS[2 * w], B0.x = CS[2 * (WCR + w)], C0.x = CS[2 * (2 * WCR + w)];
-                    }
-                    double o[2][4];
-                    const double s0 = corner_math(x0, x12.x, y0, y12.x, X0, X12.x, Y0, Y12.x, A0.x, B0.x,
-                                                  C0.x, o[0][0], o[0][1], o[0][2], o[0][3]);
-                    const double s1 = corner_math(x12.x, x12.y, y12.x, y12.y, X12.x, X12.y, Y12.x, Y12.y,
-                                                  A0.y, B0.y, C0.y, o[1][0], o[1][1], o[1][2], o[1][3]);
-#pragma unroll
-                    for (int q = 0; q < 4; q++) sts2(c0 + q * WCA, make_double2(o[0][q], o[1][q]));
-                    // sigma: this tile's corners (row < height, col < width) of the
-                    // segment's own planes (plane ib is the next segment's first)
-                    if (MODE == MODE_PCGA && I < ib && w < height && c2 < width)
-                        acc[0] += s0 * s0 + s1 * s1;
+                // ---- corners (w, c2), (w, c2+1) of plane I ------------------
+                const double* Cf = C_of(slot);
+                const double* cc = Cf + w * WCW + c2;
+                const double2 Ac = lds2(cc), Bc = lds2(cc + WCA), Ec = lds2(cc + 2 * WCA);
+                const double s0 = corner_s(x0, x12.x, y0, y12.x, X0, X12.x, Y0, Y12.x, Ac.x, Bc.x, Ec.x);
+                const double s1 = corner_s(x12.x, x12.y, y12.x, y12.y, X12.x, X12.y, Y12.x, Y12.y, Ac.y, Bc.y,
+                                           Ec.y);
+                // sigma: this tile's corners (row < height, col < width) of the
+                // segment's own planes (plane ib is the next segment's first)
+                if (MODE == MODE_PCGA && I < ib && cell_ok) acc[0] += s0 * s0 + s1 * s1;
+                // the corner fluxes (A, B, E) = s_c (a, b, e); a cell sums, over
+                // its 8 corners, sr A + st B + sp E (sr, st, sp = +1 on the
+                // corner's low side): combine along K with the right lane
+                const double Aa = s0 * Ac.x, Ab = s1 * Ac.y, Ba = s0 * Bc.x, Bb = s1 * Bc.y;
+                const double Ea = s0 * Ec.x, Eb = s1 * Ec.y;
+                double An = __shfl_down_sync(0xffffffffu, Aa, 1);
+                double Bn = __shfl_down_sync(0xffffffffu, Ba, 1);
+                double En = __shfl_down_sync(0xffffffffu, Ea, 1);
+                if (edge) An = 0.0, Bn = 0.0, En = 0.0;  // the extra column, added after the barrier
+                const double A2a = Aa + Ab, A2b = Ab + An;
+                const double B2a = Ba + Bb, B2b = Bb + Bn;
+                const double Eda = Ea - Eb, Edb = Eb - En;
+                // corner row w gives its own cell row B2 + Ed (+-A2) and the cell
+                // row above Ed - B2 (+-A2): the latter goes to warp w-1
+                if (crow && w >= 1) {
+                    sts2(XA + par * XSZ + w * WK + c2, make_double2(A2a, A2b));
+                    sts2(XY + par * XSZ + w * WK + c2, make_double2(Eda - B2a, Edb - B2b));
                 }
-                if (xr >= 0) {  // row 16 / column 64: counted by the neighbouring tile
-                    double* c0 = Cf + xr * WCW + xc;
-                    double A = c0[0], B = c0[WCA], E = c0[2 * WCA];
-                    if (last && xc == width) {
+                if (xlane) {  // extra-column corner (lane, width)
+                    double A, B, E;
+                    if (last) {
                         const double* CS = p1 + O_CS;
-                        A = CS[2 * xr], B = CS[2 * (WCR + xr)], E = CS[2 * (2 * WCR + xr)];
+                        A = CS[2 * lane], B = CS[2 * (WCR + lane)], E = CS[2 * (2 * WCR + lane)];
+                    } else {
+                        const double* c0 = Cf + lane * WCW + width;
+                        A = c0[0], B = c0[WCA], E = c0[2 * WCA];
                     }
-                    double o0, o1, o2, o3;
-                    corner_math(e0, e1, e2, e3, E0, E1, E2, E3, A, B, E, o0, o1, o2, o3);
-                    c0[0] = o0;
-                    c0[WCA] = o1;
-                    c0[2 * WCA] = o2;
-                    c0[3 * WCA] = o3;
+                    const double sx = corner_s(e0, e1, e2, e3, E0, E1, E2, E3, A, B, E);
+                    double* xo = XC + par * XCS + 4 * lane;
+                    sts2(xo, make_double2(sx * A, sx * B));
+                    xo[2] = sx * E;
                 }
                 x0 = X0, y0 = Y0, x12 = X12, y12 = Y12, e0 = E0, e1 = E1, e2 = E2, e3 = E3;
-                consumer_sync();
-                // ---- cells (w, c2..c2+1) of plane i = I-1: corner planes i
-                // (sr = +1) and I (sr = -1); out/q plane i from this stage
-                if (n >= 2 && cell_ok) {
-                    const int i = I - 1;
-                    const double* l = C_of((n - 1) % W_NSLOT) + w * WCW + c2;
-                    const double* h = Cf + w * WCW + c2;
-                    const double2 l0 = lds2(l), l2 = lds2(l + 2 * WCA + WCW);
-                    const double2 h3 = lds2(h + 3 * WCA), h1 = lds2(h + WCA + WCW);
-                    const double l1a = l[WCA + 1], l1b = l[WCA + 2];
-                    const double l3a = l[3 * WCA + WCW + 1], l3b = l[3 * WCA + WCW + 2];
-                    const double h2a = h[2 * WCA + 1], h2b = h[2 * WCA + 2];
-                    const double h0a = h[WCW + 1], h0b = h[WCW + 2];
-                    const double s0 = ((l0.x + l1a) + (l2.x + l3a)) - ((h3.x + h2a) + (h1.x + h0a));
-                    const double s1 = ((l0.y + l1b) + (l2.y + l3b)) - ((h3.y + h2b) + (h1.y + h0b));
-                    const double ivr = ivr_here;  // 1/vr of plane i = I-1
-                    const double y0 = s0 * (ivr * cw0), y1 = s1 * (ivr * cw1);
-                    const double2 qv = lds2(Q_of(slot) + w * WK + c2);
-                    double* o = a.out + (size_t)i * plane + (size_t)(j0 + w) * g.np + k0 + c2;
-                    if (MODE == MODE_RESID) {
-                        const double r0 = qv.x - y0, r1 = qv.y - y1;
-                        stg2(o, make_double2(r0, r1));
-                        const double vr = __ldg(g.vr + i);
-                        const double V0 = vr / cw0, V1 = vr / cw1;
-                        const double2 f = ld2(a.f + (o - a.out));
-                        const double2 di = ld2(a.dinv + (o - a.out));
-                        acc[0] += V0 * f.x * f.x + V1 * f.y * f.y;
-                        acc[1] += V0 * r0 * r0 + V1 * r1 * r1;
-                        acc[2] += V0 * r0 * (di.x * r0) + V1 * r1 * (di.y * r1);
-                    } else {
-                        stg2(o, make_double2(qv.x + y0, qv.y + y1));
-                    }
-                }
-                // stage n-1 is no longer read (p by corners(I), products by
-                // cells(I-1)); the combination writes went through the generic
-                // proxy, the next fill of the slot is a tensor copy
-                fence_proxy_async();
+                // q / out of plane I-1 from this stage (read before the release)
+#ifndef MAS_ANISO_QREG
+                if (n >= 2 && cell_ok) qv = lds2(Q_of(slot) + w * WK + c2);
+#endif
+                // stage n is no longer read: hand the slot back
                 __syncwarp();
-                if (lane == 0) mbar_arrive(empty0 + 8 * ((n - 1) % W_NSLOT));
+                if (lane == 0) mbar_arrive(empty0 + 8 * slot);
+                consumer_sync();
+                // ---- cells (w, c2..c2+1): corner rows w and w+1 -------------
+                if (cell_ok) {
+                    const double2 An1 = lds2(XA + par * XSZ + (w + 1) * WK + c2);
+                    const double2 Yn1 = lds2(XY + par * XSZ + (w + 1) * WK + c2);
+                    const double Sa = (B2a + Eda) + Yn1.x, Ta = A2a + An1.x;
+                    double Sb = (B2b + Edb) + Yn1.y, Tb = A2b + An1.y;
+                    if (edge) {  // the extra column's corners at rows w, w+1
+                        const double* xc0 = XC + par * XCS + 4 * w;
+                        const double2 ab0 = lds2(xc0), ab1 = lds2(xc0 + 4);
+                        Sb += (ab0.y - xc0[2]) - (ab1.y + xc0[6]);
+                        Tb += ab0.x + ab1.x;
+                    }
+                    // corner plane I is the upper-r face of cell plane I-1 (-A) and
+                    // the lower-r face of cell plane I (+A)
+                    if (n >= 2) {
+                        const double sv0 = carry.x + (Sa - Ta), sv1 = carry.y + (Sb - Tb);
+                        const int i = I - 1;
+                        const double ivr = ivr_here;  // 1/vr of plane i = I-1
+                        const double y0 = sv0 * (ivr * cw0), y1 = sv1 * (ivr * cw1);
+                        double* o = a.out + (size_t)i * plane + (size_t)(j0 + w) * g.np + k0 + c2;
+                        if (MODE == MODE_RESID) {
+                            const double r0 = qv.x - y0, r1 = qv.y - y1;
+                            stg2(o, make_double2(r0, r1));
+                            const double vr = __ldg(g.vr + i);
+                            const double V0 = vr / cw0, V1 = vr / cw1;
+                            const double2 f = ld2(a.f + (o - a.out));
+                            const double2 di = ld2(a.dinv + (o - a.out));
+                            acc[0] += V0 * f.x * f.x + V1 * f.y * f.y;
+                            acc[1] += V0 * r0 * r0 + V1 * r1 * r1;
+                            acc[2] += V0 * r0 * (di.x * r0) + V1 * r1 * (di.y * r1);
+                        } else {
+                            stg2(o, make_double2(qv.x + y0, qv.y + y1));
+                        }
+                    }
+                    carry = make_double2(Sa + Ta, Sb + Tb);
+                }
+                par ^= 1;
             }
         }
         __syncthreads();  // the next segment re-initialises the rings and barriers
