@@ -594,19 +594,6 @@ static mas_status_t ensure_prof_events(mas_op* op, int k) {
 // deciding kernel's last block sets the while-condition to 0.
 // (MAS_GRAPH_PRE=1, an experiment hook, launches iteration 1 as plain
 // kernels ahead of a graph holding only the while node, the round-1 form.)
-// kernel B visits the rows in kernel A's r-chunks, each chunk top-down, when
-// a vector fits the 126 MB L2 (reuse of what the other kernel touched last:
-// C2a +2%, C2 +0.7%, C3 unchanged); MAS_B_PLANE_ORDER=1 keeps the plane order
-// (experiment hook)
-static int b_chunk(const mas_op* op) {
-    static const bool plane_order = [] {
-        const char* e = getenv("MAS_B_PLANE_ORDER");
-        return e && atoi(e) != 0;
-    }();
-    const double vec_bytes = 8.0 * op->ncomp * op->geo.nl * (double)op->geo.plane;
-    return plane_order || vec_bytes > 126e6 ? 0 : op->chunk;
-}
-
 static mas_status_t loop_graph(mas_op* op, StencilArgs a, StreamArgs b, AnisoArgs an, bool pre_plain) {
     const int aniso_key = op->aniso ? (lpar_in_a(op) ? 2 : 1) : 0;
     if (op->gexec && op->g_x == a.x && op->g_hist == a.rho_hist && op->g_aniso == aniso_key &&
@@ -1589,7 +1576,6 @@ mas_status_t mas_op_kernel_bench(mas_op_t* op, int reps, double* a_ms, double* b
     b.r = op->r;
     b.q = op->q;
     b.dinv = op->dinv;
-    b.chunk = b_chunk(op);
     b.st = op->st;
     b.rho_hist = a.rho_hist;
     b.sigma_hist = a.sigma_hist;
@@ -1879,7 +1865,6 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
     b.r = op->r;
     b.q = op->q;
     b.dinv = op->dinv;
-    b.chunk = b_chunk(op);
     b.st = op->st;
     b.rho_hist = rho_h;
     b.sigma_hist = sig_h;
@@ -2317,7 +2302,6 @@ mas_status_t mas_stack_solve(mas_stack_t* sk, const double* const* rhs, double* 
         B.r = op->r;
         B.q = op->q;
         B.dinv = op->dinv;
-        B.chunk = b_chunk(op);
         B.st = op->st;
         B.rho_hist = A.rho_hist;
         B.sigma_hist = A.sigma_hist;

@@ -1226,23 +1226,7 @@ __global__ void __launch_bounds__(kThreads) k_pcg_b(const StreamArgs a) {
     }
     if (!brk) {
         const long long Nl = (long long)g.nl * g.plane;
-        // the (r,theta) rows in kernel A's chunk structure, each chunk's planes
-        // top-down (virtual row v -> plane i, row j; v = (s * nch + c) * nt + j,
-        // i = c * chunk + len_c - 1 - s): kernel A marches every chunk upwards,
-        // so the planes it wrote last (q still in L2) are read first, and the
-        // planes of r written last here are the ones kernel A reads first
-        const int chunk = a.chunk > 0 ? a.chunk : g.nl;
-        const int nch = (g.nl + chunk - 1) / chunk;
-        const int rows = chunk * nch * g.nt;
-        auto vrow = [&](int v, int& i, int& j) -> bool {
-            const int s = v / (nch * g.nt);
-            const int rem = v - s * (nch * g.nt);
-            const int c = rem / g.nt;
-            j = rem - c * g.nt;
-            const int len = min(chunk, g.nl - c * chunk);
-            i = c * chunk + len - 1 - s;
-            return s < len;
-        };
+        const int rows = g.nl * g.nt;
         const int half = g.np >> 1;
         // a block covers rpi whole (r,theta) rows per step when a row has
         // fewer double2 pairs than the block has threads
@@ -1256,18 +1240,12 @@ __global__ void __launch_bounds__(kThreads) k_pcg_b(const StreamArgs a) {
             const int stride = gridDim.x * rpi;
             for (int row = blockIdx.x * rpi + sub; row < rows; row += 2 * stride) {
                 const int row2 = row + stride;
-                int i1, j1, i2, j2;
-                const bool one = vrow(row, i1, j1);
-                bool two = row2 < rows && vrow(row2, i2, j2);
-                if (!one && !two) continue;
-                if (!one) {  // (ragged last chunk) only the second row: take it as the first
-                    i1 = i2, j1 = j2;
-                    two = false;
-                }
-                if (!two) i2 = i1, j2 = j1;
+                const bool two = row2 < rows;
+                const int i1 = row / g.nt, j1 = row - i1 * g.nt;
+                const int i2 = two ? row2 / g.nt : i1, j2 = two ? row2 - i2 * g.nt : j1;
                 const double w1 = __ldg(g.vr + i1) * __ldg(g.vt + j1);
                 const double w2 = __ldg(g.vr + i2) * __ldg(g.vt + j2);
-                const long long b1 = ((long long)i1 * g.nt + j1) * g.np, b2 = ((long long)i2 * g.nt + j2) * g.np;
+                const long long b1 = (long long)row * g.np, b2 = (long long)(two ? row2 : row) * g.np;
                 for (int h = col; h < half; h += tpr) {
                     const int k = 2 * h;
                     const double2 d1 = ld2(a.dinv + b1 + k), r1 = ld_cs(a.r + b1 + k), q1 = ld_cs(a.q + b1 + k);
@@ -1297,10 +1275,9 @@ __global__ void __launch_bounds__(kThreads) k_pcg_b(const StreamArgs a) {
         } else
 #endif
         for (int row = blockIdx.x * rpi + sub; row < rows; row += gridDim.x * rpi) {
-            int i, j;
-            if (!vrow(row, i, j)) continue;
+            const int i = row / g.nt, j = row - i * g.nt;
             const double wrow = __ldg(g.vr + i) * __ldg(g.vt + j);
-            const long long base = ((long long)i * g.nt + j) * g.np;
+            const long long base = (long long)row * g.np;
             for (int h = col; h < half; h += tpr) {
                 const int k = 2 * h;
                 const double2 di = ld2(a.dinv + base + k);

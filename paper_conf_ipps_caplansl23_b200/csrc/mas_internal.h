@@ -175,7 +175,6 @@ struct StreamArgs {  // kernel B
     double* x;
     const double* p[2];
     int brk_at;               // test hook (MAS_TEST_TRANSPORTS=1 + MAS_TEST_BREAKDOWN_AT=k): B(k) breaks down
-    int chunk;                // kernel A's r-chunk: rows visited chunk-wise top-down (0: plane order)
 };
 
 // ---------------------------------------------------------------------------
