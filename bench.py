@@ -229,7 +229,8 @@ def host_dram_gbs(threads: int):
         for fn in (lib.host_copy_gbs, lib.host_read_gbs):
             fn.restype = ctypes.c_double
             fn.argtypes = [ctypes.c_longlong, ctypes.c_int]
-        os.environ.setdefault("OMP_NUM_THREADS", str(threads))
+        lib.host_set_threads.argtypes = [ctypes.c_int]
+        lib.host_set_threads(int(threads))  # the oracle's 1-thread sample shares the OpenMP runtime
         cp = float(lib.host_copy_gbs(1 << 28, 3))
         rd = float(lib.host_read_gbs(1 << 28, 3))
         return max(cp, rd), cp, rd
@@ -658,15 +659,18 @@ def main():
         v, per = oracle_sample(prob, args.cpu_iters, cores)
         # the survey's single-thread point (SURVEY §8(d) timing protocol: C1
         # and C2-sized grids), fixed iterations on the same grid
+        hbw, hcp, hrd = host_dram_gbs(cores)
         v1 = per1 = None
         if cells <= 5_000_000:
             v1, per1 = oracle_sample(prob, 2, 1)
-        hbw, hcp, hrd = host_dram_gbs(cores)
         ob = oracle_bytes_per_cell(nc) * cells * v / 1e9
         cpu = {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle",
                "host_dram_gbs": hbw, "host_copy_gbs_with_write_allocate": hcp,
                "host_read_gbs": hrd, "oracle_alg_gbs": ob,
-               "oracle_frac_of_host_dram": (ob / hbw) if hbw else None,
+               # below ~256 MB per iteration the oracle's vectors live in the host caches
+               # and a DRAM fraction means nothing (C1)
+               "oracle_frac_of_host_dram": (ob / hbw) if hbw and
+               oracle_bytes_per_cell(nc) * cells >= 256e6 else None,
                "cpu_model": cpu_model(),
                "one_thread": None if v1 is None else {
                    "value": v1, "unit": UNIT, "cores": 1,

@@ -13,6 +13,12 @@
 #include <string.h>
 #include <omp.h>
 
+/* the OpenMP runtime is shared with the oracle library in bench.py's process
+ * (its 1-thread sample calls omp_set_num_threads(1)): set the team size here */
+void host_set_threads(int threads) {
+    if (threads > 0) omp_set_num_threads(threads);
+}
+
 static double* filled(long long n) {
     double* a = malloc(sizeof(double) * n);
     long long i;
