@@ -89,6 +89,43 @@ def test_apply_and_diag_match_oracle(mp, oracle_mod, shape, bc):
     np.testing.assert_allclose(host(D), Do, rtol=1e-13, atol=0)
 
 
+@pytest.mark.parametrize("shape", [(16, 24, 64), (24, 20, 70), (40, 32, 128), (7, 40, 192)])
+def test_apply_repeatable_and_per_cell(mp, oracle_mod, shape):
+    """Race sentinel for k_aniso's shared-memory hand-offs (the two-parity
+    corner-row exchange between consumer warps, the halo warp's extra column,
+    the ring slot released before the consumer barrier): 30 repeated applies
+    are bitwise identical, and every cell of c x + L_par x is within 1e-12 of
+    a local scale of the oracle: 2 max|x| times the largest diagonal D_Q of
+    the cell's 27-cell neighbourhood (the V-weighted operator is a Gram
+    matrix, so |L_PQ| <= sqrt(V_Q/V_P) sqrt(D_P D_Q); a stale or half-written
+    value in one cell is an O(1) error there, even where the V-weighted norm
+    hides it).
+    Shapes: one phi tile (64), a ragged phi tile (70 = 64 + 6), ragged theta
+    tiles, several tiles per block segment (192 = 3 phi tiles)."""
+    mesh = W.stretched_mesh(*shape)
+    _, c, kpar, b = rand_fields(shape, 3)
+    kappa = np.zeros(shape)
+    g, op = setup(mp, mesh, kappa, c, kpar, b)
+    xh = W.random_field((1,) + shape, 11)
+    x = dev(xh)
+    y0 = torch.empty_like(x)
+    op.apply(x, y0)
+    for _ in range(30):
+        y = torch.empty_like(x)
+        op.apply(x, y)
+        assert torch.equal(y, y0)
+    o = oracle_mod.Oracle(mesh, 0, 1)
+    yo = o.apply(kappa, c, xh) + o.aniso_apply(kpar, b, xh)
+    D = o.diag(kappa, c) + o.aniso_diag(kpar, b)
+    Dp = np.pad(D, ((1, 1), (1, 1), (0, 0)), mode="edge")
+    Dp = np.concatenate([Dp[:, :, -1:], Dp, Dp[:, :, :1]], axis=2)  # periodic phi
+    n0, n1, n2 = shape
+    Dn = np.max([Dp[a:a + n0, b_:b_ + n1, e:e + n2] for a in range(3) for b_ in range(3) for e in range(3)],
+                axis=0)
+    scale = 2.0 * Dn[None] * np.abs(xh).max()
+    assert (np.abs(host(y0) - yo) / scale).max() <= 1e-12
+
+
 def test_pure_field_aligned_apply(mp, oracle_mod):
     """kappa = 0: the result is c x + L_par x alone (no 7-point term to hide a
     wrong corner term behind)."""
