@@ -19,6 +19,7 @@ python bench.py --solver cg1 --no-cpu-baseline --no-e2e > $O/${TAG}_bench_C3_cg1
 python bench.py --config C3s8 --no-cpu-baseline --no-e2e > $O/${TAG}_bench_C3s8.log 2>&1
 python tools/stack_bench.py > $O/${TAG}_stack_bench.json 2> $O/${TAG}_stack_bench.err
 for f in $O/${TAG}_bench_*.log; do echo "$f: $(tail -1 $f | cut -c1-100)"; done
+[ -n "$SKIP_NCU" ] && exit 0
 $NCU --metrics gpu__time_duration.sum --clock-control none -c 400 --csv --log-file $O/${TAG}_launches_C3.csv \
   python bench.py --steps 2 --warmup 1 --no-cpu-baseline --no-e2e --no-replay > /dev/null 2>&1
 $NCU --metrics gpu__time_duration.sum --clock-control none -c 900 --csv --log-file $O/${TAG}_launches_C2a.csv \
