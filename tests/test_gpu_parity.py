@@ -166,17 +166,23 @@ def test_pcg_matches_oracle_at_tol(mp, oracle_mod, idx):
     # Residual histories: CG amplifies rounding differences; the oracle run
     # against itself with a 1e-16 relative perturbation of f already differs
     # by 1e-4..3e-3 after ~20 iterations on these stiff problems (DESIGN.md
-    # §6.2).  So: 1e-9 over the first 10 iterations; after that within 20x
-    # the oracle's own envelope measured on this very problem.
+    # §6.2).  So: 1e-9 over the first 10 iterations; after that within 4x the
+    # oracle's own envelope on this very problem, the running max over four
+    # independently perturbed oracle solves (one perturbation alone samples
+    # the rounding spread too thinly for a tight factor).
     n = min(len(hist), len(histo))
     np.testing.assert_allclose(hist[:10], histo[:10], rtol=1e-9, atol=0)
-    pert = prob.f * (1.0 + 1e-16 * np.random.default_rng(7).standard_normal(prob.f.shape))
-    prob.f = pert
-    _, _, _, _, histp = oracle_mod.solve_problem(prob)
-    m = min(n, len(histp))
-    env = np.maximum.accumulate(np.abs(histp[:m] - histo[:m]) / histo[:m])
-    dev_ = np.abs(hist[:m] - histo[:m]) / histo[:m]
-    assert (dev_ <= 20.0 * env + 1e-9).all(), (dev_.max(), env.max())
+    f0 = prob.f.copy()
+    env = np.zeros(n)
+    for seed in (7, 8, 9, 10):
+        prob.f = f0 * (1.0 + 1e-16 * np.random.default_rng(seed).standard_normal(f0.shape))
+        _, _, _, _, histp = oracle_mod.solve_problem(prob)
+        m = min(n, len(histp))
+        env[:m] = np.maximum(env[:m], np.abs(histp[:m] - histo[:m]) / histo[:m])
+    prob.f = f0
+    env = np.maximum.accumulate(env)
+    dev_ = np.abs(hist[:n] - histo[:n]) / histo[:n]
+    assert (dev_ <= 4.0 * env + 1e-9).all(), (dev_.max(), env.max(), (dev_ / (env + 1e-30)).max())
 
 
 @pytest.mark.parametrize("k", [1, 2, 7, 40])
