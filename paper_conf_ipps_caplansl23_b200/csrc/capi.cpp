@@ -623,8 +623,7 @@ static mas_status_t loop_graph(mas_op* op, StencilArgs a, StreamArgs b, AnisoArg
                 an1.u = aniso_p_halo(op, 1);
                 e = launch_aniso(MODE_PCGA, an1, op->cap_stream);
             }
-            if (e == cudaSuccess && op->tnode)
-                e = launch_pole_avg(op->geo, nc, op->q, nullptr, 0, op->geo.nl, op->cap_stream);
+            // (theta nodes: kernel B does the pole pass on q itself)
             if (e == cudaSuccess) e = launch_pcg_b(b, op->b_blocks, op->cap_stream);
             cudaGraph_t out = g;
             cudaError_t e2 = cudaStreamEndCapture(op->cap_stream, &out);
@@ -667,8 +666,6 @@ static mas_status_t loop_graph(mas_op* op, StencilArgs a, StreamArgs b, AnisoArg
                 e = launch_stencil(MODE_PCGA, nc, a, op->cap_stream);
                 an.u = aniso_p_halo(op, kk);
                 if (e == cudaSuccess && op->aniso && !lpar_in_a(op)) e = launch_aniso(MODE_PCGA, an, op->cap_stream);
-                if (e == cudaSuccess && op->tnode)
-                    e = launch_pole_avg(op->geo, nc, op->q, nullptr, 0, op->geo.nl, op->cap_stream);
                 if (e == cudaSuccess) e = launch_pcg_b(b, op->b_blocks, op->cap_stream);
             }
             cudaGraph_t out = body;
@@ -1576,6 +1573,7 @@ mas_status_t mas_op_kernel_bench(mas_op_t* op, int reps, double* a_ms, double* b
     b.r = op->r;
     b.q = op->q;
     b.dinv = op->dinv;
+    b.tnode = op->tnode;
     b.st = op->st;
     b.rho_hist = a.rho_hist;
     b.sigma_hist = a.sigma_hist;
@@ -1865,6 +1863,7 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
     b.r = op->r;
     b.q = op->q;
     b.dinv = op->dinv;
+    b.tnode = op->tnode;
     b.st = op->st;
     b.rho_hist = rho_h;
     b.sigma_hist = sig_h;
@@ -1907,8 +1906,7 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
                 an.u = aniso_p_halo(op, 1);
                 CU(launch_aniso(MODE_PCGA, an, s));
             }
-            ST(pole_pass(op, op->q, nc, s));
-            CU(launch_pcg_b(b, op->b_blocks, s));
+            CU(launch_pcg_b(b, op->b_blocks, s));  // (theta nodes: with the pole pass on q)
         }
         CU(cudaGraphLaunch(op->gexec, s));
     }
@@ -1987,10 +1985,7 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
         if (k <= maxit) {
             // virtual P2P ranks: all A(k) and k_aniso(k) done (B(k) reads slots A and C)
             if (p2p) ST(comm_vsync(comm, s));
-            if (op->tnode) {  // the caps of q = L p (theta nodes, NEXT-2)
-                ST(pole_pass(op, op->q, nc, s));
-                op->launches++;
-            }
+            // (theta nodes, NEXT-2: kernel B forms the caps of q = L p itself)
             if (pe) CU(cudaEventRecord(pe[2], s));
             CU(launch_pcg_b(b, op->b_blocks, s));
             op->launches++;
@@ -2026,7 +2021,7 @@ mas_status_t mas_pcg_solve(const mas_op_t* op_c, const double* rhs, double* x, d
     if (graph) {  // iteration 1 + 4 kernels per executed loop body (iterations 2k, 2k+1)
         const int last_a = fin.status == MAS_ERR_BREAKDOWN ? fin.iters : fin.iters + 1;
         const int bodies = last_a <= 2 ? 1 : last_a / 2;
-        const int per = 2 + (op->aniso && !lpar_in_a(op) ? 1 : 0) + (op->tnode ? 1 : 0);  // kernels per iteration
+        const int per = 2 + (op->aniso && !lpar_in_a(op) ? 1 : 0);  // kernels per iteration
         op->launches += per + 2LL * per * bodies;
     }
     if (res_hist) {
@@ -2106,8 +2101,7 @@ static cudaError_t stack_iteration(const mas_stack* sk, std::vector<StencilArgs>
     if (!with_b) return e;
     for (size_t m = 0; m < sk->ops.size() && e == cudaSuccess; m++) {
         const mas_op* op = sk->ops[m];
-        if (op->tnode) e = launch_pole_avg(op->geo, op->ncomp, op->q, nullptr, 0, op->geo.nl, s);
-        if (e == cudaSuccess) e = launch_pcg_b(b[m], op->b_blocks, s);
+        e = launch_pcg_b(b[m], op->b_blocks, s);  // (theta nodes: with the pole pass on q)
     }
     if (e == cudaSuccess) e = launch_stack_sum(ss, 1, 2, s);  // rho_k, ||r_k||^2
     return e;
@@ -2302,6 +2296,7 @@ mas_status_t mas_stack_solve(mas_stack_t* sk, const double* const* rhs, double* 
         B.r = op->r;
         B.q = op->q;
         B.dinv = op->dinv;
+        B.tnode = op->tnode;
         B.st = op->st;
         B.rho_hist = A.rho_hist;
         B.sigma_hist = A.sigma_hist;

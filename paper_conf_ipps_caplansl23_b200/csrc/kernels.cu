@@ -1183,7 +1183,11 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
 // --------------------------------------------------------------------------
 // kernel B: r -= alpha q ; z = D^-1 r ; <r,z>_V, <r,r>_V
 // --------------------------------------------------------------------------
-template <int NC>
+// TN (theta-node placement, NEXT-2 R29-R30): kernel B also does the pole pass
+// on q that k_pole_avg did between kernel A and kernel B -- one block per
+// (plane, pole) row forms the phi average of q with k_pole_avg's arithmetic
+// (same bits), then updates that row with it; the main loop skips pole rows.
+template <int NC, bool TN = false>
 __global__ void __launch_bounds__(kThreads) k_pcg_b(const StreamArgs a) {
     const PcgState* vst = a.st;
     if (__ldcg(&vst->stopped)) {
@@ -1224,6 +1228,46 @@ __global__ void __launch_bounds__(kThreads) k_pcg_b(const StreamArgs a) {
              e += (long long)gridDim.x * blockDim.x)
             a.x[e] = fma(am1, pk1[e], a.x[e]);
     }
+    if (TN && !brk) {
+        // the pole rows (j = 0, nt-1 of the theta-node rows), block-uniform loop
+        const long long Nl = (long long)g.nl * g.plane;
+        __shared__ double pws[2][kThreads / 32];
+        __shared__ double pavg;
+        for (int u = blockIdx.x; u < 2 * g.nl; u += gridDim.x) {
+            const int il = u >> 1, row = (u & 1) ? g.nt - 1 : 0;
+            const long long base = ((long long)il * g.nt + row) * g.np;
+            const double wrow = __ldg(g.vr + il) * __ldg(g.vt + row);
+            for (int c = 0; c < NC; c++) {
+                const double* qr = a.q + c * Nl + base;
+                double sq = 0.0, sw = 0.0;
+                for (int k = threadIdx.x; k < g.np; k += kThreads) {
+                    const double dp = __ldg(g.vp + k);
+                    sq = fma(dp, qr[k], sq);
+                    sw += dp;
+                }
+                sq = warp_sum(sq);
+                sw = warp_sum(sw);
+                if ((threadIdx.x & 31) == 0) pws[0][threadIdx.x >> 5] = sq, pws[1][threadIdx.x >> 5] = sw;
+                __syncthreads();
+                if (threadIdx.x == 0) {
+                    double ts = 0.0, tw = 0.0;
+                    for (int t = 0; t < kThreads / 32; t++) ts += pws[0][t], tw += pws[1][t];
+                    pavg = ts / tw;
+                }
+                __syncthreads();
+                const double qbar = pavg;
+                for (int k = threadIdx.x; k < g.np; k += kThreads) {
+                    double* rp = a.r + c * Nl + base + k;
+                    const double rv = fma(-alpha, qbar, *rp);
+                    *rp = rv;
+                    const double V = wrow * __ldg(g.vp + k);
+                    acc[0] += V * rv * (__ldg(a.dinv + base + k) * rv);
+                    acc[1] += V * rv * rv;
+                }
+                __syncthreads();  // pavg / pws reused by the next component or row
+            }
+        }
+    }
     if (!brk) {
         const long long Nl = (long long)g.nl * g.plane;
         const int rows = g.nl * g.nt;
@@ -1239,13 +1283,23 @@ __global__ void __launch_bounds__(kThreads) k_pcg_b(const StreamArgs a) {
             // step, all six loads in flight before the arithmetic
             const int stride = gridDim.x * rpi;
             for (int row = blockIdx.x * rpi + sub; row < rows; row += 2 * stride) {
-                const int row2 = row + stride;
-                const bool two = row2 < rows;
-                const int i1 = row / g.nt, j1 = row - i1 * g.nt;
+                int row1 = row, row2 = row + stride;
+                bool two = row2 < rows;
+                if (TN) {  // pole rows were done above
+                    const int jj1 = row1 % g.nt, jj2 = row2 % g.nt;
+                    const bool p1 = jj1 == 0 || jj1 == g.nt - 1, p2 = two && (jj2 == 0 || jj2 == g.nt - 1);
+                    if (p2) two = false;
+                    if (p1) {
+                        if (!two) continue;
+                        row1 = row2;
+                        two = false;
+                    }
+                }
+                const int i1 = row1 / g.nt, j1 = row1 - i1 * g.nt;
                 const int i2 = two ? row2 / g.nt : i1, j2 = two ? row2 - i2 * g.nt : j1;
                 const double w1 = __ldg(g.vr + i1) * __ldg(g.vt + j1);
                 const double w2 = __ldg(g.vr + i2) * __ldg(g.vt + j2);
-                const long long b1 = (long long)row * g.np, b2 = (long long)(two ? row2 : row) * g.np;
+                const long long b1 = (long long)row1 * g.np, b2 = (long long)(two ? row2 : row1) * g.np;
                 for (int h = col; h < half; h += tpr) {
                     const int k = 2 * h;
                     const double2 d1 = ld2(a.dinv + b1 + k), r1 = ld_cs(a.r + b1 + k), q1 = ld_cs(a.q + b1 + k);
@@ -1276,6 +1330,7 @@ __global__ void __launch_bounds__(kThreads) k_pcg_b(const StreamArgs a) {
 #endif
         for (int row = blockIdx.x * rpi + sub; row < rows; row += gridDim.x * rpi) {
             const int i = row / g.nt, j = row - i * g.nt;
+            if (TN && (j == 0 || j == g.nt - 1)) continue;  // pole rows were done above
             const double wrow = __ldg(g.vr + i) * __ldg(g.vt + j);
             const long long base = (long long)row * g.np;
             for (int h = col; h < half; h += tpr) {
@@ -1636,7 +1691,11 @@ cudaError_t launch_stack_sum(const StackStates& s, int off, int cnt, cudaStream_
 }
 
 cudaError_t launch_pcg_b(const StreamArgs& a, int nblocks, cudaStream_t s) {
-    if (a.ncomp == 1)
+    if (a.ncomp == 1 && a.tnode)
+        k_pcg_b<1, true><<<nblocks, kThreads, 0, s>>>(a);
+    else if (a.ncomp == 3 && a.tnode)
+        k_pcg_b<3, true><<<nblocks, kThreads, 0, s>>>(a);
+    else if (a.ncomp == 1)
         k_pcg_b<1><<<nblocks, kThreads, 0, s>>>(a);
     else if (a.ncomp == 3)
         k_pcg_b<3><<<nblocks, kThreads, 0, s>>>(a);

@@ -175,6 +175,7 @@ struct StreamArgs {  // kernel B
     double* x;
     const double* p[2];
     int brk_at;               // test hook (MAS_TEST_TRANSPORTS=1 + MAS_TEST_BREAKDOWN_AT=k): B(k) breaks down
+    int tnode;                // theta-node placement: kernel B does the pole pass on q first
 };
 
 // ---------------------------------------------------------------------------
