@@ -5,8 +5,10 @@ R34) at C3's size on one B200, beside C3's cell-centred 3-component solve.
 Each block is a scalar operator at its own location: v_r on the r nodes,
 v_theta on the theta nodes, v_phi on the phi nodes (workloads.
 staggered_viscosity_blocks: C3's fields evaluated there).  Per iteration each
-block runs kernel A (72 B per unknown: r, p_old, x, dinv, kappa, c read; p, q,
-x written) and kernel B (32 B: r, q, dinv read; r written), plus the
+block runs kernel A (68 B per unknown on average: r, p_old, dinv, kappa, c read,
+p, q written, and x read and written with p_(k-2) read by every second launch --
+the two-iteration x update; bench.alg_bytes_per_cell(1)) and kernel B (32 B: r,
+q, dinv read; r written), plus the
 one-warp k_stack_sum nodes.  Timed with CUDA events around mas_stack_solve
 (x reset to x0 before each step, outside the events), after warm-up.
 Prints one JSON line."""
@@ -78,7 +80,9 @@ def main():
 
     it_s, ms_s = timed(solve_s, reset_s)
     unknowns = sum(int(np.prod(b[1].shape)) for b in blocks)
-    bytes_it = 104 * unknowns
+    sys.path.insert(0, ROOT)
+    import bench  # the byte counts of the bench contract
+    bytes_it = sum(bench.alg_bytes_per_cell(1)) * unknowns  # 68 + 32 B per unknown
     sk.close()
     for o in ops:
         o.close()
