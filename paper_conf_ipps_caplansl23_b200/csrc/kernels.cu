@@ -1239,11 +1239,32 @@ __global__ void __launch_bounds__(kThreads) k_pcg_b(const StreamArgs a) {
             const double wrow = __ldg(g.vr + il) * __ldg(g.vt + row);
             for (int c = 0; c < NC; c++) {
                 const double* qr = a.q + c * Nl + base;
+                double* rr = a.r + c * Nl + base;
+                // q, r, 1/D and the phi weights of the thread's cells, loaded
+                // together (one round trip; rows of up to 4 * kThreads cells)
+                constexpr int PK = 4;
+                double qv[PK], rv0[PK], dv[PK], vp[PK];
+                const bool fits = g.np <= PK * kThreads;
+#pragma unroll
+                for (int t = 0; t < PK; t++) {
+                    const int k = threadIdx.x + t * kThreads;
+                    const bool in = fits && k < g.np;
+                    qv[t] = in ? qr[k] : 0.0;
+                    rv0[t] = in ? rr[k] : 0.0;
+                    dv[t] = in ? __ldg(a.dinv + base + k) : 0.0;
+                    vp[t] = in ? __ldg(g.vp + k) : 0.0;
+                }
                 double sq = 0.0, sw = 0.0;
-                for (int k = threadIdx.x; k < g.np; k += kThreads) {
-                    const double dp = __ldg(g.vp + k);
-                    sq = fma(dp, qr[k], sq);
-                    sw += dp;
+                if (fits) {
+#pragma unroll
+                    for (int t = 0; t < PK; t++)
+                        if (threadIdx.x + t * kThreads < g.np) sq = fma(vp[t], qv[t], sq), sw += vp[t];
+                } else {
+                    for (int k = threadIdx.x; k < g.np; k += kThreads) {
+                        const double dp = __ldg(g.vp + k);
+                        sq = fma(dp, qr[k], sq);
+                        sw += dp;
+                    }
                 }
                 sq = warp_sum(sq);
                 sw = warp_sum(sw);
@@ -1256,13 +1277,26 @@ __global__ void __launch_bounds__(kThreads) k_pcg_b(const StreamArgs a) {
                 }
                 __syncthreads();
                 const double qbar = pavg;
-                for (int k = threadIdx.x; k < g.np; k += kThreads) {
-                    double* rp = a.r + c * Nl + base + k;
-                    const double rv = fma(-alpha, qbar, *rp);
-                    *rp = rv;
-                    const double V = wrow * __ldg(g.vp + k);
-                    acc[0] += V * rv * (__ldg(a.dinv + base + k) * rv);
-                    acc[1] += V * rv * rv;
+                if (fits) {
+#pragma unroll
+                    for (int t = 0; t < PK; t++) {
+                        const int k = threadIdx.x + t * kThreads;
+                        if (k < g.np) {
+                            const double rv = fma(-alpha, qbar, rv0[t]);
+                            rr[k] = rv;
+                            const double V = wrow * vp[t];
+                            acc[0] += V * rv * (dv[t] * rv);
+                            acc[1] += V * rv * rv;
+                        }
+                    }
+                } else {
+                    for (int k = threadIdx.x; k < g.np; k += kThreads) {
+                        const double rv = fma(-alpha, qbar, rr[k]);
+                        rr[k] = rv;
+                        const double V = wrow * __ldg(g.vp + k);
+                        acc[0] += V * rv * (__ldg(a.dinv + base + k) * rv);
+                        acc[1] += V * rv * rv;
+                    }
                 }
                 __syncthreads();  // pavg / pws reused by the next component or row
             }
