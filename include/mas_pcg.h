@@ -167,7 +167,8 @@ MAS_API mas_status_t mas_op_setup(mas_grid_t* g, int ncomp, const double* kappa,
  * [tC_{j-1}, tC_j]; a pole's equation is the balance of its polar cap
  * (theta in [0, tC_0]), the phi sum of its slices' fluxes to row 1 -- the
  * paper's per-radius sum0 array reduction (Listings 3-5, P:428-445,
- * P:592-645), done on the GPU by k_pole_avg after every stencil pass.
+ * P:592-645), done on the GPU after every stencil pass (k_pole_avg; inside a
+ * solve's iterations kernel B forms the caps of q itself).
  * kappa and c may vary over a pole row's slots (each slot is a cap slice);
  * rhs and x0 pole rows are taken as one value (x0's are replaced by their
  * dp-weighted phi average; rhs must be phi-constant there).  Needs both pole
