@@ -317,6 +317,15 @@ constexpr bool kX2 = (NC == 1);
 #define MAS_PF_DIST 3
 #endif
 constexpr int kPfDist = MAS_PF_DIST;  // planes ahead of the stencil plane
+// the single-reduction kernel (CG1) streams more fields per plane (w, s and
+// its late own-only x, p loads): its prefetched lines must land closer to
+// their use or L2 evicts them first (C3 CG1: distance 2 / 3 / 4 = 534 / 474 /
+// 426 iters/s; kernel A at 3 is best: 707 against 665 at 2 or 4, r6pfab)
+#ifndef MAS_PF_DIST_CG1
+#define MAS_PF_DIST_CG1 2
+#endif
+template <int MODE>
+constexpr int kPfDistOf = MODE == MODE_CG1 ? MAS_PF_DIST_CG1 : kPfDist;
 #ifndef MAS_PF_SCALAR
 #define MAS_PF_SCALAR 0  // the scalar kernel measured slower with the prefetch (r1e)
 #endif
@@ -925,7 +934,7 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
 #ifndef MAS_NO_PREFETCH
     // the planes the march reaches before its first in-loop prefetch
     if (NC == 3 || MAS_PF_SCALAR)
-        for (int ip = ia + 1; ip < min(ia + kPfDist, ib); ip++)
+        for (int ip = ia + 1; ip < min(ia + kPfDistOf<MODE>, ib); ip++)
             plane_prefetch<MODE, NC>(a, ip, j0, k0, height, width, FIRSTK, xupd);
 #endif
     // ---- prologue: planes ia-1 (own cells only) and ia --------------------
@@ -1008,8 +1017,8 @@ __global__ void __launch_bounds__(kSThreads, NC == 1 ? MAS_MINB1 : MAS_MINB) k_s
 #ifndef MAS_NO_PREFETCH
         // 3-component kernels only: for the scalar kernel (C2: 256 work items,
         // under one wave) it measured slower (tools/abtest.sh)
-        if ((NC == 3 || MAS_PF_SCALAR) && i + kPfDist < ib)
-            plane_prefetch<MODE, NC>(a, i + kPfDist, j0, k0, height, width, FIRSTK, xupd);
+        if ((NC == 3 || MAS_PF_SCALAR) && i + kPfDistOf<MODE> < ib)
+            plane_prefetch<MODE, NC>(a, i + kPfDistOf<MODE>, j0, k0, height, width, FIRSTK, xupd);
 #endif
         if (!kIssueEarly && i + 2 <= ib && real_plane(i + 2))
             stage_issue<MODE, NC, LPAR>(a, i + 2, j0, k0, height, width, hm, FIRSTK, xupd && (i + 2 < ib),
