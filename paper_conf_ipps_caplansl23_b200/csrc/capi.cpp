@@ -854,8 +854,9 @@ static mas_status_t cg1_solve(mas_op* op, const double* fd, double* xd, double t
         CU(cudaGraphLaunch(op->gexec1, s));
     } else {
         // host-driven: launch n = 1 is the init, n = k + 1 is kernel k; stop
-        // enqueueing once the device reports a decision taken by launch <= n-1
-        for (int n = 1; n <= maxit + 1; n++) {
+        // enqueueing once the device reports a decision taken by launch <= n-1.
+        // Kernel maxit + 1 (launch maxit + 2) takes the maxit decision.
+        for (int n = 1; n <= maxit + 2; n++) {
             cudaEvent_t* pe = nullptr;
             if (op->prof) {
                 ST(ensure_prof_events(op, n));

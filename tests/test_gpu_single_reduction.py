@@ -91,6 +91,12 @@ def test_single_reduction_fixed_iterations(mp, oracle_mod, k, mk):
     assert it == ito == k
     V = oracle_mod.Oracle.for_problem(prob).volumes()
     assert rel_l2_V(V, x - prob.x0, xo - prob.x0) <= 1e-10
+    # the host-driven loop (profiling; also the virtual-rank / NCCL loops) must
+    # launch the kernel that takes the maxit decision and give the same bits
+    st2, x2, it2, rel2, hist2, _, _ = gsolve(mp, prob, tol=0.0, maxit=k, prof=True)
+    assert (st2, it2) == (st, it)
+    np.testing.assert_array_equal(x2, x)
+    np.testing.assert_array_equal(np.asarray(hist2), np.asarray(hist))
 
 
 @pytest.mark.parametrize("mk", ["viscosity", "mms"])
