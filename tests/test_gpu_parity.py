@@ -194,6 +194,18 @@ def test_pcg_fixed_iterations(mp, oracle_mod, k):
     assert it == ito == k
     V = oracle_mod.Oracle.for_problem(prob).volumes()
     assert rel_l2_V(V, x, xo) <= 1e-10
+    # the host-driven loop (profiling on) reaches the same maxit decision, bitwise
+    g2, op2 = make(mp, prob.mesh, prob.ncomp, prob.kappa, prob.c, prob.bc_inner, prob.bc_outer)
+    f2 = dev(prob.f)
+    if prob.ub_inner is not None or prob.ub_outer is not None:
+        op2.dirichlet_rhs(dev(prob.ub_inner) if prob.ub_inner is not None else None,
+                          dev(prob.ub_outer) if prob.ub_outer is not None else None, f2)
+    op2.set_profiling(True)
+    x2 = dev(prob.x0)
+    st2, it2, _, hist2 = op2.solve(f2, x2, 0.0, k, True)
+    assert (st2, it2) == (st, it)
+    np.testing.assert_array_equal(host(x2), x)
+    np.testing.assert_array_equal(np.asarray(hist2), np.asarray(hist))
 
 
 def test_pcg_edge_cases(mp, oracle_mod):
